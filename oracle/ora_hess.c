@@ -1,0 +1,605 @@
+/*
+ * ora_hess.c -- the CPU oracle (TEST INFRASTRUCTURE ONLY; see oracle.h).
+ *
+ * What each function follows:
+ *   ora_dgehd2    unblocked Householder reduction H = Q^T A Q          P:38-40 (Sec. III-A)
+ *                 with LAPACK DLARFG/DGEHD2 conventions (reading R1, R3)
+ *   ora_dorghr    Q = H(ilo) ... H(ihi-1), backward accumulation         P:40 (Q = Q1 Q2 ... Qn)
+ *   encode        r = A e, c = e^T A, kappa = e^T A e                    P:218-224 (Sec. IV-B, Fig. 3), R22
+ *   bookkeeping   Theorem 1 applied per reflector (right then left)      P:268-274 (Sec. IV-D)
+ *   verify        recompute L e, e^T L at each boundary                  P:256-260, P:272 (Sec. IV-C/F)
+ *   decode/fix    A(i,j) = r(i) - sum_{k!=j} A(i,k) (or column form)     P:278 (Sec. IV-F), R12
+ *   Q protection  Qr/Qc of the Householder vectors, checked at the end   P:266, P:278 (Sec. IV-E)
+ *   injector      XOR one bit of a binary64 word                         P:48-52 (failure model), R16
+ *
+ * The paper checks once per nb-column iteration (Alg. 3 l.12-13);
+ * the oracle runs the unblocked algorithm and verifies at the same
+ * boundaries (columns k = ilo-1 + t*nb) with the vector test of R11,
+ * recomputing the checksums from scratch (no fusion, no incremental sums).
+ */
+#include "oracle.h"
+
+#include <float.h>
+#include <math.h>
+#include <stdlib.h>
+#include <string.h>
+#ifdef _OPENMP
+#include <omp.h>
+#endif
+
+#define AT(A, lda, i, j) (A)[(size_t)(i) + (size_t)(j) * (size_t)(lda)]
+static const double EPS = DBL_EPSILON; /* 2^-52, R17 */
+
+int ora_num_threads(void) {
+#ifdef _OPENMP
+    return omp_get_max_threads();
+#else
+    return 1;
+#endif
+}
+
+double ora_flip(double *x, int bit) {
+    uint64_t u;
+    double old = *x;
+    memcpy(&u, x, 8);
+    u ^= (uint64_t)1 << (bit & 63);
+    memcpy(x, &u, 8);
+    return *x - old;
+}
+
+/* ------------------------------------------------------------------ */
+/* DLARFG (R1): given alpha and x (length m), produce beta, tau and     */
+/* scale x in place so that H [alpha; x] = [beta; 0], H = I - tau v v^T, */
+/* v = [1; x_scaled].  xnorm = 0 (or m = 0) gives tau = 0, H = I.        */
+/* ------------------------------------------------------------------ */
+static void dlarfg(int m, double *alpha, double *x, double *tau) {
+    double xnorm2 = 0.0;
+    for (int i = 0; i < m; i++) xnorm2 += x[i] * x[i];
+    double xnorm = sqrt(xnorm2);
+    if (m <= 0 || xnorm == 0.0) {
+        *tau = 0.0;
+        return;
+    }
+    double beta = -copysign(hypot(*alpha, xnorm), *alpha);
+    *tau = (beta - *alpha) / beta;
+    double scal = 1.0 / (*alpha - beta);
+    for (int i = 0; i < m; i++) x[i] *= scal;
+    *alpha = beta;
+}
+
+static int check_args(int n, int ilo, int ihi, const void *A, int lda, const void *tau) {
+    if (n < 0) return -1;
+    if (ilo < 1 || ilo > (n > 1 ? n : 1)) return -2;
+    if (ihi < (ilo < n ? ilo : n) || ihi > n) return -3;
+    if (n > 0 && A == NULL) return -4;
+    if (lda < (n > 1 ? n : 1)) return -5;
+    if (n > 1 && tau == NULL) return -6;
+    return 0;
+}
+
+/* One reflector step at column c (0-based), optionally carrying the
+ * checksum bookkeeping of Theorem 1.  y, w are workspaces of length n.
+ * Returns tau.  chk == NULL: plain DGEHD2 step. */
+typedef struct {
+    double *r, *c, *kap;     /* H checksums (length n, n, 1) */
+    double *qr, *qc, *qk;    /* Q checksums */
+} chk_t;
+
+static double reflector_step(int n, int ihi, double *A, int lda, int c,
+                             double *y, double *w, chk_t *chk) {
+    int m = ihi - c - 1;                 /* length of [alpha; x] = rows c+1..ihi-1 */
+    double tau = 0.0;
+    if (m < 1) return 0.0;
+    double *alpha = &AT(A, lda, c + 1, c);
+    double *x = &AT(A, lda, c + 2, c);   /* rows c+2..ihi-1, length m-1 */
+    double alpha0 = *alpha;
+    dlarfg(m - 1, alpha, x, &tau);
+    if (tau == 0.0) {
+        if (chk) {                       /* H(c) = I: checksums unchanged, Qc(c) = sum x */
+            double sx = 0.0;
+            for (int i = 0; i < m - 1; i++) sx += x[i];
+            chk->qc[c] = sx;
+            for (int i = 0; i < m - 1; i++) chk->qr[c + 2 + i] += x[i];
+            *chk->qk += sx;
+        }
+        return 0.0;
+    }
+    double beta = *alpha;
+    /* v(c+1) = 1 implicit, v(c+2:ihi) = x */
+#define V(i) ((i) == c + 1 ? 1.0 : AT(A, lda, (i), c))
+    double ev = 1.0;                     /* e^T v */
+    for (int i = c + 2; i < ihi; i++) ev += V(i);
+
+    if (chk) {
+        /* reduced column c: left term of its own reflector (R7): c[c] -= (e^T v)(alpha - beta) */
+        chk->c[c] -= ev * (alpha0 - beta);
+        /* Q checksums of the new Householder vector (Fig. 5) */
+        chk->qc[c] = ev - 1.0;
+        for (int i = c + 2; i < ihi; i++) chk->qr[i] += V(i);
+        *chk->qk += ev - 1.0;
+    }
+
+    /* Right step: A(0:ihi, c+1:ihi) := A (I - tau v v^T).  y = A v.  P:38 (A Q_i) */
+#pragma omp parallel for schedule(static)
+    for (int i = 0; i < ihi; i++) {
+        double s = 0.0;
+        for (int j = c + 1; j < ihi; j++) s += AT(A, lda, i, j) * V(j);
+        y[i] = s;
+    }
+    if (chk) {
+        /* Theorem 1 part 2 at reflector granularity */
+        double cv = 0.0;
+        for (int j = c + 1; j < ihi; j++) cv += chk->c[j] * V(j);
+        *chk->kap -= tau * cv * ev;
+        for (int j = c + 1; j < ihi; j++) chk->c[j] -= tau * cv * V(j);
+        for (int i = 0; i < ihi; i++) chk->r[i] -= tau * ev * y[i];
+    }
+#pragma omp parallel for schedule(static)
+    for (int j = c + 1; j < ihi; j++) {
+        double vj = tau * V(j);
+        for (int i = 0; i < ihi; i++) AT(A, lda, i, j) -= y[i] * vj;
+    }
+
+    /* Left step: A(c+1:ihi, c+1:n) := (I - tau v v^T) A.  w = v^T A.  P:38 (Q_i^{-1} A) */
+#pragma omp parallel for schedule(static)
+    for (int j = c + 1; j < n; j++) {
+        double s = 0.0;
+        for (int i = c + 1; i < ihi; i++) s += V(i) * AT(A, lda, i, j);
+        w[j] = s;
+    }
+    if (chk) {
+        /* Theorem 1 part 3 at reflector granularity */
+        double vr = 0.0;
+        for (int i = c + 1; i < ihi; i++) vr += V(i) * chk->r[i];
+        *chk->kap -= tau * ev * vr;
+        for (int i = c + 1; i < ihi; i++) chk->r[i] -= tau * vr * V(i);
+        for (int j = c + 1; j < n; j++) chk->c[j] -= tau * ev * w[j];
+    }
+#pragma omp parallel for schedule(static)
+    for (int j = c + 1; j < n; j++) {
+        double wj = tau * w[j];
+        for (int i = c + 1; i < ihi; i++) AT(A, lda, i, j) -= V(i) * wj;
+    }
+#undef V
+    return tau;
+}
+
+int ora_dgehd2(int n, int ilo, int ihi, double *A, int lda, double *tau) {
+    int info = check_args(n, ilo, ihi, A, lda, tau);
+    if (info) return info;
+    for (int c = 0; c < n - 1; c++) tau[c] = 0.0;
+    if (n <= 1) return 0;
+    double *y = (double *)calloc((size_t)n, sizeof(double));
+    double *w = (double *)calloc((size_t)n, sizeof(double));
+    for (int c = ilo - 1; c <= ihi - 2; c++) tau[c] = reflector_step(n, ihi, A, lda, c, y, w, NULL);
+    free(y);
+    free(w);
+    return 0;
+}
+
+int ora_dorghr(int n, int ilo, int ihi, const double *A, int lda, const double *tau,
+               double *Q, int ldq) {
+    int info = check_args(n, ilo, ihi, A, lda, tau);
+    if (info) return info;
+    if (Q == NULL) return -7;
+    if (ldq < (n > 1 ? n : 1)) return -8;
+    for (int j = 0; j < n; j++)
+        for (int i = 0; i < n; i++) AT(Q, ldq, i, j) = (i == j) ? 1.0 : 0.0;
+    if (n <= 1) return 0;
+    double *w = (double *)calloc((size_t)n, sizeof(double));
+    /* Q := H(c) Q for c = ihi-2 down to ilo-1; H(c) acts on rows/cols c+1..ihi-1 */
+    for (int c = ihi - 2; c >= ilo - 1; c--) {
+        double t = tau[c];
+        if (t == 0.0) continue;
+#define V(i) ((i) == c + 1 ? 1.0 : AT(A, lda, (i), c))
+#pragma omp parallel for schedule(static)
+        for (int j = c + 1; j < ihi; j++) {
+            double s = 0.0;
+            for (int i = c + 1; i < ihi; i++) s += V(i) * AT(Q, ldq, i, j);
+            w[j] = s;
+        }
+#pragma omp parallel for schedule(static)
+        for (int j = c + 1; j < ihi; j++) {
+            double wj = t * w[j];
+            for (int i = c + 1; i < ihi; i++) AT(Q, ldq, i, j) -= V(i) * wj;
+        }
+#undef V
+    }
+    free(w);
+    return 0;
+}
+
+/* ------------------------------------------------------------------ */
+/* Decoder (reading R12, "decoder v2"): never miscorrect.              */
+/* ------------------------------------------------------------------ */
+static void push_ev(ora_report *rep, int kind, int panel, int64_t i, int64_t j, double delta) {
+    if (!rep) return;
+    if (rep->nevents < ORA_MAX_EVENTS) {
+        ora_event *e = &rep->ev[rep->nevents++];
+        e->kind = kind; e->panel = panel; e->i = i; e->j = j; e->delta = delta;
+    }
+}
+
+static int bad(double d, double tau) { return !(fabs(d) <= tau); } /* NaN counts as flagged */
+
+static int approx(double a, double b, double tol) {
+    if (!isfinite(a) || !isfinite(b)) return !isfinite(a) && !isfinite(b);
+    return fabs(a - b) <= tol;
+}
+
+typedef struct { double *Dr, *Dc, sr, sc; } syn_t;
+
+static void syndromes(int n, const double *L, int ldl, const double *r, const double *c,
+                      double kap, syn_t *s) {
+#pragma omp parallel for schedule(static)
+    for (int i = 0; i < n; i++) {
+        double t = 0.0;
+        for (int j = 0; j < n; j++) t += AT(L, ldl, i, j);
+        s->Dr[i] = r[i] - t;
+    }
+#pragma omp parallel for schedule(static)
+    for (int j = 0; j < n; j++) {
+        double t = 0.0;
+        for (int i = 0; i < n; i++) t += AT(L, ldl, i, j);
+        s->Dc[j] = c[j] - t;
+    }
+    double sr = 0.0, sc = 0.0;
+    for (int i = 0; i < n; i++) sr += r[i];
+    for (int j = 0; j < n; j++) sc += c[j];
+    s->sr = sr - kap;
+    s->sc = sc - kap;
+}
+
+/* unique subset S' of idx[0..m) (size <= 3) with sum D over S' ~ target.
+ * Returns size (0..3) with members in out[], or -1 if none / not unique. */
+static int unique_subset(int m, const int *idx, const double *D, double target,
+                         double tauS, int n, int *out) {
+    double tol_base = tauS;
+    if (approx(target, 0.0, tauS)) return 0;
+    if (!isfinite(target)) {       /* a checksum word became inf/nan: take the non-finite ones */
+        int k = 0;
+        for (int a = 0; a < m; a++)
+            if (!isfinite(D[idx[a]])) { if (k == 3) return -1; out[k++] = idx[a]; }
+        return k > 0 ? k : -1;
+    }
+    if (m > 256) return -1;
+    int found = 0, best[3] = {-1, -1, -1}, bsz = 0;
+    for (int a = 0; a < m; a++) {
+        double da = D[idx[a]];
+        double tol = tol_base + 2.0 * n * EPS * fabs(da);
+        if (approx(da, target, tol)) { found++; best[0] = idx[a]; bsz = 1; }
+        for (int b = a + 1; b < m; b++) {
+            double db = D[idx[b]];
+            double tol2 = tol_base + 2.0 * n * EPS * (fabs(da) + fabs(db));
+            if (approx(da + db, target, tol2)) { found++; best[0] = idx[a]; best[1] = idx[b]; bsz = 2; }
+            for (int e = b + 1; e < m; e++) {
+                double de = D[idx[e]];
+                double tol3 = tol_base + 2.0 * n * EPS * (fabs(da) + fabs(db) + fabs(de));
+                if (approx(da + db + de, target, tol3)) {
+                    found++; best[0] = idx[a]; best[1] = idx[b]; best[2] = idx[e]; bsz = 3;
+                }
+            }
+        }
+    }
+    if (found != 1) return -1;
+    for (int k = 0; k < bsz; k++) out[k] = best[k];
+    return bsz;
+}
+
+static int in_set(int v, const int *s, int m) {
+    for (int k = 0; k < m; k++) if (s[k] == v) return 1;
+    return 0;
+}
+
+/* A(i,j) = r(i) - sum_{k != j} L(i,k)   (first formula) */
+static double fix_row(int n, double *L, int ldl, const double *r, int i, int j) {
+    double s = 0.0;
+    for (int k = 0; k < n; k++) if (k != j) s += AT(L, ldl, i, k);
+    double old = AT(L, ldl, i, j);
+    AT(L, ldl, i, j) = r[i] - s;
+    return AT(L, ldl, i, j) - old;
+}
+/* A(i,j) = c(j) - sum_{k != i} L(k,j)   (second formula) */
+static double fix_col(int n, double *L, int ldl, const double *c, int i, int j) {
+    double s = 0.0;
+    for (int k = 0; k < n; k++) if (k != i) s += AT(L, ldl, k, j);
+    double old = AT(L, ldl, i, j);
+    AT(L, ldl, i, j) = c[j] - s;
+    return AT(L, ldl, i, j) - old;
+}
+
+int ora_decode(int n, double *L, int ldl, double *r, double *c, double *kappa,
+               double tau_abs, ora_report *rep, int panel, int mode) {
+    const int evD = mode == ORA_MODE_Q ? ORA_EV_FIX_Q : ORA_EV_FIX_DATA;
+    const int evR = mode == ORA_MODE_Q ? ORA_EV_FIX_QR : ORA_EV_FIX_R;
+    const int evC = mode == ORA_MODE_Q ? ORA_EV_FIX_QC : ORA_EV_FIX_C;
+    const int evK = mode == ORA_MODE_Q ? ORA_EV_FIX_QK : ORA_EV_FIX_K;
+    double tauS = tau_abs * sqrt((double)(n > 1 ? n : 1));
+    syn_t s;
+    s.Dr = (double *)malloc(sizeof(double) * (size_t)(n > 0 ? n : 1));
+    s.Dc = (double *)malloc(sizeof(double) * (size_t)(n > 0 ? n : 1));
+    int *R = (int *)malloc(sizeof(int) * (size_t)(n > 0 ? n : 1));
+    int *C = (int *)malloc(sizeof(int) * (size_t)(n > 0 ? n : 1));
+    int *Rd = (int *)malloc(sizeof(int) * (size_t)(n > 0 ? n : 1));
+    int *Cd = (int *)malloc(sizeof(int) * (size_t)(n > 0 ? n : 1));
+    int result = 0;
+    syndromes(n, L, ldl, r, c, *kappa, &s);
+    int nR = 0, nC = 0;
+    for (int i = 0; i < n; i++) if (bad(s.Dr[i], tau_abs)) R[nR++] = i;
+    for (int j = 0; j < n; j++) if (bad(s.Dc[j], tau_abs)) C[nC++] = j;
+    int sr_ok = approx(s.sr, 0.0, tauS), sc_ok = approx(s.sc, 0.0, tauS);
+    if (nR == 0 && nC == 0 && sr_ok && sc_ok) { result = 0; goto done; }
+    push_ev(rep, ORA_EV_DETECT, panel, nR, nC, 0.0);
+    if (rep) rep->detected++;
+
+    if (nR == 0 && nC == 0) {
+        /* (1) only the corner disagrees: both sums off by the same amount */
+        if (!sr_ok && !sc_ok && approx(s.sr, s.sc, tauS)) {
+            double sr = 0.0;
+            for (int i = 0; i < n; i++) sr += r[i];
+            double old = *kappa;
+            *kappa = sr;
+            push_ev(rep, evK, panel, -1, -1, *kappa - old);
+        } else {
+            result = 2;
+            goto done;
+        }
+    } else {
+        /* (2) checksum-vector errors: unique subset whose syndrome sum explains s_r / s_c.
+         * If s_r ~ s_c != 0 the same syndrome is also produced by a corner error
+         * plus data errors (e.g. r(i), c(j) both off by -d  ==  A(i,j) and kappa
+         * both off by +d): information-theoretically ambiguous, so refuse. */
+        if (!sr_ok && !sc_ok && approx(s.sr, s.sc, tauS)) { result = 2; goto done; }
+        int Rc[3], Cc[3];
+        int nRc = unique_subset(nR, R, s.Dr, s.sr, tauS, n, Rc);
+        int nCc = unique_subset(nC, C, s.Dc, s.sc, tauS, n, Cc);
+        if (nRc < 0 || nCc < 0) { result = 2; goto done; }
+        int nRd = 0, nCd = 0;
+        for (int a = 0; a < nR; a++) if (!in_set(R[a], Rc, nRc)) Rd[nRd++] = R[a];
+        for (int a = 0; a < nC; a++) if (!in_set(C[a], Cc, nCc)) Cd[nCd++] = C[a];
+        /* (3) data errors */
+        if (nRd == 0 && nCd == 0) {
+            /* only checksum words were hit */
+        } else if (nRd == 0 || nCd == 0) {
+            result = 2; goto done;
+        } else if (nRd == 1 && nCd == 1) {
+            double tol = 2.0 * tau_abs + 2.0 * n * EPS * (fabs(s.Dr[Rd[0]]) + fabs(s.Dc[Cd[0]]));
+            if (!approx(s.Dr[Rd[0]], s.Dc[Cd[0]], tol)) { result = 2; goto done; }
+            double d = fix_row(n, L, ldl, r, Rd[0], Cd[0]);
+            push_ev(rep, evD, panel, Rd[0], Cd[0], d);
+        } else if (nRd == 1) {
+            /* one shared row, several columns: column formulas */
+            double sum = 0.0, sabs = 0.0;
+            int nonfin = 0;
+            for (int b = 0; b < nCd; b++) { sum += s.Dc[Cd[b]]; sabs += fabs(s.Dc[Cd[b]]); nonfin |= !isfinite(s.Dc[Cd[b]]); }
+            double tol = 2.0 * tauS + 2.0 * n * EPS * (sabs + fabs(s.Dr[Rd[0]]));
+            if (!nonfin && !approx(sum, s.Dr[Rd[0]], tol)) { result = 2; goto done; }
+            if (nonfin && isfinite(s.Dr[Rd[0]])) { result = 2; goto done; }
+            for (int b = 0; b < nCd; b++) {
+                double d = fix_col(n, L, ldl, c, Rd[0], Cd[b]);
+                push_ev(rep, evD, panel, Rd[0], Cd[b], d);
+            }
+        } else if (nCd == 1) {
+            /* one shared column, several rows: row formulas */
+            double sum = 0.0, sabs = 0.0;
+            int nonfin = 0;
+            for (int a = 0; a < nRd; a++) { sum += s.Dr[Rd[a]]; sabs += fabs(s.Dr[Rd[a]]); nonfin |= !isfinite(s.Dr[Rd[a]]); }
+            double tol = 2.0 * tauS + 2.0 * n * EPS * (sabs + fabs(s.Dc[Cd[0]]));
+            if (!nonfin && !approx(sum, s.Dc[Cd[0]], tol)) { result = 2; goto done; }
+            if (nonfin && isfinite(s.Dc[Cd[0]])) { result = 2; goto done; }
+            for (int a = 0; a < nRd; a++) {
+                double d = fix_row(n, L, ldl, r, Rd[a], Cd[0]);
+                push_ev(rep, evD, panel, Rd[a], Cd[0], d);
+            }
+        } else if (nRd == nCd) {
+            /* distinct rows and columns: pair by value, uniquely in both directions */
+            int *pair = (int *)malloc(sizeof(int) * (size_t)nRd);
+            int okp = 1;
+            for (int a = 0; a < nRd && okp; a++) {
+                int cnt = 0;
+                for (int b = 0; b < nCd; b++) {
+                    double tol = 2.0 * tau_abs + 2.0 * n * EPS * (fabs(s.Dr[Rd[a]]) + fabs(s.Dc[Cd[b]]));
+                    if (approx(s.Dr[Rd[a]], s.Dc[Cd[b]], tol)) { cnt++; pair[a] = b; }
+                }
+                if (cnt != 1) okp = 0;
+            }
+            for (int b = 0; b < nCd && okp; b++) {
+                int cnt = 0;
+                for (int a = 0; a < nRd; a++) {
+                    double tol = 2.0 * tau_abs + 2.0 * n * EPS * (fabs(s.Dr[Rd[a]]) + fabs(s.Dc[Cd[b]]));
+                    if (approx(s.Dr[Rd[a]], s.Dc[Cd[b]], tol)) cnt++;
+                }
+                if (cnt != 1) okp = 0;
+            }
+            if (okp)
+                for (int a = 0; a < nRd; a++) {
+                    double d = fix_row(n, L, ldl, r, Rd[a], Cd[pair[a]]);
+                    push_ev(rep, evD, panel, Rd[a], Cd[pair[a]], d);
+                }
+            free(pair);
+            if (!okp) { result = 2; goto done; }
+        } else {
+            result = 2; goto done;
+        }
+        /* (4) refresh the corrupted checksum words from the (repaired) data */
+        for (int a = 0; a < nRc; a++) {
+            int i = Rc[a];
+            double t = 0.0;
+            for (int j = 0; j < n; j++) t += AT(L, ldl, i, j);
+            double old = r[i];
+            r[i] = t;
+            push_ev(rep, evR, panel, i, -1, r[i] - old);
+        }
+        for (int b = 0; b < nCc; b++) {
+            int j = Cc[b];
+            double t = 0.0;
+            for (int i = 0; i < n; i++) t += AT(L, ldl, i, j);
+            double old = c[j];
+            c[j] = t;
+            push_ev(rep, evC, panel, -1, j, c[j] - old);
+        }
+    }
+    /* (5) re-verify: anything left is uncorrectable */
+    syndromes(n, L, ldl, r, c, *kappa, &s);
+    result = 1;
+    for (int i = 0; i < n && result == 1; i++) if (bad(s.Dr[i], tau_abs)) result = 2;
+    for (int j = 0; j < n && result == 1; j++) if (bad(s.Dc[j], tau_abs)) result = 2;
+    if (result == 1 && !(approx(s.sr, 0.0, tauS) && approx(s.sc, 0.0, tauS))) result = 2;
+done:
+    if (result == 1 && rep) rep->corrected++;
+    if (result == 2) {
+        push_ev(rep, ORA_EV_UNCORRECTABLE, panel, nR, nC, 0.0);
+        if (rep) rep->uncorrectable++;
+    }
+    free(s.Dr); free(s.Dc); free(R); free(C); free(Rd); free(Cd);
+    return result;
+}
+
+/* encode (Fig. 3, Alg. 3 l.2): r = A e, c = e^T A, kappa = e^T A e (R22) */
+void ora_encode(int n, const double *A, int lda, double *r, double *c, double *kappa) {
+    for (int i = 0; i < n; i++) {
+        double s = 0.0;
+        for (int j = 0; j < n; j++) s += AT(A, lda, i, j);
+        r[i] = s;
+    }
+    for (int j = 0; j < n; j++) {
+        double s = 0.0;
+        for (int i = 0; i < n; i++) s += AT(A, lda, i, j);
+        c[j] = s;
+    }
+    double k = 0.0;
+    for (int i = 0; i < n; i++) k += r[i];
+    *kappa = k;
+}
+
+/* ------------------------------------------------------------------ */
+/* ABFT driver                                                          */
+/* ------------------------------------------------------------------ */
+
+/* logical H matrix (R6): stored Householder vectors of finished columns
+ * (j in [ilo-1, cdone), i >= j+2) read as 0 */
+static int is_v(int i, int j, int ilo, int ihi, int cdone) {
+    return j >= ilo - 1 && j < cdone && j <= ihi - 2 && i >= j + 2 && i < ihi;
+}
+
+static void build_L(int n, const double *A, int lda, int ilo, int ihi, int cdone, double *L, int q) {
+#pragma omp parallel for schedule(static)
+    for (int j = 0; j < n; j++)
+        for (int i = 0; i < n; i++) {
+            int v = is_v(i, j, ilo, ihi, cdone);
+            AT(L, n, i, j) = (q ? v : !v) ? AT(A, lda, i, j) : 0.0;
+        }
+}
+
+static void write_back(int n, double *A, int lda, int ilo, int ihi, int cdone, const double *L, int q) {
+    for (int j = 0; j < n; j++)
+        for (int i = 0; i < n; i++) {
+            int v = is_v(i, j, ilo, ihi, cdone);
+            if (q ? v : !v) AT(A, lda, i, j) = AT(L, n, i, j);
+        }
+}
+
+static void inject(const ora_fault *f, int n, double *A, int lda, chk_t *k, ora_report *rep) {
+    double *p = NULL;
+    switch (f->site) {
+    case ORA_SITE_A: if (f->i >= 0 && f->i < n && f->j >= 0 && f->j < n) p = &AT(A, lda, f->i, f->j); break;
+    case ORA_SITE_R: if (f->i >= 0 && f->i < n) p = &k->r[f->i]; break;
+    case ORA_SITE_C: if (f->j >= 0 && f->j < n) p = &k->c[f->j]; break;
+    case ORA_SITE_K: p = k->kap; break;
+    case ORA_SITE_QR: if (f->i >= 0 && f->i < n) p = &k->qr[f->i]; break;
+    case ORA_SITE_QC: if (f->j >= 0 && f->j < n) p = &k->qc[f->j]; break;
+    }
+    if (!p) return;
+    double d = ora_flip(p, f->bit);
+    push_ev(rep, ORA_EV_INJECT, f->panel, f->i, f->j, d);
+}
+
+static double frob(int n, const double *A, int lda) {
+    double s = 0.0;
+    for (int j = 0; j < n; j++)
+        for (int i = 0; i < n; i++) s += AT(A, lda, i, j) * AT(A, lda, i, j);
+    return sqrt(s);
+}
+
+int ora_ft_dgehd2(int n, int ilo, int ihi, double *A, int lda, double *tau,
+                  int nb, double c_thr, const ora_fault *faults, int nfaults,
+                  ora_report *rep, int stop_after_panel, double *chk_out) {
+    int info = check_args(n, ilo, ihi, A, lda, tau);
+    if (info) return info;
+    if (nb < 1) return -7;
+    if (c_thr <= 0.0) c_thr = 2.0;
+    if (rep) memset(rep, 0, sizeof(*rep));
+    for (int c = 0; c < n - 1; c++) tau[c] = 0.0;
+    if (n == 0) return 0;
+
+    size_t nn = (size_t)n;
+    double *r = (double *)calloc(nn, 8), *cc = (double *)calloc(nn, 8);
+    double *qr = (double *)calloc(nn, 8), *qc = (double *)calloc(nn, 8);
+    double *y = (double *)calloc(nn, 8), *w = (double *)calloc(nn, 8);
+    double *L = (double *)malloc(nn * nn * 8);
+    double *Dr = (double *)malloc(nn * 8), *Dc = (double *)malloc(nn * 8);
+    double kap = 0.0, qk = 0.0;
+    chk_t k = {r, cc, &kap, qr, qc, &qk};
+
+    ora_encode(n, A, lda, r, cc, &kap);
+    double normF = frob(n, A, lda);              /* invariant under the similarity */
+    double tau_abs = c_thr * n * EPS * normF;    /* R10 */
+    double unit = n * EPS * (normF > 0 ? normF : 1.0);
+    int result = 0;
+
+    int c0 = ilo - 1, clast = ihi - 2;           /* reflector columns */
+    for (int c = c0; c <= clast; c++) {
+        if ((c - c0) % nb == 0) {
+            int t = (c - c0) / nb;
+            /* boundary t: inject, then verify / decode / correct (Alg. 3 l.12-15) */
+            for (int f = 0; f < nfaults; f++)
+                if (faults[f].panel == t) inject(&faults[f], n, A, lda, &k, rep);
+            build_L(n, A, lda, ilo, ihi, c, L, 0);
+            /* drift and the paper's scalar statistic (recorded; R11) */
+            {
+                double sr = 0.0, sc = 0.0, dmax = 0.0;
+                syn_t s = {Dr, Dc, 0, 0};
+                syndromes(n, L, n, r, cc, kap, &s);
+                for (int i = 0; i < n; i++) { sr += r[i]; if (fabs(Dr[i]) > dmax) dmax = fabs(Dr[i]); }
+                for (int j = 0; j < n; j++) { sc += cc[j]; if (fabs(Dc[j]) > dmax) dmax = fabs(Dc[j]); }
+                if (rep) {
+                    double ps = fabs(sr - sc) / (unit * sqrt((double)n));
+                    if (ps > rep->paper_stat_max || ps != ps) rep->paper_stat_max = ps;
+                    if (dmax / unit > rep->max_drift && dmax <= tau_abs) rep->max_drift = dmax / unit;
+                }
+            }
+            int dres = ora_decode(n, L, n, r, cc, &kap, tau_abs, rep, t, ORA_MODE_H);
+            if (dres == 2) { result = 1; goto out; }
+            if (dres == 1) write_back(n, A, lda, ilo, ihi, c, L, 0);
+        }
+        tau[c] = reflector_step(n, ihi, A, lda, c, y, w, &k);
+        if (stop_after_panel >= 0 && ((c + 1 - c0) % nb == 0 || c == clast) &&
+            (c - c0) / nb == stop_after_panel) {
+            if (chk_out) {
+                memcpy(chk_out, r, nn * 8);
+                memcpy(chk_out + n, cc, nn * 8);
+                chk_out[2 * n] = kap;
+            }
+            goto out;
+        }
+    }
+    /* end: inject AT_END faults, final H verification (a12) and Q verification */
+    for (int f = 0; f < nfaults; f++)
+        if (faults[f].panel == -1) inject(&faults[f], n, A, lda, &k, rep);
+    {
+        int cdone = clast + 1;
+        build_L(n, A, lda, ilo, ihi, cdone, L, 0);
+        int dres = ora_decode(n, L, n, r, cc, &kap, tau_abs, rep, -1, ORA_MODE_H);
+        if (dres == 2) { result = 1; goto out; }
+        if (dres == 1) write_back(n, A, lda, ilo, ihi, cdone, L, 0);
+        /* Q: logical matrix = stored Householder vectors only */
+        build_L(n, A, lda, ilo, ihi, cdone, L, 1);
+        double tauQ = c_thr * n * EPS * sqrt((double)n);
+        dres = ora_decode(n, L, n, qr, qc, &qk, tauQ, rep, -1, ORA_MODE_Q);
+        if (dres == 2) { result = 1; goto out; }
+        if (dres == 1) write_back(n, A, lda, ilo, ihi, cdone, L, 1);
+    }
+out:
+    free(r); free(cc); free(qr); free(qc); free(y); free(w); free(L); free(Dr); free(Dc);
+    return result;
+}

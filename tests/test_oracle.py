@@ -1,0 +1,364 @@
+"""Pins of the CPU oracle against things other than itself (-m "not gpu").
+
+Each test states what fixes the expected value:
+  * a library routine (LAPACK dgehrd/dorghr via scipy) for the whole reduction,
+  * the n = 3 worked example (tests/golden/n3_closed_form.json),
+  * exact special cases (already-Hessenberg, symmetric -> tridiagonal,
+    integer-valued encoding),
+  * invariants of a similarity (trace, Frobenius norm, eigenvalues, Q e1 = e1,
+    Q^T Q = I, residual),
+  * Theorem 1: maintained checksums equal recomputed ones,
+  * brute force over every <= 2-fault placement of the decoder (R12),
+  * the paper's Fig. 2 propagation pattern.
+"""
+import itertools
+import json
+import os
+
+import numpy as np
+import pytest
+from scipy.linalg import lapack
+
+import synth
+
+EPS = 2.0 ** -52
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def resid_ratio(A, H, Q):
+    n = A.shape[0]
+    return np.linalg.norm(A - Q @ H @ Q.T, 1) / (n * np.linalg.norm(A, 1) * EPS)
+
+
+def orth_ratio(Q):
+    n = Q.shape[0]
+    return np.linalg.norm(np.eye(n) - Q.T @ Q, 1) / (n * EPS)
+
+
+# ---------------------------------------------------------------- LAPACK pin
+@pytest.mark.parametrize("n,dist", [(5, "uniform"), (64, "uniform"), (64, "normal"),
+                                    (129, "normal"), (300, "uniform")])
+def test_matches_lapack_dgehrd(ora, n, dist):
+    A = synth.matrix(n, dist=dist)
+    Ao, tau = ora.dgehd2(A)
+    hq, tq, info = lapack.dgehrd(A)
+    assert info == 0
+    H, Hl = np.triu(Ao, -1), np.triu(hq, -1)
+    assert np.abs(H - Hl).max() / np.abs(Hl).max() <= 1e-12
+    assert np.abs(tau - tq[: n - 1]).max() <= 1e-12 * max(1.0, np.abs(tq).max())
+    V, Vl = np.tril(Ao, -2), np.tril(hq, -2)
+    assert np.abs(V - Vl).max() <= 1e-10
+    Q = ora.dorghr(Ao, tau)
+    Ql, info = lapack.dorghr(hq, tq)
+    assert info == 0
+    assert np.abs(Q - Ql).max() <= 1e-12
+
+
+@pytest.mark.parametrize("n,ilo,ihi", [(40, 1, 40), (40, 5, 40), (40, 1, 31), (40, 7, 29), (40, 20, 21), (40, 40, 40)])
+def test_ilo_ihi_matches_lapack(ora, n, ilo, ihi):
+    A = synth.matrix(n, seed=7 + ilo + 3 * ihi, ilo=ilo, ihi=ihi)
+    Ao, tau = ora.dgehd2(A, ilo, ihi)
+    hq, tq, info = lapack.dgehrd(A, lo=ilo - 1, hi=ihi - 1)
+    assert info == 0
+    assert np.abs(np.triu(Ao, -1) - np.triu(hq, -1)).max() <= 1e-12 * np.abs(hq).max()
+    assert np.abs(tau - tq[: n - 1]).max() <= 1e-12
+    # tau is zero outside the active block (LAPACK contract)
+    assert np.all(tau[: ilo - 1] == 0.0) and np.all(tau[max(ihi - 1, 0):] == 0.0)
+    Q = ora.dorghr(Ao, tau, ilo, ihi)
+    Ql, _ = lapack.dorghr(hq, tq, lo=ilo - 1, hi=ihi - 1)
+    assert np.abs(Q - Ql).max() <= 1e-12
+    H = np.triu(Ao, -1)
+    assert resid_ratio(A, H, Q) <= 30 and orth_ratio(Q) <= 30
+
+
+# ---------------------------------------------------------------- tiny cases
+@pytest.mark.parametrize("n", [0, 1, 2])
+def test_no_reflectors(ora, n):
+    A = synth.matrix(n) if n else np.zeros((0, 0))
+    Ao, tau = ora.dgehd2(A)
+    assert np.array_equal(Ao, A)
+    assert np.all(tau == 0.0)
+    if n:
+        assert np.array_equal(ora.dorghr(Ao, tau), np.eye(n))
+
+
+def test_n3_closed_form(ora):
+    g = json.load(open(os.path.join(GOLDEN, "n3_closed_form.json")))
+    A = np.array(g["A"], dtype=np.float64)
+    Ao, tau = ora.dgehd2(A)
+    np.testing.assert_allclose(tau, g["tau"], rtol=0, atol=1e-15)
+    assert Ao[1, 0] == g["beta"]
+    np.testing.assert_allclose(Ao[2, 0], g["v"][2], rtol=0, atol=1e-16)
+    np.testing.assert_allclose(np.triu(Ao, -1), g["H"], rtol=0, atol=4e-15)
+
+
+# ---------------------------------------------------------------- exact cases
+def test_already_hessenberg_is_identity_bitwise(ora):
+    A = synth.hessenberg_matrix(50)
+    Ao, tau = ora.dgehd2(A)
+    assert np.all(tau == 0.0)
+    assert np.array_equal(Ao, A)
+    assert np.array_equal(ora.dorghr(Ao, tau), np.eye(50))
+
+
+def test_symmetric_gives_tridiagonal(ora):
+    S = synth.symmetric_matrix(80)
+    Ao, tau = ora.dgehd2(S)
+    H = np.triu(Ao, -1)
+    assert np.abs(np.triu(H, 2)).max() <= 1e-14 * np.linalg.norm(S)
+    # and H is symmetric up to rounding
+    assert np.abs(H - H.T).max() <= 1e-13 * np.linalg.norm(S)
+
+
+def test_encoding_exact_on_integers(ora):
+    rng = np.random.default_rng(3)
+    A = rng.integers(-1000, 1000, size=(37, 37)).astype(np.float64)
+    r, c, k = ora.encode(A)
+    Ai = A.astype(np.int64)
+    assert np.array_equal(r, Ai.sum(axis=1).astype(np.float64))
+    assert np.array_equal(c, Ai.sum(axis=0).astype(np.float64))
+    assert k == float(Ai.sum())
+
+
+# ---------------------------------------------------------------- invariants
+@pytest.mark.parametrize("dist", ["uniform", "normal"])
+def test_similarity_invariants(ora, dist):
+    n = 16
+    A = synth.matrix(n, seed=99, dist=dist)
+    Ao, tau = ora.dgehd2(A)
+    H = np.triu(Ao, -1)
+    Q = ora.dorghr(Ao, tau)
+    assert abs(np.trace(H) - np.trace(A)) <= 10 * n * EPS * np.linalg.norm(A)
+    assert abs(np.linalg.norm(H) - np.linalg.norm(A)) <= 10 * n * EPS * np.linalg.norm(A)
+    ea = np.sort_complex(np.linalg.eigvals(A))
+    eh = np.sort_complex(np.linalg.eigvals(H))
+    assert np.abs(ea - eh).max() <= 1e-10 * np.linalg.norm(A)
+    e1 = np.zeros(n); e1[0] = 1.0
+    assert np.array_equal(Q @ e1, e1) and np.array_equal(Q[0], e1)
+    assert resid_ratio(A, H, Q) <= 30
+    assert orth_ratio(Q) <= 30
+
+
+@pytest.mark.parametrize("n", [256, 400])
+def test_residual_and_orthogonality_paper_magnitudes(ora, n):
+    """Table II / III: MAGMA-level residuals ~1e-18..1e-17, orthogonality ~4e-17."""
+    A = synth.matrix(n)
+    Ao, tau = ora.dgehd2(A)
+    H = np.triu(Ao, -1)
+    Q = ora.dorghr(Ao, tau)
+    paper_res = np.linalg.norm(A - Q @ H @ Q.T, 1) / (n * np.linalg.norm(A, 1))
+    paper_orth = np.linalg.norm(Q @ Q.T - np.eye(n), 1) / n
+    assert paper_res < 1e-16 and paper_orth < 1e-15
+    assert resid_ratio(A, H, Q) <= 30 and orth_ratio(Q) <= 30
+
+
+# ---------------------------------------------------------------- ABFT bookkeeping
+def _logical(Ao, ilo, ihi, cdone):
+    n = Ao.shape[0]
+    L = Ao.copy()
+    for j in range(max(ilo - 1, 0), min(cdone, ihi - 1)):
+        L[j + 2: ihi, j] = 0.0
+    return L
+
+
+@pytest.mark.parametrize("n,nb,dist,ilo,ihi", [(64, 16, "uniform", 1, 64), (200, 32, "normal", 1, 200),
+                                               (150, 32, "uniform", 4, 131)])
+def test_theorem1_checksums_at_every_boundary(ora, n, nb, dist, ilo, ihi):
+    """Theorem 1: r = L e and c = e^T L stay valid; kappa = e^T L e (R22)."""
+    A = synth.matrix(n, dist=dist, ilo=ilo, ihi=ihi)
+    normF = np.linalg.norm(A)
+    npanel = (ihi - 2 - (ilo - 1) + nb) // nb
+    for t in range(npanel):
+        info, Aw, tau, rep, chk = ora.ft_dgehd2(A, nb, ilo, ihi, stop_after_panel=t)
+        assert info == 0
+        cdone = min(ilo - 1 + (t + 1) * nb, ihi - 1)
+        L = _logical(Aw, ilo, ihi, cdone)
+        r, c, k = chk[:n], chk[n:2 * n], chk[2 * n]
+        unit = n * EPS * normF
+        assert np.abs(r - L.sum(axis=1)).max() <= 0.5 * unit
+        assert np.abs(c - L.sum(axis=0)).max() <= 0.5 * unit
+        assert abs(k - L.sum()) <= 0.5 * unit * np.sqrt(n)
+    # the fault-free run leaves A identical to the plain reduction and reports nothing
+    info, Af, tauf, rep, _ = ora.ft_dgehd2(A, nb, ilo, ihi)
+    Ao, tau = ora.dgehd2(A, ilo, ihi)
+    assert info == 0 and rep.detected == 0 and rep.nevents == 0
+    assert np.array_equal(Af, Ao) and np.array_equal(tauf, tau)
+    assert rep.max_drift < 0.5
+
+
+# ---------------------------------------------------------------- injector
+@pytest.mark.parametrize("bit", [0, 30, 51, 52, 62, 63])
+def test_flip_is_one_bit(ora, bit):
+    x = 0.7312
+    y = ora.flip(x, bit)
+    a = np.array([x]).view(np.uint64)[0]
+    b = np.array([y]).view(np.uint64)[0]
+    assert bin(int(a ^ b)).count("1") == 1 and int(a ^ b) == 1 << bit
+
+
+# ---------------------------------------------------------------- decoder truth tables
+def _decoder_case(ora, n=8, seed=0):
+    A = synth.matrix(n, seed=seed, dist="normal")
+    r, c, k = ora.encode(A)
+    tau = 2.0 * n * EPS * np.linalg.norm(A)
+    return A, r, c, k, tau
+
+
+def _apply(A, r, c, k, site, bit, ora):
+    A, r, c = A.copy(order="F"), r.copy(), c.copy()
+    kind, i, j = site
+    if kind == "A":
+        A[i, j] = ora.flip(A[i, j], bit)
+    elif kind == "r":
+        r[i] = ora.flip(r[i], bit)
+    elif kind == "c":
+        c[j] = ora.flip(c[j], bit)
+    else:
+        k = ora.flip(k, bit)
+    return A, r, c, k
+
+
+def _sites(n):
+    s = [("A", i, j) for i in range(n) for j in range(n)]
+    s += [("r", i, -1) for i in range(n)] + [("c", -1, j) for j in range(n)] + [("k", -1, -1)]
+    return s
+
+
+def _exact(A0, r0, c0, k0, L, r, c, k, n):
+    scale = n * EPS * max(1.0, np.abs(A0).max()) * 8
+    return (np.abs(L - A0).max() <= scale and np.abs(r - r0).max() <= scale * n
+            and np.abs(c - c0).max() <= scale * n and abs(k - k0) <= scale * n * n)
+
+
+@pytest.mark.parametrize("seed", [0, 1, 2])
+def test_decoder_every_single_fault_corrected(ora, seed):
+    n = 8
+    A, r, c, k, tau = _decoder_case(ora, n, seed)
+    for site in _sites(n):
+        for bit in (45, 51, 62, 63):
+            Af, rf, cf, kf = _apply(A, r, c, k, site, bit, ora)
+            res, L, r2, c2, k2, rep = ora.decode(Af, rf, cf, kf, tau)
+            assert res == 1, (site, bit, rep.events())
+            assert _exact(A, r, c, k, L, r2, c2, k2, n), (site, bit)
+
+
+@pytest.mark.parametrize("seed", [0, 1, 2])
+def test_decoder_never_miscorrects_two_faults(ora, seed):
+    """Brute force over every pair of fault sites x bit pairs (R12): exact or refused."""
+    n = 8
+    A, r, c, k, tau = _decoder_case(ora, n, seed)
+    sites = _sites(n)
+    bitpairs = [(45, 51), (51, 51), (62, 45), (63, 51), (52, 60), (62, 63)]
+    corrected = refused = 0
+    for s1, s2 in itertools.combinations(sites, 2):
+        for b1, b2 in bitpairs:
+            Af, rf, cf, kf = _apply(A, r, c, k, s1, b1, ora)
+            Af, rf, cf, kf = _apply(Af, rf, cf, kf, s2, b2, ora)
+            res, L, r2, c2, k2, rep = ora.decode(Af, rf, cf, kf, tau)
+            if res == 1:
+                assert _exact(A, r, c, k, L, r2, c2, k2, n), (s1, s2, b1, b2, rep.events())
+                corrected += 1
+            else:
+                assert res == 2, (s1, s2, b1, b2)
+                refused += 1
+    assert corrected > 0.8 * (corrected + refused)
+
+
+def test_decoder_refuses_rectangle_and_l_shape(ora):
+    """errors forming a rectangle are not correctable.  A tied rectangle and an
+    L-shape whose syndromes pair with nothing must be refused.  (With one checksum
+    pair some 3-error patterns have exactly the syndrome of a 2-error pattern; no
+    decoder can tell them apart -- DESIGN.md, decoder limits.)"""
+    n = 8
+    A, r, c, k, tau = _decoder_case(ora, n, 5)
+    for pattern in ([(1, 2, 0.25), (1, 5, 0.25), (4, 2, 0.25), (4, 5, 0.25)],
+                    [(1, 2, 0.25), (1, 5, 0.5), (4, 2, 1.0)]):
+        Af = A.copy(order="F")
+        for (i, j, d) in pattern:
+            Af[i, j] += d
+        res, *_ = ora.decode(Af, r, c, k, tau)
+        assert res == 2
+
+
+# ---------------------------------------------------------------- end-to-end fault runs
+def _fault_free(ora, A, nb, ilo=1, ihi=None):
+    Ao, tau = ora.dgehd2(A, ilo, ihi if ihi else A.shape[0])
+    return Ao, tau
+
+
+@pytest.mark.parametrize("site,i,j,bit", [
+    (0, 40, 50, 51),    # C1 default: area 2 at panel 1, bit 51
+    (0, 5, 50, 62),     # area 1 (rows above the panel), catastrophic exponent flip
+    (0, 40, 50, 63),    # sign
+    (0, 20, 16, 45),    # panel column being factorised next
+    (1, 33, -1, 55),    # r
+    (2, -1, 61, 52),    # c
+    (3, -1, -1, 48),    # kappa
+])
+def test_c1_single_fault_corrected(ora, site, i, j, bit):
+    n, nb = 64, 16
+    A = synth.matrix(n)
+    Ao, tau = _fault_free(ora, A, nb)
+    info, Af, tauf, rep, _ = ora.ft_dgehd2(A, nb, faults=[(1, site, i, j, bit)])
+    assert info == 0, rep.events()
+    ev = rep.events()
+    assert any(e[0] == "DETECT" and e[1] == 1 for e in ev)
+    if site == 0:
+        assert any(e[0] == "FIX_DATA" and e[2] == i and e[3] == j for e in ev)
+    H, Hf = np.triu(Ao, -1), np.triu(Af, -1)
+    assert np.abs(H - Hf).max() / np.abs(H).max() <= 1e-12
+    assert np.abs(tau - tauf).max() <= 1e-12
+
+
+def test_area3_fault_corrected_at_end(ora):
+    n, nb = 64, 16
+    A = synth.matrix(n)
+    Ao, tau = _fault_free(ora, A, nb)
+    # stored Householder vector (finished column 3) hit at boundary 2 (area 3)
+    info, Af, tauf, rep, _ = ora.ft_dgehd2(A, nb, faults=[(2, 0, 30, 3, 50)])
+    assert info == 0
+    assert any(e[0] == "FIX_Q" and e[2] == 30 and e[3] == 3 for e in rep.events())
+    assert np.abs(Af - Ao).max() <= 1e-14
+
+
+def test_finished_h_fault_corrected_at_end(ora):
+    n, nb = 64, 16
+    A = synth.matrix(n)
+    Ao, tau = _fault_free(ora, A, nb)
+    info, Af, tauf, rep, _ = ora.ft_dgehd2(A, nb, faults=[(-1, 0, 3, 10, 50)])
+    assert info == 0
+    assert any(e[0] == "FIX_DATA" and e[1] == -1 for e in rep.events())
+    assert np.abs(np.triu(Af, -1) - np.triu(Ao, -1)).max() <= 1e-13
+
+
+def test_simultaneous_faults(ora):
+    n, nb = 128, 32
+    A = synth.matrix(n, dist="normal")
+    Ao, tau = _fault_free(ora, A, nb)
+    faults = [(2, 0, 80, 100, 55), (2, 0, 90, 110, 47), (2, 2, -1, 120, 52)]
+    info, Af, tauf, rep, _ = ora.ft_dgehd2(A, nb, faults=faults)
+    assert info == 0, rep.events()
+    assert np.abs(np.triu(Af, -1) - np.triu(Ao, -1)).max() <= 1e-12 * np.abs(Ao).max()
+
+
+# ---------------------------------------------------------------- Fig. 2
+def test_fig2_propagation_patterns(ora):
+    """ABFT off (threshold disabled), one error after iteration 1, N=158, nb=32."""
+    n, nb = 158, 32
+    A = synth.matrix(n)
+    Ao, tau = ora.dgehd2(A)
+    off = 1e300  # no detection: the error propagates as in the paper's heat maps
+
+    def diff(i, j):
+        info, Af, tf, rep, _ = ora.ft_dgehd2(A, nb, c_thr=off, faults=[(1, 0, i, j, 52)])
+        return np.abs(Af - Ao) > 1e-12 * np.abs(Ao).max()
+
+    d = diff(53, 16)           # area 3: finished Householder vector, does not propagate
+    assert d.sum() == 1 and d[53, 16]
+    d = diff(31, 127)          # area 1: pollutes one row of H (row 31, columns after the panel)
+    rows = np.unique(np.nonzero(d)[0])
+    assert list(rows) == [31] and d[31, 33:].mean() > 0.9
+    d = diff(63, 127)          # area 2: pollutes almost all of H after column 32, and much of Q
+    H = np.triu(np.ones((n, n), bool), -1)
+    assert d[:, 33:][H[:, 33:]].mean() > 0.9
+    assert d[:, 33:][~H[:, 33:]].mean() > 0.3
