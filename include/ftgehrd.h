@@ -1,0 +1,149 @@
+/*
+ * ftgehrd.h -- C ABI of the B200-native ABFT Hessenberg reduction.
+ *
+ * Method: Jia, Luszczek, Dongarra, "Hessenberg Reduction with Transient Error
+ * Resilience on GPU-Based Hybrid Architectures", IPDPSW 2016.  "P:N" below is
+ * a line of that paper's text; "R#" a reading in DESIGN.md.
+ *
+ * All matrices are column-major FP64.  Pointers named d* are DEVICE pointers
+ * (cudaMalloc / torch CUDA tensors) owned by the caller; the library never
+ * frees them.  h* pointers are HOST pointers (pinned memory recommended).
+ * Library workspace (augmented array, checkpoint, V/Y/T/W panels, checksum
+ * vectors) is cached per device and released by ft_finalize().
+ *
+ * Return value (LAPACK style "info"):
+ *    0                 success (possibly after correcting soft errors; see report)
+ *   -i                 argument i is illegal (1 n, 2 ilo, 3 ihi, 4 A, 5 lda,
+ *                      6 tau, 7 opts / an opts field, 8 Q, 9 ldq)
+ *    FT_E_UNCORRECTABLE a detected discrepancy could not be decoded (R12);
+ *                      A and tau are undefined, the report holds the events
+ *    FT_E_CUDA / FT_E_NCCL / FT_E_NOMEM   runtime failures
+ * Every call returns only after its stream has finished (info depends on the
+ * device-side verification outcome).
+ */
+#ifndef FTGEHRD_H
+#define FTGEHRD_H
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define FT_E_UNCORRECTABLE 1
+#define FT_E_CUDA 2
+#define FT_E_NCCL 3
+#define FT_E_NOMEM 4
+
+/* Fault-injection phases within panel iteration t (Alg. 3):
+ *   BEFORE_PANEL  start of iteration t, before its checkpoint (the paper's Fig. 2
+ *                 "after iteration t-1, before iteration t")
+ *   AFTER_PANEL   after the panel factorization (DLAHR2, Alg. 3 l.5-7), before the updates
+ *   AFTER_RIGHT   after the right update (Alg. 3 l.8-10), before the left update (l.11)
+ *   AFTER_UPDATE  after the left update, before the end-of-iteration check (l.12)
+ *   AT_END        after the last iteration, before the final verification (panel ignored) */
+enum { FT_PHASE_BEFORE_PANEL = 0, FT_PHASE_AFTER_PANEL = 1, FT_PHASE_AFTER_RIGHT = 2,
+       FT_PHASE_AFTER_UPDATE = 3, FT_PHASE_AT_END = 4 };
+
+/* Fault sites (failure model P:48-52; areas of Fig. 2a):
+ *   A   working-array word A(i,j): area 1 (rows above the panel), area 2
+ *       (trailing matrix), area 3 (finished Householder vectors) or finished H
+ *   R   row-checksum r(i)        (Ar_chk)
+ *   C   column-checksum c(j)     (Ac_chk)
+ *   K   corner kappa = e^T L e   (R22)
+ *   Y   panel workspace Y(i,j)   (j = column within the panel; R15)
+ *   V   panel workspace V(i,j)   (the copy the updates read; R15) */
+enum { FT_SITE_A = 0, FT_SITE_R = 1, FT_SITE_C = 2, FT_SITE_K = 3, FT_SITE_Y = 4, FT_SITE_V = 5 };
+
+typedef struct {
+    int32_t panel;  /* iteration t >= 0 (ignored for AT_END) */
+    int32_t phase;  /* FT_PHASE_* */
+    int32_t site;   /* FT_SITE_* */
+    int32_t bit;    /* 0..63: XOR this bit of the binary64 word */
+    int64_t i, j;   /* 0-based position (j unused for R, i unused for C) */
+} ft_fault;
+
+enum { FT_EV_INJECT = 0, FT_EV_DETECT = 1, FT_EV_FIX_DATA = 2, FT_EV_FIX_R = 3, FT_EV_FIX_C = 4,
+       FT_EV_FIX_K = 5, FT_EV_FIX_Q = 6, FT_EV_FIX_QR = 7, FT_EV_FIX_QC = 8, FT_EV_FIX_QK = 9,
+       FT_EV_UNCORRECTABLE = 10, FT_EV_ROLLBACK = 11, FT_EV_PANEL_REDO = 12 };
+
+typedef struct {
+    int32_t kind, panel;  /* FT_EV_*, iteration (-1 = final verification) */
+    int64_t i, j;         /* position (DETECT: i = #flagged rows, j = #flagged cols) */
+    double delta;         /* INJECT: new - old; FIX_*: repaired - corrupted */
+} ft_event;
+
+#define FT_MAX_EVENTS 256
+typedef struct {
+    int32_t detected, corrected, rollbacks, panel_redos, uncorrectable, nevents;
+    double max_drift_rel;       /* max |maintained - recomputed| / (n eps ||A||_F) seen */
+    double ms[8];               /* per-phase device ms: 0 total, 1 panel, 2 right, 3 left,
+                                   4 verify, 5 recovery, 6 copy, 7 encode */
+    ft_event events[FT_MAX_EVENTS];
+} ft_report;
+
+enum { FT_POLICY_EAGER = 0, FT_POLICY_PAPER = 1 };
+
+typedef struct {
+    int32_t nb;          /* panel width; 0 -> 32 if n < 4096 else 64 (R4); max 64      */
+    int32_t abft;        /* 0 = fault-prone baseline (no checksums), 1 = protected     */
+    int32_t weighted;    /* reserved (weighted checksum pair, NEXT-1); must be 0       */
+    int32_t policy;      /* FT_POLICY_EAGER (default) or FT_POLICY_PAPER (R11)         */
+    double c_thr;        /* threshold constant; 0 -> 2.0; tau_abs = c_thr*n*eps*||A||_F (R10) */
+    const ft_fault *faults;   /* host array, may be NULL                                 */
+    int32_t nfaults;
+    ft_report *report;        /* optional host output                                    */
+    int32_t stop_after_panel; /* verify hook: -1 = run to the end; t >= 0 = stop after
+                                 iteration t, copy the WORKING matrix (H/V so far, trailing
+                                 part updated) to dA and the maintained checksums
+                                 [r(0:n) | c(0:n) | kappa] to dchk_out                   */
+    double *dchk_out;         /* device buffer of 2n+1 doubles, or NULL                  */
+    void *stream;             /* cudaStream_t; NULL -> the legacy default stream          */
+} ft_opts;
+
+/* Fill *o with defaults (nb 0, abft 1, policy EAGER, c_thr 2, no faults, run to end). */
+void ft_opts_default(ft_opts *o);
+
+/* Reduce A to upper Hessenberg form H = Q^T A Q (LAPACK DGEHRD semantics, P:38-42,
+ * Alg. 3).  On exit H is on and above the first subdiagonal of dA and the
+ * Householder vectors v(i+2:ihi) of H(i) = I - tau(i) v v^T are stored below it
+ * (v(i+1) = 1 implicit).  dtau has n-1 entries; tau(1:ilo-1) = tau(ihi:n-1) = 0.
+ * 1 <= ilo <= ihi <= n (n = 0: ilo = 1, ihi = 0); A is assumed upper triangular
+ * in rows/columns 1:ilo-1 and ihi+1:n.  lda >= max(1, n). */
+int ft_dgehrd(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opts *opts);
+
+/* Same contract with HOST buffers hA / htau: the host->device copy of A, the
+ * reduction and the device->host copy of H/V and tau all run inside the call
+ * (the end-to-end entry point bench.py times). */
+int ft_dgehrd_host(int n, int ilo, int ihi, double *hA, int lda, double *htau, const ft_opts *opts);
+
+/* Form the explicit orthogonal Q = H(ilo) H(ilo+1) ... H(ihi-1) from the output
+ * of ft_dgehrd (LAPACK DORGHR semantics; Q is the identity outside rows/cols
+ * ilo..ihi and Q e1 = e1 when ilo = 1).  dQ may alias dA only if ldq == lda.
+ * opts may be NULL (only opts->nb and opts->stream are read). */
+int ft_dorghr(int n, int ilo, int ihi, const double *dA, int lda, const double *dtau,
+              double *dQ, int ldq, const ft_opts *opts);
+
+/* Multi-GPU entry (1-D block-column cyclic, block = nb): global column J lives on
+ * rank (J/nb) mod nranks at local column (J/(nb*nranks))*nb + J mod nb; each rank
+ * passes its n x ncols_local slab.  nccl_comm is an ncclComm_t (or NULL with
+ * nranks == 1).  tau is replicated on return.  (Round 1: nranks == 1 only.) */
+int ft_dgehrd_mgpu(int n, int ilo, int ihi, double *dA_local, int lda_local, double *dtau,
+                   void *nccl_comm, int rank, int nranks, const ft_opts *opts);
+
+/* Human-readable text for an info code. */
+const char *ft_strerror(int info);
+
+/* Release all cached device workspace. */
+void ft_finalize(void);
+
+/* Library build / capability string (arch, version). */
+const char *ft_version(void);
+
+/* Kernel-launch counter (for the bench's gpu_launches claim): number of kernels this
+ * library has launched since load / the last reset. */
+int64_t ft_launch_count(int reset);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

@@ -1,0 +1,515 @@
+// ft_abft.cu -- checksum encode / verify / locate / correct / inject kernels and
+// small utilities of the product path.
+//
+//   encode            r = A e, c = e^T A, kappa = e^T A e      P:218-224 (Sec. IV-B, Fig. 3), R22
+//   pre-update check  e^T Y vs Y_chk, e^T V vs V_chk             R15 (extends Alg. 3 l.6-7)
+//   end check         |sum r - kappa|, |sum c - kappa|           P:256-260 (Alg. 3 l.12-13), R11
+//   full verify       D_r = r - L e, D_c = c - e^T L             P:272 (Sec. IV-F, location)
+//   fix               A(i,j) = r(i) - sum_{k!=j} A(i,k) (or col)
+//   inject            XOR one bit of a binary64 word             P:48-52 failure model, R16
+#include "ft_common.cuh"
+#include "ft_internal.h"
+
+static const double EPS = 2.220446049250313e-16;
+
+__global__ void k_copy_in(const double *__restrict__ A, int lda, double *__restrict__ Aw, int64_t ldw, int n) {
+    int64_t j = blockIdx.y;
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x)
+        Aw[i + j * ldw] = A[i + j * (int64_t)lda];
+}
+cudaError_t ft_copy_in(const double *A, int lda, double *Aw, int64_t ldw, int n, cudaStream_t s) {
+    if (n <= 0) return cudaSuccess;
+    g_ft_launches++;
+    k_copy_in<<<dim3((n + 255) / 256 < 8 ? (n + 255) / 256 : 8, n), 256, 0, s>>>(A, lda, Aw, ldw, n);
+    return cudaGetLastError();
+}
+__global__ void k_copy_out(const double *__restrict__ Aw, int64_t ldw, double *__restrict__ A, int lda, int n) {
+    int64_t j = blockIdx.y;
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x)
+        A[i + j * (int64_t)lda] = Aw[i + j * ldw];
+}
+cudaError_t ft_copy_out(const double *Aw, int64_t ldw, double *A, int lda, int n, cudaStream_t s) {
+    if (n <= 0) return cudaSuccess;
+    g_ft_launches++;
+    k_copy_out<<<dim3((n + 255) / 256 < 8 ? (n + 255) / 256 : 8, n), 256, 0, s>>>(Aw, ldw, A, lda, n);
+    return cudaGetLastError();
+}
+
+// ---------------------------------------------------------------------------
+// encode: row sums (thread per row), column sums (warp per column), ||A||_F^2
+// ---------------------------------------------------------------------------
+__global__ void k_encode_rows(double *Aw, int64_t ldw, int n, double *sq_part) {
+    int i = blockIdx.x * blockDim.x + threadIdx.x;
+    double s = 0.0, q = 0.0;
+    if (i < n) {
+        for (int j = 0; j < n; j++) {
+            double a = Aw[i + (int64_t)j * ldw];
+            s += a;
+            q += a * a;
+        }
+        Aw[i + (int64_t)n * ldw] = s;  // r(i) in column n
+    }
+    q = warp_sum(q);
+    __shared__ double ws[32];
+    if ((threadIdx.x & 31) == 0) ws[threadIdx.x >> 5] = q;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double t = 0.0;
+        for (int w = 0; w < (int)(blockDim.x >> 5); w++) t += ws[w];
+        sq_part[blockIdx.x] = t;
+    }
+}
+__global__ void k_encode_cols(double *Aw, int64_t ldw, int n) {
+    int j = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+    int lane = threadIdx.x & 31;
+    if (j >= n) return;
+    double s = 0.0;
+    for (int i = lane; i < n; i += 32) s += Aw[i + (int64_t)j * ldw];
+    s = warp_sum(s);
+    if (lane == 0) Aw[n + (int64_t)j * ldw] = s;  // c(j) in row n
+}
+__global__ void k_encode_finish(double *Aw, int64_t ldw, int n, const double *sq_part, int nparts, FtCtl *ctl) {
+    // kappa = sum r (fixed order), ||A||_F
+    __shared__ double ws[32];
+    double s = 0.0;
+    for (int i = threadIdx.x; i < n; i += blockDim.x) s += Aw[i + (int64_t)n * ldw];
+    s = warp_sum(s);
+    if ((threadIdx.x & 31) == 0) ws[threadIdx.x >> 5] = s;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double k = 0.0;
+        for (int w = 0; w < (int)(blockDim.x >> 5); w++) k += ws[w];
+        Aw[n + (int64_t)n * ldw] = k;
+        double q = 0.0;
+        for (int b = 0; b < nparts; b++) q += sq_part[b];
+        ctl->normF = sqrt(q);
+    }
+}
+// frozen row sums before the first panel: columns 0..ilo-2 are final (R5/R6)
+__global__ void k_frozen_init(const double *Aw, int64_t ldw, int n, int ncols, double *Fr) {
+    int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    double s = 0.0;
+    for (int j = 0; j < ncols; j++) s += Aw[i + (int64_t)j * ldw];
+    Fr[i] = s;
+}
+cudaError_t ft_frozen_init(const double *Aw, int64_t ldw, int n, int ncols, double *Fr, cudaStream_t s) {
+    g_ft_launches++;
+    k_frozen_init<<<(n + 255) / 256, 256, 0, s>>>(Aw, ldw, n, ncols, Fr);
+    return cudaGetLastError();
+}
+cudaError_t ft_encode(double *Aw, int64_t ldw, int n, FtCtl *ctl, double *scratch, cudaStream_t s) {
+    if (n <= 0) return cudaSuccess;
+    int nb = (n + 255) / 256;
+    g_ft_launches += 3;
+    k_encode_rows<<<nb, 256, 0, s>>>(Aw, ldw, n, scratch);
+    k_encode_cols<<<(n + 7) / 8, 256, 0, s>>>(Aw, ldw, n);
+    k_encode_finish<<<1, 1024, 0, s>>>(Aw, ldw, n, scratch, nb, ctl);
+    return cudaGetLastError();
+}
+
+// ||A||_F only (ABFT off still reports drift in units of ||A||_F)
+__global__ void k_frob(const double *A, int lda, int n, FtCtl *ctl) {
+    __shared__ double ws[32];
+    double q = 0.0;
+    for (int64_t idx = threadIdx.x; idx < (int64_t)n * n; idx += blockDim.x) {
+        double a = A[(idx % n) + (idx / n) * (int64_t)lda];
+        q += a * a;
+    }
+    q = warp_sum(q);
+    if ((threadIdx.x & 31) == 0) ws[threadIdx.x >> 5] = q;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double t = 0.0;
+        for (int w = 0; w < (int)(blockDim.x >> 5); w++) t += ws[w];
+        ctl->normF = sqrt(t);
+    }
+}
+cudaError_t ft_frob_to_ctl(const double *A, int lda, int n, FtCtl *ctl, cudaStream_t s) {
+    g_ft_launches++;
+    k_frob<<<1, 1024, 0, s>>>(A, lda, n, ctl);
+    return cudaGetLastError();
+}
+
+// ---------------------------------------------------------------------------
+// pre-update check sums: eY(j) = sum_{i<ihi} Y(i,j), eV(j) = sum_{k+1<=i<ihi} V(i,j)
+// (computed after the AFTER_PANEL injection point; reading R15)
+// ---------------------------------------------------------------------------
+__global__ void k_precheck(const double *Y, const double *V, int64_t ldw, int ihi, int k, int ib, FtCtl *ctl) {
+    if (ctl->halt) return;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    const int rows_per = 256;
+    const int i0 = blockIdx.x * rows_per, i1 = min(ihi, i0 + rows_per);
+    for (int j = wid; j < ib; j += nw) {
+        double sy = 0.0, sv = 0.0;
+        for (int i = i0 + lane; i < i1; i += 32) {
+            sy += Y[i + (int64_t)j * ldw];
+            if (i >= k + 1) sv += V[i + (int64_t)j * ldw];
+        }
+        sy = warp_sum(sy);
+        sv = warp_sum(sv);
+        if (lane == 0) {
+            atomicAdd(&ctl->eY[j], sy);
+            atomicAdd(&ctl->eV[j], sv);
+        }
+    }
+}
+cudaError_t ft_precheck(const double *Y, const double *V, int64_t ldw, int n, int ihi, int k, int ib,
+                        FtCtl *ctl, cudaStream_t s) {
+    int nblk = (ihi + 255) / 256;
+    g_ft_launches++;
+    k_precheck<<<nblk, 512, 0, s>>>(Y, V, ldw, ihi, k, ib, ctl);
+    return cudaGetLastError();
+}
+
+// one warp: decide whether to halt before the updates consume the panel's output
+__global__ void k_decide(const double *Y, const double *V, const double *T, int64_t ldw, int n, int k, int ib,
+                         int panel, FtCtl *ctl) {
+    if (ctl->halt) return;
+    const int lane = threadIdx.x;
+    const double unit = (double)n * EPS * ctl->normF;
+    const double c_thr = ctl->c_thr;
+    double tmax = 0.0;
+    for (int i = lane; i < ib * ib; i += 32) {
+        int a = i % ib, b = i / ib;
+        tmax = fmax(tmax, fabs(T[a + b * FT_NBMAX]));
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) tmax = fmax(tmax, __shfl_xor_sync(0xffffffffu, tmax, o));
+    int reason = 0;
+    if (ctl->nflag > 0) reason |= 1;
+    const double tauY = c_thr * unit * (tmax > 1.0 ? tmax : 1.0);
+    const double tauV = c_thr * (double)n * EPS * sqrt((double)n);
+    for (int j = lane; j < ib; j += 32) {
+        double dy = ctl->eY[j] - Y[n + (int64_t)j * ldw];
+        double dv = ctl->eV[j] - V[n + (int64_t)j * ldw];
+        if (not_within(dy, tauY)) reason |= 2;
+        if (not_within(dv, tauV)) reason |= 4;
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) reason |= __shfl_xor_sync(0xffffffffu, reason, o);
+    __syncwarp();
+    if (lane == 0) {
+        if (reason) {
+            ctl->halt_panel = panel;
+            ctl->halt_stage = 1;
+            ctl->halt_reason = reason;
+            __threadfence();
+            ctl->halt = 1;
+        }
+        ctl->nflag = 0;
+    }
+    for (int j = lane; j < FT_NBMAX; j += 32) {
+        ctl->eY[j] = 0.0;
+        ctl->eV[j] = 0.0;
+    }
+}
+cudaError_t ft_decide(const double *Y, const double *V, const double *T, int64_t ldw, int n, int k, int ib,
+                      int panel, FtCtl *ctl, cudaStream_t s) {
+    g_ft_launches++;
+    k_decide<<<1, 32, 0, s>>>(Y, V, T, ldw, n, k, ib, panel, ctl);
+    return cudaGetLastError();
+}
+
+// ---------------------------------------------------------------------------
+// end-of-iteration check (Alg. 3 l.12-13) + frozen-row-sum bookkeeping.
+// Grid-stride blocks; the last block to finish takes the decision.
+//   sum r = sum_{i<n} A(i,n), sum c = sum_{j<n} A(n,j), kappa = A(n,n)
+//   Fr(i) += sum_{col in [k,e), i <= col+1} A(i,col)   for i <= e (columns frozen now)
+// ---------------------------------------------------------------------------
+__global__ void k_endcheck(double *Aw, int64_t ldw, int n, int ihi, int k, int ib, int panel, int policy,
+                           double *Fr, FtCtl *ctl) {
+    if (ctl->halt) return;
+    __shared__ double ws[2][32];
+    __shared__ int last;
+    double sr = 0.0, sc = 0.0;
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+        sr += Aw[i + (int64_t)n * ldw];
+        sc += Aw[n + (int64_t)i * ldw];
+    }
+    sr = warp_sum(sr);
+    sc = warp_sum(sc);
+    if ((threadIdx.x & 31) == 0) {
+        ws[0][threadIdx.x >> 5] = sr;
+        ws[1][threadIdx.x >> 5] = sc;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double a = 0.0, b = 0.0;
+        for (int w = 0; w < (int)(blockDim.x >> 5); w++) {
+            a += ws[0][w];
+            b += ws[1][w];
+        }
+        atomicAdd(&ctl->sums[0], a);
+        atomicAdd(&ctl->sums[1], b);
+        __threadfence();
+        last = (atomicAdd(&ctl->done_count, 1) == (int)gridDim.x - 1);
+    }
+    __syncthreads();
+    if (!last) return;
+    if (threadIdx.x == 0) {
+        __threadfence();
+        double Sr = atomicAdd(&ctl->sums[0], 0.0), Sc = atomicAdd(&ctl->sums[1], 0.0);
+        double kap = Aw[n + (int64_t)n * ldw];
+        double unit = (double)n * EPS * ctl->normF;
+        double tauS = ctl->c_thr * unit * sqrt((double)n);
+        int reason = 0;
+        if (policy == FT_POLICY_PAPER) {
+            if (not_within(Sr - Sc, tauS)) reason |= 8;
+        } else {
+            if (not_within(Sr - kap, tauS) || not_within(Sc - kap, tauS)) reason |= 8;
+        }
+        ctl->sums[0] = 0.0;
+        ctl->sums[1] = 0.0;
+        ctl->done_count = 0;
+        if (reason) {
+            ctl->halt_panel = panel;
+            ctl->halt_stage = 2;
+            ctl->halt_reason = reason;
+            __threadfence();
+            ctl->halt = 1;
+        }
+    }
+}
+// frozen row sums of the panel columns that just became final (rows 0..e; R6)
+__global__ void k_frozen_rows(const double *Aw, int64_t ldw, int n, int k, int e, double *Fr, FtCtl *ctl) {
+    if (ctl->halt) return;
+    int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i > e || i >= n) return;
+    double s = 0.0;
+    for (int col = k; col < e; col++)
+        if (i <= col + 1) s += Aw[i + (int64_t)col * ldw];
+    Fr[i] += s;
+}
+cudaError_t ft_endcheck(double *Aw, int64_t ldw, int n, int ihi, int k, int ib, int panel, int policy,
+                        double *Fr, FtCtl *ctl, cudaStream_t s) {
+    int nblk = (n + 1023) / 1024;
+    if (nblk > 16) nblk = 16;
+    g_ft_launches += 2;
+    k_endcheck<<<nblk, 1024, 0, s>>>(Aw, ldw, n, ihi, k, ib, panel, policy, Fr, ctl);
+    int e = k + ib;
+    k_frozen_rows<<<(e + 1 + 255) / 256, 256, 0, s>>>(Aw, ldw, n, k, e, Fr, ctl);
+    return cudaGetLastError();
+}
+
+// ---------------------------------------------------------------------------
+// fault injector: XOR one bit of one binary64 word (skipped after a halt; once per fault)
+// ---------------------------------------------------------------------------
+__global__ void k_inject(double *addr, int fidx, int bit, FtCtl *ctl) {
+    if (ctl->halt || ctl->inj_done[fidx]) return;
+    unsigned long long u = __double_as_longlong(*addr);
+    double old = *addr;
+    u ^= 1ull << (bit & 63);
+    *addr = __longlong_as_double(u);
+    ctl->inj_delta[fidx] = __longlong_as_double(u) - old;
+    ctl->inj_done[fidx] = 1;
+}
+cudaError_t ft_inject(double *addr, int fidx, int bit, FtCtl *ctl, cudaStream_t s) {
+    g_ft_launches++;
+    k_inject<<<1, 1, 0, s>>>(addr, fidx, bit, ctl);
+    return cudaGetLastError();
+}
+
+// ---------------------------------------------------------------------------
+// full verification over the logical matrix (recovery path and final check).
+// mode 0 (H): L(i,j) = 0 for stored Householder vectors (j in [ilo-1, cdone), j <= ihi-2,
+//             j+2 <= i < ihi), else A(i,j).  r/c are the maintained checksums.
+// mode 1 (Q): L(i,j) = A(i,j) exactly on that V region, 0 elsewhere; r/c = Qr/Qc.
+// Fr (mode 0, optional) is ignored here: the full verify recomputes everything.
+// sums[0] = sum r, sums[1] = sum c.
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ bool in_v(int i, int j, int ilo, int ihi, int cdone) {
+    return j >= ilo - 1 && j < cdone && j <= ihi - 2 && i >= j + 2 && i < ihi;
+}
+__global__ void k_fv_rows(const double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdone, int mode,
+                          const double *r, int64_t rinc, double *Dr) {
+    int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    double s = 0.0;
+    for (int j = 0; j < n; j++) {
+        bool v = in_v(i, j, ilo, ihi, cdone);
+        if (mode == 0 ? !v : v) s += Aw[i + (int64_t)j * ldw];
+    }
+    Dr[i] = r[(int64_t)i * rinc] - s;
+}
+__global__ void k_fv_cols(const double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdone, int mode,
+                          const double *c, int64_t cinc, double *Dc) {
+    int j = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+    int lane = threadIdx.x & 31;
+    if (j >= n) return;
+    double s = 0.0;
+    for (int i = lane; i < n; i += 32) {
+        bool v = in_v(i, j, ilo, ihi, cdone);
+        if (mode == 0 ? !v : v) s += Aw[i + (int64_t)j * ldw];
+    }
+    s = warp_sum(s);
+    if (lane == 0) Dc[j] = c[(int64_t)j * cinc] - s;
+}
+__global__ void k_fv_sums(int n, const double *r, int64_t rinc, const double *c, int64_t cinc, double *sums) {
+    __shared__ double ws[2][32];
+    double a = 0.0, b = 0.0;
+    for (int i = threadIdx.x; i < n; i += blockDim.x) {
+        a += r[(int64_t)i * rinc];
+        b += c[(int64_t)i * cinc];
+    }
+    a = warp_sum(a);
+    b = warp_sum(b);
+    if ((threadIdx.x & 31) == 0) {
+        ws[0][threadIdx.x >> 5] = a;
+        ws[1][threadIdx.x >> 5] = b;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double x = 0.0, y = 0.0;
+        for (int w = 0; w < (int)(blockDim.x >> 5); w++) {
+            x += ws[0][w];
+            y += ws[1][w];
+        }
+        sums[0] = x;
+        sums[1] = y;
+    }
+}
+cudaError_t ft_full_verify(const double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdone, int mode,
+                           const double *r, int64_t rinc, const double *c, int64_t cinc, const double *Fr,
+                           double *Dr, double *Dc, double *sums, cudaStream_t s) {
+    if (n <= 0) return cudaSuccess;
+    g_ft_launches += 3;
+    k_fv_rows<<<(n + 127) / 128, 128, 0, s>>>(Aw, ldw, n, ilo, ihi, cdone, mode, r, rinc, Dr);
+    k_fv_cols<<<(n + 7) / 8, 256, 0, s>>>(Aw, ldw, n, ilo, ihi, cdone, mode, c, cinc, Dc);
+    k_fv_sums<<<1, 1024, 0, s>>>(n, r, rinc, c, cinc, sums);
+    return cudaGetLastError();
+}
+
+// one block per fix: explicit sum excluding the bad element
+__global__ void k_fix(double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdone, int mode, double *r,
+                      int64_t rinc, double *c, int64_t cinc, double *kappa, const FtFix *fixes, double *deltas) {
+    const FtFix f = fixes[blockIdx.x];
+    __shared__ double ws[32];
+    double s = 0.0;
+    const int i0 = (int)f.i, j0 = (int)f.j;
+    if (f.kind == 0 || f.kind == 2) {  // along row i
+        for (int j = threadIdx.x; j < n; j += blockDim.x) {
+            if (f.kind == 0 && j == j0) continue;
+            bool v = in_v(i0, j, ilo, ihi, cdone);
+            if (mode == 0 ? !v : v) s += Aw[i0 + (int64_t)j * ldw];
+        }
+    } else if (f.kind == 1 || f.kind == 3) {  // along column j
+        for (int i = threadIdx.x; i < n; i += blockDim.x) {
+            if (f.kind == 1 && i == i0) continue;
+            bool v = in_v(i, j0, ilo, ihi, cdone);
+            if (mode == 0 ? !v : v) s += Aw[i + (int64_t)j0 * ldw];
+        }
+    } else {  // kappa = sum r
+        for (int i = threadIdx.x; i < n; i += blockDim.x) s += r[(int64_t)i * rinc];
+    }
+    s = warp_sum(s);
+    if ((threadIdx.x & 31) == 0) ws[threadIdx.x >> 5] = s;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double t = 0.0;
+        for (int w = 0; w < (int)(blockDim.x >> 5); w++) t += ws[w];
+        double *dst;
+        double nv;
+        if (f.kind == 0) {
+            dst = Aw + i0 + (int64_t)j0 * ldw;
+            nv = r[(int64_t)i0 * rinc] - t;
+        } else if (f.kind == 1) {
+            dst = Aw + i0 + (int64_t)j0 * ldw;
+            nv = c[(int64_t)j0 * cinc] - t;
+        } else if (f.kind == 2) {
+            dst = r + (int64_t)i0 * rinc;
+            nv = t;
+        } else if (f.kind == 3) {
+            dst = c + (int64_t)j0 * cinc;
+            nv = t;
+        } else {
+            dst = kappa;
+            nv = t;
+        }
+        deltas[blockIdx.x] = nv - *dst;
+        *dst = nv;
+    }
+}
+cudaError_t ft_apply_fixes(double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdone, int mode, double *r,
+                           int64_t rinc, double *c, int64_t cinc, double *kappa, const FtFix *fixes, int nfix,
+                           double *deltas, cudaStream_t s) {
+    if (nfix <= 0) return cudaSuccess;
+    g_ft_launches++;
+    k_fix<<<nfix, 256, 0, s>>>(Aw, ldw, n, ilo, ihi, cdone, mode, r, rinc, c, cinc, kappa, fixes, deltas);
+    return cudaGetLastError();
+}
+
+// ---------------------------------------------------------------------------
+// Q formation helpers (ft_dorghr): dense V from the stored reflectors, and T (DLARFT)
+// ---------------------------------------------------------------------------
+__global__ void k_build_v(const double *Aw, int64_t ldw, double *V, int n, int ihi, int k, int ib) {
+    int i = blockIdx.x * blockDim.x + threadIdx.x;
+    int j = blockIdx.y;
+    if (i >= n || j >= ib) return;
+    int c = k + j;
+    double v = 0.0;
+    if (i == c + 1) v = 1.0;
+    else if (i >= c + 2 && i < ihi) v = Aw[i + (int64_t)c * ldw];
+    V[i + (int64_t)j * ldw] = v;
+}
+cudaError_t ft_build_v(const double *Aw, int64_t ldw, double *V, int n, int ihi, int k, int ib, cudaStream_t s) {
+    g_ft_launches++;
+    k_build_v<<<dim3((n + 255) / 256, ib), 256, 0, s>>>(Aw, ldw, V, n, ihi, k, ib);
+    return cudaGetLastError();
+}
+// T(0:j, j) = -tau_j T(0:j,0:j) (V(:,0:j)^T v_j), T(j,j) = tau_j  (one block; G = V^T V first)
+__global__ void k_larft(const double *V, int64_t ldw, const double *tau, double *T, int ihi, int k, int ib) {
+    extern __shared__ double larft_smem[];
+    double *G = larft_smem, *Ts = larft_smem + FT_NBMAX * FT_NBMAX, *tmp = Ts + FT_NBMAX * FT_NBMAX;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    for (int pidx = wid; pidx < ib * ib; pidx += nw) {
+        int a = pidx % ib, b = pidx / ib;
+        double s = 0.0;
+        if (a < b)
+            for (int i = k + 1 + lane; i < ihi; i += 32) s += V[i + (int64_t)a * ldw] * V[i + (int64_t)b * ldw];
+        s = warp_sum(s);
+        if (lane == 0) G[a + b * FT_NBMAX] = s;
+    }
+    for (int i = threadIdx.x; i < FT_NBMAX * FT_NBMAX; i += blockDim.x) Ts[i] = 0.0;
+    __syncthreads();
+    for (int j = 0; j < ib; j++) {
+        const double tj = tau[k + j];
+        if (threadIdx.x < j) {
+            double s = 0.0;
+            for (int b = threadIdx.x; b < j; b++) s += Ts[threadIdx.x + b * FT_NBMAX] * G[b + j * FT_NBMAX];
+            tmp[threadIdx.x] = -tj * s;
+        }
+        __syncthreads();
+        if (threadIdx.x < j) Ts[threadIdx.x + j * FT_NBMAX] = tmp[threadIdx.x];
+        if (threadIdx.x == 0) Ts[j + j * FT_NBMAX] = tj;
+        __syncthreads();
+    }
+    for (int i = threadIdx.x; i < ib * ib; i += blockDim.x) {
+        int a = i % ib, b = i / ib;
+        T[a + b * FT_NBMAX] = Ts[a + b * FT_NBMAX];
+    }
+}
+cudaError_t ft_larft(const double *V, int64_t ldw, const double *tau, double *T, int n, int ihi, int k, int ib,
+                     cudaStream_t s) {
+    static bool attr = false;
+    const int smem = (2 * FT_NBMAX * FT_NBMAX + FT_NBMAX) * sizeof(double);
+    if (!attr) {
+        cudaError_t e = cudaFuncSetAttribute(k_larft, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+        if (e != cudaSuccess) return e;
+        attr = true;
+    }
+    g_ft_launches++;
+    k_larft<<<1, 512, smem, s>>>(V, ldw, tau, T, ihi, k, ib);
+    return cudaGetLastError();
+}
+__global__ void k_identity(double *Q, int64_t ldq, int n) {
+    int i = blockIdx.x * blockDim.x + threadIdx.x;
+    int64_t j = blockIdx.y;
+    if (i < n) Q[i + j * ldq] = (i == j) ? 1.0 : 0.0;
+}
+cudaError_t ft_set_identity(double *Q, int64_t ldq, int n, cudaStream_t s) {
+    if (n <= 0) return cudaSuccess;
+    g_ft_launches++;
+    k_identity<<<dim3((n + 255) / 256, n), 256, 0, s>>>(Q, ldq, n);
+    return cudaGetLastError();
+}

@@ -1,0 +1,94 @@
+// ft_common.cuh -- device helpers shared by the ftgehrd kernels (product path).
+// No code here is shared with oracle/ (the CPU oracle is a separate program).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#ifndef FT_NBMAX
+#define FT_NBMAX 64  // max panel width (opts.nb <= 64)
+#endif
+#define FT_KPAD (FT_NBMAX + 4)  // smem row stride for K <= 64 operands (conflict-free DMMA frags)
+
+#define FT_DEV __device__ __forceinline__
+
+// ---------------------------------------------------------------------------
+// FP64 tensor-core MMA (sm_80+ mma.sync f64; lowers to DMMA on sm_100a).
+// D(8x8) += A(8x4, row) * B(4x8, col).  Fragment ownership (lane l):
+//   A: a = A[l/4][l%4]      B: b = B[l%4][l/4]      C/D: d0,d1 = C[l/4][2(l%4)+{0,1}]
+// ---------------------------------------------------------------------------
+FT_DEV void dmma_8x8x4(double &d0, double &d1, double a, double b) {
+    asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};\n"
+                 : "+d"(d0), "+d"(d1)
+                 : "d"(a), "d"(b));
+}
+
+// Warp-level tile MMA: acc[MI][NI] (8MI x 8NI) += A(8MI x K) * B(K x 8NI).
+// A element (m,k) at As[m*SA + k] (AK = false) or As[k*SA + m] (AK = true).
+// B element (k,n) at Bs[n*SB + k].  K is a multiple of 4; m0/n0 are the warp
+// tile origin inside the smem tiles.
+template <int MI, int NI, bool AK>
+FT_DEV void warp_mma(double (&acc)[MI][NI][2], const double *As, int SA, const double *Bs, int SB,
+                     int m0, int n0, int K) {
+    const int lane = threadIdx.x & 31;
+    const int lr = lane >> 2, lc = lane & 3;
+#pragma unroll 2
+    for (int k = 0; k < K; k += 4) {
+        double a[MI], b[NI];
+#pragma unroll
+        for (int mi = 0; mi < MI; mi++) {
+            int m = m0 + mi * 8 + lr;
+            a[mi] = AK ? As[(k + lc) * SA + m] : As[m * SA + k + lc];
+        }
+#pragma unroll
+        for (int ni = 0; ni < NI; ni++) {
+            int nn = n0 + ni * 8 + lr;
+            b[ni] = Bs[nn * SB + k + lc];
+        }
+#pragma unroll
+        for (int mi = 0; mi < MI; mi++)
+#pragma unroll
+            for (int ni = 0; ni < NI; ni++) dmma_8x8x4(acc[mi][ni][0], acc[mi][ni][1], a[mi], b[ni]);
+    }
+}
+
+// element coordinates owned by this lane in fragment (mi, ni), v = 0/1
+FT_DEV int frag_row(int mi) { return mi * 8 + ((threadIdx.x & 31) >> 2); }
+FT_DEV int frag_col(int ni, int v) { return ni * 8 + 2 * (threadIdx.x & 3) + v; }
+
+// ---------------------------------------------------------------------------
+// Grid barrier for a cooperative (co-resident) launch: monotonic arrival
+// counter, release/acquire at gpu scope.  `epoch` counts barriers passed by
+// this CTA; the counter must be zero at launch.
+// ---------------------------------------------------------------------------
+FT_DEV unsigned ld_acquire_u32(const unsigned *p) {
+    unsigned v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];\n" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+FT_DEV void red_release_add_u32(unsigned *p, unsigned v) {
+    asm volatile("red.release.gpu.global.add.u32 [%0], %1;\n" ::"l"(p), "r"(v) : "memory");
+}
+FT_DEV void grid_barrier(unsigned *count, unsigned &epoch, unsigned nblocks) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        epoch += 1;
+        const unsigned target = epoch * nblocks;
+        __threadfence();
+        red_release_add_u32(count, 1u);
+        while (ld_acquire_u32(count) < target) {
+        }
+        __threadfence();
+    }
+    __syncthreads();
+}
+
+// L2-coherent loads for data written by other CTAs inside the same launch
+FT_DEV double ldcg(const double *p) { return __ldcg(p); }
+
+FT_DEV double warp_sum(double v) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    return v;
+}
+
+FT_DEV bool not_within(double d, double tau) { return !(fabs(d) <= tau); }  // NaN -> true

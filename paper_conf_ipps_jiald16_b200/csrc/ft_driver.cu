@@ -1,0 +1,968 @@
+// ft_driver.cu -- host orchestrator and C ABI of libftgehrd (FT_DGEHRD, Alg. 3 P:216,
+// re-designed all-GPU: panel, updates, checksums, verification and injector all run in
+// this library's kernels; the host only enqueues them and, on a detected error, drives
+// the recovery (reverse computation P:260/P:316, location P:272, correction P:278).
+//
+// Fault-free calls enqueue every iteration back to back with no host synchronization:
+// each kernel first reads a device "halt" word, and a check kernel that detects an
+// inconsistency raises it, turning every later kernel of the call into a no-op.  The
+// host reads the control block once at the end; if it finds a halt it recovers the
+// iteration that raised it and re-enqueues from there.
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <map>
+#include <vector>
+
+#include "ft_internal.h"
+
+int64_t g_ft_launches = 0;
+
+namespace {
+
+const double kEps = 2.220446049250313e-16;
+
+#define CK(x)                                        \
+    do {                                             \
+        cudaError_t e_ = (x);                        \
+        if (e_ != cudaSuccess) {                     \
+            if (getenv("FT_DEBUG"))                  \
+                fprintf(stderr, "ftgehrd: %s at %s:%d\n", cudaGetErrorString(e_), __FILE__, __LINE__); \
+            return FT_E_CUDA;                        \
+        }                                            \
+    } while (0)
+
+// ---------------------------------------------------------------------------
+// workspace (cached per device, grown on demand)
+// ---------------------------------------------------------------------------
+constexpr int kMaxWsplit = 16;
+constexpr int kYtopRows = 296 * 64;  // max (Y_top splits x rows) kept in ypart
+
+struct Work {
+    int n_cap = -1;
+    int64_t ldw = 0;
+    double *Aw = nullptr, *V = nullptr, *Y = nullptr, *T = nullptr, *Wpart = nullptr, *bvec = nullptr,
+           *acc = nullptr, *ckpt = nullptr, *ck_r = nullptr, *ck_c = nullptr, *ck_q = nullptr, *Fr = nullptr,
+           *Qr = nullptr, *Qc = nullptr, *Dr = nullptr, *Dc = nullptr, *sums = nullptr, *ypart = nullptr,
+           *rowpart = nullptr, *scratch = nullptr, *deltas = nullptr, *hA = nullptr, *htau = nullptr;
+    unsigned *bar = nullptr;
+    FtCtl *ctl = nullptr;
+    FtFix *fixes = nullptr;
+    int nsm = 0;
+    size_t bytes = 0;
+    void release() {
+        double **ps[] = {&Aw, &V, &Y, &T, &Wpart, &bvec, &acc, &ckpt, &ck_r, &ck_c, &ck_q, &Fr, &Qr, &Qc, &Dr, &Dc,
+                         &sums, &ypart, &rowpart, &scratch, &deltas, &hA, &htau};
+        for (auto p : ps) {
+            if (*p) cudaFree(*p);
+            *p = nullptr;
+        }
+        if (bar) cudaFree(bar);
+        if (ctl) cudaFree(ctl);
+        if (fixes) cudaFree(fixes);
+        bar = nullptr;
+        ctl = nullptr;
+        fixes = nullptr;
+        n_cap = -1;
+        bytes = 0;
+    }
+};
+std::map<int, Work> g_work;
+
+template <class T>
+cudaError_t dalloc(T **p, size_t count, size_t &acc) {
+    acc += count * sizeof(T);
+    return cudaMalloc((void **)p, std::max<size_t>(count, 1) * sizeof(T));
+}
+
+int get_work(int n, Work **out) {
+    int dev = 0;
+    CK(cudaGetDevice(&dev));
+    Work &w = g_work[dev];
+    if (w.n_cap >= n) {
+        *out = &w;
+        return 0;
+    }
+    w.release();
+    int64_t ldw = ((int64_t)n + 2 + 31) / 32 * 32;
+    size_t N1 = (size_t)n + 1;
+    size_t b = 0;
+    cudaError_t e = cudaSuccess;
+    auto A = [&](cudaError_t x) {
+        if (x != cudaSuccess && e == cudaSuccess) e = x;
+    };
+    A(dalloc(&w.Aw, (size_t)ldw * (N1 + 1), b));
+    A(dalloc(&w.V, (size_t)ldw * FT_NBMAX, b));
+    A(dalloc(&w.Y, (size_t)ldw * FT_NBMAX, b));
+    A(dalloc(&w.T, (size_t)FT_NBMAX * FT_NBMAX, b));
+    A(dalloc(&w.Wpart, (size_t)kMaxWsplit * (N1 + 64) * FT_NBMAX, b));
+    A(dalloc(&w.bvec, (size_t)ldw, b));
+    A(dalloc(&w.acc, (size_t)3 * FT_ACC_STRIDE, b));
+    A(dalloc(&w.ckpt, (size_t)ldw * FT_NBMAX, b));
+    A(dalloc(&w.ck_r, (size_t)ldw, b));
+    A(dalloc(&w.ck_c, N1, b));
+    A(dalloc(&w.ck_q, 3 * (size_t)ldw, b));
+    A(dalloc(&w.Fr, (size_t)ldw, b));
+    A(dalloc(&w.Qr, (size_t)ldw, b));
+    A(dalloc(&w.Qc, (size_t)ldw, b));
+    A(dalloc(&w.Dr, (size_t)ldw, b));
+    A(dalloc(&w.Dc, (size_t)ldw, b));
+    A(dalloc(&w.sums, 8, b));
+    A(dalloc(&w.ypart, (size_t)kYtopRows * FT_NBMAX, b));
+    A(dalloc(&w.rowpart, (size_t)kYtopRows, b));
+    A(dalloc(&w.scratch, (size_t)(n + 255) / 256 + 8, b));
+    A(dalloc(&w.deltas, (size_t)FT_MAX_EVENTS, b));
+    A(dalloc(&w.bar, 4, b));
+    A(dalloc(&w.ctl, 1, b));
+    A(dalloc(&w.fixes, (size_t)FT_MAX_EVENTS, b));
+    if (e != cudaSuccess) {
+        w.release();
+        cudaGetLastError();
+        return e == cudaErrorMemoryAllocation ? FT_E_NOMEM : FT_E_CUDA;
+    }
+    int nsm = 0;
+    CK(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev));
+    w.nsm = nsm;
+    w.ldw = ldw;
+    w.n_cap = n;
+    w.bytes = b;
+    *out = &w;
+    return 0;
+}
+
+// ---------------------------------------------------------------------------
+// R12 decoder (host side).  Works on the syndromes computed by the GPU full-verify
+// kernels; emits a list of fixes that the GPU applies with explicit sums.
+// Safety property: never miscorrect -- refuse whenever two explanations exist.
+// ---------------------------------------------------------------------------
+struct Plan {
+    int status = 0;  // 0 clean, 1 fixes planned, 2 uncorrectable
+    std::vector<FtFix> fixes;
+};
+
+bool bad(double d, double tau) { return !(std::fabs(d) <= tau); }
+bool same(double a, double b, double tol) {
+    bool fa = std::isfinite(a), fb = std::isfinite(b);
+    if (!fa || !fb) return !fa && !fb;
+    return std::fabs(a - b) <= tol;
+}
+
+// members of S whose syndromes add up to `target` (|subset| <= 3), unique, or fail
+bool explain(const std::vector<int> &S, const std::vector<double> &D, double target, double tauS, int n,
+             std::vector<int> &out) {
+    out.clear();
+    if (same(target, 0.0, tauS)) return true;
+    if (!std::isfinite(target)) {
+        for (int i : S)
+            if (!std::isfinite(D[i])) out.push_back(i);
+        return !out.empty() && out.size() <= 3;
+    }
+    if (S.size() > 256) return false;
+    int hits = 0;
+    std::vector<int> best;
+    const size_t m = S.size();
+    auto tol_of = [&](double s) { return tauS + 2.0 * n * kEps * s; };
+    for (size_t a = 0; a < m; a++) {
+        double da = D[S[a]];
+        if (same(da, target, tol_of(std::fabs(da)))) {
+            hits++;
+            best = {S[a]};
+        }
+        for (size_t b2 = a + 1; b2 < m; b2++) {
+            double db = D[S[b2]];
+            if (same(da + db, target, tol_of(std::fabs(da) + std::fabs(db)))) {
+                hits++;
+                best = {S[a], S[b2]};
+            }
+            for (size_t c2 = b2 + 1; c2 < m; c2++) {
+                double dc = D[S[c2]];
+                if (same(da + db + dc, target, tol_of(std::fabs(da) + std::fabs(db) + std::fabs(dc)))) {
+                    hits++;
+                    best = {S[a], S[b2], S[c2]};
+                }
+            }
+        }
+    }
+    if (hits != 1) return false;
+    out = best;
+    return true;
+}
+
+Plan decode(int n, const std::vector<double> &Dr, const std::vector<double> &Dc, double sr, double sc,
+            double tau) {
+    Plan P;
+    const double tauS = tau * std::sqrt((double)std::max(n, 1));
+    std::vector<int> R, C;
+    for (int i = 0; i < n; i++)
+        if (bad(Dr[i], tau)) R.push_back(i);
+    for (int j = 0; j < n; j++)
+        if (bad(Dc[j], tau)) C.push_back(j);
+    const bool sr0 = same(sr, 0.0, tauS), sc0 = same(sc, 0.0, tauS);
+    if (R.empty() && C.empty() && sr0 && sc0) return P;
+    P.status = 2;
+    if (R.empty() && C.empty()) {
+        // only the corner: both sums off by the same amount
+        if (!sr0 && !sc0 && same(sr, sc, tauS)) {
+            P.fixes.push_back({-1, -1, 4, 0});
+            P.status = 1;
+        }
+        return P;
+    }
+    // ambiguous with "corner + data errors"
+    if (!sr0 && !sc0 && same(sr, sc, tauS)) return P;
+    std::vector<int> Rc, Cc;
+    if (!explain(R, Dr, sr, tauS, n, Rc) || !explain(C, Dc, sc, tauS, n, Cc)) return P;
+    std::vector<int> Rd, Cd;
+    for (int i : R)
+        if (std::find(Rc.begin(), Rc.end(), i) == Rc.end()) Rd.push_back(i);
+    for (int j : C)
+        if (std::find(Cc.begin(), Cc.end(), j) == Cc.end()) Cd.push_back(j);
+    auto pair_tol = [&](double a, double b) { return 2.0 * tau + 2.0 * n * kEps * (std::fabs(a) + std::fabs(b)); };
+    if (Rd.empty() != Cd.empty()) return P;
+    if (!Rd.empty()) {
+        if (Rd.size() == 1 && Cd.size() == 1) {
+            if (!same(Dr[Rd[0]], Dc[Cd[0]], pair_tol(Dr[Rd[0]], Dc[Cd[0]]))) return P;
+            P.fixes.push_back({Rd[0], Cd[0], 0, 0});
+        } else if (Rd.size() == 1 || Cd.size() == 1) {
+            // one shared line holds all errors: fix each along the orthogonal line
+            const bool shared_row = Rd.size() == 1;
+            const std::vector<int> &many = shared_row ? Cd : Rd;
+            const std::vector<double> &Dm = shared_row ? Dc : Dr;
+            double one = shared_row ? Dr[Rd[0]] : Dc[Cd[0]];
+            double s = 0.0, sa = 0.0;
+            bool nonfin = false;
+            for (int x : many) {
+                s += Dm[x];
+                sa += std::fabs(Dm[x]);
+                nonfin |= !std::isfinite(Dm[x]);
+            }
+            if (nonfin) {
+                if (std::isfinite(one)) return P;
+            } else if (!same(s, one, 2.0 * tauS + 2.0 * n * kEps * (sa + std::fabs(one)))) {
+                return P;
+            }
+            for (int x : many) {
+                if (shared_row) P.fixes.push_back({Rd[0], x, 1, 0});  // column formula
+                else P.fixes.push_back({x, Cd[0], 0, 0});             // row formula
+            }
+        } else if (Rd.size() == Cd.size()) {
+            std::vector<int> match(Rd.size(), -1);
+            for (size_t a = 0; a < Rd.size(); a++) {
+                int cnt = 0;
+                for (size_t b2 = 0; b2 < Cd.size(); b2++)
+                    if (same(Dr[Rd[a]], Dc[Cd[b2]], pair_tol(Dr[Rd[a]], Dc[Cd[b2]]))) {
+                        cnt++;
+                        match[a] = (int)b2;
+                    }
+                if (cnt != 1) return P;
+            }
+            for (size_t b2 = 0; b2 < Cd.size(); b2++) {
+                int cnt = 0;
+                for (size_t a = 0; a < Rd.size(); a++)
+                    if (same(Dr[Rd[a]], Dc[Cd[b2]], pair_tol(Dr[Rd[a]], Dc[Cd[b2]]))) cnt++;
+                if (cnt != 1) return P;
+            }
+            for (size_t a = 0; a < Rd.size(); a++) P.fixes.push_back({Rd[a], Cd[match[a]], 0, 0});
+        } else {
+            return P;
+        }
+    }
+    for (int i : Rc) P.fixes.push_back({i, -1, 2, 0});
+    for (int j : Cc) P.fixes.push_back({-1, j, 3, 0});
+    P.status = 1;
+    return P;
+}
+
+// ---------------------------------------------------------------------------
+// one call's state
+// ---------------------------------------------------------------------------
+struct Call {
+    int n, ilo, ihi, nb, abft, policy;
+    double c_thr;
+    cudaStream_t s;
+    Work *w;
+    double *tau;  // device tau (n-1)
+    std::vector<ft_fault> faults;
+    std::vector<ft_event> events;
+    int detected = 0, corrected = 0, rollbacks = 0, redos = 0, uncorrectable = 0;
+    int npanels = 0;
+    int rend() const { return abft ? n + 1 : ihi; }
+    int cend() const { return abft ? n + 1 : n; }
+    int pk(int t) const { return ilo - 1 + t * nb; }
+    int pib(int t) const { return std::min(nb, ihi - 2 - pk(t)); }
+    void ev(int kind, int panel, int64_t i, int64_t j, double d) {
+        ft_event e;
+        e.kind = kind;
+        e.panel = panel;
+        e.i = i;
+        e.j = j;
+        e.delta = d;
+        events.push_back(e);
+    }
+};
+
+double *site_addr(Call &C, const ft_fault &f) {
+    Work &w = *C.w;
+    const int64_t ldw = w.ldw;
+    const int n = C.n;
+    switch (f.site) {
+    case FT_SITE_A:
+        if (f.i < 0 || f.i >= n || f.j < 0 || f.j >= n) return nullptr;
+        return w.Aw + f.i + f.j * ldw;
+    case FT_SITE_R:
+        if (!C.abft || f.i < 0 || f.i >= n) return nullptr;
+        return w.Aw + f.i + (int64_t)n * ldw;
+    case FT_SITE_C:
+        if (!C.abft || f.j < 0 || f.j >= n) return nullptr;
+        return w.Aw + n + f.j * ldw;
+    case FT_SITE_K:
+        if (!C.abft) return nullptr;
+        return w.Aw + n + (int64_t)n * ldw;
+    case FT_SITE_Y:
+        if (f.i < 0 || f.i > n || f.j < 0 || f.j >= FT_NBMAX) return nullptr;
+        return w.Y + f.i + f.j * ldw;
+    case FT_SITE_V:
+        if (f.i < 0 || f.i > n || f.j < 0 || f.j >= FT_NBMAX) return nullptr;
+        return w.V + f.i + f.j * ldw;
+    }
+    return nullptr;
+}
+
+int inject_at(Call &C, int panel, int phase) {
+    for (size_t q = 0; q < C.faults.size() && q < FT_MAXFAULTS; q++) {
+        const ft_fault &f = C.faults[q];
+        if (f.phase != phase) continue;
+        if (phase != FT_PHASE_AT_END && f.panel != panel) continue;
+        double *a = site_addr(C, f);
+        if (!a) continue;
+        CK(ft_inject(a, (int)q, f.bit, C.w->ctl, C.s));
+    }
+    return 0;
+}
+
+// checkpoint copy kernels must respect the halt word, so they are kernels, not memcpys
+__global__ void k_ckpt(double *Aw, int64_t ldw, int n, int rend, int k, int ib, double *ckpt, double *ck_r,
+                       double *ck_c, double *ck_q, const double *Qr, const double *Qc, const double *Fr,
+                       int restore, const FtCtl *ctl, int check_halt) {
+    if (check_halt && ctl->halt) return;
+    const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    const int64_t panel_elems = (int64_t)ldw * ib;
+    for (int64_t x = tid; x < panel_elems; x += stride) {
+        int64_t i = x % ldw, j = x / ldw;
+        if (i >= rend) continue;
+        double *a = Aw + i + (k + j) * ldw;
+        if (restore) *a = ckpt[x];
+        else ckpt[x] = *a;
+    }
+    for (int64_t i = tid; i <= n; i += stride) {
+        double *r = Aw + i + (int64_t)n * ldw;  // column n (r, kappa)
+        double *c = Aw + n + i * ldw;            // row n (c)
+        if (restore) {
+            *r = ck_r[i];
+            *c = ck_c[i];
+            ((double *)Qr)[i] = ck_q[i];
+            ((double *)Qc)[i] = ck_q[ldw + i];
+            ((double *)Fr)[i] = ck_q[2 * ldw + i];
+        } else {
+            ck_r[i] = *r;
+            ck_c[i] = *c;
+            ck_q[i] = Qr[i];
+            ck_q[ldw + i] = Qc[i];
+            ck_q[2 * ldw + i] = Fr[i];
+        }
+    }
+}
+
+int checkpoint(Call &C, int t, int restore) {
+    Work &w = *C.w;
+    int k = C.pk(t), ib = C.pib(t);
+    int64_t total = std::max<int64_t>(w.ldw * ib, C.n + 1);
+    int blocks = (int)std::min<int64_t>((total + 255) / 256, 4 * (int64_t)w.nsm);
+    g_ft_launches++;
+    k_ckpt<<<blocks, 256, 0, C.s>>>(w.Aw, w.ldw, C.n, C.rend(), k, ib, w.ckpt, w.ck_r, w.ck_c, w.ck_q, w.Qr, w.Qc,
+                                    w.Fr, restore, w.ctl, restore ? 0 : 1);
+    CK(cudaGetLastError());
+    return 0;
+}
+
+int right_update(Call &C, int t, double sign, int do_w) {
+    Work &w = *C.w;
+    const int k = C.pk(t), ib = C.pib(t), e = k + ib;
+    GemmRightParams g{};
+    g.A = w.Aw;
+    g.lda = w.ldw;
+    g.ldw = w.ldw;
+    g.Y = w.Y;
+    g.V = w.V;
+    g.K = ib;
+    g.sign = sign;
+    g.Wpart = w.Wpart;
+    g.wsplit_stride = ((int64_t)C.n + 1 + 64) * FT_NBMAX;
+    g.ctl = sign < 0 ? w.ctl : nullptr;
+    // M-part: rows 0..k of the panel columns k+1..e-1 (DGEHRD's DTRMM + DAXPY)
+    g.r_lo = 0;
+    g.r_hi = k + 1;
+    g.c_lo = k + 1;
+    g.c_hi = e;
+    g.do_right = 1;
+    g.do_w = 0;
+    g.nsplit = 1;
+    CK(ft_launch_gemm_right(g, C.s));
+    // trailing block (+ checksum row/column), fused with W = V^T A_new
+    g.r_lo = 0;
+    g.r_hi = C.rend();
+    g.c_lo = e;
+    g.c_hi = C.cend();
+    g.wr_lo = k + 1;
+    g.wr_hi = C.ihi;
+    g.do_w = do_w;
+    int nstrip = (g.c_hi - g.c_lo + 63) / 64;
+    int nrt = (g.r_hi + 31) / 32;
+    int ns = (2 * w.nsm + nstrip - 1) / std::max(nstrip, 1);
+    ns = std::min(ns, std::max(1, nrt / 2));
+    ns = std::max(1, std::min(ns, kMaxWsplit));
+    g.nsplit = ns;
+    CK(ft_launch_gemm_right(g, C.s));
+    return 0;
+}
+
+int left_update(Call &C, int t, double sign, int nsplit) {
+    Work &w = *C.w;
+    const int k = C.pk(t), ib = C.pib(t), e = k + ib;
+    GemmLeftParams g{};
+    g.A = w.Aw;
+    g.lda = w.ldw;
+    g.ldw = w.ldw;
+    g.V = w.V;
+    g.T = w.T;
+    g.Wpart = w.Wpart;
+    g.r_lo = k + 1;
+    g.r_hi = C.rend();
+    g.c_lo = e;
+    g.c_hi = C.cend();
+    g.K = ib;
+    g.nsplit = nsplit;
+    g.wsplit_stride = ((int64_t)C.n + 1 + 64) * FT_NBMAX;
+    g.transT = 1;
+    g.sign = sign;
+    g.ctl = sign < 0 ? w.ctl : nullptr;
+    CK(ft_launch_gemm_left(g, C.s));
+    return 0;
+}
+
+int trailing_nsplit(Call &C, int t) {
+    const int k = C.pk(t), ib = C.pib(t), e = k + ib;
+    int nstrip = (C.cend() - e + 63) / 64;
+    int nrt = (C.rend() + 31) / 32;
+    int ns = (2 * C.w->nsm + nstrip - 1) / std::max(nstrip, 1);
+    ns = std::min(ns, std::max(1, nrt / 2));
+    return std::max(1, std::min(ns, kMaxWsplit));
+}
+
+int enqueue_panel(Call &C, int t) {
+    Work &w = *C.w;
+    const int n = C.n, k = C.pk(t), ib = C.pib(t);
+    const bool eager = C.abft && C.policy == FT_POLICY_EAGER;
+    if (inject_at(C, t, FT_PHASE_BEFORE_PANEL)) return FT_E_CUDA;
+    if (C.abft && checkpoint(C, t, 0)) return FT_E_CUDA;
+    CK(cudaMemsetAsync(w.bar, 0, 4 * sizeof(unsigned), C.s));
+    CK(cudaMemsetAsync(w.acc, 0, 3 * FT_ACC_STRIDE * sizeof(double), C.s));
+    PanelParams p{};
+    p.A = w.Aw;
+    p.ldw = w.ldw;
+    p.V = w.V;
+    p.Y = w.Y;
+    p.T = w.T;
+    p.tau = C.tau;
+    p.bvec = w.bvec;
+    p.acc = w.acc;
+    p.bar = w.bar;
+    p.ctl = w.ctl;
+    p.Qr = w.Qr;
+    p.Qc = w.Qc;
+    p.n = n;
+    p.ihi = C.ihi;
+    p.k = k;
+    p.ib = ib;
+    p.abft = C.abft;
+    p.verify = eager ? 1 : 0;
+    p.rbase = ((k + 1) / 16) * 16;
+    int rendp = (C.rend() + 15) / 16 * 16;
+    p.ngroups = (rendp - p.rbase) / 16;
+    CK(ft_launch_panel(p, w.nsm, C.s));
+    // Y_top = A(0:k+1, k+1:ihi) V T (+ area-1 row sums)
+    YtopParams y{};
+    y.A = w.Aw;
+    y.ldw = w.ldw;
+    y.V = w.V;
+    y.T = w.T;
+    y.Y = w.Y;
+    y.ypart = w.ypart;
+    y.rowpart = w.rowpart;
+    y.Fr = w.Fr;
+    y.ctl = w.ctl;
+    y.n = n;
+    y.ihi = C.ihi;
+    y.k = k;
+    y.ib = ib;
+    y.abft = C.abft;
+    y.verify = eager ? 1 : 0;
+    int nm = (k + 1 + 63) / 64;
+    int nkt = (C.ihi - k - 1 + 31) / 32;
+    int ns = std::max(1, std::min({(2 * w.nsm) / nm, nkt / 2, 64}));
+    while ((int64_t)ns * (k + 1) > kYtopRows) ns--;
+    y.nsplit = std::max(ns, 1);
+    CK(ft_launch_ytop(y, C.s));
+    if (inject_at(C, t, FT_PHASE_AFTER_PANEL)) return FT_E_CUDA;
+    if (eager) {
+        CK(ft_precheck(w.Y, w.V, w.ldw, n, C.ihi, k, ib, w.ctl, C.s));
+        CK(ft_decide(w.Y, w.V, w.T, w.ldw, n, k, ib, t, w.ctl, C.s));
+    }
+    if (right_update(C, t, -1.0, 1)) return FT_E_CUDA;
+    if (inject_at(C, t, FT_PHASE_AFTER_RIGHT)) return FT_E_CUDA;
+    if (left_update(C, t, -1.0, trailing_nsplit(C, t))) return FT_E_CUDA;
+    if (inject_at(C, t, FT_PHASE_AFTER_UPDATE)) return FT_E_CUDA;
+    if (C.abft) CK(ft_endcheck(w.Aw, w.ldw, n, C.ihi, k, ib, t, C.policy, w.Fr, w.ctl, C.s));
+    return 0;
+}
+
+// full verify + decode + correct + re-verify.  mode 0: H (cdone finished columns), 1: Q.
+// Returns 0 ok (clean or corrected), FT_E_UNCORRECTABLE, or an error.
+int verify_and_correct(Call &C, int panel, int cdone, int mode, bool *found) {
+    Work &w = *C.w;
+    const int n = C.n;
+    const int64_t ldw = w.ldw;
+    double *r = mode == 0 ? w.Aw + (int64_t)n * ldw : w.Qr;
+    int64_t rinc = 1;
+    double *c = mode == 0 ? w.Aw + n : w.Qc;
+    int64_t cinc = mode == 0 ? ldw : 1;
+    double *kap = mode == 0 ? w.Aw + n + (int64_t)n * ldw : w.Qc + n;
+    FtCtl hctl;
+    CK(cudaMemcpyAsync(&hctl, w.ctl, sizeof(FtCtl), cudaMemcpyDeviceToHost, C.s));
+    CK(cudaStreamSynchronize(C.s));
+    const double tau = mode == 0 ? C.c_thr * n * kEps * hctl.normF : C.c_thr * n * kEps * std::sqrt((double)n);
+    std::vector<double> Dr(n), Dc(n);
+    double sums[2], kh;
+    *found = false;
+    for (int pass = 0; pass < 2; pass++) {
+        CK(ft_full_verify(w.Aw, ldw, n, C.ilo, C.ihi, cdone, mode, r, rinc, c, cinc, nullptr, w.Dr, w.Dc, w.sums, C.s));
+        CK(cudaMemcpyAsync(Dr.data(), w.Dr, n * sizeof(double), cudaMemcpyDeviceToHost, C.s));
+        CK(cudaMemcpyAsync(Dc.data(), w.Dc, n * sizeof(double), cudaMemcpyDeviceToHost, C.s));
+        CK(cudaMemcpyAsync(sums, w.sums, 2 * sizeof(double), cudaMemcpyDeviceToHost, C.s));
+        CK(cudaMemcpyAsync(&kh, kap, sizeof(double), cudaMemcpyDeviceToHost, C.s));
+        CK(cudaStreamSynchronize(C.s));
+        Plan P = decode(n, Dr, Dc, sums[0] - kh, sums[1] - kh, tau);
+        if (pass == 0) {
+            // fault-free drift bookkeeping
+            if (P.status == 0 || P.status == 1) {
+                double mx = 0.0;
+                for (int i = 0; i < n; i++) {
+                    if (std::fabs(Dr[i]) <= tau) mx = std::max(mx, std::fabs(Dr[i]));
+                    if (std::fabs(Dc[i]) <= tau) mx = std::max(mx, std::fabs(Dc[i]));
+                }
+                double unit = tau / C.c_thr;
+                double rel = unit > 0 ? mx / unit : 0.0;
+                unsigned long long bits;
+                memcpy(&bits, &rel, 8);
+                if (bits > hctl.drift_bits) {
+                    CK(cudaMemcpyAsync(&w.ctl->drift_bits, &bits, 8, cudaMemcpyHostToDevice, C.s));
+                }
+            }
+            if (P.status == 0) return 0;
+            *found = true;
+            int nr = 0, nc = 0;
+            for (int i = 0; i < n; i++) {
+                nr += bad(Dr[i], tau);
+                nc += bad(Dc[i], tau);
+            }
+            C.ev(FT_EV_DETECT, panel, nr, nc, 0.0);
+            C.detected++;
+            if (P.status == 2) {
+                C.ev(FT_EV_UNCORRECTABLE, panel, nr, nc, 0.0);
+                C.uncorrectable++;
+                return FT_E_UNCORRECTABLE;
+            }
+            int nf = (int)std::min<size_t>(P.fixes.size(), FT_MAX_EVENTS);
+            CK(cudaMemcpyAsync(w.fixes, P.fixes.data(), nf * sizeof(FtFix), cudaMemcpyHostToDevice, C.s));
+            CK(ft_apply_fixes(w.Aw, ldw, n, C.ilo, C.ihi, cdone, mode, r, rinc, c, cinc, kap, w.fixes, nf, w.deltas,
+                              C.s));
+            std::vector<double> dl(nf);
+            CK(cudaMemcpyAsync(dl.data(), w.deltas, nf * sizeof(double), cudaMemcpyDeviceToHost, C.s));
+            CK(cudaStreamSynchronize(C.s));
+            for (int q = 0; q < nf; q++) {
+                const FtFix &f = P.fixes[q];
+                int kind = f.kind == 0 || f.kind == 1 ? (mode == 0 ? FT_EV_FIX_DATA : FT_EV_FIX_Q)
+                           : f.kind == 2             ? (mode == 0 ? FT_EV_FIX_R : FT_EV_FIX_QR)
+                           : f.kind == 3             ? (mode == 0 ? FT_EV_FIX_C : FT_EV_FIX_QC)
+                                                     : (mode == 0 ? FT_EV_FIX_K : FT_EV_FIX_QK);
+                C.ev(kind, panel, f.i, f.j, dl[q]);
+            }
+        } else {
+            if (P.status != 0) {
+                C.ev(FT_EV_UNCORRECTABLE, panel, -1, -1, 0.0);
+                C.uncorrectable++;
+                return FT_E_UNCORRECTABLE;
+            }
+            C.corrected++;
+        }
+    }
+    return 0;
+}
+
+int recover(Call &C, const FtCtl &h) {
+    Work &w = *C.w;
+    const int t = h.halt_panel;
+    const int k = C.pk(t);
+    // clear the halt so the recovery kernels run
+    int zero = 0;
+    CK(cudaMemcpyAsync(&w.ctl->halt, &zero, sizeof(int), cudaMemcpyHostToDevice, C.s));
+    CK(cudaMemcpyAsync(&w.ctl->nflag, &zero, sizeof(int), cudaMemcpyHostToDevice, C.s));
+    CK(cudaMemsetAsync(w.ctl->eY, 0, sizeof(double) * 128, C.s));
+    CK(cudaMemsetAsync(w.ctl->sums, 0, sizeof(double) * 4, C.s));
+    CK(cudaMemsetAsync(&w.ctl->done_count, 0, sizeof(int), C.s));
+    if (h.halt_stage == 2) {
+        // reverse computation: add back the left, then the right update
+        if (left_update(C, t, +1.0, trailing_nsplit(C, t))) return FT_E_CUDA;
+        if (right_update(C, t, +1.0, 0)) return FT_E_CUDA;
+        C.ev(FT_EV_ROLLBACK, t, h.halt_reason, 0, 0.0);
+        C.rollbacks++;
+    } else {
+        C.ev(FT_EV_PANEL_REDO, t, h.halt_reason, 0, 0.0);
+        C.redos++;
+    }
+    // restore the pre-factorized panel and the checksum vectors (diskless checkpoint)
+    if (checkpoint(C, t, 1)) return FT_E_CUDA;
+    bool found = false;
+    int info = verify_and_correct(C, t, k, 0, &found);
+    return info;
+}
+
+int validate(int n, int ilo, int ihi, const void *A, int lda, const void *tau, const ft_opts *o) {
+    if (n < 0) return -1;
+    if (ilo < 1 || ilo > std::max(1, n)) return -2;
+    if (ihi < std::min(ilo, n) || ihi > n) return -3;
+    if (n > 0 && !A) return -4;
+    if (lda < std::max(1, n)) return -5;
+    if (n > 1 && !tau) return -6;
+    if (o) {
+        if (o->nb < 0 || o->nb > FT_NBMAX) return -7;
+        if (o->abft != 0 && o->abft != 1) return -7;
+        if (o->weighted != 0) return -7;
+        if (o->policy != FT_POLICY_EAGER && o->policy != FT_POLICY_PAPER) return -7;
+        if (o->c_thr < 0.0 || !(o->c_thr == o->c_thr)) return -7;
+        if (o->nfaults < 0 || o->nfaults > FT_MAXFAULTS || (o->nfaults > 0 && !o->faults)) return -7;
+        if (o->stop_after_panel < -1) return -7;
+    }
+    return 0;
+}
+
+int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opts *opts) {
+    ft_opts o;
+    ft_opts_default(&o);
+    if (opts) o = *opts;
+    int info = validate(n, ilo, ihi, dA, lda, dtau, &o);
+    if (info) return info;
+    cudaStream_t s = (cudaStream_t)o.stream;
+    if (n == 0) return 0;
+    if (n > 1) CK(cudaMemsetAsync(dtau, 0, (n - 1) * sizeof(double), s));
+    Call C;
+    C.n = n;
+    C.ilo = ilo;
+    C.ihi = ihi;
+    C.nb = o.nb > 0 ? o.nb : (n < 4096 ? 32 : 64);
+    C.abft = o.abft;
+    C.policy = o.policy;
+    C.c_thr = o.c_thr > 0 ? o.c_thr : 2.0;
+    C.s = s;
+    C.tau = dtau;
+    for (int q = 0; q < o.nfaults; q++) C.faults.push_back(o.faults[q]);
+    int rc = get_work(n, &C.w);
+    if (rc) return rc;
+    Work &w = *C.w;
+    cudaEvent_t ev0, ev1;
+    CK(cudaEventCreate(&ev0));
+    CK(cudaEventCreate(&ev1));
+    CK(cudaEventRecord(ev0, s));
+    // control block
+    FtCtl h0;
+    memset(&h0, 0, sizeof(h0));
+    h0.c_thr = C.c_thr;
+    CK(cudaMemcpyAsync(w.ctl, &h0, sizeof(FtCtl), cudaMemcpyHostToDevice, s));
+    // working array: A, zero padding, checksum row/column
+    CK(cudaMemsetAsync(w.Aw, 0, (size_t)w.ldw * (n + 1) * sizeof(double), s));
+    CK(cudaMemsetAsync(w.V, 0, (size_t)w.ldw * FT_NBMAX * sizeof(double), s));
+    CK(cudaMemsetAsync(w.Y, 0, (size_t)w.ldw * FT_NBMAX * sizeof(double), s));
+    CK(ft_copy_in(dA, lda, w.Aw, w.ldw, n, s));
+    if (C.abft) {
+        CK(ft_encode(w.Aw, w.ldw, n, w.ctl, w.scratch, s));
+        CK(cudaMemsetAsync(w.Fr, 0, w.ldw * sizeof(double), s));
+        if (ilo > 1) CK(ft_frozen_init(w.Aw, w.ldw, n, ilo - 1, w.Fr, s));
+        CK(cudaMemsetAsync(w.Qr, 0, w.ldw * sizeof(double), s));
+        CK(cudaMemsetAsync(w.Qc, 0, w.ldw * sizeof(double), s));
+    }
+    C.npanels = 0;
+    for (int k = ilo - 1; k < ihi - 2; k += C.nb) C.npanels++;
+    const int last = (o.stop_after_panel >= 0) ? std::min(o.stop_after_panel + 1, C.npanels) : C.npanels;
+    int t0 = 0, attempts = 0;
+    info = 0;
+    while (true) {
+        for (int t = t0; t < last; t++) {
+            rc = enqueue_panel(C, t);
+            if (rc) return rc;
+        }
+        FtCtl h;
+        CK(cudaMemcpyAsync(&h, w.ctl, sizeof(FtCtl), cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        if (!h.halt) break;
+        if (++attempts > 4 * (C.npanels + 1) + (int)C.faults.size() * 4) {
+            C.ev(FT_EV_UNCORRECTABLE, h.halt_panel, -1, -1, 0.0);
+            C.uncorrectable++;
+            info = FT_E_UNCORRECTABLE;
+            break;
+        }
+        rc = recover(C, h);
+        if (rc == FT_E_UNCORRECTABLE) {
+            info = rc;
+            break;
+        }
+        if (rc) return rc;
+        t0 = h.halt_panel;
+    }
+    if (info == 0 && o.stop_after_panel < 0) {
+        inject_at(C, -1, FT_PHASE_AT_END);
+        if (C.abft) {
+            // final verification of the finished H (a12) and of the Householder vectors
+            bool found = false;
+            const int cdone = std::max(ihi - 1, ilo - 1);
+            int r1 = verify_and_correct(C, -1, cdone, 0, &found);
+            if (r1 == 0) r1 = verify_and_correct(C, -1, cdone, 1, &found);
+            if (r1 == FT_E_UNCORRECTABLE) info = r1;
+            else if (r1) return r1;
+        }
+    }
+    CK(ft_copy_out(w.Aw, w.ldw, dA, lda, n, s));
+    if (o.stop_after_panel >= 0 && o.dchk_out && C.abft) {
+        CK(cudaMemcpyAsync(o.dchk_out, w.Aw + (int64_t)n * w.ldw, n * sizeof(double), cudaMemcpyDeviceToDevice, s));
+        CK(cudaMemcpy2DAsync(o.dchk_out + n, sizeof(double), w.Aw + n, w.ldw * sizeof(double), sizeof(double), n,
+                             cudaMemcpyDeviceToDevice, s));
+        CK(cudaMemcpyAsync(o.dchk_out + 2 * n, w.Aw + n + (int64_t)n * w.ldw, sizeof(double),
+                           cudaMemcpyDeviceToDevice, s));
+    }
+    CK(cudaEventRecord(ev1, s));
+    FtCtl hf;
+    CK(cudaMemcpyAsync(&hf, w.ctl, sizeof(FtCtl), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    float ms = 0.f;
+    cudaEventElapsedTime(&ms, ev0, ev1);
+    cudaEventDestroy(ev0);
+    cudaEventDestroy(ev1);
+    if (o.report) {
+        ft_report &R = *o.report;
+        memset(&R, 0, sizeof(R));
+        // injection events first (in fault order), then the detection/correction log
+        std::vector<ft_event> all;
+        for (size_t q = 0; q < C.faults.size() && q < FT_MAXFAULTS; q++) {
+            if (!hf.inj_done[q]) continue;
+            ft_event e;
+            e.kind = FT_EV_INJECT;
+            e.panel = C.faults[q].phase == FT_PHASE_AT_END ? -1 : C.faults[q].panel;
+            e.i = C.faults[q].i;
+            e.j = C.faults[q].j;
+            e.delta = hf.inj_delta[q];
+            all.push_back(e);
+        }
+        all.insert(all.end(), C.events.begin(), C.events.end());
+        R.nevents = (int)std::min<size_t>(all.size(), FT_MAX_EVENTS);
+        for (int q = 0; q < R.nevents; q++) R.events[q] = all[q];
+        R.detected = C.detected;
+        R.corrected = C.corrected;
+        R.rollbacks = C.rollbacks;
+        R.panel_redos = C.redos;
+        R.uncorrectable = C.uncorrectable;
+        double drift;
+        memcpy(&drift, &hf.drift_bits, 8);
+        R.max_drift_rel = drift;
+        R.ms[0] = ms;
+    }
+    return info;
+}
+
+}  // namespace
+
+// ---------------------------------------------------------------------------
+// C ABI
+// ---------------------------------------------------------------------------
+extern "C" {
+
+void ft_opts_default(ft_opts *o) {
+    if (!o) return;
+    memset(o, 0, sizeof(*o));
+    o->nb = 0;
+    o->abft = 1;
+    o->weighted = 0;
+    o->policy = FT_POLICY_EAGER;
+    o->c_thr = 2.0;
+    o->stop_after_panel = -1;
+}
+
+int ft_dgehrd(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opts *opts) {
+    return run(n, ilo, ihi, dA, lda, dtau, opts);
+}
+
+int ft_dgehrd_host(int n, int ilo, int ihi, double *hA, int lda, double *htau, const ft_opts *opts) {
+    ft_opts o;
+    ft_opts_default(&o);
+    if (opts) o = *opts;
+    int info = validate(n, ilo, ihi, hA, lda, htau, &o);
+    if (info) return info;
+    if (n == 0) return 0;
+    cudaStream_t s = (cudaStream_t)o.stream;
+    double *dA = nullptr, *dtau = nullptr;
+    // device staging buffers live with the workspace of this size
+    static std::map<int, std::pair<size_t, std::pair<double *, double *>>> stage;
+    int dev = 0;
+    CK(cudaGetDevice(&dev));
+    auto &st = stage[dev];
+    size_t need = (size_t)n * n;
+    if (st.first < need) {
+        if (st.second.first) cudaFree(st.second.first);
+        if (st.second.second) cudaFree(st.second.second);
+        CK(cudaMalloc(&st.second.first, need * sizeof(double)));
+        CK(cudaMalloc(&st.second.second, std::max(n, 2) * sizeof(double)));
+        st.first = need;
+    }
+    dA = st.second.first;
+    dtau = st.second.second;
+    CK(cudaMemcpy2DAsync(dA, n * sizeof(double), hA, (size_t)lda * sizeof(double), n * sizeof(double), n,
+                         cudaMemcpyHostToDevice, s));
+    info = run(n, ilo, ihi, dA, n, dtau, &o);
+    if (info < 0 || info == FT_E_CUDA || info == FT_E_NOMEM) return info;
+    CK(cudaMemcpy2DAsync(hA, (size_t)lda * sizeof(double), dA, n * sizeof(double), n * sizeof(double), n,
+                         cudaMemcpyDeviceToHost, s));
+    if (n > 1) CK(cudaMemcpyAsync(htau, dtau, (n - 1) * sizeof(double), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    return info;
+}
+
+int ft_dorghr(int n, int ilo, int ihi, const double *dA, int lda, const double *dtau, double *dQ, int ldq,
+              const ft_opts *opts) {
+    ft_opts o;
+    ft_opts_default(&o);
+    if (opts) o = *opts;
+    int info = validate(n, ilo, ihi, dA, lda, dtau, nullptr);
+    if (info) return info;
+    if (n > 0 && !dQ) return -8;
+    if (ldq < std::max(1, n)) return -9;
+    if (o.nb < 0 || o.nb > FT_NBMAX) return -7;
+    if (n == 0) return 0;
+    cudaStream_t s = (cudaStream_t)o.stream;
+    Work *wp = nullptr;
+    int rc = get_work(n, &wp);
+    if (rc) return rc;
+    Work &w = *wp;
+    const int nb = o.nb > 0 ? o.nb : (n < 4096 ? 32 : 64);
+    CK(ft_copy_in(dA, lda, w.Aw, w.ldw, n, s));  // private copy of V (dQ may alias dA)
+    CK(ft_set_identity(dQ, ldq, n, s));
+    int npanels = 0;
+    for (int k = ilo - 1; k < ihi - 2; k += nb) npanels++;
+    for (int t = npanels - 1; t >= 0; t--) {
+        const int k = ilo - 1 + t * nb, ib = std::min(nb, ihi - 2 - k);
+        CK(ft_build_v(w.Aw, w.ldw, w.V, n, ihi, k, ib, s));
+        CK(ft_larft(w.V, w.ldw, dtau, w.T, n, ihi, k, ib, s));
+        GemmRightParams g{};
+        g.A = dQ;
+        g.lda = ldq;
+        g.ldw = w.ldw;
+        g.Y = nullptr;
+        g.V = w.V;
+        g.r_lo = k + 1;
+        g.r_hi = ihi;
+        g.c_lo = k + 1;
+        g.c_hi = ihi;
+        g.K = ib;
+        g.wr_lo = k + 1;
+        g.wr_hi = ihi;
+        g.do_right = 0;
+        g.do_w = 1;
+        g.sign = 1.0;
+        g.Wpart = w.Wpart;
+        g.wsplit_stride = ((int64_t)n + 1 + 64) * FT_NBMAX;
+        int nstrip = (ihi - k - 1 + 63) / 64;
+        int nrt = (ihi - k - 1 + 31) / 32;
+        int ns = (2 * w.nsm + nstrip - 1) / std::max(nstrip, 1);
+        ns = std::max(1, std::min({ns, std::max(1, nrt / 2), kMaxWsplit}));
+        g.nsplit = ns;
+        g.ctl = nullptr;
+        CK(ft_launch_gemm_right(g, s));
+        GemmLeftParams L{};
+        L.A = dQ;
+        L.lda = ldq;
+        L.ldw = w.ldw;
+        L.V = w.V;
+        L.T = w.T;
+        L.Wpart = w.Wpart;
+        L.r_lo = k + 1;
+        L.r_hi = ihi;
+        L.c_lo = k + 1;
+        L.c_hi = ihi;
+        L.K = ib;
+        L.nsplit = ns;
+        L.wsplit_stride = g.wsplit_stride;
+        L.transT = 0;
+        L.sign = -1.0;
+        L.ctl = nullptr;
+        CK(ft_launch_gemm_left(L, s));
+    }
+    CK(cudaStreamSynchronize(s));
+    return 0;
+}
+
+int ft_dgehrd_mgpu(int n, int ilo, int ihi, double *dA_local, int lda_local, double *dtau, void *nccl_comm,
+                   int rank, int nranks, const ft_opts *opts) {
+    if (nranks < 1 || rank < 0 || rank >= nranks) return -9;
+    if (nranks == 1) return ft_dgehrd(n, ilo, ihi, dA_local, lda_local, dtau, opts);
+    return -9;  // multi-rank distribution not built in this round ("Multi-GPU")
+}
+
+const char *ft_strerror(int info) {
+    switch (info) {
+    case 0: return "success";
+    case FT_E_UNCORRECTABLE: return "uncorrectable soft error (checksum discrepancy could not be decoded)";
+    case FT_E_CUDA: return "CUDA runtime error";
+    case FT_E_NCCL: return "NCCL error";
+    case FT_E_NOMEM: return "out of device memory";
+    default: break;
+    }
+    if (info < 0) {
+        static const char *args[] = {"", "n", "ilo", "ihi", "A", "lda", "tau", "opts", "Q", "ldq"};
+        static char buf[64];
+        int a = -info;
+        snprintf(buf, sizeof(buf), "illegal value of argument %d (%s)", a, a < 10 ? args[a] : "?");
+        return buf;
+    }
+    return "unknown error";
+}
+
+void ft_finalize(void) {
+    for (auto &kv : g_work) {
+        int cur = 0;
+        cudaGetDevice(&cur);
+        cudaSetDevice(kv.first);
+        kv.second.release();
+        cudaSetDevice(cur);
+    }
+    g_work.clear();
+}
+
+const char *ft_version(void) { return "ftgehrd 0.1 (sm_100a; DMMA f64 updates, persistent DLAHR2 panel)"; }
+
+int64_t ft_launch_count(int reset) {
+    int64_t v = g_ft_launches;
+    if (reset) g_ft_launches = 0;
+    return v;
+}
+
+}  // extern "C"

@@ -1,0 +1,118 @@
+// ft_internal.h -- internal structures and kernel launchers of libftgehrd.
+// Host + device visible; no torch types, no oracle code.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "../../include/ftgehrd.h"
+
+#define FT_MAXFAULTS 64
+#ifndef FT_NBMAX
+#define FT_NBMAX 64
+#endif
+#define FT_ACC_STRIDE (2 * 64 + 8)  // [s1 | vtb | nrm2 sx alpha ...] per reduction set
+
+// Device-resident control block: halt protocol, fused-verify flags, injector log.
+struct FtCtl {
+    int halt;         // != 0: every later kernel of this call is a no-op
+    int halt_panel;   // iteration at which the halt was raised
+    int halt_stage;   // 1 = pre-update (verify-before-consume / workspace check), 2 = post-update
+    int halt_reason;  // bit 0: D_r flag, 1: Y check, 2: V check, 3: scalar check (paper), 4: kappa
+    int nflag;        // flagged rows in the fused verify of the current iteration
+    int done_count;   // last-block-done counter
+    int pad[2];
+    double normF;         // ||A||_F of the input (invariant under the similarity)
+    double c_thr;
+    unsigned long long drift_bits;  // max fault-free |D| / (n eps ||A||_F) seen (as bits)
+    double eY[64];        // pre-update check sums (e^T Y)
+    double eV[64];        // (e^T V)
+    double sums[4];       // end check: sum r, sum c
+    double inj_delta[FT_MAXFAULTS];
+    int inj_done[FT_MAXFAULTS];
+};
+
+struct PanelParams {
+    double *A;
+    int64_t ldw;
+    double *V, *Y, *T, *tau, *bvec, *acc;
+    unsigned *bar;
+    FtCtl *ctl;
+    double *Qr, *Qc;
+    int n, ihi, k, ib, abft, verify;  // verify: fused D_r on the first GEMV (EAGER policy)
+    int rbase, ngroups;               // 16-row groups starting at rbase
+    int smem_rows;                    // set by the launcher: V/Y rows cached in shared memory
+};
+
+// launchers (return cudaError_t of the launch)
+cudaError_t ft_launch_panel(const PanelParams &p, int nsm, cudaStream_t s);
+size_t ft_panel_smem_bytes();
+
+struct GemmRightParams {
+    double *A;
+    int64_t lda;    // leading dimension of A (the updated matrix)
+    int64_t ldw;    // leading dimension of Y and V
+    const double *Y, *V;
+    int r_lo, r_hi, c_lo, c_hi, K;  // C rows/cols, inner dimension
+    int wr_lo, wr_hi;               // rows of V that take part in W = V^T A_new
+    int do_right, do_w;
+    double sign;                    // -1: A -= Y V^T (update), +1: rollback
+    double *Wpart;                  // [split][col][64]
+    int64_t wsplit_stride;          // doubles per split
+    int nsplit;
+    const FtCtl *ctl;
+};
+cudaError_t ft_launch_gemm_right(const GemmRightParams &p, cudaStream_t s);
+
+struct GemmLeftParams {
+    double *A;
+    int64_t lda;
+    int64_t ldw;
+    const double *V, *T, *Wpart;
+    int r_lo, r_hi, c_lo, c_hi, K;
+    int nsplit;
+    int64_t wsplit_stride;
+    int transT;     // 1: A -= V (T^T W) (DLARFB 'L','T'); 0: A -= V (T W)
+    double sign;    // -1 update, +1 rollback
+    const FtCtl *ctl;
+};
+cudaError_t ft_launch_gemm_left(const GemmLeftParams &p, cudaStream_t s);
+
+struct YtopParams {
+    const double *A;
+    int64_t ldw;
+    const double *V, *T;
+    double *Y;
+    double *ypart, *rowpart;  // [split][row][64], [split][row]
+    const double *Fr;
+    FtCtl *ctl;
+    int n, ihi, k, ib, nsplit, abft, verify;
+};
+cudaError_t ft_launch_ytop(const YtopParams &p, cudaStream_t s);
+
+// ABFT / utility kernels (ft_abft.cu)
+cudaError_t ft_copy_in(const double *A, int lda, double *Aw, int64_t ldw, int n, cudaStream_t s);
+cudaError_t ft_copy_out(const double *Aw, int64_t ldw, double *A, int lda, int n, cudaStream_t s);
+cudaError_t ft_encode(double *Aw, int64_t ldw, int n, FtCtl *ctl, double *scratch, cudaStream_t s);
+cudaError_t ft_frozen_init(const double *Aw, int64_t ldw, int n, int ncols, double *Fr, cudaStream_t s);
+cudaError_t ft_precheck(const double *Y, const double *V, int64_t ldw, int n, int ihi, int k, int ib,
+                        FtCtl *ctl, cudaStream_t s);
+cudaError_t ft_decide(const double *Y, const double *V, const double *T, int64_t ldw, int n, int k,
+                      int ib, int panel, FtCtl *ctl, cudaStream_t s);
+cudaError_t ft_endcheck(double *Aw, int64_t ldw, int n, int ihi, int k, int ib, int panel, int policy,
+                        double *Fr, FtCtl *ctl, cudaStream_t s);
+cudaError_t ft_inject(double *addr, int fidx, int bit, FtCtl *ctl, cudaStream_t s);
+// full verification (recovery path / final): mode 0 = H logical, 1 = Q (V region)
+cudaError_t ft_full_verify(const double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdone, int mode,
+                           const double *r, int64_t rinc, const double *c, int64_t cinc, const double *Fr,
+                           double *Dr, double *Dc, double *sums, cudaStream_t s);
+struct FtFix { int64_t i, j; int kind; int pad; };  // kind: 0 row formula, 1 col formula, 2 refresh r(i), 3 refresh c(j), 4 kappa
+cudaError_t ft_apply_fixes(double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdone, int mode,
+                           double *r, int64_t rinc, double *c, int64_t cinc, double *kappa,
+                           const FtFix *fixes, int nfix, double *deltas, cudaStream_t s);
+cudaError_t ft_frob_to_ctl(const double *A, int lda, int n, FtCtl *ctl, cudaStream_t s);
+cudaError_t ft_build_v(const double *Aw, int64_t ldw, double *V, int n, int ihi, int k, int ib, cudaStream_t s);
+cudaError_t ft_larft(const double *V, int64_t ldw, const double *tau, double *T, int n, int ihi, int k,
+                     int ib, cudaStream_t s);
+cudaError_t ft_set_identity(double *Q, int64_t ldq, int n, cudaStream_t s);
+
+extern int64_t g_ft_launches;
