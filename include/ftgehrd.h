@@ -143,6 +143,17 @@ const char *ft_version(void);
  * library has launched since load / the last reset. */
 int64_t ft_launch_count(int reset);
 
+/* Diagnostics (used by bench.py for the roofline of the dominant kernel).
+ * ft_debug_time_panels(1) resets and starts recording CUDA events around every panel
+ * kernel launch on its stream; ft_debug_panel_ms() / ft_debug_panel_launches() return the
+ * summed device time and launch count of completed calls.  ft_debug_probe_panel(t, dbuf)
+ * makes CTA 0 of panel t write per-column phase timestamps (%globaltimer, 16 slots per
+ * column, device buffer of 64*16 uint64) -- t = -1 disables. */
+void ft_debug_time_panels(int on);
+double ft_debug_panel_ms(void);
+int ft_debug_panel_launches(void);
+void ft_debug_probe_panel(int panel, unsigned long long *dbuf);
+
 #ifdef __cplusplus
 }
 #endif

@@ -19,6 +19,38 @@
 #include "ft_internal.h"
 
 int64_t g_ft_launches = 0;
+static int g_dbg_panel = -1;
+static unsigned long long *g_dbg_buf = nullptr;
+extern "C" void ft_debug_probe_panel(int panel, unsigned long long *dbuf) {
+    g_dbg_panel = panel;
+    g_dbg_buf = dbuf;
+}
+// live per-launch timing of the panel kernel (CUDA events on the launching stream)
+static bool g_time_panels = false;
+static double g_panel_ms = 0.0;
+static int g_panel_launches = 0;
+static std::vector<std::pair<cudaEvent_t, cudaEvent_t>> g_panel_events;
+extern "C" void ft_debug_time_panels(int on) {
+    g_time_panels = on != 0;
+    if (on) {
+        g_panel_ms = 0.0;
+        g_panel_launches = 0;
+    }
+}
+extern "C" double ft_debug_panel_ms(void) { return g_panel_ms; }
+extern "C" int ft_debug_panel_launches(void) { return g_panel_launches; }
+static void collect_panel_events() {
+    for (auto &pr : g_panel_events) {
+        float ms = 0.f;
+        if (cudaEventElapsedTime(&ms, pr.first, pr.second) == cudaSuccess) {
+            g_panel_ms += ms;
+            g_panel_launches++;
+        }
+        cudaEventDestroy(pr.first);
+        cudaEventDestroy(pr.second);
+    }
+    g_panel_events.clear();
+}
 
 namespace {
 
@@ -489,10 +521,21 @@ int enqueue_panel(Call &C, int t) {
     p.ib = ib;
     p.abft = C.abft;
     p.verify = eager ? 1 : 0;
+    p.dbg = (t == g_dbg_panel) ? g_dbg_buf : nullptr;
     p.rbase = ((k + 1) / 16) * 16;
     int rendp = (C.rend() + 15) / 16 * 16;
     p.ngroups = (rendp - p.rbase) / 16;
+    cudaEvent_t pe0 = nullptr, pe1 = nullptr;
+    if (g_time_panels) {
+        CK(cudaEventCreate(&pe0));
+        CK(cudaEventCreate(&pe1));
+        CK(cudaEventRecord(pe0, C.s));
+    }
     CK(ft_launch_panel(p, w.nsm, C.s));
+    if (g_time_panels) {
+        CK(cudaEventRecord(pe1, C.s));
+        g_panel_events.push_back({pe0, pe1});
+    }
     // Y_top = A(0:k+1, k+1:ihi) V T (+ area-1 row sums)
     YtopParams y{};
     y.A = w.Aw;
@@ -757,6 +800,7 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
     CK(cudaStreamSynchronize(s));
     float ms = 0.f;
     cudaEventElapsedTime(&ms, ev0, ev1);
+    collect_panel_events();
     cudaEventDestroy(ev0);
     cudaEventDestroy(ev1);
     if (o.report) {

@@ -41,6 +41,7 @@ struct PanelParams {
     int n, ihi, k, ib, abft, verify;  // verify: fused D_r on the first GEMV (EAGER policy)
     int rbase, ngroups;               // 16-row groups starting at rbase
     int smem_rows;                    // set by the launcher: V/Y rows cached in shared memory
+    unsigned long long *dbg;          // optional per-column phase timestamps (CTA 0), or NULL
 };
 
 // launchers (return cudaError_t of the launch)

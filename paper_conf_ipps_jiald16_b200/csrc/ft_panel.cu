@@ -62,6 +62,17 @@ __device__ __forceinline__ void block_sum3(PanelSmem &S, double &a, double &b, d
     __syncthreads();
 }
 
+__device__ __forceinline__ unsigned long long gtimer() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
+#define PROBE(slot)                                                                   \
+    do {                                                                              \
+        if (p.dbg && blockIdx.x == 0 && tid == 0 && j < 64)                           \
+            p.dbg[j * 16 + (slot)] = gtimer();                                        \
+    } while (0)
+
 __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
     if (p.ctl->halt) return;  // uniform for the whole grid (nobody writes halt in this launch)
     extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -108,6 +119,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
     for (int j = 0; j < ib; j++) {
         const int c = k + j;
         double *acc = p.acc + (j % 3) * FT_ACC_STRIDE;
+        PROBE(0);
         // ---------------- (i) b0 = A(:,c) - Y V(c,:)^T  ------------------------------
         if (tid < j) S.vrow[tid] = (tid == j - 1) ? 1.0 : ldcg(V + c + (int64_t)tid * ldw);
         __syncthreads();
@@ -126,7 +138,9 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
                 sacc = warp_sum(sacc);
                 if (lane == 0) atomicAdd(acc + jp, sacc);
             }
+            PROBE(1);
             grid_barrier(p.bar, epoch, P);
+            PROBE(2);
             // ---------------- (ii) w = T^T s1 ; b = b0 - V_aug w ----------------------
             if (tid < j) S.s1[tid] = ldcg(acc + tid);
             __syncthreads();
@@ -162,7 +176,9 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
             double *nxt = p.acc + ((j + 1) % 3) * FT_ACC_STRIDE;
             for (int i = tid; i < FT_ACC_STRIDE; i += blockDim.x) nxt[i] = 0.0;
         }
+        PROBE(3);
         grid_barrier(p.bar, epoch, P);
+        PROBE(4);
         // ---------------- (iii) DLARFG (reading R1) --------------------------------
         if (tid == 0) {
             double nrm2 = ldcg(acc + 2 * FT_NBMAX + 0);
@@ -212,6 +228,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
         } else if (cache && mine) {
             Vl[tid + j * ls] = 0.0;  // rows outside the panel take no part in the V^T b dots
         }
+        PROBE(5);
         // ---------------- (iv) the trailing GEMV, v staged in shared memory ------------
         const bool vfy = (j == 0) && p.verify;
         const int cend = vfy ? n : ihi;
@@ -251,6 +268,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
                 }
             }
         }
+        PROBE(6);
         if (gemv_on) {
             S.redy[tid] = ya;
             if (vfy) S.reds[tid] = rs;
@@ -280,6 +298,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
             }
         }
         __syncthreads();
+        PROBE(7);
         // ---------------- (v) Y(:, j), T(:, j) -------------------------------------
         if (valid) {
             double2 yy2 = S.y2[tid >> 1];
@@ -319,6 +338,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
             }
         }
         __syncthreads();
+        PROBE(8);
     }
     // Q row checksums of the new Householder vectors (Fig. 5): own data rows
     if (p.abft && datarow) {

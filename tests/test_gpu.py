@@ -1,0 +1,294 @@
+"""GPU parity tests: the CUDA path (through the C ABI) against the CPU oracle.
+
+Tolerances (readings R17/R18):
+  * H, V, tau, Q: max|x_gpu - x_ora| / max|x_ora| <= 1e-9 (norm-wise max-entry)
+  * ||A - Q H Q^T||_1 / (n ||A||_1 eps) <= 30 and ||I - Q^T Q||_1 / (n eps) <= 30
+  * checksums at an iteration boundary: |chk_gpu - chk_ora| <= 1e-10 ||A||_F
+  * fault runs: same tolerances as a fault-free run; located (i, j) equal the oracle's
+"""
+import numpy as np
+import pytest
+
+import oracle
+import synth
+
+pytestmark = pytest.mark.gpu
+EPS = 2.0 ** -52
+TOL = 1e-9
+
+torch = pytest.importorskip("torch")
+if not torch.cuda.is_available():  # pragma: no cover
+    pytest.skip("needs a CUDA device", allow_module_level=True)
+
+import paper_conf_ipps_jiald16_b200 as ft  # noqa: E402
+
+
+def rel(a, b):
+    d = np.abs(a - b).max() if a.size else 0.0
+    s = np.abs(b).max() if b.size else 1.0
+    return d / (s if s > 0 else 1.0)
+
+
+def gpu_reduce(A, ilo=1, ihi=None, lda=None, **kw):
+    n = A.shape[0]
+    if lda is None or lda == n:
+        dA = ft.fortran(torch.from_numpy(A).cuda())
+    else:  # a padded leading dimension
+        buf = torch.zeros(lda * n, dtype=torch.float64, device="cuda")
+        dA = torch.as_strided(buf, (n, n), (1, lda))
+        dA.copy_(torch.from_numpy(A).cuda())
+    tau, res = ft.dgehrd(dA, ilo=ilo, ihi=ihi, **kw)
+    torch.cuda.synchronize()
+    return dA, tau, res
+
+
+def check_against_oracle(A, dA, tau, ilo=1, ihi=None, nb=0, tol=TOL):
+    n = A.shape[0]
+    ihi = n if ihi is None else ihi
+    Ao, to = oracle.dgehd2(A, ilo, ihi)
+    Ag = dA.cpu().numpy()
+    tg = tau.cpu().numpy()[: max(n - 1, 0)]
+    H, Ho = np.triu(Ag, -1), np.triu(Ao, -1)
+    assert rel(H, Ho) <= tol, ("H", rel(H, Ho))
+    assert np.abs(tg - to).max(initial=0.0) <= tol * max(1.0, np.abs(to).max(initial=0.0)), "tau"
+    if n > 2:
+        V, Vo = np.tril(Ag, -2), np.tril(Ao, -2)
+        assert np.abs(V - Vo).max() <= tol * max(1.0, np.abs(Vo).max()), ("V", np.abs(V - Vo).max())
+    Q, info = ft.dorghr(dA, tau, ilo=ilo, ihi=ihi, nb=nb)
+    assert info == 0
+    Qg = Q.cpu().numpy()
+    Qo = oracle.dorghr(Ao, to, ilo, ihi)
+    assert np.abs(Qg - Qo).max(initial=0.0) <= tol, ("Q", np.abs(Qg - Qo).max())
+    if n:
+        an = np.linalg.norm(A, 1)
+        res = np.linalg.norm(A - Qg @ H @ Qg.T, 1) / (n * max(an, 1e-300) * EPS)
+        orth = np.linalg.norm(np.eye(n) - Qg.T @ Qg, 1) / (n * EPS)
+        assert res <= 30 and orth <= 30, (res, orth)
+    return H, Ho
+
+
+# ------------------------------------------------------------------ fault-free parity
+@pytest.mark.parametrize("n,nb", [(1, 16), (2, 16), (3, 16), (4, 16), (5, 16), (17, 16), (18, 16), (64, 16),
+                                  (100, 32), (257, 32), (300, 64), (513, 64)])
+@pytest.mark.parametrize("abft", [False, True])
+def test_parity_small(n, nb, abft):
+    A = synth.matrix(n, dist="uniform")
+    dA, tau, res = gpu_reduce(A, nb=nb, abft=abft)
+    assert res.info == 0, res.events
+    assert res.report.detected == 0 and res.report.nevents == 0, res.events
+    check_against_oracle(A, dA, tau, nb=nb)
+
+
+@pytest.mark.parametrize("n,nb,dist", [(700, 32, "normal"), (1000, 64, "uniform")])
+def test_parity_medium(n, nb, dist):
+    A = synth.matrix(n, dist=dist)
+    dA, tau, res = gpu_reduce(A, nb=nb)
+    assert res.info == 0 and res.report.detected == 0
+    check_against_oracle(A, dA, tau, nb=nb)
+    assert res.report.max_drift_rel < 0.5  # fault-free checksum drift, units of n eps ||A||_F
+
+
+def test_parity_c2_full_size():
+    """BASELINE config C2 (n = 2048, nb = 32), the bench workload, full element-wise parity."""
+    n = 2048
+    A = synth.matrix(n)
+    dA, tau, res = gpu_reduce(A, nb=32)
+    assert res.info == 0 and res.report.detected == 0
+    check_against_oracle(A, dA, tau, nb=32)
+
+
+@pytest.mark.parametrize("policy", [ft.POLICY_EAGER, ft.POLICY_PAPER])
+def test_policies_fault_free(policy):
+    A = synth.matrix(200, dist="normal")
+    dA, tau, res = gpu_reduce(A, nb=32, policy=policy)
+    assert res.info == 0 and res.report.detected == 0
+    check_against_oracle(A, dA, tau, nb=32)
+
+
+@pytest.mark.parametrize("n,ilo,ihi,nb", [(150, 4, 131, 32), (90, 1, 70, 16), (90, 20, 90, 16), (64, 30, 33, 16),
+                                         (64, 10, 10, 16)])
+@pytest.mark.parametrize("abft", [False, True])
+def test_ilo_ihi(n, ilo, ihi, nb, abft):
+    A = synth.matrix(n, seed=n + ilo + ihi, ilo=ilo, ihi=ihi)
+    dA, tau, res = gpu_reduce(A, ilo=ilo, ihi=ihi, nb=nb, abft=abft)
+    assert res.info == 0 and res.report.detected == 0, res.events
+    check_against_oracle(A, dA, tau, ilo=ilo, ihi=ihi, nb=nb)
+    tg = tau.cpu().numpy()
+    assert np.all(tg[: ilo - 1] == 0.0) and np.all(tg[max(ihi - 1, 0): n - 1] == 0.0)
+
+
+def test_padded_lda():
+    A = synth.matrix(77)
+    dA, tau, res = gpu_reduce(A, lda=83, nb=16)
+    assert res.info == 0
+    check_against_oracle(A, dA, tau, nb=16)
+
+
+def test_exact_cases():
+    """Already-Hessenberg input: tau = 0 and H = A exactly; symmetric input: tridiagonal H."""
+    A = synth.hessenberg_matrix(96)
+    dA, tau, res = gpu_reduce(A, nb=32)
+    assert np.all(tau.cpu().numpy()[:95] == 0.0)
+    assert np.array_equal(dA.cpu().numpy(), A)
+    S = synth.symmetric_matrix(96)
+    dS, tau, res = gpu_reduce(S, nb=32)
+    H = np.triu(dS.cpu().numpy(), -1)
+    assert np.abs(np.triu(H, 2)).max() <= 1e-13 * np.linalg.norm(S)
+
+
+def test_dorghr_in_place():
+    A = synth.matrix(130)
+    dA, tau, res = gpu_reduce(A, nb=32)
+    Qo = oracle.dorghr(*oracle.dgehd2(A))
+    Q, info = ft.dorghr(dA, tau, Q=dA, nb=32)  # dQ aliases dA (ldq == lda)
+    assert info == 0 and np.abs(Q.cpu().numpy() - Qo).max() <= TOL
+
+
+def test_host_entry_point():
+    A = synth.matrix(300)
+    Ah = np.asfortranarray(A.copy())
+    tau, res = ft.dgehrd_host(Ah, nb=32)
+    assert res.info == 0
+    Ao, to = oracle.dgehd2(A)
+    assert rel(np.triu(Ah, -1), np.triu(Ao, -1)) <= TOL
+    assert np.abs(tau - to).max() <= TOL
+
+
+# ------------------------------------------------------------------ checksum parity (Theorem 1)
+@pytest.mark.parametrize("n,nb", [(64, 16), (300, 32), (513, 64)])
+def test_checksums_at_every_boundary(n, nb):
+    A = synth.matrix(n, dist="normal")
+    normF = np.linalg.norm(A)
+    npanel = (n - 2 + nb - 1) // nb
+    for t in range(npanel):
+        chk = torch.zeros(2 * n + 1, dtype=torch.float64, device="cuda")
+        dA, tau, res = gpu_reduce(A, nb=nb, stop_after_panel=t, dchk_out=chk)
+        assert res.info == 0
+        info, Aw, tw, rep, chko = oracle.ft_dgehd2(A, nb, stop_after_panel=t)
+        g = chk.cpu().numpy()
+        assert np.abs(g - chko).max() <= 1e-10 * normF, (t, np.abs(g - chko).max())
+        assert rel(dA.cpu().numpy(), Aw) <= TOL, t
+
+
+# ------------------------------------------------------------------ fault injection
+def faulty(A, nb, faults, **kw):
+    return gpu_reduce(A, nb=nb, faults=faults, **kw)
+
+
+def fixes(events, kinds=("FIX_DATA", "FIX_R", "FIX_C", "FIX_K", "FIX_Q", "FIX_QR", "FIX_QC", "FIX_QK")):
+    return sorted((e[0], e[2], e[3]) for e in events if e[0] in kinds)
+
+
+ORA_SITE = {ft.SITE_A: oracle.SITE_A, ft.SITE_R: oracle.SITE_R, ft.SITE_C: oracle.SITE_C, ft.SITE_K: oracle.SITE_K}
+
+
+@pytest.mark.parametrize("site,i,j,bit", [
+    (ft.SITE_A, 40, 50, 51),   # C1 default: area 2 at panel 1, bit 51
+    (ft.SITE_A, 40, 50, 62),   # catastrophic exponent flip (R14)
+    (ft.SITE_A, 40, 50, 63),   # sign
+    (ft.SITE_A, 5, 50, 55),    # area 1 (rows above the panel)
+    (ft.SITE_A, 20, 16, 45),   # the panel column about to be factorized
+    (ft.SITE_A, 60, 63, 52),   # last row / column
+    (ft.SITE_R, 33, -1, 55),
+    (ft.SITE_R, 3, -1, 62),
+    (ft.SITE_C, -1, 61, 52),
+    (ft.SITE_C, -1, 7, 50),    # checksum of a finished column
+    (ft.SITE_K, -1, -1, 48),
+])
+def test_c1_before_panel_fault_matches_oracle(site, i, j, bit):
+    n, nb = 64, 16
+    A = synth.matrix(n)
+    dA, tau, res = faulty(A, nb, [(1, ft.PHASE_BEFORE_PANEL, site, i, j, bit)])
+    assert res.info == 0, res.events
+    check_against_oracle(A, dA, tau, nb=nb)
+    info, Af, tf, rep, _ = oracle.ft_dgehd2(A, nb, faults=[(1, ORA_SITE[site], i, j, bit)])
+    assert info == 0
+    ora_fix = [(k, a, b) for (k, a, b) in fixes(rep.events())]
+    assert fixes(res.events) == ora_fix, (res.events, rep.events())
+
+
+@pytest.mark.parametrize("bit", list(range(0, 64, 3)) + [52, 62, 63])
+@pytest.mark.parametrize("site,i,j", [(ft.SITE_A, 40, 50), (ft.SITE_A, 10, 40), (ft.SITE_R, 45, -1),
+                                      (ft.SITE_C, -1, 45)])
+def test_bit_sweep_detect_or_harmless(site, i, j, bit):
+    """R16: a flip with |delta| > tau_abs is detected and corrected; a smaller one is harmless."""
+    n, nb = 64, 16
+    A = synth.matrix(n, dist="normal")
+    dA, tau, res = faulty(A, nb, [(2, ft.PHASE_BEFORE_PANEL, site, i, j, bit)])
+    assert res.info == 0, res.events
+    check_against_oracle(A, dA, tau, nb=nb)
+    delta = [e[4] for e in res.events if e[0] == "INJECT"][0]
+    tau_abs = 2.0 * n * EPS * np.linalg.norm(A)
+    if not (abs(delta) <= tau_abs):
+        assert res.report.detected >= 1, (bit, delta, res.events)
+
+
+@pytest.mark.parametrize("phase", [ft.PHASE_AFTER_PANEL, ft.PHASE_AFTER_RIGHT, ft.PHASE_AFTER_UPDATE])
+@pytest.mark.parametrize("i,j,bit", [(40, 70, 51), (70, 90, 56), (10, 80, 63), (40, 70, 60)])
+def test_mid_iteration_faults(phase, i, j, bit):
+    n, nb = 128, 32
+    A = synth.matrix(n)
+    dA, tau, res = faulty(A, nb, [(1, phase, ft.SITE_A, i, j, bit)])
+    assert res.info == 0, res.events
+    assert res.report.detected >= 1
+    check_against_oracle(A, dA, tau, nb=nb)
+
+
+@pytest.mark.parametrize("site,i,j,bit", [(ft.SITE_Y, 50, 3, 45), (ft.SITE_Y, 100, 0, 62), (ft.SITE_Y, 10, 5, 51),
+                                          (ft.SITE_V, 60, 2, 50), (ft.SITE_V, 80, 7, 62)])
+def test_workspace_faults_redo_panel(site, i, j, bit):
+    """R15: Y/V corrupted between the panel and the updates -> pre-update check -> redo."""
+    n, nb = 128, 32
+    A = synth.matrix(n)
+    dA, tau, res = faulty(A, nb, [(1, ft.PHASE_AFTER_PANEL, site, i, j, bit)])
+    assert res.info == 0, res.events
+    assert res.report.panel_redos >= 1 or res.report.rollbacks >= 1, res.events
+    check_against_oracle(A, dA, tau, nb=nb)
+
+
+@pytest.mark.parametrize("i,j,bit", [(30, 3, 50), (100, 40, 62), (90, 70, 45)])
+def test_area3_and_finished_h_corrected_at_end(i, j, bit):
+    n, nb = 128, 32
+    A = synth.matrix(n)
+    # (i >= j+2 in a finished column: stored Householder vector; else finished H)
+    dA, tau, res = faulty(A, nb, [(0, ft.PHASE_AT_END, ft.SITE_A, i, j, bit)])
+    assert res.info == 0, res.events
+    check_against_oracle(A, dA, tau, nb=nb)
+    assert any(e[0] in ("FIX_Q", "FIX_DATA") and e[1] == -1 for e in res.events), res.events
+
+
+def test_c3_style_simultaneous_faults():
+    """C3 pattern at reduced size: two trailing flips (distinct rows/cols), a panel-workspace
+    flip (AFTER_PANEL) and a checksum flip, all in one iteration."""
+    n, nb = 512, 64
+    A = synth.matrix(n)
+    faults = [(3, ft.PHASE_BEFORE_PANEL, ft.SITE_A, 300, 400, 55),
+              (3, ft.PHASE_BEFORE_PANEL, ft.SITE_A, 350, 450, 47),
+              (3, ft.PHASE_AFTER_PANEL, ft.SITE_Y, 380, 3, 60),
+              (3, ft.PHASE_BEFORE_PANEL, ft.SITE_C, -1, 420, 52)]
+    dA, tau, res = faulty(A, nb, faults)
+    assert res.info == 0, res.events
+    check_against_oracle(A, dA, tau, nb=nb)
+    got = fixes(res.events)
+    assert ("FIX_DATA", 300, 400) in got and ("FIX_DATA", 350, 450) in got and ("FIX_C", -1, 420) in got
+
+
+def test_uncorrectable_is_reported():
+    """A rectangle of equal flips cannot be decoded: info = FT_E_UNCORRECTABLE, never a wrong answer."""
+    n, nb = 64, 16
+    A = np.ones((n, n)) + np.eye(n)  # equal entries -> equal deltas
+    f = [(1, ft.PHASE_BEFORE_PANEL, ft.SITE_A, i, j, 40) for (i, j) in [(30, 40), (30, 50), (35, 40), (35, 50)]]
+    dA, tau, res = faulty(A, nb, f)
+    assert res.info == ft.FT_E_UNCORRECTABLE
+    assert res.report.uncorrectable >= 1
+
+
+def test_abft_off_propagates_fig2():
+    """ABFT off: an error in area 2 after iteration 1 pollutes H (Fig. 2d)."""
+    n, nb = 158, 32
+    A = synth.matrix(n)
+    dA, tau, res = faulty(A, nb, [(1, ft.PHASE_BEFORE_PANEL, ft.SITE_A, 63, 127, 52)], abft=False)
+    Ao, to = oracle.dgehd2(A)
+    d = np.abs(np.triu(dA.cpu().numpy(), -1) - np.triu(Ao, -1)) > 1e-12 * np.abs(Ao).max()
+    Hm = np.triu(np.ones((n, n), bool), -1)
+    assert d[:, 33:][Hm[:, 33:]].mean() > 0.9
