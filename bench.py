@@ -246,8 +246,7 @@ def main():
         L.ft_debug_panel_ms.restype = ctypes.c_double
         L.ft_debug_panel_launches.restype = ctypes.c_int
         L.ft_debug_time_panels(1)
-        for _ in range(2):
-            one(True)
+        one(True)
         L.ft_debug_time_panels(0)
         panel_ms = L.ft_debug_panel_ms()
         nlaunch = L.ft_debug_panel_launches()

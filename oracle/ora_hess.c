@@ -357,6 +357,29 @@ int ora_decode(int n, double *L, int ldl, double *r, double *c, double *kappa,
         int nRd = 0, nCd = 0;
         for (int a = 0; a < nR; a++) if (!in_set(R[a], Rc, nRc)) Rd[nRd++] = R[a];
         for (int a = 0; a < nC; a++) if (!in_set(C[a], Cc, nCc)) Cd[nCd++] = C[a];
+        /* A flagged line with no flagged partner can only be a checksum word: when its
+         * syndrome hid inside the sum tolerance (tau < |d| <= tau*sqrt(n)), take the whole
+         * flagged set as checksum errors if it explains s_r (s_c) within that tolerance. */
+        if (nRd > 0 && nCd == 0 && nR <= 3) {
+            double sum = 0.0, sa = 0.0;
+            int small = 1; /* only syndromes that could hide inside tauS (not a cancelling pair) */
+            for (int a = 0; a < nR; a++) { sum += s.Dr[R[a]]; sa += fabs(s.Dr[R[a]]); small &= fabs(s.Dr[R[a]]) <= tauS; }
+            if (small && approx(sum, s.sr, tauS + 2.0 * n * EPS * sa)) {
+                nRc = nR;
+                for (int a = 0; a < nR; a++) Rc[a] = R[a];
+                nRd = 0;
+            }
+        }
+        if (nCd > 0 && nRd == 0 && nC <= 3) {
+            double sum = 0.0, sa = 0.0;
+            int small = 1;
+            for (int a = 0; a < nC; a++) { sum += s.Dc[C[a]]; sa += fabs(s.Dc[C[a]]); small &= fabs(s.Dc[C[a]]) <= tauS; }
+            if (small && approx(sum, s.sc, tauS + 2.0 * n * EPS * sa)) {
+                nCc = nC;
+                for (int a = 0; a < nC; a++) Cc[a] = C[a];
+                nCd = 0;
+            }
+        }
         /* (3) data errors */
         if (nRd == 0 && nCd == 0) {
             /* only checksum words were hit */

@@ -252,6 +252,26 @@ Plan decode(int n, const std::vector<double> &Dr, const std::vector<double> &Dc,
     for (int j : C)
         if (std::find(Cc.begin(), Cc.end(), j) == Cc.end()) Cd.push_back(j);
     auto pair_tol = [&](double a, double b) { return 2.0 * tau + 2.0 * n * kEps * (std::fabs(a) + std::fabs(b)); };
+    // a flagged line without a flagged partner is a checksum word whose syndrome hid inside
+    // the sum tolerance (tau < |d| <= tau sqrt(n)): accept if the whole set explains s_r / s_c
+    auto whole_set = [&](const std::vector<int> &S, const std::vector<double> &D, double target) {
+        if (S.size() > 3) return false;
+        double sum = 0.0, sa = 0.0;
+        for (int x : S) {
+            if (!(std::fabs(D[x]) <= tauS)) return false;  // large syndromes cannot hide: a cancelling pair
+            sum += D[x];
+            sa += std::fabs(D[x]);
+        }
+        return same(sum, target, tauS + 2.0 * n * kEps * sa);
+    };
+    if (!Rd.empty() && Cd.empty() && whole_set(R, Dr, sr)) {
+        Rc = R;
+        Rd.clear();
+    }
+    if (!Cd.empty() && Rd.empty() && whole_set(C, Dc, sc)) {
+        Cc = C;
+        Cd.clear();
+    }
     if (Rd.empty() != Cd.empty()) return P;
     if (!Rd.empty()) {
         if (Rd.size() == 1 && Cd.size() == 1) {

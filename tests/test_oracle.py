@@ -362,3 +362,20 @@ def test_fig2_propagation_patterns(ora):
     H = np.triu(np.ones((n, n), bool), -1)
     assert d[:, 33:][H[:, 33:]].mean() > 0.9
     assert d[:, 33:][~H[:, 33:]].mean() > 0.3
+
+
+@pytest.mark.parametrize("seed", [0, 1])
+def test_decoder_borderline_flips_never_refused_or_wrong(ora, seed):
+    """Flips whose syndrome sits between tau_abs and tau_abs*sqrt(n) (the sum tolerance):
+    every single checksum-word flip is corrected, every data flip is corrected or left
+    below the detection threshold (R16), none is refused or miscorrected."""
+    n = 16
+    A = synth.matrix(n, seed=seed, dist="normal")
+    r, c, k = ora.encode(A)
+    tau = 2.0 * n * EPS * np.linalg.norm(A)
+    for bit in range(0, 20):
+        for site in [("r", 3, -1), ("c", -1, 5), ("A", 7, 9), ("A", 0, 15)]:
+            Af, rf, cf, kf = _apply(A, r, c, k, site, bit, ora)
+            res, L, r2, c2, k2, rep = ora.decode(Af, rf, cf, kf, tau)
+            assert res in (0, 1), (site, bit, rep.events())
+            assert np.abs(L - A).max() <= 2 * tau, (site, bit)
