@@ -276,8 +276,8 @@ def test_c3_style_simultaneous_faults():
 def test_uncorrectable_is_reported():
     """A rectangle of equal flips cannot be decoded: info = FT_E_UNCORRECTABLE, never a wrong answer."""
     n, nb = 64, 16
-    A = np.ones((n, n)) + np.eye(n)  # equal entries -> equal deltas
-    f = [(1, ft.PHASE_BEFORE_PANEL, ft.SITE_A, i, j, 40) for (i, j) in [(30, 40), (30, 50), (35, 40), (35, 50)]]
+    A = np.ones((n, n)) + np.eye(n)  # entries 1.0: flipping mantissa bit 51 adds exactly +0.5 to each
+    f = [(0, ft.PHASE_BEFORE_PANEL, ft.SITE_A, i, j, 51) for (i, j) in [(30, 40), (30, 50), (35, 40), (35, 50)]]
     dA, tau, res = faulty(A, nb, f)
     assert res.info == ft.FT_E_UNCORRECTABLE
     assert res.report.uncorrectable >= 1
