@@ -51,6 +51,45 @@ FT_DEV void warp_mma(double (&acc)[MI][NI][2], const double *As, int SA, const d
     }
 }
 
+// Same with both operand layouts selectable: A(m,k) at As[m*SA+k] (AK=false) or
+// As[k*SA+m] (AK=true); B(k,n) at Bs[n*SB+k] (BK=false) or Bs[k*SB+n] (BK=true).
+// With strides = 4 (mod 16) doubles every fragment load is bank-conflict free.
+template <int MI, int NI, bool AK, bool BK>
+FT_DEV void warp_mma2(double (&acc)[MI][NI][2], const double *As, int SA, const double *Bs, int SB, int m0,
+                      int n0, int K) {
+    const int lane = threadIdx.x & 31;
+    const int lr = lane >> 2, lc = lane & 3;
+#pragma unroll 4
+    for (int k = 0; k < K; k += 4) {
+        double a[MI], b[NI];
+#pragma unroll
+        for (int mi = 0; mi < MI; mi++) {
+            int m = m0 + mi * 8 + lr;
+            a[mi] = AK ? As[(k + lc) * SA + m] : As[m * SA + k + lc];
+        }
+#pragma unroll
+        for (int ni = 0; ni < NI; ni++) {
+            int nn = n0 + ni * 8 + lr;
+            b[ni] = BK ? Bs[(k + lc) * SB + nn] : Bs[nn * SB + k + lc];
+        }
+#pragma unroll
+        for (int mi = 0; mi < MI; mi++)
+#pragma unroll
+            for (int ni = 0; ni < NI; ni++) dmma_8x8x4(acc[mi][ni][0], acc[mi][ni][1], a[mi], b[ni]);
+    }
+}
+
+// 16-byte asynchronous global->shared copy (LDGSTS); src_bytes < 16 zero-fills the tail
+FT_DEV void cp_async16(void *smem, const void *gmem, int src_bytes) {
+    unsigned s = (unsigned)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(s), "l"(gmem), "r"(src_bytes) : "memory");
+}
+FT_DEV void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
+template <int N>
+FT_DEV void cp_async_wait() {
+    asm volatile("cp.async.wait_group %0;\n" ::"n"(N) : "memory");
+}
+
 // element coordinates owned by this lane in fragment (mi, ni), v = 0/1
 FT_DEV int frag_row(int mi) { return mi * 8 + ((threadIdx.x & 31) >> 2); }
 FT_DEV int frag_col(int ni, int v) { return ni * 8 + 2 * (threadIdx.x & 3) + v; }

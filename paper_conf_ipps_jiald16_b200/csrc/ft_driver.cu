@@ -929,7 +929,25 @@ int ft_dorghr(int n, int ilo, int ihi, const double *dA, int lda, const double *
     Work &w = *wp;
     const int nb = o.nb > 0 ? o.nb : (n < 4096 ? 32 : 64);
     CK(ft_copy_in(dA, lda, w.Aw, w.ldw, n, s));  // private copy of V (dQ may alias dA)
-    CK(ft_set_identity(dQ, ldq, n, s));
+    // the DMMA tiles move 16-byte chunks: work in an aligned scratch if dQ / ldq are not
+    double *Qw = dQ;
+    int64_t ldqw = ldq;
+    static std::map<int, std::pair<size_t, double *>> qscratch;
+    if ((ldq & 1) || (((uintptr_t)dQ) & 15)) {
+        int dev = 0;
+        CK(cudaGetDevice(&dev));
+        auto &qs = qscratch[dev];
+        size_t need = (size_t)w.ldw * n;
+        if (qs.first < need) {
+            if (qs.second) cudaFree(qs.second);
+            qs.second = nullptr;
+            CK(cudaMalloc(&qs.second, need * sizeof(double)));
+            qs.first = need;
+        }
+        Qw = qs.second;
+        ldqw = w.ldw;
+    }
+    CK(ft_set_identity(Qw, ldqw, n, s));
     int npanels = 0;
     for (int k = ilo - 1; k < ihi - 2; k += nb) npanels++;
     for (int t = npanels - 1; t >= 0; t--) {
@@ -937,8 +955,8 @@ int ft_dorghr(int n, int ilo, int ihi, const double *dA, int lda, const double *
         CK(ft_build_v(w.Aw, w.ldw, w.V, n, ihi, k, ib, s));
         CK(ft_larft(w.V, w.ldw, dtau, w.T, n, ihi, k, ib, s));
         GemmRightParams g{};
-        g.A = dQ;
-        g.lda = ldq;
+        g.A = Qw;
+        g.lda = ldqw;
         g.ldw = w.ldw;
         g.Y = nullptr;
         g.V = w.V;
@@ -962,8 +980,8 @@ int ft_dorghr(int n, int ilo, int ihi, const double *dA, int lda, const double *
         g.ctl = nullptr;
         CK(ft_launch_gemm_right(g, s));
         GemmLeftParams L{};
-        L.A = dQ;
-        L.lda = ldq;
+        L.A = Qw;
+        L.lda = ldqw;
         L.ldw = w.ldw;
         L.V = w.V;
         L.T = w.T;
@@ -980,6 +998,9 @@ int ft_dorghr(int n, int ilo, int ihi, const double *dA, int lda, const double *
         L.ctl = nullptr;
         CK(ft_launch_gemm_left(L, s));
     }
+    if (Qw != dQ)
+        CK(cudaMemcpy2DAsync(dQ, (size_t)ldq * sizeof(double), Qw, (size_t)ldqw * sizeof(double),
+                             (size_t)n * sizeof(double), n, cudaMemcpyDeviceToDevice, s));
     CK(cudaStreamSynchronize(s));
     return 0;
 }

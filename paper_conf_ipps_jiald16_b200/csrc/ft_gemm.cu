@@ -15,130 +15,126 @@
 #include "ft_common.cuh"
 #include "ft_internal.h"
 
-#define GB_N 64   // strip width
+#define GB_N 64   // strip width (columns of the updated matrix per CTA)
 #define GB_M 32   // row tile
-#define GT 128    // threads
-#define CS_LD (GB_M + 4)
+#define GT 128    // threads (4 warps)
+#define TS (GB_M + 4)   // smem stride of row-indexed tiles (36 = 4 mod 16: conflict-free)
 
-struct RightSmem {
-    double Vs[GB_N * FT_KPAD];  // V(cols, :)   [col][j]
-    double Ys[GB_M * FT_KPAD];  // sign*Y(rows,:) [row][j]
-    double Vt[GB_M * FT_KPAD];  // V(rows, :)   [row][j]  (W operand)
-    double Cs[GB_N * CS_LD];    // C tile        [col][row]
+template <int KT>
+struct RightSmemT {
+    double Vs[KT][GB_N + 4];  // V(cols, j) as [j][col]: B operand of the right update (k-major)
+    struct Stage {
+        double Cs[GB_N][TS];  // C tile [col][row] (column-major, as in HBM)
+        double Ys[KT][TS];    // Y(rows, j) as [j][row]
+        double Vt[KT][TS];    // V(rows, j) as [j][row]: A operand of W = V^T C
+    } st[2];
 };
 
-// load a [GB_M x KT] column-major block (rows r.., columns 0..KT-1 of M, ld) into smem
-// as [row][j] (stride FT_KPAD), scaled; zero outside rows [lo, hi) and columns [0, K).
-// All loads of a thread are issued before any store (memory-level parallelism).
+// stage loaders (cp.async 16 B chunks; rows >= hi of the tile are zero-filled, never read)
+__device__ __forceinline__ void issue_ctile(double (*Cs)[TS], const double *A, int64_t lda, int cb, int r, int hi,
+                                            int ncols) {
+    for (int q = threadIdx.x; q < GB_N * (GB_M / 2); q += GT) {
+        int cc = q / (GB_M / 2), m2 = (q % (GB_M / 2)) * 2;
+        int rows_left = hi - (r + m2);
+        int bytes = (cc < ncols) ? (rows_left >= 2 ? 16 : (rows_left == 1 ? 8 : 0)) : 0;
+        const double *src = bytes ? A + (int64_t)(cb + cc) * lda + r + m2 : A;
+        cp_async16(&Cs[cc][m2], src, bytes);
+    }
+}
 template <int KT>
-__device__ __forceinline__ void load_rows_rowmajor(double *dst, const double *M, int64_t ld, int r, int K, int lo,
-                                                   int hi, double scale) {
-    constexpr int PER = GB_M * KT / GT;
-    double v[PER];
-#pragma unroll
-    for (int u = 0; u < PER; u++) {
-        int i = threadIdx.x + u * GT;
-        int m = i % GB_M, jj = i / GB_M;
-        int rr = r + m;
-        v[u] = (jj < K && rr >= lo && rr < hi) ? M[rr + (int64_t)jj * ld] * scale : 0.0;
-    }
-#pragma unroll
-    for (int u = 0; u < PER; u++) {
-        int i = threadIdx.x + u * GT;
-        dst[(i % GB_M) * FT_KPAD + i / GB_M] = v[u];
+__device__ __forceinline__ void issue_jtile(double (*T)[TS], const double *M, int64_t ld, int r, int K) {
+    for (int q = threadIdx.x; q < KT * (GB_M / 2); q += GT) {
+        int jj = q / (GB_M / 2), m2 = (q % (GB_M / 2)) * 2;
+        int bytes = jj < K ? 16 : 0;
+        const double *src = bytes ? M + (int64_t)jj * ld + r + m2 : M;
+        cp_async16(&T[jj][m2], src, bytes);
     }
 }
-// V(cols, 0:KT) for a 64-column strip -> smem [col][j]
+// zero rows of a [KT][TS] tile outside [lo, hi) (tile rows r .. r+GB_M)
 template <int KT>
-__device__ __forceinline__ void load_strip_rowmajor(double *dst, const double *M, int64_t ld, int c0, int K, int ncols) {
-    constexpr int PER = GB_N * KT / GT;
-#pragma unroll 8
-    for (int u = 0; u < PER; u++) {
-        int i = threadIdx.x + u * GT;
-        int m = i % GB_N, jj = i / GB_N;
-        dst[m * FT_KPAD + jj] = (jj < K && m < ncols) ? M[(c0 + m) + (int64_t)jj * ld] : 0.0;
+__device__ __forceinline__ void mask_jtile(double (*T)[TS], int r, int lo, int hi) {
+    if (r >= lo && r + GB_M <= hi) return;
+    for (int q = threadIdx.x; q < KT * GB_M; q += GT) {
+        int jj = q / GB_M, m = q % GB_M;
+        if (r + m < lo || r + m >= hi) T[jj][m] = 0.0;
     }
 }
-// C tile (GB_M rows x GB_N cols) -> registers (8 double2 per thread) -> smem [col][row];
-// only rows m in [mlo, mhi) of the tile are touched in global memory (others read as 0)
-__device__ __forceinline__ void load_ctile(double *Cs, const double *A, int64_t lda, int cb, int r, int mlo, int mhi,
-                                           int ncols, bool vec_ok) {
-    constexpr int PER = GB_N * (GB_M / 2) / GT;
-    double2 v[PER];
-#pragma unroll
-    for (int u = 0; u < PER; u++) {
-        int i = threadIdx.x + u * GT;
-        int cc = i / (GB_M / 2), m2 = (i % (GB_M / 2)) * 2;
-        v[u] = make_double2(0.0, 0.0);
-        if (cc < ncols) {
-            const double *src = A + (int64_t)(cb + cc) * lda + r + m2;
-            if (vec_ok && m2 >= mlo && m2 + 1 < mhi) {
-                v[u] = *reinterpret_cast<const double2 *>(src);
-            } else {
-                if (m2 >= mlo && m2 < mhi) v[u].x = src[0];
-                if (m2 + 1 >= mlo && m2 + 1 < mhi) v[u].y = src[1];
-            }
-        }
-    }
-#pragma unroll
-    for (int u = 0; u < PER; u++) {
-        int i = threadIdx.x + u * GT;
-        int cc = i / (GB_M / 2), m2 = (i % (GB_M / 2)) * 2;
-        *reinterpret_cast<double2 *>(&Cs[cc * CS_LD + m2]) = v[u];
-    }
-}
-__device__ __forceinline__ void store_ctile(const double *Cs, double *A, int64_t lda, int cb, int r, int mlo, int mhi,
-                                            int ncols, bool vec_ok) {
-    constexpr int PER = GB_N * (GB_M / 2) / GT;
-#pragma unroll
-    for (int u = 0; u < PER; u++) {
-        int i = threadIdx.x + u * GT;
-        int cc = i / (GB_M / 2), m2 = (i % (GB_M / 2)) * 2;
+__device__ __forceinline__ void store_ctile2(double (*Cs)[TS], double *A, int64_t lda, int cb, int r, int lo, int hi,
+                                             int ncols) {
+    for (int q = threadIdx.x; q < GB_N * (GB_M / 2); q += GT) {
+        int cc = q / (GB_M / 2), m2 = (q % (GB_M / 2)) * 2;
         if (cc >= ncols) continue;
-        double *dst = A + (int64_t)(cb + cc) * lda + r + m2;
-        double2 v = *reinterpret_cast<const double2 *>(&Cs[cc * CS_LD + m2]);
-        if (vec_ok && m2 >= mlo && m2 + 1 < mhi) {
+        int row = r + m2;
+        double *dst = A + (int64_t)(cb + cc) * lda + row;
+        double2 v = *reinterpret_cast<const double2 *>(&Cs[cc][m2]);
+        if (row >= lo && row + 1 < hi) {
             *reinterpret_cast<double2 *>(dst) = v;
         } else {
-            if (m2 >= mlo && m2 < mhi) dst[0] = v.x;
-            if (m2 + 1 >= mlo && m2 + 1 < mhi) dst[1] = v.y;
+            if (row >= lo && row < hi) dst[0] = v.x;
+            if (row + 1 >= lo && row + 1 < hi) dst[1] = v.y;
         }
     }
 }
 
+// ---------------------------------------------------------------------------
+// Right update A(rows, cols) += sign * Y V(cols,:)^T, fused W = V(wrows,:)^T A_new
+// ---------------------------------------------------------------------------
 template <int KT>
-__global__ void __launch_bounds__(GT, 2) k_gemm_right(GemmRightParams p) {
+__global__ void __launch_bounds__(GT) k_gemm_right(GemmRightParams p) {
     if (p.ctl && p.ctl->halt) return;
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    RightSmem &S = *reinterpret_cast<RightSmem *>(smem_raw);
+    RightSmemT<KT> &S = *reinterpret_cast<RightSmemT<KT> *>(smem_raw);
     const int warp = threadIdx.x >> 5;
     const int cb = p.c_lo + blockIdx.x * GB_N;
     const int ncols = min(GB_N, p.c_hi - cb);
     const int K = p.K;
-    const bool vec_ok = ((p.lda & 1) == 0) && ((((uintptr_t)p.A) & 15) == 0);
-    // row tiles are aligned to absolute multiples of GB_M (16-byte aligned columns)
-    const int rbase = (p.r_lo / GB_M) * GB_M;
+    const double sg = p.sign;
+    const int rbase = (p.r_lo / GB_M) * GB_M;  // 256-byte aligned tiles
     const int nrt = (p.r_hi - rbase + GB_M - 1) / GB_M;
     const int t0 = (int)((long long)blockIdx.y * nrt / gridDim.y);
     const int t1 = (int)((long long)(blockIdx.y + 1) * nrt / gridDim.y);
 
-    if (p.do_right) load_strip_rowmajor<KT>(S.Vs, p.V, p.ldw, cb, K, ncols);
-    double wacc[4][4][2];
+    // V(cols, :) once per CTA, [j][col]
+    if (p.do_right)
+        for (int q = threadIdx.x; q < KT * GB_N; q += GT) {
+            int jj = q / GB_N, cc = q % GB_N;
+            S.Vs[jj][cc] = (jj < K && cc < ncols) ? p.V[(cb + cc) + (int64_t)jj * p.ldw] : 0.0;
+        }
+    constexpr int WMI = 4, WNI = KT == 64 ? 4 : 2;  // W warp tile: 32 j x (8*WNI) cols
+    double wacc[WMI][WNI][2];
 #pragma unroll
-    for (int a = 0; a < 4; a++)
+    for (int a = 0; a < WMI; a++)
 #pragma unroll
-        for (int b = 0; b < 4; b++) wacc[a][b][0] = wacc[a][b][1] = 0.0;
+        for (int b = 0; b < WNI; b++) wacc[a][b][0] = wacc[a][b][1] = 0.0;
+    const int wm0 = KT == 64 ? (warp >> 1) * 32 : 0;
+    const int wn0 = KT == 64 ? (warp & 1) * 32 : warp * 16;
 
+    auto issue = [&](int tt, int s) {
+        const int r = rbase + tt * GB_M;
+        const int hi = min(r + GB_M, p.r_hi);
+        issue_ctile(S.st[s].Cs, p.A, p.lda, cb, r, hi, ncols);
+        if (p.do_right) issue_jtile<KT>(S.st[s].Ys, p.Y, p.ldw, r, K);
+        if (p.do_w) issue_jtile<KT>(S.st[s].Vt, p.V, p.ldw, r, K);
+        cp_async_commit();
+    };
+    if (t0 < t1) issue(t0, 0);
     for (int tt = t0; tt < t1; tt++) {
+        const int s = (tt - t0) & 1;
         const int r = rbase + tt * GB_M;
         const int lo = max(r, p.r_lo), hi = min(r + GB_M, p.r_hi);
+        if (tt + 1 < t1) {
+            issue(tt + 1, s ^ 1);
+            cp_async_wait<1>();
+        } else {
+            cp_async_wait<0>();
+        }
         __syncthreads();
-        if (p.do_right) load_rows_rowmajor<KT>(S.Ys, p.Y, p.ldw, r, K, lo, hi, p.sign);
-        if (p.do_w) load_rows_rowmajor<KT>(S.Vt, p.V, p.ldw, r, K, max(lo, p.wr_lo), min(hi, p.wr_hi), 1.0);
-        load_ctile(S.Cs, p.A, p.lda, cb, r, lo - r, hi - r, ncols, vec_ok);
-        __syncthreads();
+        auto &St = S.st[s];
+        if (p.do_w) {
+            mask_jtile<KT>(St.Vt, r, max(lo, p.wr_lo), min(hi, p.wr_hi));
+        }
         if (p.do_right) {
-            // warp owns rows 0..31 x cols warp*16 .. +16; rows outside [lo, hi) carry Y = 0
+            // C' = C + sg * Y V^T:  acc = sg*C ; acc += Y V^T ; C' = sg*acc
             double acc[4][2][2];
 #pragma unroll
             for (int mi = 0; mi < 4; mi++)
@@ -146,47 +142,45 @@ __global__ void __launch_bounds__(GT, 2) k_gemm_right(GemmRightParams p) {
                 for (int ni = 0; ni < 2; ni++)
 #pragma unroll
                     for (int v = 0; v < 2; v++)
-                        acc[mi][ni][v] = S.Cs[(warp * 16 + frag_col(ni, v)) * CS_LD + frag_row(mi)];
-            warp_mma<4, 2, false>(acc, S.Ys, FT_KPAD, S.Vs, FT_KPAD, 0, warp * 16, KT);
-            __syncwarp();
+                        acc[mi][ni][v] = sg * St.Cs[warp * 16 + frag_col(ni, v)][frag_row(mi)];
+            warp_mma2<4, 2, true, true>(acc, &St.Ys[0][0], TS, &S.Vs[0][0], GB_N + 4, 0, warp * 16, KT);
 #pragma unroll
             for (int mi = 0; mi < 4; mi++)
 #pragma unroll
                 for (int ni = 0; ni < 2; ni++)
 #pragma unroll
                     for (int v = 0; v < 2; v++)
-                        S.Cs[(warp * 16 + frag_col(ni, v)) * CS_LD + frag_row(mi)] = acc[mi][ni][v];
+                        St.Cs[warp * 16 + frag_col(ni, v)][frag_row(mi)] = sg * acc[mi][ni][v];
             __syncthreads();
-            store_ctile(S.Cs, p.A, p.lda, cb, r, lo - r, hi - r, ncols, vec_ok);
+            store_ctile2(St.Cs, p.A, p.lda, cb, r, lo, hi, ncols);
+        } else if (p.do_w) {
+            __syncthreads();
         }
         if (p.do_w) {
-            // W (KT x 64) += V_tile^T (KT x 32) * C (32 x 64); warp tile 32 x 32
-            const int wm0 = (warp >> 1) * 32, wn0 = (warp & 1) * 32;
-            if (wm0 < KT) warp_mma<4, 4, true>(wacc, S.Vt, FT_KPAD, S.Cs, CS_LD, wm0, wn0, GB_M);
+            // rows outside [lo, hi) of the C tile are stale/zero, Vt is zero there
+            warp_mma2<WMI, WNI, false, false>(wacc, &St.Vt[0][0], TS, &St.Cs[0][0], TS, wm0, wn0, GB_M);
         }
+        __syncthreads();
     }
     if (p.do_w) {
-        const int wm0 = (warp >> 1) * 32, wn0 = (warp & 1) * 32;
         double *Wp = p.Wpart + (int64_t)blockIdx.y * p.wsplit_stride;
-        if (wm0 < KT) {
 #pragma unroll
-            for (int mi = 0; mi < 4; mi++)
+        for (int mi = 0; mi < WMI; mi++)
 #pragma unroll
-                for (int ni = 0; ni < 4; ni++)
+            for (int ni = 0; ni < WNI; ni++)
 #pragma unroll
-                    for (int v = 0; v < 2; v++) {
-                        int jj = wm0 + frag_row(mi);
-                        int cc = wn0 + frag_col(ni, v);
-                        if (jj < K && cc < ncols) Wp[(int64_t)(cb + cc) * FT_NBMAX + jj] = wacc[mi][ni][v];
-                    }
-        }
+                for (int v = 0; v < 2; v++) {
+                    int jj = wm0 + frag_row(mi);
+                    int cc = wn0 + frag_col(ni, v);
+                    if (jj < K && cc < ncols) Wp[(int64_t)(cb + cc) * FT_NBMAX + jj] = wacc[mi][ni][v];
+                }
     }
 }
 
 template <int KT>
 static cudaError_t launch_right_kt(const GemmRightParams &p, cudaStream_t s) {
     static bool attr = false;
-    size_t smem = sizeof(RightSmem);
+    size_t smem = sizeof(RightSmemT<KT>);
     if (!attr) {
         cudaError_t e = cudaFuncSetAttribute(k_gemm_right<KT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return e;
@@ -200,100 +194,116 @@ static cudaError_t launch_right_kt(const GemmRightParams &p, cudaStream_t s) {
 }
 cudaError_t ft_launch_gemm_right(const GemmRightParams &p, cudaStream_t s) {
     if (p.r_hi <= p.r_lo || p.c_hi <= p.c_lo || p.K <= 0) return cudaSuccess;
+    const bool aligned = (p.lda % 2 == 0) && ((((uintptr_t)p.A) & 15) == 0) && (p.ldw % 2 == 0) &&
+                         ((((uintptr_t)p.V) & 15) == 0) && (!p.do_right || ((((uintptr_t)p.Y) & 15) == 0));
+    if (!aligned) return cudaErrorInvalidValue;  // the library only passes 16-byte aligned operands
     return p.K <= 32 ? launch_right_kt<32>(p, s) : launch_right_kt<64>(p, s);
 }
 
 // ---------------------------------------------------------------------------
 // Left update: A(rows, cols) += sign * V(rows,:) (op(T) W(:, cols))
 // ---------------------------------------------------------------------------
-struct LeftSmem {
-    double Wp[GB_N * FT_KPAD];  // sign*op(T) W [col][j]
+template <int KT>
+struct LeftSmemT {
+    double Wp[GB_N][KT + 4];  // op(T) W as [col][j]: B operand (n-major)
     union {
-        struct {                // prologue only
-            double Ts[FT_NBMAX * FT_NBMAX];
-            double Wr[GB_N * FT_KPAD];  // raw W [col][j]
+        struct {
+            double Ts[KT][KT];
+            double Wr[GB_N][KT + 4];
         } pro;
-        struct {                // main loop
-            double Vt[GB_M * FT_KPAD];
-            double Cs[GB_N * CS_LD];
-        } main;
+        struct {
+            double Cs[GB_N][TS];
+            double Vt[KT][TS];
+        } st[2];
     } u;
 };
 
 template <int KT>
-__global__ void __launch_bounds__(GT, 2) k_gemm_left(GemmLeftParams p) {
+__global__ void __launch_bounds__(GT) k_gemm_left(GemmLeftParams p) {
     if (p.ctl && p.ctl->halt) return;
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    LeftSmem &S = *reinterpret_cast<LeftSmem *>(smem_raw);
+    LeftSmemT<KT> &S = *reinterpret_cast<LeftSmemT<KT> *>(smem_raw);
     const int warp = threadIdx.x >> 5;
     const int cb = p.c_lo + blockIdx.x * GB_N;
     const int ncols = min(GB_N, p.c_hi - cb);
     const int K = p.K;
-    const bool vec_ok = ((p.lda & 1) == 0) && ((((uintptr_t)p.A) & 15) == 0);
+    const double sg = p.sign;
     const int rbase = (p.r_lo / GB_M) * GB_M;
     const int nrt = (p.r_hi - rbase + GB_M - 1) / GB_M;
     const int t0 = (int)((long long)blockIdx.y * nrt / gridDim.y);
     const int t1 = (int)((long long)(blockIdx.y + 1) * nrt / gridDim.y);
 
-    for (int i = threadIdx.x; i < K * K; i += blockDim.x) {
-        int a = i % K, b = i / K;
-        S.u.pro.Ts[a + b * FT_NBMAX] = p.T[a + b * FT_NBMAX];
+    for (int i = threadIdx.x; i < KT * KT; i += GT) {
+        int a = i % KT, b = i / KT;
+        S.u.pro.Ts[b][a] = (a < K && b < K) ? p.T[a + b * FT_NBMAX] : 0.0;  // Ts[b][a] = T(a,b)
     }
-    for (int i = threadIdx.x; i < GB_N * KT; i += blockDim.x) {
+    for (int i = threadIdx.x; i < GB_N * KT; i += GT) {
         int jj = i % KT, cc = i / KT;
         double sacc = 0.0;
         if (cc < ncols && jj < K)
             for (int sp = 0; sp < p.nsplit; sp++)
                 sacc += p.Wpart[sp * p.wsplit_stride + (int64_t)(cb + cc) * FT_NBMAX + jj];
-        S.u.pro.Wr[cc * FT_KPAD + jj] = sacc;
+        S.u.pro.Wr[cc][jj] = sacc;
     }
     __syncthreads();
-    // Wp(a, col) = sign * sum_b op(T)(a, b) W(b, col);  T upper triangular
-    for (int i = threadIdx.x; i < GB_N * KT; i += blockDim.x) {
+    // Wp(col, a) = sum_b op(T)(a, b) W(b, col);  T upper triangular
+    for (int i = threadIdx.x; i < GB_N * KT; i += GT) {
         int a = i % KT, cc = i / KT;
         double sacc = 0.0;
         if (a < K) {
             if (p.transT) {
-                for (int b = 0; b <= a; b++) sacc += S.u.pro.Ts[b + a * FT_NBMAX] * S.u.pro.Wr[cc * FT_KPAD + b];
+                for (int b = 0; b <= a; b++) sacc += S.u.pro.Ts[a][b] * S.u.pro.Wr[cc][b];  // T(b,a)
             } else {
-                for (int b = a; b < K; b++) sacc += S.u.pro.Ts[a + b * FT_NBMAX] * S.u.pro.Wr[cc * FT_KPAD + b];
+                for (int b = a; b < K; b++) sacc += S.u.pro.Ts[b][a] * S.u.pro.Wr[cc][b];  // T(a,b)
             }
         }
-        S.Wp[cc * FT_KPAD + a] = p.sign * sacc;
+        S.Wp[cc][a] = sacc;
     }
+    __syncthreads();
+    auto issue = [&](int tt, int s) {
+        const int r = rbase + tt * GB_M;
+        const int hi = min(r + GB_M, p.r_hi);
+        issue_ctile(S.u.st[s].Cs, p.A, p.lda, cb, r, hi, ncols);
+        issue_jtile<KT>(S.u.st[s].Vt, p.V, p.ldw, r, K);
+        cp_async_commit();
+    };
+    if (t0 < t1) issue(t0, 0);
     for (int tt = t0; tt < t1; tt++) {
+        const int s = (tt - t0) & 1;
         const int r = rbase + tt * GB_M;
         const int lo = max(r, p.r_lo), hi = min(r + GB_M, p.r_hi);
+        if (tt + 1 < t1) {
+            issue(tt + 1, s ^ 1);
+            cp_async_wait<1>();
+        } else {
+            cp_async_wait<0>();
+        }
         __syncthreads();
-        load_rows_rowmajor<KT>(S.u.main.Vt, p.V, p.ldw, r, K, lo, hi, 1.0);
-        load_ctile(S.u.main.Cs, p.A, p.lda, cb, r, lo - r, hi - r, ncols, vec_ok);
-        __syncthreads();
+        auto &St = S.u.st[s];
         double acc[4][2][2];
 #pragma unroll
         for (int mi = 0; mi < 4; mi++)
 #pragma unroll
             for (int ni = 0; ni < 2; ni++)
 #pragma unroll
-                for (int v = 0; v < 2; v++)
-                    acc[mi][ni][v] = S.u.main.Cs[(warp * 16 + frag_col(ni, v)) * CS_LD + frag_row(mi)];
-        warp_mma<4, 2, false>(acc, S.u.main.Vt, FT_KPAD, S.Wp, FT_KPAD, 0, warp * 16, KT);
-        __syncwarp();
+                for (int v = 0; v < 2; v++) acc[mi][ni][v] = sg * St.Cs[warp * 16 + frag_col(ni, v)][frag_row(mi)];
+        warp_mma2<4, 2, true, false>(acc, &St.Vt[0][0], TS, &S.Wp[0][0], KT + 4, 0, warp * 16, KT);
 #pragma unroll
         for (int mi = 0; mi < 4; mi++)
 #pragma unroll
             for (int ni = 0; ni < 2; ni++)
 #pragma unroll
-                for (int v = 0; v < 2; v++)
-                    S.u.main.Cs[(warp * 16 + frag_col(ni, v)) * CS_LD + frag_row(mi)] = acc[mi][ni][v];
+                for (int v = 0; v < 2; v++) St.Cs[warp * 16 + frag_col(ni, v)][frag_row(mi)] = sg * acc[mi][ni][v];
         __syncthreads();
-        store_ctile(S.u.main.Cs, p.A, p.lda, cb, r, lo - r, hi - r, ncols, vec_ok);
+        store_ctile2(St.Cs, p.A, p.lda, cb, r, lo, hi, ncols);
+        __syncthreads();
     }
 }
 
 template <int KT>
 static cudaError_t launch_left_kt(const GemmLeftParams &p, cudaStream_t s) {
     static bool attr = false;
-    size_t smem = sizeof(LeftSmem);
+    size_t smem = sizeof(LeftSmemT<KT>);
     if (!attr) {
         cudaError_t e = cudaFuncSetAttribute(k_gemm_left<KT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return e;
@@ -310,6 +320,9 @@ static cudaError_t launch_left_kt(const GemmLeftParams &p, cudaStream_t s) {
 }
 cudaError_t ft_launch_gemm_left(const GemmLeftParams &p, cudaStream_t s) {
     if (p.r_hi <= p.r_lo || p.c_hi <= p.c_lo || p.K <= 0) return cudaSuccess;
+    const bool aligned = (p.lda % 2 == 0) && ((((uintptr_t)p.A) & 15) == 0) && (p.ldw % 2 == 0) &&
+                         ((((uintptr_t)p.V) & 15) == 0);
+    if (!aligned) return cudaErrorInvalidValue;
     return p.K <= 32 ? launch_left_kt<32>(p, s) : launch_left_kt<64>(p, s);
 }
 
