@@ -513,3 +513,15 @@ cudaError_t ft_set_identity(double *Q, int64_t ldq, int n, cudaStream_t s) {
     k_identity<<<dim3((n + 255) / 256, n), 256, 0, s>>>(Q, ldq, n);
     return cudaGetLastError();
 }
+
+__global__ void k_zero_if_running(double *p, size_t n, const FtCtl *ctl) {
+    if (ctl && ctl->halt) return;
+    for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) p[i] = 0.0;
+}
+cudaError_t ft_zero_if_running(double *p, size_t n, const FtCtl *ctl, cudaStream_t s) {
+    g_ft_launches++;
+    int blocks = (int)((n + 1023) / 1024);
+    if (blocks > 592) blocks = 592;
+    k_zero_if_running<<<blocks, 256, 0, s>>>(p, n, ctl);
+    return cudaGetLastError();
+}

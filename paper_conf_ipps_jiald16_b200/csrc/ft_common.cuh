@@ -112,11 +112,11 @@ FT_DEV void grid_barrier(unsigned *count, unsigned &epoch, unsigned nblocks) {
     if (threadIdx.x == 0) {
         epoch += 1;
         const unsigned target = epoch * nblocks;
-        __threadfence();
+        // release is cumulative over the CTA's writes ordered before it by bar.sync;
+        // the acquire load orders everything after it (PTX memory model)
         red_release_add_u32(count, 1u);
         while (ld_acquire_u32(count) < target) {
         }
-        __threadfence();
     }
     __syncthreads();
 }

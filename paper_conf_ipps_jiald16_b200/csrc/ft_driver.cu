@@ -21,6 +21,8 @@
 int64_t g_ft_launches = 0;
 static int g_dbg_panel = -1;
 static unsigned long long *g_dbg_buf = nullptr;
+static int g_dbg_mode = 0;
+extern "C" void ft_debug_ablate(int mode) { g_dbg_mode = mode; }
 extern "C" void ft_debug_probe_panel(int panel, unsigned long long *dbuf) {
     g_dbg_panel = panel;
     g_dbg_buf = dbuf;
@@ -75,6 +77,7 @@ constexpr int kYtopRows = 296 * 64;  // max (Y_top splits x rows) kept in ypart
 struct Work {
     int n_cap = -1;
     int64_t ldw = 0;
+    double *Wt = nullptr;
     double *Aw = nullptr, *V = nullptr, *Y = nullptr, *T = nullptr, *Wpart = nullptr, *bvec = nullptr,
            *acc = nullptr, *ckpt = nullptr, *ck_r = nullptr, *ck_c = nullptr, *ck_q = nullptr, *Fr = nullptr,
            *Qr = nullptr, *Qc = nullptr, *Dr = nullptr, *Dc = nullptr, *sums = nullptr, *ypart = nullptr,
@@ -85,7 +88,7 @@ struct Work {
     int nsm = 0;
     size_t bytes = 0;
     void release() {
-        double **ps[] = {&Aw, &V, &Y, &T, &Wpart, &bvec, &acc, &ckpt, &ck_r, &ck_c, &ck_q, &Fr, &Qr, &Qc, &Dr, &Dc,
+        double **ps[] = {&Wt, &Aw, &V, &Y, &T, &Wpart, &bvec, &acc, &ckpt, &ck_r, &ck_c, &ck_q, &Fr, &Qr, &Qc, &Dr, &Dc,
                          &sums, &ypart, &rowpart, &scratch, &deltas, &hA, &htau};
         for (auto p : ps) {
             if (*p) cudaFree(*p);
@@ -130,6 +133,7 @@ int get_work(int n, Work **out) {
     A(dalloc(&w.Y, (size_t)ldw * FT_NBMAX, b));
     A(dalloc(&w.T, (size_t)FT_NBMAX * FT_NBMAX, b));
     A(dalloc(&w.Wpart, (size_t)kMaxWsplit * (N1 + 64) * FT_NBMAX, b));
+    A(dalloc(&w.Wt, (N1 + 64) * FT_NBMAX, b));
     A(dalloc(&w.bvec, (size_t)ldw, b));
     A(dalloc(&w.acc, (size_t)3 * FT_ACC_STRIDE, b));
     A(dalloc(&w.ckpt, (size_t)ldw * FT_NBMAX, b));
@@ -477,6 +481,8 @@ int right_update(Call &C, int t, double sign, int do_w) {
     ns = std::min(ns, std::max(1, nrt / 2));
     ns = std::max(1, std::min(ns, kMaxWsplit));
     g.nsplit = ns;
+    // zero W with a halt-aware kernel: after a halt, W of the halted iteration is needed by the rollback
+    if (do_w && ns > 1) CK(ft_zero_if_running(w.Wpart, (size_t)(C.n + 1 + 64) * FT_NBMAX, w.ctl, C.s));
     CK(ft_launch_gemm_right(g, C.s));
     return 0;
 }
@@ -491,6 +497,7 @@ int left_update(Call &C, int t, double sign, int nsplit) {
     g.V = w.V;
     g.T = w.T;
     g.Wpart = w.Wpart;
+    g.Wt = w.Wt;
     g.r_lo = k + 1;
     g.r_hi = C.rend();
     g.c_lo = e;
@@ -542,6 +549,7 @@ int enqueue_panel(Call &C, int t) {
     p.abft = C.abft;
     p.verify = eager ? 1 : 0;
     p.dbg = (t == g_dbg_panel) ? g_dbg_buf : nullptr;
+    p.dbg_mode = (t == g_dbg_panel) ? g_dbg_mode : 0;
     p.rbase = ((k + 1) / 16) * 16;
     int rendp = (C.rend() + 15) / 16 * 16;
     p.ngroups = (rendp - p.rbase) / 16;
@@ -978,6 +986,7 @@ int ft_dorghr(int n, int ilo, int ihi, const double *dA, int lda, const double *
         ns = std::max(1, std::min({ns, std::max(1, nrt / 2), kMaxWsplit}));
         g.nsplit = ns;
         g.ctl = nullptr;
+        if (ns > 1) CK(cudaMemsetAsync(w.Wpart, 0, (size_t)(n + 1 + 64) * FT_NBMAX * sizeof(double), s));
         CK(ft_launch_gemm_right(g, s));
         GemmLeftParams L{};
         L.A = Qw;
@@ -986,6 +995,7 @@ int ft_dorghr(int n, int ilo, int ihi, const double *dA, int lda, const double *
         L.V = w.V;
         L.T = w.T;
         L.Wpart = w.Wpart;
+        L.Wt = w.Wt;
         L.r_lo = k + 1;
         L.r_hi = ihi;
         L.c_lo = k + 1;

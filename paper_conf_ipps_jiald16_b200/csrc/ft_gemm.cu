@@ -95,11 +95,20 @@ __global__ void __launch_bounds__(GT) k_gemm_right(GemmRightParams p) {
     const int t1 = (int)((long long)(blockIdx.y + 1) * nrt / gridDim.y);
 
     // V(cols, :) once per CTA, [j][col]
-    if (p.do_right)
-        for (int q = threadIdx.x; q < KT * GB_N; q += GT) {
-            int jj = q / GB_N, cc = q % GB_N;
-            S.Vs[jj][cc] = (jj < K && cc < ncols) ? p.V[(cb + cc) + (int64_t)jj * p.ldw] : 0.0;
+    if (p.do_right) {
+        constexpr int PER = KT * GB_N / GT;
+        double tmp[PER];
+#pragma unroll
+        for (int u = 0; u < PER; u++) {
+            int q = threadIdx.x + u * GT, jj = q / GB_N, cc = q % GB_N;
+            tmp[u] = (jj < K && cc < ncols) ? __ldg(p.V + (cb + cc) + (int64_t)jj * p.ldw) : 0.0;
         }
+#pragma unroll
+        for (int u = 0; u < PER; u++) {
+            int q = threadIdx.x + u * GT;
+            S.Vs[q / GB_N][q % GB_N] = tmp[u];
+        }
+    }
     constexpr int WMI = 4, WNI = KT == 64 ? 4 : 2;  // W warp tile: 32 j x (8*WNI) cols
     double wacc[WMI][WNI][2];
 #pragma unroll
@@ -163,7 +172,8 @@ __global__ void __launch_bounds__(GT) k_gemm_right(GemmRightParams p) {
         __syncthreads();
     }
     if (p.do_w) {
-        double *Wp = p.Wpart + (int64_t)blockIdx.y * p.wsplit_stride;
+        // row splits of a strip accumulate into one W (fp64 RED at L2; W zeroed by the host)
+        double *Wp = p.Wpart;
 #pragma unroll
         for (int mi = 0; mi < WMI; mi++)
 #pragma unroll
@@ -172,7 +182,11 @@ __global__ void __launch_bounds__(GT) k_gemm_right(GemmRightParams p) {
                 for (int v = 0; v < 2; v++) {
                     int jj = wm0 + frag_row(mi);
                     int cc = wn0 + frag_col(ni, v);
-                    if (jj < K && cc < ncols) Wp[(int64_t)(cb + cc) * FT_NBMAX + jj] = wacc[mi][ni][v];
+                    if (jj < K && cc < ncols) {
+                        double *dst = Wp + (int64_t)(cb + cc) * FT_NBMAX + jj;
+                        if (gridDim.y == 1) *dst = wacc[mi][ni][v];
+                        else atomicAdd(dst, wacc[mi][ni][v]);
+                    }
                 }
     }
 }
@@ -206,17 +220,44 @@ cudaError_t ft_launch_gemm_right(const GemmRightParams &p, cudaStream_t s) {
 template <int KT>
 struct LeftSmemT {
     double Wp[GB_N][KT + 4];  // op(T) W as [col][j]: B operand (n-major)
-    union {
-        struct {
-            double Ts[KT][KT];
-            double Wr[GB_N][KT + 4];
-        } pro;
-        struct {
-            double Cs[GB_N][TS];
-            double Vt[KT][TS];
-        } st[2];
-    } u;
+    struct {
+        double Cs[GB_N][TS];
+        double Vt[KT][TS];
+    } st[2];
 };
+
+// W'(col, a) = sum_b op(T)(a, b) W(b, col), T upper triangular; W, W' stored [col][64]
+__global__ void k_wprep(const double *__restrict__ W, const double *__restrict__ T, double *__restrict__ Wt,
+                        int c_lo, int c_hi, int K, int transT, const FtCtl *ctl) {
+    if (ctl && ctl->halt) return;
+    __shared__ double Ts[FT_NBMAX][FT_NBMAX + 1];
+    for (int i = threadIdx.x; i < K * K; i += blockDim.x) {
+        int a = i % K, b = i / K;
+        Ts[a][b] = T[a + b * FT_NBMAX];
+    }
+    __syncthreads();
+    const int a = threadIdx.x % FT_NBMAX;
+    const int col = c_lo + blockIdx.x * (blockDim.x / FT_NBMAX) + threadIdx.x / FT_NBMAX;
+    if (col >= c_hi || a >= K) return;
+    const double *w = W + (int64_t)col * FT_NBMAX;
+    double s0 = 0.0, s1 = 0.0;
+    if (transT) {
+        int b = 0;
+        for (; b + 1 <= a; b += 2) {
+            s0 += Ts[b][a] * w[b];
+            s1 += Ts[b + 1][a] * w[b + 1];
+        }
+        if (b <= a) s0 += Ts[b][a] * w[b];
+    } else {
+        int b = a;
+        for (; b + 1 < K; b += 2) {
+            s0 += Ts[a][b] * w[b];
+            s1 += Ts[a][b + 1] * w[b + 1];
+        }
+        if (b < K) s0 += Ts[a][b] * w[b];
+    }
+    Wt[(int64_t)col * FT_NBMAX + a] = s0 + s1;
+}
 
 template <int KT>
 __global__ void __launch_bounds__(GT) k_gemm_left(GemmLeftParams p) {
@@ -233,41 +274,22 @@ __global__ void __launch_bounds__(GT) k_gemm_left(GemmLeftParams p) {
     const int t0 = (int)((long long)blockIdx.y * nrt / gridDim.y);
     const int t1 = (int)((long long)(blockIdx.y + 1) * nrt / gridDim.y);
 
-    for (int i = threadIdx.x; i < KT * KT; i += GT) {
-        int a = i % KT, b = i / KT;
-        S.u.pro.Ts[b][a] = (a < K && b < K) ? p.T[a + b * FT_NBMAX] : 0.0;  // Ts[b][a] = T(a,b)
+    // W' for this strip: [col][j] rows of 64 doubles in HBM -> [col][KT+4] in smem
+    for (int q = threadIdx.x; q < GB_N * (KT / 2); q += GT) {
+        int cc = q / (KT / 2), j2 = (q % (KT / 2)) * 2;
+        int bytes = cc < ncols ? 16 : 0;
+        const double *src = bytes ? p.Wpart + (int64_t)(cb + cc) * FT_NBMAX + j2 : p.Wpart;
+        cp_async16(&S.Wp[cc][j2], src, bytes);
     }
-    for (int i = threadIdx.x; i < GB_N * KT; i += GT) {
-        int jj = i % KT, cc = i / KT;
-        double sacc = 0.0;
-        if (cc < ncols && jj < K)
-            for (int sp = 0; sp < p.nsplit; sp++)
-                sacc += p.Wpart[sp * p.wsplit_stride + (int64_t)(cb + cc) * FT_NBMAX + jj];
-        S.u.pro.Wr[cc][jj] = sacc;
-    }
-    __syncthreads();
-    // Wp(col, a) = sum_b op(T)(a, b) W(b, col);  T upper triangular
-    for (int i = threadIdx.x; i < GB_N * KT; i += GT) {
-        int a = i % KT, cc = i / KT;
-        double sacc = 0.0;
-        if (a < K) {
-            if (p.transT) {
-                for (int b = 0; b <= a; b++) sacc += S.u.pro.Ts[a][b] * S.u.pro.Wr[cc][b];  // T(b,a)
-            } else {
-                for (int b = a; b < K; b++) sacc += S.u.pro.Ts[b][a] * S.u.pro.Wr[cc][b];  // T(a,b)
-            }
-        }
-        S.Wp[cc][a] = sacc;
-    }
-    __syncthreads();
     auto issue = [&](int tt, int s) {
         const int r = rbase + tt * GB_M;
         const int hi = min(r + GB_M, p.r_hi);
-        issue_ctile(S.u.st[s].Cs, p.A, p.lda, cb, r, hi, ncols);
-        issue_jtile<KT>(S.u.st[s].Vt, p.V, p.ldw, r, K);
+        issue_ctile(S.st[s].Cs, p.A, p.lda, cb, r, hi, ncols);
+        issue_jtile<KT>(S.st[s].Vt, p.V, p.ldw, r, K);
         cp_async_commit();
     };
     if (t0 < t1) issue(t0, 0);
+    else cp_async_commit();
     for (int tt = t0; tt < t1; tt++) {
         const int s = (tt - t0) & 1;
         const int r = rbase + tt * GB_M;
@@ -279,7 +301,7 @@ __global__ void __launch_bounds__(GT) k_gemm_left(GemmLeftParams p) {
             cp_async_wait<0>();
         }
         __syncthreads();
-        auto &St = S.u.st[s];
+        auto &St = S.st[s];
         double acc[4][2][2];
 #pragma unroll
         for (int mi = 0; mi < 4; mi++)
@@ -314,8 +336,13 @@ static cudaError_t launch_left_kt(const GemmLeftParams &p, cudaStream_t s) {
     int ny = (2 * 148 + nstrip - 1) / nstrip;
     if (ny > nrt / 2) ny = nrt / 2;
     if (ny < 1) ny = 1;
-    g_ft_launches++;
-    k_gemm_left<KT><<<dim3(nstrip, ny), GT, smem, s>>>(p);
+    g_ft_launches += 2;
+    const int per = GT / FT_NBMAX;  // columns per k_wprep block
+    k_wprep<<<(p.c_hi - p.c_lo + per - 1) / per, GT, 0, s>>>(p.Wpart, p.T, p.Wt, p.c_lo, p.c_hi, p.K, p.transT,
+                                                              p.ctl);
+    GemmLeftParams q = p;
+    q.Wpart = p.Wt;  // the main kernel reads W' = op(T) W
+    k_gemm_left<KT><<<dim3(nstrip, ny), GT, smem, s>>>(q);
     return cudaGetLastError();
 }
 cudaError_t ft_launch_gemm_left(const GemmLeftParams &p, cudaStream_t s) {

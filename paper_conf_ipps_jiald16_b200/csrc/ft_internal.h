@@ -42,6 +42,7 @@ struct PanelParams {
     int rbase, ngroups;               // 16-row groups starting at rbase
     int smem_rows;                    // set by the launcher: V/Y rows cached in shared memory
     unsigned long long *dbg;          // optional per-column phase timestamps (CTA 0), or NULL
+    int dbg_mode;                     // timing ablations (wrong results): 1 no grid barriers, 2 no GEMV, 4 no atomics
 };
 
 // launchers (return cudaError_t of the launch)
@@ -68,7 +69,8 @@ struct GemmLeftParams {
     double *A;
     int64_t lda;
     int64_t ldw;
-    const double *V, *T, *Wpart;
+    const double *V, *T, *Wpart;  // Wpart: W = V^T A (accumulated, [col][64])
+    double *Wt;                     // scratch for W' = op(T) W ([col][64])
     int r_lo, r_hi, c_lo, c_hi, K;
     int nsplit;
     int64_t wsplit_stride;
@@ -101,6 +103,7 @@ cudaError_t ft_decide(const double *Y, const double *V, const double *T, int64_t
                       int ib, int panel, FtCtl *ctl, cudaStream_t s);
 cudaError_t ft_endcheck(double *Aw, int64_t ldw, int n, int ihi, int k, int ib, int panel, int policy,
                         double *Fr, FtCtl *ctl, cudaStream_t s);
+cudaError_t ft_zero_if_running(double *p, size_t n, const FtCtl *ctl, cudaStream_t s);
 cudaError_t ft_inject(double *addr, int fidx, int bit, FtCtl *ctl, cudaStream_t s);
 // full verification (recovery path / final): mode 0 = H logical, 1 = Q (V region)
 cudaError_t ft_full_verify(const double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdone, int mode,

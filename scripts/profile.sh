@@ -10,8 +10,8 @@ ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/
     python scratch/prof1.py 2048 1 > /dev/null 2>&1
 ncu --set full --clock-control none --import-source on -k regex:k_panel -s 10 -c 1 -o $OUT/prof_panel \
     python scratch/prof1.py 2048 1 > /dev/null 2>&1
-ncu --set full --clock-control none --import-source on -k regex:k_gemm_right -s 21 -c 1 -o $OUT/prof_right \
+ncu --set full --clock-control none --import-source on -k regex:k_gemm_right -s 41 -c 1 -o $OUT/prof_right \
     python scratch/prof1.py 2048 1 > /dev/null 2>&1
-ncu --set full --clock-control none --import-source on -k regex:k_gemm_left -s 10 -c 1 -o $OUT/prof_left \
+ncu --set full --clock-control none --import-source on -k regex:k_gemm_left -s 20 -c 1 -o $OUT/prof_left \
     python scratch/prof1.py 2048 1 > /dev/null 2>&1
 ls -la $OUT
