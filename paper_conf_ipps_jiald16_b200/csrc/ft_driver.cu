@@ -135,7 +135,7 @@ int get_work(int n, Work **out) {
     A(dalloc(&w.Wpart, (size_t)kMaxWsplit * (N1 + 64) * FT_NBMAX, b));
     A(dalloc(&w.Wt, (N1 + 64) * FT_NBMAX, b));
     A(dalloc(&w.bvec, (size_t)ldw, b));
-    A(dalloc(&w.acc, (size_t)3 * FT_ACC_STRIDE, b));
+    A(dalloc(&w.acc, (size_t)FT_ACC_SETS * FT_ACC_STRIDE, b));
     A(dalloc(&w.ckpt, (size_t)ldw * FT_NBMAX, b));
     A(dalloc(&w.ck_r, (size_t)ldw, b));
     A(dalloc(&w.ck_c, N1, b));
@@ -521,14 +521,21 @@ int trailing_nsplit(Call &C, int t) {
     return std::max(1, std::min(ns, kMaxWsplit));
 }
 
+// panel-kernel sync state: barrier counters and accumulator sets must be zero when a
+// sequence of panel launches starts (the kernels recycle them afterwards)
+int reset_panel_state(Call &C) {
+    Work &w = *C.w;
+    CK(cudaMemsetAsync(w.bar, 0, 4 * sizeof(unsigned), C.s));
+    CK(cudaMemsetAsync(w.acc, 0, (size_t)FT_ACC_SETS * FT_ACC_STRIDE * sizeof(double), C.s));
+    return 0;
+}
+
 int enqueue_panel(Call &C, int t) {
     Work &w = *C.w;
     const int n = C.n, k = C.pk(t), ib = C.pib(t);
     const bool eager = C.abft && C.policy == FT_POLICY_EAGER;
     if (inject_at(C, t, FT_PHASE_BEFORE_PANEL)) return FT_E_CUDA;
     if (C.abft && checkpoint(C, t, 0)) return FT_E_CUDA;
-    CK(cudaMemsetAsync(w.bar, 0, 4 * sizeof(unsigned), C.s));
-    CK(cudaMemsetAsync(w.acc, 0, 3 * FT_ACC_STRIDE * sizeof(double), C.s));
     PanelParams p{};
     p.A = w.Aw;
     p.ldw = w.ldw;
@@ -538,7 +545,8 @@ int enqueue_panel(Call &C, int t) {
     p.tau = C.tau;
     p.bvec = w.bvec;
     p.acc = w.acc;
-    p.bar = w.bar;
+    p.bar = w.bar + (t & 1);
+    p.bar_next = w.bar + ((t + 1) & 1);
     p.ctl = w.ctl;
     p.Qr = w.Qr;
     p.Qc = w.Qc;
@@ -550,9 +558,10 @@ int enqueue_panel(Call &C, int t) {
     p.verify = eager ? 1 : 0;
     p.dbg = (t == g_dbg_panel) ? g_dbg_buf : nullptr;
     p.dbg_mode = (t == g_dbg_panel) ? g_dbg_mode : 0;
-    p.rbase = ((k + 1) / 16) * 16;
-    int rendp = (C.rend() + 15) / 16 * 16;
-    p.ngroups = (rendp - p.rbase) / 16;
+    const int gr = ft_panel_group_rows();
+    p.rbase = ((k + 1) / gr) * gr;
+    int rendp = (C.rend() + gr - 1) / gr * gr;
+    p.ngroups = (rendp - p.rbase) / gr;
     cudaEvent_t pe0 = nullptr, pe1 = nullptr;
     if (g_time_panels) {
         CK(cudaEventCreate(&pe0));
@@ -706,6 +715,7 @@ int recover(Call &C, const FtCtl &h) {
     }
     // restore the pre-factorized panel and the checksum vectors (diskless checkpoint)
     if (checkpoint(C, t, 1)) return FT_E_CUDA;
+    if (reset_panel_state(C)) return FT_E_CUDA;
     bool found = false;
     int info = verify_and_correct(C, t, k, 0, &found);
     return info;
@@ -767,6 +777,8 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
     CK(cudaMemsetAsync(w.V, 0, (size_t)w.ldw * FT_NBMAX * sizeof(double), s));
     CK(cudaMemsetAsync(w.Y, 0, (size_t)w.ldw * FT_NBMAX * sizeof(double), s));
     CK(ft_copy_in(dA, lda, w.Aw, w.ldw, n, s));
+    CK(cudaMemsetAsync(w.bvec, 0, (size_t)w.ldw * sizeof(double), s));  // b(q >= ihi) must read 0
+    if (reset_panel_state(C)) return FT_E_CUDA;
     if (C.abft) {
         CK(ft_encode(w.Aw, w.ldw, n, w.ctl, w.scratch, s));
         CK(cudaMemsetAsync(w.Fr, 0, w.ldw * sizeof(double), s));

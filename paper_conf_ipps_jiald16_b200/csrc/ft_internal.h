@@ -11,6 +11,7 @@
 #define FT_NBMAX 64
 #endif
 #define FT_ACC_STRIDE (2 * 64 + 8)  // [s1 | vtb | nrm2 sx alpha ...] per reduction set
+#define FT_ACC_SETS 4               // sets indexed by the global column mod 4 (recycled in-kernel)
 
 // Device-resident control block: halt protocol, fused-verify flags, injector log.
 struct FtCtl {
@@ -35,12 +36,12 @@ struct PanelParams {
     double *A;
     int64_t ldw;
     double *V, *Y, *T, *tau, *bvec, *acc;
-    unsigned *bar;
+    unsigned *bar;       // grid-barrier counter of this launch (zero at launch)
+    unsigned *bar_next;  // the next panel launch's counter (zeroed by this launch)
     FtCtl *ctl;
     double *Qr, *Qc;
     int n, ihi, k, ib, abft, verify;  // verify: fused D_r on the first GEMV (EAGER policy)
-    int rbase, ngroups;               // 16-row groups starting at rbase
-    int smem_rows;                    // set by the launcher: V/Y rows cached in shared memory
+    int rbase, ngroups;               // ft_panel_group_rows()-row groups starting at rbase
     unsigned long long *dbg;          // optional per-column phase timestamps (CTA 0), or NULL
     int dbg_mode;                     // timing ablations (wrong results): 1 no grid barriers, 2 no GEMV, 4 no atomics
 };
@@ -48,6 +49,7 @@ struct PanelParams {
 // launchers (return cudaError_t of the launch)
 cudaError_t ft_launch_panel(const PanelParams &p, int nsm, cudaStream_t s);
 size_t ft_panel_smem_bytes();
+int ft_panel_group_rows();
 
 struct GemmRightParams {
     double *A;

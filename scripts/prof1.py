@@ -1,0 +1,88 @@
+#!/usr/bin/env python3
+"""Profiling driver: run `reps` ABFT reductions of the synthetic n x n matrix (one GPU).
+
+  python scripts/prof1.py N [reps] [--nb NB] [--abft 0|1] [--probe PANEL] [--ablate MODE]
+
+Prints per-call milliseconds (CUDA events), the panel kernel's share (live events) and,
+with --probe, the per-column phase timestamps (clock64 cycles, CTA 0) of one panel.
+Used under ncu (scripts/profile.sh) and for quick timing; never a bench value.
+"""
+import argparse
+import ctypes
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("n", type=int)
+    ap.add_argument("reps", type=int, nargs="?", default=1)
+    ap.add_argument("--nb", type=int, default=0)
+    ap.add_argument("--abft", type=int, default=1)
+    ap.add_argument("--probe", type=int, default=-1)
+    ap.add_argument("--ablate", type=int, default=0)
+    a = ap.parse_args()
+    import torch
+
+    import paper_conf_ipps_jiald16_b200 as ft
+    import synth
+
+    n = a.n
+    A = synth.matrix(n)
+    dA0 = ft.fortran(torch.from_numpy(A).cuda())
+    dA = ft.fortran(torch.empty((n, n), dtype=torch.float64, device="cuda"))
+    tau = torch.zeros(n, dtype=torch.float64, device="cuda")
+    L = ft.lib()
+    L.ft_debug_time_panels.argtypes = [ctypes.c_int]
+    L.ft_debug_panel_ms.restype = ctypes.c_double
+    L.ft_debug_panel_launches.restype = ctypes.c_int
+    dbg = None
+    if a.probe >= 0:
+        dbg = torch.zeros(2048, dtype=torch.int64, device="cuda")
+        L.ft_debug_probe_panel.argtypes = [ctypes.c_int, ctypes.c_void_p]
+        L.ft_debug_probe_panel(a.probe, ctypes.c_void_p(dbg.data_ptr()))
+        L.ft_debug_ablate.argtypes = [ctypes.c_int]
+        L.ft_debug_ablate(a.ablate)
+    s = torch.cuda.current_stream()
+    for it in range(a.reps):
+        dA.copy_(dA0)
+        L.ft_debug_time_panels(1)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(s)
+        _, res = ft.dgehrd(dA, tau=tau, nb=a.nb, abft=bool(a.abft), stream=s)
+        e1.record(s)
+        torch.cuda.synchronize()
+        L.ft_debug_time_panels(0)
+        ms = e0.elapsed_time(e1)
+        pms = L.ft_debug_panel_ms()
+        print(f"rep {it}: n={n} info={res.info} {ms:.3f} ms  panel {pms:.3f} ms "
+              f"({L.ft_debug_panel_launches()} launches, {100 * pms / ms:.1f}%)  "
+              f"{10 / 3 * n ** 3 / ms / 1e6:.1f} Gflop/s", flush=True)
+    if dbg is not None:
+        d = dbg.cpu().numpy()
+        names = {0: "start", 1: "s1_dots", 2: "sync1", 3: "w", 4: "x_dots", 5: "sync2", 6: "dlarfg",
+                 7: "gemv", 8: "red_sync", 9: "y_v_t"}
+        order = [0, 1, 2, 3, 4, 5, 6, 7, 8, 9]
+        tot = {}
+        ncol = 0
+        for j in range(64):
+            row = d[j * 16: j * 16 + 16]
+            if row[0] == 0:
+                continue
+            ncol += 1
+            prev = row[0]
+            for sl in order[1:]:
+                if row[sl] == 0:
+                    continue
+                tot[names[sl]] = tot.get(names[sl], 0) + (row[sl] - prev)
+                prev = row[sl]
+        print(f"probe panel {a.probe}: {ncol} columns, mean cycles per column by phase:")
+        for k2, v in tot.items():
+            print(f"  {k2:10s} {v / max(ncol, 1):10.0f}")
+
+
+if __name__ == "__main__":
+    main()

@@ -7,11 +7,11 @@ mkdir -p $OUT
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,clocks.mem --format=csv > $OUT/gpu.txt
 python bench.py --steps 5 --warmup 3 > $OUT/bench.json 2> $OUT/bench.err
 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches.csv \
-    python scratch/prof1.py 2048 1 > /dev/null 2>&1
+    python scripts/prof1.py 2048 1 > /dev/null 2>&1
 ncu --set full --clock-control none --import-source on -k regex:k_panel -s 10 -c 1 -o $OUT/prof_panel \
-    python scratch/prof1.py 2048 1 > /dev/null 2>&1
+    python scripts/prof1.py 2048 1 > /dev/null 2>&1
 ncu --set full --clock-control none --import-source on -k regex:k_gemm_right -s 41 -c 1 -o $OUT/prof_right \
-    python scratch/prof1.py 2048 1 > /dev/null 2>&1
+    python scripts/prof1.py 2048 1 > /dev/null 2>&1
 ncu --set full --clock-control none --import-source on -k regex:k_gemm_left -s 20 -c 1 -o $OUT/prof_left \
-    python scratch/prof1.py 2048 1 > /dev/null 2>&1
+    python scripts/prof1.py 2048 1 > /dev/null 2>&1
 ls -la $OUT
