@@ -71,7 +71,7 @@ const double kEps = 2.220446049250313e-16;
 // ---------------------------------------------------------------------------
 // workspace (cached per device, grown on demand)
 // ---------------------------------------------------------------------------
-constexpr int kMaxWsplit = 16;
+constexpr int kMaxWsplit = FT_WSPLIT_MAX;
 constexpr int kYtopRows = 296 * 64;  // max (Y_top splits x rows) kept in ypart
 
 struct Work {
@@ -465,7 +465,7 @@ int right_update(Call &C, int t, double sign, int do_w) {
     g.c_hi = e;
     g.do_right = 1;
     g.do_w = 0;
-    g.nsplit = 1;
+    g.nsplit = ft_gemm_splits(g.r_lo, g.r_hi, g.c_lo, g.c_hi, w.nsm);
     CK(ft_launch_gemm_right(g, C.s));
     // trailing block (+ checksum row/column), fused with W = V^T A_new
     g.r_lo = 0;
@@ -475,14 +475,7 @@ int right_update(Call &C, int t, double sign, int do_w) {
     g.wr_lo = k + 1;
     g.wr_hi = C.ihi;
     g.do_w = do_w;
-    int nstrip = (g.c_hi - g.c_lo + 63) / 64;
-    int nrt = (g.r_hi + 31) / 32;
-    int ns = (2 * w.nsm + nstrip - 1) / std::max(nstrip, 1);
-    ns = std::min(ns, std::max(1, nrt / 2));
-    ns = std::max(1, std::min(ns, kMaxWsplit));
-    g.nsplit = ns;
-    // zero W with a halt-aware kernel: after a halt, W of the halted iteration is needed by the rollback
-    if (do_w && ns > 1) CK(ft_zero_if_running(w.Wpart, (size_t)(C.n + 1 + 64) * FT_NBMAX, w.ctl, C.s));
+    g.nsplit = ft_gemm_splits(g.r_lo, g.r_hi, g.c_lo, g.c_hi, w.nsm);
     CK(ft_launch_gemm_right(g, C.s));
     return 0;
 }
@@ -513,12 +506,8 @@ int left_update(Call &C, int t, double sign, int nsplit) {
 }
 
 int trailing_nsplit(Call &C, int t) {
-    const int k = C.pk(t), ib = C.pib(t), e = k + ib;
-    int nstrip = (C.cend() - e + 63) / 64;
-    int nrt = (C.rend() + 31) / 32;
-    int ns = (2 * C.w->nsm + nstrip - 1) / std::max(nstrip, 1);
-    ns = std::min(ns, std::max(1, nrt / 2));
-    return std::max(1, std::min(ns, kMaxWsplit));
+    const int e = C.pk(t) + C.pib(t);
+    return ft_gemm_splits(0, C.rend(), e, C.cend(), C.w->nsm);
 }
 
 // panel-kernel sync state: barrier counters and accumulator sets must be zero when a
@@ -992,13 +981,9 @@ int ft_dorghr(int n, int ilo, int ihi, const double *dA, int lda, const double *
         g.sign = 1.0;
         g.Wpart = w.Wpart;
         g.wsplit_stride = ((int64_t)n + 1 + 64) * FT_NBMAX;
-        int nstrip = (ihi - k - 1 + 63) / 64;
-        int nrt = (ihi - k - 1 + 31) / 32;
-        int ns = (2 * w.nsm + nstrip - 1) / std::max(nstrip, 1);
-        ns = std::max(1, std::min({ns, std::max(1, nrt / 2), kMaxWsplit}));
+        const int ns = ft_gemm_splits(k + 1, ihi, k + 1, ihi, w.nsm);
         g.nsplit = ns;
         g.ctl = nullptr;
-        if (ns > 1) CK(cudaMemsetAsync(w.Wpart, 0, (size_t)(n + 1 + 64) * FT_NBMAX * sizeof(double), s));
         CK(ft_launch_gemm_right(g, s));
         GemmLeftParams L{};
         L.A = Qw;

@@ -7,186 +7,186 @@
 // the column checksum c -- so Theorem 1 is carried by the same tiles.
 // Rollback (reverse computation, Alg. 3 l.14) is the same kernels with sign +1.
 //
-// Tiling: a CTA owns a 64-column strip and a contiguous row range; it walks the rows in
-// 32-row tiles staged in shared memory (coalesced 16-byte loads), the MMA is
-// mma.sync.m8n8k4.f64 (SASS DMMA) on 4 warps.  W partials are written per row split and
-// reduced (with T^T) in the prologue of the left-update kernel, so both passes are
-// deterministic.
 #include "ft_common.cuh"
 #include "ft_internal.h"
 
-#define GB_N 64   // strip width (columns of the updated matrix per CTA)
-#define GB_M 32   // row tile
-#define GT 128    // threads (4 warps)
-#define TS (GB_M + 4)   // smem stride of row-indexed tiles (36 = 4 mod 16: conflict-free)
+// Tiling (both kernels): a CTA owns a 64-column strip and a contiguous range of 64-row
+// tiles.  The MMA is formulated on the transpose, D = C^T (cols x rows), so that an
+// accumulator fragment holds two CONSECUTIVE rows of one column: the C tile moves between
+// HBM and the DMMA accumulators with 16-byte vector loads/stores and never touches shared
+// memory.  The small operands (V, Y, W') are k-major cp.async tiles in shared memory with
+// a stride of 68 doubles (= 4 mod 16: every fragment load is bank-conflict free).
+//   right:  D(cols, rows) += V(cols, :) Y(rows, :)^T,  then  W^T(cols, :) += C_new^T V(rows, :)
+//           -- C_new^T as the A operand comes from the accumulators by an in-warp shuffle
+//   left:   D(cols, rows) += W'^T(cols, :) V(rows, :)^T
+// W partials are written per row split and summed (with op(T)) by k_wprep, so every pass
+// is deterministic.
+#define UB 64   // tile rows / strip columns
+#define UT 256  // threads (8 warps)
+#define SK 68   // smem stride of the k-major operand tiles
+
+int ft_gemm_splits(int r_lo, int r_hi, int c_lo, int c_hi, int nsm) {
+    const int nstrip = (c_hi - c_lo + UB - 1) / UB;
+    const int nrt = (r_hi - (r_lo / UB) * UB + UB - 1) / UB;
+    int ns = (2 * nsm + nstrip - 1) / (nstrip > 0 ? nstrip : 1);
+    if (ns > nrt) ns = nrt;
+    if (ns > FT_WSPLIT_MAX) ns = FT_WSPLIT_MAX;
+    return ns < 1 ? 1 : ns;
+}
 
 template <int KT>
 struct RightSmemT {
-    double Vs[KT][GB_N + 4];  // V(cols, j) as [j][col]: B operand of the right update (k-major)
-    struct Stage {
-        double Cs[GB_N][TS];  // C tile [col][row] (column-major, as in HBM)
-        double Ys[KT][TS];    // Y(rows, j) as [j][row]
-        double Vt[KT][TS];    // V(rows, j) as [j][row]: A operand of W = V^T C
-    } st[2];
+    double Vc[KT][SK];  // V(cols, k) as [k][col]   (A operand of the right update)
+    double Ys[KT][SK];  // Y(rows, k) as [k][row]   (B operand of the right update)
+    double Vr[KT][SK];  // V(rows, j) as [j][row]   (B operand of W^T = C_new^T V)
 };
 
-// stage loaders (cp.async 16 B chunks; rows >= hi of the tile are zero-filled, never read)
-__device__ __forceinline__ void issue_ctile(double (*Cs)[TS], const double *A, int64_t lda, int cb, int r, int hi,
-                                            int ncols) {
-    for (int q = threadIdx.x; q < GB_N * (GB_M / 2); q += GT) {
-        int cc = q / (GB_M / 2), m2 = (q % (GB_M / 2)) * 2;
-        int rows_left = hi - (r + m2);
-        int bytes = (cc < ncols) ? (rows_left >= 2 ? 16 : (rows_left == 1 ? 8 : 0)) : 0;
-        const double *src = bytes ? A + (int64_t)(cb + cc) * lda + r + m2 : A;
-        cp_async16(&Cs[cc][m2], src, bytes);
-    }
-}
+// k-major operand tile: M(r .. r+63, 0:KT) (column-major, leading dim ld) -> T[k][row];
+// rows >= hi and k >= K are zero-filled
 template <int KT>
-__device__ __forceinline__ void issue_jtile(double (*T)[TS], const double *M, int64_t ld, int r, int K) {
-    for (int q = threadIdx.x; q < KT * (GB_M / 2); q += GT) {
-        int jj = q / (GB_M / 2), m2 = (q % (GB_M / 2)) * 2;
-        int bytes = jj < K ? 16 : 0;
-        const double *src = bytes ? M + (int64_t)jj * ld + r + m2 : M;
-        cp_async16(&T[jj][m2], src, bytes);
+__device__ __forceinline__ void issue_ktile(double (*T)[SK], const double *M, int64_t ld, int r, int hi, int K) {
+    for (int q = threadIdx.x; q < KT * (UB / 2); q += UT) {
+        const int kk = q / (UB / 2), m2 = (q % (UB / 2)) * 2;
+        const int left = hi - (r + m2);
+        const int bytes = kk < K ? (left >= 2 ? 16 : (left == 1 ? 8 : 0)) : 0;
+        cp_async16(&T[kk][m2], bytes ? M + (int64_t)kk * ld + r + m2 : M, bytes);
     }
 }
-// zero rows of a [KT][TS] tile outside [lo, hi) (tile rows r .. r+GB_M)
-template <int KT>
-__device__ __forceinline__ void mask_jtile(double (*T)[TS], int r, int lo, int hi) {
-    if (r >= lo && r + GB_M <= hi) return;
-    for (int q = threadIdx.x; q < KT * GB_M; q += GT) {
-        int jj = q / GB_M, m = q % GB_M;
-        if (r + m < lo || r + m >= hi) T[jj][m] = 0.0;
-    }
+
+// acc(pair) <- C(row, row+1 ; col) with rows outside [lo, hi) (or a missing column) as 0
+__device__ __forceinline__ double2 load_pair(const double *colp, int row, int lo, int hi, bool colok) {
+    double2 v = make_double2(0.0, 0.0);
+    if (!colok) return v;
+    if (row >= lo && row + 1 < hi) return *reinterpret_cast<const double2 *>(colp + row);
+    if (row >= lo && row < hi) v.x = colp[row];
+    if (row + 1 >= lo && row + 1 < hi) v.y = colp[row + 1];
+    return v;
 }
-__device__ __forceinline__ void store_ctile2(double (*Cs)[TS], double *A, int64_t lda, int cb, int r, int lo, int hi,
-                                             int ncols) {
-    for (int q = threadIdx.x; q < GB_N * (GB_M / 2); q += GT) {
-        int cc = q / (GB_M / 2), m2 = (q % (GB_M / 2)) * 2;
-        if (cc >= ncols) continue;
-        int row = r + m2;
-        double *dst = A + (int64_t)(cb + cc) * lda + row;
-        double2 v = *reinterpret_cast<const double2 *>(&Cs[cc][m2]);
-        if (row >= lo && row + 1 < hi) {
-            *reinterpret_cast<double2 *>(dst) = v;
-        } else {
-            if (row >= lo && row < hi) dst[0] = v.x;
-            if (row + 1 >= lo && row + 1 < hi) dst[1] = v.y;
-        }
+__device__ __forceinline__ void store_pair(double *colp, int row, int lo, int hi, bool colok, double x, double y) {
+    if (!colok) return;
+    if (row >= lo && row + 1 < hi) {
+        *reinterpret_cast<double2 *>(colp + row) = make_double2(x, y);
+        return;
     }
+    if (row >= lo && row < hi) colp[row] = x;
+    if (row + 1 >= lo && row + 1 < hi) colp[row + 1] = y;
 }
 
 // ---------------------------------------------------------------------------
 // Right update A(rows, cols) += sign * Y V(cols,:)^T, fused W = V(wrows,:)^T A_new
+// warp w owns columns w*8 .. w*8+7 of the strip and all 64 rows of a tile (8 fragments)
 // ---------------------------------------------------------------------------
 template <int KT>
-__global__ void __launch_bounds__(GT) k_gemm_right(GemmRightParams p) {
+__global__ void __launch_bounds__(UT, 2) k_gemm_right(GemmRightParams p) {
     if (p.ctl && p.ctl->halt) return;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     RightSmemT<KT> &S = *reinterpret_cast<RightSmemT<KT> *>(smem_raw);
-    const int warp = threadIdx.x >> 5;
-    const int cb = p.c_lo + blockIdx.x * GB_N;
-    const int ncols = min(GB_N, p.c_hi - cb);
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int lr = lane >> 2, lc = lane & 3;
+    const int cb = p.c_lo + blockIdx.x * UB;
+    const int ncols = min(UB, p.c_hi - cb);
     const int K = p.K;
     const double sg = p.sign;
-    const int rbase = (p.r_lo / GB_M) * GB_M;  // 256-byte aligned tiles
-    const int nrt = (p.r_hi - rbase + GB_M - 1) / GB_M;
+    const int rbase = (p.r_lo / UB) * UB;
+    const int nrt = (p.r_hi - rbase + UB - 1) / UB;
     const int t0 = (int)((long long)blockIdx.y * nrt / gridDim.y);
     const int t1 = (int)((long long)(blockIdx.y + 1) * nrt / gridDim.y);
+    constexpr int NJ = KT / 8;
+    const int wcol = warp * 8 + lr;  // this lane's column inside the strip (D row)
+    const bool colok = wcol < ncols;
+    double *colp = p.A + (int64_t)(cb + (colok ? wcol : 0)) * p.lda;
 
-    // V(cols, :) once per CTA, [j][col]
-    if (p.do_right) {
-        constexpr int PER = KT * GB_N / GT;
-        double tmp[PER];
-#pragma unroll
-        for (int u = 0; u < PER; u++) {
-            int q = threadIdx.x + u * GT, jj = q / GB_N, cc = q % GB_N;
-            tmp[u] = (jj < K && cc < ncols) ? __ldg(p.V + (cb + cc) + (int64_t)jj * p.ldw) : 0.0;
-        }
-#pragma unroll
-        for (int u = 0; u < PER; u++) {
-            int q = threadIdx.x + u * GT;
-            S.Vs[q / GB_N][q % GB_N] = tmp[u];
+    if (p.do_right) {  // V(cols, :) once per CTA (plain loads: cb may be odd)
+        for (int i = tid; i < KT * UB; i += UT) {
+            const int kk = i / UB, cc = i % UB;
+            S.Vc[kk][cc] = (kk < K && cc < ncols) ? __ldg(p.V + (cb + cc) + (int64_t)kk * p.ldw) : 0.0;
         }
     }
-    constexpr int WMI = 4, WNI = KT == 64 ? 4 : 2;  // W warp tile: 32 j x (8*WNI) cols
-    double wacc[WMI][WNI][2];
+    double wacc[NJ][2];
 #pragma unroll
-    for (int a = 0; a < WMI; a++)
-#pragma unroll
-        for (int b = 0; b < WNI; b++) wacc[a][b][0] = wacc[a][b][1] = 0.0;
-    const int wm0 = KT == 64 ? (warp >> 1) * 32 : 0;
-    const int wn0 = KT == 64 ? (warp & 1) * 32 : warp * 16;
+    for (int a = 0; a < NJ; a++) wacc[a][0] = wacc[a][1] = 0.0;
 
-    auto issue = [&](int tt, int s) {
-        const int r = rbase + tt * GB_M;
-        const int hi = min(r + GB_M, p.r_hi);
-        issue_ctile(S.st[s].Cs, p.A, p.lda, cb, r, hi, ncols);
-        if (p.do_right) issue_jtile<KT>(S.st[s].Ys, p.Y, p.ldw, r, K);
-        if (p.do_w) issue_jtile<KT>(S.st[s].Vt, p.V, p.ldw, r, K);
+    // pipeline invariant at the top of tile tt: groups [Ys(tt), Vr(tt)] in flight
+    if (t0 < t1) {
+        if (p.do_right) issue_ktile<KT>(S.Ys, p.Y, p.ldw, rbase + t0 * UB, p.r_hi, K);
         cp_async_commit();
-    };
-    if (t0 < t1) issue(t0, 0);
-    for (int tt = t0; tt < t1; tt++) {
-        const int s = (tt - t0) & 1;
-        const int r = rbase + tt * GB_M;
-        const int lo = max(r, p.r_lo), hi = min(r + GB_M, p.r_hi);
-        if (tt + 1 < t1) {
-            issue(tt + 1, s ^ 1);
-            cp_async_wait<1>();
-        } else {
-            cp_async_wait<0>();
-        }
-        __syncthreads();
-        auto &St = S.st[s];
-        if (p.do_w) {
-            mask_jtile<KT>(St.Vt, r, max(lo, p.wr_lo), min(hi, p.wr_hi));
-        }
-        if (p.do_right) {
-            // C' = C + sg * Y V^T:  acc = sg*C ; acc += Y V^T ; C' = sg*acc
-            double acc[4][2][2];
-#pragma unroll
-            for (int mi = 0; mi < 4; mi++)
-#pragma unroll
-                for (int ni = 0; ni < 2; ni++)
-#pragma unroll
-                    for (int v = 0; v < 2; v++)
-                        acc[mi][ni][v] = sg * St.Cs[warp * 16 + frag_col(ni, v)][frag_row(mi)];
-            warp_mma2<4, 2, true, true>(acc, &St.Ys[0][0], TS, &S.Vs[0][0], GB_N + 4, 0, warp * 16, KT);
-#pragma unroll
-            for (int mi = 0; mi < 4; mi++)
-#pragma unroll
-                for (int ni = 0; ni < 2; ni++)
-#pragma unroll
-                    for (int v = 0; v < 2; v++)
-                        St.Cs[warp * 16 + frag_col(ni, v)][frag_row(mi)] = sg * acc[mi][ni][v];
-            __syncthreads();
-            store_ctile2(St.Cs, p.A, p.lda, cb, r, lo, hi, ncols);
-        } else if (p.do_w) {
-            __syncthreads();
-        }
-        if (p.do_w) {
-            // rows outside [lo, hi) of the C tile are stale/zero, Vt is zero there
-            warp_mma2<WMI, WNI, false, false>(wacc, &St.Vt[0][0], TS, &St.Cs[0][0], TS, wm0, wn0, GB_M);
-        }
-        __syncthreads();
+        if (p.do_w) issue_ktile<KT>(S.Vr, p.V, p.ldw, rbase + t0 * UB, p.r_hi, K);
+        cp_async_commit();
     }
+    for (int tt = t0; tt < t1; tt++) {
+        const int r = rbase + tt * UB;
+        const int lo = max(r, p.r_lo), hi = min(r + UB, p.r_hi);
+        double acc[8][2];
+#pragma unroll
+        for (int ni = 0; ni < 8; ni++) {
+            const double2 c = load_pair(colp, r + ni * 8 + 2 * lc, lo, hi, colok);
+            acc[ni][0] = sg * c.x;
+            acc[ni][1] = sg * c.y;
+        }
+        cp_async_wait<1>();
+        __syncthreads();
+        if (p.do_right) {
+#pragma unroll 4
+            for (int k0 = 0; k0 < KT; k0 += 4) {
+                const double a = S.Vc[k0 + lc][wcol];
+                double b[8];
+#pragma unroll
+                for (int ni = 0; ni < 8; ni++) b[ni] = S.Ys[k0 + lc][ni * 8 + lr];
+#pragma unroll
+                for (int ni = 0; ni < 8; ni++) dmma_8x8x4(acc[ni][0], acc[ni][1], a, b[ni]);
+            }
+#pragma unroll
+            for (int ni = 0; ni < 8; ni++) {
+                acc[ni][0] *= sg;
+                acc[ni][1] *= sg;
+                store_pair(colp, r + ni * 8 + 2 * lc, lo, hi, colok, acc[ni][0], acc[ni][1]);
+            }
+        }
+        __syncthreads();  // every warp is done with Ys(tt)
+        if (p.do_right && tt + 1 < t1) issue_ktile<KT>(S.Ys, p.Y, p.ldw, r + UB, p.r_hi, K);
+        cp_async_commit();
+        if (p.do_w) {
+            cp_async_wait<1>();
+            __syncthreads();
+            // only rows in [wr_lo, wr_hi) take part in W
+            const int wlo = max(lo, p.wr_lo), whi = min(hi, p.wr_hi);
+#pragma unroll
+            for (int ni = 0; ni < 8; ni++) {
+                const int row = r + ni * 8 + 2 * lc;
+                if (row < wlo || row >= whi) acc[ni][0] = 0.0;
+                if (row + 1 < wlo || row + 1 >= whi) acc[ni][1] = 0.0;
+            }
+            // W^T(cols, j) += C_new^T(cols, rows) V(rows, j); the A fragment (col lr, row
+            // ks*4 + lc) sits in lane lr*4 + 2h + lc/2, element lc & 1 (ks = 2 ni + h)
+#pragma unroll
+            for (int ks = 0; ks < 16; ks++) {
+                const int ni = ks >> 1, h = ks & 1;
+                const int src = lr * 4 + 2 * h + (lc >> 1);
+                const double x0 = __shfl_sync(0xffffffffu, acc[ni][0], src);
+                const double x1 = __shfl_sync(0xffffffffu, acc[ni][1], src);
+                const double a = (lc & 1) ? x1 : x0;
+#pragma unroll
+                for (int nj = 0; nj < NJ; nj++) {
+                    const double b = S.Vr[nj * 8 + lr][ks * 4 + lc];
+                    dmma_8x8x4(wacc[nj][0], wacc[nj][1], a, b);
+                }
+            }
+            __syncthreads();  // every warp is done with Vr(tt)
+            if (tt + 1 < t1) issue_ktile<KT>(S.Vr, p.V, p.ldw, r + UB, p.r_hi, K);
+        }
+        cp_async_commit();
+    }
+    cp_async_wait<0>();
     if (p.do_w) {
-        // row splits of a strip accumulate into one W (fp64 RED at L2; W zeroed by the host)
-        double *Wp = p.Wpart;
+        // deterministic partial of this row split: Wpart[split][col][j]
+        double *Wp = p.Wpart + (int64_t)blockIdx.y * p.wsplit_stride;
+        if (colok)
 #pragma unroll
-        for (int mi = 0; mi < WMI; mi++)
-#pragma unroll
-            for (int ni = 0; ni < WNI; ni++)
+            for (int nj = 0; nj < NJ; nj++)
 #pragma unroll
                 for (int v = 0; v < 2; v++) {
-                    int jj = wm0 + frag_row(mi);
-                    int cc = wn0 + frag_col(ni, v);
-                    if (jj < K && cc < ncols) {
-                        double *dst = Wp + (int64_t)(cb + cc) * FT_NBMAX + jj;
-                        if (gridDim.y == 1) *dst = wacc[mi][ni][v];
-                        else atomicAdd(dst, wacc[mi][ni][v]);
-                    }
+                    const int jj = nj * 8 + 2 * lc + v;
+                    if (jj < K) Wp[(int64_t)(cb + wcol) * FT_NBMAX + jj] = wacc[nj][v];
                 }
     }
 }
@@ -194,20 +194,21 @@ __global__ void __launch_bounds__(GT) k_gemm_right(GemmRightParams p) {
 template <int KT>
 static cudaError_t launch_right_kt(const GemmRightParams &p, cudaStream_t s) {
     static bool attr = false;
-    size_t smem = sizeof(RightSmemT<KT>);
+    const size_t smem = sizeof(RightSmemT<KT>);
     if (!attr) {
         cudaError_t e = cudaFuncSetAttribute(k_gemm_right<KT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return e;
         attr = true;
     }
-    int nstrip = (p.c_hi - p.c_lo + GB_N - 1) / GB_N;
-    int ny = p.nsplit > 0 ? p.nsplit : 1;
+    const int nstrip = (p.c_hi - p.c_lo + UB - 1) / UB;
+    const int ny = p.nsplit > 0 ? p.nsplit : 1;
     g_ft_launches++;
-    k_gemm_right<KT><<<dim3(nstrip, ny), GT, smem, s>>>(p);
+    k_gemm_right<KT><<<dim3(nstrip, ny), UT, smem, s>>>(p);
     return cudaGetLastError();
 }
 cudaError_t ft_launch_gemm_right(const GemmRightParams &p, cudaStream_t s) {
     if (p.r_hi <= p.r_lo || p.c_hi <= p.c_lo || p.K <= 0) return cudaSuccess;
+    if (p.do_w && p.nsplit > FT_WSPLIT_MAX) return cudaErrorInvalidValue;
     const bool aligned = (p.lda % 2 == 0) && ((((uintptr_t)p.A) & 15) == 0) && (p.ldw % 2 == 0) &&
                          ((((uintptr_t)p.V) & 15) == 0) && (!p.do_right || ((((uintptr_t)p.Y) & 15) == 0));
     if (!aligned) return cudaErrorInvalidValue;  // the library only passes 16-byte aligned operands
@@ -216,133 +217,145 @@ cudaError_t ft_launch_gemm_right(const GemmRightParams &p, cudaStream_t s) {
 
 // ---------------------------------------------------------------------------
 // Left update: A(rows, cols) += sign * V(rows,:) (op(T) W(:, cols))
+// warp (wc, wr) owns columns wc*16 .. +16 and rows wr*32 .. +32 of a 64 x 64 tile
 // ---------------------------------------------------------------------------
 template <int KT>
 struct LeftSmemT {
-    double Wp[GB_N][KT + 4];  // op(T) W as [col][j]: B operand (n-major)
-    struct {
-        double Cs[GB_N][TS];
-        double Vt[KT][TS];
-    } st[2];
+    double Wc[KT][SK];     // W' = op(T) W as [k][col]  (A operand, W'^T)
+    double Vr[2][KT][SK];  // V(rows, k) as [k][row]    (B operand), double-buffered
 };
 
-// W'(col, a) = sum_b op(T)(a, b) W(b, col), T upper triangular; W, W' stored [col][64]
-__global__ void k_wprep(const double *__restrict__ W, const double *__restrict__ T, double *__restrict__ Wt,
-                        int c_lo, int c_hi, int K, int transT, const FtCtl *ctl) {
+// W'(col, a) = sum_b op(T)(a, b) W(b, col), W = sum over the row-split partials (fixed
+// order); T upper triangular; W partials [split][col][64], W' [col][64]
+__global__ void k_wprep(const double *__restrict__ Wpart, int64_t wstride, int nsplit,
+                        const double *__restrict__ T, double *__restrict__ Wt, int c_lo, int c_hi, int K,
+                        int transT, const FtCtl *ctl) {
     if (ctl && ctl->halt) return;
     __shared__ double Ts[FT_NBMAX][FT_NBMAX + 1];
+    __shared__ double Ws[UT / FT_NBMAX][FT_NBMAX];
     for (int i = threadIdx.x; i < K * K; i += blockDim.x) {
         int a = i % K, b = i / K;
         Ts[a][b] = T[a + b * FT_NBMAX];
     }
+    const int a = threadIdx.x % FT_NBMAX, cl = threadIdx.x / FT_NBMAX;
+    const int col = c_lo + blockIdx.x * (blockDim.x / FT_NBMAX) + cl;
+    double w = 0.0;
+    if (col < c_hi && a < K)
+        for (int sp = 0; sp < nsplit; sp++) w += Wpart[(int64_t)sp * wstride + (int64_t)col * FT_NBMAX + a];
+    Ws[cl][a] = w;
     __syncthreads();
-    const int a = threadIdx.x % FT_NBMAX;
-    const int col = c_lo + blockIdx.x * (blockDim.x / FT_NBMAX) + threadIdx.x / FT_NBMAX;
     if (col >= c_hi || a >= K) return;
-    const double *w = W + (int64_t)col * FT_NBMAX;
     double s0 = 0.0, s1 = 0.0;
     if (transT) {
         int b = 0;
         for (; b + 1 <= a; b += 2) {
-            s0 += Ts[b][a] * w[b];
-            s1 += Ts[b + 1][a] * w[b + 1];
+            s0 += Ts[b][a] * Ws[cl][b];
+            s1 += Ts[b + 1][a] * Ws[cl][b + 1];
         }
-        if (b <= a) s0 += Ts[b][a] * w[b];
+        if (b <= a) s0 += Ts[b][a] * Ws[cl][b];
     } else {
         int b = a;
         for (; b + 1 < K; b += 2) {
-            s0 += Ts[a][b] * w[b];
-            s1 += Ts[a][b + 1] * w[b + 1];
+            s0 += Ts[a][b] * Ws[cl][b];
+            s1 += Ts[a][b + 1] * Ws[cl][b + 1];
         }
-        if (b < K) s0 += Ts[a][b] * w[b];
+        if (b < K) s0 += Ts[a][b] * Ws[cl][b];
     }
     Wt[(int64_t)col * FT_NBMAX + a] = s0 + s1;
 }
 
 template <int KT>
-__global__ void __launch_bounds__(GT) k_gemm_left(GemmLeftParams p) {
+__global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
     if (p.ctl && p.ctl->halt) return;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     LeftSmemT<KT> &S = *reinterpret_cast<LeftSmemT<KT> *>(smem_raw);
-    const int warp = threadIdx.x >> 5;
-    const int cb = p.c_lo + blockIdx.x * GB_N;
-    const int ncols = min(GB_N, p.c_hi - cb);
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int lr = lane >> 2, lc = lane & 3;
+    const int wc = warp & 3, wr = warp >> 2;
+    const int cb = p.c_lo + blockIdx.x * UB;
+    const int ncols = min(UB, p.c_hi - cb);
     const int K = p.K;
     const double sg = p.sign;
-    const int rbase = (p.r_lo / GB_M) * GB_M;
-    const int nrt = (p.r_hi - rbase + GB_M - 1) / GB_M;
+    const int rbase = (p.r_lo / UB) * UB;
+    const int nrt = (p.r_hi - rbase + UB - 1) / UB;
     const int t0 = (int)((long long)blockIdx.y * nrt / gridDim.y);
     const int t1 = (int)((long long)(blockIdx.y + 1) * nrt / gridDim.y);
 
-    // W' for this strip: [col][j] rows of 64 doubles in HBM -> [col][KT+4] in smem
-    for (int q = threadIdx.x; q < GB_N * (KT / 2); q += GT) {
-        int cc = q / (KT / 2), j2 = (q % (KT / 2)) * 2;
-        int bytes = cc < ncols ? 16 : 0;
-        const double *src = bytes ? p.Wpart + (int64_t)(cb + cc) * FT_NBMAX + j2 : p.Wpart;
-        cp_async16(&S.Wp[cc][j2], src, bytes);
+    if (t0 < t1) issue_ktile<KT>(S.Vr[0], p.V, p.ldw, rbase + t0 * UB, p.r_hi, K);
+    cp_async_commit();
+    // W'^T for the strip: Wt [col][64] -> Wc[k][col]
+    for (int i = tid; i < KT * UB; i += UT) {
+        const int cc = i / KT, kk = i % KT;
+        S.Wc[kk][cc] = (kk < K && cc < ncols) ? p.Wpart[(int64_t)(cb + cc) * FT_NBMAX + kk] : 0.0;
     }
-    auto issue = [&](int tt, int s) {
-        const int r = rbase + tt * GB_M;
-        const int hi = min(r + GB_M, p.r_hi);
-        issue_ctile(S.st[s].Cs, p.A, p.lda, cb, r, hi, ncols);
-        issue_jtile<KT>(S.st[s].Vt, p.V, p.ldw, r, K);
-        cp_async_commit();
-    };
-    if (t0 < t1) issue(t0, 0);
-    else cp_async_commit();
+    int cols[2];
+    bool colok[2];
+    double *colp[2];
+#pragma unroll
+    for (int mi = 0; mi < 2; mi++) {
+        cols[mi] = wc * 16 + mi * 8 + lr;
+        colok[mi] = cols[mi] < ncols;
+        colp[mi] = p.A + (int64_t)(cb + (colok[mi] ? cols[mi] : 0)) * p.lda;
+    }
     for (int tt = t0; tt < t1; tt++) {
-        const int s = (tt - t0) & 1;
-        const int r = rbase + tt * GB_M;
-        const int lo = max(r, p.r_lo), hi = min(r + GB_M, p.r_hi);
-        if (tt + 1 < t1) {
-            issue(tt + 1, s ^ 1);
-            cp_async_wait<1>();
-        } else {
-            cp_async_wait<0>();
+        const int st = (tt - t0) & 1;
+        const int r = rbase + tt * UB;
+        const int lo = max(r, p.r_lo), hi = min(r + UB, p.r_hi);
+        double acc[2][4][2];
+#pragma unroll
+        for (int mi = 0; mi < 2; mi++)
+#pragma unroll
+            for (int ni = 0; ni < 4; ni++) {
+                const double2 c = load_pair(colp[mi], r + wr * 32 + ni * 8 + 2 * lc, lo, hi, colok[mi]);
+                acc[mi][ni][0] = sg * c.x;
+                acc[mi][ni][1] = sg * c.y;
+            }
+        if (tt + 1 < t1) issue_ktile<KT>(S.Vr[st ^ 1], p.V, p.ldw, r + UB, p.r_hi, K);
+        cp_async_commit();
+        cp_async_wait<1>();
+        __syncthreads();
+#pragma unroll 4
+        for (int k0 = 0; k0 < KT; k0 += 4) {
+            double a[2], b[4];
+#pragma unroll
+            for (int mi = 0; mi < 2; mi++) a[mi] = S.Wc[k0 + lc][wc * 16 + mi * 8 + lr];
+#pragma unroll
+            for (int ni = 0; ni < 4; ni++) b[ni] = S.Vr[st][k0 + lc][wr * 32 + ni * 8 + lr];
+#pragma unroll
+            for (int mi = 0; mi < 2; mi++)
+#pragma unroll
+                for (int ni = 0; ni < 4; ni++) dmma_8x8x4(acc[mi][ni][0], acc[mi][ni][1], a[mi], b[ni]);
         }
-        __syncthreads();
-        auto &St = S.st[s];
-        double acc[4][2][2];
 #pragma unroll
-        for (int mi = 0; mi < 4; mi++)
+        for (int mi = 0; mi < 2; mi++)
 #pragma unroll
-            for (int ni = 0; ni < 2; ni++)
-#pragma unroll
-                for (int v = 0; v < 2; v++) acc[mi][ni][v] = sg * St.Cs[warp * 16 + frag_col(ni, v)][frag_row(mi)];
-        warp_mma2<4, 2, true, false>(acc, &St.Vt[0][0], TS, &S.Wp[0][0], KT + 4, 0, warp * 16, KT);
-#pragma unroll
-        for (int mi = 0; mi < 4; mi++)
-#pragma unroll
-            for (int ni = 0; ni < 2; ni++)
-#pragma unroll
-                for (int v = 0; v < 2; v++) St.Cs[warp * 16 + frag_col(ni, v)][frag_row(mi)] = sg * acc[mi][ni][v];
-        __syncthreads();
-        store_ctile2(St.Cs, p.A, p.lda, cb, r, lo, hi, ncols);
-        __syncthreads();
+            for (int ni = 0; ni < 4; ni++)
+                store_pair(colp[mi], r + wr * 32 + ni * 8 + 2 * lc, lo, hi, colok[mi], sg * acc[mi][ni][0],
+                           sg * acc[mi][ni][1]);
+        __syncthreads();  // Vr[st] is refilled two tiles later
     }
+    cp_async_wait<0>();
 }
 
 template <int KT>
 static cudaError_t launch_left_kt(const GemmLeftParams &p, cudaStream_t s) {
     static bool attr = false;
-    size_t smem = sizeof(LeftSmemT<KT>);
+    const size_t smem = sizeof(LeftSmemT<KT>);
     if (!attr) {
         cudaError_t e = cudaFuncSetAttribute(k_gemm_left<KT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return e;
         attr = true;
     }
-    int nstrip = (p.c_hi - p.c_lo + GB_N - 1) / GB_N;
-    int nrt = (p.r_hi - (p.r_lo / GB_M) * GB_M + GB_M - 1) / GB_M;
-    int ny = (2 * 148 + nstrip - 1) / nstrip;
-    if (ny > nrt / 2) ny = nrt / 2;
-    if (ny < 1) ny = 1;
+    const int nstrip = (p.c_hi - p.c_lo + UB - 1) / UB;
+    int nsm = 148;
+    const int ny = ft_gemm_splits(p.r_lo, p.r_hi, p.c_lo, p.c_hi, nsm);
     g_ft_launches += 2;
-    const int per = GT / FT_NBMAX;  // columns per k_wprep block
-    k_wprep<<<(p.c_hi - p.c_lo + per - 1) / per, GT, 0, s>>>(p.Wpart, p.T, p.Wt, p.c_lo, p.c_hi, p.K, p.transT,
-                                                              p.ctl);
+    const int per = UT / FT_NBMAX;  // columns per k_wprep block
+    k_wprep<<<(p.c_hi - p.c_lo + per - 1) / per, UT, 0, s>>>(p.Wpart, p.wsplit_stride, p.nsplit > 0 ? p.nsplit : 1,
+                                                              p.T, p.Wt, p.c_lo, p.c_hi, p.K, p.transT, p.ctl);
     GemmLeftParams q = p;
     q.Wpart = p.Wt;  // the main kernel reads W' = op(T) W
-    k_gemm_left<KT><<<dim3(nstrip, ny), GT, smem, s>>>(q);
+    k_gemm_left<KT><<<dim3(nstrip, ny), UT, smem, s>>>(q);
     return cudaGetLastError();
 }
 cudaError_t ft_launch_gemm_left(const GemmLeftParams &p, cudaStream_t s) {
@@ -366,7 +379,7 @@ struct YtopSmem {
     double rsum[YT_M];
 };
 
-__global__ void __launch_bounds__(GT) k_ytop_partial(YtopParams p) {
+__global__ void __launch_bounds__(128) k_ytop_partial(YtopParams p) {
     if (p.ctl->halt) return;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     YtopSmem &S = *reinterpret_cast<YtopSmem *>(smem_raw);
@@ -466,7 +479,7 @@ cudaError_t ft_launch_ytop(const YtopParams &p, cudaStream_t s) {
     }
     int nm = (p.k + 1 + YT_M - 1) / YT_M;
     g_ft_launches += 2;
-    k_ytop_partial<<<dim3(nm, p.nsplit), GT, smem, s>>>(p);
+    k_ytop_partial<<<dim3(nm, p.nsplit), 128, smem, s>>>(p);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
     k_ytop_finalize<<<(p.k + 1 + YF_R - 1) / YF_R, YF_R * 64, 0, s>>>(p);

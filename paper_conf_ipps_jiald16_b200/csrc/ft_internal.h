@@ -60,21 +60,24 @@ struct GemmRightParams {
     int wr_lo, wr_hi;               // rows of V that take part in W = V^T A_new
     int do_right, do_w;
     double sign;                    // -1: A -= Y V^T (update), +1: rollback
-    double *Wpart;                  // [split][col][64]
+    double *Wpart;                  // W partials [split][col][64] (one per row split, no atomics)
     int64_t wsplit_stride;          // doubles per split
-    int nsplit;
+    int nsplit;                     // row splits (grid.y); use ft_gemm_splits()
     const FtCtl *ctl;
 };
 cudaError_t ft_launch_gemm_right(const GemmRightParams &p, cudaStream_t s);
+#define FT_WSPLIT_MAX 16  // max row splits of the right update (deterministic W partials)
+// row splits the right-update launch uses for this block (the left update's k_wprep sums them)
+int ft_gemm_splits(int r_lo, int r_hi, int c_lo, int c_hi, int nsm);
 
 struct GemmLeftParams {
     double *A;
     int64_t lda;
     int64_t ldw;
-    const double *V, *T, *Wpart;  // Wpart: W = V^T A (accumulated, [col][64])
+    const double *V, *T, *Wpart;  // Wpart: the right update's W partials [split][col][64]
     double *Wt;                     // scratch for W' = op(T) W ([col][64])
     int r_lo, r_hi, c_lo, c_hi, K;
-    int nsplit;
+    int nsplit;     // number of W partials to sum (the right update's splits)
     int64_t wsplit_stride;
     int transT;     // 1: A -= V (T^T W) (DLARFB 'L','T'); 0: A -= V (T W)
     double sign;    // -1 update, +1 rollback
