@@ -25,13 +25,26 @@
 #define UT 256  // threads (8 warps)
 #define SK 68   // smem stride of the k-major operand tiles
 
+// Row splits per strip: minimise waves * tiles-per-CTA for 2 resident CTAs per SM (the
+// grid is nstrip x ns CTAs; a ragged last wave idles SMs).
+static int best_splits(int nstrip, int nrt, int nsm, int cap) {
+    const int slots = 2 * nsm;
+    int best = 1;
+    long long best_cost = -1;
+    for (int ns = 1; ns <= cap && ns <= nrt; ns++) {
+        const long long waves = ((long long)nstrip * ns + slots - 1) / slots;
+        const long long cost = waves * ((nrt + ns - 1) / ns);
+        if (best_cost < 0 || cost < best_cost) {
+            best_cost = cost;
+            best = ns;
+        }
+    }
+    return best;
+}
 int ft_gemm_splits(int r_lo, int r_hi, int c_lo, int c_hi, int nsm) {
     const int nstrip = (c_hi - c_lo + UB - 1) / UB;
     const int nrt = (r_hi - (r_lo / UB) * UB + UB - 1) / UB;
-    int ns = (2 * nsm + nstrip - 1) / (nstrip > 0 ? nstrip : 1);
-    if (ns > nrt) ns = nrt;
-    if (ns > FT_WSPLIT_MAX) ns = FT_WSPLIT_MAX;
-    return ns < 1 ? 1 : ns;
+    return best_splits(nstrip > 0 ? nstrip : 1, nrt > 0 ? nrt : 1, nsm, FT_WSPLIT_MAX);
 }
 
 template <int KT>
@@ -116,10 +129,12 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_right(GemmRightParams p) {
     for (int tt = t0; tt < t1; tt++) {
         const int r = rbase + tt * UB;
         const int lo = max(r, p.r_lo), hi = min(r + UB, p.r_hi);
+        const bool full = lo == r && hi == r + UB && ncols == UB;  // interior tile: no masks
         double acc[8][2];
 #pragma unroll
         for (int ni = 0; ni < 8; ni++) {
-            const double2 c = load_pair(colp, r + ni * 8 + 2 * lc, lo, hi, colok);
+            const int row = r + ni * 8 + 2 * lc;
+            const double2 c = full ? *reinterpret_cast<const double2 *>(colp + row) : load_pair(colp, row, lo, hi, colok);
             acc[ni][0] = sg * c.x;
             acc[ni][1] = sg * c.y;
         }
@@ -139,7 +154,9 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_right(GemmRightParams p) {
             for (int ni = 0; ni < 8; ni++) {
                 acc[ni][0] *= sg;
                 acc[ni][1] *= sg;
-                store_pair(colp, r + ni * 8 + 2 * lc, lo, hi, colok, acc[ni][0], acc[ni][1]);
+                const int row = r + ni * 8 + 2 * lc;
+                if (full) *reinterpret_cast<double2 *>(colp + row) = make_double2(acc[ni][0], acc[ni][1]);
+                else store_pair(colp, row, lo, hi, colok, acc[ni][0], acc[ni][1]);
             }
         }
         __syncthreads();  // every warp is done with Ys(tt)
@@ -301,12 +318,15 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
         const int st = (tt - t0) & 1;
         const int r = rbase + tt * UB;
         const int lo = max(r, p.r_lo), hi = min(r + UB, p.r_hi);
+        const bool full = lo == r && hi == r + UB && ncols == UB;  // interior tile: no masks
         double acc[2][4][2];
 #pragma unroll
         for (int mi = 0; mi < 2; mi++)
 #pragma unroll
             for (int ni = 0; ni < 4; ni++) {
-                const double2 c = load_pair(colp[mi], r + wr * 32 + ni * 8 + 2 * lc, lo, hi, colok[mi]);
+                const int row = r + wr * 32 + ni * 8 + 2 * lc;
+                const double2 c = full ? *reinterpret_cast<const double2 *>(colp[mi] + row)
+                                       : load_pair(colp[mi], row, lo, hi, colok[mi]);
                 acc[mi][ni][0] = sg * c.x;
                 acc[mi][ni][1] = sg * c.y;
             }
@@ -329,9 +349,12 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
 #pragma unroll
         for (int mi = 0; mi < 2; mi++)
 #pragma unroll
-            for (int ni = 0; ni < 4; ni++)
-                store_pair(colp[mi], r + wr * 32 + ni * 8 + 2 * lc, lo, hi, colok[mi], sg * acc[mi][ni][0],
-                           sg * acc[mi][ni][1]);
+            for (int ni = 0; ni < 4; ni++) {
+                const int row = r + wr * 32 + ni * 8 + 2 * lc;
+                const double x = sg * acc[mi][ni][0], y = sg * acc[mi][ni][1];
+                if (full) *reinterpret_cast<double2 *>(colp[mi] + row) = make_double2(x, y);
+                else store_pair(colp[mi], row, lo, hi, colok[mi], x, y);
+            }
         __syncthreads();  // Vr[st] is refilled two tiles later
     }
     cp_async_wait<0>();
@@ -347,8 +370,14 @@ static cudaError_t launch_left_kt(const GemmLeftParams &p, cudaStream_t s) {
         attr = true;
     }
     const int nstrip = (p.c_hi - p.c_lo + UB - 1) / UB;
-    int nsm = 148;
-    const int ny = ft_gemm_splits(p.r_lo, p.r_hi, p.c_lo, p.c_hi, nsm);
+    static int nsm = 0;
+    if (!nsm) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    }
+    const int nrt = (p.r_hi - (p.r_lo / UB) * UB + UB - 1) / UB;
+    const int ny = best_splits(nstrip, nrt, nsm, 1 << 20);
     g_ft_launches += 2;
     const int per = UT / FT_NBMAX;  // columns per k_wprep block
     k_wprep<<<(p.c_hi - p.c_lo + per - 1) / per, UT, 0, s>>>(p.Wpart, p.wsplit_stride, p.nsplit > 0 ? p.nsplit : 1,
