@@ -135,7 +135,7 @@ int get_work(int n, Work **out) {
     A(dalloc(&w.Wpart, (size_t)kMaxWsplit * (N1 + 64) * FT_NBMAX, b));
     A(dalloc(&w.Wt, (N1 + 64) * FT_NBMAX, b));
     A(dalloc(&w.bvec, (size_t)ldw, b));
-    A(dalloc(&w.acc, (size_t)FT_ACC_SETS * FT_ACC_STRIDE, b));
+    A(dalloc(&w.acc, (size_t)FT_ACC_SETS * FT_ACC_SET_DOUBLES, b));
     A(dalloc(&w.ckpt, (size_t)ldw * FT_NBMAX, b));
     A(dalloc(&w.ck_r, (size_t)ldw, b));
     A(dalloc(&w.ck_c, N1, b));
@@ -515,7 +515,7 @@ int trailing_nsplit(Call &C, int t) {
 int reset_panel_state(Call &C) {
     Work &w = *C.w;
     CK(cudaMemsetAsync(w.bar, 0, 4 * sizeof(unsigned), C.s));
-    CK(cudaMemsetAsync(w.acc, 0, (size_t)FT_ACC_SETS * FT_ACC_STRIDE * sizeof(double), C.s));
+    CK(cudaMemsetAsync(w.acc, 0, (size_t)FT_ACC_SETS * FT_ACC_SET_DOUBLES * sizeof(double), C.s));
     return 0;
 }
 

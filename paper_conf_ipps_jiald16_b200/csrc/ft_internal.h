@@ -12,6 +12,8 @@
 #endif
 #define FT_ACC_STRIDE (2 * 64 + 8)  // [s1 | vtb | nrm2 sx alpha ...] per reduction set
 #define FT_ACC_SETS 4               // sets indexed by the global column mod 4 (recycled in-kernel)
+#define FT_ACC_PAD 32               // doubles between accumulators: one 256-byte block (own L2 slice) each
+#define FT_ACC_SET_DOUBLES (FT_ACC_STRIDE * FT_ACC_PAD)
 
 // Device-resident control block: halt protocol, fused-verify flags, injector log.
 struct FtCtl {

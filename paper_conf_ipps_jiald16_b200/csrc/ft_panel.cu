@@ -18,20 +18,32 @@
 //  * rows [rbase, rend) are split into 8-row groups, contiguous per CTA; each CTA owns
 //    its rows for the whole panel (b, V, Y rows cached in shared memory), so y needs no
 //    cross-CTA reduction and every small dot is a CTA partial + one fp64 atomic;
-//  * exactly two grid syncs per column, each followed by ONE L2 round trip;
-//  * the GEMV starts right after sync #2 on the UNSCALED b,
+//  * warp 0 is the CONTROL warp: it runs the whole column chain (i)-(iii), (v) warp-
+//    synchronously (lane = row for row dots, lane = output for column dots, no CTA-wide
+//    barriers) and the two grid syncs per column; warps 1..15 only stream A for the
+//    GEMV.  The two roles meet at two named barriers per column (GO, DONE);
+//  * the GEMV runs on the UNSCALED b right after sync #2,
 //        y = A(:, c+1) + scale * A(:, c+2:ihi) b(c+2:ihi),   scale = 1/(alpha - beta),
-//    while warp 0 evaluates DLARFG, so the reflector scalars are off the critical path;
+//    while the control warp evaluates DLARFG, T(:, j) and the stores of V(:, j) and the
+//    reduced column, so only the Y(:, j) step follows the GEMV on the critical path;
 //  * accumulator sets are indexed by the global column (mod 4) and recycled in-kernel,
 //    barrier counters alternate between consecutive panel launches: no memsets per panel.
 #include "ft_common.cuh"
 #include "ft_internal.h"
 
+#include <cstdlib>
+
 #define PT 512        // threads per CTA
 #define NW (PT / 32)  // warps per CTA
+#define NGW (NW - 1)  // GEMV warps (warp 0 is the control warp)
 #define GR 8          // row-group granularity (64 bytes of a column)
 #define VS 65         // shared-memory row stride of the V / Y row caches (doubles)
 #define RMAX PT       // max rows per CTA
+#define BAR_GO 1      // named barrier: b(c+2:ihi) is published, start the GEMV
+#define BAR_DONE 2    // named barrier: GEMV partials are in shared memory
+#ifndef GB
+#define GB 8          // GEMV load batch (double2 of A + b per lane)
+#endif
 
 // accumulator set layout (FT_ACC_STRIDE doubles): [0,64) s1 = V^T b0 | [64,128) V^T x |
 // 128 ||x||^2 | 129 e^T x | 130 alpha
@@ -45,8 +57,12 @@ struct PanelSmem {
     double vrow[FT_NBMAX];              // V(c, 0:j) of the current column
     double w[FT_NBMAX];                 // T^T s1
     double t[FT_NBMAX];                 // V^T v
+    double s1[FT_NBMAX];                // V^T b0 (reduced)
     double scal[8];                     // tau, beta, scale, vchk, alpha
-    double bsm[RMAX];                   // b of the own rows (masked) for the column dots
+    double acol[RMAX];                  // A(row, c) of the own rows
+    double anext[RMAX];                 // A(row, c+1)
+    double b0[RMAX];                    // b0 (rows), then b
+    double bm[RMAX];                    // masked b0 / x for the column dots
     double2 red[PT];                    // GEMV partials  (y pairs)
     double2 rsr[PT];                    // GEMV partials  (row sums, verify pass)
     // followed (dynamic part) by the CTA's rows of V and Y when they fit: [R][VS] each
@@ -56,15 +72,24 @@ size_t ft_panel_smem_bytes() { return sizeof(PanelSmem); }
 
 #define PROBE(slot)                                                                   \
     do {                                                                              \
-        if (p.dbg && blockIdx.x == 0 && tid == 0 && j < 64)                           \
+        if (p.dbg && blockIdx.x == 0 && lane == 0 && j < 64)                          \
             p.dbg[j * 16 + (slot)] = clock64();                                       \
     } while (0)
 
-// sum over the L lanes of an aligned lane group (L a power of two <= 32)
-__device__ __forceinline__ double group_sum(double v, int L) {
-#pragma unroll 1
-    for (int o = L >> 1; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
-    return v;
+__device__ __forceinline__ void named_bar(int id) { asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(PT) : "memory"); }
+
+// grid barrier driven by one warp: lane 0 arrives (release) and polls (acquire); the
+// warp-level barriers order the other lanes' accesses around it
+__device__ __forceinline__ void warp_grid_barrier(unsigned *count, unsigned &epoch, unsigned nblocks) {
+    __syncwarp();
+    if ((threadIdx.x & 31) == 0) {
+        epoch += 1;
+        const unsigned target = epoch * nblocks;
+        red_release_add_u32(count, 1u);
+        while (ld_acquire_u32(count) < target) {
+        }
+    }
+    __syncwarp();
 }
 
 // DLARFG scalars (reading R1), out of line: one copy of the sqrt / division code
@@ -85,13 +110,20 @@ __device__ __noinline__ Refl dlarfg_scalars(double nrm2, double alpha, bool triv
     return r;
 }
 
-// lanes per output for J column dots (L * J <= PT), as log2
-__device__ __forceinline__ int coldot_log2L(int J) { return J <= 16 ? 5 : (J <= 32 ? 4 : (J <= 64 ? 3 : 2)); }
-
-__device__ __forceinline__ int pow2_floor(int x) {
-    int p = 1;
-    while (p * 2 <= x) p *= 2;
-    return p;
+// sum_{jp < J} X[jp * cs] * z[jp] with four independent chains
+__device__ __forceinline__ double dotj(const double *X, int64_t cs, const double *z, int J) {
+    double s0 = 0.0, s1 = 0.0, s2 = 0.0, s3 = 0.0;
+    int jp = 0;
+#pragma unroll 1
+    for (; jp + 3 < J; jp += 4) {
+        s0 += X[jp * cs] * z[jp];
+        s1 += X[(jp + 1) * cs] * z[jp + 1];
+        s2 += X[(jp + 2) * cs] * z[jp + 2];
+        s3 += X[(jp + 3) * cs] * z[jp + 3];
+    }
+#pragma unroll 1
+    for (; jp < J; jp++) s0 += X[jp * cs] * z[jp];
+    return (s0 + s1) + (s2 + s3);
 }
 
 template <bool CACHE>
@@ -111,8 +143,6 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
     double *__restrict__ A = p.A;
     double *__restrict__ V = p.V;
     double *__restrict__ Y = p.Y;
-    unsigned epoch = 0;
-    if (blockIdx.x == 0 && tid == 0) *p.bar_next = 0u;  // the next panel launch's counter
 
     // own rows of V and Y: [rl][jp] in shared memory (write-through to global) when they fit
     double *Vl = CACHE ? reinterpret_cast<double *>(smem_raw + sizeof(PanelSmem)) : V + r0;
@@ -120,136 +150,187 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
     constexpr int64_t XR = CACHE ? VS : 1;  // row stride
     const int64_t XC = CACHE ? 1 : ldw;     // column stride
 
-    // row-dot mapping: tpr lanes per own row
-    const int tpr = min(8, pow2_floor(PT / R));
-    const int tsh = __ffs(tpr) - 1;
-    const int rl = tid >> tsh, lr = tid & (tpr - 1);
-    const int row = r0 + rl;
-    const bool mine = rl < R;
-    const bool datarow = mine && row >= k + 1 && row < ihi;
-    const bool chkrow = mine && p.abft && row == n;
-    const bool valid = datarow || chkrow;
-    const bool leader = mine && lr == 0;
-
-    // GEMV mapping: row pair rp, column lane cl (R2p lanes per column; pow2 when <= 32 so
-    // the lanes of one row pair are shuffle-reducible inside a warp)
+    // GEMV partial layout (shared by both roles): R2p lanes per column, a power of two
+    // when <= 32 so the lanes of one row pair are shuffle-reducible inside a warp
     int R2p = R2;
     if (R2 <= 32) {
         R2p = 1;
         while (R2p < R2) R2p *= 2;
     }
-    const int ncl = PT / R2p;
-    const int rp = tid % R2p, cl = tid / R2p;
-    const bool gemv_on = rp < R2 && cl < ncl;
-    const int npart = R2p <= 32 ? NW : ncl;  // partials per row pair after the warp stage
-    const double2 *__restrict__ A2 = reinterpret_cast<const double2 *>(A + r0);
-    const int64_t ldw2 = ldw >> 1;
-
-    const double c_thr = p.ctl->c_thr;
-    const double tau_abs = c_thr * (double)n * 2.220446049250313e-16 * p.ctl->normF;
+    const int ncl = (NGW * 32) / R2p;
+    const int npart = R2p <= 32 ? NGW : ncl;  // partials per row pair
 
 #pragma unroll 1
     for (int i = tid; i < FT_NBMAX * (FT_NBMAX + 1); i += PT) (&S.Ts[0][0])[i] = 0.0;
-    double acol = (leader && valid) ? A[row + (int64_t)k * ldw] : 0.0;  // A(row, c)
+    for (int rl = tid; rl < R; rl += PT) {
+        const int row = r0 + rl;
+        const bool valid = (row >= k + 1 && row < ihi) || (p.abft && row == n);
+        S.acol[rl] = valid ? A[row + (int64_t)k * ldw] : 0.0;
+    }
     __syncthreads();
 
+    if (wid > 0) {
+        // ======================= GEMV warps =============================================
+        const int gt = tid - 32;
+        const int rp = gt % R2p, cl = gt / R2p;
+        const bool gemv_on = rp < R2 && cl < ncl;
+        const double2 *__restrict__ A2 = reinterpret_cast<const double2 *>(A + r0);
+        const int64_t ldw2 = ldw >> 1;
+        const double *bv = p.bvec;  // b(q) for c+2 <= q < ihi; zero for q >= ihi
+#pragma unroll 1
+        for (int j = 0; j < ib; j++) {
+            const int c = k + j;
+            const bool vfy = (j == 0) && p.verify;
+            const int cend = vfy ? n : ihi;
+            named_bar(BAR_GO);
+            double2 ya = make_double2(0.0, 0.0), rs = make_double2(0.0, 0.0);
+            if (gemv_on && !(p.dbg_mode & 2)) {
+                // b is read with plain (L1-allocating) loads: the control warp's acquire at
+                // sync #2 invalidated this SM's L1 (CCTL.IVALL) before BAR_GO released us
+                int col = c + 2 + cl;
+#pragma unroll 1
+                for (; col + (GB - 1) * ncl < cend; col += GB * ncl) {
+                    double2 a[GB];
+                    double v[GB];
+#pragma unroll
+                    for (int u = 0; u < GB; u++) {
+                        const int q = col + u * ncl;
+                        a[u] = A2[(int64_t)q * ldw2 + rp];
+                        v[u] = bv[q];
+                    }
+#pragma unroll
+                    for (int u = 0; u < GB; u++) {
+                        ya.x += a[u].x * v[u];
+                        ya.y += a[u].y * v[u];
+                        rs.x += a[u].x;  // row sums: used by the verify pass only (cheap, memory-bound loop)
+                        rs.y += a[u].y;
+                    }
+                }
+#pragma unroll 1
+                for (; col < cend; col += ncl) {
+                    const double2 a = A2[(int64_t)col * ldw2 + rp];
+                    const double v = bv[col];
+                    ya.x += a.x * v;
+                    ya.y += a.y * v;
+                    rs.x += a.x;
+                    rs.y += a.y;
+                }
+            }
+            if (R2p <= 32) {
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1)
+                    if (o >= R2p) {
+                        ya.x += __shfl_xor_sync(0xffffffffu, ya.x, o);
+                        ya.y += __shfl_xor_sync(0xffffffffu, ya.y, o);
+                        if (vfy) {
+                            rs.x += __shfl_xor_sync(0xffffffffu, rs.x, o);
+                            rs.y += __shfl_xor_sync(0xffffffffu, rs.y, o);
+                        }
+                    }
+                if (lane < R2p) {
+                    S.red[(wid - 1) * R2p + lane] = ya;
+                    if (vfy) S.rsr[(wid - 1) * R2p + lane] = rs;
+                }
+            } else if (cl < ncl) {
+                S.red[cl * R2p + rp] = ya;
+                if (vfy) S.rsr[cl * R2p + rp] = rs;
+            }
+            named_bar(BAR_DONE);
+        }
+        return;
+    }
+
+    // ======================= control warp =================================================
+    unsigned epoch = 0;
+    if (blockIdx.x == 0 && lane == 0) *p.bar_next = 0u;  // the next panel launch's counter
+    const double c_thr = p.ctl->c_thr;
+    const double tau_abs = c_thr * (double)n * 2.220446049250313e-16 * p.ctl->normF;
+    auto is_data = [&](int row) { return row >= k + 1 && row < ihi; };
+    auto is_valid = [&](int row) { return (row >= k + 1 && row < ihi) || (p.abft && row == n); };
+
+#pragma unroll 1
     for (int j = 0; j < ib; j++) {
         const int c = k + j;
-        double *acc = p.acc + (c & 3) * FT_ACC_STRIDE;
-        // A(row, c+1): the first term of y, and the next column's acol (column c+1 is not
-        // modified while column c is processed)
-        const double anext = (leader && valid) ? A[row + (int64_t)(c + 1) * ldw] : 0.0;
+        double *acc = p.acc + (c & 3) * FT_ACC_SET_DOUBLES;  // accumulator i at acc[i * FT_ACC_PAD]
+        // A(row, c+1) of the first two row chunks: issued now, consumed after the GEMV
+        double an0 = 0.0, an1 = 0.0;
+        if (lane < R && is_valid(r0 + lane)) an0 = A[(r0 + lane) + (int64_t)(c + 1) * ldw];
+        if (lane + 32 < R && is_valid(r0 + lane + 32)) an1 = A[(r0 + lane + 32) + (int64_t)(c + 1) * ldw];
         PROBE(0);
-        // ---------------- (i) b0 = A(:,c) - Y V(c,:)^T ------------------------------------
-        double b0 = acol;
+        // ---------------- (i) b0 = A(:,c) - Y V(c,:)^T, s1 = V^T b0 -----------------------
         if (j > 0) {
-            double sacc = 0.0;
-            if (mine)
 #pragma unroll 1
-                for (int jp = lr; jp < j; jp += tpr) sacc += Yl[rl * XR + jp * XC] * S.vrow[jp];
-            b0 = acol - group_sum(sacc, tpr);
-            if (leader) S.bsm[rl] = datarow ? b0 : 0.0;
-            __syncthreads();
-            // s1 = V^T b0 over the data rows: one partial per CTA and output
-            {
-                const int lg = coldot_log2L(j), L = 1 << lg;
-                const int o = tid >> lg, lc = tid & (L - 1);
-                double s = 0.0;
-                if (o < j)
+            for (int rl = lane; rl < R; rl += 32) {
+                const double b0 = S.acol[rl] - dotj(Yl + rl * XR, XC, S.vrow, j);
+                S.b0[rl] = b0;
+                S.bm[rl] = is_data(r0 + rl) ? b0 : 0.0;
+            }
+            __syncwarp();
 #pragma unroll 1
-                    for (int t2 = lc; t2 < R; t2 += L) s += Vl[t2 * XR + o * XC] * S.bsm[t2];
-                s = group_sum(s, L);
-                if (o < j && lc == 0 && !(p.dbg_mode & 4)) atomicAdd(acc + o, s);
+            for (int o = lane; o < j; o += 32) {
+                const double s = dotj(Vl + o * XC, XR, S.bm, R);
+                if (!(p.dbg_mode & 4)) atomicAdd(acc + o * FT_ACC_PAD, s);
             }
             PROBE(1);
-            if (!(p.dbg_mode & 1)) grid_barrier(p.bar, epoch, P);
+            if (!(p.dbg_mode & 1)) warp_grid_barrier(p.bar, epoch, P);
             PROBE(2);
-            // w = T^T s1 (8 lanes per output, s1 read straight from L2)
-            {
-                const int a = tid >> 3, q = tid & 7;
-                double s = 0.0;
-#pragma unroll
-                for (int u = 0; u < FT_NBMAX / 8; u++) {
-                    const int bb = q + 8 * u;
-                    if (a < j && bb <= a) s += S.Ts[bb][a] * ldcg(acc + bb);
-                }
-                s += __shfl_xor_sync(0xffffffffu, s, 1);
-                s += __shfl_xor_sync(0xffffffffu, s, 2);
-                s += __shfl_xor_sync(0xffffffffu, s, 4);
-                if (a < j && q == 0) S.w[a] = s;
-            }
-            __syncthreads();
-            PROBE(3);
-        }
-        // ---------------- (ii) b = b0 - V w --------------------------------------------------
-        double b = b0;
-        if (j > 0) {
-            double sacc = 0.0;
-            if (mine)
+            // w = T^T s1
+            if (lane < j) S.s1[lane] = ldcg(acc + lane * FT_ACC_PAD);
+            if (lane + 32 < j) S.s1[lane + 32] = ldcg(acc + (lane + 32) * FT_ACC_PAD);
+            __syncwarp();
 #pragma unroll 1
-                for (int jp = lr; jp < j; jp += tpr) sacc += Vl[rl * XR + jp * XC] * S.w[jp];
-            b = b0 - group_sum(sacc, tpr);
+            for (int a = lane; a < j; a += 32) S.w[a] = dotj(&S.Ts[0][a], FT_NBMAX + 1, S.s1, a + 1);
+            __syncwarp();
+            // ---------------- (ii) b = b0 - V w ---------------------------------------------
+#pragma unroll 1
+            for (int rl = lane; rl < R; rl += 32) S.b0[rl] -= dotj(Vl + rl * XR, XC, S.w, j);
+        } else {
+#pragma unroll 1
+            for (int rl = lane; rl < R; rl += 32) S.b0[rl] = S.acol[rl];
         }
-        const bool xrow = datarow && row >= c + 2;
-        if (leader) {
-            S.bsm[rl] = xrow ? b : 0.0;
+        PROBE(3);
+        // publish x = b(c+2:ihi) for the GEMV, alpha = b(c+1); column dots of x
+#pragma unroll 1
+        for (int rl = lane; rl < R; rl += 32) {
+            const int row = r0 + rl;
+            const double b = S.b0[rl];
+            const bool xrow = is_data(row) && row >= c + 2;
+            S.bm[rl] = xrow ? b : 0.0;
             if (xrow) p.bvec[row] = b;
-            if (datarow && row == c + 1) acc[ACC_ALPHA] = b;  // alpha: a single writer
+            if (row == c + 1) acc[ACC_ALPHA * FT_ACC_PAD] = b;  // alpha: a single writer
         }
-        __syncthreads();
-        // V^T x (jp < j), ||x||^2 (jp = j), e^T x (jp = j + 1) over the own x rows
-        {
-            const int J = j + 2;
-            const int lg = coldot_log2L(J), L = 1 << lg;
-            const int o = tid >> lg, lc = tid & (L - 1);
-            double s = 0.0;
-            if (o < J)
+        __syncwarp();
 #pragma unroll 1
-                for (int t2 = lc; t2 < R; t2 += L) {
-                    const double bt = S.bsm[t2];
-                    s += (o < j ? Vl[t2 * XR + o * XC] : (o == j ? bt : 1.0)) * bt;
-                }
-            s = group_sum(s, L);
-            if (o < J && lc == 0 && !(p.dbg_mode & 4))
-                atomicAdd(acc + (o < j ? ACC_VTB + o : (o == j ? ACC_NRM : ACC_SX)), s);
+        for (int o = lane; o < j + 2; o += 32) {
+            double s;
+            if (o < j) s = dotj(Vl + o * XC, XR, S.bm, R);
+            else if (o == j) s = dotj(S.bm, 1, S.bm, R);
+            else {
+                s = 0.0;
+                for (int rl = 0; rl < R; rl++) s += S.bm[rl];
+            }
+            if (!(p.dbg_mode & 4)) atomicAdd(acc + (o < j ? ACC_VTB + o : (o == j ? ACC_NRM : ACC_SX)) * FT_ACC_PAD, s);
         }
         PROBE(4);
-        if (!(p.dbg_mode & 1)) grid_barrier(p.bar, epoch, P);
+        if (!(p.dbg_mode & 1)) warp_grid_barrier(p.bar, epoch, P);
         PROBE(5);
-        // ---------------- (iii) DLARFG (reading R1) in warp 0, concurrent with the GEMV -------
-        if (wid == 0) {
-            const double nrm2 = ldcg(acc + ACC_NRM), sx = ldcg(acc + ACC_SX), alpha = ldcg(acc + ACC_ALPHA);
+        named_bar(BAR_GO);  // the GEMV warps start on the unscaled b
+        // ---------------- (iii) DLARFG (reading R1), concurrent with the GEMV ---------------
+        {
+            const double nrm2 = ldcg(acc + ACC_NRM * FT_ACC_PAD), sx = ldcg(acc + ACC_SX * FT_ACC_PAD),
+                         alpha = ldcg(acc + ACC_ALPHA * FT_ACC_PAD);
             double vn0 = 0.0, vt0 = 0.0, vn1 = 0.0, vt1 = 0.0;
             if (lane < j) {
                 vn0 = ldcg(V + (c + 1) + (int64_t)lane * ldw);
-                vt0 = ldcg(acc + ACC_VTB + lane);
+                vt0 = ldcg(acc + (ACC_VTB + lane) * FT_ACC_PAD);
             }
             if (lane + 32 < j) {
                 vn1 = ldcg(V + (c + 1) + (int64_t)(lane + 32) * ldw);
-                vt1 = ldcg(acc + ACC_VTB + lane + 32);
+                vt1 = ldcg(acc + (ACC_VTB + lane + 32) * FT_ACC_PAD);
             }
             const Refl rf = dlarfg_scalars(nrm2, alpha, c + 2 >= ihi);
             const double tau = rf.tau, beta = rf.beta, scale = rf.scale;
+            const double vchk = 1.0 + scale * sx;  // V_chk(j) = e^T v
             // t = V^T v = V(c+1,:)^T + scale * V^T x; V(c+1, :) is also the next column's vrow
             if (lane < j) {
                 S.t[lane] = vn0 + scale * vt0;
@@ -262,101 +343,25 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
             if (lane == 0) {
                 S.vrow[j] = 1.0;
                 S.scal[0] = tau;
-                S.scal[1] = beta;
                 S.scal[2] = scale;
-                S.scal[3] = 1.0 + scale * sx;  // V_chk(j) = e^T v
-                S.scal[4] = alpha;
             }
-        }
-        PROBE(6);
-        // ---------------- (iv) the trailing GEMV on the unscaled b ---------------------------
-        const bool vfy = (j == 0) && p.verify;
-        const int cend = vfy ? n : ihi;
-        double2 ya = make_double2(0.0, 0.0), rs = make_double2(0.0, 0.0);
-        if (gemv_on && !(p.dbg_mode & 2)) {
-            const double *bv = p.bvec;  // b(q) for c+2 <= q < ihi; zero for q >= ihi
-            int col = c + 2 + cl;
+            __syncwarp();
+            // T(a, j) = -tau * sum_{b=a}^{j-1} T(a, b) t(b), T(j, j) = tau
 #pragma unroll 1
-            for (; col + 7 * ncl < cend; col += 8 * ncl) {
-                double2 a[8];
-                double v[8];
-#pragma unroll
-                for (int u = 0; u < 8; u++) {
-                    const int q = col + u * ncl;
-                    a[u] = A2[(int64_t)q * ldw2 + rp];
-                    v[u] = ldcg(bv + q);
-                }
-#pragma unroll
-                for (int u = 0; u < 8; u++) {
-                    ya.x += a[u].x * v[u];
-                    ya.y += a[u].y * v[u];
-                    rs.x += a[u].x;  // row sums: used by the verify pass only (cheap, HBM-bound loop)
-                    rs.y += a[u].y;
-                }
-            }
+            for (int a = lane; a < j; a += 32) S.Ts[a][j] = -tau * dotj(&S.Ts[a][a], 1, S.t + a, j - a);
+            if (lane == 0) S.Ts[j][j] = tau;
+            // V(:, j) and the reduced column c of the own rows
 #pragma unroll 1
-            for (; col < cend; col += ncl) {
-                const double2 a = A2[(int64_t)col * ldw2 + rp];
-                const double v = ldcg(bv + col);
-                ya.x += a.x * v;
-                ya.y += a.y * v;
-                rs.x += a.x;
-                rs.y += a.y;
-            }
-        }
-        PROBE(7);
-        // partials: shuffle over the lanes of a row pair inside the warp, then shared memory
-        if (R2p <= 32) {
-#pragma unroll
-            for (int o = 1; o < 32; o <<= 1)
-                if (o >= R2p) {
-                    ya.x += __shfl_xor_sync(0xffffffffu, ya.x, o);
-                    ya.y += __shfl_xor_sync(0xffffffffu, ya.y, o);
-                    if (vfy) {
-                        rs.x += __shfl_xor_sync(0xffffffffu, rs.x, o);
-                        rs.y += __shfl_xor_sync(0xffffffffu, rs.y, o);
-                    }
-                }
-            if (lane < R2p) {
-                S.red[wid * R2p + lane] = ya;
-                if (vfy) S.rsr[wid * R2p + lane] = rs;
-            }
-        } else if (cl < ncl) {
-            S.red[cl * R2p + rp] = ya;
-            if (vfy) S.rsr[cl * R2p + rp] = rs;
-        }
-        // (zero the accumulator set of column c+2 (= that of column c-2): every CTA has
-        // finished reading it, and column c+2 starts adding into it after two more syncs)
-        if (blockIdx.x == 0)
-            for (int i = tid; i < FT_ACC_STRIDE; i += PT) p.acc[((c + 2) & 3) * FT_ACC_STRIDE + i] = 0.0;
-        __syncthreads();
-        PROBE(8);
-        // ---------------- (v) Y(:, j), T(:, j), V(:, j), reduced column c -------------------
-        const double tau = S.scal[0], scale = S.scal[2];
-        {
-            double sacc = 0.0;
-            if (mine)
-#pragma unroll 1
-                for (int jp = lr; jp < j; jp += tpr) sacc += Yl[rl * XR + jp * XC] * S.t[jp];
-            sacc = group_sum(sacc, tpr);
-            if (leader) {
-                if (valid) {
-                    double yb = 0.0;
-                    const int pr = rl >> 1;
-#pragma unroll 1
-                    for (int q = 0; q < npart; q++) {
-                        const double2 u = S.red[q * R2p + pr];
-                        yb += (rl & 1) ? u.y : u.x;
-                    }
-                    const double yy = tau * (anext + scale * yb - sacc);
-                    Y[row + (int64_t)j * ldw] = yy;
-                    if (CACHE) Yl[rl * XR + j * XC] = yy;
-                    const double beta = S.scal[1], vchk = S.scal[3], alpha = S.scal[4];
+            for (int rl = lane; rl < R; rl += 32) {
+                const int row = r0 + rl;
+                const double b = S.b0[rl];
+                if (row == n && p.abft) {
+                    V[row + (int64_t)j * ldw] = vchk;
+                    if (CACHE) Vl[rl * XR + j * XC] = vchk;
+                    A[row + (int64_t)c * ldw] = (tau != 0.0) ? b - vchk * (alpha - beta) : b;  // left term (R7)
+                } else if (is_data(row)) {
                     double vv, av;
-                    if (chkrow) {
-                        vv = vchk;
-                        av = (tau != 0.0) ? b - vchk * (alpha - beta) : b;  // left term of reflector j (R7)
-                    } else if (row <= c) {
+                    if (row <= c) {
                         vv = 0.0;
                         av = b;
                     } else if (row == c + 1) {
@@ -369,15 +374,62 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
                     V[row + (int64_t)j * ldw] = vv;
                     if (CACHE) Vl[rl * XR + j * XC] = vv;
                     A[row + (int64_t)c * ldw] = av;
-                    if (vfy && datarow) {
+                } else if (CACHE) {
+                    Vl[rl * XR + j * XC] = 0.0;  // rows outside the panel take no part in the dots
+                }
+            }
+            if (blockIdx.x == 0 && lane == 0) {
+                p.tau[c] = tau;
+                if (p.abft) {
+                    p.Qc[c] = vchk - 1.0;   // Q column checksum
+                    p.Qc[n] += vchk - 1.0;  // corner of the Q checksums
+                }
+            }
+            // recycle the accumulator set of column c+2 (= that of column c-2): every CTA has
+            // finished reading it, and column c+2 adds into it only after two more syncs
+            if (blockIdx.x == 0)
+                for (int i = lane; i < FT_ACC_STRIDE; i += 32) p.acc[((c + 2) & 3) * FT_ACC_SET_DOUBLES + i * FT_ACC_PAD] = 0.0;
+            if (lane < R) S.anext[lane] = an0;
+            if (lane + 32 < R) S.anext[lane + 32] = an1;
+            for (int rl = lane + 64; rl < R; rl += 32)
+                S.anext[rl] = is_valid(r0 + rl) ? A[(r0 + rl) + (int64_t)(c + 1) * ldw] : 0.0;
+        }
+        PROBE(6);
+        named_bar(BAR_DONE);  // GEMV partials ready
+        PROBE(7);
+        // ---------------- (v) Y(:, j) = tau (y - Y t) ----------------------------------------
+        {
+            const double tau = S.scal[0], scale = S.scal[2];
+            const bool vfy = (j == 0) && p.verify;
+#pragma unroll 1
+            for (int rl = lane; rl < R; rl += 32) {
+                const int row = r0 + rl;
+                const double an = S.anext[rl];
+                if (is_valid(row)) {
+                    const int pr = rl >> 1;
+                    double y0 = 0.0, y1 = 0.0;
+                    int q = 0;
+#pragma unroll 1
+                    for (; q + 1 < npart; q += 2) {
+                        const double2 u0 = S.red[q * R2p + pr], u1 = S.red[(q + 1) * R2p + pr];
+                        y0 += (rl & 1) ? u0.y : u0.x;
+                        y1 += (rl & 1) ? u1.y : u1.x;
+                    }
+                    if (q < npart) {
+                        const double2 u0 = S.red[q * R2p + pr];
+                        y0 += (rl & 1) ? u0.y : u0.x;
+                    }
+                    const double yy = tau * (an + scale * (y0 + y1) - dotj(Yl + rl * XR, XC, S.t, j));
+                    Y[row + (int64_t)j * ldw] = yy;
+                    if (CACHE) Yl[rl * XR + j * XC] = yy;
+                    if (vfy && is_data(row)) {
                         // D_r(row) = r(row) - sum_{col >= k} L(row, col); columns < k are logical zero
                         double rsum = 0.0;
-#pragma unroll 1
-                        for (int q = 0; q < npart; q++) {
-                            const double2 u = S.rsr[q * R2p + pr];
+                        for (int q2 = 0; q2 < npart; q2++) {
+                            const double2 u = S.rsr[q2 * R2p + pr];
                             rsum += (rl & 1) ? u.y : u.x;
                         }
-                        rsum += b0 + anext;
+                        rsum += S.acol[rl] + an;
                         const double d = A[row + (int64_t)n * ldw] - rsum;
                         if (not_within(d, tau_abs)) {
                             atomicAdd(&p.ctl->nflag, 1);
@@ -386,45 +438,25 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
                             atomicMax(&p.ctl->drift_bits, (unsigned long long)__double_as_longlong(rel));
                         }
                     }
-                } else if (CACHE) {
-                    Vl[rl * XR + j * XC] = 0.0;  // rows outside the panel take no part in the dots
                 }
+                S.acol[rl] = an;
             }
+            __syncwarp();
         }
-        {   // T(a, j) = -tau * sum_{b=a}^{j-1} T(a, b) t(b), 8 lanes per output
-            const int a = tid >> 3, q = tid & 7;
-            double s = 0.0;
-            if (a < j)
-                for (int bb = a + q; bb < j; bb += 8) s += S.Ts[a][bb] * S.t[bb];
-            s += __shfl_xor_sync(0xffffffffu, s, 1);
-            s += __shfl_xor_sync(0xffffffffu, s, 2);
-            s += __shfl_xor_sync(0xffffffffu, s, 4);
-            if (a < j && q == 0) S.Ts[a][j] = -tau * s;
-            if (tid == 0) S.Ts[j][j] = tau;
-        }
-        if (blockIdx.x == 0 && tid == 0) {
-            p.tau[c] = tau;
-            if (p.abft) {
-                const double vchk = S.scal[3];
-                p.Qc[c] = vchk - 1.0;   // Q column checksum
-                p.Qc[n] += vchk - 1.0;  // corner of the Q checksums
-            }
-        }
-        acol = anext;
-        __syncthreads();
-        PROBE(9);
+        PROBE(8);
     }
     // Q row checksums of the new Householder vectors (Fig. 5): own data rows
-    if (p.abft && leader && datarow) {
-        double s = 0.0;
-#pragma unroll 1
-        for (int jj = 0; jj < ib; jj++)
-            if (row >= k + jj + 2) s += Vl[rl * XR + jj * XC];
-        p.Qr[row] += s;
-    }
+    if (p.abft)
+        for (int rl = lane; rl < R; rl += 32) {
+            const int row = r0 + rl;
+            if (!is_data(row)) continue;
+            double s = 0.0;
+            for (int jj = 0; jj < ib; jj++)
+                if (row >= k + jj + 2) s += Vl[rl * XR + jj * XC];
+            p.Qr[row] += s;
+        }
     if (blockIdx.x == 0)
-#pragma unroll 1
-        for (int i = tid; i < ib * ib; i += PT) {
+        for (int i = lane; i < ib * ib; i += 32) {
             int a = i % ib, bb = i / ib;
             p.T[a + bb * FT_NBMAX] = S.Ts[a][bb];
         }
@@ -441,6 +473,12 @@ cudaError_t ft_launch_panel(const PanelParams &p, int nsm, cudaStream_t s) {
         e = cudaFuncSetAttribute(k_panel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem);
         if (e != cudaSuccess) return e;
     }
+    static int ctas = -1;
+    if (ctas < 0) {
+        const char *e = getenv("FT_PANEL_CTAS");  // experiment knob: cap on the panel grid
+        ctas = e ? atoi(e) : 0;
+    }
+    if (ctas > 0 && ctas < nsm) nsm = ctas;
     int grid = nsm < p.ngroups ? nsm : p.ngroups;
     if (grid < 1) grid = 1;
     // rows per CTA (max over CTAs) and whether their V/Y rows fit next to the fixed part

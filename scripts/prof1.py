@@ -63,9 +63,9 @@ def main():
               f"{10 / 3 * n ** 3 / ms / 1e6:.1f} Gflop/s", flush=True)
     if dbg is not None:
         d = dbg.cpu().numpy()
-        names = {0: "start", 1: "s1_dots", 2: "sync1", 3: "w", 4: "x_dots", 5: "sync2", 6: "dlarfg",
-                 7: "gemv", 8: "red_sync", 9: "y_v_t"}
-        order = [0, 1, 2, 3, 4, 5, 6, 7, 8, 9]
+        names = {0: "start", 1: "s1_dots", 2: "sync1", 3: "w_b", 4: "x_dots", 5: "sync2", 6: "cw_dlarfg_T_V",
+                 7: "gemv_wait", 8: "y_step"}
+        order = [0, 1, 2, 3, 4, 5, 6, 7, 8]
         tot = {}
         ncol = 0
         for j in range(64):
