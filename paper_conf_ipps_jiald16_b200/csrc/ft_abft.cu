@@ -36,28 +36,63 @@ cudaError_t ft_copy_out(const double *Aw, int64_t ldw, double *A, int lda, int n
 }
 
 // ---------------------------------------------------------------------------
-// encode: row sums (thread per row), column sums (warp per column), ||A||_F^2
+// encode: row sums as 2-D tiled partial sums (thread per row, 64-column chunks, fixed-order
+// finish: deterministic), column sums (warp per column), ||A||_F^2
 // ---------------------------------------------------------------------------
-__global__ void k_encode_rows(double *Aw, int64_t ldw, int n, double *sq_part) {
-    int i = blockIdx.x * blockDim.x + threadIdx.x;
+#define LS_RB 256  // rows per block of the row-sum passes
+static int ls_chunks(int n) {  // column chunks (<= 64): partials fit the 64 x ldw scratch
+    int cb = (n + 63) / 64;
+    if (cb < 32) cb = 32;
+    return (n + cb - 1) / cb;
+}
+// rowpart[chunk][i] = sum_{j in chunk} w(i,j) A(i,j), w = 1 (mode -1: encode), the logical-H
+// mask (mode 0) or the Householder-vector mask (mode 1); sq_part[block] = sum A^2 (encode)
+__device__ __forceinline__ bool in_v(int i, int j, int ilo, int ihi, int cdone) {
+    return j >= ilo - 1 && j < cdone && j <= ihi - 2 && i >= j + 2 && i < ihi;
+}
+__global__ void __launch_bounds__(LS_RB) k_rowsum_part(const double *__restrict__ Aw, int64_t ldw, int n, int nchunk,
+                                                       int mode, int ilo, int ihi, int cdone, double *rowpart,
+                                                       double *sq_part) {
+    const int i = blockIdx.x * LS_RB + threadIdx.x;
+    const int cw = (n + nchunk - 1) / nchunk;
+    const int j0 = blockIdx.y * cw, j1 = min(n, j0 + cw);
     double s = 0.0, q = 0.0;
     if (i < n) {
-        for (int j = 0; j < n; j++) {
-            double a = Aw[i + (int64_t)j * ldw];
-            s += a;
-            q += a * a;
+        const double *a = Aw + i;
+        if (mode < 0) {
+            for (int j = j0; j < j1; j++) {
+                const double x = a[(int64_t)j * ldw];
+                s += x;
+                q += x * x;
+            }
+        } else {
+            for (int j = j0; j < j1; j++) {
+                const bool v = in_v(i, j, ilo, ihi, cdone);
+                if (mode == 0 ? !v : v) s += a[(int64_t)j * ldw];
+            }
         }
-        Aw[i + (int64_t)n * ldw] = s;  // r(i) in column n
+        rowpart[(int64_t)blockIdx.y * n + i] = s;
     }
-    q = warp_sum(q);
-    __shared__ double ws[32];
-    if ((threadIdx.x & 31) == 0) ws[threadIdx.x >> 5] = q;
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        double t = 0.0;
-        for (int w = 0; w < (int)(blockDim.x >> 5); w++) t += ws[w];
-        sq_part[blockIdx.x] = t;
+    if (sq_part) {
+        q = warp_sum(q);
+        __shared__ double ws[LS_RB / 32];
+        if ((threadIdx.x & 31) == 0) ws[threadIdx.x >> 5] = q;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            double t = 0.0;
+            for (int w = 0; w < LS_RB / 32; w++) t += ws[w];
+            sq_part[blockIdx.y * gridDim.x + blockIdx.x] = t;
+        }
     }
+}
+// out[i * oinc] = (base ? base[i * binc] : 0) - / + sum_chunk rowpart[chunk][i]
+__global__ void k_rowsum_finish(const double *rowpart, int n, int nchunk, const double *base, int64_t binc,
+                                double *out, int64_t oinc) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    double s = 0.0;
+    for (int c = 0; c < nchunk; c++) s += rowpart[(int64_t)c * n + i];
+    out[(int64_t)i * oinc] = base ? base[(int64_t)i * binc] - s : s;
 }
 __global__ void k_encode_cols(double *Aw, int64_t ldw, int n) {
     int j = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
@@ -98,13 +133,15 @@ cudaError_t ft_frozen_init(const double *Aw, int64_t ldw, int n, int ncols, doub
     k_frozen_init<<<(n + 255) / 256, 256, 0, s>>>(Aw, ldw, n, ncols, Fr);
     return cudaGetLastError();
 }
-cudaError_t ft_encode(double *Aw, int64_t ldw, int n, FtCtl *ctl, double *scratch, cudaStream_t s) {
+cudaError_t ft_encode(double *Aw, int64_t ldw, int n, FtCtl *ctl, double *scratch, double *linepart,
+                      cudaStream_t s) {
     if (n <= 0) return cudaSuccess;
-    int nb = (n + 255) / 256;
-    g_ft_launches += 3;
-    k_encode_rows<<<nb, 256, 0, s>>>(Aw, ldw, n, scratch);
+    const int nrb = (n + LS_RB - 1) / LS_RB, nch = ls_chunks(n);
+    g_ft_launches += 4;
+    k_rowsum_part<<<dim3(nrb, nch), LS_RB, 0, s>>>(Aw, ldw, n, nch, -1, 0, 0, 0, linepart, scratch);
+    k_rowsum_finish<<<(n + 255) / 256, 256, 0, s>>>(linepart, n, nch, nullptr, 0, Aw + (int64_t)n * ldw, 1);
     k_encode_cols<<<(n + 7) / 8, 256, 0, s>>>(Aw, ldw, n);
-    k_encode_finish<<<1, 1024, 0, s>>>(Aw, ldw, n, scratch, nb, ctl);
+    k_encode_finish<<<1, 1024, 0, s>>>(Aw, ldw, n, scratch, nrb * nch, ctl);
     return cudaGetLastError();
 }
 
@@ -318,20 +355,6 @@ cudaError_t ft_inject(double *addr, int fidx, int bit, FtCtl *ctl, cudaStream_t 
 // Fr (mode 0, optional) is ignored here: the full verify recomputes everything.
 // sums[0] = sum r, sums[1] = sum c.
 // ---------------------------------------------------------------------------
-__device__ __forceinline__ bool in_v(int i, int j, int ilo, int ihi, int cdone) {
-    return j >= ilo - 1 && j < cdone && j <= ihi - 2 && i >= j + 2 && i < ihi;
-}
-__global__ void k_fv_rows(const double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdone, int mode,
-                          const double *r, int64_t rinc, double *Dr) {
-    int i = blockIdx.x * blockDim.x + threadIdx.x;
-    if (i >= n) return;
-    double s = 0.0;
-    for (int j = 0; j < n; j++) {
-        bool v = in_v(i, j, ilo, ihi, cdone);
-        if (mode == 0 ? !v : v) s += Aw[i + (int64_t)j * ldw];
-    }
-    Dr[i] = r[(int64_t)i * rinc] - s;
-}
 __global__ void k_fv_cols(const double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdone, int mode,
                           const double *c, int64_t cinc, double *Dc) {
     int j = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
@@ -371,10 +394,12 @@ __global__ void k_fv_sums(int n, const double *r, int64_t rinc, const double *c,
 }
 cudaError_t ft_full_verify(const double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdone, int mode,
                            const double *r, int64_t rinc, const double *c, int64_t cinc, const double *Fr,
-                           double *Dr, double *Dc, double *sums, cudaStream_t s) {
+                           double *Dr, double *Dc, double *sums, double *linepart, cudaStream_t s) {
     if (n <= 0) return cudaSuccess;
-    g_ft_launches += 3;
-    k_fv_rows<<<(n + 127) / 128, 128, 0, s>>>(Aw, ldw, n, ilo, ihi, cdone, mode, r, rinc, Dr);
+    g_ft_launches += 4;
+    const int nrb = (n + LS_RB - 1) / LS_RB, nch = ls_chunks(n);
+    k_rowsum_part<<<dim3(nrb, nch), LS_RB, 0, s>>>(Aw, ldw, n, nch, mode, ilo, ihi, cdone, linepart, nullptr);
+    k_rowsum_finish<<<(n + 255) / 256, 256, 0, s>>>(linepart, n, nch, r, rinc, Dr, 1);
     k_fv_cols<<<(n + 7) / 8, 256, 0, s>>>(Aw, ldw, n, ilo, ihi, cdone, mode, c, cinc, Dc);
     k_fv_sums<<<1, 1024, 0, s>>>(n, r, rinc, c, cinc, sums);
     return cudaGetLastError();

@@ -81,20 +81,23 @@ struct Work {
     double *Aw = nullptr, *V = nullptr, *Y = nullptr, *T = nullptr, *Wpart = nullptr, *bvec = nullptr,
            *acc = nullptr, *ckpt = nullptr, *ck_r = nullptr, *ck_c = nullptr, *ck_q = nullptr, *Fr = nullptr,
            *Qr = nullptr, *Qc = nullptr, *Dr = nullptr, *Dc = nullptr, *sums = nullptr, *ypart = nullptr,
-           *rowpart = nullptr, *scratch = nullptr, *deltas = nullptr, *hA = nullptr, *htau = nullptr;
+           *rowpart = nullptr, *linepart = nullptr, *scratch = nullptr, *deltas = nullptr, *hA = nullptr, *htau = nullptr;
     unsigned *bar = nullptr;
+    int *strip_done = nullptr;
     FtCtl *ctl = nullptr;
     FtFix *fixes = nullptr;
     int nsm = 0;
     size_t bytes = 0;
     void release() {
         double **ps[] = {&Wt, &Aw, &V, &Y, &T, &Wpart, &bvec, &acc, &ckpt, &ck_r, &ck_c, &ck_q, &Fr, &Qr, &Qc, &Dr, &Dc,
-                         &sums, &ypart, &rowpart, &scratch, &deltas, &hA, &htau};
+                         &sums, &ypart, &rowpart, &linepart, &scratch, &deltas, &hA, &htau};
         for (auto p : ps) {
             if (*p) cudaFree(*p);
             *p = nullptr;
         }
         if (bar) cudaFree(bar);
+        if (strip_done) cudaFree(strip_done);
+        strip_done = nullptr;
         if (ctl) cudaFree(ctl);
         if (fixes) cudaFree(fixes);
         bar = nullptr;
@@ -148,9 +151,11 @@ int get_work(int n, Work **out) {
     A(dalloc(&w.sums, 8, b));
     A(dalloc(&w.ypart, (size_t)kYtopRows * FT_NBMAX, b));
     A(dalloc(&w.rowpart, (size_t)kYtopRows, b));
-    A(dalloc(&w.scratch, (size_t)(n + 255) / 256 + 8, b));
+    A(dalloc(&w.scratch, (size_t)64 * ((n + 255) / 256) + 8, b));
+    A(dalloc(&w.linepart, (size_t)64 * ldw, b));
     A(dalloc(&w.deltas, (size_t)FT_MAX_EVENTS, b));
     A(dalloc(&w.bar, 4, b));
+    A(dalloc(&w.strip_done, (N1 + 63) / 64 + 2, b));
     A(dalloc(&w.ctl, 1, b));
     A(dalloc(&w.fixes, (size_t)FT_MAX_EVENTS, b));
     if (e != cudaSuccess) {
@@ -158,6 +163,9 @@ int get_work(int n, Work **out) {
         cudaGetLastError();
         return e == cudaErrorMemoryAllocation ? FT_E_NOMEM : FT_E_CUDA;
     }
+    CK(cudaMemset(w.strip_done, 0, ((N1 + 63) / 64 + 2) * sizeof(int)));  // self-resetting afterwards
+    CK(cudaMemset(w.V, 0, (size_t)ldw * FT_NBMAX * sizeof(double)));
+    CK(cudaMemset(w.Y, 0, (size_t)ldw * FT_NBMAX * sizeof(double)));
     int nsm = 0;
     CK(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev));
     w.nsm = nsm;
@@ -386,6 +394,12 @@ double *site_addr(Call &C, const ft_fault &f) {
     return nullptr;
 }
 
+bool has_fault(const Call &C, int panel, int phase) {
+    for (size_t q = 0; q < C.faults.size() && q < FT_MAXFAULTS; q++)
+        if (C.faults[q].phase == phase && (phase == FT_PHASE_AT_END || C.faults[q].panel == panel)) return true;
+    return false;
+}
+
 int inject_at(Call &C, int panel, int phase) {
     for (size_t q = 0; q < C.faults.size() && q < FT_MAXFAULTS; q++) {
         const ft_fault &f = C.faults[q];
@@ -458,16 +472,14 @@ int right_update(Call &C, int t, double sign, int do_w) {
     g.Wpart = w.Wpart;
     g.wsplit_stride = ((int64_t)C.n + 1 + 64) * FT_NBMAX;
     g.ctl = sign < 0 ? w.ctl : nullptr;
-    // M-part: rows 0..k of the panel columns k+1..e-1 (DGEHRD's DTRMM + DAXPY)
-    g.r_lo = 0;
-    g.r_hi = k + 1;
-    g.c_lo = k + 1;
-    g.c_hi = e;
+    // M-part: rows 0..k of the panel columns k+1..e-1 (DGEHRD's DTRMM + DAXPY), as one extra
+    // strip of the trailing launch
+    g.has_m = 1;
+    g.m_r_hi = k + 1;
+    g.m_c_lo = k + 1;
+    g.m_c_hi = e;
+    // trailing block (+ checksum row/column), fused with W = V^T A_new and W' = T^T W
     g.do_right = 1;
-    g.do_w = 0;
-    g.nsplit = ft_gemm_splits(g.r_lo, g.r_hi, g.c_lo, g.c_hi, w.nsm);
-    CK(ft_launch_gemm_right(g, C.s));
-    // trailing block (+ checksum row/column), fused with W = V^T A_new
     g.r_lo = 0;
     g.r_hi = C.rend();
     g.c_lo = e;
@@ -476,11 +488,17 @@ int right_update(Call &C, int t, double sign, int do_w) {
     g.wr_hi = C.ihi;
     g.do_w = do_w;
     g.nsplit = ft_gemm_splits(g.r_lo, g.r_hi, g.c_lo, g.c_hi, w.nsm);
+    if (do_w) {
+        g.Wt = w.Wt;
+        g.T = w.T;
+        g.transT = 1;
+        g.strip_done = w.strip_done;
+    }
     CK(ft_launch_gemm_right(g, C.s));
     return 0;
 }
 
-int left_update(Call &C, int t, double sign, int nsplit) {
+int left_update(Call &C, int t, double sign, int nsplit, int endcheck = 0) {
     Work &w = *C.w;
     const int k = C.pk(t), ib = C.pib(t), e = k + ib;
     GemmLeftParams g{};
@@ -501,6 +519,13 @@ int left_update(Call &C, int t, double sign, int nsplit) {
     g.transT = 1;
     g.sign = sign;
     g.ctl = sign < 0 ? w.ctl : nullptr;
+    g.wt_ready = 1;  // W' was formed by the right-update launch (and is kept for a rollback)
+    g.endcheck = endcheck;
+    g.panel = t;
+    g.policy = C.policy;
+    g.n = C.n;
+    g.Fr = w.Fr;
+    g.ectl = w.ctl;
     CK(ft_launch_gemm_left(g, C.s));
     return 0;
 }
@@ -524,8 +549,14 @@ int enqueue_panel(Call &C, int t) {
     const int n = C.n, k = C.pk(t), ib = C.pib(t);
     const bool eager = C.abft && C.policy == FT_POLICY_EAGER;
     if (inject_at(C, t, FT_PHASE_BEFORE_PANEL)) return FT_E_CUDA;
-    if (C.abft && checkpoint(C, t, 0)) return FT_E_CUDA;
     PanelParams p{};
+    if (C.abft) {  // the panel kernel takes the diskless checkpoint in its prologue
+        p.ckpt = w.ckpt;
+        p.ck_r = w.ck_r;
+        p.ck_c = w.ck_c;
+        p.ck_q = w.ck_q;
+        p.Fr = w.Fr;
+    }
     p.A = w.Aw;
     p.ldw = w.ldw;
     p.V = w.V;
@@ -545,6 +576,8 @@ int enqueue_panel(Call &C, int t) {
     p.ib = ib;
     p.abft = C.abft;
     p.verify = eager ? 1 : 0;
+    const bool fuse_pre = eager && !has_fault(C, t, FT_PHASE_AFTER_PANEL);
+    p.precheck_sums = fuse_pre ? 1 : 0;
     p.dbg = (t == g_dbg_panel) ? g_dbg_buf : nullptr;
     p.dbg_mode = (t == g_dbg_panel) ? g_dbg_mode : 0;
     const int gr = ft_panel_group_rows();
@@ -579,6 +612,8 @@ int enqueue_panel(Call &C, int t) {
     y.ib = ib;
     y.abft = C.abft;
     y.verify = eager ? 1 : 0;
+    y.decide = fuse_pre ? 1 : 0;
+    y.panel = t;
     int nm = (k + 1 + 63) / 64;
     int nkt = (C.ihi - k - 1 + 31) / 32;
     int ns = std::max(1, std::min({(2 * w.nsm) / nm, nkt / 2, 64}));
@@ -586,15 +621,18 @@ int enqueue_panel(Call &C, int t) {
     y.nsplit = std::max(ns, 1);
     CK(ft_launch_ytop(y, C.s));
     if (inject_at(C, t, FT_PHASE_AFTER_PANEL)) return FT_E_CUDA;
-    if (eager) {
+    if (eager && !fuse_pre) {
+        // a fault is scheduled after the panel: recompute the check sums after it
+        CK(cudaMemsetAsync(w.ctl->eY, 0, sizeof(double) * 2 * FT_NBMAX, C.s));
         CK(ft_precheck(w.Y, w.V, w.ldw, n, C.ihi, k, ib, w.ctl, C.s));
         CK(ft_decide(w.Y, w.V, w.T, w.ldw, n, k, ib, t, w.ctl, C.s));
     }
     if (right_update(C, t, -1.0, 1)) return FT_E_CUDA;
     if (inject_at(C, t, FT_PHASE_AFTER_RIGHT)) return FT_E_CUDA;
-    if (left_update(C, t, -1.0, trailing_nsplit(C, t))) return FT_E_CUDA;
+    const bool fuse_end = C.abft && !has_fault(C, t, FT_PHASE_AFTER_UPDATE);
+    if (left_update(C, t, -1.0, trailing_nsplit(C, t), fuse_end ? 1 : 0)) return FT_E_CUDA;
     if (inject_at(C, t, FT_PHASE_AFTER_UPDATE)) return FT_E_CUDA;
-    if (C.abft) CK(ft_endcheck(w.Aw, w.ldw, n, C.ihi, k, ib, t, C.policy, w.Fr, w.ctl, C.s));
+    if (C.abft && !fuse_end) CK(ft_endcheck(w.Aw, w.ldw, n, C.ihi, k, ib, t, C.policy, w.Fr, w.ctl, C.s));
     return 0;
 }
 
@@ -617,7 +655,8 @@ int verify_and_correct(Call &C, int panel, int cdone, int mode, bool *found) {
     double sums[2], kh;
     *found = false;
     for (int pass = 0; pass < 2; pass++) {
-        CK(ft_full_verify(w.Aw, ldw, n, C.ilo, C.ihi, cdone, mode, r, rinc, c, cinc, nullptr, w.Dr, w.Dc, w.sums, C.s));
+        CK(ft_full_verify(w.Aw, ldw, n, C.ilo, C.ihi, cdone, mode, r, rinc, c, cinc, nullptr, w.Dr, w.Dc, w.sums,
+                          w.linepart, C.s));
         CK(cudaMemcpyAsync(Dr.data(), w.Dr, n * sizeof(double), cudaMemcpyDeviceToHost, C.s));
         CK(cudaMemcpyAsync(Dc.data(), w.Dc, n * sizeof(double), cudaMemcpyDeviceToHost, C.s));
         CK(cudaMemcpyAsync(sums, w.sums, 2 * sizeof(double), cudaMemcpyDeviceToHost, C.s));
@@ -691,7 +730,7 @@ int recover(Call &C, const FtCtl &h) {
     CK(cudaMemcpyAsync(&w.ctl->nflag, &zero, sizeof(int), cudaMemcpyHostToDevice, C.s));
     CK(cudaMemsetAsync(w.ctl->eY, 0, sizeof(double) * 128, C.s));
     CK(cudaMemsetAsync(w.ctl->sums, 0, sizeof(double) * 4, C.s));
-    CK(cudaMemsetAsync(&w.ctl->done_count, 0, sizeof(int), C.s));
+    CK(cudaMemsetAsync(&w.ctl->done_count, 0, 3 * sizeof(int), C.s));  // done_count, done_ytop, done_left
     if (h.halt_stage == 2) {
         // reverse computation: add back the left, then the right update
         if (left_update(C, t, +1.0, trailing_nsplit(C, t))) return FT_E_CUDA;
@@ -769,7 +808,7 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
     CK(cudaMemsetAsync(w.bvec, 0, (size_t)w.ldw * sizeof(double), s));  // b(q >= ihi) must read 0
     if (reset_panel_state(C)) return FT_E_CUDA;
     if (C.abft) {
-        CK(ft_encode(w.Aw, w.ldw, n, w.ctl, w.scratch, s));
+        CK(ft_encode(w.Aw, w.ldw, n, w.ctl, w.scratch, w.linepart, s));
         CK(cudaMemsetAsync(w.Fr, 0, w.ldw * sizeof(double), s));
         if (ilo > 1) CK(ft_frozen_init(w.Aw, w.ldw, n, ilo - 1, w.Fr, s));
         CK(cudaMemsetAsync(w.Qr, 0, w.ldw * sizeof(double), s));
@@ -984,6 +1023,10 @@ int ft_dorghr(int n, int ilo, int ihi, const double *dA, int lda, const double *
         const int ns = ft_gemm_splits(k + 1, ihi, k + 1, ihi, w.nsm);
         g.nsplit = ns;
         g.ctl = nullptr;
+        g.Wt = w.Wt;
+        g.T = w.T;
+        g.transT = 0;
+        g.strip_done = w.strip_done;
         CK(ft_launch_gemm_right(g, s));
         GemmLeftParams L{};
         L.A = Qw;
@@ -1003,6 +1046,7 @@ int ft_dorghr(int n, int ilo, int ihi, const double *dA, int lda, const double *
         L.transT = 0;
         L.sign = -1.0;
         L.ctl = nullptr;
+        L.wt_ready = 1;
         CK(ft_launch_gemm_left(L, s));
     }
     if (Qw != dQ)

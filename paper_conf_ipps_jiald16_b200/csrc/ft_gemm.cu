@@ -96,12 +96,16 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_right(GemmRightParams p) {
     RightSmemT<KT> &S = *reinterpret_cast<RightSmemT<KT> *>(smem_raw);
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int lr = lane >> 2, lc = lane & 3;
-    const int cb = p.c_lo + blockIdx.x * UB;
-    const int ncols = min(UB, p.c_hi - cb);
+    // the last strip of the grid is the M-part when present (rows 0..m_r_hi, no W)
+    const bool mpart = p.has_m && blockIdx.x == gridDim.x - 1;
+    const int r_lo = mpart ? 0 : p.r_lo, r_hi = mpart ? p.m_r_hi : p.r_hi;
+    const int do_w = mpart ? 0 : p.do_w;
+    const int cb = mpart ? p.m_c_lo : p.c_lo + blockIdx.x * UB;
+    const int ncols = min(UB, (mpart ? p.m_c_hi : p.c_hi) - cb);
     const int K = p.K;
     const double sg = p.sign;
-    const int rbase = (p.r_lo / UB) * UB;
-    const int nrt = (p.r_hi - rbase + UB - 1) / UB;
+    const int rbase = (r_lo / UB) * UB;
+    const int nrt = (r_hi - rbase + UB - 1) / UB;
     const int t0 = (int)((long long)blockIdx.y * nrt / gridDim.y);
     const int t1 = (int)((long long)(blockIdx.y + 1) * nrt / gridDim.y);
     constexpr int NJ = KT / 8;
@@ -121,14 +125,14 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_right(GemmRightParams p) {
 
     // pipeline invariant at the top of tile tt: groups [Ys(tt), Vr(tt)] in flight
     if (t0 < t1) {
-        if (p.do_right) issue_ktile<KT>(S.Ys, p.Y, p.ldw, rbase + t0 * UB, p.r_hi, K);
+        if (p.do_right) issue_ktile<KT>(S.Ys, p.Y, p.ldw, rbase + t0 * UB, r_hi, K);
         cp_async_commit();
-        if (p.do_w) issue_ktile<KT>(S.Vr, p.V, p.ldw, rbase + t0 * UB, p.r_hi, K);
+        if (do_w) issue_ktile<KT>(S.Vr, p.V, p.ldw, rbase + t0 * UB, r_hi, K);
         cp_async_commit();
     }
     for (int tt = t0; tt < t1; tt++) {
         const int r = rbase + tt * UB;
-        const int lo = max(r, p.r_lo), hi = min(r + UB, p.r_hi);
+        const int lo = max(r, r_lo), hi = min(r + UB, r_hi);
         const bool full = lo == r && hi == r + UB && ncols == UB;  // interior tile: no masks
         double acc[8][2];
 #pragma unroll
@@ -160,9 +164,9 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_right(GemmRightParams p) {
             }
         }
         __syncthreads();  // every warp is done with Ys(tt)
-        if (p.do_right && tt + 1 < t1) issue_ktile<KT>(S.Ys, p.Y, p.ldw, r + UB, p.r_hi, K);
+        if (p.do_right && tt + 1 < t1) issue_ktile<KT>(S.Ys, p.Y, p.ldw, r + UB, r_hi, K);
         cp_async_commit();
-        if (p.do_w) {
+        if (do_w) {
             cp_async_wait<1>();
             __syncthreads();
             // only rows in [wr_lo, wr_hi) take part in W
@@ -189,12 +193,12 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_right(GemmRightParams p) {
                 }
             }
             __syncthreads();  // every warp is done with Vr(tt)
-            if (tt + 1 < t1) issue_ktile<KT>(S.Vr, p.V, p.ldw, r + UB, p.r_hi, K);
+            if (tt + 1 < t1) issue_ktile<KT>(S.Vr, p.V, p.ldw, r + UB, r_hi, K);
         }
         cp_async_commit();
     }
     cp_async_wait<0>();
-    if (p.do_w) {
+    if (do_w) {
         // deterministic partial of this row split: Wpart[split][col][j]
         double *Wp = p.Wpart + (int64_t)blockIdx.y * p.wsplit_stride;
         if (colok)
@@ -205,6 +209,54 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_right(GemmRightParams p) {
                     const int jj = nj * 8 + 2 * lc + v;
                     if (jj < K) Wp[(int64_t)(cb + wcol) * FT_NBMAX + jj] = wacc[nj][v];
                 }
+        if (p.Wt) {
+            // the last CTA of the strip sums the partials (fixed order) and forms W' = op(T) W
+            __shared__ int last;
+            __threadfence();
+            __syncthreads();
+            if (tid == 0) last = atomicAdd(&p.strip_done[blockIdx.x], 1) == (int)gridDim.y - 1;
+            __syncthreads();
+            if (last) {
+                __threadfence();
+                double(*Ts)[SK] = S.Vc;  // reuse: T as Ts[a][b] (KT x KT)
+                double(*Ws)[SK] = S.Ys;  // W as Ws[col][b] (64 x KT): spans Ys and Vr (contiguous)
+                for (int i = tid; i < KT * KT; i += UT) {
+                    const int a = i % KT, b = i / KT;
+                    Ts[a][b] = (a < K && b < K) ? p.T[a + b * FT_NBMAX] : 0.0;
+                }
+                for (int i = tid; i < UB * KT; i += UT) {
+                    const int cc = i / KT, b = i % KT;
+                    double w = 0.0;
+                    if (cc < ncols && b < K)
+                        for (int sp = 0; sp < (int)gridDim.y; sp++)
+                            w += __ldcg(p.Wpart + (int64_t)sp * p.wsplit_stride + (int64_t)(cb + cc) * FT_NBMAX + b);
+                    Ws[cc][b] = w;
+                }
+                __syncthreads();
+                for (int i = tid; i < UB * KT; i += UT) {
+                    const int cc = i / KT, a = i % KT;
+                    if (cc >= ncols || a >= K) continue;
+                    double s0 = 0.0, s1 = 0.0;
+                    if (p.transT) {  // W'(a) = sum_{b <= a} T(b, a) W(b)
+                        int b = 0;
+                        for (; b + 1 <= a; b += 2) {
+                            s0 += Ts[b][a] * Ws[cc][b];
+                            s1 += Ts[b + 1][a] * Ws[cc][b + 1];
+                        }
+                        if (b <= a) s0 += Ts[b][a] * Ws[cc][b];
+                    } else {  // W'(a) = sum_{b >= a} T(a, b) W(b)
+                        int b = a;
+                        for (; b + 1 < K; b += 2) {
+                            s0 += Ts[a][b] * Ws[cc][b];
+                            s1 += Ts[a][b + 1] * Ws[cc][b + 1];
+                        }
+                        if (b < K) s0 += Ts[a][b] * Ws[cc][b];
+                    }
+                    p.Wt[(int64_t)(cb + cc) * FT_NBMAX + a] = s0 + s1;
+                }
+                if (tid == 0) p.strip_done[blockIdx.x] = 0;
+            }
+        }
     }
 }
 
@@ -217,14 +269,31 @@ static cudaError_t launch_right_kt(const GemmRightParams &p, cudaStream_t s) {
         if (e != cudaSuccess) return e;
         attr = true;
     }
-    const int nstrip = (p.c_hi - p.c_lo + UB - 1) / UB;
+    const int nstrip = (p.c_hi - p.c_lo + UB - 1) / UB + (p.has_m ? 1 : 0);
     const int ny = p.nsplit > 0 ? p.nsplit : 1;
     g_ft_launches++;
     k_gemm_right<KT><<<dim3(nstrip, ny), UT, smem, s>>>(p);
     return cudaGetLastError();
 }
 cudaError_t ft_launch_gemm_right(const GemmRightParams &p, cudaStream_t s) {
-    if (p.r_hi <= p.r_lo || p.c_hi <= p.c_lo || p.K <= 0) return cudaSuccess;
+    if (p.K <= 0) return cudaSuccess;
+    if (p.r_hi <= p.r_lo || p.c_hi <= p.c_lo) {  // no trailing block: at most the M-part
+        if (!p.has_m || p.m_r_hi <= 0 || p.m_c_hi <= p.m_c_lo) return cudaSuccess;
+        GemmRightParams q = p;
+        q.has_m = 0;
+        q.r_lo = 0;
+        q.r_hi = p.m_r_hi;
+        q.c_lo = p.m_c_lo;
+        q.c_hi = p.m_c_hi;
+        q.do_w = 0;
+        q.Wt = nullptr;
+        return ft_launch_gemm_right(q, s);
+    }
+    if (p.has_m && (p.m_r_hi <= 0 || p.m_c_hi <= p.m_c_lo)) {
+        GemmRightParams q = p;
+        q.has_m = 0;
+        return ft_launch_gemm_right(q, s);
+    }
     if (p.do_w && p.nsplit > FT_WSPLIT_MAX) return cudaErrorInvalidValue;
     const bool aligned = (p.lda % 2 == 0) && ((((uintptr_t)p.A) & 15) == 0) && (p.ldw % 2 == 0) &&
                          ((((uintptr_t)p.V) & 15) == 0) && (!p.do_right || ((((uintptr_t)p.Y) & 15) == 0));
@@ -300,6 +369,18 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
 
     if (t0 < t1) issue_ktile<KT>(S.Vr[0], p.V, p.ldw, rbase + t0 * UB, p.r_hi, K);
     cp_async_commit();
+    if (p.endcheck) {
+        // frozen row sums of the panel columns k..e-1 (final now, untouched by this kernel; R6):
+        // Fr(i) += sum_{col in [k,e), i <= col+1} A(i, col) for i <= e
+        const int k = p.r_lo - 1, e = p.c_lo;
+        const int nb = gridDim.x * gridDim.y, b = blockIdx.y * gridDim.x + blockIdx.x;
+        for (int i = b * UT + tid; i <= e && i < p.n; i += nb * UT) {
+            double s = 0.0;
+            for (int col = k; col < e; col++)
+                if (i <= col + 1) s += p.A[i + (int64_t)col * p.lda];
+            p.Fr[i] += s;
+        }
+    }
     // W'^T for the strip: Wt [col][64] -> Wc[k][col]
     for (int i = tid; i < KT * UB; i += UT) {
         const int cc = i / KT, kk = i % KT;
@@ -358,6 +439,53 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
         __syncthreads();  // Vr[st] is refilled two tiles later
     }
     cp_async_wait<0>();
+    if (!p.endcheck) return;
+    // fused end-of-iteration check (Alg. 3 l.12-13; R11/R22): once every CTA has finished, the
+    // last one compares sum r and sum c with kappa (EAGER) or with each other (PAPER)
+    __shared__ int last;
+    __shared__ double red2[2][UT / 32];
+    __threadfence();
+    __syncthreads();
+    if (tid == 0) last = atomicAdd(&p.ectl->done_left, 1) == (int)(gridDim.x * gridDim.y) - 1;
+    __syncthreads();
+    if (!last) return;
+    __threadfence();
+    const int n = p.n;
+    double sr = 0.0, sc = 0.0;
+    for (int i = tid; i < n; i += UT) {
+        sr += __ldcg(p.A + i + (int64_t)n * p.lda);
+        sc += __ldcg(p.A + n + (int64_t)i * p.lda);
+    }
+    sr = warp_sum(sr);
+    sc = warp_sum(sc);
+    if (lane == 0) {
+        red2[0][warp] = sr;
+        red2[1][warp] = sc;
+    }
+    __syncthreads();
+    if (tid != 0) return;
+    double Sr = 0.0, Sc = 0.0;
+    for (int w = 0; w < UT / 32; w++) {
+        Sr += red2[0][w];
+        Sc += red2[1][w];
+    }
+    FtCtl *ctl = p.ectl;
+    const double kap = __ldcg(p.A + n + (int64_t)n * p.lda);
+    const double tauS = ctl->c_thr * (double)n * 2.220446049250313e-16 * ctl->normF * sqrt((double)n);
+    int reason = 0;
+    if (p.policy == FT_POLICY_PAPER) {
+        if (not_within(Sr - Sc, tauS)) reason |= 8;
+    } else {
+        if (not_within(Sr - kap, tauS) || not_within(Sc - kap, tauS)) reason |= 8;
+    }
+    ctl->done_left = 0;
+    if (reason) {
+        ctl->halt_panel = p.panel;
+        ctl->halt_stage = 2;
+        ctl->halt_reason = reason;
+        __threadfence();
+        ctl->halt = 1;
+    }
 }
 
 template <int KT>
@@ -378,10 +506,14 @@ static cudaError_t launch_left_kt(const GemmLeftParams &p, cudaStream_t s) {
     }
     const int nrt = (p.r_hi - (p.r_lo / UB) * UB + UB - 1) / UB;
     const int ny = best_splits(nstrip, nrt, nsm, 1 << 20);
-    g_ft_launches += 2;
-    const int per = UT / FT_NBMAX;  // columns per k_wprep block
-    k_wprep<<<(p.c_hi - p.c_lo + per - 1) / per, UT, 0, s>>>(p.Wpart, p.wsplit_stride, p.nsplit > 0 ? p.nsplit : 1,
-                                                              p.T, p.Wt, p.c_lo, p.c_hi, p.K, p.transT, p.ctl);
+    if (!p.wt_ready) {
+        g_ft_launches++;
+        const int per = UT / FT_NBMAX;  // columns per k_wprep block
+        k_wprep<<<(p.c_hi - p.c_lo + per - 1) / per, UT, 0, s>>>(p.Wpart, p.wsplit_stride,
+                                                                  p.nsplit > 0 ? p.nsplit : 1, p.T, p.Wt, p.c_lo,
+                                                                  p.c_hi, p.K, p.transT, p.ctl);
+    }
+    g_ft_launches++;
     GemmLeftParams q = p;
     q.Wpart = p.Wt;  // the main kernel reads W' = op(T) W
     k_gemm_left<KT><<<dim3(nstrip, ny), UT, smem, s>>>(q);
@@ -468,6 +600,7 @@ __global__ void __launch_bounds__(YF_R * 64) k_ytop_finalize(YtopParams p) {
     if (p.ctl->halt) return;
     __shared__ double Ts[FT_NBMAX * FT_NBMAX];
     __shared__ double y0[YF_R][FT_NBMAX + 1];
+    __shared__ int last;
     const int jb = threadIdx.x & 63, rl = threadIdx.x >> 6;
     const int row = blockIdx.x * YF_R + rl;
     const int ib = p.ib;
@@ -481,13 +614,12 @@ __global__ void __launch_bounds__(YF_R * 64) k_ytop_finalize(YtopParams p) {
             acc += p.ypart[(int64_t)sp * (p.k + 1) * FT_NBMAX + (int64_t)row * FT_NBMAX + jb];
     y0[rl][jb] = acc;
     __syncthreads();
-    if (row > p.k) return;
-    if (jb < ib) {
-        double s = 0.0;
-        for (int b = 0; b <= jb; b++) s += y0[rl][b] * Ts[b + jb * FT_NBMAX];
-        p.Y[row + (int64_t)jb * p.ldw] = s;
+    double yv = 0.0;
+    if (row <= p.k && jb < ib) {
+        for (int b = 0; b <= jb; b++) yv += y0[rl][b] * Ts[b + jb * FT_NBMAX];
+        p.Y[row + (int64_t)jb * p.ldw] = yv;
     }
-    if (p.verify && jb == 0) {
+    if (p.verify && row <= p.k && jb == 0) {
         double rsum = 0.0;
         for (int sp = 0; sp < p.nsplit; sp++) rsum += p.rowpart[(int64_t)sp * (p.k + 1) + row];
         rsum += p.A[row + (int64_t)p.k * p.ldw];
@@ -495,6 +627,56 @@ __global__ void __launch_bounds__(YF_R * 64) k_ytop_finalize(YtopParams p) {
         double d = p.A[row + (int64_t)p.n * p.ldw] - p.Fr[row] - rsum;
         double tau_abs = p.ctl->c_thr * (double)p.n * 2.220446049250313e-16 * p.ctl->normF;
         if (not_within(d, tau_abs)) atomicAdd(&p.ctl->nflag, 1);
+    }
+    if (!p.decide) return;
+    // fused pre-update check (reading R15): e^T Y of rows 0..k, then the last block decides
+    __syncthreads();
+    y0[rl][jb] = yv;
+    __syncthreads();
+    if (rl == 0 && jb < ib) {
+        double s = 0.0;
+        for (int q = 0; q < YF_R; q++) s += y0[q][jb];
+        atomicAdd(&p.ctl->eY[jb], s);
+    }
+    __threadfence();
+    __syncthreads();
+    if (threadIdx.x == 0) last = atomicAdd(&p.ctl->done_ytop, 1) == (int)gridDim.x - 1;
+    __syncthreads();
+    if (!last || threadIdx.x >= 32) return;
+    __threadfence();
+    FtCtl *ctl = p.ctl;
+    const int lane = threadIdx.x, n = p.n;
+    const double unit = (double)n * 2.220446049250313e-16 * ctl->normF;
+    double tmax = 0.0;
+    for (int i = lane; i < ib * ib; i += 32) tmax = fmax(tmax, fabs(Ts[(i % ib) + (i / ib) * FT_NBMAX]));
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) tmax = fmax(tmax, __shfl_xor_sync(0xffffffffu, tmax, o));
+    int reason = 0;
+    if (atomicAdd(&ctl->nflag, 0) > 0) reason |= 1;
+    const double tauY = ctl->c_thr * unit * (tmax > 1.0 ? tmax : 1.0);
+    const double tauV = ctl->c_thr * (double)n * 2.220446049250313e-16 * sqrt((double)n);
+    for (int j = lane; j < ib; j += 32) {
+        const double dy = __ldcg(&ctl->eY[j]) - p.Y[n + (int64_t)j * p.ldw];
+        const double dv = __ldcg(&ctl->eV[j]) - p.V[n + (int64_t)j * p.ldw];
+        if (not_within(dy, tauY)) reason |= 2;
+        if (not_within(dv, tauV)) reason |= 4;
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) reason |= __shfl_xor_sync(0xffffffffu, reason, o);
+    for (int j = lane; j < FT_NBMAX; j += 32) {
+        ctl->eY[j] = 0.0;
+        ctl->eV[j] = 0.0;
+    }
+    if (lane == 0) {
+        ctl->nflag = 0;
+        ctl->done_ytop = 0;
+        if (reason) {
+            ctl->halt_panel = p.panel;
+            ctl->halt_stage = 1;
+            ctl->halt_reason = reason;
+            __threadfence();
+            ctl->halt = 1;
+        }
     }
 }
 

@@ -22,8 +22,9 @@ struct FtCtl {
     int halt_stage;   // 1 = pre-update (verify-before-consume / workspace check), 2 = post-update
     int halt_reason;  // bit 0: D_r flag, 1: Y check, 2: V check, 3: scalar check (paper), 4: kappa
     int nflag;        // flagged rows in the fused verify of the current iteration
-    int done_count;   // last-block-done counter
-    int pad[2];
+    int done_count;   // last-block-done counter (k_endcheck)
+    int done_ytop;    // last-block-done counter (fused pre-update decision in the Y_top finalize)
+    int done_left;    // last-CTA-done counter (fused end-of-iteration check in the left update)
     double normF;         // ||A||_F of the input (invariant under the similarity)
     double c_thr;
     unsigned long long drift_bits;  // max fault-free |D| / (n eps ||A||_F) seen (as bits)
@@ -44,6 +45,9 @@ struct PanelParams {
     double *Qr, *Qc;
     int n, ihi, k, ib, abft, verify;  // verify: fused D_r on the first GEMV (EAGER policy)
     int rbase, ngroups;               // ft_panel_group_rows()-row groups starting at rbase
+    // diskless checkpoint of the panel, taken in the kernel's prologue, or NULL
+    double *ckpt, *ck_r, *ck_c, *ck_q, *Fr;
+    int precheck_sums;  // add e^T Y, e^T V of the own rows into ctl->eY / eV (fused pre-update check)
     unsigned long long *dbg;          // optional per-column phase timestamps (CTA 0), or NULL
     int dbg_mode;                     // timing ablations (wrong results): 1 no grid barriers, 2 no GEMV, 4 no atomics
 };
@@ -66,6 +70,14 @@ struct GemmRightParams {
     int64_t wsplit_stride;          // doubles per split
     int nsplit;                     // row splits (grid.y); use ft_gemm_splits()
     const FtCtl *ctl;
+    // optional M-part (DGEHRD's DTRMM + DAXPY on rows 0..m_r_hi-1 of columns m_c_lo..m_c_hi-1),
+    // run as one extra strip of the same launch (no W)
+    int has_m, m_c_lo, m_c_hi, m_r_hi;
+    // W' = op(T) W formed by the last CTA of each strip (the left update's operand), if Wt != NULL
+    double *Wt;
+    const double *T;
+    int transT;
+    int *strip_done;  // per-strip arrival counters (zero; reset by their last CTA)
 };
 cudaError_t ft_launch_gemm_right(const GemmRightParams &p, cudaStream_t s);
 #define FT_WSPLIT_MAX 16  // max row splits of the right update (deterministic W partials)
@@ -84,6 +96,11 @@ struct GemmLeftParams {
     int transT;     // 1: A -= V (T^T W) (DLARFB 'L','T'); 0: A -= V (T W)
     double sign;    // -1 update, +1 rollback
     const FtCtl *ctl;
+    int wt_ready;   // 1: Wt already holds op(T) W (formed by the right-update launch)
+    // fused end-of-iteration check (Alg. 3 l.12-13) + frozen row sums; last CTA decides
+    int endcheck, panel, policy, n;
+    double *Fr;
+    FtCtl *ectl;
 };
 cudaError_t ft_launch_gemm_left(const GemmLeftParams &p, cudaStream_t s);
 
@@ -96,13 +113,16 @@ struct YtopParams {
     const double *Fr;
     FtCtl *ctl;
     int n, ihi, k, ib, nsplit, abft, verify;
+    int decide;  // fused pre-update check (R15): add e^T Y of rows 0..k, last block decides
+    int panel;
 };
 cudaError_t ft_launch_ytop(const YtopParams &p, cudaStream_t s);
 
 // ABFT / utility kernels (ft_abft.cu)
 cudaError_t ft_copy_in(const double *A, int lda, double *Aw, int64_t ldw, int n, cudaStream_t s);
 cudaError_t ft_copy_out(const double *Aw, int64_t ldw, double *A, int lda, int n, cudaStream_t s);
-cudaError_t ft_encode(double *Aw, int64_t ldw, int n, FtCtl *ctl, double *scratch, cudaStream_t s);
+cudaError_t ft_encode(double *Aw, int64_t ldw, int n, FtCtl *ctl, double *scratch, double *linepart,
+                      cudaStream_t s);
 cudaError_t ft_frozen_init(const double *Aw, int64_t ldw, int n, int ncols, double *Fr, cudaStream_t s);
 cudaError_t ft_precheck(const double *Y, const double *V, int64_t ldw, int n, int ihi, int k, int ib,
                         FtCtl *ctl, cudaStream_t s);
@@ -115,7 +135,7 @@ cudaError_t ft_inject(double *addr, int fidx, int bit, FtCtl *ctl, cudaStream_t 
 // full verification (recovery path / final): mode 0 = H logical, 1 = Q (V region)
 cudaError_t ft_full_verify(const double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdone, int mode,
                            const double *r, int64_t rinc, const double *c, int64_t cinc, const double *Fr,
-                           double *Dr, double *Dc, double *sums, cudaStream_t s);
+                           double *Dr, double *Dc, double *sums, double *linepart, cudaStream_t s);
 struct FtFix { int64_t i, j; int kind; int pad; };  // kind: 0 row formula, 1 col formula, 2 refresh r(i), 3 refresh c(j), 4 kappa
 cudaError_t ft_apply_fixes(double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdone, int mode,
                            double *r, int64_t rinc, double *c, int64_t cinc, double *kappa,

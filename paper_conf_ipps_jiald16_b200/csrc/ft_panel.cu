@@ -162,6 +162,29 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
 
 #pragma unroll 1
     for (int i = tid; i < FT_NBMAX * (FT_NBMAX + 1); i += PT) (&S.Ts[0][0])[i] = 0.0;
+    if (p.ckpt) {
+        // diskless checkpoint of the panel columns, r, c, kappa, Qr, Qc, Fr, taken
+        // before anything is modified: own rows by their owner, c by the owner of row n (it
+        // rewrites c(k:e)), the rest grid-strided; all of it precedes this CTA's first arrival
+        const int rend = p.abft ? n + 1 : ihi;
+        for (int x = tid; x < R * ib; x += PT) {
+            const int rl = x % R, jj = x / R, row = r0 + rl;
+            if (row < rend) p.ckpt[row + (int64_t)jj * ldw] = A[row + (int64_t)(k + jj) * ldw];
+        }
+        const int gstride = (int)P * PT, g = blockIdx.x * PT + tid;
+        for (int x = g; x < p.rbase * ib; x += gstride) {
+            const int i = x % p.rbase, jj = x / p.rbase;
+            p.ckpt[i + (int64_t)jj * ldw] = A[i + (int64_t)(k + jj) * ldw];
+        }
+        for (int i = g; i <= n; i += gstride) {
+            p.ck_r[i] = A[i + (int64_t)n * ldw];
+            p.ck_q[i] = p.Qr[i];
+            p.ck_q[ldw + i] = p.Qc[i];
+            p.ck_q[2 * ldw + i] = p.Fr[i];
+        }
+        if (r0 <= n && n < r1)
+            for (int i = tid; i <= n; i += PT) p.ck_c[i] = A[n + (int64_t)i * ldw];
+    }
     for (int rl = tid; rl < R; rl += PT) {
         const int row = r0 + rl;
         const bool valid = (row >= k + 1 && row < ihi) || (p.abft && row == n);
@@ -454,6 +477,17 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
             for (int jj = 0; jj < ib; jj++)
                 if (row >= k + jj + 2) s += Vl[rl * XR + jj * XC];
             p.Qr[row] += s;
+        }
+    if (p.precheck_sums)  // e^T Y, e^T V over the own data rows (pre-update check R15, fused)
+        for (int jj = lane; jj < ib; jj += 32) {
+            double sy = 0.0, sv = 0.0;
+            for (int rl = 0; rl < R; rl++)
+                if (is_data(r0 + rl)) {
+                    sy += Yl[rl * XR + jj * XC];
+                    sv += Vl[rl * XR + jj * XC];
+                }
+            atomicAdd(&p.ctl->eY[jj], sy);
+            atomicAdd(&p.ctl->eV[jj], sv);
         }
     if (blockIdx.x == 0)
         for (int i = lane; i < ib * ib; i += 32) {
