@@ -35,6 +35,19 @@ cudaError_t ft_copy_out(const double *Aw, int64_t ldw, double *A, int lda, int n
     return cudaGetLastError();
 }
 
+// control block initialisation as a kernel (capturable into a CUDA graph)
+__global__ void k_ctl_init(FtCtl *ctl, double c_thr) {
+    unsigned *w = reinterpret_cast<unsigned *>(ctl);
+    for (size_t i = threadIdx.x; i < sizeof(FtCtl) / sizeof(unsigned); i += blockDim.x) w[i] = 0u;
+    __syncthreads();
+    if (threadIdx.x == 0) ctl->c_thr = c_thr;
+}
+cudaError_t ft_ctl_init(FtCtl *ctl, double c_thr, cudaStream_t s) {
+    g_ft_launches++;
+    k_ctl_init<<<1, 256, 0, s>>>(ctl, c_thr);
+    return cudaGetLastError();
+}
+
 // ---------------------------------------------------------------------------
 // encode: row sums as 2-D tiled partial sums (thread per row, 64-column chunks, fixed-order
 // finish: deterministic), column sums (warp per column), ||A||_F^2

@@ -14,6 +14,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <map>
+#include <tuple>
 #include <vector>
 
 #include "ft_internal.h"
@@ -84,6 +85,7 @@ struct Work {
            *rowpart = nullptr, *linepart = nullptr, *scratch = nullptr, *deltas = nullptr, *hA = nullptr, *htau = nullptr;
     unsigned *bar = nullptr;
     int *strip_done = nullptr;
+    cudaStream_t cap_stream = nullptr;  // graph capture stream (library-owned)
     FtCtl *ctl = nullptr;
     FtFix *fixes = nullptr;
     int nsm = 0;
@@ -109,6 +111,35 @@ struct Work {
 };
 std::map<int, Work> g_work;
 
+// CUDA graphs of fault-free calls, keyed by device, shape, options and caller buffers
+struct GraphKey {
+    int dev, n, ilo, ihi, nb, abft, policy;
+    double c_thr;
+    const void *dA;
+    int lda;
+    const void *dtau;
+    bool operator<(const GraphKey &o) const {
+        return std::tie(dev, n, ilo, ihi, nb, abft, policy, c_thr, dA, lda, dtau) <
+               std::tie(o.dev, o.n, o.ilo, o.ihi, o.nb, o.abft, o.policy, o.c_thr, o.dA, o.lda, o.dtau);
+    }
+};
+struct GraphEntry {
+    cudaGraphExec_t exec = nullptr;
+    int64_t launches = 0;
+    bool failed = false;
+};
+std::map<GraphKey, GraphEntry> g_graphs;
+void drop_graphs(int dev) {
+    for (auto it = g_graphs.begin(); it != g_graphs.end();) {
+        if (it->first.dev == dev) {
+            if (it->second.exec) cudaGraphExecDestroy(it->second.exec);
+            it = g_graphs.erase(it);
+        } else {
+            ++it;
+        }
+    }
+}
+
 template <class T>
 cudaError_t dalloc(T **p, size_t count, size_t &acc) {
     acc += count * sizeof(T);
@@ -123,6 +154,7 @@ int get_work(int n, Work **out) {
         *out = &w;
         return 0;
     }
+    drop_graphs(dev);  // captured graphs hold the old workspace pointers
     w.release();
     int64_t ldw = ((int64_t)n + 2 + 31) / 32 * 32;
     size_t N1 = (size_t)n + 1;
@@ -749,6 +781,30 @@ int recover(Call &C, const FtCtl &h) {
     return info;
 }
 
+// start of a call: control block, working array (A, zero padding, checksum row/column,
+// P:218-224), panel sync state, encode (Alg. 3 l.2), Q checksums
+int enqueue_start(Call &C, const double *dA, int lda) {
+    Work &w = *C.w;
+    const int n = C.n;
+    cudaStream_t s = C.s;
+    if (n > 1) CK(cudaMemsetAsync(C.tau, 0, (n - 1) * sizeof(double), s));
+    CK(ft_ctl_init(w.ctl, C.c_thr, s));
+    CK(cudaMemsetAsync(w.Aw, 0, (size_t)w.ldw * (n + 1) * sizeof(double), s));
+    CK(cudaMemsetAsync(w.V, 0, (size_t)w.ldw * FT_NBMAX * sizeof(double), s));
+    CK(cudaMemsetAsync(w.Y, 0, (size_t)w.ldw * FT_NBMAX * sizeof(double), s));
+    CK(ft_copy_in(dA, lda, w.Aw, w.ldw, n, s));
+    CK(cudaMemsetAsync(w.bvec, 0, (size_t)w.ldw * sizeof(double), s));  // b(q >= ihi) must read 0
+    if (reset_panel_state(C)) return FT_E_CUDA;
+    if (C.abft) {
+        CK(ft_encode(w.Aw, w.ldw, n, w.ctl, w.scratch, w.linepart, s));
+        CK(cudaMemsetAsync(w.Fr, 0, w.ldw * sizeof(double), s));
+        if (C.ilo > 1) CK(ft_frozen_init(w.Aw, w.ldw, n, C.ilo - 1, w.Fr, s));
+        CK(cudaMemsetAsync(w.Qr, 0, w.ldw * sizeof(double), s));
+        CK(cudaMemsetAsync(w.Qc, 0, w.ldw * sizeof(double), s));
+    }
+    return 0;
+}
+
 int validate(int n, int ilo, int ihi, const void *A, int lda, const void *tau, const ft_opts *o) {
     if (n < 0) return -1;
     if (ilo < 1 || ilo > std::max(1, n)) return -2;
@@ -776,7 +832,6 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
     if (info) return info;
     cudaStream_t s = (cudaStream_t)o.stream;
     if (n == 0) return 0;
-    if (n > 1) CK(cudaMemsetAsync(dtau, 0, (n - 1) * sizeof(double), s));
     Call C;
     C.n = n;
     C.ilo = ilo;
@@ -795,29 +850,62 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
     CK(cudaEventCreate(&ev0));
     CK(cudaEventCreate(&ev1));
     CK(cudaEventRecord(ev0, s));
-    // control block
-    FtCtl h0;
-    memset(&h0, 0, sizeof(h0));
-    h0.c_thr = C.c_thr;
-    CK(cudaMemcpyAsync(w.ctl, &h0, sizeof(FtCtl), cudaMemcpyHostToDevice, s));
-    // working array: A, zero padding, checksum row/column
-    CK(cudaMemsetAsync(w.Aw, 0, (size_t)w.ldw * (n + 1) * sizeof(double), s));
-    CK(cudaMemsetAsync(w.V, 0, (size_t)w.ldw * FT_NBMAX * sizeof(double), s));
-    CK(cudaMemsetAsync(w.Y, 0, (size_t)w.ldw * FT_NBMAX * sizeof(double), s));
-    CK(ft_copy_in(dA, lda, w.Aw, w.ldw, n, s));
-    CK(cudaMemsetAsync(w.bvec, 0, (size_t)w.ldw * sizeof(double), s));  // b(q >= ihi) must read 0
-    if (reset_panel_state(C)) return FT_E_CUDA;
-    if (C.abft) {
-        CK(ft_encode(w.Aw, w.ldw, n, w.ctl, w.scratch, w.linepart, s));
-        CK(cudaMemsetAsync(w.Fr, 0, w.ldw * sizeof(double), s));
-        if (ilo > 1) CK(ft_frozen_init(w.Aw, w.ldw, n, ilo - 1, w.Fr, s));
-        CK(cudaMemsetAsync(w.Qr, 0, w.ldw * sizeof(double), s));
-        CK(cudaMemsetAsync(w.Qc, 0, w.ldw * sizeof(double), s));
-    }
     C.npanels = 0;
     for (int k = ilo - 1; k < ihi - 2; k += C.nb) C.npanels++;
     const int last = (o.stop_after_panel >= 0) ? std::min(o.stop_after_panel + 1, C.npanels) : C.npanels;
-    int t0 = 0, attempts = 0;
+    // Fault-free calls replay one CUDA graph of the whole launch sequence (start-up kernels and
+    // every iteration), captured on the second call with the same shape and buffers; the halt
+    // protocol is unchanged (a halted graph's remaining kernels are no-ops, recovery follows).
+    const bool graphable = C.faults.empty() && o.stop_after_panel < 0 && g_dbg_panel < 0 && !g_time_panels &&
+                           !getenv("FT_NO_GRAPH");
+    bool launched = false;
+    if (graphable) {
+        int dev = 0;
+        CK(cudaGetDevice(&dev));
+        GraphKey key{dev, n, ilo, ihi, C.nb, C.abft, C.policy, C.c_thr, (const void *)dA, lda, (const void *)dtau};
+        auto it = g_graphs.find(key);
+        if (it != g_graphs.end() && it->second.exec) {
+            CK(cudaGraphLaunch(it->second.exec, s));
+            g_ft_launches += it->second.launches;
+            launched = true;
+        } else if (it != g_graphs.end() && !it->second.failed) {  // second call: capture
+            // record on a library-owned stream (the caller's may be the legacy default stream,
+            // which cannot capture); the graph is then launched on the caller's stream
+            cudaGraph_t graph = nullptr;
+            const int64_t l0 = g_ft_launches;
+            if (!w.cap_stream) CK(cudaStreamCreateWithFlags(&w.cap_stream, cudaStreamNonBlocking));
+            int rc2 = 1;
+            cudaError_t ce = cudaStreamBeginCapture(w.cap_stream, cudaStreamCaptureModeThreadLocal);
+            if (ce == cudaSuccess) {
+                C.s = w.cap_stream;
+                rc2 = enqueue_start(C, dA, lda);
+                for (int t = 0; t < last && !rc2; t++) rc2 = enqueue_panel(C, t);
+                ce = cudaStreamEndCapture(w.cap_stream, &graph);
+                C.s = s;
+            }
+            cudaGraphExec_t exec = nullptr;
+            if (!rc2 && ce == cudaSuccess && graph && cudaGraphInstantiate(&exec, graph, 0) == cudaSuccess) {
+                it->second.exec = exec;
+                it->second.launches = g_ft_launches - l0;
+                g_ft_launches = l0;
+                CK(cudaGraphLaunch(exec, s));
+                g_ft_launches += it->second.launches;
+                launched = true;
+            } else {
+                g_ft_launches = l0;
+                cudaGetLastError();
+                it->second.failed = true;
+            }
+            if (graph) cudaGraphDestroy(graph);
+        } else {
+            g_graphs[key] = GraphEntry{};
+        }
+    }
+    if (!launched) {
+        rc = enqueue_start(C, dA, lda);
+        if (rc) return rc;
+    }
+    int t0 = launched ? last : 0, attempts = 0;
     info = 0;
     while (true) {
         for (int t = t0; t < last; t++) {
@@ -1083,6 +1171,7 @@ const char *ft_strerror(int info) {
 }
 
 void ft_finalize(void) {
+    for (auto &kv : g_work) drop_graphs(kv.first);
     for (auto &kv : g_work) {
         int cur = 0;
         cudaGetDevice(&cur);

@@ -119,6 +119,7 @@ struct YtopParams {
 cudaError_t ft_launch_ytop(const YtopParams &p, cudaStream_t s);
 
 // ABFT / utility kernels (ft_abft.cu)
+cudaError_t ft_ctl_init(FtCtl *ctl, double c_thr, cudaStream_t s);
 cudaError_t ft_copy_in(const double *A, int lda, double *Aw, int64_t ldw, int n, cudaStream_t s);
 cudaError_t ft_copy_out(const double *Aw, int64_t ldw, double *A, int lda, int n, cudaStream_t s);
 cudaError_t ft_encode(double *Aw, int64_t ldw, int n, FtCtl *ctl, double *scratch, double *linepart,

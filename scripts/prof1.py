@@ -24,6 +24,7 @@ def main():
     ap.add_argument("--abft", type=int, default=1)
     ap.add_argument("--probe", type=int, default=-1)
     ap.add_argument("--ablate", type=int, default=0)
+    ap.add_argument("--no-panel-timing", action="store_true", help="leave panel events off (CUDA graphs enabled)")
     a = ap.parse_args()
     import torch
 
@@ -49,7 +50,7 @@ def main():
     s = torch.cuda.current_stream()
     for it in range(a.reps):
         dA.copy_(dA0)
-        L.ft_debug_time_panels(1)
+        L.ft_debug_time_panels(0 if a.no_panel_timing else 1)
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(s)
         _, res = ft.dgehrd(dA, tau=tau, nb=a.nb, abft=bool(a.abft), stream=s)

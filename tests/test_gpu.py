@@ -97,6 +97,34 @@ def test_parity_c2_full_size():
     check_against_oracle(A, dA, tau, nb=32)
 
 
+@pytest.mark.parametrize("n,nb,abft", [(600, 32, True), (600, 32, False), (1100, 64, True)])
+def test_graph_replay(n, nb, abft):
+    """Repeated fault-free calls on the same buffers: the 2nd call captures a CUDA graph, later
+    calls replay it; every result must match the oracle, and a fault run on the same buffers
+    (direct launches) must still detect and correct."""
+    A = synth.matrix(n)
+    At = torch.from_numpy(A).cuda()
+    dA = ft.fortran(torch.empty((n, n), dtype=torch.float64, device="cuda"))
+    tau = torch.zeros(n, dtype=torch.float64, device="cuda")
+    Ho = None
+    for it in range(4):
+        dA.copy_(At)
+        _, res = ft.dgehrd(dA, tau=tau, nb=nb, abft=abft)
+        torch.cuda.synchronize()
+        assert res.info == 0 and res.report.detected == 0, (it, res.events)
+        H = np.triu(dA.cpu().numpy(), -1)
+        if Ho is None:
+            Ao, _ = oracle.dgehd2(A)
+            Ho = np.triu(Ao, -1)
+        assert rel(H, Ho) <= TOL, (it, rel(H, Ho))
+    if abft:
+        dA.copy_(At)
+        _, res = ft.dgehrd(dA, tau=tau, nb=nb, faults=[(1, ft.PHASE_BEFORE_PANEL, ft.SITE_A, n // 2, n // 2 + 9, 55)])
+        torch.cuda.synchronize()
+        assert res.info == 0 and any(e[0] == "FIX_DATA" for e in res.events), res.events
+        assert rel(np.triu(dA.cpu().numpy(), -1), Ho) <= TOL
+
+
 @pytest.mark.parametrize("policy", [ft.POLICY_EAGER, ft.POLICY_PAPER])
 def test_policies_fault_free(policy):
     A = synth.matrix(200, dist="normal")
