@@ -84,6 +84,11 @@ FT_DEV void cp_async16(void *smem, const void *gmem, int src_bytes) {
     unsigned s = (unsigned)__cvta_generic_to_shared(smem);
     asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(s), "l"(gmem), "r"(src_bytes) : "memory");
 }
+// 8-byte asynchronous global->shared copy (LDGSTS); src_bytes = 0 zero-fills
+FT_DEV void cp_async8(void *smem, const void *gmem, int src_bytes) {
+    unsigned s = (unsigned)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(s), "l"(gmem), "r"(src_bytes) : "memory");
+}
 FT_DEV void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
 template <int N>
 FT_DEV void cp_async_wait() {
@@ -123,6 +128,24 @@ FT_DEV void grid_barrier(unsigned *count, unsigned &epoch, unsigned nblocks) {
 
 // L2-coherent loads for data written by other CTAs inside the same launch
 FT_DEV double ldcg(const double *p) { return __ldcg(p); }
+
+// sum_{i < N} p[i * stride] (L2-coherent loads), eight loads in flight at a time; fixed
+// summation order for a given N (deterministic)
+FT_DEV double sum_strided(const double *p, int64_t stride, int N) {
+    double s0 = 0.0, s1 = 0.0, s2 = 0.0, s3 = 0.0;
+    int i = 0;
+    for (; i + 8 <= N; i += 8) {
+        double v[8];
+#pragma unroll
+        for (int u = 0; u < 8; u++) v[u] = __ldcg(p + (int64_t)(i + u) * stride);
+        s0 += v[0] + v[4];
+        s1 += v[1] + v[5];
+        s2 += v[2] + v[6];
+        s3 += v[3] + v[7];
+    }
+    for (; i < N; i++) s0 += __ldcg(p + (int64_t)i * stride);
+    return (s0 + s1) + (s2 + s3);
+}
 
 FT_DEV double warp_sum(double v) {
 #pragma unroll

@@ -114,9 +114,10 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_right(GemmRightParams p) {
     double *colp = p.A + (int64_t)(cb + (colok ? wcol : 0)) * p.lda;
 
     if (p.do_right) {  // V(cols, :) once per CTA (plain loads: cb may be odd)
-        for (int i = tid; i < KT * UB; i += UT) {
+        for (int i = tid; i < KT * UB; i += UT) {  // asynchronous: joins the first Ys group
             const int kk = i / UB, cc = i % UB;
-            S.Vc[kk][cc] = (kk < K && cc < ncols) ? __ldg(p.V + (cb + cc) + (int64_t)kk * p.ldw) : 0.0;
+            const bool ok = kk < K && cc < ncols;
+            cp_async8(&S.Vc[kk][cc], ok ? p.V + (cb + cc) + (int64_t)kk * p.ldw : p.V, ok ? 8 : 0);
         }
     }
     double wacc[NJ][2];
@@ -222,16 +223,18 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_right(GemmRightParams p) {
                 double(*Ws)[SK] = S.Ys;  // W as Ws[col][b] (64 x KT): spans Ys and Vr (contiguous)
                 for (int i = tid; i < KT * KT; i += UT) {
                     const int a = i % KT, b = i / KT;
-                    Ts[a][b] = (a < K && b < K) ? p.T[a + b * FT_NBMAX] : 0.0;
+                    const bool ok = a < K && b < K;
+                    cp_async8(&Ts[a][b], ok ? p.T + a + b * FT_NBMAX : p.T, ok ? 8 : 0);
                 }
+                cp_async_commit();
                 for (int i = tid; i < UB * KT; i += UT) {
                     const int cc = i / KT, b = i % KT;
                     double w = 0.0;
                     if (cc < ncols && b < K)
-                        for (int sp = 0; sp < (int)gridDim.y; sp++)
-                            w += __ldcg(p.Wpart + (int64_t)sp * p.wsplit_stride + (int64_t)(cb + cc) * FT_NBMAX + b);
+                        w = sum_strided(p.Wpart + (int64_t)(cb + cc) * FT_NBMAX + b, p.wsplit_stride, (int)gridDim.y);
                     Ws[cc][b] = w;
                 }
+                cp_async_wait<0>();
                 __syncthreads();
                 for (int i = tid; i < UB * KT; i += UT) {
                     const int cc = i / KT, a = i % KT;
@@ -326,8 +329,7 @@ __global__ void k_wprep(const double *__restrict__ Wpart, int64_t wstride, int n
     const int a = threadIdx.x % FT_NBMAX, cl = threadIdx.x / FT_NBMAX;
     const int col = c_lo + blockIdx.x * (blockDim.x / FT_NBMAX) + cl;
     double w = 0.0;
-    if (col < c_hi && a < K)
-        for (int sp = 0; sp < nsplit; sp++) w += Wpart[(int64_t)sp * wstride + (int64_t)col * FT_NBMAX + a];
+    if (col < c_hi && a < K) w = sum_strided(Wpart + (int64_t)col * FT_NBMAX + a, wstride, nsplit);
     Ws[cl][a] = w;
     __syncthreads();
     if (col >= c_hi || a >= K) return;
@@ -367,6 +369,12 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
     const int t0 = (int)((long long)blockIdx.y * nrt / gridDim.y);
     const int t1 = (int)((long long)(blockIdx.y + 1) * nrt / gridDim.y);
 
+    // W'^T for the strip: Wt [col][64] -> Wc[k][col] (asynchronous, with the first V tile)
+    for (int i = tid; i < KT * UB; i += UT) {
+        const int cc = i / KT, kk = i % KT;
+        const bool ok = kk < K && cc < ncols;
+        cp_async8(&S.Wc[kk][cc], ok ? p.Wpart + (int64_t)(cb + cc) * FT_NBMAX + kk : p.Wpart, ok ? 8 : 0);
+    }
     if (t0 < t1) issue_ktile<KT>(S.Vr[0], p.V, p.ldw, rbase + t0 * UB, p.r_hi, K);
     cp_async_commit();
     if (p.endcheck) {
@@ -375,16 +383,9 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
         const int k = p.r_lo - 1, e = p.c_lo;
         const int nb = gridDim.x * gridDim.y, b = blockIdx.y * gridDim.x + blockIdx.x;
         for (int i = b * UT + tid; i <= e && i < p.n; i += nb * UT) {
-            double s = 0.0;
-            for (int col = k; col < e; col++)
-                if (i <= col + 1) s += p.A[i + (int64_t)col * p.lda];
-            p.Fr[i] += s;
+            const int c0 = i - 1 > k ? i - 1 : k;  // columns col >= i - 1 hold row i's H entries
+            p.Fr[i] += c0 < e ? sum_strided(p.A + i + (int64_t)c0 * p.lda, p.lda, e - c0) : 0.0;
         }
-    }
-    // W'^T for the strip: Wt [col][64] -> Wc[k][col]
-    for (int i = tid; i < KT * UB; i += UT) {
-        const int cc = i / KT, kk = i % KT;
-        S.Wc[kk][cc] = (kk < K && cc < ncols) ? p.Wpart[(int64_t)(cb + cc) * FT_NBMAX + kk] : 0.0;
     }
     int cols[2];
     bool colok[2];
@@ -452,9 +453,12 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
     __threadfence();
     const int n = p.n;
     double sr = 0.0, sc = 0.0;
-    for (int i = tid; i < n; i += UT) {
-        sr += __ldcg(p.A + i + (int64_t)n * p.lda);
-        sc += __ldcg(p.A + n + (int64_t)i * p.lda);
+    {
+        const int per = (n + UT - 1) / UT, i0 = tid * per, cnt = min(per, n - i0);
+        if (cnt > 0) {
+            sr = sum_strided(p.A + i0 + (int64_t)n * p.lda, 1, cnt);
+            sc = sum_strided(p.A + n + (int64_t)i0 * p.lda, p.lda, cnt);
+        }
     }
     sr = warp_sum(sr);
     sc = warp_sum(sc);
@@ -535,9 +539,8 @@ cudaError_t ft_launch_gemm_left(const GemmLeftParams &p, cudaStream_t s) {
 #define YT_M 64
 #define YT_K 32
 struct YtopSmem {
-    double As[YT_K * (YT_M + 4)];        // A tile [col][row]
-    double Vs[FT_NBMAX * (YT_K + 4)];    // V [j][col]
-    double rsum[YT_M];
+    double As[2][YT_K * (YT_M + 4)];      // A tile [col][row], double-buffered
+    double Vs[2][FT_NBMAX * (YT_K + 4)];  // V [j][col]
 };
 
 __global__ void __launch_bounds__(128) k_ytop_partial(YtopParams p) {
@@ -558,28 +561,38 @@ __global__ void __launch_bounds__(128) k_ytop_partial(YtopParams p) {
 #pragma unroll
         for (int b = 0; b < 8; b++) acc[a][b][0] = acc[a][b][1] = 0.0;
     double rs = 0.0;
-    for (int kt = kt0; kt < kt1; kt++) {
+    // stage k-tile kt into buffer st with cp.async (every load in flight at once)
+    auto issue = [&](int kt, int st) {
         const int kc = K0 + kt * YT_K;
         const int nk = min(YT_K, K1 - kc);
-        __syncthreads();
         for (int i = threadIdx.x; i < YT_K * YT_M; i += blockDim.x) {
-            int m = i % YT_M, kk = i / YT_M;
-            double v = 0.0;
-            if (m < mrows && kk < nk) v = p.A[(m_lo + m) + (int64_t)(kc + kk) * p.ldw];
-            S.As[kk * (YT_M + 4) + m] = v;
+            const int m = i % YT_M, kk = i / YT_M;
+            const bool ok = m < mrows && kk < nk;
+            cp_async8(&S.As[st][kk * (YT_M + 4) + m], ok ? p.A + (m_lo + m) + (int64_t)(kc + kk) * p.ldw : p.A,
+                      ok ? 8 : 0);
         }
         for (int i = threadIdx.x; i < FT_NBMAX * YT_K; i += blockDim.x) {
-            int kk = i % YT_K, jj = i / YT_K;
-            double v = 0.0;
-            if (jj < ib && kk < nk) v = p.V[(kc + kk) + (int64_t)jj * p.ldw];
-            S.Vs[jj * (YT_K + 4) + kk] = v;
+            const int kk = i % YT_K, jj = i / YT_K;
+            const bool ok = jj < ib && kk < nk;
+            cp_async8(&S.Vs[st][jj * (YT_K + 4) + kk], ok ? p.V + (kc + kk) + (int64_t)jj * p.ldw : p.V, ok ? 8 : 0);
         }
+    };
+    if (kt0 < kt1) issue(kt0, 0);
+    cp_async_commit();
+    for (int kt = kt0; kt < kt1; kt++) {
+        const int st = (kt - kt0) & 1;
+        const int nk = min(YT_K, K1 - (K0 + kt * YT_K));
+        if (kt + 1 < kt1) issue(kt + 1, st ^ 1);
+        cp_async_commit();
+        cp_async_wait<1>();
         __syncthreads();
         if (p.verify && threadIdx.x < YT_M)
-            for (int kk = 0; kk < nk; kk++) rs += S.As[kk * (YT_M + 4) + threadIdx.x];
+            for (int kk = 0; kk < nk; kk++) rs += S.As[st][kk * (YT_M + 4) + threadIdx.x];
         // warp tile: rows warp*16..+16, cols 0..63 (MI=2, NI=8)
-        warp_mma<2, 8, true>(acc, S.As, YT_M + 4, S.Vs, YT_K + 4, warp * 16, 0, YT_K);
+        warp_mma<2, 8, true>(acc, S.As[st], YT_M + 4, S.Vs[st], YT_K + 4, warp * 16, 0, YT_K);
+        __syncthreads();  // buffer st is refilled by the next iteration's issue
     }
+    cp_async_wait<0>();
     double *yp = p.ypart + (int64_t)blockIdx.y * (int64_t)(p.k + 1) * FT_NBMAX;
 #pragma unroll
     for (int mi = 0; mi < 2; mi++)
@@ -610,8 +623,7 @@ __global__ void __launch_bounds__(YF_R * 64) k_ytop_finalize(YtopParams p) {
     }
     double acc = 0.0;
     if (row <= p.k && jb < ib)
-        for (int sp = 0; sp < p.nsplit; sp++)
-            acc += p.ypart[(int64_t)sp * (p.k + 1) * FT_NBMAX + (int64_t)row * FT_NBMAX + jb];
+        acc = sum_strided(p.ypart + (int64_t)row * FT_NBMAX + jb, (int64_t)(p.k + 1) * FT_NBMAX, p.nsplit);
     y0[rl][jb] = acc;
     __syncthreads();
     double yv = 0.0;
@@ -621,9 +633,9 @@ __global__ void __launch_bounds__(YF_R * 64) k_ytop_finalize(YtopParams p) {
     }
     if (p.verify && row <= p.k && jb == 0) {
         double rsum = 0.0;
-        for (int sp = 0; sp < p.nsplit; sp++) rsum += p.rowpart[(int64_t)sp * (p.k + 1) + row];
+        rsum = sum_strided(p.rowpart + row, p.k + 1, p.nsplit);
         rsum += p.A[row + (int64_t)p.k * p.ldw];
-        for (int col = p.ihi; col < p.n; col++) rsum += p.A[row + (int64_t)col * p.ldw];
+        if (p.ihi < p.n) rsum += sum_strided(p.A + row + (int64_t)p.ihi * p.ldw, p.ldw, p.n - p.ihi);
         double d = p.A[row + (int64_t)p.n * p.ldw] - p.Fr[row] - rsum;
         double tau_abs = p.ctl->c_thr * (double)p.n * 2.220446049250313e-16 * p.ctl->normF;
         if (not_within(d, tau_abs)) atomicAdd(&p.ctl->nflag, 1);

@@ -39,8 +39,7 @@
 #define GR 8          // row-group granularity (64 bytes of a column)
 #define VS 65         // shared-memory row stride of the V / Y row caches (doubles)
 #define RMAX PT       // max rows per CTA
-#define BAR_GO 1      // named barrier: b(c+2:ihi) is published, start the GEMV
-#define BAR_DONE 2    // named barrier: GEMV partials are in shared memory
+#define NSLOT (PT / 8)  // 8-lane groups per CTA (rows / outputs handled at once)
 #ifndef GB
 #define GB 8          // GEMV load batch (double2 of A + b per lane)
 #endif
@@ -70,27 +69,18 @@ struct PanelSmem {
 
 size_t ft_panel_smem_bytes() { return sizeof(PanelSmem); }
 
+// timing probes (debug hook): CTA 0's timestamps at dbg[j*16 + slot]; the max over CTAs of
+// the cycles since the CTA's previous probe at dbg[1024 + j*16 + slot]
 #define PROBE(slot)                                                                   \
     do {                                                                              \
-        if (p.dbg && blockIdx.x == 0 && lane == 0 && j < 64)                          \
-            p.dbg[j * 16 + (slot)] = clock64();                                       \
+        if (p.dbg && tid == 0 && j < 64) {                                            \
+            const long long now_ = clock64();                                         \
+            if (blockIdx.x == 0) p.dbg[j * 16 + (slot)] = now_;                       \
+            if ((slot) != 0)                                                          \
+                atomicMax(p.dbg + 1024 + j * 16 + (slot), (unsigned long long)(now_ - probe_last)); \
+            probe_last = now_;                                                        \
+        }                                                                             \
     } while (0)
-
-__device__ __forceinline__ void named_bar(int id) { asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(PT) : "memory"); }
-
-// grid barrier driven by one warp: lane 0 arrives (release) and polls (acquire); the
-// warp-level barriers order the other lanes' accesses around it
-__device__ __forceinline__ void warp_grid_barrier(unsigned *count, unsigned &epoch, unsigned nblocks) {
-    __syncwarp();
-    if ((threadIdx.x & 31) == 0) {
-        epoch += 1;
-        const unsigned target = epoch * nblocks;
-        red_release_add_u32(count, 1u);
-        while (ld_acquire_u32(count) < target) {
-        }
-    }
-    __syncwarp();
-}
 
 // DLARFG scalars (reading R1), out of line: one copy of the sqrt / division code
 struct Refl {
@@ -126,6 +116,14 @@ __device__ __forceinline__ double dotj(const double *X, int64_t cs, const double
     return (s0 + s1) + (s2 + s3);
 }
 
+// 8-lane group sum (lanes g = 0..7 of an aligned group); every lane of the warp must call it
+__device__ __forceinline__ double group8_sum(double v) {
+    v += __shfl_xor_sync(0xffffffffu, v, 4);
+    v += __shfl_xor_sync(0xffffffffu, v, 2);
+    v += __shfl_xor_sync(0xffffffffu, v, 1);
+    return v;
+}
+
 template <bool CACHE>
 __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
     if (p.ctl->halt) return;  // uniform for the whole grid (nobody writes halt in this launch)
@@ -133,6 +131,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
     PanelSmem &S = *reinterpret_cast<PanelSmem *>(smem_raw);
 
     const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+    const int slot = tid >> 3, g = tid & 7;  // 8-lane groups: NSLOT row / output slots
     const unsigned P = gridDim.x;
     const int g0 = (int)((long long)blockIdx.x * p.ngroups / P);
     const int g1 = (int)((long long)(blockIdx.x + 1) * p.ngroups / P);
@@ -150,8 +149,8 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
     constexpr int64_t XR = CACHE ? VS : 1;  // row stride
     const int64_t XC = CACHE ? 1 : ldw;     // column stride
 
-    // GEMV partial layout (shared by both roles): R2p lanes per column, a power of two
-    // when <= 32 so the lanes of one row pair are shuffle-reducible inside a warp
+    // GEMV partial layout: R2p lanes per column, a power of two when <= 32 so the lanes of
+    // one row pair are shuffle-reducible inside a warp
     int R2p = R2;
     if (R2 <= 32) {
         R2p = 1;
@@ -159,6 +158,83 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
     }
     const int ncl = (NGW * 32) / R2p;
     const int npart = R2p <= 32 ? NGW : ncl;  // partials per row pair
+
+    auto is_data = [&](int row) { return row >= k + 1 && row < ihi; };
+    auto is_valid = [&](int row) { return (row >= k + 1 && row < ihi) || (p.abft && row == n); };
+
+    // ---- CTA-parallel building blocks of the column chain --------------------------------
+    // row dot of row rl (an 8-lane group per row): sum_{jp < J} X(rl, jp) z[jp], J <= 64.
+    // Fully unrolled with predication: all operand loads are in flight at once.
+    auto rowdot = [&](const double *X, int rl, const double *z, int J) -> double {
+        double s0 = 0.0, s1 = 0.0;
+        if (rl < R) {
+            const double *x = X + rl * XR;
+#pragma unroll
+            for (int u = 0; u < FT_NBMAX / 8; u += 2) {
+                const int ja = g + 8 * u, jb = ja + 8;
+                if (ja < J) s0 += x[ja * XC] * z[ja];
+                if (jb < J) s1 += x[jb * XC] * z[jb];
+            }
+        }
+        return group8_sum(s0 + s1);
+    };
+    // column dots over the own rows, CTA partial added into the accumulators:
+    // out[o] = sum_rl X(rl, o) zr[rl] (o < J); extras: out[J] = zr.zr, out[J+1] = sum zr.
+    // An aligned group of LPO lanes per output (4..32: ~2 rows per lane, LPO * outputs <= PT),
+    // lanes stride the rows, shuffle tree inside the warp; the group leader adds the CTA
+    // partial into the accumulator.  No shared-memory pass, no CTA barrier.
+    auto coldot_add = [&](const double *X, const double *zr, int J, bool extras, double *acc, int acc_o0,
+                          int acc_extra0) {
+        const int NO = J + (extras ? 2 : 0);
+        // lanes per output: ~2 rows per lane, at most 32, at most PT / NO (a power of two)
+        int LPO = 4;
+        while (LPO < 32 && 2 * LPO < R && (2 * LPO) * NO <= PT) LPO *= 2;
+        const int o = tid / LPO, gl = tid & (LPO - 1);
+        if ((wid * 32) / LPO >= NO) return;  // warp without outputs (warp-uniform)
+        double s = 0.0;
+        if (o < NO) {
+            double s1 = 0.0;
+#pragma unroll 1
+            for (int rb = gl; rb < R; rb += 4 * LPO) {
+#pragma unroll
+                for (int u = 0; u < 4; u++) {
+                    const int rl = rb + u * LPO;
+                    if (rl < R) {
+                        const double z = zr[rl];
+                        const double t = (o < J ? X[rl * XR + o * XC] : (o == J ? z : 1.0)) * z;
+                        if (u & 1) s1 += t;
+                        else s += t;
+                    }
+                }
+            }
+            s += s1;
+        }
+#pragma unroll
+        for (int off = 16; off > 0; off >>= 1)
+            if (off < LPO) s += __shfl_xor_sync(0xffffffffu, s, off);
+        if (o < NO && gl == 0 && !(p.dbg_mode & 4)) {
+            const int dst = o < J ? acc_o0 + o : acc_extra0 + (o - J);
+            atomicAdd(acc + dst * FT_ACC_PAD, s);
+        }
+    };
+    // grid barrier: thread 0 arrives (release, cumulative over the CTA's writes ordered by the
+    // bar.sync) and polls (acquire); `after` runs in warp 0 right after the poll succeeds, so
+    // the control loads it issues are at the head of the SM's memory queue (ahead of the GEMV)
+    auto grid_sync = [&](unsigned &epoch, auto after) {
+        __syncthreads();
+        if (wid == 0) {
+            if (lane == 0 && !(p.dbg_mode & 1)) {
+                epoch += 1;
+                const unsigned target = epoch * P;
+                red_release_add_u32(p.bar, 1u);
+                while (ld_acquire_u32(p.bar) < target) {
+                }
+            }
+            __syncwarp();
+            after();
+        }
+        __syncthreads();
+    };
 
 #pragma unroll 1
     for (int i = tid; i < FT_NBMAX * (FT_NBMAX + 1); i += PT) (&S.Ts[0][0])[i] = 0.0;
@@ -171,12 +247,12 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
             const int rl = x % R, jj = x / R, row = r0 + rl;
             if (row < rend) p.ckpt[row + (int64_t)jj * ldw] = A[row + (int64_t)(k + jj) * ldw];
         }
-        const int gstride = (int)P * PT, g = blockIdx.x * PT + tid;
-        for (int x = g; x < p.rbase * ib; x += gstride) {
+        const int gstride = (int)P * PT, gi = blockIdx.x * PT + tid;
+        for (int x = gi; x < p.rbase * ib; x += gstride) {
             const int i = x % p.rbase, jj = x / p.rbase;
             p.ckpt[i + (int64_t)jj * ldw] = A[i + (int64_t)(k + jj) * ldw];
         }
-        for (int i = g; i <= n; i += gstride) {
+        for (int i = gi; i <= n; i += gstride) {
             p.ck_r[i] = A[i + (int64_t)n * ldw];
             p.ck_q[i] = p.Qr[i];
             p.ck_q[ldw + i] = p.Qc[i];
@@ -187,29 +263,120 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
     }
     for (int rl = tid; rl < R; rl += PT) {
         const int row = r0 + rl;
-        const bool valid = (row >= k + 1 && row < ihi) || (p.abft && row == n);
-        S.acol[rl] = valid ? A[row + (int64_t)k * ldw] : 0.0;
+        S.acol[rl] = is_valid(row) ? A[row + (int64_t)k * ldw] : 0.0;
     }
+    if (tid == 0 && blockIdx.x == 0) *p.bar_next = 0u;  // the next panel launch's counter
     __syncthreads();
 
-    if (wid > 0) {
-        // ======================= GEMV warps =============================================
-        const int gt = tid - 32;
-        const int rp = gt % R2p, cl = gt / R2p;
-        const bool gemv_on = rp < R2 && cl < ncl;
-        const double2 *__restrict__ A2 = reinterpret_cast<const double2 *>(A + r0);
-        const int64_t ldw2 = ldw >> 1;
-        const double *bv = p.bvec;  // b(q) for c+2 <= q < ihi; zero for q >= ihi
+    unsigned epoch = 0;
+    long long probe_last = 0;
+    double qc_corner = 0.0;  // corner of the Q checksums: sum of this panel's Qc (CTA 0, thread 0)
+    const double c_thr = p.ctl->c_thr;
+    const double tau_abs = c_thr * (double)n * 2.220446049250313e-16 * p.ctl->normF;
+
 #pragma unroll 1
-        for (int j = 0; j < ib; j++) {
-            const int c = k + j;
+    for (int j = 0; j < ib; j++) {
+        const int c = k + j;
+        double *acc = p.acc + (c & 3) * FT_ACC_SET_DOUBLES;  // accumulator i at acc[i * FT_ACC_PAD]
+        // A(row, c+1) of the own rows (thread = row): issued now, parked in smem before the GEMV
+        double an_reg = 0.0;
+        if (tid < R && is_valid(r0 + tid)) an_reg = A[(r0 + tid) + (int64_t)(c + 1) * ldw];
+        PROBE(0);
+        // ---------------- (i) b0 = A(:,c) - Y V(c,:)^T, s1 = V^T b0 ---------------------------
+        if (j > 0) {
+#pragma unroll 1
+            for (int base = 0; base < R; base += NSLOT) {
+                if (base + 4 * wid >= R) break;  // no rows for this warp (warp-uniform)
+                const int rl = base + slot;
+                const double yv = rowdot(Yl, rl, S.vrow, j);
+                if (rl < R && g == 0) {
+                    const double b0 = S.acol[rl] - yv;
+                    S.b0[rl] = b0;
+                    S.bm[rl] = is_data(r0 + rl) ? b0 : 0.0;
+                }
+            }
+            PROBE(10);
+            __syncthreads();
+            PROBE(11);
+            coldot_add(Vl, S.bm, j, false, acc, 0, 0);
+            PROBE(1);
+            grid_sync(epoch, [&]() {
+                if (lane < j) S.s1[lane] = ldcg(acc + lane * FT_ACC_PAD);
+                if (lane + 32 < j) S.s1[lane + 32] = ldcg(acc + (lane + 32) * FT_ACC_PAD);
+            });
+            PROBE(2);
+            // w = T^T s1 (an 8-lane group per output)
+            {
+                double s0 = 0.0, s1 = 0.0;
+                if (4 * wid < j) {
+                if (slot < j)
+#pragma unroll
+                    for (int u = 0; u < FT_NBMAX / 8; u += 2) {
+                        const int ba = g + 8 * u, bb = ba + 8;
+                        if (ba <= slot) s0 += S.Ts[ba][slot] * S.s1[ba];
+                        if (bb <= slot) s1 += S.Ts[bb][slot] * S.s1[bb];
+                    }
+                const double s = group8_sum(s0 + s1);
+                if (slot < j && g == 0) S.w[slot] = s;
+                }
+            }
+            __syncthreads();
+        }
+        // ---------------- (ii) b = b0 - V w; publish x = b(c+2:ihi) for the GEMV, alpha = b(c+1)
+        auto publish = [&](int rl, double b) {
+            const int row = r0 + rl;
+            const bool xrow = is_data(row) && row >= c + 2;
+            S.b0[rl] = b;
+            S.bm[rl] = xrow ? b : 0.0;
+            if (xrow) p.bvec[row] = b;
+            if (row == c + 1) acc[ACC_ALPHA * FT_ACC_PAD] = b;  // alpha: a single writer
+        };
+        if (j > 0) {
+#pragma unroll 1
+            for (int base = 0; base < R; base += NSLOT) {
+                if (base + 4 * wid >= R) break;
+                const int rl = base + slot;
+                const double vw = rowdot(Vl, rl, S.w, j);
+                if (rl < R && g == 0) publish(rl, S.b0[rl] - vw);
+            }
+        } else {
+            for (int rl = tid; rl < R; rl += PT) publish(rl, S.acol[rl]);
+        }
+        __syncthreads();
+        PROBE(3);
+        coldot_add(Vl, S.bm, j, true, acc, ACC_VTB, ACC_NRM);
+        if (tid < R) S.anext[tid] = an_reg;
+        PROBE(4);
+        // control scalars of DLARFG, loaded by warp 0 as soon as the barrier opens
+        double nrm2 = 0.0, sx = 0.0, alpha = 0.0, vn0 = 0.0, vt0 = 0.0, vn1 = 0.0, vt1 = 0.0;
+        grid_sync(epoch, [&]() {
+            nrm2 = ldcg(acc + ACC_NRM * FT_ACC_PAD);
+            sx = ldcg(acc + ACC_SX * FT_ACC_PAD);
+            alpha = ldcg(acc + ACC_ALPHA * FT_ACC_PAD);
+            if (lane < j) {
+                vn0 = ldcg(V + (c + 1) + (int64_t)lane * ldw);
+                vt0 = ldcg(acc + (ACC_VTB + lane) * FT_ACC_PAD);
+            }
+            if (lane + 32 < j) {
+                vn1 = ldcg(V + (c + 1) + (int64_t)(lane + 32) * ldw);
+                vt1 = ldcg(acc + (ACC_VTB + lane + 32) * FT_ACC_PAD);
+            }
+        });
+        PROBE(5);
+        if (wid > 0) {
+            // ======================= GEMV warps: y = A(:, c+1:) v on the unscaled b ===========
+            const int gt = tid - 32;
+            const int rp = gt % R2p, cl = gt / R2p;
+            const bool gemv_on = rp < R2 && cl < ncl;
+            const double2 *__restrict__ A2 = reinterpret_cast<const double2 *>(A + r0);
+            const int64_t ldw2 = ldw >> 1;
+            const double *bv = p.bvec;  // b(q) for c+2 <= q < ihi; zero for q >= ihi
             const bool vfy = (j == 0) && p.verify;
             const int cend = vfy ? n : ihi;
-            named_bar(BAR_GO);
             double2 ya = make_double2(0.0, 0.0), rs = make_double2(0.0, 0.0);
             if (gemv_on && !(p.dbg_mode & 2)) {
-                // b is read with plain (L1-allocating) loads: the control warp's acquire at
-                // sync #2 invalidated this SM's L1 (CCTL.IVALL) before BAR_GO released us
+                // b is read with plain (L1-allocating) loads: the acquire at the grid barrier
+                // invalidated this SM's L1 before the trailing bar.sync released us
                 int col = c + 2 + cl;
 #pragma unroll 1
                 for (; col + (GB - 1) * ncl < cend; col += GB * ncl) {
@@ -229,14 +396,22 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
                         rs.y += a[u].y;
                     }
                 }
-#pragma unroll 1
-                for (; col < cend; col += ncl) {
-                    const double2 a = A2[(int64_t)col * ldw2 + rp];
-                    const double v = bv[col];
-                    ya.x += a.x * v;
-                    ya.y += a.y * v;
-                    rs.x += a.x;
-                    rs.y += a.y;
+                if (col < cend) {  // ragged tail: one predicated batch (all loads in flight together)
+                    double2 a[GB];
+                    double v[GB];
+#pragma unroll
+                    for (int u = 0; u < GB; u++) {
+                        const int q = col + u * ncl;
+                        a[u] = q < cend ? A2[(int64_t)q * ldw2 + rp] : make_double2(0.0, 0.0);
+                        v[u] = q < cend ? bv[q] : 0.0;
+                    }
+#pragma unroll
+                    for (int u = 0; u < GB; u++) {
+                        ya.x += a[u].x * v[u];
+                        ya.y += a[u].y * v[u];
+                        rs.x += a[u].x;
+                        rs.y += a[u].y;
+                    }
                 }
             }
             if (R2p <= 32) {
@@ -258,99 +433,8 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
                 S.red[cl * R2p + rp] = ya;
                 if (vfy) S.rsr[cl * R2p + rp] = rs;
             }
-            named_bar(BAR_DONE);
-        }
-        return;
-    }
-
-    // ======================= control warp =================================================
-    unsigned epoch = 0;
-    if (blockIdx.x == 0 && lane == 0) *p.bar_next = 0u;  // the next panel launch's counter
-    const double c_thr = p.ctl->c_thr;
-    const double tau_abs = c_thr * (double)n * 2.220446049250313e-16 * p.ctl->normF;
-    auto is_data = [&](int row) { return row >= k + 1 && row < ihi; };
-    auto is_valid = [&](int row) { return (row >= k + 1 && row < ihi) || (p.abft && row == n); };
-
-#pragma unroll 1
-    for (int j = 0; j < ib; j++) {
-        const int c = k + j;
-        double *acc = p.acc + (c & 3) * FT_ACC_SET_DOUBLES;  // accumulator i at acc[i * FT_ACC_PAD]
-        // A(row, c+1) of the first two row chunks: issued now, consumed after the GEMV
-        double an0 = 0.0, an1 = 0.0;
-        if (lane < R && is_valid(r0 + lane)) an0 = A[(r0 + lane) + (int64_t)(c + 1) * ldw];
-        if (lane + 32 < R && is_valid(r0 + lane + 32)) an1 = A[(r0 + lane + 32) + (int64_t)(c + 1) * ldw];
-        PROBE(0);
-        // ---------------- (i) b0 = A(:,c) - Y V(c,:)^T, s1 = V^T b0 -----------------------
-        if (j > 0) {
-#pragma unroll 1
-            for (int rl = lane; rl < R; rl += 32) {
-                const double b0 = S.acol[rl] - dotj(Yl + rl * XR, XC, S.vrow, j);
-                S.b0[rl] = b0;
-                S.bm[rl] = is_data(r0 + rl) ? b0 : 0.0;
-            }
-            __syncwarp();
-#pragma unroll 1
-            for (int o = lane; o < j; o += 32) {
-                const double s = dotj(Vl + o * XC, XR, S.bm, R);
-                if (!(p.dbg_mode & 4)) atomicAdd(acc + o * FT_ACC_PAD, s);
-            }
-            PROBE(1);
-            if (!(p.dbg_mode & 1)) warp_grid_barrier(p.bar, epoch, P);
-            PROBE(2);
-            // w = T^T s1
-            if (lane < j) S.s1[lane] = ldcg(acc + lane * FT_ACC_PAD);
-            if (lane + 32 < j) S.s1[lane + 32] = ldcg(acc + (lane + 32) * FT_ACC_PAD);
-            __syncwarp();
-#pragma unroll 1
-            for (int a = lane; a < j; a += 32) S.w[a] = dotj(&S.Ts[0][a], FT_NBMAX + 1, S.s1, a + 1);
-            __syncwarp();
-            // ---------------- (ii) b = b0 - V w ---------------------------------------------
-#pragma unroll 1
-            for (int rl = lane; rl < R; rl += 32) S.b0[rl] -= dotj(Vl + rl * XR, XC, S.w, j);
         } else {
-#pragma unroll 1
-            for (int rl = lane; rl < R; rl += 32) S.b0[rl] = S.acol[rl];
-        }
-        PROBE(3);
-        // publish x = b(c+2:ihi) for the GEMV, alpha = b(c+1); column dots of x
-#pragma unroll 1
-        for (int rl = lane; rl < R; rl += 32) {
-            const int row = r0 + rl;
-            const double b = S.b0[rl];
-            const bool xrow = is_data(row) && row >= c + 2;
-            S.bm[rl] = xrow ? b : 0.0;
-            if (xrow) p.bvec[row] = b;
-            if (row == c + 1) acc[ACC_ALPHA * FT_ACC_PAD] = b;  // alpha: a single writer
-        }
-        __syncwarp();
-#pragma unroll 1
-        for (int o = lane; o < j + 2; o += 32) {
-            double s;
-            if (o < j) s = dotj(Vl + o * XC, XR, S.bm, R);
-            else if (o == j) s = dotj(S.bm, 1, S.bm, R);
-            else {
-                s = 0.0;
-                for (int rl = 0; rl < R; rl++) s += S.bm[rl];
-            }
-            if (!(p.dbg_mode & 4)) atomicAdd(acc + (o < j ? ACC_VTB + o : (o == j ? ACC_NRM : ACC_SX)) * FT_ACC_PAD, s);
-        }
-        PROBE(4);
-        if (!(p.dbg_mode & 1)) warp_grid_barrier(p.bar, epoch, P);
-        PROBE(5);
-        named_bar(BAR_GO);  // the GEMV warps start on the unscaled b
-        // ---------------- (iii) DLARFG (reading R1), concurrent with the GEMV ---------------
-        {
-            const double nrm2 = ldcg(acc + ACC_NRM * FT_ACC_PAD), sx = ldcg(acc + ACC_SX * FT_ACC_PAD),
-                         alpha = ldcg(acc + ACC_ALPHA * FT_ACC_PAD);
-            double vn0 = 0.0, vt0 = 0.0, vn1 = 0.0, vt1 = 0.0;
-            if (lane < j) {
-                vn0 = ldcg(V + (c + 1) + (int64_t)lane * ldw);
-                vt0 = ldcg(acc + (ACC_VTB + lane) * FT_ACC_PAD);
-            }
-            if (lane + 32 < j) {
-                vn1 = ldcg(V + (c + 1) + (int64_t)(lane + 32) * ldw);
-                vt1 = ldcg(acc + (ACC_VTB + lane + 32) * FT_ACC_PAD);
-            }
+            // ======================= control warp: (iii) DLARFG (R1), V(:, j) ================
             const Refl rf = dlarfg_scalars(nrm2, alpha, c + 2 >= ihi);
             const double tau = rf.tau, beta = rf.beta, scale = rf.scale;
             const double vchk = 1.0 + scale * sx;  // V_chk(j) = e^T v
@@ -368,11 +452,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
                 S.scal[0] = tau;
                 S.scal[2] = scale;
             }
-            __syncwarp();
-            // T(a, j) = -tau * sum_{b=a}^{j-1} T(a, b) t(b), T(j, j) = tau
-#pragma unroll 1
-            for (int a = lane; a < j; a += 32) S.Ts[a][j] = -tau * dotj(&S.Ts[a][a], 1, S.t + a, j - a);
-            if (lane == 0) S.Ts[j][j] = tau;
+            PROBE(9);
             // V(:, j) and the reduced column c of the own rows
 #pragma unroll 1
             for (int rl = lane; rl < R; rl += 32) {
@@ -404,73 +484,98 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
             if (blockIdx.x == 0 && lane == 0) {
                 p.tau[c] = tau;
                 if (p.abft) {
-                    p.Qc[c] = vchk - 1.0;   // Q column checksum
-                    p.Qc[n] += vchk - 1.0;  // corner of the Q checksums
+                    p.Qc[c] = vchk - 1.0;  // Q column checksum
+                    qc_corner += vchk - 1.0;
                 }
             }
             // recycle the accumulator set of column c+2 (= that of column c-2): every CTA has
             // finished reading it, and column c+2 adds into it only after two more syncs
             if (blockIdx.x == 0)
                 for (int i = lane; i < FT_ACC_STRIDE; i += 32) p.acc[((c + 2) & 3) * FT_ACC_SET_DOUBLES + i * FT_ACC_PAD] = 0.0;
-            if (lane < R) S.anext[lane] = an0;
-            if (lane + 32 < R) S.anext[lane + 32] = an1;
-            for (int rl = lane + 64; rl < R; rl += 32)
-                S.anext[rl] = is_valid(r0 + rl) ? A[(r0 + rl) + (int64_t)(c + 1) * ldw] : 0.0;
+            PROBE(6);
         }
-        PROBE(6);
-        named_bar(BAR_DONE);  // GEMV partials ready
+        __syncthreads();  // GEMV partials, tau / scale / t, V(:, j) are in shared memory
         PROBE(7);
-        // ---------------- (v) Y(:, j) = tau (y - Y t) ----------------------------------------
+        // ---------------- (v) Y(:, j) = tau (y - Y t) (an 8-lane group per row) -----------------
         {
             const double tau = S.scal[0], scale = S.scal[2];
             const bool vfy = (j == 0) && p.verify;
-#pragma unroll 1
-            for (int rl = lane; rl < R; rl += 32) {
-                const int row = r0 + rl;
-                const double an = S.anext[rl];
-                if (is_valid(row)) {
-                    const int pr = rl >> 1;
-                    double y0 = 0.0, y1 = 0.0;
-                    int q = 0;
-#pragma unroll 1
-                    for (; q + 1 < npart; q += 2) {
-                        const double2 u0 = S.red[q * R2p + pr], u1 = S.red[(q + 1) * R2p + pr];
-                        y0 += (rl & 1) ? u0.y : u0.x;
-                        y1 += (rl & 1) ? u1.y : u1.x;
+            {   // T(a, j) = -tau * sum_{b=a}^{j-1} T(a, b) t(b), T(j, j) = tau (8 lanes per a)
+                double s0 = 0.0, s1 = 0.0;
+                if (4 * wid < j) {
+                if (slot < j)
+#pragma unroll
+                    for (int u = 0; u < FT_NBMAX / 8; u += 2) {
+                        const int ba = slot + g + 8 * u, bb = ba + 8;
+                        if (ba < j) s0 += S.Ts[slot][ba] * S.t[ba];
+                        if (bb < j) s1 += S.Ts[slot][bb] * S.t[bb];
                     }
-                    if (q < npart) {
-                        const double2 u0 = S.red[q * R2p + pr];
-                        y0 += (rl & 1) ? u0.y : u0.x;
+                const double s = group8_sum(s0 + s1);
+                if (slot < j && g == 0) S.Ts[slot][j] = -tau * s;
+                }
+                if (tid == 0) S.Ts[j][j] = tau;
+            }
+            PROBE(12);
+#pragma unroll 1
+            for (int base = 0; base < R; base += NSLOT) {
+                if (base + 4 * wid >= R) break;
+                const int rl = base + slot;
+                const bool on = rl < R && is_valid(r0 + rl);
+                const int pr = rl >> 1, hi = rl & 1;
+                // lane partial of scale * y - Y(rl, :) t: GEMV partials q = g, g + 8 (npart <= 15)
+                double ya = 0.0, yb = 0.0, rsum = 0.0;
+                if (on) {
+#pragma unroll
+                    for (int u = 0; u < 2; u++) {
+                        const int q = g + 8 * u;
+                        if (q < npart) {
+                            const double2 w2 = S.red[q * R2p + pr];
+                            ya += scale * (hi ? w2.y : w2.x);
+                            if (vfy) {
+                                const double2 r2 = S.rsr[q * R2p + pr];
+                                rsum += hi ? r2.y : r2.x;
+                            }
+                        }
                     }
-                    const double yy = tau * (an + scale * (y0 + y1) - dotj(Yl + rl * XR, XC, S.t, j));
-                    Y[row + (int64_t)j * ldw] = yy;
-                    if (CACHE) Yl[rl * XR + j * XC] = yy;
-                    if (vfy && is_data(row)) {
-                        // D_r(row) = r(row) - sum_{col >= k} L(row, col); columns < k are logical zero
-                        double rsum = 0.0;
-                        for (int q2 = 0; q2 < npart; q2++) {
-                            const double2 u = S.rsr[q2 * R2p + pr];
-                            rsum += (rl & 1) ? u.y : u.x;
-                        }
-                        rsum += S.acol[rl] + an;
-                        const double d = A[row + (int64_t)n * ldw] - rsum;
-                        if (not_within(d, tau_abs)) {
-                            atomicAdd(&p.ctl->nflag, 1);
-                        } else if (tau_abs > 0.0) {
-                            const double rel = fabs(d) / (tau_abs / c_thr);
-                            atomicMax(&p.ctl->drift_bits, (unsigned long long)__double_as_longlong(rel));
-                        }
+#pragma unroll
+                    for (int u = 0; u < FT_NBMAX / 8; u += 2) {
+                        const int ja = g + 8 * u, jb = ja + 8;
+                        if (ja < j) ya -= Yl[rl * XR + ja * XC] * S.t[ja];
+                        if (jb < j) yb -= Yl[rl * XR + jb * XC] * S.t[jb];
                     }
                 }
-                S.acol[rl] = an;
+                const double ysum = group8_sum(ya + yb);
+                if (vfy) rsum = group8_sum(rsum);
+                if (rl < R && g == 0) {
+                    const int row = r0 + rl;
+                    const double an = S.anext[rl];
+                    if (on) {
+                        const double yy = tau * (an + ysum);
+                        Y[row + (int64_t)j * ldw] = yy;
+                        if (CACHE) Yl[rl * XR + j * XC] = yy;
+                        if (vfy && is_data(row)) {
+                            // D_r(row) = r(row) - sum_{col >= k} L(row, col); columns < k are logical zero
+                            rsum += S.acol[rl] + an;
+                            const double d = A[row + (int64_t)n * ldw] - rsum;
+                            if (not_within(d, tau_abs)) {
+                                atomicAdd(&p.ctl->nflag, 1);
+                            } else if (tau_abs > 0.0) {
+                                const double rel = fabs(d) / (tau_abs / c_thr);
+                                atomicMax(&p.ctl->drift_bits, (unsigned long long)__double_as_longlong(rel));
+                            }
+                        }
+                    }
+                    S.acol[rl] = an;
+                }
             }
-            __syncwarp();
+            PROBE(13);
+            __syncthreads();
         }
         PROBE(8);
     }
     // Q row checksums of the new Householder vectors (Fig. 5): own data rows
     if (p.abft)
-        for (int rl = lane; rl < R; rl += 32) {
+        for (int rl = tid; rl < R; rl += PT) {
             const int row = r0 + rl;
             if (!is_data(row)) continue;
             double s = 0.0;
@@ -478,19 +583,17 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
                 if (row >= k + jj + 2) s += Vl[rl * XR + jj * XC];
             p.Qr[row] += s;
         }
-    if (p.precheck_sums)  // e^T Y, e^T V over the own data rows (pre-update check R15, fused)
-        for (int jj = lane; jj < ib; jj += 32) {
-            double sy = 0.0, sv = 0.0;
-            for (int rl = 0; rl < R; rl++)
-                if (is_data(r0 + rl)) {
-                    sy += Yl[rl * XR + jj * XC];
-                    sv += Vl[rl * XR + jj * XC];
-                }
-            atomicAdd(&p.ctl->eY[jj], sy);
-            atomicAdd(&p.ctl->eV[jj], sv);
-        }
+    if (p.precheck_sums && tid < 2 * ib) {  // e^T Y, e^T V over the own data rows (pre-update check R15, fused)
+        const int jj = tid % ib;
+        const double *X = tid < ib ? Yl : Vl;
+        double s = 0.0;
+        for (int rl = 0; rl < R; rl++)
+            if (is_data(r0 + rl)) s += X[rl * XR + jj * XC];
+        atomicAdd(tid < ib ? &p.ctl->eY[jj] : &p.ctl->eV[jj], s);
+    }
+    if (blockIdx.x == 0 && tid == 0 && p.abft) p.Qc[n] += qc_corner;
     if (blockIdx.x == 0)
-        for (int i = lane; i < ib * ib; i += 32) {
+        for (int i = tid; i < ib * ib; i += PT) {
             int a = i % ib, bb = i / ib;
             p.T[a + bb * FT_NBMAX] = S.Ts[a][bb];
         }

@@ -64,9 +64,10 @@ def main():
               f"{10 / 3 * n ** 3 / ms / 1e6:.1f} Gflop/s", flush=True)
     if dbg is not None:
         d = dbg.cpu().numpy()
-        names = {0: "start", 1: "s1_dots", 2: "sync1", 3: "w_b", 4: "x_dots", 5: "sync2", 6: "cw_dlarfg_T_V",
-                 7: "gemv_wait", 8: "y_step"}
-        order = [0, 1, 2, 3, 4, 5, 6, 7, 8]
+        names = {0: "start", 10: "b0_rowdot", 11: "b0_bar", 1: "s1_coldot", 2: "sync1", 3: "w_b", 4: "x_dots",
+                 5: "sync2", 9: "cw_dlarfg", 6: "cw_V_stores", 7: "gemv_wait", 12: "T_col", 13: "y_rows",
+                 8: "y_bar"}
+        order = [0, 10, 11, 1, 2, 3, 4, 5, 9, 6, 7, 12, 13, 8]
         tot = {}
         ncol = 0
         for j in range(64):
@@ -80,9 +81,16 @@ def main():
                     continue
                 tot[names[sl]] = tot.get(names[sl], 0) + (row[sl] - prev)
                 prev = row[sl]
-        print(f"probe panel {a.probe}: {ncol} columns, mean cycles per column by phase:")
+        mx = {}
+        for j in range(64):
+            row = d[1024 + j * 16: 1024 + j * 16 + 16]
+            for sl in order[1:]:
+                if row[sl] > 0:
+                    mx[names[sl]] = mx.get(names[sl], 0) + row[sl]
+        print(f"probe panel {a.probe}: {ncol} columns, mean cycles per column by phase "
+              f"(CTA 0 | max over CTAs of the phase):")
         for k2, v in tot.items():
-            print(f"  {k2:10s} {v / max(ncol, 1):10.0f}")
+            print(f"  {k2:12s} {v / max(ncol, 1):10.0f} {mx.get(k2, 0) / max(ncol, 1):10.0f}")
 
 
 if __name__ == "__main__":
