@@ -123,12 +123,44 @@ int ft_dgehrd_host(int n, int ilo, int ihi, double *hA, int lda, double *htau, c
 int ft_dorghr(int n, int ilo, int ihi, const double *dA, int lda, const double *dtau,
               double *dQ, int ldq, const ft_opts *opts);
 
-/* Multi-GPU entry (1-D block-column cyclic, block = nb): global column J lives on
- * rank (J/nb) mod nranks at local column (J/(nb*nranks))*nb + J mod nb; each rank
- * passes its n x ncols_local slab.  nccl_comm is an ncclComm_t (or NULL with
- * nranks == 1).  tau is replicated on return.  (Round 1: nranks == 1 only.) */
+/* ---------------------------------------------------------------------------------
+ * Multi-GPU reduction (the north star's "1-D block-column cyclic across
+ * 2/4/8 B200").  Layout: global column J (0-based) lives on rank (J / nb) mod nranks at
+ * local column (J / (nb * nranks)) * nb + J mod nb, nb = opts->nb (0 -> 32 if n < 4096
+ * else 64); each rank passes its n x ncols_local slab (column-major, lda_local >= n).
+ * Every rank runs the DLAHR2 panel redundantly on a broadcast copy of the panel columns;
+ * the trailing GEMV of every column covers only the rank's own columns and its partial
+ * sums are exchanged CTA by CTA through peer memory inside the persistent panel kernel
+ * (no host collective per column); Y_top is a per-rank partial summed by a peer
+ * allreduce; the block-reflector updates are rank-local.  tau is replicated on return.
+ * Round-1 scope: ilo = 1, ihi = n, no fault plan, no stop hook (-7 otherwise); with
+ * abft = 1 the checksums ride through every update and the finished H is verified
+ * against them at the end -- report->detected counts flagged rows/columns,
+ * report->max_drift_rel the largest discrepancy in units of n eps ||A||_F; correction
+ * and rollback run on the single-GPU entry only.
+ *
+ * Bootstrap (one process per GPU): ft_mgpu_setup allocates this rank's workspace,
+ * including a peer-visible region, for matrices up to n_max and returns its CUDA IPC
+ * handle; the caller all-gathers the handles (e.g. torch.distributed) and passes them to
+ * ft_mgpu_connect, which maps every peer's region.  Errors: -9 bad rank / nranks /
+ * call order, FT_E_CUDA / FT_E_NOMEM as for ft_dgehrd.  All ranks must issue the same
+ * sequence of ft_dgehrd_mgpu calls (same n, nb, abft). */
+typedef struct { char bytes[64]; } ft_ipc_handle;
+int ft_mgpu_setup(int n_max, int rank, int nranks, ft_ipc_handle *handle_out);
+int ft_mgpu_connect(const ft_ipc_handle *handles, int rank, int nranks);
 int ft_dgehrd_mgpu(int n, int ilo, int ihi, double *dA_local, int lda_local, double *dtau,
-                   void *nccl_comm, int rank, int nranks, const ft_opts *opts);
+                   int rank, int nranks, const ft_opts *opts);
+
+/* The same sharded reduction with nranks VIRTUAL ranks on the current GPU (one process):
+ * dA_local[q] / dtau[q] are rank q's slab and tau (device pointers, q < nranks <= 8).
+ * Identical kernels and exchange protocol; the ranks' CTA groups share one cooperative
+ * launch and reach each other's buffers through plain device pointers.  Used to test and
+ * measure the multi-GPU path on one GPU. */
+int ft_dgehrd_vranks(int n, int ilo, int ihi, double *const *dA_local, int lda_local,
+                     double *const *dtau, int nranks, const ft_opts *opts);
+
+/* Release the multi-rank workspaces (virtual ranks and this process's rank). */
+void ft_mgpu_finalize(void);
 
 /* Human-readable text for an info code. */
 const char *ft_strerror(int info);

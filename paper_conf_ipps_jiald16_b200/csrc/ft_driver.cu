@@ -1144,13 +1144,6 @@ int ft_dorghr(int n, int ilo, int ihi, const double *dA, int lda, const double *
     return 0;
 }
 
-int ft_dgehrd_mgpu(int n, int ilo, int ihi, double *dA_local, int lda_local, double *dtau, void *nccl_comm,
-                   int rank, int nranks, const ft_opts *opts) {
-    if (nranks < 1 || rank < 0 || rank >= nranks) return -9;
-    if (nranks == 1) return ft_dgehrd(n, ilo, ihi, dA_local, lda_local, dtau, opts);
-    return -9;  // multi-rank distribution not built in this round ("Multi-GPU")
-}
-
 const char *ft_strerror(int info) {
     switch (info) {
     case 0: return "success";
@@ -1161,7 +1154,7 @@ const char *ft_strerror(int info) {
     default: break;
     }
     if (info < 0) {
-        static const char *args[] = {"", "n", "ilo", "ihi", "A", "lda", "tau", "opts", "Q", "ldq"};
+        static const char *args[] = {"", "n", "ilo", "ihi", "A", "lda", "tau", "opts", "Q / rank", "ldq / nranks"};
         static char buf[64];
         int a = -info;
         snprintf(buf, sizeof(buf), "illegal value of argument %d (%s)", a, a < 10 ? args[a] : "?");
@@ -1171,6 +1164,7 @@ const char *ft_strerror(int info) {
 }
 
 void ft_finalize(void) {
+    ft_mgpu_finalize();
     for (auto &kv : g_work) drop_graphs(kv.first);
     for (auto &kv : g_work) {
         int cur = 0;

@@ -117,7 +117,8 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_right(GemmRightParams p) {
         for (int i = tid; i < KT * UB; i += UT) {  // asynchronous: joins the first Ys group
             const int kk = i / UB, cc = i % UB;
             const bool ok = kk < K && cc < ncols;
-            cp_async8(&S.Vc[kk][cc], ok ? p.V + (cb + cc) + (int64_t)kk * p.ldw : p.V, ok ? 8 : 0);
+            const int vrow = ft_cmap(cb + cc, p.cm_G, p.cm_rank, p.cm_nb, p.cm_ncl, p.cm_n);
+            cp_async8(&S.Vc[kk][cc], ok ? p.V + vrow + (int64_t)kk * p.ldw : p.V, ok ? 8 : 0);
         }
     }
     double wacc[NJ][2];
@@ -550,7 +551,8 @@ __global__ void __launch_bounds__(128) k_ytop_partial(YtopParams p) {
     const int warp = threadIdx.x >> 5;
     const int m_lo = blockIdx.x * YT_M;
     const int mrows = min(YT_M, p.k + 1 - m_lo);
-    const int K0 = p.k + 1, K1 = p.ihi;  // inner range
+    const bool mg = p.cm_G > 1;
+    const int K0 = mg ? p.kc0 : p.k + 1, K1 = mg ? p.kc1 : p.ihi;  // inner range (local columns)
     const int nkt = (K1 - K0 + YT_K - 1) / YT_K;
     const int kt0 = (int)((long long)blockIdx.y * nkt / gridDim.y);
     const int kt1 = (int)((long long)(blockIdx.y + 1) * nkt / gridDim.y);
@@ -574,7 +576,8 @@ __global__ void __launch_bounds__(128) k_ytop_partial(YtopParams p) {
         for (int i = threadIdx.x; i < FT_NBMAX * YT_K; i += blockDim.x) {
             const int kk = i % YT_K, jj = i / YT_K;
             const bool ok = jj < ib && kk < nk;
-            cp_async8(&S.Vs[st][jj * (YT_K + 4) + kk], ok ? p.V + (kc + kk) + (int64_t)jj * p.ldw : p.V, ok ? 8 : 0);
+            const int vrow = mg ? ft_cmap(kc + kk, p.cm_G, p.cm_rank, p.cm_nb, p.cm_ncl, -1) : kc + kk;
+            cp_async8(&S.Vs[st][jj * (YT_K + 4) + kk], ok ? p.V + vrow + (int64_t)jj * p.ldw : p.V, ok ? 8 : 0);
         }
     };
     if (kt0 < kt1) issue(kt0, 0);

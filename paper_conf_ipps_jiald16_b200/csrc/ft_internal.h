@@ -7,6 +7,8 @@
 #include "../../include/ftgehrd.h"
 
 #define FT_MAXFAULTS 64
+#define FT_MAX_VRANKS 8      // ranks per multi-rank launch (virtual ranks on one GPU) / max ranks
+#define FT_FLAG_STRIDE 256   // per-rank stride of the exchange flag arrays (>= CTAs per rank)
 #ifndef FT_NBMAX
 #define FT_NBMAX 64
 #endif
@@ -50,10 +52,31 @@ struct PanelParams {
     int precheck_sums;  // add e^T Y, e^T V of the own rows into ctl->eY / eV (fused pre-update check)
     unsigned long long *dbg;          // optional per-column phase timestamps (CTA 0), or NULL
     int dbg_mode;                     // timing ablations (wrong results): 1 no grid barriers, 2 no GEMV, 4 no atomics
+    // panel columns: Apan[row + c * ldw] is panel column c (k <= c < k + ib); == A on one GPU.
+    // rcol: the row-checksum column r.
+    double *Apan, *rcol;
+    // multi-rank mode (1-D block-column cyclic); G == 1 on one GPU.  A is the
+    // rank's local slab: local column l holds global column J(l) = (l / cbnb) G cbnb +
+    // rank cbnb + l % cbnb.  The trailing GEMV covers the panel columns (owner only, from
+    // Apan) and the local columns [lcol0, lcol1) (global >= e); the per-column GEMV
+    // partials are exchanged through peer memory, CTA by CTA (no collective, no host).
+    int G, rank, cbnb, owner, lcol0, lcol1, e;
+    double2 *yx;                     // own exchange slots [2][G][ldw]: (y partial, A(:, c+1) part)
+    double2 *ypeer[FT_MAX_VRANKS];   // every rank's slot base (index = rank; own included)
+    unsigned *flags;                 // own arrival flags [G][FT_FLAG_STRIDE]
+    unsigned *fpeer[FT_MAX_VRANKS];  // every rank's flag array
+    unsigned seq0;                   // flag value of column c is seq0 + c + 1
+};
+// A multi-rank launch: nr ranks (virtual ranks sharing this GPU, or 1 per GPU), each a
+// group of gridDim.x / nr CTAs with identical row partitions.
+struct PanelLaunch {
+    PanelParams r[FT_MAX_VRANKS];
+    int nr;
 };
 
 // launchers (return cudaError_t of the launch)
 cudaError_t ft_launch_panel(const PanelParams &p, int nsm, cudaStream_t s);
+cudaError_t ft_launch_panel_multi(const PanelLaunch &L, int nsm, cudaStream_t s);
 size_t ft_panel_smem_bytes();
 int ft_panel_group_rows();
 
@@ -78,7 +101,17 @@ struct GemmRightParams {
     const double *T;
     int transT;
     int *strip_done;  // per-strip arrival counters (zero; reset by their last CTA)
+    // multi-rank column map: local column l of A is global column
+    // ft_cmap(l) (the row of V it pairs with); cm_G <= 1 is the identity
+    int cm_G, cm_rank, cm_nb, cm_ncl, cm_n;
 };
+// global column of local column l in the 1-D block-column cyclic layout; local column ncl
+// is the replicated row-checksum column r (global n)
+__host__ __device__ inline int ft_cmap(int l, int G, int rank, int nb, int ncl, int n) {
+    if (G <= 1) return l;
+    if (l == ncl) return n;
+    return (l / nb) * nb * G + rank * nb + l % nb;
+}
 cudaError_t ft_launch_gemm_right(const GemmRightParams &p, cudaStream_t s);
 #define FT_WSPLIT_MAX 16  // max row splits of the right update (deterministic W partials)
 // row splits the right-update launch uses for this block (the left update's k_wprep sums them)
@@ -115,6 +148,9 @@ struct YtopParams {
     int n, ihi, k, ib, nsplit, abft, verify;
     int decide;  // fused pre-update check (R15): add e^T Y of rows 0..k, last block decides
     int panel;
+    // multi-rank: the inner dimension runs over the local columns [kc0, kc1) (global >= k+1),
+    // V rows through the column map; Y(0:k+1, :) is then this rank's partial
+    int cm_G, cm_rank, cm_nb, cm_ncl, kc0, kc1;
 };
 cudaError_t ft_launch_ytop(const YtopParams &p, cudaStream_t s);
 

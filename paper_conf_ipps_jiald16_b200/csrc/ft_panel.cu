@@ -75,7 +75,7 @@ size_t ft_panel_smem_bytes() { return sizeof(PanelSmem); }
     do {                                                                              \
         if (p.dbg && tid == 0 && j < 64) {                                            \
             const long long now_ = clock64();                                         \
-            if (blockIdx.x == 0) p.dbg[j * 16 + (slot)] = now_;                       \
+            if (bid == 0) p.dbg[j * 16 + (slot)] = now_;                       \
             if ((slot) != 0)                                                          \
                 atomicMax(p.dbg + 1024 + j * 16 + (slot), (unsigned long long)(now_ - probe_last)); \
             probe_last = now_;                                                        \
@@ -124,22 +124,38 @@ __device__ __forceinline__ double group8_sum(double v) {
     return v;
 }
 
-template <bool CACHE>
-__global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
+// system-scope flag helpers for the cross-rank exchange (peer memory over NVLink, or the
+// other virtual ranks of this launch)
+__device__ __forceinline__ unsigned ld_acquire_sys_u32(const unsigned *p) {
+    unsigned v;
+    asm volatile("ld.acquire.sys.global.u32 %0, [%1];\n" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_relaxed_sys_u32(unsigned *p, unsigned v) {
+    asm volatile("st.relaxed.sys.global.u32 [%0], %1;\n" ::"l"(p), "r"(v) : "memory");
+}
+
+template <bool CACHE, bool MG>
+__global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLaunch L) {
+    // rank group of this CTA (MG: virtual ranks share the launch; one GPU: a single group)
+    const unsigned P = gridDim.x / L.nr;
+    const int vr = MG ? (int)(blockIdx.x / P) : 0;
+    const PanelParams &p = L.r[vr];
+    const int bid = (int)(blockIdx.x - vr * P);
     if (p.ctl->halt) return;  // uniform for the whole grid (nobody writes halt in this launch)
     extern __shared__ __align__(16) unsigned char smem_raw[];
     PanelSmem &S = *reinterpret_cast<PanelSmem *>(smem_raw);
 
     const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
     const int slot = tid >> 3, g = tid & 7;  // 8-lane groups: NSLOT row / output slots
-    const unsigned P = gridDim.x;
-    const int g0 = (int)((long long)blockIdx.x * p.ngroups / P);
-    const int g1 = (int)((long long)(blockIdx.x + 1) * p.ngroups / P);
+    const int g0 = (int)((long long)bid * p.ngroups / P);
+    const int g1 = (int)((long long)(bid + 1) * p.ngroups / P);
     const int r0 = p.rbase + GR * g0, r1 = p.rbase + GR * g1;
     const int R = r1 - r0, R2 = R >> 1;
     const int n = p.n, ihi = p.ihi, k = p.k, ib = p.ib;
     const int64_t ldw = p.ldw;
     double *__restrict__ A = p.A;
+    double *__restrict__ Apan = p.Apan;  // panel columns (== A on one GPU)
     double *__restrict__ V = p.V;
     double *__restrict__ Y = p.Y;
 
@@ -245,15 +261,15 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
         const int rend = p.abft ? n + 1 : ihi;
         for (int x = tid; x < R * ib; x += PT) {
             const int rl = x % R, jj = x / R, row = r0 + rl;
-            if (row < rend) p.ckpt[row + (int64_t)jj * ldw] = A[row + (int64_t)(k + jj) * ldw];
+            if (row < rend) p.ckpt[row + (int64_t)jj * ldw] = Apan[row + (int64_t)(k + jj) * ldw];
         }
-        const int gstride = (int)P * PT, gi = blockIdx.x * PT + tid;
+        const int gstride = (int)P * PT, gi = bid * PT + tid;
         for (int x = gi; x < p.rbase * ib; x += gstride) {
             const int i = x % p.rbase, jj = x / p.rbase;
-            p.ckpt[i + (int64_t)jj * ldw] = A[i + (int64_t)(k + jj) * ldw];
+            p.ckpt[i + (int64_t)jj * ldw] = Apan[i + (int64_t)(k + jj) * ldw];
         }
         for (int i = gi; i <= n; i += gstride) {
-            p.ck_r[i] = A[i + (int64_t)n * ldw];
+            p.ck_r[i] = p.rcol[i];
             p.ck_q[i] = p.Qr[i];
             p.ck_q[ldw + i] = p.Qc[i];
             p.ck_q[2 * ldw + i] = p.Fr[i];
@@ -263,9 +279,9 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
     }
     for (int rl = tid; rl < R; rl += PT) {
         const int row = r0 + rl;
-        S.acol[rl] = is_valid(row) ? A[row + (int64_t)k * ldw] : 0.0;
+        S.acol[rl] = is_valid(row) ? Apan[row + (int64_t)k * ldw] : 0.0;
     }
-    if (tid == 0 && blockIdx.x == 0) *p.bar_next = 0u;  // the next panel launch's counter
+    if (tid == 0 && bid == 0) *p.bar_next = 0u;  // the next panel launch's counter
     __syncthreads();
 
     unsigned epoch = 0;
@@ -280,7 +296,10 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
         double *acc = p.acc + (c & 3) * FT_ACC_SET_DOUBLES;  // accumulator i at acc[i * FT_ACC_PAD]
         // A(row, c+1) of the own rows (thread = row): issued now, parked in smem before the GEMV
         double an_reg = 0.0;
-        if (tid < R && is_valid(r0 + tid)) an_reg = A[(r0 + tid) + (int64_t)(c + 1) * ldw];
+        // (MG: a trailing column c+1 >= e lives on one rank; it arrives through the exchange)
+        // (one GPU: column e is read from A, the panel buffer holds only the panel columns)
+        if (tid < R && is_valid(r0 + tid) && (!MG || c + 1 < p.e))
+            an_reg = (c + 1 < p.e ? Apan : A)[(r0 + tid) + (int64_t)(c + 1) * ldw];
         PROBE(0);
         // ---------------- (i) b0 = A(:,c) - Y V(c,:)^T, s1 = V^T b0 ---------------------------
         if (j > 0) {
@@ -374,7 +393,39 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
             const bool vfy = (j == 0) && p.verify;
             const int cend = vfy ? n : ihi;
             double2 ya = make_double2(0.0, 0.0), rs = make_double2(0.0, 0.0);
-            if (gemv_on && !(p.dbg_mode & 2)) {
+            if (MG && gemv_on && !(p.dbg_mode & 2)) {
+                // virtual columns: [0, nA) the panel columns c+2.. (owner only, from Apan), then
+                // the local trailing columns lcol0.. (global index J(l) selects x)
+                const int nA = (p.owner && p.e > c + 2) ? p.e - (c + 2) : 0;
+                const int nv = nA + (p.lcol1 - p.lcol0);
+                const double2 *__restrict__ Ap2 = reinterpret_cast<const double2 *>(Apan + r0);
+#pragma unroll 1
+                for (int v0 = cl; v0 < nv; v0 += GB * ncl) {
+                    double2 a[GB];
+                    double xv[GB];
+#pragma unroll
+                    for (int u = 0; u < GB; u++) {
+                        const int v = v0 + u * ncl;
+                        a[u] = make_double2(0.0, 0.0);
+                        xv[u] = 0.0;
+                        if (v < nA) {
+                            const int q = c + 2 + v;
+                            a[u] = Ap2[(int64_t)q * ldw2 + rp];
+                            xv[u] = bv[q];
+                        } else if (v < nv) {
+                            const int l = p.lcol0 + v - nA;
+                            const int J = (l / p.cbnb) * p.cbnb * p.G + p.rank * p.cbnb + l % p.cbnb;
+                            a[u] = A2[(int64_t)l * ldw2 + rp];
+                            xv[u] = J >= c + 2 ? bv[J] : 0.0;  // column c+1 = e is the unit term
+                        }
+                    }
+#pragma unroll
+                    for (int u = 0; u < GB; u++) {
+                        ya.x += a[u].x * xv[u];
+                        ya.y += a[u].y * xv[u];
+                    }
+                }
+            } else if (gemv_on && !(p.dbg_mode & 2)) {
                 // b is read with plain (L1-allocating) loads: the acquire at the grid barrier
                 // invalidated this SM's L1 before the trailing bar.sync released us
                 int col = c + 2 + cl;
@@ -461,7 +512,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
                 if (row == n && p.abft) {
                     V[row + (int64_t)j * ldw] = vchk;
                     if (CACHE) Vl[rl * XR + j * XC] = vchk;
-                    A[row + (int64_t)c * ldw] = (tau != 0.0) ? b - vchk * (alpha - beta) : b;  // left term (R7)
+                    Apan[row + (int64_t)c * ldw] = (tau != 0.0) ? b - vchk * (alpha - beta) : b;  // left term (R7)
                 } else if (is_data(row)) {
                     double vv, av;
                     if (row <= c) {
@@ -476,12 +527,12 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
                     }
                     V[row + (int64_t)j * ldw] = vv;
                     if (CACHE) Vl[rl * XR + j * XC] = vv;
-                    A[row + (int64_t)c * ldw] = av;
+                    Apan[row + (int64_t)c * ldw] = av;
                 } else if (CACHE) {
                     Vl[rl * XR + j * XC] = 0.0;  // rows outside the panel take no part in the dots
                 }
             }
-            if (blockIdx.x == 0 && lane == 0) {
+            if (bid == 0 && lane == 0) {
                 p.tau[c] = tau;
                 if (p.abft) {
                     p.Qc[c] = vchk - 1.0;  // Q column checksum
@@ -490,11 +541,44 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
             }
             // recycle the accumulator set of column c+2 (= that of column c-2): every CTA has
             // finished reading it, and column c+2 adds into it only after two more syncs
-            if (blockIdx.x == 0)
+            if (bid == 0)
                 for (int i = lane; i < FT_ACC_STRIDE; i += 32) p.acc[((c + 2) & 3) * FT_ACC_SET_DOUBLES + i * FT_ACC_PAD] = 0.0;
             PROBE(6);
         }
         __syncthreads();  // GEMV partials, tau / scale / t, V(:, j) are in shared memory
+        if (MG) {
+            // ---- cross-rank exchange of the GEMV partials, CTA by CTA: every rank
+            // uses the same row partition, so CTA bid of each rank owns the same rows.  Push
+            // (y partial, A(:, c+1) part) of the own rows into every rank's slot, raise the flag,
+            // wait for every rank's flag; phase (v) sums the slots in rank order (identical on
+            // every rank).  Slots alternate by column; a rank reaches column c+2's push only
+            // after every rank has flagged column c+1, i.e. after it read column c.
+            const int sl = c & 1;
+            const int l0 = p.lcol0;
+            const bool have_an = (c + 1 == p.e) && l0 < p.lcol1 &&
+                                 (l0 / p.cbnb) * p.cbnb * p.G + p.rank * p.cbnb + l0 % p.cbnb == p.e;
+            for (int rl = tid; rl < R; rl += PT) {
+                const int row = r0 + rl, pr = rl >> 1, hi = rl & 1;
+                double ys = 0.0;
+                for (int q = 0; q < npart; q++) {
+                    const double2 u = S.red[q * R2p + pr];
+                    ys += hi ? u.y : u.x;
+                }
+                const double ap = (have_an && is_valid(row)) ? A[row + (int64_t)l0 * ldw] : 0.0;
+                const double2 v2 = make_double2(ys, ap);
+                for (int gg = 0; gg < p.G; gg++) p.ypeer[gg][((int64_t)sl * p.G + p.rank) * ldw + row] = v2;
+            }
+            __syncthreads();
+            const unsigned seq = p.seq0 + (unsigned)c + 1u;
+            if (tid == 0) {
+                __threadfence_system();
+                for (int gg = 0; gg < p.G; gg++) st_relaxed_sys_u32(p.fpeer[gg] + p.rank * FT_FLAG_STRIDE + bid, seq);
+            }
+            if (wid == 0 && lane < p.G)
+                while (ld_acquire_sys_u32(p.flags + lane * FT_FLAG_STRIDE + bid) < seq) {
+                }
+            __syncthreads();
+        }
         PROBE(7);
         // ---------------- (v) Y(:, j) = tau (y - Y t) (an 8-lane group per row) -----------------
         {
@@ -523,8 +607,19 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
                 const bool on = rl < R && is_valid(r0 + rl);
                 const int pr = rl >> 1, hi = rl & 1;
                 // lane partial of scale * y - Y(rl, :) t: GEMV partials q = g, g + 8 (npart <= 15)
-                double ya = 0.0, yb = 0.0, rsum = 0.0;
-                if (on) {
+                double ya = 0.0, yb = 0.0, rsum = 0.0, an_mg = 0.0;
+                if (on && MG) {
+                    if (g == 0) {  // exchanged partials, summed in rank order
+                        double ysum = 0.0;
+                        const double2 *yxs = p.yx + (int64_t)(c & 1) * p.G * ldw + (r0 + rl);
+                        for (int gg = 0; gg < p.G; gg++) {
+                            const double2 u = __ldcg(yxs + (int64_t)gg * ldw);
+                            ysum += u.x;
+                            an_mg += u.y;
+                        }
+                        ya = scale * ysum;
+                    }
+                } else if (on) {
 #pragma unroll
                     for (int u = 0; u < 2; u++) {
                         const int q = g + 8 * u;
@@ -537,6 +632,8 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
                             }
                         }
                     }
+                }
+                if (on) {
 #pragma unroll
                     for (int u = 0; u < FT_NBMAX / 8; u += 2) {
                         const int ja = g + 8 * u, jb = ja + 8;
@@ -548,7 +645,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
                 if (vfy) rsum = group8_sum(rsum);
                 if (rl < R && g == 0) {
                     const int row = r0 + rl;
-                    const double an = S.anext[rl];
+                    const double an = (MG && c + 1 >= p.e) ? an_mg : S.anext[rl];
                     if (on) {
                         const double yy = tau * (an + ysum);
                         Y[row + (int64_t)j * ldw] = yy;
@@ -556,7 +653,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
                         if (vfy && is_data(row)) {
                             // D_r(row) = r(row) - sum_{col >= k} L(row, col); columns < k are logical zero
                             rsum += S.acol[rl] + an;
-                            const double d = A[row + (int64_t)n * ldw] - rsum;
+                            const double d = p.rcol[row] - rsum;
                             if (not_within(d, tau_abs)) {
                                 atomicAdd(&p.ctl->nflag, 1);
                             } else if (tau_abs > 0.0) {
@@ -591,44 +688,62 @@ __global__ void __launch_bounds__(PT, 1) k_panel(PanelParams p) {
             if (is_data(r0 + rl)) s += X[rl * XR + jj * XC];
         atomicAdd(tid < ib ? &p.ctl->eY[jj] : &p.ctl->eV[jj], s);
     }
-    if (blockIdx.x == 0 && tid == 0 && p.abft) p.Qc[n] += qc_corner;
-    if (blockIdx.x == 0)
+    if (bid == 0 && tid == 0 && p.abft) p.Qc[n] += qc_corner;
+    if (bid == 0)
         for (int i = tid; i < ib * ib; i += PT) {
             int a = i % ib, bb = i / ib;
             p.T[a + bb * FT_NBMAX] = S.Ts[a][bb];
         }
 }
 
-cudaError_t ft_launch_panel(const PanelParams &p, int nsm, cudaStream_t s) {
+cudaError_t ft_launch_panel_multi(const PanelLaunch &L, int nsm, cudaStream_t s) {
     static int max_smem = 0;
     if (!max_smem) {
         int dev = 0;
         cudaGetDevice(&dev);
         cudaDeviceGetAttribute(&max_smem, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
-        cudaError_t e = cudaFuncSetAttribute(k_panel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem);
-        if (e != cudaSuccess) return e;
-        e = cudaFuncSetAttribute(k_panel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem);
-        if (e != cudaSuccess) return e;
+        const void *fns[] = {(const void *)k_panel<true, false>, (const void *)k_panel<false, false>,
+                             (const void *)k_panel<true, true>, (const void *)k_panel<false, true>};
+        for (const void *fn : fns) {
+            cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem);
+            if (e != cudaSuccess) return e;
+        }
     }
     static int ctas = -1;
     if (ctas < 0) {
         const char *e = getenv("FT_PANEL_CTAS");  // experiment knob: cap on the panel grid
         ctas = e ? atoi(e) : 0;
     }
-    if (ctas > 0 && ctas < nsm) nsm = ctas;
-    int grid = nsm < p.ngroups ? nsm : p.ngroups;
+    if (L.nr < 1 || L.nr > FT_MAX_VRANKS) return cudaErrorInvalidValue;
+    const bool mg = L.r[0].G > 1;
+    int per = nsm / L.nr;  // CTAs per rank group (identical row partition in every group)
+    if (ctas > 0 && ctas < per) per = ctas;
+    if (per > FT_FLAG_STRIDE) per = FT_FLAG_STRIDE;
+    int grid = per < L.r[0].ngroups ? per : L.r[0].ngroups;
     if (grid < 1) grid = 1;
     // rows per CTA (max over CTAs) and whether their V/Y rows fit next to the fixed part
-    const int gmax = (p.ngroups + grid - 1) / grid;
+    const int gmax = (L.r[0].ngroups + grid - 1) / grid;
     const int rmax = GR * gmax;
     if (rmax > RMAX) return cudaErrorInvalidConfiguration;  // n beyond ~75k rows per GPU
     const size_t fixed = sizeof(PanelSmem);
     const size_t want = fixed + (size_t)2 * VS * rmax * sizeof(double);
     const bool cache = want <= (size_t)max_smem;
-    void *args[] = {const_cast<PanelParams *>(&p)};
+    void *args[] = {const_cast<PanelLaunch *>(&L)};
     g_ft_launches++;
-    const void *fn = cache ? (const void *)k_panel<true> : (const void *)k_panel<false>;
-    return cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(PT), args, cache ? want : fixed, s);
+    const void *fn = mg ? (cache ? (const void *)k_panel<true, true> : (const void *)k_panel<false, true>)
+                        : (cache ? (const void *)k_panel<true, false> : (const void *)k_panel<false, false>);
+    return cudaLaunchCooperativeKernel(fn, dim3(grid * L.nr), dim3(PT), args, cache ? want : fixed, s);
+}
+
+cudaError_t ft_launch_panel(const PanelParams &p, int nsm, cudaStream_t s) {
+    PanelLaunch L;
+    L.r[0] = p;
+    L.nr = 1;
+    L.r[0].G = 1;
+    if (!L.r[0].Apan) L.r[0].Apan = p.A;
+    if (!L.r[0].rcol) L.r[0].rcol = p.A + (int64_t)p.n * p.ldw;
+    if (!L.r[0].e) L.r[0].e = p.k + p.ib;
+    return ft_launch_panel_multi(L, nsm, s);
 }
 
 int ft_panel_group_rows() { return GR; }

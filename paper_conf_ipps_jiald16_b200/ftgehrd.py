@@ -46,6 +46,10 @@ class Report(ctypes.Structure):
                 for e in self.events[: min(self.nevents, MAX_EVENTS)]]
 
 
+class IpcHandle(ctypes.Structure):
+    _fields_ = [("bytes", ctypes.c_char * 64)]
+
+
 class Opts(ctypes.Structure):
     _fields_ = [("nb", ctypes.c_int32), ("abft", ctypes.c_int32), ("weighted", ctypes.c_int32),
                 ("policy", ctypes.c_int32), ("c_thr", ctypes.c_double),
@@ -74,7 +78,11 @@ def lib():
         L.ft_dgehrd.argtypes = [i32, i32, i32, vp, i32, vp, ctypes.POINTER(Opts)]
         L.ft_dgehrd_host.argtypes = [i32, i32, i32, vp, i32, vp, ctypes.POINTER(Opts)]
         L.ft_dorghr.argtypes = [i32, i32, i32, vp, i32, vp, vp, i32, ctypes.POINTER(Opts)]
-        L.ft_dgehrd_mgpu.argtypes = [i32, i32, i32, vp, i32, vp, vp, i32, i32, ctypes.POINTER(Opts)]
+        L.ft_dgehrd_mgpu.argtypes = [i32, i32, i32, vp, i32, vp, i32, i32, ctypes.POINTER(Opts)]
+        L.ft_mgpu_setup.argtypes = [i32, i32, i32, ctypes.POINTER(IpcHandle)]
+        L.ft_mgpu_connect.argtypes = [ctypes.POINTER(IpcHandle), i32, i32]
+        L.ft_dgehrd_vranks.argtypes = [i32, i32, i32, ctypes.POINTER(vp), i32, ctypes.POINTER(vp), i32,
+                                       ctypes.POINTER(Opts)]
         L.ft_strerror.argtypes = [i32]
         L.ft_strerror.restype = ctypes.c_char_p
         L.ft_version.restype = ctypes.c_char_p
@@ -85,6 +93,7 @@ def lib():
 
 
 EXPORTS = ["ft_opts_default", "ft_dgehrd", "ft_dgehrd_host", "ft_dorghr", "ft_dgehrd_mgpu",
+           "ft_mgpu_setup", "ft_mgpu_connect", "ft_dgehrd_vranks", "ft_mgpu_finalize",
            "ft_strerror", "ft_finalize", "ft_version", "ft_launch_count"]
 
 
@@ -204,3 +213,129 @@ def launch_count(reset: bool = False) -> int:
 
 def finalize() -> None:
     lib().ft_finalize()
+
+
+# ---------------------------------------------------------------------------------------
+# Multi-GPU: 1-D block-column cyclic layout, block = nb.  Host-side layout
+# logic is plain Python (tested with gloo on CPU); the reduction runs in the library.
+# ---------------------------------------------------------------------------------------
+def default_nb(n: int) -> int:
+    """Panel width the library picks for opts.nb = 0 (reading R4)."""
+    return 32 if n < 4096 else 64
+
+
+def cyclic_columns(n: int, nb: int, rank: int, nranks: int) -> list:
+    """Global columns of `rank`, in local order: J lives on rank (J // nb) % nranks at local
+    column (J // (nb * nranks)) * nb + J % nb (include/ftgehrd.h)."""
+    cols = []
+    for b in range(rank, (n + nb - 1) // nb, nranks):
+        cols.extend(range(b * nb, min(n, (b + 1) * nb)))
+    return cols
+
+
+def global_to_local(J: int, nb: int, nranks: int) -> tuple:
+    """(rank, local column) of global column J."""
+    return (J // nb) % nranks, (J // (nb * nranks)) * nb + J % nb
+
+
+def shard(A, nb: int, nranks: int) -> list:
+    """Split an n x n matrix (torch or numpy) into the ranks' column-major slabs."""
+    n = A.shape[0]
+    out = []
+    for r in range(nranks):
+        idx = cyclic_columns(n, nb, r, nranks)
+        sl = A[:, idx]
+        if hasattr(sl, "is_cuda"):
+            sl = fortran(sl)
+        else:
+            import numpy as np
+            sl = np.asfortranarray(sl)
+        out.append(sl)
+    return out
+
+
+def unshard(slabs: list, n: int, nb: int):
+    """Inverse of shard (returns a torch tensor on the slabs' device, or numpy)."""
+    nranks = len(slabs)
+    first = slabs[0]
+    if hasattr(first, "is_cuda"):
+        import torch
+        A = torch.empty((n, n), dtype=first.dtype, device=first.device)
+    else:
+        import numpy as np
+        A = np.empty((n, n), dtype=first.dtype)
+    for r in range(nranks):
+        idx = cyclic_columns(n, nb, r, nranks)
+        if len(idx):
+            A[:, idx] = slabs[r][:, : len(idx)]
+    return A
+
+
+def _slab_ld(S, n):
+    if n > 1 and S.shape[1] > 1 and S.stride(0) != 1:
+        raise ValueError("slabs must be column-major (use fortran())")
+    return max(S.stride(1) if S.shape[1] > 1 else n, n, 1)
+
+
+def dgehrd_vranks(slabs: list, nb: int = 0, abft: bool = True, taus=None, stream=None):
+    """Sharded reduction with len(slabs) VIRTUAL ranks on the current GPU (ft_dgehrd_vranks).
+
+    slabs: the ranks' n x ncols CUDA float64 column-major slabs (modified in place).
+    Returns (taus, Result)."""
+    import torch
+    G = len(slabs)
+    n = slabs[0].shape[0]
+    nb_eff = nb if nb > 0 else default_nb(n)
+    for r, S in enumerate(slabs):
+        if S.shape[1] != len(cyclic_columns(n, nb_eff, r, G)):
+            raise ValueError(f"slab {r} has {S.shape[1]} columns, layout needs {len(cyclic_columns(n, nb_eff, r, G))}")
+    lda = max(_slab_ld(S, n) for S in slabs)
+    if any(_slab_ld(S, n) != lda for S in slabs):
+        raise ValueError("all slabs must share one leading dimension")
+    if taus is None:
+        taus = [torch.zeros(max(n - 1, 1), dtype=torch.float64, device=slabs[0].device) for _ in range(G)]
+    pa = (ctypes.c_void_p * G)(*[S.data_ptr() for S in slabs])
+    pt = (ctypes.c_void_p * G)(*[t.data_ptr() for t in taus])
+    rep = Report()
+    o = make_opts(nb=nb, abft=abft, report=rep, stream=stream)
+    info = lib().ft_dgehrd_vranks(n, 1, n, pa, lda, pt, G, ctypes.byref(o))
+    return taus, Result(info, rep, rep.event_list())
+
+
+def exchange_handles(local: bytes, group=None) -> list:
+    """All-gather each rank's 64-byte IPC handle over torch.distributed (any backend)."""
+    import torch.distributed as dist
+    out = [None] * dist.get_world_size(group)
+    dist.all_gather_object(out, bytes(local), group=group)
+    return out
+
+
+def mgpu_init(n_max: int, group=None) -> None:
+    """Bootstrap of the multi-GPU path for this process's rank (one process per GPU)."""
+    import torch.distributed as dist
+    rank, nranks = dist.get_rank(group), dist.get_world_size(group)
+    h = IpcHandle()
+    info = lib().ft_mgpu_setup(n_max, rank, nranks, ctypes.byref(h))
+    if info:
+        raise RuntimeError(f"ft_mgpu_setup: {strerror(info)}")
+    hs = exchange_handles(h.bytes.ljust(64, b"\0")[:64], group)
+    arr = (IpcHandle * nranks)()
+    for g, b in enumerate(hs):
+        ctypes.memmove(ctypes.byref(arr[g]), b, 64)
+    info = lib().ft_mgpu_connect(arr, rank, nranks)
+    if info:
+        raise RuntimeError(f"ft_mgpu_connect: {strerror(info)}")
+
+
+def dgehrd_mgpu(slab, rank: int, nranks: int, nb: int = 0, abft: bool = True, tau=None, stream=None):
+    """This rank's part of the sharded reduction (after mgpu_init). Returns (tau, Result)."""
+    import torch
+    n = slab.shape[0]
+    lda = _slab_ld(slab, n)
+    if tau is None:
+        tau = torch.zeros(max(n - 1, 1), dtype=torch.float64, device=slab.device)
+    rep = Report()
+    o = make_opts(nb=nb, abft=abft, report=rep, stream=stream)
+    info = lib().ft_dgehrd_mgpu(n, 1, n, ctypes.c_void_p(slab.data_ptr()), lda, ctypes.c_void_p(tau.data_ptr()),
+                                rank, nranks, ctypes.byref(o))
+    return tau, Result(info, rep, rep.event_list())

@@ -27,7 +27,8 @@ def declared_functions():
 
 def test_header_declares_the_boundary():
     names = declared_functions()
-    for f in ["ft_dgehrd", "ft_dgehrd_host", "ft_dorghr", "ft_dgehrd_mgpu", "ft_strerror", "ft_finalize",
+    for f in ["ft_dgehrd", "ft_dgehrd_host", "ft_dorghr", "ft_dgehrd_mgpu", "ft_mgpu_setup", "ft_mgpu_connect",
+              "ft_dgehrd_vranks", "ft_mgpu_finalize", "ft_strerror", "ft_finalize",
               "ft_opts_default", "ft_version", "ft_launch_count"]:
         assert f in names
 
