@@ -149,6 +149,100 @@ def run_reference(args, rank: int, world: int):
     print(json.dumps(line), flush=True)
 
 
+def run_sharded(args, rank: int, world: int, local: int, dist):
+    """N > 1: ONE n x n reduction, 1-D block-column cyclic over the N GPUs (SURVEY 8(e));
+    the per-column GEMV partials move through peer memory inside the panel kernel.  Strong
+    scaling: value = steps * 10/3 n^3 / (max over ranks of the summed step times)."""
+    import ctypes
+
+    import numpy as np
+    import torch
+
+    import paper_conf_ipps_jiald16_b200 as ft
+    import synth
+
+    n, nb = args.n, args.nb
+    A = synth.matrix(n)  # the same matrix on every rank (seed 20160523 + n)
+    cols = ft.cyclic_columns(n, nb, rank, world)
+    slab0 = ft.fortran(torch.from_numpy(np.ascontiguousarray(A[:, cols])).cuda())
+    slab = slab0.clone()
+    slab = ft.fortran(slab)
+    tau = torch.zeros(n, dtype=torch.float64, device="cuda")
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda")
+    stream = torch.cuda.current_stream()
+    ft.mgpu_init(n)
+
+    def one(abft: bool):
+        slab.copy_(slab0)
+        flush.fill_(1.0)
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        _, res = ft.dgehrd_mgpu(slab, rank, world, nb=nb, abft=abft, tau=tau, stream=stream)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        if res.info != 0:
+            raise RuntimeError(f"ft_dgehrd_mgpu info={res.info}: {ft.strerror(res.info)}")
+        return e0.elapsed_time(e1), res
+
+    for _ in range(args.warmup):
+        one(True)
+        one(False)
+    sampler = ClockSampler(local)
+    sampler.start()
+    dist.barrier()
+    torch.cuda.synchronize()
+    launches0 = ft.launch_count()
+    on_ms = [one(True)[0] for _ in range(args.steps)]
+    launches = ft.launch_count() - launches0
+    off_ms = [one(False)[0] for _ in range(args.steps)]
+    torch.cuda.synchronize()
+    dist.barrier()
+    clocks = sampler.stop()
+    tt = torch.tensor([sum(on_ms) / 1e3, sum(off_ms) / 1e3], dtype=torch.float64, device="cuda")
+    dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+    T_on, T_off = tt.tolist()
+    value = args.steps * flops(n) / T_on / 1e9
+    # e2e: this rank's slab from pinned host memory, the reduction, H/V slab + tau back
+    hs0 = slab0.cpu().pin_memory()
+    hs = torch.empty_like(hs0).pin_memory()
+    htau = torch.zeros(n, dtype=torch.float64).pin_memory()
+    times = []
+    for it in range(args.warmup + args.steps):
+        flush.fill_(1.0)
+        torch.cuda.synchronize()
+        dist.barrier()
+        t0 = time.perf_counter()
+        slab.copy_(hs0, non_blocking=True)
+        _, res = ft.dgehrd_mgpu(slab, rank, world, nb=nb, abft=True, tau=tau, stream=stream)
+        hs.copy_(slab, non_blocking=True)
+        htau.copy_(tau, non_blocking=True)
+        torch.cuda.synchronize()
+        t1 = time.perf_counter()
+        if it >= args.warmup:
+            times.append(t1 - t0)
+    te = torch.tensor([sum(times)], dtype=torch.float64, device="cuda")
+    dist.all_reduce(te, op=dist.ReduceOp.MAX)
+    e2e = {"value": len(times) * flops(n) / te.item() / 1e9, "unit": "Gflop/s",
+           "h2d_bytes_per_step": 8 * n * len(cols), "d2h_bytes_per_step": 8 * n * len(cols) + 8 * n,
+           "api": "ft_dgehrd_mgpu (per-rank slab from pinned host memory)"}
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": "Gflop/s", "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": 1e3 * T_on / args.steps, "higher_is_better": True,
+                "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+                "data": "synthetic U(0,1) (splitmix64 counter generator, seed 20160523+n)",
+                "config": {"workload": f"C4-style: one n={n} nb={nb} ABFT reduction, 1-D block-column cyclic "
+                                       f"over {world} GPUs", "n": n, "nb": nb, "abft": 1,
+                           "l2": "flushed between steps (256 MiB write), input restored outside the timed events",
+                           "parallelism": f"column-cyclic x{world} (peer-memory exchange per column)"},
+                "abft_overhead_pct": 100.0 * (T_on - T_off) / T_off,
+                "abft_off_value": args.steps * flops(n) / T_off / 1e9,
+                "ms_per_step_abft_off": 1e3 * T_off / args.steps, "roofline": None, "cpu_baseline": None,
+                "e2e": e2e, "gpu_launches": launches, "clocks": clocks}
+        print(json.dumps(line), flush=True)
+    dist.destroy_process_group()
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -158,6 +252,8 @@ def main():
     ap.add_argument("--nb", type=int, default=32)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--replicas", action="store_true",
+                    help="N > 1: independent replicas instead of one sharded reduction")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
 
@@ -184,6 +280,9 @@ def main():
         dist = tdist
 
     n, nb = args.n, args.nb
+    if world > 1 and not args.replicas:
+        run_sharded(args, rank, world, local, dist)
+        return
     A = synth.matrix(n, seed=synth.default_seed(n) + rank)
     dA0 = ft.fortran(torch.from_numpy(A).cuda())
     dA = ft.fortran(torch.empty((n, n), dtype=torch.float64, device="cuda"))
