@@ -143,7 +143,15 @@ FT_DEV double sum_strided(const double *p, int64_t stride, int N) {
         s2 += v[2] + v[6];
         s3 += v[3] + v[7];
     }
-    for (; i < N; i++) s0 += __ldcg(p + (int64_t)i * stride);
+    if (i < N) {  // remainder: one predicated batch (all loads in flight together)
+        double v[8];
+#pragma unroll
+        for (int u = 0; u < 8; u++) v[u] = i + u < N ? __ldcg(p + (int64_t)(i + u) * stride) : 0.0;
+        s0 += v[0] + v[4];
+        s1 += v[1] + v[5];
+        s2 += v[2] + v[6];
+        s3 += v[3] + v[7];
+    }
     return (s0 + s1) + (s2 + s3);
 }
 

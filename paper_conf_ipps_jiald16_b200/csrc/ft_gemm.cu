@@ -25,10 +25,10 @@
 #define UT 256  // threads (8 warps)
 #define SK 68   // smem stride of the k-major operand tiles
 
-// Row splits per strip: minimise waves * tiles-per-CTA for 2 resident CTAs per SM (the
+// Row splits per strip: minimise waves * tiles-per-CTA for one resident CTA per SM (the
 // grid is nstrip x ns CTAs; a ragged last wave idles SMs).
 static int best_splits(int nstrip, int nrt, int nsm, int cap) {
-    const int slots = 2 * nsm;
+    const int slots = nsm;  // one CTA per SM (the C tile of the next iteration is prefetched in registers)
     int best = 1;
     long long best_cost = -1;
     for (int ns = 1; ns <= cap && ns <= nrt; ns++) {
@@ -90,7 +90,7 @@ __device__ __forceinline__ void store_pair(double *colp, int row, int lo, int hi
 // warp w owns columns w*8 .. w*8+7 of the strip and all 64 rows of a tile (8 fragments)
 // ---------------------------------------------------------------------------
 template <int KT>
-__global__ void __launch_bounds__(UT, 2) k_gemm_right(GemmRightParams p) {
+__global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
     if (p.ctl && p.ctl->halt) return;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     RightSmemT<KT> &S = *reinterpret_cast<RightSmemT<KT> *>(smem_raw);
@@ -132,6 +132,19 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_right(GemmRightParams p) {
         if (do_w) issue_ktile<KT>(S.Vr, p.V, p.ldw, rbase + t0 * UB, r_hi, K);
         cp_async_commit();
     }
+    // C tile of tile tt into registers (16-byte loads; masked pairs at the edges)
+    auto load_c = [&](int tt, double2 (&dst)[8]) {
+        const int r = rbase + tt * UB;
+        const int lo = max(r, r_lo), hi = min(r + UB, r_hi);
+        const bool full = lo == r && hi == r + UB && ncols == UB;
+#pragma unroll
+        for (int ni = 0; ni < 8; ni++) {
+            const int row = r + ni * 8 + 2 * lc;
+            dst[ni] = full ? *reinterpret_cast<const double2 *>(colp + row) : load_pair(colp, row, lo, hi, colok);
+        }
+    };
+    double2 cn[8];  // the next tile's C, prefetched a whole tile ahead
+    if (t0 < t1) load_c(t0, cn);
     for (int tt = t0; tt < t1; tt++) {
         const int r = rbase + tt * UB;
         const int lo = max(r, r_lo), hi = min(r + UB, r_hi);
@@ -139,11 +152,10 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_right(GemmRightParams p) {
         double acc[8][2];
 #pragma unroll
         for (int ni = 0; ni < 8; ni++) {
-            const int row = r + ni * 8 + 2 * lc;
-            const double2 c = full ? *reinterpret_cast<const double2 *>(colp + row) : load_pair(colp, row, lo, hi, colok);
-            acc[ni][0] = sg * c.x;
-            acc[ni][1] = sg * c.y;
+            acc[ni][0] = sg * cn[ni].x;
+            acc[ni][1] = sg * cn[ni].y;
         }
+        if (tt + 1 < t1) load_c(tt + 1, cn);
         cp_async_wait<1>();
         __syncthreads();
         if (p.do_right) {
@@ -354,7 +366,7 @@ __global__ void k_wprep(const double *__restrict__ Wpart, int64_t wstride, int n
 }
 
 template <int KT>
-__global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
+__global__ void __launch_bounds__(UT, 1) k_gemm_left(GemmLeftParams p) {
     if (p.ctl && p.ctl->halt) return;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     LeftSmemT<KT> &S = *reinterpret_cast<LeftSmemT<KT> *>(smem_raw);
@@ -378,16 +390,6 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
     }
     if (t0 < t1) issue_ktile<KT>(S.Vr[0], p.V, p.ldw, rbase + t0 * UB, p.r_hi, K);
     cp_async_commit();
-    if (p.endcheck) {
-        // frozen row sums of the panel columns k..e-1 (final now, untouched by this kernel; R6):
-        // Fr(i) += sum_{col in [k,e), i <= col+1} A(i, col) for i <= e
-        const int k = p.r_lo - 1, e = p.c_lo;
-        const int nb = gridDim.x * gridDim.y, b = blockIdx.y * gridDim.x + blockIdx.x;
-        for (int i = b * UT + tid; i <= e && i < p.n; i += nb * UT) {
-            const int c0 = i - 1 > k ? i - 1 : k;  // columns col >= i - 1 hold row i's H entries
-            p.Fr[i] += c0 < e ? sum_strided(p.A + i + (int64_t)c0 * p.lda, p.lda, e - c0) : 0.0;
-        }
-    }
     int cols[2];
     bool colok[2];
     double *colp[2];
@@ -397,6 +399,21 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
         colok[mi] = cols[mi] < ncols;
         colp[mi] = p.A + (int64_t)(cb + (colok[mi] ? cols[mi] : 0)) * p.lda;
     }
+    auto load_c = [&](int tt, double2 (&dst)[2][4]) {
+        const int r = rbase + tt * UB;
+        const int lo = max(r, p.r_lo), hi = min(r + UB, p.r_hi);
+        const bool full = lo == r && hi == r + UB && ncols == UB;
+#pragma unroll
+        for (int mi = 0; mi < 2; mi++)
+#pragma unroll
+            for (int ni = 0; ni < 4; ni++) {
+                const int row = r + wr * 32 + ni * 8 + 2 * lc;
+                dst[mi][ni] = full ? *reinterpret_cast<const double2 *>(colp[mi] + row)
+                                   : load_pair(colp[mi], row, lo, hi, colok[mi]);
+            }
+    };
+    double2 cn[2][4];  // the next tile's C, prefetched a whole tile ahead
+    if (t0 < t1) load_c(t0, cn);
     for (int tt = t0; tt < t1; tt++) {
         const int st = (tt - t0) & 1;
         const int r = rbase + tt * UB;
@@ -407,12 +424,10 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
         for (int mi = 0; mi < 2; mi++)
 #pragma unroll
             for (int ni = 0; ni < 4; ni++) {
-                const int row = r + wr * 32 + ni * 8 + 2 * lc;
-                const double2 c = full ? *reinterpret_cast<const double2 *>(colp[mi] + row)
-                                       : load_pair(colp[mi], row, lo, hi, colok[mi]);
-                acc[mi][ni][0] = sg * c.x;
-                acc[mi][ni][1] = sg * c.y;
+                acc[mi][ni][0] = sg * cn[mi][ni].x;
+                acc[mi][ni][1] = sg * cn[mi][ni].y;
             }
+        if (tt + 1 < t1) load_c(tt + 1, cn);
         if (tt + 1 < t1) issue_ktile<KT>(S.Vr[st ^ 1], p.V, p.ldw, r + UB, p.r_hi, K);
         cp_async_commit();
         cp_async_wait<1>();
@@ -441,6 +456,16 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
         __syncthreads();  // Vr[st] is refilled two tiles later
     }
     cp_async_wait<0>();
+    if (p.endcheck) {  // (after the tiles: off the C-load critical path)
+        // frozen row sums of the panel columns k..e-1 (final now, untouched by this kernel; R6):
+        // Fr(i) += sum_{col in [k,e), i <= col+1} A(i, col) for i <= e
+        const int k = p.r_lo - 1, e = p.c_lo;
+        const int nb = gridDim.x * gridDim.y, b = blockIdx.y * gridDim.x + blockIdx.x;
+        for (int i = b * UT + tid; i <= e && i < p.n; i += nb * UT) {
+            const int c0 = i - 1 > k ? i - 1 : k;  // columns col >= i - 1 hold row i's H entries
+            p.Fr[i] += c0 < e ? sum_strided(p.A + i + (int64_t)c0 * p.lda, p.lda, e - c0) : 0.0;
+        }
+    }
     if (!p.endcheck) return;
     // fused end-of-iteration check (Alg. 3 l.12-13; R11/R22): once every CTA has finished, the
     // last one compares sum r and sum c with kappa (EAGER) or with each other (PAPER)

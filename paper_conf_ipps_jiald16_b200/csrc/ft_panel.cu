@@ -303,20 +303,8 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
         PROBE(0);
         // ---------------- (i) b0 = A(:,c) - Y V(c,:)^T, s1 = V^T b0 ---------------------------
         if (j > 0) {
-#pragma unroll 1
-            for (int base = 0; base < R; base += NSLOT) {
-                if (base + 4 * wid >= R) break;  // no rows for this warp (warp-uniform)
-                const int rl = base + slot;
-                const double yv = rowdot(Yl, rl, S.vrow, j);
-                if (rl < R && g == 0) {
-                    const double b0 = S.acol[rl] - yv;
-                    S.b0[rl] = b0;
-                    S.bm[rl] = is_data(r0 + rl) ? b0 : 0.0;
-                }
-            }
-            PROBE(10);
-            __syncthreads();
-            PROBE(11);
+            // b0 = A(:, c) - Y V(c, :)^T of the own rows was formed by the previous column's
+            // step (v) (S.b0 / S.bm): only the column dots remain here
             coldot_add(Vl, S.bm, j, false, acc, 0, 0);
             PROBE(1);
             grid_sync(epoch, [&]() {
@@ -584,24 +572,34 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
         {
             const double tau = S.scal[0], scale = S.scal[2];
             const bool vfy = (j == 0) && p.verify;
-            {   // T(a, j) = -tau * sum_{b=a}^{j-1} T(a, b) t(b), T(j, j) = tau (8 lanes per a)
-                double s0 = 0.0, s1 = 0.0;
-                if (4 * wid < j) {
-                if (slot < j)
-#pragma unroll
-                    for (int u = 0; u < FT_NBMAX / 8; u += 2) {
-                        const int ba = slot + g + 8 * u, bb = ba + 8;
-                        if (ba < j) s0 += S.Ts[slot][ba] * S.t[ba];
-                        if (bb < j) s1 += S.Ts[slot][bb] * S.t[bb];
-                    }
-                const double s = group8_sum(s0 + s1);
-                if (slot < j && g == 0) S.Ts[slot][j] = -tau * s;
-                }
-                if (tid == 0) S.Ts[j][j] = tau;
-            }
-            PROBE(12);
+            // small row blocks: the T column (warps 8..15) runs beside the Y rows (warps 0..7)
+            const bool split = R <= 32;
+            if (!split || wid >= 8) {
+                // T(a, j) = -tau * sum_{b=a}^{j-1} T(a, b) t(b), T(j, j) = tau (8 lanes per a)
+                const int tslot = split ? slot - 32 : slot, tw = split ? wid - 8 : wid;
+                const int nsl = split ? 32 : NSLOT;
 #pragma unroll 1
-            for (int base = 0; base < R; base += NSLOT) {
+                for (int a0 = 0; a0 < j; a0 += nsl) {
+                    if (a0 + 4 * tw >= j) break;  // warp-uniform
+                    const int a = a0 + tslot;
+                    double s0 = 0.0, s1 = 0.0;
+                    if (a < j)
+#pragma unroll
+                        for (int u = 0; u < FT_NBMAX / 8; u += 2) {
+                            const int ba = a + g + 8 * u, bb = ba + 8;
+                            if (ba < j) s0 += S.Ts[a][ba] * S.t[ba];
+                            if (bb < j) s1 += S.Ts[a][bb] * S.t[bb];
+                        }
+                    const double sT = group8_sum(s0 + s1);
+                    if (a < j && g == 0) S.Ts[a][j] = -tau * sT;
+                }
+            }
+            if (tid == 0) S.Ts[j][j] = tau;
+            PROBE(12);
+            const int rslots = split ? 32 : NSLOT;
+#pragma unroll 1
+            for (int base = 0; base < R; base += rslots) {
+                if (split && wid >= 8) break;
                 if (base + 4 * wid >= R) break;
                 const int rl = base + slot;
                 const bool on = rl < R && is_valid(r0 + rl);
@@ -633,23 +631,37 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
                         }
                     }
                 }
+                // with the same Y row loads: P1 = Y(rl, :) V(c+1, :)^T (S.vrow), which gives the
+                // next column's b0 = A(:, c+1) - Y(:, 0:j) V(c+1, 0:j)^T = an - P1 - Y(:, j)
+                double pa = 0.0, pb = 0.0;
                 if (on) {
 #pragma unroll
                     for (int u = 0; u < FT_NBMAX / 8; u += 2) {
                         const int ja = g + 8 * u, jb = ja + 8;
-                        if (ja < j) ya -= Yl[rl * XR + ja * XC] * S.t[ja];
-                        if (jb < j) yb -= Yl[rl * XR + jb * XC] * S.t[jb];
+                        if (ja < j) {
+                            const double yv = Yl[rl * XR + ja * XC];
+                            ya -= yv * S.t[ja];
+                            pa += yv * S.vrow[ja];
+                        }
+                        if (jb < j) {
+                            const double yv = Yl[rl * XR + jb * XC];
+                            yb -= yv * S.t[jb];
+                            pb += yv * S.vrow[jb];
+                        }
                     }
                 }
                 const double ysum = group8_sum(ya + yb);
+                const double p1 = group8_sum(pa + pb);
                 if (vfy) rsum = group8_sum(rsum);
                 if (rl < R && g == 0) {
                     const int row = r0 + rl;
                     const double an = (MG && c + 1 >= p.e) ? an_mg : S.anext[rl];
+                    double b0n = 0.0;
                     if (on) {
                         const double yy = tau * (an + ysum);
                         Y[row + (int64_t)j * ldw] = yy;
                         if (CACHE) Yl[rl * XR + j * XC] = yy;
+                        b0n = an - p1 - yy;
                         if (vfy && is_data(row)) {
                             // D_r(row) = r(row) - sum_{col >= k} L(row, col); columns < k are logical zero
                             rsum += S.acol[rl] + an;
@@ -663,6 +675,8 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
                         }
                     }
                     S.acol[rl] = an;
+                    S.b0[rl] = b0n;
+                    S.bm[rl] = is_data(row) ? b0n : 0.0;
                 }
             }
             PROBE(13);
