@@ -25,10 +25,10 @@
 #define UT 256  // threads (8 warps)
 #define SK 68   // smem stride of the k-major operand tiles
 
-// Row splits per strip: minimise waves * tiles-per-CTA for one resident CTA per SM (the
-// grid is nstrip x ns CTAs; a ragged last wave idles SMs).
-static int best_splits(int nstrip, int nrt, int nsm, int cap) {
-    const int slots = nsm;  // one CTA per SM (the C tile of the next iteration is prefetched in registers)
+// Row splits per strip: minimise waves * tiles-per-CTA for per_sm resident CTAs per SM
+// (the grid is nstrip x ns CTAs; a ragged last wave idles SMs).
+static int best_splits(int nstrip, int nrt, int nsm, int cap, int per_sm) {
+    const int slots = per_sm * nsm;
     int best = 1;
     long long best_cost = -1;
     for (int ns = 1; ns <= cap && ns <= nrt; ns++) {
@@ -44,7 +44,8 @@ static int best_splits(int nstrip, int nrt, int nsm, int cap) {
 int ft_gemm_splits(int r_lo, int r_hi, int c_lo, int c_hi, int nsm) {
     const int nstrip = (c_hi - c_lo + UB - 1) / UB;
     const int nrt = (r_hi - (r_lo / UB) * UB + UB - 1) / UB;
-    return best_splits(nstrip > 0 ? nstrip : 1, nrt > 0 ? nrt : 1, nsm, FT_WSPLIT_MAX);
+    // right update: one CTA per SM (the next C tile is prefetched in registers)
+    return best_splits(nstrip > 0 ? nstrip : 1, nrt > 0 ? nrt : 1, nsm, FT_WSPLIT_MAX, 1);
 }
 
 template <int KT>
@@ -366,7 +367,7 @@ __global__ void k_wprep(const double *__restrict__ Wpart, int64_t wstride, int n
 }
 
 template <int KT>
-__global__ void __launch_bounds__(UT, 1) k_gemm_left(GemmLeftParams p) {
+__global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
     if (p.ctl && p.ctl->halt) return;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     LeftSmemT<KT> &S = *reinterpret_cast<LeftSmemT<KT> *>(smem_raw);
@@ -399,21 +400,6 @@ __global__ void __launch_bounds__(UT, 1) k_gemm_left(GemmLeftParams p) {
         colok[mi] = cols[mi] < ncols;
         colp[mi] = p.A + (int64_t)(cb + (colok[mi] ? cols[mi] : 0)) * p.lda;
     }
-    auto load_c = [&](int tt, double2 (&dst)[2][4]) {
-        const int r = rbase + tt * UB;
-        const int lo = max(r, p.r_lo), hi = min(r + UB, p.r_hi);
-        const bool full = lo == r && hi == r + UB && ncols == UB;
-#pragma unroll
-        for (int mi = 0; mi < 2; mi++)
-#pragma unroll
-            for (int ni = 0; ni < 4; ni++) {
-                const int row = r + wr * 32 + ni * 8 + 2 * lc;
-                dst[mi][ni] = full ? *reinterpret_cast<const double2 *>(colp[mi] + row)
-                                   : load_pair(colp[mi], row, lo, hi, colok[mi]);
-            }
-    };
-    double2 cn[2][4];  // the next tile's C, prefetched a whole tile ahead
-    if (t0 < t1) load_c(t0, cn);
     for (int tt = t0; tt < t1; tt++) {
         const int st = (tt - t0) & 1;
         const int r = rbase + tt * UB;
@@ -424,10 +410,12 @@ __global__ void __launch_bounds__(UT, 1) k_gemm_left(GemmLeftParams p) {
         for (int mi = 0; mi < 2; mi++)
 #pragma unroll
             for (int ni = 0; ni < 4; ni++) {
-                acc[mi][ni][0] = sg * cn[mi][ni].x;
-                acc[mi][ni][1] = sg * cn[mi][ni].y;
+                const int row = r + wr * 32 + ni * 8 + 2 * lc;
+                const double2 c = full ? *reinterpret_cast<const double2 *>(colp[mi] + row)
+                                       : load_pair(colp[mi], row, lo, hi, colok[mi]);
+                acc[mi][ni][0] = sg * c.x;
+                acc[mi][ni][1] = sg * c.y;
             }
-        if (tt + 1 < t1) load_c(tt + 1, cn);
         if (tt + 1 < t1) issue_ktile<KT>(S.Vr[st ^ 1], p.V, p.ldw, r + UB, p.r_hi, K);
         cp_async_commit();
         cp_async_wait<1>();
@@ -535,7 +523,7 @@ static cudaError_t launch_left_kt(const GemmLeftParams &p, cudaStream_t s) {
         cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
     }
     const int nrt = (p.r_hi - (p.r_lo / UB) * UB + UB - 1) / UB;
-    const int ny = best_splits(nstrip, nrt, nsm, 1 << 20);
+    const int ny = best_splits(nstrip, nrt, nsm, 1 << 20, 2);  // two resident CTAs per SM
     if (!p.wt_ready) {
         g_ft_launches++;
         const int per = UT / FT_NBMAX;  // columns per k_wprep block
