@@ -490,7 +490,7 @@ int checkpoint(Call &C, int t, int restore) {
     return 0;
 }
 
-int right_update(Call &C, int t, double sign, int do_w) {
+int right_update(Call &C, int t, double sign, int do_w, bool precheck = false) {
     Work &w = *C.w;
     const int k = C.pk(t), ib = C.pib(t), e = k + ib;
     GemmRightParams g{};
@@ -526,11 +526,16 @@ int right_update(Call &C, int t, double sign, int do_w) {
         g.transT = 1;
         g.strip_done = w.strip_done;
     }
+    if (precheck) {  // fused pre-update check (R15), decided by every CTA before it touches A
+        g.pre_ctl = w.ctl;
+        g.pre_n = C.n;
+        g.pre_panel = t;
+    }
     CK(ft_launch_gemm_right(g, C.s));
     return 0;
 }
 
-int left_update(Call &C, int t, double sign, int nsplit, int endcheck = 0) {
+int left_update(Call &C, int t, double sign, int nsplit, int endcheck = 0, bool pre_reset = false) {
     Work &w = *C.w;
     const int k = C.pk(t), ib = C.pib(t), e = k + ib;
     GemmLeftParams g{};
@@ -558,6 +563,7 @@ int left_update(Call &C, int t, double sign, int nsplit, int endcheck = 0) {
     g.n = C.n;
     g.Fr = w.Fr;
     g.ectl = w.ctl;
+    g.pre_reset = pre_reset ? w.ctl : nullptr;
     CK(ft_launch_gemm_left(g, C.s));
     return 0;
 }
@@ -659,10 +665,10 @@ int enqueue_panel(Call &C, int t) {
         CK(ft_precheck(w.Y, w.V, w.ldw, n, C.ihi, k, ib, w.ctl, C.s));
         CK(ft_decide(w.Y, w.V, w.T, w.ldw, n, k, ib, t, w.ctl, C.s));
     }
-    if (right_update(C, t, -1.0, 1)) return FT_E_CUDA;
+    if (right_update(C, t, -1.0, 1, fuse_pre)) return FT_E_CUDA;
     if (inject_at(C, t, FT_PHASE_AFTER_RIGHT)) return FT_E_CUDA;
     const bool fuse_end = C.abft && !has_fault(C, t, FT_PHASE_AFTER_UPDATE);
-    if (left_update(C, t, -1.0, trailing_nsplit(C, t), fuse_end ? 1 : 0)) return FT_E_CUDA;
+    if (left_update(C, t, -1.0, trailing_nsplit(C, t), fuse_end ? 1 : 0, fuse_pre)) return FT_E_CUDA;
     if (inject_at(C, t, FT_PHASE_AFTER_UPDATE)) return FT_E_CUDA;
     if (C.abft && !fuse_end) CK(ft_endcheck(w.Aw, w.ldw, n, C.ihi, k, ib, t, C.policy, w.Fr, w.ctl, C.s));
     return 0;

@@ -90,9 +90,50 @@ __device__ __forceinline__ void store_pair(double *colp, int row, int lo, int hi
 // Right update A(rows, cols) += sign * Y V(cols,:)^T, fused W = V(wrows,:)^T A_new
 // warp w owns columns w*8 .. w*8+7 of the strip and all 64 rows of a tile (8 fragments)
 // ---------------------------------------------------------------------------
+// the fused pre-update check (R15), evaluated redundantly by warp 0 of every CTA on the same
+// inputs (so every CTA takes the same decision); returns the reason bits
+__device__ int pre_update_reason(const GemmRightParams &p) {
+    const FtCtl *ctl = p.pre_ctl;
+    const int lane = threadIdx.x & 31, n = p.pre_n, ib = p.K;
+    const double eps = 2.220446049250313e-16;
+    const double unit = (double)n * eps * ctl->normF;
+    const double tmax = __ldcg(&ctl->tmax);
+    const double tauY = ctl->c_thr * unit * (tmax > 1.0 ? tmax : 1.0);
+    const double tauV = ctl->c_thr * (double)n * eps * sqrt((double)n);
+    int reason = __ldcg(&ctl->nflag) > 0 ? 1 : 0;
+    for (int j = lane; j < ib; j += 32) {
+        const double dy = __ldcg(&ctl->eY[j]) - __ldcg(p.Y + n + (int64_t)j * p.ldw);
+        const double dv = __ldcg(&ctl->eV[j]) - __ldcg(p.V + n + (int64_t)j * p.ldw);
+        if (not_within(dy, tauY)) reason |= 2;
+        if (not_within(dv, tauV)) reason |= 4;
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) reason |= __shfl_xor_sync(0xffffffffu, reason, o);
+    return reason;
+}
+
 template <int KT>
 __global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
     if (p.ctl && p.ctl->halt) return;
+    if (p.pre_ctl) {
+        __shared__ int s_reason;
+        if (threadIdx.x < 32) {
+            const int reason = pre_update_reason(p);
+            if (threadIdx.x == 0) s_reason = reason;
+        }
+        __syncthreads();
+        if (s_reason) {
+            if (threadIdx.x == 0 && blockIdx.x == 0 && blockIdx.y == 0) {
+                FtCtl *ctl = p.pre_ctl;
+                ctl->halt_panel = p.pre_panel;
+                ctl->halt_stage = 1;
+                ctl->halt_reason = s_reason;
+                __threadfence();
+                ctl->halt = 1;
+            }
+            return;  // nothing consumed: the panel is redone from its checkpoint
+        }
+    }
     extern __shared__ __align__(16) unsigned char smem_raw[];
     RightSmemT<KT> &S = *reinterpret_cast<RightSmemT<KT> *>(smem_raw);
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -382,6 +423,13 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
     const int nrt = (p.r_hi - rbase + UB - 1) / UB;
     const int t0 = (int)((long long)blockIdx.y * nrt / gridDim.y);
     const int t1 = (int)((long long)(blockIdx.y + 1) * nrt / gridDim.y);
+    if (p.pre_reset && blockIdx.x == 0 && blockIdx.y == 0) {  // the right update has read them
+        for (int j = tid; j < FT_NBMAX; j += UT) {
+            p.pre_reset->eY[j] = 0.0;
+            p.pre_reset->eV[j] = 0.0;
+        }
+        if (tid == 0) p.pre_reset->nflag = 0;
+    }
 
     // W'^T for the strip: Wt [col][64] -> Wc[k][col] (asynchronous, with the first V tile)
     for (int i = tid; i < KT * UB; i += UT) {
@@ -447,11 +495,14 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
     if (p.endcheck) {  // (after the tiles: off the C-load critical path)
         // frozen row sums of the panel columns k..e-1 (final now, untouched by this kernel; R6):
         // Fr(i) += sum_{col in [k,e), i <= col+1} A(i, col) for i <= e
+        // one (row, 8-column chunk) per thread: a single round trip, partial sums by atomics
         const int k = p.r_lo - 1, e = p.c_lo;
+        const int nch = (e - k + 7) / 8, rows = min(e + 1, p.n);
         const int nb = gridDim.x * gridDim.y, b = blockIdx.y * gridDim.x + blockIdx.x;
-        for (int i = b * UT + tid; i <= e && i < p.n; i += nb * UT) {
-            const int c0 = i - 1 > k ? i - 1 : k;  // columns col >= i - 1 hold row i's H entries
-            p.Fr[i] += c0 < e ? sum_strided(p.A + i + (int64_t)c0 * p.lda, p.lda, e - c0) : 0.0;
+        for (int x = b * UT + tid; x < rows * nch; x += nb * UT) {
+            const int i = x % rows, q = x / rows;
+            const int c0 = max(i - 1 > k ? i - 1 : k, k + 8 * q), c1 = min(e, k + 8 * q + 8);
+            if (c0 < c1) atomicAdd(p.Fr + i, sum_strided(p.A + i + (int64_t)c0 * p.lda, p.lda, c1 - c0));
         }
     }
     if (!p.endcheck) return;
@@ -629,7 +680,6 @@ __global__ void __launch_bounds__(YF_R * 64) k_ytop_finalize(YtopParams p) {
     if (p.ctl->halt) return;
     __shared__ double Ts[FT_NBMAX * FT_NBMAX];
     __shared__ double y0[YF_R][FT_NBMAX + 1];
-    __shared__ int last;
     const int jb = threadIdx.x & 63, rl = threadIdx.x >> 6;
     const int row = blockIdx.x * YF_R + rl;
     const int ib = p.ib;
@@ -657,7 +707,7 @@ __global__ void __launch_bounds__(YF_R * 64) k_ytop_finalize(YtopParams p) {
         if (not_within(d, tau_abs)) atomicAdd(&p.ctl->nflag, 1);
     }
     if (!p.decide) return;
-    // fused pre-update check (reading R15): e^T Y of rows 0..k, then the last block decides
+    // fused pre-update check (reading R15): e^T Y of rows 0..k
     __syncthreads();
     y0[rl][jb] = yv;
     __syncthreads();
@@ -666,46 +716,7 @@ __global__ void __launch_bounds__(YF_R * 64) k_ytop_finalize(YtopParams p) {
         for (int q = 0; q < YF_R; q++) s += y0[q][jb];
         atomicAdd(&p.ctl->eY[jb], s);
     }
-    __threadfence();
-    __syncthreads();
-    if (threadIdx.x == 0) last = atomicAdd(&p.ctl->done_ytop, 1) == (int)gridDim.x - 1;
-    __syncthreads();
-    if (!last || threadIdx.x >= 32) return;
-    __threadfence();
-    FtCtl *ctl = p.ctl;
-    const int lane = threadIdx.x, n = p.n;
-    const double unit = (double)n * 2.220446049250313e-16 * ctl->normF;
-    double tmax = 0.0;
-    for (int i = lane; i < ib * ib; i += 32) tmax = fmax(tmax, fabs(Ts[(i % ib) + (i / ib) * FT_NBMAX]));
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) tmax = fmax(tmax, __shfl_xor_sync(0xffffffffu, tmax, o));
-    int reason = 0;
-    if (atomicAdd(&ctl->nflag, 0) > 0) reason |= 1;
-    const double tauY = ctl->c_thr * unit * (tmax > 1.0 ? tmax : 1.0);
-    const double tauV = ctl->c_thr * (double)n * 2.220446049250313e-16 * sqrt((double)n);
-    for (int j = lane; j < ib; j += 32) {
-        const double dy = __ldcg(&ctl->eY[j]) - p.Y[n + (int64_t)j * p.ldw];
-        const double dv = __ldcg(&ctl->eV[j]) - p.V[n + (int64_t)j * p.ldw];
-        if (not_within(dy, tauY)) reason |= 2;
-        if (not_within(dv, tauV)) reason |= 4;
-    }
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) reason |= __shfl_xor_sync(0xffffffffu, reason, o);
-    for (int j = lane; j < FT_NBMAX; j += 32) {
-        ctl->eY[j] = 0.0;
-        ctl->eV[j] = 0.0;
-    }
-    if (lane == 0) {
-        ctl->nflag = 0;
-        ctl->done_ytop = 0;
-        if (reason) {
-            ctl->halt_panel = p.panel;
-            ctl->halt_stage = 1;
-            ctl->halt_reason = reason;
-            __threadfence();
-            ctl->halt = 1;
-        }
-    }
+    // the decision itself is taken by every CTA of the right update (GemmRightParams::pre_ctl)
 }
 
 cudaError_t ft_launch_ytop(const YtopParams &p, cudaStream_t s) {

@@ -33,6 +33,7 @@ struct FtCtl {
     double eY[64];        // pre-update check sums (e^T Y)
     double eV[64];        // (e^T V)
     double sums[4];       // end check: sum r, sum c
+    double tmax;          // max |T| of the last panel (written by the panel kernel; pre-update tolerance)
     double inj_delta[FT_MAXFAULTS];
     int inj_done[FT_MAXFAULTS];
 };
@@ -104,6 +105,10 @@ struct GemmRightParams {
     // multi-rank column map: local column l of A is global column
     // ft_cmap(l) (the row of V it pairs with); cm_G <= 1 is the identity
     int cm_G, cm_rank, cm_nb, cm_ncl, cm_n;
+    // fused pre-update check (reading R15, EAGER): every CTA evaluates e^T Y = Y_chk, e^T V = V_chk
+    // and the fused D_r flag count before touching A; a failed check halts the whole launch
+    FtCtl *pre_ctl;  // non-NULL: evaluate the check (pre_n, pre_panel)
+    int pre_n, pre_panel;
 };
 // global column of local column l in the 1-D block-column cyclic layout; local column ncl
 // is the replicated row-checksum column r (global n)
@@ -134,6 +139,7 @@ struct GemmLeftParams {
     int endcheck, panel, policy, n;
     double *Fr;
     FtCtl *ectl;
+    FtCtl *pre_reset;  // non-NULL: CTA (0,0) clears the fused pre-update sums for the next panel
 };
 cudaError_t ft_launch_gemm_left(const GemmLeftParams &p, cudaStream_t s);
 

@@ -703,11 +703,25 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
         atomicAdd(tid < ib ? &p.ctl->eY[jj] : &p.ctl->eV[jj], s);
     }
     if (bid == 0 && tid == 0 && p.abft) p.Qc[n] += qc_corner;
-    if (bid == 0)
+    if (bid == 0) {
+        double tm = 0.0;
         for (int i = tid; i < ib * ib; i += PT) {
             int a = i % ib, bb = i / ib;
             p.T[a + bb * FT_NBMAX] = S.Ts[a][bb];
+            tm = fmax(tm, fabs(S.Ts[a][bb]));
         }
+        if (p.precheck_sums) {  // max |T| for the pre-update tolerance (R15), read by the right update
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) tm = fmax(tm, __shfl_xor_sync(0xffffffffu, tm, o));
+            if (lane == 0) S.red[wid].x = tm;
+            __syncthreads();
+            if (tid == 0) {
+                double m = 0.0;
+                for (int w = 0; w < NW; w++) m = fmax(m, S.red[w].x);
+                p.ctl->tmax = m;
+            }
+        }
+    }
 }
 
 cudaError_t ft_launch_panel_multi(const PanelLaunch &L, int nsm, cudaStream_t s) {
