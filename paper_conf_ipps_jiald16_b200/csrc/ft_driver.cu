@@ -79,7 +79,7 @@ struct Work {
     int n_cap = -1;
     int64_t ldw = 0;
     double *Wt = nullptr;
-    double *Aw = nullptr, *V = nullptr, *Y = nullptr, *T = nullptr, *Wpart = nullptr, *bvec = nullptr,
+    double *Aw = nullptr, *V = nullptr, *Y = nullptr, *Z = nullptr, *T = nullptr, *Wpart = nullptr, *bvec = nullptr,
            *acc = nullptr, *ckpt = nullptr, *ck_r = nullptr, *ck_c = nullptr, *ck_q = nullptr, *Fr = nullptr,
            *Qr = nullptr, *Qc = nullptr, *Dr = nullptr, *Dc = nullptr, *sums = nullptr, *ypart = nullptr,
            *rowpart = nullptr, *linepart = nullptr, *scratch = nullptr, *deltas = nullptr, *hA = nullptr, *htau = nullptr;
@@ -91,7 +91,7 @@ struct Work {
     int nsm = 0;
     size_t bytes = 0;
     void release() {
-        double **ps[] = {&Wt, &Aw, &V, &Y, &T, &Wpart, &bvec, &acc, &ckpt, &ck_r, &ck_c, &ck_q, &Fr, &Qr, &Qc, &Dr, &Dc,
+        double **ps[] = {&Wt, &Aw, &V, &Y, &Z, &T, &Wpart, &bvec, &acc, &ckpt, &ck_r, &ck_c, &ck_q, &Fr, &Qr, &Qc, &Dr, &Dc,
                          &sums, &ypart, &rowpart, &linepart, &scratch, &deltas, &hA, &htau};
         for (auto p : ps) {
             if (*p) cudaFree(*p);
@@ -169,7 +169,8 @@ int get_work(int n, Work **out) {
     A(dalloc(&w.T, (size_t)FT_NBMAX * FT_NBMAX, b));
     A(dalloc(&w.Wpart, (size_t)kMaxWsplit * (N1 + 64) * FT_NBMAX, b));
     A(dalloc(&w.Wt, (N1 + 64) * FT_NBMAX, b));
-    A(dalloc(&w.bvec, (size_t)ldw, b));
+    A(dalloc(&w.Z, (size_t)ldw * FT_NBMAX, b));
+    A(dalloc(&w.bvec, (size_t)4 * ldw, b));
     A(dalloc(&w.acc, (size_t)FT_ACC_SETS * FT_ACC_SET_DOUBLES, b));
     A(dalloc(&w.ckpt, (size_t)ldw * FT_NBMAX, b));
     A(dalloc(&w.ck_r, (size_t)ldw, b));
@@ -602,6 +603,7 @@ int enqueue_panel(Call &C, int t) {
     p.T = w.T;
     p.tau = C.tau;
     p.bvec = w.bvec;
+    p.Z = w.Z;
     p.acc = w.acc;
     p.bar = w.bar + (t & 1);
     p.bar_next = w.bar + ((t + 1) & 1);
@@ -799,7 +801,7 @@ int enqueue_start(Call &C, const double *dA, int lda) {
     CK(cudaMemsetAsync(w.V, 0, (size_t)w.ldw * FT_NBMAX * sizeof(double), s));
     CK(cudaMemsetAsync(w.Y, 0, (size_t)w.ldw * FT_NBMAX * sizeof(double), s));
     CK(ft_copy_in(dA, lda, w.Aw, w.ldw, n, s));
-    CK(cudaMemsetAsync(w.bvec, 0, (size_t)w.ldw * sizeof(double), s));  // b(q >= ihi) must read 0
+    CK(cudaMemsetAsync(w.bvec, 0, (size_t)4 * w.ldw * sizeof(double), s));  // b(q >= ihi) must read 0
     if (reset_panel_state(C)) return FT_E_CUDA;
     if (C.abft) {
         CK(ft_encode(w.Aw, w.ldw, n, w.ctl, w.scratch, w.linepart, s));

@@ -12,7 +12,7 @@
 #ifndef FT_NBMAX
 #define FT_NBMAX 64
 #endif
-#define FT_ACC_STRIDE (2 * 64 + 8)  // [s1 | vtb | nrm2 sx alpha ...] per reduction set
+#define FT_ACC_STRIDE (3 * 64 + 8)  // [s1 | sx | scalars | V^T x] per reduction set (ft_panel.cu ACC_*)
 #define FT_ACC_SETS 4               // sets indexed by the global column mod 4 (recycled in-kernel)
 #define FT_ACC_PAD 32               // doubles between accumulators: one 256-byte block (own L2 slice) each
 #define FT_ACC_SET_DOUBLES (FT_ACC_STRIDE * FT_ACC_PAD)
@@ -41,7 +41,9 @@ struct FtCtl {
 struct PanelParams {
     double *A;
     int64_t ldw;
-    double *V, *Y, *T, *tau, *bvec, *acc;
+    double *V, *Y, *T, *tau, *acc;
+    double *bvec;        // [4][ldw]: b0 of columns c (parity c & 1), x of the explicit path (2 + parity)
+    double *Z;           // ldw x FT_NBMAX: A(:, c+2:) V_x of the own rows when they do not fit in smem
     unsigned *bar;       // grid-barrier counter of this launch (zero at launch)
     unsigned *bar_next;  // the next panel launch's counter (zeroed by this launch)
     FtCtl *ctl;
@@ -52,7 +54,8 @@ struct PanelParams {
     double *ckpt, *ck_r, *ck_c, *ck_q, *Fr;
     int precheck_sums;  // add e^T Y, e^T V of the own rows into ctl->eY / eV (fused pre-update check)
     unsigned long long *dbg;          // optional per-column phase timestamps (CTA 0), or NULL
-    int dbg_mode;                     // timing ablations (wrong results): 1 no grid barriers, 2 no GEMV, 4 no atomics
+    int dbg_mode;                     // timing ablations (wrong results): 1 no grid barriers, 2 no GEMV, 4 no atomics;
+                                      // 8: every column on the explicit (two-reduction) path (exact)
     // panel columns: Apan[row + c * ldw] is panel column c (k <= c < k + ib); == A on one GPU.
     // rcol: the row-checksum column r.
     double *Apan, *rcol;

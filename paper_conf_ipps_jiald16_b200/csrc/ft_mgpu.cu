@@ -243,7 +243,7 @@ SymLayout sym_layout(int64_t ldw, int G) {
 struct MgRank {
     int dev = -1, n_cap = -1, G = 0, rank = 0;
     int64_t ldw = 0;
-    double *Aw = nullptr, *V = nullptr, *Y = nullptr, *T = nullptr, *Wpart = nullptr, *Wt = nullptr, *bvec = nullptr,
+    double *Aw = nullptr, *V = nullptr, *Y = nullptr, *Z = nullptr, *T = nullptr, *Wpart = nullptr, *Wt = nullptr, *bvec = nullptr,
            *acc = nullptr, *Qr = nullptr, *Qc = nullptr, *ypart = nullptr, *rowpart = nullptr, *vec = nullptr,
            *vec2 = nullptr;
     unsigned *bar = nullptr;
@@ -265,7 +265,7 @@ struct MgRank {
     unsigned *flags(int g) const { return reinterpret_cast<unsigned *>(peer[g] + lay.flags); }
     unsigned *xflags(int g) const { return reinterpret_cast<unsigned *>(peer[g] + lay.xflags); }
     void release() {
-        double **ps[] = {&Aw, &V, &Y, &T, &Wpart, &Wt, &bvec, &acc, &Qr, &Qc, &ypart, &rowpart, &vec, &vec2};
+        double **ps[] = {&Aw, &V, &Y, &Z, &T, &Wpart, &Wt, &bvec, &acc, &Qr, &Qc, &ypart, &rowpart, &vec, &vec2};
         for (auto p : ps) {
             if (*p) cudaFree(*p);
             *p = nullptr;
@@ -311,7 +311,8 @@ int mg_alloc(MgRank &R, int n, int G, int rank) {
     A(cudaMalloc(&R.T, (size_t)FT_NBMAX * FT_NBMAX * sizeof(double)));
     A(cudaMalloc(&R.Wpart, (size_t)kMaxWsplitM * (N1 + 64) * FT_NBMAX * sizeof(double)));
     A(cudaMalloc(&R.Wt, (N1 + 64) * FT_NBMAX * sizeof(double)));
-    A(cudaMalloc(&R.bvec, (size_t)ldw * sizeof(double)));
+    A(cudaMalloc(&R.Z, (size_t)ldw * FT_NBMAX * sizeof(double)));
+    A(cudaMalloc(&R.bvec, (size_t)4 * ldw * sizeof(double)));
     A(cudaMalloc(&R.acc, (size_t)FT_ACC_SETS * FT_ACC_SET_DOUBLES * sizeof(double)));
     A(cudaMalloc(&R.Qr, (size_t)ldw * sizeof(double)));
     A(cudaMalloc(&R.Qc, (size_t)ldw * sizeof(double)));
@@ -412,7 +413,7 @@ int mg_run(MgCall &C, ft_report *rep) {
         CK(cudaMemsetAsync(R.Aw, 0, (size_t)ldw * (ncl + 1) * sizeof(double), s));
         CK(cudaMemsetAsync(R.V, 0, (size_t)ldw * FT_NBMAX * sizeof(double), s));
         CK(cudaMemsetAsync(R.Y, 0, (size_t)ldw * FT_NBMAX * sizeof(double), s));
-        CK(cudaMemsetAsync(R.bvec, 0, (size_t)ldw * sizeof(double), s));
+        CK(cudaMemsetAsync(R.bvec, 0, (size_t)4 * ldw * sizeof(double), s));
         CK(cudaMemsetAsync(R.bar, 0, 4 * sizeof(unsigned), s));
         CK(cudaMemsetAsync(R.acc, 0, (size_t)FT_ACC_SETS * FT_ACC_SET_DOUBLES * sizeof(double), s));
         CK(cudaMemsetAsync(R.Qr, 0, ldw * sizeof(double), s));
@@ -481,6 +482,7 @@ int mg_run(MgCall &C, ft_report *rep) {
             p.T = R.T;
             p.tau = C.dtau[q];
             p.bvec = R.bvec;
+            p.Z = R.Z;
             p.acc = R.acc;
             p.bar = R.bar + (t & 1);
             p.bar_next = R.bar + ((t + 1) & 1);

@@ -3,10 +3,10 @@
 // One cooperative launch factorizes one panel of ib columns (DLAHR2, Alg. 2 l.4 /
 // Alg. 3 l.5; LAPACK reading R2).  For column c = k + j:
 //   (i)   b0 = A(k+1:n, c) - Y(k+1:n, 0:j) V(c, 0:j)^T                [row-local]
-//   (ii)  b  = b0 - V T^T (V^T b0)                                    [grid sync #1: s1 = V^T b0]
-//   (iii) DLARFG on (b(c+1), b(c+2:n)) -> beta, tau, v                [grid sync #2: ||x||^2, V^T x, e^T x]
-//   (iv)  y = A(k+1:n, c+1:ihi) v   -- the trailing GEMV, ~83% of the  [row-split, no reduction]
-//         roofline time of the whole reduction
+//   (ii)  b  = b0 - V T^T (V^T b0)
+//   (iii) DLARFG on (b(c+1), b(c+2:n)) -> beta, tau, v
+//   (iv)  y = A(k+1:n, c+1:ihi) v   -- the trailing GEMV, ~83% of the roofline time of the
+//         whole reduction
 //   (v)   t = V^T v, Y(:, j) = tau (y - Y t), T(0:j, j) = -tau T t, T(j,j) = tau
 // With ABFT the checksum row n rides as one more row of b / Y / V (V_aug(n,:) =
 // e^T V = V_chk, Y_aug(n,:) = e^T Y = Y_chk; Alg. 3 l.6-7, readings R7/R8), and the
@@ -14,28 +14,45 @@
 // row-checksum discrepancy D_r = r - L e is evaluated BEFORE the panel's output is
 // consumed by the updates (verify-before-consume, reading R11/R14).
 //
-// Latency design (the column chain is serial: n-2 dependent steps, SURVEY 7 "hard parts"):
-//  * rows [rbase, rend) are split into 8-row groups, contiguous per CTA; each CTA owns
-//    its rows for the whole panel (b, V, Y rows cached in shared memory), so y needs no
-//    cross-CTA reduction and every small dot is a CTA partial + one fp64 atomic;
-//  * warp 0 is the CONTROL warp: it runs the whole column chain (i)-(iii), (v) warp-
-//    synchronously (lane = row for row dots, lane = output for column dots, no CTA-wide
-//    barriers) and the two grid syncs per column; warps 1..15 only stream A for the
-//    GEMV.  The two roles meet at two named barriers per column (GO, DONE);
-//  * the GEMV runs on the UNSCALED b right after sync #2,
-//        y = A(:, c+1) + scale * A(:, c+2:ihi) b(c+2:ihi),   scale = 1/(alpha - beta),
-//    while the control warp evaluates DLARFG, T(:, j) and the stores of V(:, j) and the
-//    reduced column, so only the Y(:, j) step follows the GEMV on the critical path;
-//  * accumulator sets are indexed by the global column (mod 4) and recycled in-kernel,
-//    barrier counters alternate between consecutive panel launches: no memsets per panel.
+// ONE grid-wide reduction per column (the column chain is serial: n-2 dependent steps, and a
+// grid sync with its reduction costs ~2 us on B200, profiles/r01/mb_sync*.txt, mb_ll.txt).
+// Steps (ii)-(iii) are evaluated from b0 alone: the CTAs reduce s1 = V^T b0, sx = V_x^T b0_x,
+// bb = ||b0_x||^2 and e^T b0_x (x = rows >= c+2), and every CTA derives, with w = T^T s1,
+//     ||x||^2 = bb - 2 w.sx + w^T G w,   G = V_x^T V_x (Gram, carried and downdated per column)
+//     alpha = b0(c+1) - V(c+1,:) w,      t = V^T v = V(c+1,:)^T + scale (sx - G w)
+// and the GEMV runs on b0 itself (it was published before the sync):
+//     y = A(:, c+1) + scale (A(:, c+2:) b0_x - Z w),   Z = A(:, c+2:) V_x  (carried per row)
+// A cancellation guard (||x||^2 < (bb + w^T G w)/64) sends a column to the explicit path
+// (x = b0 - V w published, second reduction, GEMV on x): identical results up to rounding.
+// scripts/proto_onesync.py checks the algebra against the plain loop.
+//
+// Layout: rows [rbase, rend) are split into 8-row groups, contiguous per CTA; each CTA owns
+// its rows for the whole panel (b, V, Y, Z rows cached in shared memory when they fit), so y
+// needs no cross-CTA reduction.  After the sync warps 1..15 stream A for the GEMV while
+// warp 0 evaluates the column's scalars; the combine (an 8-lane group per row) then forms
+// V(:, j), Y(:, j), Z(:, j) and the next column's b0 and its reduction partials.
+// Accumulator sets are indexed by the global column (mod 4) and recycled in-kernel,
+// barrier counters alternate between consecutive panel launches: no memsets per panel.
 #include "ft_common.cuh"
 #include "ft_internal.h"
 
+#include <cstdio>
 #include <cstdlib>
 
 #define PT 512        // threads per CTA
 #define NW (PT / 32)  // warps per CTA
-#define NGW (NW - 1)  // GEMV warps (warp 0 is the control warp)
+// GEMV warps: the 12 warps of SM sub-partitions 1..3 (warp w runs on sub-partition w % 4).
+// Sub-partition 0 (warps 0, 4, 8, 12) is kept free of the GEMV's load flood, so the control
+// warp's shared-memory chain is not queued behind it.
+#define NGW (3 * NW / 4)
+#define IS_GEMV_WARP(w) (((w) & 3) != 0)
+#define GEMV_IDX(w) ((w) - ((w) >> 2) - 1)
+// helpers: warps 4, 8, 12 (sub-partition 0, no GEMV) form T(:, j) and the carried Gram while the
+// GEMV streams and then stay detached until the next grid sync; the other 13 warps ("workers",
+// index wid - wid / 4) run the combine and the column dots, synchronised by named barrier 2
+#define IS_HELPER(w) (((w) & 3) == 0 && (w) != 0)
+#define NWK (NW - NW / 4 + 1)  // worker warps
+#define WKT (32 * NWK)         // worker threads
 #define GR 8          // row-group granularity (64 bytes of a column)
 #define VS 65         // shared-memory row stride of the V / Y row caches (doubles)
 #define RMAX PT       // max rows per CTA
@@ -43,28 +60,36 @@
 #ifndef GB
 #define GB 8          // GEMV load batch (double2 of A + b per lane)
 #endif
+#define GAMMA (1.0 / 64.0)  // cancellation guard of the one-reduction column (see above)
 
-// accumulator set layout (FT_ACC_STRIDE doubles): [0,64) s1 = V^T b0 | [64,128) V^T x |
-// 128 ||x||^2 | 129 e^T x | 130 alpha
-#define ACC_VTB 64
-#define ACC_NRM 128
-#define ACC_SX 129
-#define ACC_ALPHA 130
+// accumulator set layout (FT_ACC_STRIDE doubles, each accumulator on its own 256-byte block)
+#define ACC_S1 0      // [0, 64)   s1 = V^T b0 (data rows)
+#define ACC_SX 64     // [64, 128) V_x^T b0_x (data rows >= c+2)
+#define ACC_BB 128    // b0_x . b0_x
+#define ACC_EB 129    // e^T b0_x
+#define ACC_B0 130    // b0(c+1) (single writer: the row's owner)
+#define ACC_FNRM 131  // explicit path: ||x||^2
+#define ACC_FEX 132   //                e^T x
+#define ACC_FAL 133   //                alpha = b(c+1) (single writer)
+#define ACC_FVX 136   // [136, 200)     V^T x
+static_assert(ACC_FVX + FT_NBMAX <= FT_ACC_STRIDE, "accumulator set too small");
+
+enum { SC_TAU, SC_BETA, SC_SCALE, SC_ALPHA, SC_VCHK, SC_Q, SC_XX, SC_FB };
 
 struct PanelSmem {
     double Ts[FT_NBMAX][FT_NBMAX + 1];  // Ts[a][b] = T(a, b)
-    double vrow[FT_NBMAX];              // V(c, 0:j) of the current column
-    double w[FT_NBMAX];                 // T^T s1
-    double t[FT_NBMAX];                 // V^T v
-    double s1[FT_NBMAX];                // V^T b0 (reduced)
-    double scal[8];                     // tau, beta, scale, vchk, alpha
+    double Gp[FT_NBMAX][FT_NBMAX + 1];  // Gram of V over rows >= c+1 (downdated by row c+1 in use)
+    double s1[FT_NBMAX], w[FT_NBMAX], t[FT_NBMAX], ep[FT_NBMAX];  // ep: e^T V over rows >= c+1
+    double vr1[FT_NBMAX + 1];           // V(c+1, 0:j)
+    double scal[16];                    // SC_*
     double acol[RMAX];                  // A(row, c) of the own rows
     double anext[RMAX];                 // A(row, c+1)
-    double b0[RMAX];                    // b0 (rows), then b
-    double bm[RMAX];                    // masked b0 / x for the column dots
+    double b0[RMAX];                    // b0 of the current column
+    double bmA[RMAX];                   // b0 masked to the data rows
+    double bmX[RMAX];                   // b0 (or x) masked to the data rows >= c+2
     double2 red[PT];                    // GEMV partials  (y pairs)
     double2 rsr[PT];                    // GEMV partials  (row sums, verify pass)
-    // followed (dynamic part) by the CTA's rows of V and Y when they fit: [R][VS] each
+    // followed (dynamic part) by the CTA's rows of V, Y and Z when they fit: [R][VS] each
 };
 
 size_t ft_panel_smem_bytes() { return sizeof(PanelSmem); }
@@ -86,7 +111,7 @@ size_t ft_panel_smem_bytes() { return sizeof(PanelSmem); }
 struct Refl {
     double tau, beta, scale;
 };
-__device__ __noinline__ Refl dlarfg_scalars(double nrm2, double alpha, bool trivial) {
+__device__ __forceinline__ Refl dlarfg_scalars(double nrm2, double alpha, bool trivial) {
     Refl r;
     if (nrm2 == 0.0 || trivial) {
         r.tau = 0.0;  // H = I, x left untouched (it is zero)
@@ -94,26 +119,13 @@ __device__ __noinline__ Refl dlarfg_scalars(double nrm2, double alpha, bool triv
         r.scale = 1.0;
     } else {
         r.beta = -copysign(sqrt(alpha * alpha + nrm2), alpha);  // -sign(alpha) hypot(alpha, ||x||)
-        r.tau = (r.beta - alpha) / r.beta;
-        r.scale = 1.0 / (alpha - r.beta);
+        // tau = (beta - alpha) / beta, scale = 1 / (alpha - beta): two independent reciprocals
+        // (correctly rounded) instead of two dependent divisions
+        const double rb = __drcp_rn(r.beta), rs = __drcp_rn(alpha - r.beta);
+        r.tau = (r.beta - alpha) * rb;
+        r.scale = rs;
     }
     return r;
-}
-
-// sum_{jp < J} X[jp * cs] * z[jp] with four independent chains
-__device__ __forceinline__ double dotj(const double *X, int64_t cs, const double *z, int J) {
-    double s0 = 0.0, s1 = 0.0, s2 = 0.0, s3 = 0.0;
-    int jp = 0;
-#pragma unroll 1
-    for (; jp + 3 < J; jp += 4) {
-        s0 += X[jp * cs] * z[jp];
-        s1 += X[(jp + 1) * cs] * z[jp + 1];
-        s2 += X[(jp + 2) * cs] * z[jp + 2];
-        s3 += X[(jp + 3) * cs] * z[jp + 3];
-    }
-#pragma unroll 1
-    for (; jp < J; jp++) s0 += X[jp * cs] * z[jp];
-    return (s0 + s1) + (s2 + s3);
 }
 
 // 8-lane group sum (lanes g = 0..7 of an aligned group); every lane of the warp must call it
@@ -122,6 +134,55 @@ __device__ __forceinline__ double group8_sum(double v) {
     v += __shfl_xor_sync(0xffffffffu, v, 2);
     v += __shfl_xor_sync(0xffffffffu, v, 1);
     return v;
+}
+
+// T(:, j) and the carried Gram / e^T V of the next column, from the column's scalars in smem;
+// threads t0 = 0..nthr-1 (whole warps) of the calling warps take part.  It runs in helper
+// warps concurrently with the GEMV (and on the explicit path after it).  Out of line on purpose:
+// inlined into the column loop (as a lambda or a forceinline function) the T(j, j) store was
+// addressed from a register not yet defined for the current column (nvcc 12.9, sm_100a).
+__device__ __noinline__ void tcol_gram(PanelSmem &S, const int j, const int t0, const int nthr, const bool last) {
+    const double tau = S.scal[SC_TAU], scale = S.scal[SC_SCALE];
+    // T(a, j) = -tau sum_{b=a}^{j-1} T(a, b) t(b), an 8-lane group per a
+    const int sl = t0 >> 3, gg = t0 & 7, nsl = nthr >> 3;
+    for (int a0 = 0; a0 < j; a0 += nsl) {
+        const int a = a0 + sl;
+        double s0 = 0.0, s1 = 0.0;
+        if (a < j)
+#pragma unroll
+            for (int u = 0; u < FT_NBMAX / 8; u += 2) {
+                const int ba = gg + 8 * u, bb2 = ba + 8;
+                if (ba < j) s0 += S.Ts[a][ba] * S.t[ba];
+                if (bb2 < j) s1 += S.Ts[a][bb2] * S.t[bb2];
+            }
+        const double s = group8_sum(s0 + s1);
+        if (a < j && gg == 0) S.Ts[a][j] = -tau * s;
+    }
+    if (t0 == 0) S.Ts[j][j] = tau;
+    if (!last) {
+        // Gram of V over rows >= c+2 (the downdate by row c+1 of the matrix in use), new
+        // row/column j = t - V(c+1,:), scale^2 ||x||^2; the next column downdates by row c+2.
+        // Thread (a, half) updates half of row a: independent read-modify-writes, pipelined.
+        const double xx = S.scal[SC_XX];
+        const int J1 = j + 1;
+        for (int r = t0; r < 2 * J1; r += nthr) {
+            const int a = r >> 1, h = r & 1;
+            const double va = S.vr1[a];
+            if (a < j) {
+#pragma unroll 4
+                for (int b2 = h; b2 < j; b2 += 2) S.Gp[a][b2] -= va * S.vr1[b2];
+                if (h == 0) {
+                    const double g = S.t[a] - va;
+                    S.Gp[a][j] = g;
+                    S.Gp[j][a] = g;
+                }
+            } else if (h == 0) {
+                S.Gp[j][j] = scale * scale * xx;
+            }
+        }
+        // e^T V over rows >= c+2
+        for (int a = t0; a <= j; a += nthr) S.ep[a] = a < j ? S.ep[a] - S.vr1[a] : S.scal[SC_VCHK] - 1.0;
+    }
 }
 
 // system-scope flag helpers for the cross-rank exchange (peer memory over NVLink, or the
@@ -148,6 +209,8 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
 
     const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
     const int slot = tid >> 3, g = tid & 7;  // 8-lane groups: NSLOT row / output slots
+    const bool helper = IS_HELPER(wid);
+    const int widx = wid - (wid >> 2), wtid = widx * 32 + lane;  // worker warp / thread index
     const int g0 = (int)((long long)bid * p.ngroups / P);
     const int g1 = (int)((long long)(bid + 1) * p.ngroups / P);
     const int r0 = p.rbase + GR * g0, r1 = p.rbase + GR * g1;
@@ -159,9 +222,11 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
     double *__restrict__ V = p.V;
     double *__restrict__ Y = p.Y;
 
-    // own rows of V and Y: [rl][jp] in shared memory (write-through to global) when they fit
+    // own rows of V, Y and Z: [rl][jp] in shared memory (V, Y write-through to global) when
+    // they fit, else the global arrays (Z: p.Z)
     double *Vl = CACHE ? reinterpret_cast<double *>(smem_raw + sizeof(PanelSmem)) : V + r0;
     double *Yl = CACHE ? Vl + (int64_t)VS * R : Y + r0;
+    double *Zl = CACHE ? Yl + (int64_t)VS * R : p.Z + r0;
     constexpr int64_t XR = CACHE ? VS : 1;  // row stride
     const int64_t XC = CACHE ? 1 : ldw;     // column stride
 
@@ -180,7 +245,6 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
 
     // ---- CTA-parallel building blocks of the column chain --------------------------------
     // row dot of row rl (an 8-lane group per row): sum_{jp < J} X(rl, jp) z[jp], J <= 64.
-    // Fully unrolled with predication: all operand loads are in flight at once.
     auto rowdot = [&](const double *X, int rl, const double *z, int J) -> double {
         double s0 = 0.0, s1 = 0.0;
         if (rl < R) {
@@ -194,43 +258,52 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
         }
         return group8_sum(s0 + s1);
     };
-    // column dots over the own rows, CTA partial added into the accumulators:
-    // out[o] = sum_rl X(rl, o) zr[rl] (o < J); extras: out[J] = zr.zr, out[J+1] = sum zr.
-    // An aligned group of LPO lanes per output (4..32: ~2 rows per lane, LPO * outputs <= PT),
-    // lanes stride the rows, shuffle tree inside the warp; the group leader adds the CTA
-    // partial into the accumulator.  No shared-memory pass, no CTA barrier.
-    auto coldot_add = [&](const double *X, const double *zr, int J, bool extras, double *acc, int acc_o0,
-                          int acc_extra0) {
-        const int NO = J + (extras ? 2 : 0);
-        // lanes per output: ~2 rows per lane, at most 32, at most PT / NO (a power of two)
+    // column dots over the own rows of V, CTA partials added into the accumulators:
+    //   o < JA:            sum_rl V(rl, o) zA[rl]        -> acc[oA + o]
+    //   JA <= o < JA + JB: sum_rl V(rl, o - JA) zB[rl]   -> acc[oB + o - JA]
+    //   then zB.zB -> acc[oE], sum zB -> acc[oE + 1]
+    // An aligned group of LPO lanes per output (4..32, ~2 rows per lane), lanes stride the
+    // rows, shuffle tree inside the warp; the group leader adds the CTA partial.
+    auto coldot_add = [&](const double *zA, int JA, const double *zB, int JB, double *acc, int oA, int oB,
+                          int oE) {
+        const int NO = JA + JB + 2;
         int LPO = 4;
-        while (LPO < 32 && 2 * LPO < R && (2 * LPO) * NO <= PT) LPO *= 2;
-        const int o = tid / LPO, gl = tid & (LPO - 1);
-        if ((wid * 32) / LPO >= NO) return;  // warp without outputs (warp-uniform)
-        double s = 0.0;
-        if (o < NO) {
-            double s1 = 0.0;
+        while (LPO < 32 && 2 * LPO < R && (2 * LPO) * NO <= WKT) LPO *= 2;
+        if (helper) return;
+        // output blocks of WKT / LPO (two when 4 lanes per output do not cover NO <= 128)
 #pragma unroll 1
-            for (int rb = gl; rb < R; rb += 4 * LPO) {
+        for (int ob = 0; ob < NO; ob += WKT / LPO) {
+            const int o = ob + wtid / LPO, gl = wtid & (LPO - 1);
+            if (ob + (widx * 32) / LPO >= NO) break;  // warp without outputs (warp-uniform)
+            double s = 0.0;
+            if (o < NO) {
+                const bool ua = o < JA;
+                const double *zr = ua ? zA : zB;
+                const int col = ua ? o : o - JA;
+                const int kind = o < JA + JB ? 0 : (o == JA + JB ? 1 : 2);
+                double s1 = 0.0;
+#pragma unroll 1
+                for (int rb = gl; rb < R; rb += 4 * LPO) {
 #pragma unroll
-                for (int u = 0; u < 4; u++) {
-                    const int rl = rb + u * LPO;
-                    if (rl < R) {
-                        const double z = zr[rl];
-                        const double t = (o < J ? X[rl * XR + o * XC] : (o == J ? z : 1.0)) * z;
-                        if (u & 1) s1 += t;
-                        else s += t;
+                    for (int u = 0; u < 4; u++) {
+                        const int rl = rb + u * LPO;
+                        if (rl < R) {
+                            const double z = zr[rl];
+                            const double t = (kind == 0 ? Vl[rl * XR + col * XC] : (kind == 1 ? z : 1.0)) * z;
+                            if (u & 1) s1 += t;
+                            else s += t;
+                        }
                     }
                 }
+                s += s1;
             }
-            s += s1;
-        }
 #pragma unroll
-        for (int off = 16; off > 0; off >>= 1)
-            if (off < LPO) s += __shfl_xor_sync(0xffffffffu, s, off);
-        if (o < NO && gl == 0 && !(p.dbg_mode & 4)) {
-            const int dst = o < J ? acc_o0 + o : acc_extra0 + (o - J);
-            atomicAdd(acc + dst * FT_ACC_PAD, s);
+            for (int off = 16; off > 0; off >>= 1)
+                if (off < LPO) s += __shfl_xor_sync(0xffffffffu, s, off);
+            if (o < NO && gl == 0 && !(p.dbg_mode & 4)) {
+                const int dst = o < JA ? oA + o : (o < JA + JB ? oB + o - JA : oE + (o - JA - JB));
+                atomicAdd(acc + dst * FT_ACC_PAD, s);
+            }
         }
     };
     // grid barrier: thread 0 arrives (release, cumulative over the CTA's writes ordered by the
@@ -252,8 +325,117 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
         __syncthreads();
     };
 
+    unsigned epoch = 0;
+    long long probe_last = 0;
+    int j = 0;  // (PROBE)
+    // ======================= the trailing GEMV (warps with IS_GEMV_WARP) =========================
+    // partials of A(rows, c+2:cend) bv(c+2:cend) (and of the row sums when vfy) into S.red / S.rsr
+    auto gemv = [&](const double *bv, int c, bool vfy) {
+        const int gt = GEMV_IDX(wid) * 32 + lane;
+        const int rp = gt % R2p, cl = gt / R2p;
+        const bool gemv_on = rp < R2 && cl < ncl;
+        const double2 *__restrict__ A2 = reinterpret_cast<const double2 *>(A + r0);
+        const int64_t ldw2 = ldw >> 1;
+        const int cend = vfy ? n : ihi;
+        double2 ya = make_double2(0.0, 0.0), rs = make_double2(0.0, 0.0);
+        if (MG && gemv_on && !(p.dbg_mode & 2)) {
+            // virtual columns: [0, nA) the panel columns c+2.. (owner only, from Apan), then
+            // the local trailing columns lcol0.. (global index J(l) selects the operand)
+            const int nA = (p.owner && p.e > c + 2) ? p.e - (c + 2) : 0;
+            const int nv = nA + (p.lcol1 - p.lcol0);
+            const double2 *__restrict__ Ap2 = reinterpret_cast<const double2 *>(Apan + r0);
 #pragma unroll 1
-    for (int i = tid; i < FT_NBMAX * (FT_NBMAX + 1); i += PT) (&S.Ts[0][0])[i] = 0.0;
+            for (int v0 = cl; v0 < nv; v0 += GB * ncl) {
+                double2 a[GB];
+                double xv[GB];
+#pragma unroll
+                for (int u = 0; u < GB; u++) {
+                    const int v = v0 + u * ncl;
+                    a[u] = make_double2(0.0, 0.0);
+                    xv[u] = 0.0;
+                    if (v < nA) {
+                        const int q = c + 2 + v;
+                        a[u] = Ap2[(int64_t)q * ldw2 + rp];
+                        xv[u] = bv[q];
+                    } else if (v < nv) {
+                        const int l = p.lcol0 + v - nA;
+                        const int J = (l / p.cbnb) * p.cbnb * p.G + p.rank * p.cbnb + l % p.cbnb;
+                        a[u] = A2[(int64_t)l * ldw2 + rp];
+                        xv[u] = J >= c + 2 ? bv[J] : 0.0;  // column c+1 = e is the unit term
+                    }
+                }
+#pragma unroll
+                for (int u = 0; u < GB; u++) {
+                    ya.x += a[u].x * xv[u];
+                    ya.y += a[u].y * xv[u];
+                }
+            }
+        } else if (gemv_on && !(p.dbg_mode & 2)) {
+            // bv is read with plain (L1-allocating) loads: the acquire at the grid barrier
+            // invalidated this SM's L1 before the trailing bar.sync released us
+            int col = c + 2 + cl;
+#pragma unroll 1
+            for (; col + (GB - 1) * ncl < cend; col += GB * ncl) {
+                double2 a[GB];
+                double v[GB];
+#pragma unroll
+                for (int u = 0; u < GB; u++) {
+                    const int q = col + u * ncl;
+                    a[u] = A2[(int64_t)q * ldw2 + rp];
+                    v[u] = bv[q];
+                }
+#pragma unroll
+                for (int u = 0; u < GB; u++) {
+                    ya.x += a[u].x * v[u];
+                    ya.y += a[u].y * v[u];
+                    rs.x += a[u].x;  // row sums: used by the verify pass only (cheap, memory-bound loop)
+                    rs.y += a[u].y;
+                }
+            }
+            if (col < cend) {  // ragged tail: one predicated batch (all loads in flight together)
+                double2 a[GB];
+                double v[GB];
+#pragma unroll
+                for (int u = 0; u < GB; u++) {
+                    const int q = col + u * ncl;
+                    a[u] = q < cend ? A2[(int64_t)q * ldw2 + rp] : make_double2(0.0, 0.0);
+                    v[u] = q < cend ? bv[q] : 0.0;
+                }
+#pragma unroll
+                for (int u = 0; u < GB; u++) {
+                    ya.x += a[u].x * v[u];
+                    ya.y += a[u].y * v[u];
+                    rs.x += a[u].x;
+                    rs.y += a[u].y;
+                }
+            }
+        }
+        if (R2p <= 32) {
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1)
+                if (o >= R2p) {
+                    ya.x += __shfl_xor_sync(0xffffffffu, ya.x, o);
+                    ya.y += __shfl_xor_sync(0xffffffffu, ya.y, o);
+                    if (vfy) {
+                        rs.x += __shfl_xor_sync(0xffffffffu, rs.x, o);
+                        rs.y += __shfl_xor_sync(0xffffffffu, rs.y, o);
+                    }
+                }
+            if (lane < R2p) {
+                S.red[GEMV_IDX(wid) * R2p + lane] = ya;
+                if (vfy) S.rsr[GEMV_IDX(wid) * R2p + lane] = rs;
+            }
+        } else if (cl < ncl) {
+            S.red[cl * R2p + rp] = ya;
+            if (vfy) S.rsr[cl * R2p + rp] = rs;
+        }
+    };
+
+#pragma unroll 1
+    for (int i = tid; i < FT_NBMAX * (FT_NBMAX + 1); i += PT) {
+        (&S.Ts[0][0])[i] = 0.0;
+        (&S.Gp[0][0])[i] = 0.0;
+    }
     if (p.ckpt) {
         // diskless checkpoint of the panel columns, r, c, kappa, Qr, Qc, Fr, taken
         // before anything is modified: own rows by their owner, c by the owner of row n (it
@@ -277,268 +459,249 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
         if (r0 <= n && n < r1)
             for (int i = tid; i <= n; i += PT) p.ck_c[i] = A[n + (int64_t)i * ldw];
     }
-    for (int rl = tid; rl < R; rl += PT) {
-        const int row = r0 + rl;
-        S.acol[rl] = is_valid(row) ? Apan[row + (int64_t)k * ldw] : 0.0;
+    {
+        // column k: b0 = A(:, k); publish its x part (rows >= k+2) and b0(k+1)
+        double *acc0 = p.acc + (k & 3) * FT_ACC_SET_DOUBLES;
+        double *bv0 = p.bvec + (int64_t)(k & 1) * ldw;
+        for (int rl = tid; rl < R; rl += PT) {
+            const int row = r0 + rl;
+            const double b = is_valid(row) ? Apan[row + (int64_t)k * ldw] : 0.0;
+            const bool d = is_data(row), xr = d && row >= k + 2;
+            S.acol[rl] = b;
+            S.b0[rl] = b;
+            S.bmA[rl] = d ? b : 0.0;
+            S.bmX[rl] = xr ? b : 0.0;
+            if (xr) bv0[row] = b;
+            if (row == k + 1 && d) acc0[ACC_B0 * FT_ACC_PAD] = b;
+        }
     }
+    if (tid < FT_NBMAX) S.ep[tid] = 0.0;
     if (tid == 0 && bid == 0) *p.bar_next = 0u;  // the next panel launch's counter
     __syncthreads();
 
-    unsigned epoch = 0;
-    long long probe_last = 0;
     double qc_corner = 0.0;  // corner of the Q checksums: sum of this panel's Qc (CTA 0, thread 0)
     const double c_thr = p.ctl->c_thr;
     const double tau_abs = c_thr * (double)n * 2.220446049250313e-16 * p.ctl->normF;
+    // lanes per row in the combine: a whole warp per row for small row blocks
+    const int lpr = R <= NWK ? 32 : (R <= 2 * NWK ? 16 : 8);
+    const int gl = wtid & (lpr - 1), grp = wtid / lpr, ngrp = WKT / lpr;
+    auto gsum = [&](double v) {  // sum over the lpr lanes of a row group
+#pragma unroll
+        for (int off = 16; off > 0; off >>= 1)
+            if (off < lpr) v += __shfl_xor_sync(0xffffffffu, v, off);
+        return v;
+    };
+    // A(row, c+1) of the own rows (thread = row), loaded one column ahead
+    // (MG: a trailing column c+1 >= e lives on one rank; it arrives through the exchange)
+    // (one GPU: column e is read from A, the panel buffer holds only the panel columns)
+    double an_reg = 0.0;
+    if (!helper && wtid < R && is_valid(r0 + wtid) && (!MG || k + 1 < p.e))
+        an_reg = (k + 1 < p.e ? Apan : A)[(r0 + wtid) + (int64_t)(k + 1) * ldw];
 
 #pragma unroll 1
-    for (int j = 0; j < ib; j++) {
+    for (j = 0; j < ib; j++) {
         const int c = k + j;
+        const bool last = j + 1 == ib;
+        const bool trivial = c + 2 >= ihi;  // the last reflector of the active block: tau = 0
         double *acc = p.acc + (c & 3) * FT_ACC_SET_DOUBLES;  // accumulator i at acc[i * FT_ACC_PAD]
-        // A(row, c+1) of the own rows (thread = row): issued now, parked in smem before the GEMV
-        double an_reg = 0.0;
-        // (MG: a trailing column c+1 >= e lives on one rank; it arrives through the exchange)
-        // (one GPU: column e is read from A, the panel buffer holds only the panel columns)
-        if (tid < R && is_valid(r0 + tid) && (!MG || c + 1 < p.e))
-            an_reg = (c + 1 < p.e ? Apan : A)[(r0 + tid) + (int64_t)(c + 1) * ldw];
+        const double *bv0 = p.bvec + (int64_t)(c & 1) * ldw;  // b0(c+2:ihi) (GEMV operand)
+        double *bvx = p.bvec + (int64_t)(2 + (c & 1)) * ldw;   // x = b(c+2:ihi) (explicit-path operand)
+        const bool vfy = (j == 0) && p.verify;
+        if (!helper && wtid < R) S.anext[wtid] = an_reg;
+        an_reg = 0.0;
+        if (!helper && !last && wtid < R && is_valid(r0 + wtid) && (!MG || c + 2 < p.e))
+            an_reg = (c + 2 < p.e ? Apan : A)[(r0 + wtid) + (int64_t)(c + 2) * ldw];
         PROBE(0);
-        // ---------------- (i) b0 = A(:,c) - Y V(c,:)^T, s1 = V^T b0 ---------------------------
-        if (j > 0) {
-            // b0 = A(:, c) - Y V(c, :)^T of the own rows was formed by the previous column's
-            // step (v) (S.b0 / S.bm): only the column dots remain here
-            coldot_add(Vl, S.bm, j, false, acc, 0, 0);
-            PROBE(1);
-            grid_sync(epoch, [&]() {
-                if (lane < j) S.s1[lane] = ldcg(acc + lane * FT_ACC_PAD);
-                if (lane + 32 < j) S.s1[lane + 32] = ldcg(acc + (lane + 32) * FT_ACC_PAD);
-            });
-            PROBE(2);
-            // w = T^T s1 (an 8-lane group per output)
-            {
-                double s0 = 0.0, s1 = 0.0;
-                if (4 * wid < j) {
-                if (slot < j)
+        // ---------------- the column's only grid reduction: s1 = V^T b0, sx = V_x^T b0_x,
+        // bb = b0_x.b0_x, eb = e^T b0_x (x = data rows >= c+2); b0(c+1) was stored by its owner
+        coldot_add(S.bmA, j, S.bmX, j, acc, ACC_S1, ACC_SX, ACC_BB);
+        PROBE(1);
+        double s1a = 0.0, s1b = 0.0, sxa = 0.0, sxb = 0.0, vra = 0.0, vrb = 0.0, bb = 0.0, eb = 0.0, b0c1 = 0.0;
+        grid_sync(epoch, [&]() {
+            bb = ldcg(acc + ACC_BB * FT_ACC_PAD);
+            eb = ldcg(acc + ACC_EB * FT_ACC_PAD);
+            b0c1 = ldcg(acc + ACC_B0 * FT_ACC_PAD);
+            if (lane < j) {
+                s1a = ldcg(acc + (ACC_S1 + lane) * FT_ACC_PAD);
+                sxa = ldcg(acc + (ACC_SX + lane) * FT_ACC_PAD);
+                vra = ldcg(V + (c + 1) + (int64_t)lane * ldw);
+            }
+            if (lane + 32 < j) {
+                s1b = ldcg(acc + (ACC_S1 + lane + 32) * FT_ACC_PAD);
+                sxb = ldcg(acc + (ACC_SX + lane + 32) * FT_ACC_PAD);
+                vrb = ldcg(V + (c + 1) + (int64_t)(lane + 32) * ldw);
+            }
+        });
+        PROBE(2);
+        if (IS_GEMV_WARP(wid)) {
+            // speculative: y = A(:, c+1) + scale (A(:, c+2:) b0_x - Z w); MG takes the explicit path
+            if (!MG) gemv(bv0, c, vfy);
+        } else if (wid == 0) {
+            // ======================= control warp: the column's scalars from the reduction =======
+            //   w = T^T s1,  G w = Gp w - V(c+1,:)^T q  (G = V_x^T V_x),  q = V(c+1,:) w
+            //   ||x||^2 = bb - 2 w.sx + w.Gp w - q^2,  alpha = b0(c+1) - q,  e^T x = eb - ep.w + q
+            //   t = V^T v = V(c+1,:)^T + scale (sx - G w)
+            // (lane o holds outputs o and o + 32; operand loads are issued 8 rows at a time)
+            const int la = lane, lb = lane + 32;
+            if (la < j) {
+                S.s1[la] = s1a;
+                S.vr1[la] = vra;
+            }
+            if (lb < j) {
+                S.s1[lb] = s1b;
+                S.vr1[lb] = vrb;
+            }
+            __syncwarp();
+            PROBE(10);
+            double wa0 = 0.0, wa1 = 0.0, wb0 = 0.0, wb1 = 0.0;  // T is upper triangular, zero beyond j
 #pragma unroll
-                    for (int u = 0; u < FT_NBMAX / 8; u += 2) {
-                        const int ba = g + 8 * u, bb = ba + 8;
-                        if (ba <= slot) s0 += S.Ts[ba][slot] * S.s1[ba];
-                        if (bb <= slot) s1 += S.Ts[bb][slot] * S.s1[bb];
+            for (int a0 = 0; a0 < FT_NBMAX; a0 += 8) {
+                if (a0 < j) {
+                    double sv[8], ta[8], tb[8];
+#pragma unroll
+                    for (int u = 0; u < 8; u++) {
+                        sv[u] = a0 + u < j ? S.s1[a0 + u] : 0.0;
+                        ta[u] = S.Ts[a0 + u][la];
+                        tb[u] = S.Ts[a0 + u][lb];
                     }
-                const double s = group8_sum(s0 + s1);
-                if (slot < j && g == 0) S.w[slot] = s;
+#pragma unroll
+                    for (int u = 0; u < 8; u += 2) {
+                        wa0 += ta[u] * sv[u];
+                        wb0 += tb[u] * sv[u];
+                        wa1 += ta[u + 1] * sv[u + 1];
+                        wb1 += tb[u + 1] * sv[u + 1];
+                    }
                 }
             }
-            __syncthreads();
+            const double wa = la < j ? wa0 + wa1 : 0.0, wb = lb < j ? wb0 + wb1 : 0.0;
+            S.w[la] = wa;
+            S.w[lb] = wb;
+            __syncwarp();
+            PROBE(11);
+            double ga0 = 0.0, ga1 = 0.0, gb0 = 0.0, gb1 = 0.0;  // Gp is zero beyond j, so is w
+#pragma unroll
+            for (int a0 = 0; a0 < FT_NBMAX; a0 += 8) {
+                if (a0 < j) {
+                    double wv[8], xa[8], xb[8];
+#pragma unroll
+                    for (int u = 0; u < 8; u++) {
+                        wv[u] = S.w[a0 + u];
+                        xa[u] = S.Gp[la][a0 + u];
+                        xb[u] = S.Gp[lb][a0 + u];
+                    }
+#pragma unroll
+                    for (int u = 0; u < 8; u += 2) {
+                        ga0 += xa[u] * wv[u];
+                        gb0 += xb[u] * wv[u];
+                        ga1 += xa[u + 1] * wv[u + 1];
+                        gb1 += xb[u + 1] * wv[u + 1];
+                    }
+                }
+            }
+            const double gpa = ga0 + ga1, gpb = gb0 + gb1;
+            const double epa = la < j ? S.ep[la] : 0.0, epb = lb < j ? S.ep[lb] : 0.0;
+            double q = vra * wa + vrb * wb, sw = sxa * wa + sxb * wb, ew = epa * wa + epb * wb;
+            double wgw = wa * gpa + wb * gpb;
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) {
+                q += __shfl_xor_sync(0xffffffffu, q, o);
+                sw += __shfl_xor_sync(0xffffffffu, sw, o);
+                ew += __shfl_xor_sync(0xffffffffu, ew, o);
+                wgw += __shfl_xor_sync(0xffffffffu, wgw, o);
+            }
+            wgw -= q * q;  // w^T G w
+            PROBE(12);
+            const double xx = bb - 2.0 * sw + wgw;
+            const double alpha = b0c1 - q;
+            const double ex = trivial ? 0.0 : eb - ew + q;
+            // cancellation guard: the expansion loses ~log2((bb + wGw) / xx) bits; below 1/64
+            // the column takes the explicit two-reduction path (uniform: every CTA sees the same
+            // sums).  MG: always explicit (the ranks' sums differ in rounding, the path must not)
+            const bool fast = !MG && !(p.dbg_mode & 8) && (trivial || xx >= GAMMA * (bb + wgw));
+            if (fast) {
+                const Refl rf = dlarfg_scalars(xx, alpha, trivial);
+                if (la < j) S.t[la] = vra + (trivial ? 0.0 : rf.scale * (sxa - (gpa - vra * q)));
+                if (lb < j) S.t[lb] = vrb + (trivial ? 0.0 : rf.scale * (sxb - (gpb - vrb * q)));
+                if (lane == 0) {
+                    S.scal[SC_TAU] = rf.tau;
+                    S.scal[SC_BETA] = rf.beta;
+                    S.scal[SC_SCALE] = rf.scale;
+                    S.scal[SC_ALPHA] = alpha;
+                    S.scal[SC_VCHK] = 1.0 + rf.scale * ex;
+                    S.scal[SC_XX] = trivial ? 0.0 : xx;
+                }
+            }
+            if (lane == 0) {
+                S.scal[SC_Q] = q;
+                S.scal[SC_FB] = fast ? 0.0 : 1.0;
+            }
+            PROBE(9);
+            __syncwarp();  // bar.arrive is .aligned: the whole warp, converged, after lane 0's stores
+            asm volatile("bar.arrive 1, 128;\n" ::: "memory");  // the scalars are in smem: helpers go
+        } else {
+            // helpers (warps 4, 8, 12: sub-partition 0, no GEMV): T(:, j) and the carried Gram
+            // while the GEMV streams (skipped on the explicit path: done after its second sync)
+            __syncwarp();
+            asm volatile("bar.sync 1, 128;\n" ::: "memory");
+            if (S.scal[SC_FB] == 0.0 && !MG && !(p.dbg_mode & 16)) tcol_gram(S, j, ((wid >> 2) - 1) * 32 + lane, 96, last);
         }
-        // ---------------- (ii) b = b0 - V w; publish x = b(c+2:ihi) for the GEMV, alpha = b(c+1)
-        auto publish = [&](int rl, double b) {
-            const int row = r0 + rl;
-            const bool xrow = is_data(row) && row >= c + 2;
-            S.b0[rl] = b;
-            S.bm[rl] = xrow ? b : 0.0;
-            if (xrow) p.bvec[row] = b;
-            if (row == c + 1) acc[ACC_ALPHA * FT_ACC_PAD] = b;  // alpha: a single writer
-        };
-        if (j > 0) {
+        if (!helper) {  // workers: GEMV partials, the column's scalars
+            __syncwarp();
+            asm volatile("bar.sync 2, %0;\n" ::"n"(WKT) : "memory");
+        }
+        PROBE(3);
+        const bool fb = S.scal[SC_FB] != 0.0;  // grid-uniform
+        // helpers are done with this column unless the explicit path, MG or the ablation needs them
+        if (helper && !fb && !MG && !(p.dbg_mode & 16)) continue;
+        if (fb) {
+            // ---- explicit path: x = b0 - V w of the own rows, second reduction, GEMV on x
 #pragma unroll 1
             for (int base = 0; base < R; base += NSLOT) {
                 if (base + 4 * wid >= R) break;
                 const int rl = base + slot;
                 const double vw = rowdot(Vl, rl, S.w, j);
-                if (rl < R && g == 0) publish(rl, S.b0[rl] - vw);
+                if (rl < R && g == 0) {
+                    const int row = r0 + rl;
+                    const double x = S.b0[rl] - vw;
+                    const bool xr = is_data(row) && row >= c + 2;
+                    S.bmX[rl] = xr ? x : 0.0;
+                    if (xr) bvx[row] = x;
+                    if (row == c + 1 && is_data(row)) acc[ACC_FAL * FT_ACC_PAD] = x;
+                }
             }
-        } else {
-            for (int rl = tid; rl < R; rl += PT) publish(rl, S.acol[rl]);
+            __syncthreads();
+            coldot_add(nullptr, 0, S.bmX, j, acc, 0, ACC_FVX, ACC_FNRM);
+            double fnrm = 0.0, fex = 0.0, fal = 0.0, fva = 0.0, fvb = 0.0;
+            grid_sync(epoch, [&]() {
+                fnrm = ldcg(acc + ACC_FNRM * FT_ACC_PAD);
+                fex = ldcg(acc + ACC_FEX * FT_ACC_PAD);
+                fal = ldcg(acc + ACC_FAL * FT_ACC_PAD);
+                if (lane < j) fva = ldcg(acc + (ACC_FVX + lane) * FT_ACC_PAD);
+                if (lane + 32 < j) fvb = ldcg(acc + (ACC_FVX + lane + 32) * FT_ACC_PAD);
+            });
+            if (IS_GEMV_WARP(wid)) {
+                gemv(bvx, c, false);
+            } else if (wid == 0) {
+                const Refl rf = dlarfg_scalars(fnrm, fal, trivial);
+                if (lane < j) S.t[lane] = S.vr1[lane] + rf.scale * fva;
+                if (lane + 32 < j) S.t[lane + 32] = S.vr1[lane + 32] + rf.scale * fvb;
+                if (lane == 0) {
+                    S.scal[SC_TAU] = rf.tau;
+                    S.scal[SC_BETA] = rf.beta;
+                    S.scal[SC_SCALE] = rf.scale;
+                    S.scal[SC_ALPHA] = fal;
+                    S.scal[SC_VCHK] = 1.0 + rf.scale * fex;
+                    S.scal[SC_XX] = fnrm;
+                }
+            }
+            __syncthreads();
+            if (!IS_GEMV_WARP(wid)) tcol_gram(S, j, (wid >> 2) * 32 + lane, 128, last);  // warps 0, 4, 8, 12
         }
-        __syncthreads();
-        PROBE(3);
-        coldot_add(Vl, S.bm, j, true, acc, ACC_VTB, ACC_NRM);
-        if (tid < R) S.anext[tid] = an_reg;
-        PROBE(4);
-        // control scalars of DLARFG, loaded by warp 0 as soon as the barrier opens
-        double nrm2 = 0.0, sx = 0.0, alpha = 0.0, vn0 = 0.0, vt0 = 0.0, vn1 = 0.0, vt1 = 0.0;
-        grid_sync(epoch, [&]() {
-            nrm2 = ldcg(acc + ACC_NRM * FT_ACC_PAD);
-            sx = ldcg(acc + ACC_SX * FT_ACC_PAD);
-            alpha = ldcg(acc + ACC_ALPHA * FT_ACC_PAD);
-            if (lane < j) {
-                vn0 = ldcg(V + (c + 1) + (int64_t)lane * ldw);
-                vt0 = ldcg(acc + (ACC_VTB + lane) * FT_ACC_PAD);
-            }
-            if (lane + 32 < j) {
-                vn1 = ldcg(V + (c + 1) + (int64_t)(lane + 32) * ldw);
-                vt1 = ldcg(acc + (ACC_VTB + lane + 32) * FT_ACC_PAD);
-            }
-        });
-        PROBE(5);
-        if (wid > 0) {
-            // ======================= GEMV warps: y = A(:, c+1:) v on the unscaled b ===========
-            const int gt = tid - 32;
-            const int rp = gt % R2p, cl = gt / R2p;
-            const bool gemv_on = rp < R2 && cl < ncl;
-            const double2 *__restrict__ A2 = reinterpret_cast<const double2 *>(A + r0);
-            const int64_t ldw2 = ldw >> 1;
-            const double *bv = p.bvec;  // b(q) for c+2 <= q < ihi; zero for q >= ihi
-            const bool vfy = (j == 0) && p.verify;
-            const int cend = vfy ? n : ihi;
-            double2 ya = make_double2(0.0, 0.0), rs = make_double2(0.0, 0.0);
-            if (MG && gemv_on && !(p.dbg_mode & 2)) {
-                // virtual columns: [0, nA) the panel columns c+2.. (owner only, from Apan), then
-                // the local trailing columns lcol0.. (global index J(l) selects x)
-                const int nA = (p.owner && p.e > c + 2) ? p.e - (c + 2) : 0;
-                const int nv = nA + (p.lcol1 - p.lcol0);
-                const double2 *__restrict__ Ap2 = reinterpret_cast<const double2 *>(Apan + r0);
-#pragma unroll 1
-                for (int v0 = cl; v0 < nv; v0 += GB * ncl) {
-                    double2 a[GB];
-                    double xv[GB];
-#pragma unroll
-                    for (int u = 0; u < GB; u++) {
-                        const int v = v0 + u * ncl;
-                        a[u] = make_double2(0.0, 0.0);
-                        xv[u] = 0.0;
-                        if (v < nA) {
-                            const int q = c + 2 + v;
-                            a[u] = Ap2[(int64_t)q * ldw2 + rp];
-                            xv[u] = bv[q];
-                        } else if (v < nv) {
-                            const int l = p.lcol0 + v - nA;
-                            const int J = (l / p.cbnb) * p.cbnb * p.G + p.rank * p.cbnb + l % p.cbnb;
-                            a[u] = A2[(int64_t)l * ldw2 + rp];
-                            xv[u] = J >= c + 2 ? bv[J] : 0.0;  // column c+1 = e is the unit term
-                        }
-                    }
-#pragma unroll
-                    for (int u = 0; u < GB; u++) {
-                        ya.x += a[u].x * xv[u];
-                        ya.y += a[u].y * xv[u];
-                    }
-                }
-            } else if (gemv_on && !(p.dbg_mode & 2)) {
-                // b is read with plain (L1-allocating) loads: the acquire at the grid barrier
-                // invalidated this SM's L1 before the trailing bar.sync released us
-                int col = c + 2 + cl;
-#pragma unroll 1
-                for (; col + (GB - 1) * ncl < cend; col += GB * ncl) {
-                    double2 a[GB];
-                    double v[GB];
-#pragma unroll
-                    for (int u = 0; u < GB; u++) {
-                        const int q = col + u * ncl;
-                        a[u] = A2[(int64_t)q * ldw2 + rp];
-                        v[u] = bv[q];
-                    }
-#pragma unroll
-                    for (int u = 0; u < GB; u++) {
-                        ya.x += a[u].x * v[u];
-                        ya.y += a[u].y * v[u];
-                        rs.x += a[u].x;  // row sums: used by the verify pass only (cheap, memory-bound loop)
-                        rs.y += a[u].y;
-                    }
-                }
-                if (col < cend) {  // ragged tail: one predicated batch (all loads in flight together)
-                    double2 a[GB];
-                    double v[GB];
-#pragma unroll
-                    for (int u = 0; u < GB; u++) {
-                        const int q = col + u * ncl;
-                        a[u] = q < cend ? A2[(int64_t)q * ldw2 + rp] : make_double2(0.0, 0.0);
-                        v[u] = q < cend ? bv[q] : 0.0;
-                    }
-#pragma unroll
-                    for (int u = 0; u < GB; u++) {
-                        ya.x += a[u].x * v[u];
-                        ya.y += a[u].y * v[u];
-                        rs.x += a[u].x;
-                        rs.y += a[u].y;
-                    }
-                }
-            }
-            if (R2p <= 32) {
-#pragma unroll
-                for (int o = 1; o < 32; o <<= 1)
-                    if (o >= R2p) {
-                        ya.x += __shfl_xor_sync(0xffffffffu, ya.x, o);
-                        ya.y += __shfl_xor_sync(0xffffffffu, ya.y, o);
-                        if (vfy) {
-                            rs.x += __shfl_xor_sync(0xffffffffu, rs.x, o);
-                            rs.y += __shfl_xor_sync(0xffffffffu, rs.y, o);
-                        }
-                    }
-                if (lane < R2p) {
-                    S.red[(wid - 1) * R2p + lane] = ya;
-                    if (vfy) S.rsr[(wid - 1) * R2p + lane] = rs;
-                }
-            } else if (cl < ncl) {
-                S.red[cl * R2p + rp] = ya;
-                if (vfy) S.rsr[cl * R2p + rp] = rs;
-            }
-        } else {
-            // ======================= control warp: (iii) DLARFG (R1), V(:, j) ================
-            const Refl rf = dlarfg_scalars(nrm2, alpha, c + 2 >= ihi);
-            const double tau = rf.tau, beta = rf.beta, scale = rf.scale;
-            const double vchk = 1.0 + scale * sx;  // V_chk(j) = e^T v
-            // t = V^T v = V(c+1,:)^T + scale * V^T x; V(c+1, :) is also the next column's vrow
-            if (lane < j) {
-                S.t[lane] = vn0 + scale * vt0;
-                S.vrow[lane] = vn0;
-            }
-            if (lane + 32 < j) {
-                S.t[lane + 32] = vn1 + scale * vt1;
-                S.vrow[lane + 32] = vn1;
-            }
-            if (lane == 0) {
-                S.vrow[j] = 1.0;
-                S.scal[0] = tau;
-                S.scal[2] = scale;
-            }
-            PROBE(9);
-            // V(:, j) and the reduced column c of the own rows
-#pragma unroll 1
-            for (int rl = lane; rl < R; rl += 32) {
-                const int row = r0 + rl;
-                const double b = S.b0[rl];
-                if (row == n && p.abft) {
-                    V[row + (int64_t)j * ldw] = vchk;
-                    if (CACHE) Vl[rl * XR + j * XC] = vchk;
-                    Apan[row + (int64_t)c * ldw] = (tau != 0.0) ? b - vchk * (alpha - beta) : b;  // left term (R7)
-                } else if (is_data(row)) {
-                    double vv, av;
-                    if (row <= c) {
-                        vv = 0.0;
-                        av = b;
-                    } else if (row == c + 1) {
-                        vv = 1.0;
-                        av = beta;
-                    } else {
-                        vv = scale * b;
-                        av = vv;
-                    }
-                    V[row + (int64_t)j * ldw] = vv;
-                    if (CACHE) Vl[rl * XR + j * XC] = vv;
-                    Apan[row + (int64_t)c * ldw] = av;
-                } else if (CACHE) {
-                    Vl[rl * XR + j * XC] = 0.0;  // rows outside the panel take no part in the dots
-                }
-            }
-            if (bid == 0 && lane == 0) {
-                p.tau[c] = tau;
-                if (p.abft) {
-                    p.Qc[c] = vchk - 1.0;  // Q column checksum (P:266)
-                    qc_corner += vchk - 1.0;
-                }
-            }
-            // recycle the accumulator set of column c+2 (= that of column c-2): every CTA has
-            // finished reading it, and column c+2 adds into it only after two more syncs
-            if (bid == 0)
-                for (int i = lane; i < FT_ACC_STRIDE; i += 32) p.acc[((c + 2) & 3) * FT_ACC_SET_DOUBLES + i * FT_ACC_PAD] = 0.0;
-            PROBE(6);
-        }
-        __syncthreads();  // GEMV partials, tau / scale / t, V(:, j) are in shared memory
         if (MG) {
             // ---- cross-rank exchange of the GEMV partials, CTA by CTA: every rank
             // uses the same row partition, so CTA bid of each rank owns the same rows.  Push
             // (y partial, A(:, c+1) part) of the own rows into every rank's slot, raise the flag,
-            // wait for every rank's flag; phase (v) sums the slots in rank order (identical on
+            // wait for every rank's flag; the combine sums the slots in rank order (identical on
             // every rank).  Slots alternate by column; a rank reaches column c+2's push only
             // after every rank has flagged column c+1, i.e. after it read column c.
             const int sl = c & 1;
@@ -567,101 +730,116 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
                 }
             __syncthreads();
         }
+        if ((p.dbg_mode & 16) && !fb) {
+            __syncthreads();
+            if (!IS_GEMV_WARP(wid)) tcol_gram(S, j, (wid >> 2) * 32 + lane, 128, last);
+            __syncthreads();
+        }
         PROBE(7);
-        // ---------------- (v) Y(:, j) = tau (y - Y t) (an 8-lane group per row) -----------------
+        // ---------------- combine (lpr lanes per row): with g = the GEMV result,
+        //   x = b0 - V w -> V(:, j), reduced column c;   u = scale (g - Z w) (fast) | scale g
+        //   y = A(:, c+1) + u,  Y(:, j) = tau (y - Y t);  Z(:, j) = u;  Z -= A(:, c+1) V(c+1, :)
+        //   next column's b0 = A(:, c+1) - Y(:, 0:j+1) V(c+1, 0:j+1)^T
         {
-            const double tau = S.scal[0], scale = S.scal[2];
-            const bool vfy = (j == 0) && p.verify;
-            // small row blocks: the T column (warps 8..15) runs beside the Y rows (warps 0..7)
-            const bool split = R <= 32;
-            if (!split || wid >= 8) {
-                // T(a, j) = -tau * sum_{b=a}^{j-1} T(a, b) t(b), T(j, j) = tau (8 lanes per a)
-                const int tslot = split ? slot - 32 : slot, tw = split ? wid - 8 : wid;
-                const int nsl = split ? 32 : NSLOT;
+            const double tau = S.scal[SC_TAU], beta = S.scal[SC_BETA], scale = S.scal[SC_SCALE];
+            const double alpha = S.scal[SC_ALPHA], vchk = S.scal[SC_VCHK], q = S.scal[SC_Q];
+            double *accn = p.acc + ((c + 1) & 3) * FT_ACC_SET_DOUBLES;
+            double *bvn = p.bvec + (int64_t)((c + 1) & 1) * ldw;
 #pragma unroll 1
-                for (int a0 = 0; a0 < j; a0 += nsl) {
-                    if (a0 + 4 * tw >= j) break;  // warp-uniform
-                    const int a = a0 + tslot;
-                    double s0 = 0.0, s1 = 0.0;
-                    if (a < j)
-#pragma unroll
-                        for (int u = 0; u < FT_NBMAX / 8; u += 2) {
-                            const int ba = a + g + 8 * u, bb = ba + 8;
-                            if (ba < j) s0 += S.Ts[a][ba] * S.t[ba];
-                            if (bb < j) s1 += S.Ts[a][bb] * S.t[bb];
-                        }
-                    const double sT = group8_sum(s0 + s1);
-                    if (a < j && g == 0) S.Ts[a][j] = -tau * sT;
-                }
-            }
-            if (tid == 0) S.Ts[j][j] = tau;
-            PROBE(12);
-            const int rslots = split ? 32 : NSLOT;
-#pragma unroll 1
-            for (int base = 0; base < R; base += rslots) {
-                if (split && wid >= 8) break;
-                if (base + 4 * wid >= R) break;
-                const int rl = base + slot;
+            for (int base = 0; base < R; base += ngrp) {
+                if (helper || base + (widx * 32) / lpr >= R) break;  // warp-uniform: no row for this warp
+                const int rl = base + grp;
                 const bool on = rl < R && is_valid(r0 + rl);
                 const int pr = rl >> 1, hi = rl & 1;
-                // lane partial of scale * y - Y(rl, :) t: GEMV partials q = g, g + 8 (npart <= 15)
-                double ya = 0.0, yb = 0.0, rsum = 0.0, an_mg = 0.0;
+                double gp = 0.0, rsum = 0.0, an_mg = 0.0;
                 if (on && MG) {
-                    if (g == 0) {  // exchanged partials, summed in rank order
-                        double ysum = 0.0;
+                    if (gl == 0) {  // exchanged partials, summed in rank order
                         const double2 *yxs = p.yx + (int64_t)(c & 1) * p.G * ldw + (r0 + rl);
                         for (int gg = 0; gg < p.G; gg++) {
                             const double2 u = __ldcg(yxs + (int64_t)gg * ldw);
-                            ysum += u.x;
+                            gp += u.x;
                             an_mg += u.y;
                         }
-                        ya = scale * ysum;
                     }
                 } else if (on) {
-#pragma unroll
-                    for (int u = 0; u < 2; u++) {
-                        const int q = g + 8 * u;
-                        if (q < npart) {
-                            const double2 w2 = S.red[q * R2p + pr];
-                            ya += scale * (hi ? w2.y : w2.x);
-                            if (vfy) {
-                                const double2 r2 = S.rsr[q * R2p + pr];
-                                rsum += hi ? r2.y : r2.x;
-                            }
+                    for (int qq = gl; qq < npart; qq += lpr) {
+                        const double2 w2 = S.red[qq * R2p + pr];
+                        gp += hi ? w2.y : w2.x;
+                        if (vfy) {
+                            const double2 r2 = S.rsr[qq * R2p + pr];
+                            rsum += hi ? r2.y : r2.x;
                         }
                     }
                 }
-                // with the same Y row loads: P1 = Y(rl, :) V(c+1, :)^T (S.vrow), which gives the
-                // next column's b0 = A(:, c+1) - Y(:, 0:j) V(c+1, 0:j)^T = an - P1 - Y(:, j)
-                double pa = 0.0, pb = 0.0;
+                double zw = 0.0, vw = 0.0, yt = 0.0, yr = 0.0;
                 if (on) {
-#pragma unroll
-                    for (int u = 0; u < FT_NBMAX / 8; u += 2) {
-                        const int ja = g + 8 * u, jb = ja + 8;
-                        if (ja < j) {
-                            const double yv = Yl[rl * XR + ja * XC];
-                            ya -= yv * S.t[ja];
-                            pa += yv * S.vrow[ja];
-                        }
-                        if (jb < j) {
-                            const double yv = Yl[rl * XR + jb * XC];
-                            yb -= yv * S.t[jb];
-                            pb += yv * S.vrow[jb];
-                        }
+                    const double anl = S.anext[rl];
+#pragma unroll 2
+                    for (int i = gl; i < j; i += lpr) {
+                        const double wi = S.w[i], vri = S.vr1[i], ti = S.t[i];
+                        double *zp = Zl + rl * XR + i * XC;
+                        const double z = *zp, vv = Vl[rl * XR + i * XC], yv = Yl[rl * XR + i * XC];
+                        zw += z * wi;
+                        vw += vv * wi;
+                        yt += yv * ti;
+                        yr += yv * vri;
+                        if (!last) *zp = z - anl * vri;
                     }
                 }
-                const double ysum = group8_sum(ya + yb);
-                const double p1 = group8_sum(pa + pb);
-                if (vfy) rsum = group8_sum(rsum);
-                if (rl < R && g == 0) {
+                PROBE(14);
+                // six group sums, interleaved (independent shuffle chains)
+#pragma unroll
+                for (int off = 16; off > 0; off >>= 1) {
+                    if (off < lpr) {
+                        const double a0 = __shfl_xor_sync(0xffffffffu, gp, off);
+                        const double a1 = __shfl_xor_sync(0xffffffffu, zw, off);
+                        const double a2 = __shfl_xor_sync(0xffffffffu, vw, off);
+                        const double a3 = __shfl_xor_sync(0xffffffffu, yt, off);
+                        const double a4 = __shfl_xor_sync(0xffffffffu, yr, off);
+                        const double a5 = __shfl_xor_sync(0xffffffffu, rsum, off);
+                        gp += a0;
+                        zw += a1;
+                        vw += a2;
+                        yt += a3;
+                        yr += a4;
+                        rsum += a5;
+                    }
+                }
+                PROBE(15);
+                if (rl < R && gl == 0) {
                     const int row = r0 + rl;
                     const double an = (MG && c + 1 >= p.e) ? an_mg : S.anext[rl];
                     double b0n = 0.0;
                     if (on) {
-                        const double yy = tau * (an + ysum);
+                        const double b = S.b0[rl] - vw;  // b = b0 - V T^T V^T b0 (step ii)
+                        // V(:, j) and the reduced column c of the own rows (step iii)
+                        if (row == n && p.abft) {
+                            V[row + (int64_t)j * ldw] = vchk;
+                            if (CACHE) Vl[rl * XR + j * XC] = vchk;
+                            Apan[row + (int64_t)c * ldw] = (tau != 0.0) ? b - vchk * (alpha - beta) : b;  // left term (R7)
+                        } else {
+                            double vv, av;
+                            if (row <= c) {
+                                vv = 0.0;
+                                av = b;
+                            } else if (row == c + 1) {
+                                vv = 1.0;
+                                av = beta;
+                            } else {
+                                vv = scale * b;
+                                av = vv;
+                            }
+                            V[row + (int64_t)j * ldw] = vv;
+                            if (CACHE) Vl[rl * XR + j * XC] = vv;
+                            Apan[row + (int64_t)c * ldw] = av;
+                        }
+                        // steps (iv)-(v)
+                        const double u = fb ? scale * gp : scale * (gp - (zw - an * q));
+                        if (!last) Zl[rl * XR + j * XC] = u;
+                        const double yy = tau * (an + u - yt);
                         Y[row + (int64_t)j * ldw] = yy;
                         if (CACHE) Yl[rl * XR + j * XC] = yy;
-                        b0n = an - p1 - yy;
+                        b0n = an - yr - yy;
                         if (vfy && is_data(row)) {
                             // D_r(row) = r(row) - sum_{col >= k} L(row, col); columns < k are logical zero
                             rsum += S.acol[rl] + an;
@@ -673,17 +851,41 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
                                 atomicMax(&p.ctl->drift_bits, (unsigned long long)__double_as_longlong(rel));
                             }
                         }
+                    } else if (CACHE) {
+                        Vl[rl * XR + j * XC] = 0.0;  // rows outside the panel take no part in the dots
                     }
                     S.acol[rl] = an;
                     S.b0[rl] = b0n;
-                    S.bm[rl] = is_data(row) ? b0n : 0.0;
+                    if (!last) {  // publish the next column's b0
+                        const bool d = on && is_data(row), xr = d && row >= c + 3;
+                        S.bmA[rl] = d ? b0n : 0.0;
+                        S.bmX[rl] = xr ? b0n : 0.0;
+                        if (xr) bvn[row] = b0n;
+                        if (row == c + 2 && d) accn[ACC_B0 * FT_ACC_PAD] = b0n;
+                    }
                 }
             }
             PROBE(13);
-            __syncthreads();
+            if (bid == 0 && tid == 0) {
+                p.tau[c] = tau;
+                if (p.abft) {
+                    p.Qc[c] = vchk - 1.0;  // Q column checksum (P:266)
+                    qc_corner += vchk - 1.0;
+                }
+            }
+            // recycle the accumulator set of column c+2 (= that of column c-2): every CTA has
+            // finished reading it, and column c+2 adds into it only after two more syncs
+            if (bid == 0 && wid == NW - 1)
+                for (int i = lane; i < FT_ACC_STRIDE; i += 32)
+                    p.acc[((c + 2) & 3) * FT_ACC_SET_DOUBLES + i * FT_ACC_PAD] = 0.0;
+            if (!helper) {  // workers: the next column's b0 and masks are in smem
+                __syncwarp();
+                asm volatile("bar.sync 2, %0;\n" ::"n"(WKT) : "memory");
+            }
         }
         PROBE(8);
     }
+    __syncthreads();  // the helpers' last T column
     // Q row checksums of the new Householder vectors (Fig. 5): own data rows
     if (p.abft)
         for (int rl = tid; rl < R; rl += PT) {
@@ -737,10 +939,14 @@ cudaError_t ft_launch_panel_multi(const PanelLaunch &L, int nsm, cudaStream_t s)
             if (e != cudaSuccess) return e;
         }
     }
-    static int ctas = -1;
+    static int ctas = -1, explicit_path = 0;
     if (ctas < 0) {
         const char *e = getenv("FT_PANEL_CTAS");  // experiment knob: cap on the panel grid
         ctas = e ? atoi(e) : 0;
+        const char *x = getenv("FT_PANEL_EXPLICIT");  // experiment knob: every column on the explicit path
+        explicit_path = x ? atoi(x) : 0;
+        const char *d = getenv("FT_PANEL_DBG");  // experiment knob: dbg_mode bits for every launch
+        if (d) explicit_path |= atoi(d) << 8;
     }
     if (L.nr < 1 || L.nr > FT_MAX_VRANKS) return cudaErrorInvalidValue;
     const bool mg = L.r[0].G > 1;
@@ -749,14 +955,21 @@ cudaError_t ft_launch_panel_multi(const PanelLaunch &L, int nsm, cudaStream_t s)
     if (per > FT_FLAG_STRIDE) per = FT_FLAG_STRIDE;
     int grid = per < L.r[0].ngroups ? per : L.r[0].ngroups;
     if (grid < 1) grid = 1;
-    // rows per CTA (max over CTAs) and whether their V/Y rows fit next to the fixed part
+    // rows per CTA (max over CTAs) and whether their V/Y/Z rows fit next to the fixed part
     const int gmax = (L.r[0].ngroups + grid - 1) / grid;
     const int rmax = GR * gmax;
-    if (rmax > RMAX) return cudaErrorInvalidConfiguration;  // n beyond ~75k rows per GPU
+    if (rmax > WKT) return cudaErrorInvalidConfiguration;  // n beyond ~61k rows per GPU
     const size_t fixed = sizeof(PanelSmem);
-    const size_t want = fixed + (size_t)2 * VS * rmax * sizeof(double);
+    const size_t want = fixed + (size_t)3 * VS * rmax * sizeof(double);
     const bool cache = want <= (size_t)max_smem;
-    void *args[] = {const_cast<PanelLaunch *>(&L)};
+    PanelLaunch Lx;
+    const PanelLaunch *Lp = &L;
+    if (explicit_path) {
+        Lx = L;
+        for (int i = 0; i < Lx.nr; i++) Lx.r[i].dbg_mode |= ((explicit_path & 0xff) ? 8 : 0) | (explicit_path >> 8);
+        Lp = &Lx;
+    }
+    void *args[] = {const_cast<PanelLaunch *>(Lp)};
     g_ft_launches++;
     const void *fn = mg ? (cache ? (const void *)k_panel<true, true> : (const void *)k_panel<false, true>)
                         : (cache ? (const void *)k_panel<true, false> : (const void *)k_panel<false, false>);

@@ -64,10 +64,9 @@ def main():
               f"{10 / 3 * n ** 3 / ms / 1e6:.1f} Gflop/s", flush=True)
     if dbg is not None:
         d = dbg.cpu().numpy()
-        names = {0: "start", 10: "b0_rowdot", 11: "b0_bar", 1: "s1_coldot", 2: "sync1", 3: "w_b", 4: "x_dots",
-                 5: "sync2", 9: "cw_dlarfg", 6: "cw_V_stores", 7: "gemv_wait", 12: "T_col", 13: "y_rows",
-                 8: "y_bar"}
-        order = [0, 10, 11, 1, 2, 3, 4, 5, 9, 6, 7, 12, 13, 8]
+        names = {0: "start", 1: "coldot", 2: "sync", 10: "c_loads", 11: "c_w", 12: "c_Gw_shfl", 9: "c_dlarfg",
+                 3: "gemv_join", 7: "explicit/xchg", 14: "cmb_dots", 15: "cmb_gsum", 13: "cmb_leader", 8: "T_G_bar"}
+        order = [0, 1, 2, 10, 11, 12, 9, 3, 7, 14, 15, 13, 8]
         tot = {}
         ncol = 0
         for j in range(64):
