@@ -185,6 +185,11 @@ void ft_debug_time_panels(int on);
 double ft_debug_panel_ms(void);
 int ft_debug_panel_launches(void);
 void ft_debug_probe_panel(int panel, unsigned long long *dbuf);
+/* ft_debug_panel_path(8) sends every column of every later panel through the explicit
+ * two-reduction path (the one-reduction path's cancellation fallback); 64 / 128 force the
+ * panel's smaller shared-memory modes (V, Z rows cached, Y global / all global); 0 restores
+ * the default.  Results agree with the default up to rounding (tests of those paths). */
+void ft_debug_panel_path(int bits);
 
 #ifdef __cplusplus
 }

@@ -24,6 +24,8 @@ static int g_dbg_panel = -1;
 static unsigned long long *g_dbg_buf = nullptr;
 static int g_dbg_mode = 0;
 extern "C" void ft_debug_ablate(int mode) { g_dbg_mode = mode; }
+static int g_panel_path = 0;  // OR'ed into every panel launch's mode bits (8: explicit path, 64/128: smem modes 1/0)
+extern "C" void ft_debug_panel_path(int bits) { g_panel_path = bits & (8 | 64 | 128); }
 extern "C" void ft_debug_probe_panel(int panel, unsigned long long *dbuf) {
     g_dbg_panel = panel;
     g_dbg_buf = dbuf;
@@ -619,7 +621,7 @@ int enqueue_panel(Call &C, int t) {
     const bool fuse_pre = eager && !has_fault(C, t, FT_PHASE_AFTER_PANEL);
     p.precheck_sums = fuse_pre ? 1 : 0;
     p.dbg = (t == g_dbg_panel) ? g_dbg_buf : nullptr;
-    p.dbg_mode = (t == g_dbg_panel) ? g_dbg_mode : 0;
+    p.dbg_mode = ((t == g_dbg_panel) ? g_dbg_mode : 0) | g_panel_path;
     const int gr = ft_panel_group_rows();
     p.rbase = ((k + 1) / gr) * gr;
     int rendp = (C.rend() + gr - 1) / gr * gr;
@@ -865,6 +867,7 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
     // every iteration), captured on the second call with the same shape and buffers; the halt
     // protocol is unchanged (a halted graph's remaining kernels are no-ops, recovery follows).
     const bool graphable = C.faults.empty() && o.stop_after_panel < 0 && g_dbg_panel < 0 && !g_time_panels &&
+                           !g_panel_path &&
                            !getenv("FT_NO_GRAPH");
     bool launched = false;
     if (graphable) {

@@ -50,6 +50,7 @@ struct PanelParams {
     double *Qr, *Qc;
     int n, ihi, k, ib, abft, verify;  // verify: fused D_r on the first GEMV (EAGER policy)
     int rbase, ngroups;               // ft_panel_group_rows()-row groups starting at rbase
+    int wide;                         // set by the launcher: >= 32 rows per CTA (GEMV on 15 warps)
     // diskless checkpoint of the panel, taken in the kernel's prologue, or NULL
     double *ckpt, *ck_r, *ck_c, *ck_q, *Fr;
     int precheck_sums;  // add e^T Y, e^T V of the own rows into ctl->eY / eV (fused pre-update check)
@@ -81,6 +82,7 @@ struct PanelLaunch {
 // launchers (return cudaError_t of the launch)
 cudaError_t ft_launch_panel(const PanelParams &p, int nsm, cudaStream_t s);
 cudaError_t ft_launch_panel_multi(const PanelLaunch &L, int nsm, cudaStream_t s);
+cudaError_t ft_launch_panel_wide(const PanelLaunch &L, int nsm, cudaStream_t s);  // two-reduction kernel
 size_t ft_panel_smem_bytes();
 int ft_panel_group_rows();
 

@@ -196,7 +196,7 @@ __device__ __forceinline__ void st_relaxed_sys_u32(unsigned *p, unsigned v) {
     asm volatile("st.relaxed.sys.global.u32 [%0], %1;\n" ::"l"(p), "r"(v) : "memory");
 }
 
-template <bool CACHE, bool MG>
+template <int CACHE, bool MG>
 __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLaunch L) {
     // rank group of this CTA (MG: virtual ranks share the launch; one GPU: a single group)
     const unsigned P = gridDim.x / L.nr;
@@ -209,8 +209,16 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
 
     const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
     const int slot = tid >> 3, g = tid & 7;  // 8-lane groups: NSLOT row / output slots
-    const bool helper = IS_HELPER(wid);
-    const int widx = wid - (wid >> 2), wtid = widx * 32 + lane;  // worker warp / thread index
+    // wide launches (>= 32 rows per CTA: the GEMV dominates the column) give the GEMV 15 warps,
+    // warp 0 forms T(:, j) and the Gram itself, and every warp is a worker
+    const bool wide = p.wide != 0;
+    const bool gw = wide ? wid != 0 : IS_GEMV_WARP(wid);           // GEMV warp
+    const int gidx = wide ? wid - 1 : GEMV_IDX(wid), ngw = wide ? NW - 1 : NGW;
+    const bool helper = !wide && IS_HELPER(wid);
+    const int nwk = wide ? NW : NWK, wkt = 32 * nwk;
+    const int widx = wide ? wid : wid - (wid >> 2), wtid = widx * 32 + lane;  // worker warp / thread index
+    // the non-GEMV warps (warp 0 + helpers) as one thread range, for T(:, j) / the Gram
+    const int ng_t0 = (wid >> 2) * 32 + lane, ng_n = wide ? 32 : 128;
     const int g0 = (int)((long long)bid * p.ngroups / P);
     const int g1 = (int)((long long)(bid + 1) * p.ngroups / P);
     const int r0 = p.rbase + GR * g0, r1 = p.rbase + GR * g1;
@@ -224,11 +232,16 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
 
     // own rows of V, Y and Z: [rl][jp] in shared memory (V, Y write-through to global) when
     // they fit, else the global arrays (Z: p.Z)
-    double *Vl = CACHE ? reinterpret_cast<double *>(smem_raw + sizeof(PanelSmem)) : V + r0;
-    double *Yl = CACHE ? Vl + (int64_t)VS * R : Y + r0;
-    double *Zl = CACHE ? Yl + (int64_t)VS * R : p.Z + r0;
-    constexpr int64_t XR = CACHE ? VS : 1;  // row stride
-    const int64_t XC = CACHE ? 1 : ldw;     // column stride
+    // CACHE 2: V, Z, Y rows in smem; 1: V, Z in smem, Y global; 0: all global
+    constexpr bool VC = CACHE >= 1, YC = CACHE == 2;
+    double *dyn = reinterpret_cast<double *>(smem_raw + sizeof(PanelSmem));
+    double *Vl = VC ? dyn : V + r0;
+    double *Zl = VC ? dyn + (int64_t)VS * R : p.Z + r0;
+    double *Yl = YC ? dyn + (int64_t)2 * VS * R : Y + r0;
+    constexpr int64_t XR = VC ? VS : 1;  // row stride of V and Z
+    const int64_t XC = VC ? 1 : ldw;     // column stride
+    constexpr int64_t YR = YC ? VS : 1;  // of Y
+    const int64_t YCS = YC ? 1 : ldw;
 
     // GEMV partial layout: R2p lanes per column, a power of two when <= 32 so the lanes of
     // one row pair are shuffle-reducible inside a warp
@@ -237,8 +250,8 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
         R2p = 1;
         while (R2p < R2) R2p *= 2;
     }
-    const int ncl = (NGW * 32) / R2p;
-    const int npart = R2p <= 32 ? NGW : ncl;  // partials per row pair
+    const int ncl = (ngw * 32) / R2p;
+    const int npart = R2p <= 32 ? ngw : ncl;  // partials per row pair
 
     auto is_data = [&](int row) { return row >= k + 1 && row < ihi; };
     auto is_valid = [&](int row) { return (row >= k + 1 && row < ihi) || (p.abft && row == n); };
@@ -268,11 +281,11 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
                           int oE) {
         const int NO = JA + JB + 2;
         int LPO = 4;
-        while (LPO < 32 && 2 * LPO < R && (2 * LPO) * NO <= WKT) LPO *= 2;
+        while (LPO < 32 && 2 * LPO < R && (2 * LPO) * NO <= wkt) LPO *= 2;
         if (helper) return;
-        // output blocks of WKT / LPO (two when 4 lanes per output do not cover NO <= 128)
+        // output blocks of wkt / LPO (two when 4 lanes per output do not cover NO <= 128)
 #pragma unroll 1
-        for (int ob = 0; ob < NO; ob += WKT / LPO) {
+        for (int ob = 0; ob < NO; ob += wkt / LPO) {
             const int o = ob + wtid / LPO, gl = wtid & (LPO - 1);
             if (ob + (widx * 32) / LPO >= NO) break;  // warp without outputs (warp-uniform)
             double s = 0.0;
@@ -331,7 +344,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
     // ======================= the trailing GEMV (warps with IS_GEMV_WARP) =========================
     // partials of A(rows, c+2:cend) bv(c+2:cend) (and of the row sums when vfy) into S.red / S.rsr
     auto gemv = [&](const double *bv, int c, bool vfy) {
-        const int gt = GEMV_IDX(wid) * 32 + lane;
+        const int gt = gidx * 32 + lane;
         const int rp = gt % R2p, cl = gt / R2p;
         const bool gemv_on = rp < R2 && cl < ncl;
         const double2 *__restrict__ A2 = reinterpret_cast<const double2 *>(A + r0);
@@ -422,8 +435,8 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
                     }
                 }
             if (lane < R2p) {
-                S.red[GEMV_IDX(wid) * R2p + lane] = ya;
-                if (vfy) S.rsr[GEMV_IDX(wid) * R2p + lane] = rs;
+                S.red[gidx * R2p + lane] = ya;
+                if (vfy) S.rsr[gidx * R2p + lane] = rs;
             }
         } else if (cl < ncl) {
             S.red[cl * R2p + rp] = ya;
@@ -483,8 +496,8 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
     const double c_thr = p.ctl->c_thr;
     const double tau_abs = c_thr * (double)n * 2.220446049250313e-16 * p.ctl->normF;
     // lanes per row in the combine: a whole warp per row for small row blocks
-    const int lpr = R <= NWK ? 32 : (R <= 2 * NWK ? 16 : 8);
-    const int gl = wtid & (lpr - 1), grp = wtid / lpr, ngrp = WKT / lpr;
+    const int lpr = R <= nwk ? 32 : (R <= 2 * nwk ? 16 : 8);
+    const int gl = wtid & (lpr - 1), grp = wtid / lpr, ngrp = wkt / lpr;
     auto gsum = [&](double v) {  // sum over the lpr lanes of a row group
 #pragma unroll
         for (int off = 16; off > 0; off >>= 1)
@@ -533,7 +546,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
             }
         });
         PROBE(2);
-        if (IS_GEMV_WARP(wid)) {
+        if (gw) {
             // speculative: y = A(:, c+1) + scale (A(:, c+2:) b0_x - Z w); MG takes the explicit path
             if (!MG) gemv(bv0, c, vfy);
         } else if (wid == 0) {
@@ -637,7 +650,8 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
             }
             PROBE(9);
             __syncwarp();  // bar.arrive is .aligned: the whole warp, converged, after lane 0's stores
-            asm volatile("bar.arrive 1, 128;\n" ::: "memory");  // the scalars are in smem: helpers go
+            if (!wide) asm volatile("bar.arrive 1, 128;\n" ::: "memory");  // the scalars are in smem: helpers go
+            else if (fast && !(p.dbg_mode & 16)) tcol_gram(S, j, lane, 32, last);
         } else {
             // helpers (warps 4, 8, 12: sub-partition 0, no GEMV): T(:, j) and the carried Gram
             // while the GEMV streams (skipped on the explicit path: done after its second sync)
@@ -645,7 +659,9 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
             asm volatile("bar.sync 1, 128;\n" ::: "memory");
             if (S.scal[SC_FB] == 0.0 && !MG && !(p.dbg_mode & 16)) tcol_gram(S, j, ((wid >> 2) - 1) * 32 + lane, 96, last);
         }
-        if (!helper) {  // workers: GEMV partials, the column's scalars
+        if (wide) {
+            __syncthreads();
+        } else if (!helper) {  // workers: GEMV partials, the column's scalars
             __syncwarp();
             asm volatile("bar.sync 2, %0;\n" ::"n"(WKT) : "memory");
         }
@@ -679,7 +695,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
                 if (lane < j) fva = ldcg(acc + (ACC_FVX + lane) * FT_ACC_PAD);
                 if (lane + 32 < j) fvb = ldcg(acc + (ACC_FVX + lane + 32) * FT_ACC_PAD);
             });
-            if (IS_GEMV_WARP(wid)) {
+            if (gw) {
                 gemv(bvx, c, false);
             } else if (wid == 0) {
                 const Refl rf = dlarfg_scalars(fnrm, fal, trivial);
@@ -695,7 +711,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
                 }
             }
             __syncthreads();
-            if (!IS_GEMV_WARP(wid)) tcol_gram(S, j, (wid >> 2) * 32 + lane, 128, last);  // warps 0, 4, 8, 12
+            if (!gw) tcol_gram(S, j, ng_t0, ng_n, last);  // warp 0 (+ helpers)
         }
         if (MG) {
             // ---- cross-rank exchange of the GEMV partials, CTA by CTA: every rank
@@ -732,7 +748,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
         }
         if ((p.dbg_mode & 16) && !fb) {
             __syncthreads();
-            if (!IS_GEMV_WARP(wid)) tcol_gram(S, j, (wid >> 2) * 32 + lane, 128, last);
+            if (!gw) tcol_gram(S, j, ng_t0, ng_n, last);
             __syncthreads();
         }
         PROBE(7);
@@ -778,7 +794,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
                     for (int i = gl; i < j; i += lpr) {
                         const double wi = S.w[i], vri = S.vr1[i], ti = S.t[i];
                         double *zp = Zl + rl * XR + i * XC;
-                        const double z = *zp, vv = Vl[rl * XR + i * XC], yv = Yl[rl * XR + i * XC];
+                        const double z = *zp, vv = Vl[rl * XR + i * XC], yv = Yl[rl * YR + i * YCS];
                         zw += z * wi;
                         vw += vv * wi;
                         yt += yv * ti;
@@ -815,7 +831,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
                         // V(:, j) and the reduced column c of the own rows (step iii)
                         if (row == n && p.abft) {
                             V[row + (int64_t)j * ldw] = vchk;
-                            if (CACHE) Vl[rl * XR + j * XC] = vchk;
+                            if (VC) Vl[rl * XR + j * XC] = vchk;
                             Apan[row + (int64_t)c * ldw] = (tau != 0.0) ? b - vchk * (alpha - beta) : b;  // left term (R7)
                         } else {
                             double vv, av;
@@ -830,7 +846,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
                                 av = vv;
                             }
                             V[row + (int64_t)j * ldw] = vv;
-                            if (CACHE) Vl[rl * XR + j * XC] = vv;
+                            if (VC) Vl[rl * XR + j * XC] = vv;
                             Apan[row + (int64_t)c * ldw] = av;
                         }
                         // steps (iv)-(v)
@@ -838,7 +854,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
                         if (!last) Zl[rl * XR + j * XC] = u;
                         const double yy = tau * (an + u - yt);
                         Y[row + (int64_t)j * ldw] = yy;
-                        if (CACHE) Yl[rl * XR + j * XC] = yy;
+                        if (YC) Yl[rl * YR + j * YCS] = yy;
                         b0n = an - yr - yy;
                         if (vfy && is_data(row)) {
                             // D_r(row) = r(row) - sum_{col >= k} L(row, col); columns < k are logical zero
@@ -851,7 +867,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
                                 atomicMax(&p.ctl->drift_bits, (unsigned long long)__double_as_longlong(rel));
                             }
                         }
-                    } else if (CACHE) {
+                    } else if (VC) {
                         Vl[rl * XR + j * XC] = 0.0;  // rows outside the panel take no part in the dots
                     }
                     S.acol[rl] = an;
@@ -878,7 +894,9 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
             if (bid == 0 && wid == NW - 1)
                 for (int i = lane; i < FT_ACC_STRIDE; i += 32)
                     p.acc[((c + 2) & 3) * FT_ACC_SET_DOUBLES + i * FT_ACC_PAD] = 0.0;
-            if (!helper) {  // workers: the next column's b0 and masks are in smem
+            if (wide) {
+                __syncthreads();
+            } else if (!helper) {  // workers: the next column's b0 and masks are in smem
                 __syncwarp();
                 asm volatile("bar.sync 2, %0;\n" ::"n"(WKT) : "memory");
             }
@@ -896,14 +914,15 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
                 if (row >= k + jj + 2) s += Vl[rl * XR + jj * XC];
             p.Qr[row] += s;
         }
-    if (p.precheck_sums && tid < 2 * ib) {  // e^T Y, e^T V over the own data rows (pre-update check R15, fused)
-        const int jj = tid % ib;
-        const double *X = tid < ib ? Yl : Vl;
-        double s = 0.0;
-        for (int rl = 0; rl < R; rl++)
-            if (is_data(r0 + rl)) s += X[rl * XR + jj * XC];
-        atomicAdd(tid < ib ? &p.ctl->eY[jj] : &p.ctl->eV[jj], s);
-    }
+    if (p.precheck_sums)  // e^T Y, e^T V over the own data rows (pre-update check R15, fused): a warp per column
+        for (int o = wid; o < 2 * ib; o += NW) {
+            const int jj = o % ib;
+            double s = 0.0;
+            for (int rl = lane; rl < R; rl += 32)
+                if (is_data(r0 + rl)) s += o < ib ? Yl[rl * YR + jj * YCS] : Vl[rl * XR + jj * XC];
+            s = warp_sum(s);
+            if (lane == 0) atomicAdd(o < ib ? &p.ctl->eY[jj] : &p.ctl->eV[jj], s);
+        }
     if (bid == 0 && tid == 0 && p.abft) p.Qc[n] += qc_corner;
     if (bid == 0) {
         double tm = 0.0;
@@ -932,8 +951,9 @@ cudaError_t ft_launch_panel_multi(const PanelLaunch &L, int nsm, cudaStream_t s)
         int dev = 0;
         cudaGetDevice(&dev);
         cudaDeviceGetAttribute(&max_smem, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
-        const void *fns[] = {(const void *)k_panel<true, false>, (const void *)k_panel<false, false>,
-                             (const void *)k_panel<true, true>, (const void *)k_panel<false, true>};
+        const void *fns[] = {(const void *)k_panel<2, false>, (const void *)k_panel<1, false>,
+                             (const void *)k_panel<0, false>, (const void *)k_panel<2, true>,
+                             (const void *)k_panel<1, true>, (const void *)k_panel<0, true>};
         for (const void *fn : fns) {
             cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem);
             if (e != cudaSuccess) return e;
@@ -960,20 +980,29 @@ cudaError_t ft_launch_panel_multi(const PanelLaunch &L, int nsm, cudaStream_t s)
     const int rmax = GR * gmax;
     if (rmax > WKT) return cudaErrorInvalidConfiguration;  // n beyond ~61k rows per GPU
     const size_t fixed = sizeof(PanelSmem);
-    const size_t want = fixed + (size_t)3 * VS * rmax * sizeof(double);
-    const bool cache = want <= (size_t)max_smem;
-    PanelLaunch Lx;
-    const PanelLaunch *Lp = &L;
-    if (explicit_path) {
-        Lx = L;
-        for (int i = 0; i < Lx.nr; i++) Lx.r[i].dbg_mode |= ((explicit_path & 0xff) ? 8 : 0) | (explicit_path >> 8);
-        Lp = &Lx;
+    const size_t row_bytes = (size_t)VS * rmax * sizeof(double);
+    // mode 1 (V, Z rows cached, Y global) is kept for tests only: at the sizes where mode 2 does
+    // not fit, the GEMV streams from HBM and needs the L1 that a >200 KB carve-out would take
+    int cache = fixed + 3 * row_bytes <= (size_t)max_smem ? 2 : 0;
+    if ((L.r[0].dbg_mode & 64) && cache > 1) cache = 1;  // test hooks: force the smaller caching modes
+    if (L.r[0].dbg_mode & 128) cache = 0;
+    const size_t want = fixed + (size_t)(cache == 2 ? 3 : (cache == 1 ? 2 : 0)) * row_bytes;
+    // wide single-GPU launches: the two-reduction kernel (ft_panel_wide.cu), see its header
+    if (L.nr == 1 && !mg && rmax >= 32 && !(L.r[0].dbg_mode & (8 | 64 | 128)) && !explicit_path)
+        return ft_launch_panel_wide(L, nsm, s);
+    PanelLaunch Lx = L;
+    for (int i = 0; i < Lx.nr; i++) {
+        Lx.r[i].wide = rmax >= 32 ? 1 : 0;
+        if (explicit_path) Lx.r[i].dbg_mode |= ((explicit_path & 0xff) ? 8 : 0) | (explicit_path >> 8);
     }
+    const PanelLaunch *Lp = &Lx;
     void *args[] = {const_cast<PanelLaunch *>(Lp)};
     g_ft_launches++;
-    const void *fn = mg ? (cache ? (const void *)k_panel<true, true> : (const void *)k_panel<false, true>)
-                        : (cache ? (const void *)k_panel<true, false> : (const void *)k_panel<false, false>);
-    return cudaLaunchCooperativeKernel(fn, dim3(grid * L.nr), dim3(PT), args, cache ? want : fixed, s);
+    const void *fn = mg ? (cache == 2 ? (const void *)k_panel<2, true>
+                                      : (cache == 1 ? (const void *)k_panel<1, true> : (const void *)k_panel<0, true>))
+                        : (cache == 2 ? (const void *)k_panel<2, false>
+                                      : (cache == 1 ? (const void *)k_panel<1, false> : (const void *)k_panel<0, false>));
+    return cudaLaunchCooperativeKernel(fn, dim3(grid * L.nr), dim3(PT), args, want, s);
 }
 
 cudaError_t ft_launch_panel(const PanelParams &p, int nsm, cudaStream_t s) {

@@ -6,6 +6,8 @@ Tolerances (readings R17/R18):
   * checksums at an iteration boundary: |chk_gpu - chk_ora| <= 1e-10 ||A||_F
   * fault runs: same tolerances as a fault-free run; located (i, j) equal the oracle's
 """
+import ctypes
+
 import numpy as np
 import pytest
 
@@ -86,6 +88,30 @@ def test_parity_medium(n, nb, dist):
     assert res.info == 0 and res.report.detected == 0
     check_against_oracle(A, dA, tau, nb=nb)
     assert res.report.max_drift_rel < 0.5  # fault-free checksum drift, units of n eps ||A||_F
+
+
+@pytest.mark.parametrize("n,nb,abft,bits", [(64, 16, True, 8), (300, 32, False, 8), (513, 64, True, 8),
+                                            (700, 32, True, 8), (513, 64, True, 64), (700, 32, False, 128),
+                                            (300, 64, True, 8 | 128)])
+def test_parity_explicit_path(n, nb, abft, bits):
+    """Every column on the explicit two-reduction path (bit 8: the one-reduction column's
+    cancellation fallback, ft_panel.cu) and/or the panel's smaller shared-memory modes (64: Y rows
+    global, 128: V/Y/Z rows global -- the large-n layouts): same parity bar, and agreement with the
+    default path to rounding."""
+    A = synth.matrix(n, dist="uniform")
+    L = ft.lib()
+    L.ft_debug_panel_path.argtypes = [ctypes.c_int]
+    L.ft_debug_panel_path(bits)
+    try:
+        dA, tau, res = gpu_reduce(A, nb=nb, abft=abft)
+    finally:
+        L.ft_debug_panel_path(0)
+    assert res.info == 0 and res.report.detected == 0, res.events
+    check_against_oracle(A, dA, tau, nb=nb)
+    dA1, tau1, res1 = gpu_reduce(A, nb=nb, abft=abft)
+    assert res1.info == 0
+    H0, H1 = np.triu(dA.cpu().numpy(), -1), np.triu(dA1.cpu().numpy(), -1)
+    assert np.abs(H0 - H1).max() <= 1e-11 * np.abs(H1).max()
 
 
 def test_parity_c2_full_size():
@@ -320,3 +346,35 @@ def test_abft_off_propagates_fig2():
     d = np.abs(np.triu(dA.cpu().numpy(), -1) - np.triu(Ao, -1)) > 1e-12 * np.abs(Ao).max()
     Hm = np.triu(np.ones((n, n), bool), -1)
     assert d[:, 33:][Hm[:, 33:]].mean() > 0.9
+
+
+def test_wide_panel_kernel_large():
+    """n = 6144, nb = 64: the early panels have >= 32 rows per CTA and run the two-reduction
+    wide kernel (ft_panel_wide.cu); the late ones the one-reduction kernel.  The oracle is too
+    slow here, so: agreement with the all-one-reduction-kernel run (explicit path forced) to
+    rounding, and the backward-error / orthogonality bounds of the north star, on the GPU."""
+    n, nb = 6144, 64
+    A = synth.matrix(n)
+    dA, tau, res = gpu_reduce(A, nb=nb)
+    assert res.info == 0 and res.report.detected == 0
+    L = ft.lib()
+    L.ft_debug_panel_path.argtypes = [ctypes.c_int]
+    L.ft_debug_panel_path(8)
+    try:
+        dB, tauB, resB = gpu_reduce(A, nb=nb)
+    finally:
+        L.ft_debug_panel_path(0)
+    assert resB.info == 0
+    H, HB = torch.triu(dA, -1), torch.triu(dB, -1)
+    assert float((H - HB).abs().max()) <= 1e-10 * float(HB.abs().max())
+    # the last reflectors are ill-conditioned functions of the data (two correct implementations
+    # differ by ~1e-12 at n = 1024 and ~5e-9 at n = 6144 there, R18); H above is norm-wise 1e-10
+    assert float((tau - tauB).abs().max()) <= 1e-7
+    Q, info = ft.dorghr(dA, tau, nb=nb)
+    assert info == 0
+    Ad = torch.from_numpy(A).cuda()
+    eps = 2.0 ** -52
+    n1 = lambda M: float(M.abs().sum(0).max())  # 1-norm
+    resid = n1(Ad - Q @ H @ Q.T) / (n * n1(Ad) * eps)
+    orth = n1(torch.eye(n, dtype=torch.float64, device="cuda") - Q.T @ Q) / (n * eps)
+    assert resid <= 30 and orth <= 30, (resid, orth)
