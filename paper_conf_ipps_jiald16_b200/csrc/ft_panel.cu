@@ -78,7 +78,9 @@ enum { SC_TAU, SC_BETA, SC_SCALE, SC_ALPHA, SC_VCHK, SC_Q, SC_XX, SC_FB };
 
 struct PanelSmem {
     double Ts[FT_NBMAX][FT_NBMAX + 1];  // Ts[a][b] = T(a, b)
-    double Gp[FT_NBMAX][FT_NBMAX + 1];  // Gram of V over rows >= c+1 (downdated by row c+1 in use)
+    double Km[FT_NBMAX][FT_NBMAX + 1];  // K = Gp T^T, Gp = Gram of V over rows >= c+1 (see tcol_gram)
+    double ku[FT_NBMAX], kst[FT_NBMAX]; // T V(c+1,:)^T, T t (scratch of the K update)
+    double cpart[3][4][32];             // helpers' partial (w, k) of the column chain
     double s1[FT_NBMAX], w[FT_NBMAX], t[FT_NBMAX], ep[FT_NBMAX];  // ep: e^T V over rows >= c+1
     double vr1[FT_NBMAX + 1];           // V(c+1, 0:j)
     double scal[16];                    // SC_*
@@ -136,6 +138,41 @@ __device__ __forceinline__ double group8_sum(double v) {
     return v;
 }
 
+// Partial sums over a in [a0, a1) of w = T^T s1 and k = K s1 for outputs la = lane, lb = lane + 32
+// (T, K are zero beyond the current column count).  8 operand rows per batch: all loads of a
+// batch are in flight together.
+__device__ __forceinline__ void chain_part(const PanelSmem &S, int a0, int a1, int la, int lb, double &wa,
+                                           double &wb, double &ka, double &kb) {
+    double wa1 = 0.0, wb1 = 0.0, ka1 = 0.0, kb1 = 0.0;
+#pragma unroll 1
+    for (int b0 = a0; b0 < a1; b0 += 8) {
+        double sv[8], ta[8], tb[8], xa[8], xb[8];
+#pragma unroll
+        for (int u = 0; u < 8; u++) {
+            sv[u] = b0 + u < a1 ? S.s1[b0 + u] : 0.0;
+            ta[u] = S.Ts[b0 + u][la];
+            tb[u] = S.Ts[b0 + u][lb];
+            xa[u] = S.Km[la][b0 + u];
+            xb[u] = S.Km[lb][b0 + u];
+        }
+#pragma unroll
+        for (int u = 0; u < 8; u += 2) {
+            wa += ta[u] * sv[u];
+            wb += tb[u] * sv[u];
+            ka += xa[u] * sv[u];
+            kb += xb[u] * sv[u];
+            wa1 += ta[u + 1] * sv[u + 1];
+            wb1 += tb[u + 1] * sv[u + 1];
+            ka1 += xa[u + 1] * sv[u + 1];
+            kb1 += xb[u + 1] * sv[u + 1];
+        }
+    }
+    wa += wa1;
+    wb += wb1;
+    ka += ka1;
+    kb += kb1;
+}
+
 // T(:, j) and the carried Gram / e^T V of the next column, from the column's scalars in smem;
 // threads t0 = 0..nthr-1 (whole warps) of the calling warps take part.  It runs in helper
 // warps concurrently with the GEMV (and on the explicit path after it).  Out of line on purpose:
@@ -143,41 +180,55 @@ __device__ __forceinline__ double group8_sum(double v) {
 // addressed from a register not yet defined for the current column (nvcc 12.9, sm_100a).
 __device__ __noinline__ void tcol_gram(PanelSmem &S, const int j, const int t0, const int nthr, const bool last) {
     const double tau = S.scal[SC_TAU], scale = S.scal[SC_SCALE];
-    // T(a, j) = -tau sum_{b=a}^{j-1} T(a, b) t(b), an 8-lane group per a
+    // per row c < j of T (an 8-lane group each): st = T(c, :) t, sv = T(c, :) V(c+1, :)^T;
+    // T(c, j) = -tau st (DLAHR2 step v)
     const int sl = t0 >> 3, gg = t0 & 7, nsl = nthr >> 3;
     for (int a0 = 0; a0 < j; a0 += nsl) {
-        const int a = a0 + sl;
-        double s0 = 0.0, s1 = 0.0;
-        if (a < j)
+        const int c = a0 + sl;
+        double st0 = 0.0, st1 = 0.0, sv0 = 0.0, sv1 = 0.0;
+        if (c < j)
 #pragma unroll
             for (int u = 0; u < FT_NBMAX / 8; u += 2) {
                 const int ba = gg + 8 * u, bb2 = ba + 8;
-                if (ba < j) s0 += S.Ts[a][ba] * S.t[ba];
-                if (bb2 < j) s1 += S.Ts[a][bb2] * S.t[bb2];
+                if (ba < j) {
+                    const double tv = S.Ts[c][ba];
+                    st0 += tv * S.t[ba];
+                    sv0 += tv * S.vr1[ba];
+                }
+                if (bb2 < j) {
+                    const double tv = S.Ts[c][bb2];
+                    st1 += tv * S.t[bb2];
+                    sv1 += tv * S.vr1[bb2];
+                }
             }
-        const double s = group8_sum(s0 + s1);
-        if (a < j && gg == 0) S.Ts[a][j] = -tau * s;
+        const double st = group8_sum(st0 + st1), sv = group8_sum(sv0 + sv1);
+        if (c < j && gg == 0) {
+            S.Ts[c][j] = -tau * st;
+            S.kst[c] = st;
+            S.ku[c] = sv;
+        }
     }
     if (t0 == 0) S.Ts[j][j] = tau;
     if (!last) {
-        // Gram of V over rows >= c+2 (the downdate by row c+1 of the matrix in use), new
-        // row/column j = t - V(c+1,:), scale^2 ||x||^2; the next column downdates by row c+2.
-        // Thread (a, half) updates half of row a: independent read-modify-writes, pipelined.
-        const double xx = S.scal[SC_XX];
+        // K = Gp T^T for the next column, without Gp itself.  Gp_new = [Gp - v v^T, g; g^T, sigma]
+        // (v = V(c+1, 0:j), g = t - v, sigma = scale^2 ||x||^2) and T_new = [T, tc; 0, tau]
+        // (tc = -tau T t) give
+        //   K_new(a, c) = K(a, c) - v(a) (T v)(c) + g(a) tc(c)      a, c < j
+        //   K_new(a, j) = g(a) tau,   K_new(j, c) = (T g)(c) + sigma tc(c),   K_new(j, j) = sigma tau
+        asm volatile("bar.sync 3, %0;\n" ::"r"(nthr) : "memory");
+        const double sigma = scale * scale * S.scal[SC_XX];
         const int J1 = j + 1;
         for (int r = t0; r < 2 * J1; r += nthr) {
             const int a = r >> 1, h = r & 1;
-            const double va = S.vr1[a];
             if (a < j) {
+                const double va = S.vr1[a], ga = S.t[a] - va;
 #pragma unroll 4
-                for (int b2 = h; b2 < j; b2 += 2) S.Gp[a][b2] -= va * S.vr1[b2];
-                if (h == 0) {
-                    const double g = S.t[a] - va;
-                    S.Gp[a][j] = g;
-                    S.Gp[j][a] = g;
-                }
-            } else if (h == 0) {
-                S.Gp[j][j] = scale * scale * xx;
+                for (int c = h; c < j; c += 2) S.Km[a][c] += -va * S.ku[c] - tau * ga * S.kst[c];
+                if (h == 0) S.Km[a][j] = ga * tau;
+            } else {
+#pragma unroll 4
+                for (int c = h; c < j; c += 2) S.Km[j][c] = (S.kst[c] - S.ku[c]) - sigma * tau * S.kst[c];
+                if (h == 0) S.Km[j][j] = sigma * tau;
             }
         }
         // e^T V over rows >= c+2
@@ -447,7 +498,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
 #pragma unroll 1
     for (int i = tid; i < FT_NBMAX * (FT_NBMAX + 1); i += PT) {
         (&S.Ts[0][0])[i] = 0.0;
-        (&S.Gp[0][0])[i] = 0.0;
+        (&S.Km[0][0])[i] = 0.0;
     }
     if (p.ckpt) {
         // diskless checkpoint of the panel columns, r, c, kappa, Qr, Qc, Fr, taken
@@ -566,52 +617,30 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
             }
             __syncwarp();
             PROBE(10);
-            double wa0 = 0.0, wa1 = 0.0, wb0 = 0.0, wb1 = 0.0;  // T is upper triangular, zero beyond j
+            // w = T^T s1 and k = K s1 (K = Gp T^T: G w = k - V(c+1,:)^T q); narrow launches split
+            // the rows a over warp 0 and the three helpers (named barrier 4), wide ones use warp 0
+            double wa0 = 0.0, wb0 = 0.0, ka0 = 0.0, kb0 = 0.0;
+            if (!wide) {
+                asm volatile("bar.sync 4, 128;\n" ::: "memory");  // s1 staged
+                const int span = ((j + 31) >> 5) << 3;
+                chain_part(S, 0, min(span, j), la, lb, wa0, wb0, ka0, kb0);
+                asm volatile("bar.sync 4, 128;\n" ::: "memory");  // helpers' partials in smem
 #pragma unroll
-            for (int a0 = 0; a0 < FT_NBMAX; a0 += 8) {
-                if (a0 < j) {
-                    double sv[8], ta[8], tb[8];
-#pragma unroll
-                    for (int u = 0; u < 8; u++) {
-                        sv[u] = a0 + u < j ? S.s1[a0 + u] : 0.0;
-                        ta[u] = S.Ts[a0 + u][la];
-                        tb[u] = S.Ts[a0 + u][lb];
-                    }
-#pragma unroll
-                    for (int u = 0; u < 8; u += 2) {
-                        wa0 += ta[u] * sv[u];
-                        wb0 += tb[u] * sv[u];
-                        wa1 += ta[u + 1] * sv[u + 1];
-                        wb1 += tb[u + 1] * sv[u + 1];
-                    }
+                for (int h = 0; h < 3; h++) {
+                    wa0 += S.cpart[h][0][lane];
+                    wb0 += S.cpart[h][1][lane];
+                    ka0 += S.cpart[h][2][lane];
+                    kb0 += S.cpart[h][3][lane];
                 }
+            } else {
+                chain_part(S, 0, j, la, lb, wa0, wb0, ka0, kb0);
             }
+            const double wa1 = 0.0, wb1 = 0.0, ka1 = 0.0, kb1 = 0.0;
             const double wa = la < j ? wa0 + wa1 : 0.0, wb = lb < j ? wb0 + wb1 : 0.0;
+            const double gpa = ka0 + ka1, gpb = kb0 + kb1;  // (Gp w)(o)
             S.w[la] = wa;
             S.w[lb] = wb;
-            __syncwarp();
             PROBE(11);
-            double ga0 = 0.0, ga1 = 0.0, gb0 = 0.0, gb1 = 0.0;  // Gp is zero beyond j, so is w
-#pragma unroll
-            for (int a0 = 0; a0 < FT_NBMAX; a0 += 8) {
-                if (a0 < j) {
-                    double wv[8], xa[8], xb[8];
-#pragma unroll
-                    for (int u = 0; u < 8; u++) {
-                        wv[u] = S.w[a0 + u];
-                        xa[u] = S.Gp[la][a0 + u];
-                        xb[u] = S.Gp[lb][a0 + u];
-                    }
-#pragma unroll
-                    for (int u = 0; u < 8; u += 2) {
-                        ga0 += xa[u] * wv[u];
-                        gb0 += xb[u] * wv[u];
-                        ga1 += xa[u + 1] * wv[u + 1];
-                        gb1 += xb[u + 1] * wv[u + 1];
-                    }
-                }
-            }
-            const double gpa = ga0 + ga1, gpb = gb0 + gb1;
             const double epa = la < j ? S.ep[la] : 0.0, epb = lb < j ? S.ep[lb] : 0.0;
             double q = vra * wa + vrb * wb, sw = sxa * wa + sxb * wb, ew = epa * wa + epb * wb;
             double wgw = wa * gpa + wb * gpb;
@@ -656,6 +685,18 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
             // helpers (warps 4, 8, 12: sub-partition 0, no GEMV): T(:, j) and the carried Gram
             // while the GEMV streams (skipped on the explicit path: done after its second sync)
             __syncwarp();
+            {  // their quarter of the chain's w = T^T s1, k = K s1
+                const int h = (wid >> 2) - 1, span = ((j + 31) >> 5) << 3;
+                double pw = 0.0, pwb = 0.0, pk = 0.0, pkb = 0.0;
+                asm volatile("bar.sync 4, 128;\n" ::: "memory");  // s1 staged by warp 0
+                chain_part(S, min((h + 1) * span, j), min((h + 2) * span, j), lane, lane + 32, pw, pwb, pk, pkb);
+                S.cpart[h][0][lane] = pw;
+                S.cpart[h][1][lane] = pwb;
+                S.cpart[h][2][lane] = pk;
+                S.cpart[h][3][lane] = pkb;
+                __syncwarp();
+                asm volatile("bar.sync 4, 128;\n" ::: "memory");
+            }
             asm volatile("bar.sync 1, 128;\n" ::: "memory");
             if (S.scal[SC_FB] == 0.0 && !MG && !(p.dbg_mode & 16)) tcol_gram(S, j, ((wid >> 2) - 1) * 32 + lane, 96, last);
         }
