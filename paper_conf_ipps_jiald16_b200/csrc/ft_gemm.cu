@@ -448,6 +448,19 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
         colok[mi] = cols[mi] < ncols;
         colp[mi] = p.A + (int64_t)(cb + (colok[mi] ? cols[mi] : 0)) * p.lda;
     }
+    // fused end check: this CTA's share of sum r and sum c -- the entries it writes (column n:
+    // r(k+1:n), row n: c(e:n)) in the tile epilogues, and a grid-strided slice of the entries
+    // this launch does not touch (r(0:k+1), c(0:e), final since the right update / panel)
+    double es_r = 0.0, es_c = 0.0;
+    const int en = p.n;
+    if (p.endcheck) {
+        const int nb = gridDim.x * gridDim.y, b = blockIdx.y * gridDim.x + blockIdx.x;
+        const int nr = p.r_lo, ncc = p.c_lo;  // r(0:k+1), c(0:e)
+        for (int x = b * UT + tid; x < nr + ncc; x += nb * UT) {
+            if (x < nr) es_r += __ldcg(p.A + x + (int64_t)en * p.lda);
+            else es_c += __ldcg(p.A + en + (int64_t)(x - nr) * p.lda);
+        }
+    }
     for (int tt = t0; tt < t1; tt++) {
         const int st = (tt - t0) & 1;
         const int r = rbase + tt * UB;
@@ -488,6 +501,17 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
                 const double x = sg * acc[mi][ni][0], y = sg * acc[mi][ni][1];
                 if (full) *reinterpret_cast<double2 *>(colp[mi] + row) = make_double2(x, y);
                 else store_pair(colp[mi], row, lo, hi, colok[mi], x, y);
+                if (p.endcheck && colok[mi]) {
+                    const int gc = cb + cols[mi];
+                    const bool in0 = row >= lo && row < hi, in1 = row + 1 >= lo && row + 1 < hi;
+                    if (gc == en) {  // r entries (kappa = row n excluded)
+                        if (in0 && row < en) es_r += x;
+                        if (in1 && row + 1 < en) es_r += y;
+                    } else if (gc < en) {  // c entries
+                        if (in0 && row == en) es_c += x;
+                        if (in1 && row + 1 == en) es_c += y;
+                    }
+                }
             }
         __syncthreads();  // Vr[st] is refilled two tiles later
     }
@@ -506,38 +530,36 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
         }
     }
     if (!p.endcheck) return;
-    // fused end-of-iteration check (Alg. 3 l.12-13; R11/R22): once every CTA has finished, the
-    // last one compares sum r and sum c with kappa (EAGER) or with each other (PAPER)
+    // fused end-of-iteration check (Alg. 3 l.12-13; R11/R22): the CTA's partial sums go into
+    // ctl->sums[2:4]; once every CTA has finished, the last one compares sum r and sum c with
+    // kappa (EAGER) or with each other (PAPER)
     __shared__ int last;
     __shared__ double red2[2][UT / 32];
-    __threadfence();
+    es_r = warp_sum(es_r);
+    es_c = warp_sum(es_c);
+    if (lane == 0) {
+        red2[0][warp] = es_r;
+        red2[1][warp] = es_c;
+    }
     __syncthreads();
-    if (tid == 0) last = atomicAdd(&p.ectl->done_left, 1) == (int)(gridDim.x * gridDim.y) - 1;
+    if (tid == 0) {
+        double a = 0.0, b = 0.0;
+        for (int w = 0; w < UT / 32; w++) {
+            a += red2[0][w];
+            b += red2[1][w];
+        }
+        atomicAdd(&p.ectl->sums[2], a);
+        atomicAdd(&p.ectl->sums[3], b);
+        __threadfence();
+        last = atomicAdd(&p.ectl->done_left, 1) == (int)(gridDim.x * gridDim.y) - 1;
+    }
     __syncthreads();
-    if (!last) return;
+    if (!last || tid != 0) return;
     __threadfence();
     const int n = p.n;
-    double sr = 0.0, sc = 0.0;
-    {
-        const int per = (n + UT - 1) / UT, i0 = tid * per, cnt = min(per, n - i0);
-        if (cnt > 0) {
-            sr = sum_strided(p.A + i0 + (int64_t)n * p.lda, 1, cnt);
-            sc = sum_strided(p.A + n + (int64_t)i0 * p.lda, p.lda, cnt);
-        }
-    }
-    sr = warp_sum(sr);
-    sc = warp_sum(sc);
-    if (lane == 0) {
-        red2[0][warp] = sr;
-        red2[1][warp] = sc;
-    }
-    __syncthreads();
-    if (tid != 0) return;
-    double Sr = 0.0, Sc = 0.0;
-    for (int w = 0; w < UT / 32; w++) {
-        Sr += red2[0][w];
-        Sc += red2[1][w];
-    }
+    const double Sr = __ldcg(&p.ectl->sums[2]), Sc = __ldcg(&p.ectl->sums[3]);
+    p.ectl->sums[2] = 0.0;
+    p.ectl->sums[3] = 0.0;
     FtCtl *ctl = p.ectl;
     const double kap = __ldcg(p.A + n + (int64_t)n * p.lda);
     const double tauS = ctl->c_thr * (double)n * 2.220446049250313e-16 * ctl->normF * sqrt((double)n);

@@ -502,8 +502,8 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
     }
     if (p.ckpt) {
         // diskless checkpoint of the panel columns, r, c, kappa, Qr, Qc, Fr, taken
-        // before anything is modified: own rows by their owner, c by the owner of row n (it
-        // rewrites c(k:e)), the rest grid-strided; all of it precedes this CTA's first arrival
+        // before anything is modified: own rows by their owner, the rest grid-strided; all of it
+        // precedes this CTA's first arrival
         const int rend = p.abft ? n + 1 : ihi;
         for (int x = tid; x < R * ib; x += PT) {
             const int rl = x % R, jj = x / R, row = r0 + rl;
@@ -520,8 +520,9 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
             p.ck_q[ldw + i] = p.Qc[i];
             p.ck_q[2 * ldw + i] = p.Fr[i];
         }
-        if (r0 <= n && n < r1)
-            for (int i = tid; i <= n; i += PT) p.ck_c[i] = A[n + (int64_t)i * ldw];
+        // the checksum row c, grid-strided: every copy precedes its CTA's first arrival, and the
+        // owner of row n rewrites c(k:e) only after that first grid sync
+        for (int i = gi; i <= n; i += gstride) p.ck_c[i] = A[n + (int64_t)i * ldw];
     }
     {
         // column k: b0 = A(:, k); publish its x part (rows >= k+2) and b0(k+1)

@@ -261,8 +261,8 @@ __global__ void __launch_bounds__(PT, 1) k_panel_wide(const __grid_constant__ Pa
     for (int i = tid; i < FT_NBMAX * (FT_NBMAX + 1); i += PT) (&S.Ts[0][0])[i] = 0.0;
     if (p.ckpt) {
         // diskless checkpoint of the panel columns, r, c, kappa, Qr, Qc, Fr, taken
-        // before anything is modified: own rows by their owner, c by the owner of row n (it
-        // rewrites c(k:e)), the rest grid-strided; all of it precedes this CTA's first arrival
+        // before anything is modified: own rows by their owner, the rest grid-strided; all of it
+        // precedes this CTA's first arrival
         const int rend = p.abft ? n + 1 : ihi;
         for (int x = tid; x < R * ib; x += PT) {
             const int rl = x % R, jj = x / R, row = r0 + rl;
@@ -279,8 +279,9 @@ __global__ void __launch_bounds__(PT, 1) k_panel_wide(const __grid_constant__ Pa
             p.ck_q[ldw + i] = p.Qc[i];
             p.ck_q[2 * ldw + i] = p.Fr[i];
         }
-        if (r0 <= n && n < r1)
-            for (int i = tid; i <= n; i += PT) p.ck_c[i] = A[n + (int64_t)i * ldw];
+        // the checksum row c, grid-strided: every copy precedes its CTA's first arrival, and the
+        // owner of row n rewrites c(k:e) only after that first grid sync
+        for (int i = gi; i <= n; i += gstride) p.ck_c[i] = A[n + (int64_t)i * ldw];
     }
     for (int rl = tid; rl < R; rl += PT) {
         const int row = r0 + rl;
