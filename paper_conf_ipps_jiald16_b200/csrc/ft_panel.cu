@@ -548,7 +548,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
     const double c_thr = p.ctl->c_thr;
     const double tau_abs = c_thr * (double)n * 2.220446049250313e-16 * p.ctl->normF;
     // lanes per row in the combine: a whole warp per row for small row blocks
-    const int lpr = R <= nwk ? 32 : (R <= 2 * nwk ? 16 : 8);
+    const int lpr = 8;  // 8 lanes per row: 3 shuffle rounds (a round costs ~4 dependent FMAs)
     const int gl = wtid & (lpr - 1), grp = wtid / lpr, ngrp = wkt / lpr;
     auto gsum = [&](double v) {  // sum over the lpr lanes of a row group
 #pragma unroll
