@@ -88,6 +88,8 @@ struct Work {
     unsigned *bar = nullptr;
     int *strip_done = nullptr;
     cudaStream_t cap_stream = nullptr;  // graph capture stream (library-owned)
+    cudaStream_t copy_stream = nullptr; // host-buffer calls: D2H of finished columns beside the panels
+    cudaEvent_t copy_ev = nullptr;
     FtCtl *ctl = nullptr;
     FtFix *fixes = nullptr;
     int nsm = 0;
@@ -387,6 +389,11 @@ struct Call {
     std::vector<ft_event> events;
     int detected = 0, corrected = 0, rollbacks = 0, redos = 0, uncorrectable = 0;
     int npanels = 0;
+    // host-buffer call (ft_dgehrd_host): the input is copied straight into the working array and
+    // every iteration's finished columns [k, e) are copied back on w->copy_stream while the
+    // following panels run (they are never touched again, except by a recovery: re-copied)
+    double *hA = nullptr;
+    int64_t hlda = 0;
     int rend() const { return abft ? n + 1 : ihi; }
     int cend() const { return abft ? n + 1 : n; }
     int pk(int t) const { return ilo - 1 + t * nb; }
@@ -675,6 +682,13 @@ int enqueue_panel(Call &C, int t) {
     if (left_update(C, t, -1.0, trailing_nsplit(C, t), fuse_end ? 1 : 0, fuse_pre)) return FT_E_CUDA;
     if (inject_at(C, t, FT_PHASE_AFTER_UPDATE)) return FT_E_CUDA;
     if (C.abft && !fuse_end) CK(ft_endcheck(w.Aw, w.ldw, n, C.ihi, k, ib, t, C.policy, w.Fr, w.ctl, C.s));
+    if (C.hA) {  // columns [k, e) are final: back to the host beside the next panels
+        CK(cudaEventRecord(w.copy_ev, C.s));
+        CK(cudaStreamWaitEvent(w.copy_stream, w.copy_ev, 0));
+        CK(cudaMemcpy2DAsync(C.hA + (int64_t)k * C.hlda, (size_t)C.hlda * sizeof(double), w.Aw + (int64_t)k * w.ldw,
+                             (size_t)w.ldw * sizeof(double), n * sizeof(double), ib, cudaMemcpyDeviceToHost,
+                             w.copy_stream));
+    }
     return 0;
 }
 
@@ -802,7 +816,11 @@ int enqueue_start(Call &C, const double *dA, int lda) {
     CK(cudaMemsetAsync(w.Aw, 0, (size_t)w.ldw * (n + 1) * sizeof(double), s));
     CK(cudaMemsetAsync(w.V, 0, (size_t)w.ldw * FT_NBMAX * sizeof(double), s));
     CK(cudaMemsetAsync(w.Y, 0, (size_t)w.ldw * FT_NBMAX * sizeof(double), s));
-    CK(ft_copy_in(dA, lda, w.Aw, w.ldw, n, s));
+    if (C.hA)
+        CK(cudaMemcpy2DAsync(w.Aw, (size_t)w.ldw * sizeof(double), C.hA, (size_t)C.hlda * sizeof(double),
+                             n * sizeof(double), n, cudaMemcpyHostToDevice, s));
+    else
+        CK(ft_copy_in(dA, lda, w.Aw, w.ldw, n, s));
     CK(cudaMemsetAsync(w.bvec, 0, (size_t)4 * w.ldw * sizeof(double), s));  // b(q >= ihi) must read 0
     if (reset_panel_state(C)) return FT_E_CUDA;
     if (C.abft) {
@@ -834,11 +852,12 @@ int validate(int n, int ilo, int ihi, const void *A, int lda, const void *tau, c
     return 0;
 }
 
-int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opts *opts) {
+int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opts *opts, double *hA = nullptr,
+        int hlda = 0) {
     ft_opts o;
     ft_opts_default(&o);
     if (opts) o = *opts;
-    int info = validate(n, ilo, ihi, dA, lda, dtau, &o);
+    int info = validate(n, ilo, ihi, hA ? hA : dA, hA ? hlda : lda, dtau, &o);
     if (info) return info;
     cudaStream_t s = (cudaStream_t)o.stream;
     if (n == 0) return 0;
@@ -856,6 +875,12 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
     int rc = get_work(n, &C.w);
     if (rc) return rc;
     Work &w = *C.w;
+    if (hA && o.stop_after_panel < 0) {
+        C.hA = hA;
+        C.hlda = hlda;
+        if (!w.copy_stream) CK(cudaStreamCreateWithFlags(&w.copy_stream, cudaStreamNonBlocking));
+        if (!w.copy_ev) CK(cudaEventCreateWithFlags(&w.copy_ev, cudaEventDisableTiming));
+    }
     cudaEvent_t ev0, ev1;
     CK(cudaEventCreate(&ev0));
     CK(cudaEventCreate(&ev1));
@@ -873,7 +898,8 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
     if (graphable) {
         int dev = 0;
         CK(cudaGetDevice(&dev));
-        GraphKey key{dev, n, ilo, ihi, C.nb, C.abft, C.policy, C.c_thr, (const void *)dA, lda, (const void *)dtau};
+        GraphKey key{dev, n, ilo, ihi, C.nb, C.abft, C.policy, C.c_thr, C.hA ? (const void *)C.hA : (const void *)dA,
+                     C.hA ? (int)C.hlda : lda, (const void *)dtau};
         auto it = g_graphs.find(key);
         if (it != g_graphs.end() && it->second.exec) {
             CK(cudaGraphLaunch(it->second.exec, s));
@@ -891,6 +917,11 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
                 C.s = w.cap_stream;
                 rc2 = enqueue_start(C, dA, lda);
                 for (int t = 0; t < last && !rc2; t++) rc2 = enqueue_panel(C, t);
+                if (C.hA && !rc2) {  // join the copy stream back into the capture
+                    if (cudaEventRecord(w.copy_ev, w.copy_stream) != cudaSuccess ||
+                        cudaStreamWaitEvent(w.cap_stream, w.copy_ev, 0) != cudaSuccess)
+                        rc2 = 1;
+                }
                 ce = cudaStreamEndCapture(w.cap_stream, &graph);
                 C.s = s;
             }
@@ -953,7 +984,29 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
             else if (r1) return r1;
         }
     }
-    CK(ft_copy_out(w.Aw, w.ldw, dA, lda, n, s));
+    if (C.hA) {
+        // join the column copies, then the columns no iteration finished ([0, ilo-1), the last
+        // ones) -- or all of them if a recovery or the final verification touched the matrix
+        CK(cudaEventRecord(w.copy_ev, w.copy_stream));
+        CK(cudaStreamWaitEvent(s, w.copy_ev, 0));
+        const bool touched = attempts > 0 || C.corrected > 0 || C.detected > 0;
+        const int k0 = touched ? n : ilo - 1;
+        const int e1 = touched ? 0 : (C.npanels > 0 ? C.pk(C.npanels - 1) + C.pib(C.npanels - 1) : 0);
+        auto d2h = [&](int c0, int c1) -> cudaError_t {
+            if (c1 <= c0) return cudaSuccess;
+            return cudaMemcpy2DAsync(C.hA + (int64_t)c0 * C.hlda, (size_t)C.hlda * sizeof(double),
+                                     w.Aw + (int64_t)c0 * w.ldw, (size_t)w.ldw * sizeof(double), n * sizeof(double),
+                                     c1 - c0, cudaMemcpyDeviceToHost, s);
+        };
+        if (touched) {
+            CK(d2h(0, n));
+        } else {
+            CK(d2h(0, std::min(k0, n)));
+            CK(d2h(std::max(e1, k0), n));
+        }
+    } else {
+        CK(ft_copy_out(w.Aw, w.ldw, dA, lda, n, s));
+    }
     if (o.stop_after_panel >= 0 && o.dchk_out && C.abft) {
         CK(cudaMemcpyAsync(o.dchk_out, w.Aw + (int64_t)n * w.ldw, n * sizeof(double), cudaMemcpyDeviceToDevice, s));
         CK(cudaMemcpy2DAsync(o.dchk_out + n, sizeof(double), w.Aw + n, w.ldw * sizeof(double), sizeof(double), n,
@@ -1031,28 +1084,32 @@ int ft_dgehrd_host(int n, int ilo, int ihi, double *hA, int lda, double *htau, c
     if (info) return info;
     if (n == 0) return 0;
     cudaStream_t s = (cudaStream_t)o.stream;
-    double *dA = nullptr, *dtau = nullptr;
-    // device staging buffers live with the workspace of this size
-    static std::map<int, std::pair<size_t, std::pair<double *, double *>>> stage;
+    // device tau lives with the workspace of this size; A goes straight into the working array
+    static std::map<int, std::pair<int, double *>> stage;
     int dev = 0;
     CK(cudaGetDevice(&dev));
     auto &st = stage[dev];
-    size_t need = (size_t)n * n;
-    if (st.first < need) {
-        if (st.second.first) cudaFree(st.second.first);
-        if (st.second.second) cudaFree(st.second.second);
-        CK(cudaMalloc(&st.second.first, need * sizeof(double)));
-        CK(cudaMalloc(&st.second.second, std::max(n, 2) * sizeof(double)));
-        st.first = need;
+    if (st.first < n) {
+        if (st.second) cudaFree(st.second);
+        CK(cudaMalloc(&st.second, std::max(n, 2) * sizeof(double)));
+        st.first = n;
     }
-    dA = st.second.first;
-    dtau = st.second.second;
-    CK(cudaMemcpy2DAsync(dA, n * sizeof(double), hA, (size_t)lda * sizeof(double), n * sizeof(double), n,
-                         cudaMemcpyHostToDevice, s));
-    info = run(n, ilo, ihi, dA, n, dtau, &o);
+    double *dtau = st.second;
+    if (o.stop_after_panel >= 0) {  // verify-hook calls: plain staging through a device copy
+        double *dA = nullptr;
+        CK(cudaMalloc(&dA, (size_t)n * n * sizeof(double)));
+        CK(cudaMemcpy2DAsync(dA, n * sizeof(double), hA, (size_t)lda * sizeof(double), n * sizeof(double), n,
+                             cudaMemcpyHostToDevice, s));
+        info = run(n, ilo, ihi, dA, n, dtau, &o);
+        if (!(info < 0 || info == FT_E_CUDA || info == FT_E_NOMEM))
+            CK(cudaMemcpy2DAsync(hA, (size_t)lda * sizeof(double), dA, n * sizeof(double), n * sizeof(double), n,
+                                 cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        cudaFree(dA);
+    } else {
+        info = run(n, ilo, ihi, nullptr, lda, dtau, &o, hA, lda);
+    }
     if (info < 0 || info == FT_E_CUDA || info == FT_E_NOMEM) return info;
-    CK(cudaMemcpy2DAsync(hA, (size_t)lda * sizeof(double), dA, n * sizeof(double), n * sizeof(double), n,
-                         cudaMemcpyDeviceToHost, s));
     if (n > 1) CK(cudaMemcpyAsync(htau, dtau, (n - 1) * sizeof(double), cudaMemcpyDeviceToHost, s));
     CK(cudaStreamSynchronize(s));
     return info;
