@@ -80,7 +80,6 @@ struct PanelSmem {
     double Ts[FT_NBMAX][FT_NBMAX + 1];  // Ts[a][b] = T(a, b)
     double Km[FT_NBMAX][FT_NBMAX + 1];  // K = Gp T^T, Gp = Gram of V over rows >= c+1 (see tcol_gram)
     double ku[FT_NBMAX], kst[FT_NBMAX]; // T V(c+1,:)^T, T t (scratch of the K update)
-    double cpart[3][4][32];             // helpers' partial (w, k) of the column chain
     double s1[FT_NBMAX], w[FT_NBMAX], t[FT_NBMAX], ep[FT_NBMAX];  // ep: e^T V over rows >= c+1
     double vr1[FT_NBMAX + 1];           // V(c+1, 0:j)
     double scal[16];                    // SC_*
@@ -618,24 +617,10 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
             }
             __syncwarp();
             PROBE(10);
-            // w = T^T s1 and k = K s1 (K = Gp T^T: G w = k - V(c+1,:)^T q); narrow launches split
-            // the rows a over warp 0 and the three helpers (named barrier 4), wide ones use warp 0
+            // w = T^T s1 and k = K s1 (K = Gp T^T: G w = k - V(c+1,:)^T q).  (Splitting this pass
+            // over warp 0 and the helpers was measured slower: the chunk is latency-bound.)
             double wa0 = 0.0, wb0 = 0.0, ka0 = 0.0, kb0 = 0.0;
-            if (!wide) {
-                asm volatile("bar.sync 4, 128;\n" ::: "memory");  // s1 staged
-                const int span = ((j + 31) >> 5) << 3;
-                chain_part(S, 0, min(span, j), la, lb, wa0, wb0, ka0, kb0);
-                asm volatile("bar.sync 4, 128;\n" ::: "memory");  // helpers' partials in smem
-#pragma unroll
-                for (int h = 0; h < 3; h++) {
-                    wa0 += S.cpart[h][0][lane];
-                    wb0 += S.cpart[h][1][lane];
-                    ka0 += S.cpart[h][2][lane];
-                    kb0 += S.cpart[h][3][lane];
-                }
-            } else {
-                chain_part(S, 0, j, la, lb, wa0, wb0, ka0, kb0);
-            }
+            chain_part(S, 0, j, la, lb, wa0, wb0, ka0, kb0);
             const double wa1 = 0.0, wb1 = 0.0, ka1 = 0.0, kb1 = 0.0;
             const double wa = la < j ? wa0 + wa1 : 0.0, wb = lb < j ? wb0 + wb1 : 0.0;
             const double gpa = ka0 + ka1, gpb = kb0 + kb1;  // (Gp w)(o)
@@ -686,18 +671,6 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
             // helpers (warps 4, 8, 12: sub-partition 0, no GEMV): T(:, j) and the carried Gram
             // while the GEMV streams (skipped on the explicit path: done after its second sync)
             __syncwarp();
-            {  // their quarter of the chain's w = T^T s1, k = K s1
-                const int h = (wid >> 2) - 1, span = ((j + 31) >> 5) << 3;
-                double pw = 0.0, pwb = 0.0, pk = 0.0, pkb = 0.0;
-                asm volatile("bar.sync 4, 128;\n" ::: "memory");  // s1 staged by warp 0
-                chain_part(S, min((h + 1) * span, j), min((h + 2) * span, j), lane, lane + 32, pw, pwb, pk, pkb);
-                S.cpart[h][0][lane] = pw;
-                S.cpart[h][1][lane] = pwb;
-                S.cpart[h][2][lane] = pk;
-                S.cpart[h][3][lane] = pkb;
-                __syncwarp();
-                asm volatile("bar.sync 4, 128;\n" ::: "memory");
-            }
             asm volatile("bar.sync 1, 128;\n" ::: "memory");
             if (S.scal[SC_FB] == 0.0 && !MG && !(p.dbg_mode & 16)) tcol_gram(S, j, ((wid >> 2) - 1) * 32 + lane, 96, last);
         }

@@ -64,9 +64,10 @@ def main():
               f"{10 / 3 * n ** 3 / ms / 1e6:.1f} Gflop/s", flush=True)
     if dbg is not None:
         d = dbg.cpu().numpy()
-        names = {0: "start", 1: "coldot", 2: "sync", 10: "c_loads", 11: "c_w", 12: "c_Gw_shfl", 9: "c_dlarfg",
+        names = {0: "start", 1: "coldot", 2: "sync", 10: "c_loads", 4: "c_bar4a", 5: "c_part", 6: "c_bar4b",
+                 11: "c_w", 12: "c_Gw_shfl", 9: "c_dlarfg",
                  3: "gemv_join", 7: "explicit/xchg", 14: "cmb_dots", 15: "cmb_gsum", 13: "cmb_leader", 8: "T_G_bar"}
-        order = [0, 1, 2, 10, 11, 12, 9, 3, 7, 14, 15, 13, 8]
+        order = [0, 1, 2, 10, 4, 5, 6, 11, 12, 9, 3, 7, 14, 15, 13, 8]
         tot = {}
         ncol = 0
         for j in range(64):
