@@ -28,7 +28,7 @@ def dlarfg(alpha, xx):
     return (beta - alpha) / beta, beta, 1.0 / (alpha - beta)
 
 
-def panel(A, k, ib, onesync, gamma, stats):
+def panel(A, k, ib, onesync, gamma, stats, carry_k=False):
     n = A.shape[0]
     A0 = A.copy()
     rows = np.arange(n)
@@ -37,6 +37,7 @@ def panel(A, k, ib, onesync, gamma, stats):
     T = np.zeros((ib, ib))
     Z = np.zeros((n, ib))
     G = np.zeros((ib, ib))
+    Km = np.zeros((ib, ib))  # K = Gp T^T (carry_k): G w = K s1 - V(c+1,:)^T q
     tprev = None
     for j in range(ib):
         c = k + j
@@ -60,7 +61,14 @@ def panel(A, k, ib, onesync, gamma, stats):
             Z[:, :j] -= np.outer(A0[:, c + 1], vr1)
         w = T[:j, :j].T @ s1
         fast = onesync
-        if onesync:
+        if onesync and carry_k:
+            Gw = Km[:j, :j] @ s1 - vr1 * (vr1 @ w)
+            xx = bb - 2.0 * (w @ sx) + w @ Gw
+            alpha = b0c1 - vr1 @ w
+            if not (xx >= gamma * (bb + w @ Gw)):
+                fast = False
+                stats["trip"] += 1
+        elif onesync:
             Gw = G[:j, :j] @ w
             xx = bb - 2.0 * (w @ sx) + w @ Gw
             alpha = b0c1 - vr1 @ w
@@ -84,13 +92,25 @@ def panel(A, k, ib, onesync, gamma, stats):
         if fast:
             g = A0[:, c + 2:] @ b0[c + 2:]
             u = scale * (g - Z[:, :j] @ w)
-            t = vr1 + scale * (sx - G[:j, :j] @ w)
+            t = vr1 + scale * (sx - Gw)
         else:
             u = scale * (A0[:, c + 2:] @ b[c + 2:])
             t = V[:, :j].T @ v
         Z[:, j] = u
         y = np.where(act, A0[:, c + 1] + u, 0.0)
         Y[:, j] = np.where(act, tau * (y - Y[:, :j] @ t), 0.0)
+        if carry_k:  # K_new = Gp_new T_new^T by the rank-2 update of ft_panel.cu (tcol_gram)
+            st = T[:j, :j] @ t
+            su = T[:j, :j] @ vr1
+            g_ = t - vr1
+            sigma = scale * scale * xx
+            tc = -tau * st
+            Kn = np.zeros((ib, ib))
+            Kn[:j, :j] = Km[:j, :j] - np.outer(vr1, su) + np.outer(g_, tc)
+            Kn[:j, j] = g_ * tau
+            Kn[j, :j] = (st - su) + sigma * tc
+            Kn[j, j] = sigma * tau
+            Km = Kn
         T[:j, j] = -tau * (T[:j, :j] @ t)
         T[j, j] = tau
         tprev, xxprev, scaleprev = t, xx, scale
@@ -98,7 +118,7 @@ def panel(A, k, ib, onesync, gamma, stats):
     return V, Y, T
 
 
-def blocked(A, nb, onesync, gamma=1.0 / 64, stats=None):
+def blocked(A, nb, onesync, gamma=1.0 / 64, stats=None, carry_k=False):
     A = A.copy()
     n = A.shape[0]
     tau = np.zeros(n - 1)
@@ -107,7 +127,7 @@ def blocked(A, nb, onesync, gamma=1.0 / 64, stats=None):
         ib = min(nb, n - 2 - k)
         e = k + ib
         A0 = A.copy()
-        V, Y, T = panel(A, k, ib, onesync, gamma, stats)
+        V, Y, T = panel(A, k, ib, onesync, gamma, stats, carry_k)
         tau[k:e] = np.diag(T)
         Ytop = A0[: k + 1, k + 1:] @ V[k + 1:, :] @ T
         Yf = Y.copy()
