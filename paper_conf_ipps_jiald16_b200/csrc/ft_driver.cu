@@ -394,6 +394,10 @@ struct Call {
     // following panels run (they are never touched again, except by a recovery: re-copied)
     double *hA = nullptr;
     int64_t hlda = 0;
+    // Y_top fused into the panel (small n: every panel launch is narrow): the rows above the
+    // panel ride through the panel's GEMV and Y recurrence (DLAHRD's formulation), and the
+    // M-part of the right update is the b0 of those rows (written by the panel)
+    bool fused_ytop = false;
     int rend() const { return abft ? n + 1 : ihi; }
     int cend() const { return abft ? n + 1 : n; }
     int pk(int t) const { return ilo - 1 + t * nb; }
@@ -515,8 +519,8 @@ int right_update(Call &C, int t, double sign, int do_w, bool precheck = false) {
     g.wsplit_stride = ((int64_t)C.n + 1 + 64) * FT_NBMAX;
     g.ctl = sign < 0 ? w.ctl : nullptr;
     // M-part: rows 0..k of the panel columns k+1..e-1 (DGEHRD's DTRMM + DAXPY), as one extra
-    // strip of the trailing launch
-    g.has_m = 1;
+    // strip of the trailing launch (done by the panel itself when Y_top is fused)
+    g.has_m = (C.fused_ytop && sign < 0) ? 0 : 1;
     g.m_r_hi = k + 1;
     g.m_c_lo = k + 1;
     g.m_c_hi = e;
@@ -630,7 +634,8 @@ int enqueue_panel(Call &C, int t) {
     p.dbg = (t == g_dbg_panel) ? g_dbg_buf : nullptr;
     p.dbg_mode = ((t == g_dbg_panel) ? g_dbg_mode : 0) | g_panel_path;
     const int gr = ft_panel_group_rows();
-    p.rbase = ((k + 1) / gr) * gr;
+    p.rbase = C.fused_ytop ? 0 : ((k + 1) / gr) * gr;
+    p.ytop = C.fused_ytop ? 1 : 0;
     int rendp = (C.rend() + gr - 1) / gr * gr;
     p.ngroups = (rendp - p.rbase) / gr;
     cudaEvent_t pe0 = nullptr, pe1 = nullptr;
@@ -644,7 +649,7 @@ int enqueue_panel(Call &C, int t) {
         CK(cudaEventRecord(pe1, C.s));
         g_panel_events.push_back({pe0, pe1});
     }
-    // Y_top = A(0:k+1, k+1:ihi) V T (+ area-1 row sums)
+    // Y_top = A(0:k+1, k+1:ihi) V T (+ area-1 row sums), unless the panel formed it
     YtopParams y{};
     y.A = w.Aw;
     y.ldw = w.ldw;
@@ -668,7 +673,7 @@ int enqueue_panel(Call &C, int t) {
     int ns = std::max(1, std::min({(2 * w.nsm) / nm, nkt / 2, 64}));
     while ((int64_t)ns * (k + 1) > kYtopRows) ns--;
     y.nsplit = std::max(ns, 1);
-    CK(ft_launch_ytop(y, C.s));
+    if (!C.fused_ytop) CK(ft_launch_ytop(y, C.s));
     if (inject_at(C, t, FT_PHASE_AFTER_PANEL)) return FT_E_CUDA;
     if (eager && !fuse_pre) {
         // a fault is scheduled after the panel: recompute the check sums after it
@@ -875,6 +880,8 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
     int rc = get_work(n, &C.w);
     if (rc) return rc;
     Work &w = *C.w;
+    // Y_top fused into the panel when every panel launch is narrow (<= 24 rows per CTA)
+    C.fused_ytop = (n + 1 + 7) / 8 <= 3 * w.nsm && !getenv("FT_NO_FUSED_YTOP");
     if (hA && o.stop_after_panel < 0) {
         C.hA = hA;
         C.hlda = hlda;

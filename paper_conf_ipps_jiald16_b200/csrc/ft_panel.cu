@@ -304,7 +304,11 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
     const int npart = R2p <= 32 ? ngw : ncl;  // partials per row pair
 
     auto is_data = [&](int row) { return row >= k + 1 && row < ihi; };
-    auto is_valid = [&](int row) { return (row >= k + 1 && row < ihi) || (p.abft && row == n); };
+    // fused Y_top: the rows 0..k above the panel take part in the GEMV, Y, Z and b0 (their b0 is
+    // the M-part of DGEHRD), never in the column dots, V or the reflectors
+    const bool ytop = p.ytop != 0;
+    auto is_top = [&](int row) { return ytop && row <= k; };
+    auto is_valid = [&](int row) { return (row >= k + 1 && row < ihi) || (p.abft && row == n) || (ytop && row <= k); };
 
     // ---- CTA-parallel building blocks of the column chain --------------------------------
     // row dot of row rl (an 8-lane group per row): sum_{jp < J} X(rl, jp) z[jp], J <= 64.
@@ -871,10 +875,11 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
                         Y[row + (int64_t)j * ldw] = yy;
                         if (YC) Yl[rl * YR + j * YCS] = yy;
                         b0n = an - yr - yy;
-                        if (vfy && is_data(row)) {
+                        if (vfy && (is_data(row) || is_top(row))) {
                             // D_r(row) = r(row) - sum_{col >= k} L(row, col); columns < k are logical zero
+                            // for data rows, the frozen finished-H sums Fr for the rows above (area 1)
                             rsum += S.acol[rl] + an;
-                            const double d = p.rcol[row] - rsum;
+                            const double d = p.rcol[row] - (is_top(row) ? p.Fr[row] : 0.0) - rsum;
                             if (not_within(d, tau_abs)) {
                                 atomicAdd(&p.ctl->nflag, 1);
                             } else if (tau_abs > 0.0) {
@@ -934,7 +939,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
             const int jj = o % ib;
             double s = 0.0;
             for (int rl = lane; rl < R; rl += 32)
-                if (is_data(r0 + rl)) s += o < ib ? Yl[rl * YR + jj * YCS] : Vl[rl * XR + jj * XC];
+                if (is_data(r0 + rl) || is_top(r0 + rl)) s += o < ib ? Yl[rl * YR + jj * YCS] : Vl[rl * XR + jj * XC];
             s = warp_sum(s);
             if (lane == 0) atomicAdd(o < ib ? &p.ctl->eY[jj] : &p.ctl->eV[jj], s);
         }
