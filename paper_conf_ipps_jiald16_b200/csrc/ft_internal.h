@@ -52,6 +52,7 @@ struct PanelParams {
     int rbase, ngroups;               // ft_panel_group_rows()-row groups starting at rbase
     int wide;                         // set by the launcher: >= 32 rows per CTA (GEMV on 15 warps)
     int ytop;                         // rows 0..k ride along (rbase = 0): Y_top and the M-part by the panel
+    int ncc;                          // set by the launcher: trailing columns whose row slabs live in smem
     // diskless checkpoint of the panel, taken in the kernel's prologue, or NULL
     double *ckpt, *ck_r, *ck_c, *ck_q, *Fr;
     int precheck_sums;  // add e^T Y, e^T V of the own rows into ctl->eY / eV (fused pre-update check)

@@ -36,6 +36,7 @@
 #include "ft_common.cuh"
 #include "ft_internal.h"
 
+#include <algorithm>
 #include <cstdio>
 #include <cstdlib>
 
@@ -288,6 +289,9 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
     double *Vl = VC ? dyn : V + r0;
     double *Zl = VC ? dyn + (int64_t)VS * R : p.Z + r0;
     double *Yl = YC ? dyn + (int64_t)2 * VS * R : Y + r0;
+    // the CTA's row slab of the columns [k+2, k+2+ncc) at panel start ([col][R]), mode 2 only
+    const int ncc = (CACHE == 2 && !MG) ? p.ncc : 0;
+    double *Ac = dyn + (int64_t)3 * VS * R;
     constexpr int64_t XR = VC ? VS : 1;  // row stride of V and Z
     const int64_t XC = VC ? 1 : ldw;     // column stride
     constexpr int64_t YR = YC ? VS : 1;  // of Y
@@ -439,43 +443,51 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
             }
         } else if (gemv_on && !(p.dbg_mode & 2)) {
             // bv is read with plain (L1-allocating) loads: the acquire at the grid barrier
-            // invalidated this SM's L1 before the trailing bar.sync released us
-            int col = c + 2 + cl;
+            // invalidated this SM's L1 before the trailing bar.sync released us.
+            // Columns [k+2, k+2+ncc) come from the CTA's shared-memory copy of its row slab
+            // (loaded once per panel), the rest from L2 / HBM.
+            auto run = [&](const double2 *__restrict__ base, int64_t cs2, int coff, int cbeg, int cstop) {
+                int col = cbeg + cl;
 #pragma unroll 1
-            for (; col + (GB - 1) * ncl < cend; col += GB * ncl) {
-                double2 a[GB];
-                double v[GB];
+                for (; col + (GB - 1) * ncl < cstop; col += GB * ncl) {
+                    double2 a[GB];
+                    double v[GB];
 #pragma unroll
-                for (int u = 0; u < GB; u++) {
-                    const int q = col + u * ncl;
-                    a[u] = A2[(int64_t)q * ldw2 + rp];
-                    v[u] = bv[q];
-                }
+                    for (int u = 0; u < GB; u++) {
+                        const int q = col + u * ncl;
+                        a[u] = base[(int64_t)(q - coff) * cs2 + rp];
+                        v[u] = bv[q];
+                    }
 #pragma unroll
-                for (int u = 0; u < GB; u++) {
-                    ya.x += a[u].x * v[u];
-                    ya.y += a[u].y * v[u];
-                    rs.x += a[u].x;  // row sums: used by the verify pass only (cheap, memory-bound loop)
-                    rs.y += a[u].y;
+                    for (int u = 0; u < GB; u++) {
+                        ya.x += a[u].x * v[u];
+                        ya.y += a[u].y * v[u];
+                        rs.x += a[u].x;  // row sums: used by the verify pass only (cheap, memory-bound loop)
+                        rs.y += a[u].y;
+                    }
                 }
-            }
-            if (col < cend) {  // ragged tail: one predicated batch (all loads in flight together)
-                double2 a[GB];
-                double v[GB];
+                if (col < cstop) {  // ragged tail: one predicated batch (all loads in flight together)
+                    double2 a[GB];
+                    double v[GB];
 #pragma unroll
-                for (int u = 0; u < GB; u++) {
-                    const int q = col + u * ncl;
-                    a[u] = q < cend ? A2[(int64_t)q * ldw2 + rp] : make_double2(0.0, 0.0);
-                    v[u] = q < cend ? bv[q] : 0.0;
-                }
+                    for (int u = 0; u < GB; u++) {
+                        const int q = col + u * ncl;
+                        a[u] = q < cstop ? base[(int64_t)(q - coff) * cs2 + rp] : make_double2(0.0, 0.0);
+                        v[u] = q < cstop ? bv[q] : 0.0;
+                    }
 #pragma unroll
-                for (int u = 0; u < GB; u++) {
-                    ya.x += a[u].x * v[u];
-                    ya.y += a[u].y * v[u];
-                    rs.x += a[u].x;
-                    rs.y += a[u].y;
+                    for (int u = 0; u < GB; u++) {
+                        ya.x += a[u].x * v[u];
+                        ya.y += a[u].y * v[u];
+                        rs.x += a[u].x;
+                        rs.y += a[u].y;
+                    }
                 }
-            }
+            };
+            const int csplit = min(cend, k + 2 + ncc);
+            if (c + 2 < csplit) run(reinterpret_cast<const double2 *>(Ac), R2, k + 2, c + 2, csplit);
+            const int cbeg = max(c + 2, csplit);
+            if (cbeg < cend) run(A2, ldw2, 0, cbeg, cend);
         }
         if (R2p <= 32) {
 #pragma unroll
@@ -544,6 +556,17 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
         }
     }
     if (tid < FT_NBMAX) S.ep[tid] = 0.0;
+    if (ncc > 0) {
+        // the row slab of columns [k+2, k+2+ncc) into shared memory: at panel start they hold
+        // A0, and column c's GEMV reads only columns >= c+2, which this panel has not written yet
+        const int R2c = R >> 1;
+        for (int x = tid; x < ncc * R2c; x += PT) {
+            const int cc = x / R2c, rq = x - cc * R2c;
+            cp_async16(Ac + (int64_t)cc * R + 2 * rq, A + (r0 + 2 * rq) + (int64_t)(k + 2 + cc) * ldw, 16);
+        }
+        cp_async_commit();
+        cp_async_wait<0>();
+    }
     if (tid == 0 && bid == 0) *p.bar_next = 0u;  // the next panel launch's counter
     __syncthreads();
 
@@ -1006,13 +1029,28 @@ cudaError_t ft_launch_panel_multi(const PanelLaunch &L, int nsm, cudaStream_t s)
     int cache = fixed + 3 * row_bytes <= (size_t)max_smem ? 2 : 0;
     if ((L.r[0].dbg_mode & 64) && cache > 1) cache = 1;  // test hooks: force the smaller caching modes
     if (L.r[0].dbg_mode & 128) cache = 0;
-    const size_t want = fixed + (size_t)(cache == 2 ? 3 : (cache == 1 ? 2 : 0)) * row_bytes;
+    size_t want = fixed + (size_t)(cache == 2 ? 3 : (cache == 1 ? 2 : 0)) * row_bytes;
+    // mode 2, one GPU: the rest of shared memory caches the CTAs' row slabs of the first trailing
+    // columns for the whole panel (each column's GEMV would otherwise re-read them from L2)
+    int ncc = 0;
+    if (cache == 2 && !mg) {
+        static int ncc_cap = -1;
+        if (ncc_cap < 0) {
+            const char *e = getenv("FT_PANEL_NCC");  // experiment knob: cap on the cached columns
+            ncc_cap = e ? atoi(e) : 1 << 30;
+        }
+        ncc = (int)(((size_t)max_smem - want) / ((size_t)rmax * sizeof(double)));
+        ncc = std::min(ncc, std::min(ncc_cap, L.r[0].n - L.r[0].k - 2));
+        if (ncc < 0) ncc = 0;
+        want += (size_t)ncc * rmax * sizeof(double);
+    }
     // wide single-GPU launches: the two-reduction kernel (ft_panel_wide.cu), see its header
     if (L.nr == 1 && !mg && rmax >= 32 && !(L.r[0].dbg_mode & (8 | 64 | 128)) && !explicit_path)
         return ft_launch_panel_wide(L, nsm, s);
     PanelLaunch Lx = L;
     for (int i = 0; i < Lx.nr; i++) {
         Lx.r[i].wide = rmax >= 32 ? 1 : 0;
+        Lx.r[i].ncc = ncc;
         if (explicit_path) Lx.r[i].dbg_mode |= ((explicit_path & 0xff) ? 8 : 0) | (explicit_path >> 8);
     }
     const PanelLaunch *Lp = &Lx;
