@@ -91,6 +91,7 @@ struct PanelSmem {
     double bmX[RMAX];                   // b0 (or x) masked to the data rows >= c+2
     double2 red[PT];                    // GEMV partials  (y pairs)
     double2 rsr[PT];                    // GEMV partials  (row sums, verify pass)
+    unsigned long long drift;           // max fault-free |D_r| of the CTA's rows (reduced once per panel)
     // followed (dynamic part) by the CTA's rows of V, Y and Z when they fit: [R][VS] each
 };
 
@@ -568,6 +569,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
         cp_async_wait<0>();
     }
     if (tid == 0 && bid == 0) *p.bar_next = 0u;  // the next panel launch's counter
+    if (tid == 0) S.drift = 0ull;
     __syncthreads();
 
     double qc_corner = 0.0;  // corner of the Q checksums: sum of this panel's Qc (CTA 0, thread 0)
@@ -907,7 +909,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
                                 atomicAdd(&p.ctl->nflag, 1);
                             } else if (tau_abs > 0.0) {
                                 const double rel = fabs(d) / (tau_abs / c_thr);
-                                atomicMax(&p.ctl->drift_bits, (unsigned long long)__double_as_longlong(rel));
+                                atomicMax(&S.drift, (unsigned long long)__double_as_longlong(rel));  // smem: one global max per CTA
                             }
                         }
                     } else if (VC) {
@@ -947,6 +949,8 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
         PROBE(8);
     }
     __syncthreads();  // the helpers' last T column
+    __syncthreads();
+    if (tid == 0 && S.drift) atomicMax(&p.ctl->drift_bits, S.drift);
     // Q row checksums of the new Householder vectors (Fig. 5): own data rows
     if (p.abft)
         for (int rl = tid; rl < R; rl += PT) {

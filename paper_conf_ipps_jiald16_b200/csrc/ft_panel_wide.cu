@@ -70,6 +70,7 @@ struct PanelSmemW {
     double bm[RMAX];                    // masked b0 / x for the column dots
     double2 red[PT];                    // GEMV partials  (y pairs)
     double2 rsr[PT];                    // GEMV partials  (row sums, verify pass)
+    unsigned long long drift;           // max fault-free |D_r| of the CTA's rows (reduced once per panel)
     // followed (dynamic part) by the CTA's rows of V and Y when they fit: [R][VS] each
 };
 
@@ -288,6 +289,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel_wide(const __grid_constant__ Pa
         S.acol[rl] = is_valid(row) ? Apan[row + (int64_t)k * ldw] : 0.0;
     }
     if (tid == 0 && bid == 0) *p.bar_next = 0u;  // the next panel launch's counter
+    if (tid == 0) S.drift = 0ull;
     __syncthreads();
 
     unsigned epoch = 0;
@@ -676,7 +678,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel_wide(const __grid_constant__ Pa
                                 atomicAdd(&p.ctl->nflag, 1);
                             } else if (tau_abs > 0.0) {
                                 const double rel = fabs(d) / (tau_abs / c_thr);
-                                atomicMax(&p.ctl->drift_bits, (unsigned long long)__double_as_longlong(rel));
+                                atomicMax(&S.drift, (unsigned long long)__double_as_longlong(rel));  // smem: one global max per CTA
                             }
                         }
                     }
@@ -690,6 +692,8 @@ __global__ void __launch_bounds__(PT, 1) k_panel_wide(const __grid_constant__ Pa
         }
         PROBE(8);
     }
+    __syncthreads();
+    if (tid == 0 && S.drift) atomicMax(&p.ctl->drift_bits, S.drift);
     // Q row checksums of the new Householder vectors (Fig. 5): own data rows
     if (p.abft)
         for (int rl = tid; rl < R; rl += PT) {
