@@ -115,25 +115,25 @@ __device__ int pre_update_reason(const GemmRightParams &p) {
 template <int KT>
 __global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
     if (p.ctl && p.ctl->halt) return;
-    if (p.pre_ctl) {
-        __shared__ int s_reason;
-        if (threadIdx.x < 32) {
-            const int reason = pre_update_reason(p);
-            if (threadIdx.x == 0) s_reason = reason;
-        }
-        __syncthreads();
-        if (s_reason) {
-            if (threadIdx.x == 0 && blockIdx.x == 0 && blockIdx.y == 0) {
-                FtCtl *ctl = p.pre_ctl;
-                ctl->halt_panel = p.pre_panel;
-                ctl->halt_stage = 1;
-                ctl->halt_reason = s_reason;
-                __threadfence();
-                ctl->halt = 1;
-            }
-            return;  // nothing consumed: the panel is redone from its checkpoint
-        }
+    // fused pre-update check: warp 0 evaluates it while the other warps start the operand and
+    // C-tile loads; the decision is read at the first tile's barrier, before any store
+    __shared__ int s_reason;
+    if (p.pre_ctl && threadIdx.x < 32) {
+        const int reason = pre_update_reason(p);
+        if (threadIdx.x == 0) s_reason = reason;
     }
+    auto pre_abort = [&]() -> bool {  // after a __syncthreads that follows the evaluation
+        if (!p.pre_ctl || !s_reason) return false;
+        if (threadIdx.x == 0 && blockIdx.x == 0 && blockIdx.y == 0) {
+            FtCtl *ctl = p.pre_ctl;
+            ctl->halt_panel = p.pre_panel;
+            ctl->halt_stage = 1;
+            ctl->halt_reason = s_reason;
+            __threadfence();
+            ctl->halt = 1;
+        }
+        return true;  // nothing consumed: the panel is redone from its checkpoint
+    };
     extern __shared__ __align__(16) unsigned char smem_raw[];
     RightSmemT<KT> &S = *reinterpret_cast<RightSmemT<KT> *>(smem_raw);
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -200,6 +200,7 @@ __global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
         if (tt + 1 < t1) load_c(tt + 1, cn);
         cp_async_wait<1>();
         __syncthreads();
+        if (tt == t0 && pre_abort()) return;
         if (p.do_right) {
 #pragma unroll 4
             for (int k0 = 0; k0 < KT; k0 += 4) {
@@ -254,6 +255,10 @@ __global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
         cp_async_commit();
     }
     cp_async_wait<0>();
+    if (t0 >= t1) {  // no tile: take the pre-update decision here (no strip counter on a halt)
+        __syncthreads();
+        if (pre_abort()) return;
+    }
     if (do_w) {
         // deterministic partial of this row split: Wpart[split][col][j]
         double *Wp = p.Wpart + (int64_t)blockIdx.y * p.wsplit_stride;
