@@ -287,35 +287,53 @@ __global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
                     cp_async8(&Ts[a][b], ok ? p.T + a + b * FT_NBMAX : p.T, ok ? 8 : 0);
                 }
                 cp_async_commit();
-                for (int i = tid; i < UB * KT; i += UT) {
-                    const int cc = i / KT, b = i % KT;
-                    double w = 0.0;
-                    if (cc < ncols && b < K)
-                        w = sum_strided(p.Wpart + (int64_t)(cb + cc) * FT_NBMAX + b, p.wsplit_stride, (int)gridDim.y);
-                    Ws[cc][b] = w;
+                // W = sum of the row-split partials (fixed order), all of this thread's elements
+                // at once: their loads are in flight together (one round trip per 16)
+                constexpr int NE = UB * KT / UT;  // elements per thread
+                const int ns = (int)gridDim.y;
+                double wv[NE];
+#pragma unroll
+                for (int m = 0; m < NE; m++) wv[m] = 0.0;
+#pragma unroll 1
+                for (int sp = 0; sp < ns; sp += 2) {
+                    double v0[NE], v1[NE];
+#pragma unroll
+                    for (int m = 0; m < NE; m++) {
+                        const int i = tid + m * UT, cc = i / KT, bb = i % KT;
+                        const bool ok = cc < ncols && bb < K;
+                        const double *src = p.Wpart + (int64_t)(cb + cc) * FT_NBMAX + bb + (int64_t)sp * p.wsplit_stride;
+                        v0[m] = ok ? __ldcg(src) : 0.0;
+                        v1[m] = (ok && sp + 1 < ns) ? __ldcg(src + p.wsplit_stride) : 0.0;
+                    }
+#pragma unroll
+                    for (int m = 0; m < NE; m++) wv[m] += v0[m] + v1[m];
+                }
+#pragma unroll
+                for (int m = 0; m < NE; m++) {
+                    const int i = tid + m * UT;
+                    Ws[i / KT][i % KT] = wv[m];
                 }
                 cp_async_wait<0>();
                 __syncthreads();
-                for (int i = tid; i < UB * KT; i += UT) {
-                    const int cc = i / KT, a = i % KT;
-                    if (cc >= ncols || a >= K) continue;
-                    double s0 = 0.0, s1 = 0.0;
-                    if (p.transT) {  // W'(a) = sum_{b <= a} T(b, a) W(b)
-                        int b = 0;
-                        for (; b + 1 <= a; b += 2) {
-                            s0 += Ts[b][a] * Ws[cc][b];
-                            s1 += Ts[b + 1][a] * Ws[cc][b + 1];
-                        }
-                        if (b <= a) s0 += Ts[b][a] * Ws[cc][b];
-                    } else {  // W'(a) = sum_{b >= a} T(a, b) W(b)
-                        int b = a;
-                        for (; b + 1 < K; b += 2) {
-                            s0 += Ts[a][b] * Ws[cc][b];
-                            s1 += Ts[a][b + 1] * Ws[cc][b + 1];
-                        }
-                        if (b < K) s0 += Ts[a][b] * Ws[cc][b];
+                // W' = op(T) W: this thread's NE outputs as independent chains (one pass over b)
+                double so[NE];
+#pragma unroll
+                for (int m = 0; m < NE; m++) so[m] = 0.0;
+#pragma unroll 2
+                for (int bb = 0; bb < K; bb++) {
+#pragma unroll
+                    for (int m = 0; m < NE; m++) {
+                        const int i = tid + m * UT, cc = i / KT, a = i % KT;
+                        // transT: W'(a) = sum_{b <= a} T(b, a) W(b); else sum_{b >= a} T(a, b) W(b)
+                        const bool on = p.transT ? bb <= a : bb >= a;
+                        const double tv = p.transT ? Ts[bb][a] : Ts[a][bb];
+                        if (on) so[m] += tv * Ws[cc][bb];
                     }
-                    p.Wt[(int64_t)(cb + cc) * FT_NBMAX + a] = s0 + s1;
+                }
+#pragma unroll
+                for (int m = 0; m < NE; m++) {
+                    const int i = tid + m * UT, cc = i / KT, a = i % KT;
+                    if (cc < ncols && a < K) p.Wt[(int64_t)(cb + cc) * FT_NBMAX + a] = so[m];
                 }
                 if (tid == 0) p.strip_done[blockIdx.x] = 0;
             }
