@@ -733,13 +733,32 @@ __global__ void __launch_bounds__(YF_R * 64) k_ytop_finalize(YtopParams p) {
         Ts[a + b * FT_NBMAX] = p.T[a + b * FT_NBMAX];
     }
     double acc = 0.0;
-    if (row <= p.k && jb < ib)
-        acc = sum_strided(p.ypart + (int64_t)row * FT_NBMAX + jb, (int64_t)(p.k + 1) * FT_NBMAX, p.nsplit);
+    if (row <= p.k && jb < ib) {
+        // the split partials, 16 loads in flight at a time (fixed summation order)
+        const double *src = p.ypart + (int64_t)row * FT_NBMAX + jb;
+        const int64_t st = (int64_t)(p.k + 1) * FT_NBMAX;
+        for (int s0 = 0; s0 < p.nsplit; s0 += 16) {
+            double v[16];
+#pragma unroll
+            for (int u = 0; u < 16; u++) v[u] = s0 + u < p.nsplit ? __ldcg(src + (int64_t)(s0 + u) * st) : 0.0;
+#pragma unroll
+            for (int u = 0; u < 16; u++) acc += v[u];
+        }
+    }
     y0[rl][jb] = acc;
     __syncthreads();
     double yv = 0.0;
     if (row <= p.k && jb < ib) {
-        for (int b = 0; b <= jb; b++) yv += y0[rl][b] * Ts[b + jb * FT_NBMAX];
+        double y1 = 0.0, y2 = 0.0, y3 = 0.0;  // four independent chains
+        int b = 0;
+        for (; b + 3 <= jb; b += 4) {
+            yv += y0[rl][b] * Ts[b + jb * FT_NBMAX];
+            y1 += y0[rl][b + 1] * Ts[b + 1 + jb * FT_NBMAX];
+            y2 += y0[rl][b + 2] * Ts[b + 2 + jb * FT_NBMAX];
+            y3 += y0[rl][b + 3] * Ts[b + 3 + jb * FT_NBMAX];
+        }
+        for (; b <= jb; b++) yv += y0[rl][b] * Ts[b + jb * FT_NBMAX];
+        yv = (yv + y1) + (y2 + y3);
         p.Y[row + (int64_t)jb * p.ldw] = yv;
     }
     if (p.verify && row <= p.k && jb == 0) {
