@@ -339,6 +339,40 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
     auto coldot_add = [&](const double *zA, int JA, const double *zB, int JB, double *acc, int oA, int oB,
                           int oE) {
         const int NO = JA + JB + 2;
+        if (R <= 32) {
+            // small row blocks: one worker lane per output, a plain loop over the rows (two
+            // chains), no shuffles
+            if (helper) return;
+            for (int o = wtid; o < NO; o += wkt) {
+                const bool ua = o < JA;
+                const double *zr = ua ? zA : zB;
+                const int col = ua ? o : o - JA;
+                const int kind = o < JA + JB ? 0 : (o == JA + JB ? 1 : 2);
+                double s0 = 0.0, s1 = 0.0;
+                if (kind == 0) {
+                    const double *vc = Vl + col * XC;
+                    int rl = 0;
+#pragma unroll 4
+                    for (; rl + 1 < R; rl += 2) {
+                        s0 += vc[rl * XR] * zr[rl];
+                        s1 += vc[(rl + 1) * XR] * zr[rl + 1];
+                    }
+                    if (rl < R) s0 += vc[rl * XR] * zr[rl];
+                } else {
+#pragma unroll 4
+                    for (int rl = 0; rl < R; rl++) {
+                        const double z = zr[rl];
+                        if (kind == 1) s0 += z * z;
+                        else s0 += z;
+                    }
+                }
+                if (!(p.dbg_mode & 4)) {
+                    const int dst = o < JA ? oA + o : (o < JA + JB ? oB + o - JA : oE + (o - JA - JB));
+                    atomicAdd(acc + dst * FT_ACC_PAD, s0 + s1);
+                }
+            }
+            return;
+        }
         int LPO = 4;
         while (LPO < 32 && 2 * LPO < R && (2 * LPO) * NO <= wkt) LPO *= 2;
         if (helper) return;
@@ -576,7 +610,8 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
     const double c_thr = p.ctl->c_thr;
     const double tau_abs = c_thr * (double)n * 2.220446049250313e-16 * p.ctl->normF;
     // lanes per row in the combine: a whole warp per row for small row blocks
-    const int lpr = 8;  // 8 lanes per row: 3 shuffle rounds (a round costs ~4 dependent FMAs)
+    // lanes per row in the combine (8: 3 shuffle rounds; measured faster than 1 or 32)
+    const int lpr = 8;
     const int gl = wtid & (lpr - 1), grp = wtid / lpr, ngrp = wkt / lpr;
     auto gsum = [&](double v) {  // sum over the lpr lanes of a row group
 #pragma unroll
