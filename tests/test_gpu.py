@@ -114,6 +114,16 @@ def test_parity_explicit_path(n, nb, abft, bits):
     assert np.abs(H0 - H1).max() <= 1e-11 * np.abs(H1).max()
 
 
+def test_parity_unfused_ytop():
+    """n = 2600 (> 2560): Y_top by its own GEMM kernels, the M-part by the right update, every
+    panel launch still narrow (the one-reduction kernel) -- the full oracle bar."""
+    n = 2600
+    A = synth.matrix(n)
+    dA, tau, res = gpu_reduce(A, nb=32)
+    assert res.info == 0 and res.report.detected == 0
+    check_against_oracle(A, dA, tau, nb=32)
+
+
 def test_parity_c2_full_size():
     """BASELINE config C2 (n = 2048, nb = 32), the bench workload, full element-wise parity."""
     n = 2048
