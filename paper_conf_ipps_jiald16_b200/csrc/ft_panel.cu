@@ -55,7 +55,7 @@
 #define NWK (NW - NW / 4 + 1)  // worker warps
 #define WKT (32 * NWK)         // worker threads
 #define GR 8          // row-group granularity (64 bytes of a column)
-#define VS 65         // shared-memory row stride of the V / Y row caches (doubles)
+#define VS 68         // row stride of the V / Y / Z row caches (doubles; = 4 mod 16: the combine's 8-lane row groups hit distinct banks)
 #define RMAX PT       // max rows per CTA
 #define NSLOT (PT / 8)  // 8-lane groups per CTA (rows / outputs handled at once)
 #ifndef GB
@@ -307,6 +307,9 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
     }
     const int ncl = (ngw * 32) / R2p;
     const int npart = R2p <= 32 ? ngw : ncl;  // partials per row pair
+    // stride of the partials in S.red / S.rsr: R2p + 1 (odd) when a warp's R2p lanes write one
+    // partial each, so the combine's 8 lanes of a row read 8 partials from distinct banks
+    const int RSt = R2p <= 32 ? R2p + 1 : R2p;
 
     auto is_data = [&](int row) { return row >= k + 1 && row < ihi; };
     // fused Y_top: the rows 0..k above the panel take part in the GEMV, Y, Z and b0 (their b0 is
@@ -536,12 +539,12 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
                     }
                 }
             if (lane < R2p) {
-                S.red[gidx * R2p + lane] = ya;
-                if (vfy) S.rsr[gidx * R2p + lane] = rs;
+                S.red[gidx * RSt + lane] = ya;
+                if (vfy) S.rsr[gidx * RSt + lane] = rs;
             }
         } else if (cl < ncl) {
-            S.red[cl * R2p + rp] = ya;
-            if (vfy) S.rsr[cl * R2p + rp] = rs;
+            S.red[cl * RSt + rp] = ya;
+            if (vfy) S.rsr[cl * RSt + rp] = rs;
         }
     };
 
@@ -807,7 +810,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
                 const int row = r0 + rl, pr = rl >> 1, hi = rl & 1;
                 double ys = 0.0;
                 for (int q = 0; q < npart; q++) {
-                    const double2 u = S.red[q * R2p + pr];
+                    const double2 u = S.red[q * RSt + pr];
                     ys += hi ? u.y : u.x;
                 }
                 const double ap = (have_an && is_valid(row)) ? A[row + (int64_t)l0 * ldw] : 0.0;
@@ -858,10 +861,10 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
                     }
                 } else if (on) {
                     for (int qq = gl; qq < npart; qq += lpr) {
-                        const double2 w2 = S.red[qq * R2p + pr];
+                        const double2 w2 = S.red[qq * RSt + pr];
                         gp += hi ? w2.y : w2.x;
                         if (vfy) {
-                            const double2 r2 = S.rsr[qq * R2p + pr];
+                            const double2 r2 = S.rsr[qq * RSt + pr];
                             rsum += hi ? r2.y : r2.x;
                         }
                     }
