@@ -190,6 +190,11 @@ void ft_debug_probe_panel(int panel, unsigned long long *dbuf);
  * panel's smaller shared-memory modes (V, Z rows cached, Y global / all global); 0 restores
  * the default.  Results agree with the default up to rounding (tests of those paths). */
 void ft_debug_panel_path(int bits);
+/* ft_debug_left_fold(0) makes the ABFT left update carry the checksum row c and column r as
+ * an extra DMMA tile row / column strip (the round-1 layout) instead of folding them into
+ * the CTAs of the last tile row / strip (1, the default).  Results agree
+ * up to rounding; CUDA-graph replay is off while 0. */
+void ft_debug_left_fold(int on);
 
 #ifdef __cplusplus
 }

@@ -26,6 +26,8 @@ static int g_dbg_mode = 0;
 extern "C" void ft_debug_ablate(int mode) { g_dbg_mode = mode; }
 static int g_panel_path = 0;  // OR'ed into every panel launch's mode bits (8: explicit path, 64/128: smem modes 1/0)
 extern "C" void ft_debug_panel_path(int bits) { g_panel_path = bits & (8 | 64 | 128); }
+static int g_left_fold = 1;  // ABFT left update: checksum row/column folded (1) or as DMMA tiles (0)
+extern "C" void ft_debug_left_fold(int on) { g_left_fold = on ? 1 : 0; }
 extern "C" void ft_debug_probe_panel(int panel, unsigned long long *dbuf) {
     g_dbg_panel = panel;
     g_dbg_buf = dbuf;
@@ -578,6 +580,7 @@ int left_update(Call &C, int t, double sign, int nsplit, int endcheck = 0, bool 
     g.Fr = w.Fr;
     g.ectl = w.ctl;
     g.pre_reset = pre_reset ? w.ctl : nullptr;
+    g.fold = C.abft ? g_left_fold : 0;
     CK(ft_launch_gemm_left(g, C.s));
     return 0;
 }
@@ -901,7 +904,7 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
     // every iteration), captured on the second call with the same shape and buffers; the halt
     // protocol is unchanged (a halted graph's remaining kernels are no-ops, recovery follows).
     const bool graphable = C.faults.empty() && o.stop_after_panel < 0 && g_dbg_panel < 0 && !g_time_panels &&
-                           !g_panel_path &&
+                           !g_panel_path && g_left_fold &&
                            !getenv("FT_NO_GRAPH");
     bool launched = false;
     if (graphable) {

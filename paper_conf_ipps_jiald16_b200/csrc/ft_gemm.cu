@@ -390,6 +390,8 @@ template <int KT>
 struct LeftSmemT {
     double Wc[KT][SK];     // W' = op(T) W as [k][col]  (A operand, W'^T)
     double Vr[2][KT][SK];  // V(rows, k) as [k][row]    (B operand), double-buffered
+    double Wr[KT];         // fold: W'(:, n), the r column's coefficients
+    double Vn[KT];         // fold: V(n, :) = V_chk
 };
 
 // W'(col, a) = sum_b op(T)(a, b) W(b, col), W = sum over the row-split partials (fixed
@@ -433,6 +435,27 @@ __global__ void k_wprep(const double *__restrict__ Wpart, int64_t wstride, int n
 template <int KT>
 __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
     if (p.ctl && p.ctl->halt) return;
+    if (blockIdx.y >= p.ny) {
+        // frozen row sums of the panel columns k..e-1 (final now, untouched by this launch; R6):
+        // Fr(i) += sum_{col in [max(k, i-1), e)} A(i, col) for i <= e -- one row per thread in
+        // extra CTA rows of the grid, so the tile CTAs (few at late panels) carry no serial tail
+        const int k = p.r_lo - 1, e = p.c_lo, rows = min(e + 1, p.n);
+        const int i = ((blockIdx.y - p.ny) * gridDim.x + blockIdx.x) * UT + threadIdx.x;
+        if (i >= rows) return;
+        const double *a = p.A + i;
+        double s0 = 0.0, s1 = 0.0, s2 = 0.0, s3 = 0.0;
+        int c = max(k, i - 1);
+#pragma unroll 4
+        for (; c + 4 <= e; c += 4) {
+            s0 += __ldcg(a + (int64_t)c * p.lda);
+            s1 += __ldcg(a + (int64_t)(c + 1) * p.lda);
+            s2 += __ldcg(a + (int64_t)(c + 2) * p.lda);
+            s3 += __ldcg(a + (int64_t)(c + 3) * p.lda);
+        }
+        for (; c < e; c++) s0 += __ldcg(a + (int64_t)c * p.lda);
+        p.Fr[i] += (s0 + s1) + (s2 + s3);
+        return;
+    }
     extern __shared__ __align__(16) unsigned char smem_raw[];
     LeftSmemT<KT> &S = *reinterpret_cast<LeftSmemT<KT> *>(smem_raw);
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -444,8 +467,8 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
     const double sg = p.sign;
     const int rbase = (p.r_lo / UB) * UB;
     const int nrt = (p.r_hi - rbase + UB - 1) / UB;
-    const int t0 = (int)((long long)blockIdx.y * nrt / gridDim.y);
-    const int t1 = (int)((long long)(blockIdx.y + 1) * nrt / gridDim.y);
+    const int t0 = (int)((long long)blockIdx.y * nrt / p.ny);
+    const int t1 = (int)((long long)(blockIdx.y + 1) * nrt / p.ny);
     if (p.pre_reset && blockIdx.x == 0 && blockIdx.y == 0) {  // the right update has read them
         for (int j = tid; j < FT_NBMAX; j += UT) {
             p.pre_reset->eY[j] = 0.0;
@@ -462,6 +485,11 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
     }
     if (t0 < t1) issue_ktile<KT>(S.Vr[0], p.V, p.ldw, rbase + t0 * UB, p.r_hi, K);
     cp_async_commit();
+    // fold (ABFT): column n (r) rides with the last strip, row n (c) with the last row tile
+    if (p.fold && tid < KT) {
+        S.Wr[tid] = tid < K ? p.Wpart[(int64_t)p.n * FT_NBMAX + tid] : 0.0;
+        S.Vn[tid] = tid < K ? p.V[p.n + (int64_t)tid * p.ldw] : 0.0;
+    }
     int cols[2];
     bool colok[2];
     double *colp[2];
@@ -474,10 +502,19 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
     // fused end check: this CTA's share of sum r and sum c -- the entries it writes (column n:
     // r(k+1:n), row n: c(e:n)) in the tile epilogues, and a grid-strided slice of the entries
     // this launch does not touch (r(0:k+1), c(0:e), final since the right update / panel)
+    // With the fold only the CTAs that write r or c (last strip, last tile row) take part:
+    // the other CTAs skip the tail, so the serialised same-address atomics of the last-CTA
+    // protocol scale with gx + gy instead of gx * gy (one CTA per tile at large n)
     double es_r = 0.0, es_c = 0.0;
     const int en = p.n;
-    if (p.endcheck) {
-        const int nb = gridDim.x * gridDim.y, b = blockIdx.y * gridDim.x + blockIdx.x;
+    const bool fold_col = p.fold && blockIdx.x == gridDim.x - 1;
+    const bool fold_row = p.fold && (int)blockIdx.y == p.ny - 1;
+    const bool part = !p.fold || fold_col || fold_row;
+    const int pidx = !p.fold ? (int)(blockIdx.y * gridDim.x + blockIdx.x)
+                             : (fold_col ? (int)blockIdx.y : p.ny + (int)blockIdx.x);
+    const int pcnt = !p.fold ? (int)gridDim.x * p.ny : (int)gridDim.x + p.ny - 1;
+    if (p.endcheck && part) {
+        const int nb = pcnt, b = pidx;
         const int nr = p.r_lo, ncc = p.c_lo;  // r(0:k+1), c(0:e)
         for (int x = b * UT + tid; x < nr + ncc; x += nb * UT) {
             if (x < nr) es_r += __ldcg(p.A + x + (int64_t)en * p.lda);
@@ -536,23 +573,58 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
                     }
                 }
             }
+        if (fold_col) {  // r(rows) += sg V(rows, :) W'(:, n): 4 lanes per row, two chains each
+            const int rr = tid >> 2, q4 = tid & 3;
+            double s0 = 0.0, s1 = 0.0;
+#pragma unroll
+            for (int kk = q4; kk < KT; kk += 8) {
+                s0 += S.Vr[st][kk][rr] * S.Wr[kk];
+                s1 += S.Vr[st][kk + 4][rr] * S.Wr[kk + 4];
+            }
+            s0 += s1;
+            s0 += __shfl_xor_sync(0xffffffffu, s0, 1);
+            s0 += __shfl_xor_sync(0xffffffffu, s0, 2);
+            const int row = r + rr;
+            if (q4 == 0 && row >= lo && row < hi) {
+                double *pr = p.A + row + (int64_t)p.n * p.lda;
+                const double v = *pr + sg * s0;
+                *pr = v;
+                es_r += v;
+            }
+        }
         __syncthreads();  // Vr[st] is refilled two tiles later
     }
     cp_async_wait<0>();
-    if (p.endcheck) {  // (after the tiles: off the C-load critical path)
-        // frozen row sums of the panel columns k..e-1 (final now, untouched by this kernel; R6):
-        // Fr(i) += sum_{col in [k,e), i <= col+1} A(i, col) for i <= e
-        // one (row, 8-column chunk) per thread: a single round trip, partial sums by atomics
-        const int k = p.r_lo - 1, e = p.c_lo;
-        const int nch = (e - k + 7) / 8, rows = min(e + 1, p.n);
-        const int nb = gridDim.x * gridDim.y, b = blockIdx.y * gridDim.x + blockIdx.x;
-        for (int x = b * UT + tid; x < rows * nch; x += nb * UT) {
-            const int i = x % rows, q = x / rows;
-            const int c0 = max(i - 1 > k ? i - 1 : k, k + 8 * q), c1 = min(e, k + 8 * q + 8);
-            if (c0 < c1) atomicAdd(p.Fr + i, sum_strided(p.A + i + (int64_t)c0 * p.lda, p.lda, c1 - c0));
+    if (fold_row) {  // c(cols) += sg V(n, :) W'(:, cols), and kappa with the last strip
+        __syncthreads();  // Wc landed (cp.async) for every thread
+        const int cc = tid >> 2, q4 = tid & 3;
+        double s0 = 0.0, s1 = 0.0, k0 = 0.0, k1 = 0.0;
+#pragma unroll
+        for (int kk = q4; kk < KT; kk += 8) {
+            s0 += S.Vn[kk] * S.Wc[kk][cc];
+            s1 += S.Vn[kk + 4] * S.Wc[kk + 4][cc];
+            k0 += S.Vn[kk] * S.Wr[kk];
+            k1 += S.Vn[kk + 4] * S.Wr[kk + 4];
+        }
+        s0 += s1;
+        s0 += __shfl_xor_sync(0xffffffffu, s0, 1);
+        s0 += __shfl_xor_sync(0xffffffffu, s0, 2);
+        k0 += k1;
+        k0 += __shfl_xor_sync(0xffffffffu, k0, 1);
+        k0 += __shfl_xor_sync(0xffffffffu, k0, 2);
+        if (q4 == 0 && cc < ncols) {
+            double *pc = p.A + p.n + (int64_t)(cb + cc) * p.lda;
+            const double v = *pc + sg * s0;
+            *pc = v;
+            es_c += v;
+        }
+        if (fold_col && tid == 0) {
+            double *pk = p.A + p.n + (int64_t)p.n * p.lda;
+            *pk = *pk + sg * k0;
         }
     }
-    if (!p.endcheck) return;
+    if (p.fold && part) __threadfence();  // the fold's stores precede this CTA's done_left increment
+    if (!p.endcheck || !part) return;
     // fused end-of-iteration check (Alg. 3 l.12-13; R11/R22): the CTA's partial sums go into
     // ctl->sums[2:4]; once every CTA has finished, the last one compares sum r and sum c with
     // kappa (EAGER) or with each other (PAPER)
@@ -574,7 +646,7 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
         atomicAdd(&p.ectl->sums[2], a);
         atomicAdd(&p.ectl->sums[3], b);
         __threadfence();
-        last = atomicAdd(&p.ectl->done_left, 1) == (int)(gridDim.x * gridDim.y) - 1;
+        last = atomicAdd(&p.ectl->done_left, 1) == pcnt - 1;
     }
     __syncthreads();
     if (!last || tid != 0) return;
@@ -611,14 +683,19 @@ static cudaError_t launch_left_kt(const GemmLeftParams &p, cudaStream_t s) {
         if (e != cudaSuccess) return e;
         attr = true;
     }
-    const int nstrip = (p.c_hi - p.c_lo + UB - 1) / UB;
+    // fold: tiles cover rows [r_lo, r_hi-1) and columns [c_lo, c_hi-1); the checksum row and
+    // column (index n) are folded into the last tile row / strip
+    const bool fold = p.fold && p.r_hi - 1 == p.n && p.c_hi - 1 == p.n && p.r_hi - 1 > p.r_lo &&
+                      p.c_hi - 1 > p.c_lo && p.wt_ready;
+    const int r_hi = fold ? p.r_hi - 1 : p.r_hi, c_hi = fold ? p.c_hi - 1 : p.c_hi;
+    const int nstrip = (c_hi - p.c_lo + UB - 1) / UB;
     static int nsm = 0;
     if (!nsm) {
         int dev = 0;
         cudaGetDevice(&dev);
         cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
     }
-    const int nrt = (p.r_hi - (p.r_lo / UB) * UB + UB - 1) / UB;
+    const int nrt = (r_hi - (p.r_lo / UB) * UB + UB - 1) / UB;
     const int ny = best_splits(nstrip, nrt, nsm, 1 << 20, 2);  // two resident CTAs per SM
     if (!p.wt_ready) {
         g_ft_launches++;
@@ -630,7 +707,16 @@ static cudaError_t launch_left_kt(const GemmLeftParams &p, cudaStream_t s) {
     g_ft_launches++;
     GemmLeftParams q = p;
     q.Wpart = p.Wt;  // the main kernel reads W' = op(T) W
-    k_gemm_left<KT><<<dim3(nstrip, ny), UT, smem, s>>>(q);
+    q.fold = fold ? 1 : 0;
+    q.r_hi = r_hi;
+    q.c_hi = c_hi;
+    q.ny = ny;
+    int nyf = 0;  // extra CTA rows for the frozen row sums (one row of A per thread)
+    if (p.endcheck) {
+        const int rows = std::min(p.c_lo + 1, p.n);
+        nyf = ((rows + UT - 1) / UT + nstrip - 1) / nstrip;
+    }
+    k_gemm_left<KT><<<dim3(nstrip, ny + nyf), UT, smem, s>>>(q);
     return cudaGetLastError();
 }
 cudaError_t ft_launch_gemm_left(const GemmLeftParams &p, cudaStream_t s) {

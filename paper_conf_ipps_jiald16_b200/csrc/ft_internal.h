@@ -147,6 +147,12 @@ struct GemmLeftParams {
     double *Fr;
     FtCtl *ectl;
     FtCtl *pre_reset;  // non-NULL: CTA (0,0) clears the fused pre-update sums for the next panel
+    // 1: row r_hi-1 and column c_hi-1 are the checksum row c and column r (= n, ABFT); they are
+    // updated by CUDA-core dot products in the CTAs owning the last row tile / column strip
+    // instead of as an extra 64-row tile and 64-column strip of DMMA work (n % 64 == 0 would
+    // otherwise add a whole strip and tile row for one column / one row)
+    int fold;
+    int ny;  // set by the launcher: CTA rows that own tiles (rows >= ny form the frozen row sums)
 };
 cudaError_t ft_launch_gemm_left(const GemmLeftParams &p, cudaStream_t s);
 

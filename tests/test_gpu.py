@@ -249,7 +249,7 @@ def test_host_entry_with_fault():
 
 
 # ------------------------------------------------------------------ checksum parity (Theorem 1)
-@pytest.mark.parametrize("n,nb", [(64, 16), (300, 32), (513, 64)])
+@pytest.mark.parametrize("n,nb", [(64, 16), (300, 32), (513, 64), (256, 64), (320, 32)])
 def test_checksums_at_every_boundary(n, nb):
     A = synth.matrix(n, dist="normal")
     normF = np.linalg.norm(A)
@@ -262,6 +262,32 @@ def test_checksums_at_every_boundary(n, nb):
         g = chk.cpu().numpy()
         assert np.abs(g - chko).max() <= 1e-10 * normF, (t, np.abs(g - chko).max())
         assert rel(dA.cpu().numpy(), Aw) <= TOL, t
+
+
+@pytest.mark.parametrize("n,nb", [(256, 64), (320, 32), (513, 64), (1024, 32)])
+def test_left_update_fold_matches_tiles(n, nb):
+    """The ABFT left update's checksum row/column folded into the last tile row / strip
+    (default) against the same row/column as extra DMMA tiles (ft_debug_left_fold(0)): H, tau
+    and the maintained checksums at a mid boundary agree to rounding; both meet the oracle."""
+    A = synth.matrix(n, dist="normal")
+    L = ft.lib()
+    L.ft_debug_left_fold.argtypes = [ctypes.c_int]
+    t = ((n - 2 + nb - 1) // nb) // 2
+    out = []
+    for fold in (1, 0):
+        L.ft_debug_left_fold(fold)
+        try:
+            chk = torch.zeros(2 * n + 1, dtype=torch.float64, device="cuda")
+            dAs, _, rs = gpu_reduce(A, nb=nb, stop_after_panel=t, dchk_out=chk)
+            dA, tau, res = gpu_reduce(A, nb=nb)
+        finally:
+            L.ft_debug_left_fold(1)
+        assert rs.info == 0 and res.info == 0 and res.report.detected == 0, res.events
+        check_against_oracle(A, dA, tau, nb=nb)
+        out.append((dA.cpu().numpy(), chk.cpu().numpy()))
+    (H1, c1), (H0, c0) = out
+    assert rel(np.triu(H1, -1), np.triu(H0, -1)) <= 1e-11  # panel atomics: rounding-level run-to-run
+    assert np.abs(c1 - c0).max() <= 1e-11 * np.linalg.norm(A)
 
 
 # ------------------------------------------------------------------ fault injection
