@@ -7,6 +7,8 @@
 // the column checksum c -- so Theorem 1 is carried by the same tiles.
 // Rollback (reverse computation, Alg. 3 l.14) is the same kernels with sign +1.
 //
+#include <cstdlib>
+
 #include "ft_common.cuh"
 #include "ft_internal.h"
 
@@ -27,13 +29,14 @@
 
 // Row splits per strip: minimise waves * tiles-per-CTA for per_sm resident CTAs per SM
 // (the grid is nstrip x ns CTAs; a ragged last wave idles SMs).
-static int best_splits(int nstrip, int nrt, int nsm, int cap, int per_sm) {
+// ovh: fixed per-CTA cost (prologue: operand strip load, pipeline fill) in quarter tiles
+static int best_splits(int nstrip, int nrt, int nsm, int cap, int per_sm, int ovh = 0) {
     const int slots = per_sm * nsm;
     int best = 1;
     long long best_cost = -1;
     for (int ns = 1; ns <= cap && ns <= nrt; ns++) {
         const long long waves = ((long long)nstrip * ns + slots - 1) / slots;
-        const long long cost = waves * ((nrt + ns - 1) / ns);
+        const long long cost = waves * (4 * ((nrt + ns - 1) / ns) + ovh);
         if (best_cost < 0 || cost < best_cost) {
             best_cost = cost;
             best = ns;
@@ -696,7 +699,10 @@ static cudaError_t launch_left_kt(const GemmLeftParams &p, cudaStream_t s) {
         cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
     }
     const int nrt = (r_hi - (p.r_lo / UB) * UB + UB - 1) / UB;
-    const int ny = best_splits(nstrip, nrt, nsm, 1 << 20, 2);  // two resident CTAs per SM
+    // per-CTA prologue of half a tile (W' strip + first V tile): measured best of 0 / 2 / 4 / 8 at
+    // n = 8192 / 16384 (profiles/r01/s8/left_ovh.txt); FT_LEFT_OVH overrides for sweeps
+    static const int ovh = getenv("FT_LEFT_OVH") ? atoi(getenv("FT_LEFT_OVH")) : 2;
+    const int ny = best_splits(nstrip, nrt, nsm, 1 << 20, 2, ovh);  // two resident CTAs per SM
     if (!p.wt_ready) {
         g_ft_launches++;
         const int per = UT / FT_NBMAX;  // columns per k_wprep block
