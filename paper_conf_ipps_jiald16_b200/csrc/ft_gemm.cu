@@ -48,7 +48,8 @@ int ft_gemm_splits(int r_lo, int r_hi, int c_lo, int c_hi, int nsm) {
     const int nstrip = (c_hi - c_lo + UB - 1) / UB;
     const int nrt = (r_hi - (r_lo / UB) * UB + UB - 1) / UB;
     // right update: one CTA per SM (the next C tile is prefetched in registers)
-    return best_splits(nstrip > 0 ? nstrip : 1, nrt > 0 ? nrt : 1, nsm, FT_WSPLIT_MAX, 1);
+    static const int ovh = getenv("FT_RIGHT_OVH") ? atoi(getenv("FT_RIGHT_OVH")) : 0;
+    return best_splits(nstrip > 0 ? nstrip : 1, nrt > 0 ? nrt : 1, nsm, FT_WSPLIT_MAX, 1, ovh);
 }
 
 template <int KT>
