@@ -447,17 +447,18 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
         const int i = ((blockIdx.y - p.ny) * gridDim.x + blockIdx.x) * UT + threadIdx.x;
         if (i >= rows) return;
         const double *a = p.A + i;
-        double s0 = 0.0, s1 = 0.0, s2 = 0.0, s3 = 0.0;
+        // all of a row's loads in flight together (<= 64 columns): 8 at a time into 8 chains
+        double s[8] = {0.0, 0.0, 0.0, 0.0, 0.0, 0.0, 0.0, 0.0};
         int c = max(k, i - 1);
-#pragma unroll 4
-        for (; c + 4 <= e; c += 4) {
-            s0 += __ldcg(a + (int64_t)c * p.lda);
-            s1 += __ldcg(a + (int64_t)(c + 1) * p.lda);
-            s2 += __ldcg(a + (int64_t)(c + 2) * p.lda);
-            s3 += __ldcg(a + (int64_t)(c + 3) * p.lda);
+#pragma unroll 8
+        for (; c + 8 <= e; c += 8) {
+#pragma unroll
+            for (int u = 0; u < 8; u++) s[u] += __ldcg(a + (int64_t)(c + u) * p.lda);
         }
-        for (; c < e; c++) s0 += __ldcg(a + (int64_t)c * p.lda);
-        p.Fr[i] += (s0 + s1) + (s2 + s3);
+#pragma unroll
+        for (int u = 0; u < 7; u++)
+            if (c + u < e) s[u] += __ldcg(a + (int64_t)(c + u) * p.lda);
+        p.Fr[i] += ((s[0] + s[1]) + (s[2] + s[3])) + ((s[4] + s[5]) + (s[6] + s[7]));
         return;
     }
     extern __shared__ __align__(16) unsigned char smem_raw[];
