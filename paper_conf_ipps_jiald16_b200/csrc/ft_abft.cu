@@ -199,8 +199,8 @@ __global__ void k_precheck(const double *Y, const double *V, int64_t ldw, int ih
         sy = warp_sum(sy);
         sv = warp_sum(sv);
         if (lane == 0) {
-            atomicAdd(&ctl->eY[j], sy);
-            atomicAdd(&ctl->eV[j], sv);
+            atomicAdd(&ctl->eY[j * FT_ESTR], sy);
+            atomicAdd(&ctl->eV[j * FT_ESTR], sv);
         }
     }
 }
@@ -231,8 +231,8 @@ __global__ void k_decide(const double *Y, const double *V, const double *T, int6
     const double tauY = c_thr * unit * (tmax > 1.0 ? tmax : 1.0);
     const double tauV = c_thr * (double)n * EPS * sqrt((double)n);
     for (int j = lane; j < ib; j += 32) {
-        double dy = ctl->eY[j] - Y[n + (int64_t)j * ldw];
-        double dv = ctl->eV[j] - V[n + (int64_t)j * ldw];
+        double dy = ctl->eY[j * FT_ESTR] - Y[n + (int64_t)j * ldw];
+        double dv = ctl->eV[j * FT_ESTR] - V[n + (int64_t)j * ldw];
         if (not_within(dy, tauY)) reason |= 2;
         if (not_within(dv, tauV)) reason |= 4;
     }
@@ -250,8 +250,8 @@ __global__ void k_decide(const double *Y, const double *V, const double *T, int6
         ctl->nflag = 0;
     }
     for (int j = lane; j < FT_NBMAX; j += 32) {
-        ctl->eY[j] = 0.0;
-        ctl->eV[j] = 0.0;
+        ctl->eY[j * FT_ESTR] = 0.0;
+        ctl->eV[j * FT_ESTR] = 0.0;
     }
 }
 cudaError_t ft_decide(const double *Y, const double *V, const double *T, int64_t ldw, int n, int k, int ib,

@@ -680,7 +680,7 @@ int enqueue_panel(Call &C, int t) {
     if (inject_at(C, t, FT_PHASE_AFTER_PANEL)) return FT_E_CUDA;
     if (eager && !fuse_pre) {
         // a fault is scheduled after the panel: recompute the check sums after it
-        CK(cudaMemsetAsync(w.ctl->eY, 0, sizeof(double) * 2 * FT_NBMAX, C.s));
+        CK(cudaMemsetAsync(w.ctl->eY, 0, sizeof(double) * 2 * FT_NBMAX * FT_ESTR, C.s));
         CK(ft_precheck(w.Y, w.V, w.ldw, n, C.ihi, k, ib, w.ctl, C.s));
         CK(ft_decide(w.Y, w.V, w.T, w.ldw, n, k, ib, t, w.ctl, C.s));
     }
@@ -792,7 +792,7 @@ int recover(Call &C, const FtCtl &h) {
     int zero = 0;
     CK(cudaMemcpyAsync(&w.ctl->halt, &zero, sizeof(int), cudaMemcpyHostToDevice, C.s));
     CK(cudaMemcpyAsync(&w.ctl->nflag, &zero, sizeof(int), cudaMemcpyHostToDevice, C.s));
-    CK(cudaMemsetAsync(w.ctl->eY, 0, sizeof(double) * 128, C.s));
+    CK(cudaMemsetAsync(w.ctl->eY, 0, sizeof(double) * 2 * FT_NBMAX * FT_ESTR, C.s));
     CK(cudaMemsetAsync(w.ctl->sums, 0, sizeof(double) * 4, C.s));
     CK(cudaMemsetAsync(&w.ctl->done_count, 0, 3 * sizeof(int), C.s));  // done_count, done_ytop, done_left
     if (h.halt_stage == 2) {

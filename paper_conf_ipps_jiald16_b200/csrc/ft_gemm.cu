@@ -106,8 +106,8 @@ __device__ int pre_update_reason(const GemmRightParams &p) {
     const double tauV = ctl->c_thr * (double)n * eps * sqrt((double)n);
     int reason = __ldcg(&ctl->nflag) > 0 ? 1 : 0;
     for (int j = lane; j < ib; j += 32) {
-        const double dy = __ldcg(&ctl->eY[j]) - __ldcg(p.Y + n + (int64_t)j * p.ldw);
-        const double dv = __ldcg(&ctl->eV[j]) - __ldcg(p.V + n + (int64_t)j * p.ldw);
+        const double dy = __ldcg(&ctl->eY[j * FT_ESTR]) - __ldcg(p.Y + n + (int64_t)j * p.ldw);
+        const double dv = __ldcg(&ctl->eV[j * FT_ESTR]) - __ldcg(p.V + n + (int64_t)j * p.ldw);
         if (not_within(dy, tauY)) reason |= 2;
         if (not_within(dv, tauV)) reason |= 4;
     }
@@ -476,8 +476,8 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
     const int t1 = (int)((long long)(blockIdx.y + 1) * nrt / p.ny);
     if (p.pre_reset && blockIdx.x == 0 && blockIdx.y == 0) {  // the right update has read them
         for (int j = tid; j < FT_NBMAX; j += UT) {
-            p.pre_reset->eY[j] = 0.0;
-            p.pre_reset->eV[j] = 0.0;
+            p.pre_reset->eY[j * FT_ESTR] = 0.0;
+            p.pre_reset->eV[j * FT_ESTR] = 0.0;
         }
         if (tid == 0) p.pre_reset->nflag = 0;
     }
@@ -872,7 +872,7 @@ __global__ void __launch_bounds__(YF_R * 64) k_ytop_finalize(YtopParams p) {
     if (rl == 0 && jb < ib) {
         double s = 0.0;
         for (int q = 0; q < YF_R; q++) s += y0[q][jb];
-        atomicAdd(&p.ctl->eY[jb], s);
+        atomicAdd(&p.ctl->eY[jb * FT_ESTR], s);
     }
     // the decision itself is taken by every CTA of the right update (GemmRightParams::pre_ctl)
 }

@@ -12,6 +12,7 @@
 #ifndef FT_NBMAX
 #define FT_NBMAX 64
 #endif
+#define FT_ESTR 4  // doubles per pre-update check sum (FtCtl::eY / eV)
 #define FT_ACC_STRIDE (3 * 64 + 8)  // [s1 | sx | scalars | V^T x] per reduction set (ft_panel.cu ACC_*)
 #define FT_ACC_SETS 4               // sets indexed by the global column mod 4 (recycled in-kernel)
 #define FT_ACC_PAD 32               // doubles between accumulators: one 256-byte block (own L2 slice) each
@@ -30,8 +31,10 @@ struct FtCtl {
     double normF;         // ||A||_F of the input (invariant under the similarity)
     double c_thr;
     unsigned long long drift_bits;  // max fault-free |D| / (n eps ||A||_F) seen (as bits)
-    double eY[64];        // pre-update check sums (e^T Y)
-    double eV[64];        // (e^T V)
+    // pre-update check sums e^T Y, e^T V of column j at [j * FT_ESTR]: one 32-byte sector per
+    // column, so the per-CTA atomics of different columns do not serialise on shared sectors
+    double eY[64 * FT_ESTR];
+    double eV[64 * FT_ESTR];
     double sums[4];       // end check: sum r, sum c
     double tmax;          // max |T| of the last panel (written by the panel kernel; pre-update tolerance)
     double inj_delta[FT_MAXFAULTS];

@@ -1006,7 +1006,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
             for (int rl = lane; rl < R; rl += 32)
                 if (is_data(r0 + rl) || is_top(r0 + rl)) s += o < ib ? Yl[rl * YR + jj * YCS] : Vl[rl * XR + jj * XC];
             s = warp_sum(s);
-            if (lane == 0) atomicAdd(o < ib ? &p.ctl->eY[jj] : &p.ctl->eV[jj], s);
+            if (lane == 0) atomicAdd(o < ib ? &p.ctl->eY[jj * FT_ESTR] : &p.ctl->eV[jj * FT_ESTR], s);
         }
     if (bid == 0 && tid == 0 && p.abft) p.Qc[n] += qc_corner;
     if (bid == 0) {

@@ -710,7 +710,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel_wide(const __grid_constant__ Pa
         double s = 0.0;
         for (int rl = 0; rl < R; rl++)
             if (is_data(r0 + rl)) s += X[rl * XR + jj * XC];
-        atomicAdd(tid < ib ? &p.ctl->eY[jj] : &p.ctl->eV[jj], s);
+        atomicAdd(tid < ib ? &p.ctl->eY[jj * FT_ESTR] : &p.ctl->eV[jj * FT_ESTR], s);
     }
     if (bid == 0 && tid == 0 && p.abft) p.Qc[n] += qc_corner;
     if (bid == 0) {
