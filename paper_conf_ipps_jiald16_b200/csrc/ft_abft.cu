@@ -73,12 +73,14 @@ __global__ void __launch_bounds__(LS_RB) k_rowsum_part(const double *__restrict_
     if (i < n) {
         const double *a = Aw + i;
         if (mode < 0) {
+#pragma unroll 8
             for (int j = j0; j < j1; j++) {
                 const double x = a[(int64_t)j * ldw];
                 s += x;
                 q += x * x;
             }
         } else {
+#pragma unroll 8
             for (int j = j0; j < j1; j++) {
                 const bool v = in_v(i, j, ilo, ihi, cdone);
                 if (mode == 0 ? !v : v) s += a[(int64_t)j * ldw];
@@ -117,20 +119,27 @@ __global__ void k_encode_cols(double *Aw, int64_t ldw, int n) {
     if (lane == 0) Aw[n + (int64_t)j * ldw] = s;  // c(j) in row n
 }
 __global__ void k_encode_finish(double *Aw, int64_t ldw, int n, const double *sq_part, int nparts, FtCtl *ctl) {
-    // kappa = sum r (fixed order), ||A||_F
-    __shared__ double ws[32];
-    double s = 0.0;
+    // kappa = sum r, ||A||_F^2 = sum of the squares' partials (both in a fixed order: strided
+    // per thread, then warps, then thread 0 over the warps)
+    __shared__ double ws[32], wq[32];
+    double s = 0.0, q = 0.0;
     for (int i = threadIdx.x; i < n; i += blockDim.x) s += Aw[i + (int64_t)n * ldw];
+    for (int b = threadIdx.x; b < nparts; b += blockDim.x) q += sq_part[b];
     s = warp_sum(s);
-    if ((threadIdx.x & 31) == 0) ws[threadIdx.x >> 5] = s;
+    q = warp_sum(q);
+    if ((threadIdx.x & 31) == 0) {
+        ws[threadIdx.x >> 5] = s;
+        wq[threadIdx.x >> 5] = q;
+    }
     __syncthreads();
     if (threadIdx.x == 0) {
-        double k = 0.0;
-        for (int w = 0; w < (int)(blockDim.x >> 5); w++) k += ws[w];
+        double k = 0.0, qq = 0.0;
+        for (int w = 0; w < (int)(blockDim.x >> 5); w++) {
+            k += ws[w];
+            qq += wq[w];
+        }
         Aw[n + (int64_t)n * ldw] = k;
-        double q = 0.0;
-        for (int b = 0; b < nparts; b++) q += sq_part[b];
-        ctl->normF = sqrt(q);
+        ctl->normF = sqrt(qq);
     }
 }
 // frozen row sums before the first panel: columns 0..ilo-2 are final (R5/R6)
