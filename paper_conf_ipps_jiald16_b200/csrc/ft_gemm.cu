@@ -439,12 +439,13 @@ __global__ void k_wprep(const double *__restrict__ Wpart, int64_t wstride, int n
 template <int KT>
 __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
     if (p.ctl && p.ctl->halt) return;
-    if (blockIdx.y >= p.ny) {
+    if ((int)blockIdx.y < p.nyf) {
         // frozen row sums of the panel columns k..e-1 (final now, untouched by this launch; R6):
         // Fr(i) += sum_{col in [max(k, i-1), e)} A(i, col) for i <= e -- one row per thread in
-        // extra CTA rows of the grid, so the tile CTAs (few at late panels) carry no serial tail
+        // extra CTA rows of the grid, so the tile CTAs (few at late panels) carry no serial tail;
+        // they come first in the grid (scheduled first, off the launch's tail)
         const int k = p.r_lo - 1, e = p.c_lo, rows = min(e + 1, p.n);
-        const int i = ((blockIdx.y - p.ny) * gridDim.x + blockIdx.x) * UT + threadIdx.x;
+        const int i = (blockIdx.y * gridDim.x + blockIdx.x) * UT + threadIdx.x;
         if (i >= rows) return;
         const double *a = p.A + i;
         // all of a row's loads in flight together (<= 64 columns): 8 at a time into 8 chains
@@ -466,15 +467,18 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int lr = lane >> 2, lc = lane & 3;
     const int wc = warp & 3, wr = warp >> 2;
-    const int cb = p.c_lo + blockIdx.x * UB;
+    // strips and row splits in reverse grid order: the CTAs of the last strip and the last row
+    // split (the fold and the end-check tail) are scheduled first
+    const int bx = (int)gridDim.x - 1 - (int)blockIdx.x, by = p.ny - 1 - ((int)blockIdx.y - p.nyf);
+    const int cb = p.c_lo + bx * UB;
     const int ncols = min(UB, p.c_hi - cb);
     const int K = p.K;
     const double sg = p.sign;
     const int rbase = (p.r_lo / UB) * UB;
     const int nrt = (p.r_hi - rbase + UB - 1) / UB;
-    const int t0 = (int)((long long)blockIdx.y * nrt / p.ny);
-    const int t1 = (int)((long long)(blockIdx.y + 1) * nrt / p.ny);
-    if (p.pre_reset && blockIdx.x == 0 && blockIdx.y == 0) {  // the right update has read them
+    const int t0 = (int)((long long)by * nrt / p.ny);
+    const int t1 = (int)((long long)(by + 1) * nrt / p.ny);
+    if (p.pre_reset && bx == 0 && by == 0) {  // the right update has read them
         for (int j = tid; j < FT_NBMAX; j += UT) {
             p.pre_reset->eY[j * FT_ESTR] = 0.0;
             p.pre_reset->eV[j * FT_ESTR] = 0.0;
@@ -512,11 +516,10 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
     // protocol scale with gx + gy instead of gx * gy (one CTA per tile at large n)
     double es_r = 0.0, es_c = 0.0;
     const int en = p.n;
-    const bool fold_col = p.fold && blockIdx.x == gridDim.x - 1;
-    const bool fold_row = p.fold && (int)blockIdx.y == p.ny - 1;
+    const bool fold_col = p.fold && bx == (int)gridDim.x - 1;
+    const bool fold_row = p.fold && by == p.ny - 1;
     const bool part = !p.fold || fold_col || fold_row;
-    const int pidx = !p.fold ? (int)(blockIdx.y * gridDim.x + blockIdx.x)
-                             : (fold_col ? (int)blockIdx.y : p.ny + (int)blockIdx.x);
+    const int pidx = !p.fold ? by * (int)gridDim.x + bx : (fold_col ? by : p.ny + bx);
     const int pcnt = !p.fold ? (int)gridDim.x * p.ny : (int)gridDim.x + p.ny - 1;
     if (p.endcheck && part) {
         const int nb = pcnt, b = pidx;
@@ -724,6 +727,7 @@ static cudaError_t launch_left_kt(const GemmLeftParams &p, cudaStream_t s) {
         const int rows = std::min(p.c_lo + 1, p.n);
         nyf = ((rows + UT - 1) / UT + nstrip - 1) / nstrip;
     }
+    q.nyf = nyf;
     k_gemm_left<KT><<<dim3(nstrip, ny + nyf), UT, smem, s>>>(q);
     return cudaGetLastError();
 }

@@ -155,7 +155,7 @@ struct GemmLeftParams {
     // instead of as an extra 64-row tile and 64-column strip of DMMA work (n % 64 == 0 would
     // otherwise add a whole strip and tile row for one column / one row)
     int fold;
-    int ny;  // set by the launcher: CTA rows that own tiles (rows >= ny form the frozen row sums)
+    int ny, nyf;  // set by the launcher: CTA rows [0, nyf) form the frozen row sums, the next ny own tiles
 };
 cudaError_t ft_launch_gemm_left(const GemmLeftParams &p, cudaStream_t s);
 
