@@ -28,6 +28,18 @@
 #endif
 
 #define AT(A, lda, i, j) (A)[(size_t)(i) + (size_t)(j) * (size_t)(lda)]
+/* rows per block of the streamed row-wise sums (memory order only): one block per thread,
+ * a multiple of 8 rows, at most 4096 (the block's accumulators stay in L2) */
+static int row_block(int m) {
+    int nt = 1;
+#ifdef _OPENMP
+    nt = omp_get_max_threads();
+#endif
+    int rb = (m + nt - 1) / nt;
+    rb = (rb + 7) / 8 * 8;
+    if (rb > 4096) rb = 4096;
+    return rb < 8 ? 8 : rb;
+}
 static const double EPS = DBL_EPSILON; /* 2^-52, R17 */
 
 int ora_num_threads(void) {
@@ -119,12 +131,18 @@ static double reflector_step(int n, int ihi, double *A, int lda, int c,
         *chk->qk += ev - 1.0;
     }
 
-    /* Right step: A(0:ihi, c+1:ihi) := A (I - tau v v^T).  y = A v.  P:38 (A Q_i) */
+    /* Right step: A(0:ihi, c+1:ihi) := A (I - tau v v^T).  y = A v.  P:38 (A Q_i)
+     * y(i) = sum_j A(i,j) v(j), j increasing -- the loop nest runs j-outer over a block of
+     * rows so the column-major matrix streams; every y(i) sees the same additions in the
+     * same order as the plain dot (bitwise identical; -ffp-contract=off). */
 #pragma omp parallel for schedule(static)
-    for (int i = 0; i < ihi; i++) {
-        double s = 0.0;
-        for (int j = c + 1; j < ihi; j++) s += AT(A, lda, i, j) * V(j);
-        y[i] = s;
+    for (int i0 = 0; i0 < ihi; i0 += row_block(ihi)) {
+        const int rb = row_block(ihi), i1 = i0 + rb < ihi ? i0 + rb : ihi;
+        for (int i = i0; i < i1; i++) y[i] = 0.0;
+        for (int j = c + 1; j < ihi; j++) {
+            const double vj = V(j);
+            for (int i = i0; i < i1; i++) y[i] += AT(A, lda, i, j) * vj;
+        }
     }
     if (chk) {
         /* Theorem 1 part 2 at reflector granularity */
@@ -229,14 +247,22 @@ static int approx(double a, double b, double tol) {
 
 typedef struct { double *Dr, *Dc, sr, sc; } syn_t;
 
+/* row sums t(i) = sum_j L(i,j), j increasing (blocked over rows, column-major streaming;
+ * the same order of additions as the plain per-row loop) */
+static void row_sums(int n, const double *L, int ldl, double *t) {
+#pragma omp parallel for schedule(static)
+    for (int i0 = 0; i0 < n; i0 += row_block(n)) {
+        const int rb = row_block(n), i1 = i0 + rb < n ? i0 + rb : n;
+        for (int i = i0; i < i1; i++) t[i] = 0.0;
+        for (int j = 0; j < n; j++)
+            for (int i = i0; i < i1; i++) t[i] += AT(L, ldl, i, j);
+    }
+}
+
 static void syndromes(int n, const double *L, int ldl, const double *r, const double *c,
                       double kap, syn_t *s) {
-#pragma omp parallel for schedule(static)
-    for (int i = 0; i < n; i++) {
-        double t = 0.0;
-        for (int j = 0; j < n; j++) t += AT(L, ldl, i, j);
-        s->Dr[i] = r[i] - t;
-    }
+    row_sums(n, L, ldl, s->Dr);
+    for (int i = 0; i < n; i++) s->Dr[i] = r[i] - s->Dr[i];
 #pragma omp parallel for schedule(static)
     for (int j = 0; j < n; j++) {
         double t = 0.0;
@@ -480,11 +506,7 @@ done:
 
 /* encode (Fig. 3, Alg. 3 l.2): r = A e, c = e^T A, kappa = e^T A e (R22) */
 void ora_encode(int n, const double *A, int lda, double *r, double *c, double *kappa) {
-    for (int i = 0; i < n; i++) {
-        double s = 0.0;
-        for (int j = 0; j < n; j++) s += AT(A, lda, i, j);
-        r[i] = s;
-    }
+    row_sums(n, A, lda, r);
     for (int j = 0; j < n; j++) {
         double s = 0.0;
         for (int i = 0; i < n; i++) s += AT(A, lda, i, j);
