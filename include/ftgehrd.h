@@ -20,6 +20,10 @@
  *    FT_E_CUDA / FT_E_NCCL / FT_E_NOMEM   runtime failures
  * Every call returns only after its stream has finished (info depends on the
  * device-side verification outcome).
+ *
+ * Threading: the library is NOT reentrant.  Its workspace, cached CUDA graphs and
+ * counters are per device and process-global; calls from several host threads
+ * (on one device or several) must be serialised by the caller.
  */
 #ifndef FTGEHRD_H
 #define FTGEHRD_H
@@ -51,8 +55,10 @@ enum { FT_PHASE_BEFORE_PANEL = 0, FT_PHASE_AFTER_PANEL = 1, FT_PHASE_AFTER_RIGHT
  *   C   column-checksum c(j)     (Ac_chk)
  *   K   corner kappa = e^T L e   (R22)
  *   Y   panel workspace Y(i,j)   (j = column within the panel; R15)
- *   V   panel workspace V(i,j)   (the copy the updates read; R15) */
-enum { FT_SITE_A = 0, FT_SITE_R = 1, FT_SITE_C = 2, FT_SITE_K = 3, FT_SITE_Y = 4, FT_SITE_V = 5 };
+ *   V   panel workspace V(i,j)   (the copy the updates read; R15)
+ *   T   block-reflector factor T(i,j), 0 <= i, j < 64 (the nb x nb upper triangle is what the
+ *       left update W' = T^T V^T A reads; R15 extended to T) */
+enum { FT_SITE_A = 0, FT_SITE_R = 1, FT_SITE_C = 2, FT_SITE_K = 3, FT_SITE_Y = 4, FT_SITE_V = 5, FT_SITE_T = 6 };
 
 typedef struct {
     int32_t panel;  /* iteration t >= 0 (ignored for AT_END) */
@@ -195,6 +201,9 @@ void ft_debug_panel_path(int bits);
  * the CTAs of the last tile row / strip (1, the default).  Results agree
  * up to rounding; CUDA-graph replay is off while 0. */
 void ft_debug_left_fold(int on);
+/* Number of panel launches that ran the two-reduction wide kernel (>= 32 rows per CTA, the large-n
+ * path) since load / the last reset: tests use it to show which panel kernel a run exercised. */
+int64_t ft_debug_wide_launches(int reset);
 
 #ifdef __cplusplus
 }

@@ -538,12 +538,13 @@ __global__ void k_larft(const double *V, int64_t ldw, const double *tau, double 
 }
 cudaError_t ft_larft(const double *V, int64_t ldw, const double *tau, double *T, int n, int ihi, int k, int ib,
                      cudaStream_t s) {
-    static bool attr = false;
+    static unsigned attr = 0;
+    const unsigned dbit = ft_dev_bit();
     const int smem = (2 * FT_NBMAX * FT_NBMAX + FT_NBMAX) * sizeof(double);
-    if (!attr) {
+    if (!(attr & dbit)) {
         cudaError_t e = cudaFuncSetAttribute(k_larft, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
         if (e != cudaSuccess) return e;
-        attr = true;
+        attr |= dbit;
     }
     g_ft_launches++;
     k_larft<<<1, 512, smem, s>>>(V, ldw, tau, T, ihi, k, ib);

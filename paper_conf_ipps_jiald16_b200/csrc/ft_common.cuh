@@ -162,3 +162,24 @@ FT_DEV double warp_sum(double v) {
 }
 
 FT_DEV bool not_within(double d, double tau) { return !(fabs(d) <= tau); }  // NaN -> true
+
+// Checksum of row r of the block-reflector factor T over the entries the updates read (the upper
+// triangle, T(r, c) for r <= c < K; reading R15 extended to T).  Four consecutive lanes
+// per row (q = 0..3 takes c = r+q, r+q+4, ...), combined by xor shuffles: the same additions in
+// the same order wherever it is evaluated, so a fault-free recomputation matches the checksum the
+// panel stored.  get(r, c) returns T(r, c); every lane of the 4-lane group must call it.
+template <class F>
+FT_DEV void t_row_checksum(F get, int r, int q, int K, double &s, double &sa) {
+    s = 0.0;
+    sa = 0.0;
+    if (r < K)
+        for (int c = r + q; c < K; c += 4) {
+            const double v = get(r, c);
+            s += v;
+            sa += fabs(v);
+        }
+    s += __shfl_xor_sync(0xffffffffu, s, 1);
+    sa += __shfl_xor_sync(0xffffffffu, sa, 1);
+    s += __shfl_xor_sync(0xffffffffu, s, 2);
+    sa += __shfl_xor_sync(0xffffffffu, sa, 2);
+}

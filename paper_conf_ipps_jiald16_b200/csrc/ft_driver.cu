@@ -20,6 +20,12 @@
 #include "ft_internal.h"
 
 int64_t g_ft_launches = 0;
+int64_t g_ft_wide_launches = 0;
+extern "C" int64_t ft_debug_wide_launches(int reset) {
+    const int64_t v = g_ft_wide_launches;
+    if (reset) g_ft_wide_launches = 0;
+    return v;
+}
 static int g_dbg_panel = -1;
 static unsigned long long *g_dbg_buf = nullptr;
 static int g_dbg_mode = 0;
@@ -438,6 +444,9 @@ double *site_addr(Call &C, const ft_fault &f) {
     case FT_SITE_V:
         if (f.i < 0 || f.i > n || f.j < 0 || f.j >= FT_NBMAX) return nullptr;
         return w.V + f.i + f.j * ldw;
+    case FT_SITE_T:
+        if (f.i < 0 || f.i >= FT_NBMAX || f.j < 0 || f.j >= FT_NBMAX) return nullptr;
+        return w.T + f.i + f.j * FT_NBMAX;
     }
     return nullptr;
 }
@@ -542,6 +551,7 @@ int right_update(Call &C, int t, double sign, int do_w, bool precheck = false) {
         g.transT = 1;
         g.strip_done = w.strip_done;
     }
+    g.tctl = (C.abft && sign < 0 && do_w) ? w.ctl : nullptr;  // T checksum where W' = T^T W is formed
     if (precheck) {  // fused pre-update check (R15), decided by every CTA before it touches A
         g.pre_ctl = w.ctl;
         g.pre_n = C.n;
@@ -581,6 +591,7 @@ int left_update(Call &C, int t, double sign, int nsplit, int endcheck = 0, bool 
     g.ectl = w.ctl;
     g.pre_reset = pre_reset ? w.ctl : nullptr;
     g.fold = C.abft ? g_left_fold : 0;
+    g.tctl = (C.abft && sign < 0) ? w.ctl : nullptr;
     CK(ft_launch_gemm_left(g, C.s));
     return 0;
 }
@@ -795,7 +806,14 @@ int recover(Call &C, const FtCtl &h) {
     CK(cudaMemsetAsync(w.ctl->eY, 0, sizeof(double) * 2 * FT_NBMAX * FT_ESTR, C.s));
     CK(cudaMemsetAsync(w.ctl->sums, 0, sizeof(double) * 4, C.s));
     CK(cudaMemsetAsync(&w.ctl->done_count, 0, 3 * sizeof(int), C.s));  // done_count, done_ytop, done_left
-    if (h.halt_stage == 2) {
+    CK(cudaMemsetAsync(&w.ctl->tbad, 0, sizeof(int), C.s));
+    if (h.halt_stage == 3) {
+        // the right update ran with a T that failed its checksum (W' is void, the left update did not
+        // run): undo the right update only, then redo the panel from its checkpoint
+        if (right_update(C, t, +1.0, 0)) return FT_E_CUDA;
+        C.ev(FT_EV_ROLLBACK, t, h.halt_reason, 0, 0.0);
+        C.rollbacks++;
+    } else if (h.halt_stage == 2) {
         // reverse computation: add back the left, then the right update
         if (left_update(C, t, +1.0, trailing_nsplit(C, t))) return FT_E_CUDA;
         if (right_update(C, t, +1.0, 0)) return FT_E_CUDA;

@@ -319,6 +319,17 @@ __global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
                 }
                 cp_async_wait<0>();
                 __syncthreads();
+                if (p.tctl) {
+                    // T checksum (R15 extended to T): the T this CTA is about to consume against the
+                    // row sums the panel stored with it; a mismatch flags the iteration (tbad) and the
+                    // left-update launch raises the halt (the right update itself completes in full)
+                    double ts, tsa;
+                    t_row_checksum([&](int a, int bb) { return Ts[a][bb]; }, tid >> 2, tid & 3, K, ts, tsa);
+                    const int a = tid >> 2;
+                    if ((tid & 3) == 0 && a < K &&
+                        not_within(ts - __ldcg(&p.tctl->tchk[a]), (double)K * 2.220446049250313e-16 * tsa))
+                        p.tctl->tbad = 1;
+                }
                 // W' = op(T) W: this thread's NE outputs as independent chains (one pass over b)
                 double so[NE];
 #pragma unroll
@@ -347,12 +358,13 @@ __global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
 
 template <int KT>
 static cudaError_t launch_right_kt(const GemmRightParams &p, cudaStream_t s) {
-    static bool attr = false;
+    static unsigned attr = 0;
+    const unsigned dbit = ft_dev_bit();
     const size_t smem = sizeof(RightSmemT<KT>);
-    if (!attr) {
+    if (!(attr & dbit)) {
         cudaError_t e = cudaFuncSetAttribute(k_gemm_right<KT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return e;
-        attr = true;
+        attr |= dbit;
     }
     const int nstrip = (p.c_hi - p.c_lo + UB - 1) / UB + (p.has_m ? 1 : 0);
     const int ny = p.nsplit > 0 ? p.nsplit : 1;
@@ -439,6 +451,17 @@ __global__ void k_wprep(const double *__restrict__ Wpart, int64_t wstride, int n
 template <int KT>
 __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
     if (p.ctl && p.ctl->halt) return;
+    if (p.tctl && __ldcg(&p.tctl->tbad)) {  // the right update consumed a corrupted T: nothing here runs
+        if (blockIdx.x == 0 && blockIdx.y == 0 && threadIdx.x == 0) {
+            FtCtl *ctl = p.tctl;
+            ctl->halt_panel = p.panel;
+            ctl->halt_stage = 3;
+            ctl->halt_reason = 32;
+            __threadfence();
+            ctl->halt = 1;
+        }
+        return;
+    }
     if ((int)blockIdx.y < p.nyf) {
         // frozen row sums of the panel columns k..e-1 (final now, untouched by this launch; R6):
         // Fr(i) += sum_{col in [max(k, i-1), e)} A(i, col) for i <= e -- one row per thread in
@@ -684,12 +707,13 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
 
 template <int KT>
 static cudaError_t launch_left_kt(const GemmLeftParams &p, cudaStream_t s) {
-    static bool attr = false;
+    static unsigned attr = 0;
+    const unsigned dbit = ft_dev_bit();
     const size_t smem = sizeof(LeftSmemT<KT>);
-    if (!attr) {
+    if (!(attr & dbit)) {
         cudaError_t e = cudaFuncSetAttribute(k_gemm_left<KT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return e;
-        attr = true;
+        attr |= dbit;
     }
     // fold: tiles cover rows [r_lo, r_hi-1) and columns [c_lo, c_hi-1); the checksum row and
     // column (index n) are folded into the last tile row / strip
@@ -882,12 +906,13 @@ __global__ void __launch_bounds__(YF_R * 64) k_ytop_finalize(YtopParams p) {
 }
 
 cudaError_t ft_launch_ytop(const YtopParams &p, cudaStream_t s) {
-    static bool attr = false;
+    static unsigned attr = 0;
+    const unsigned dbit = ft_dev_bit();
     size_t smem = sizeof(YtopSmem);
-    if (!attr) {
+    if (!(attr & dbit)) {
         cudaError_t e = cudaFuncSetAttribute(k_ytop_partial, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return e;
-        attr = true;
+        attr |= dbit;
     }
     int nm = (p.k + 1 + YT_M - 1) / YT_M;
     g_ft_launches += 2;

@@ -22,8 +22,9 @@
 struct FtCtl {
     int halt;         // != 0: every later kernel of this call is a no-op
     int halt_panel;   // iteration at which the halt was raised
-    int halt_stage;   // 1 = pre-update (verify-before-consume / workspace check), 2 = post-update
-    int halt_reason;  // bit 0: D_r flag, 1: Y check, 2: V check, 3: scalar check (paper), 4: kappa
+    int halt_stage;   // 1 = pre-update (verify-before-consume / workspace check), 2 = post-update,
+                      // 3 = T checksum failed after the right update (only the right update to undo)
+    int halt_reason;  // bit 0: D_r flag, 1: Y check, 2: V check, 3: scalar check (paper), 4: kappa, 5: T check
     int nflag;        // flagged rows in the fused verify of the current iteration
     int done_count;   // last-block-done counter (k_endcheck)
     int done_ytop;    // last-block-done counter (fused pre-update decision in the Y_top finalize)
@@ -37,6 +38,12 @@ struct FtCtl {
     double eV[64 * FT_ESTR];
     double sums[4];       // end check: sum r, sum c
     double tmax;          // max |T| of the last panel (written by the panel kernel; pre-update tolerance)
+    // T checksum (reading R15 extended to T): row sums of the upper triangle of the panel's T, written
+    // by the panel kernel with T; re-evaluated from T in memory by the right-update CTAs that form
+    // W' = T^T W.  A mismatch sets tbad (the right update has then been applied in full); the left
+    // update launch turns it into a halt of stage 3 (roll back the right update, redo the panel)
+    double tchk[64];
+    int tbad;
     double inj_delta[FT_MAXFAULTS];
     int inj_done[FT_MAXFAULTS];
 };
@@ -119,6 +126,9 @@ struct GemmRightParams {
     // and the fused D_r flag count before touching A; a failed check halts the whole launch
     FtCtl *pre_ctl;  // non-NULL: evaluate the check (pre_n, pre_panel)
     int pre_n, pre_panel;
+    // T checksum check (ABFT): the last CTA of each strip verifies the T it read against ctl->tchk
+    // before forming W' = op(T) W; on a mismatch it sets ctl->tbad (non-NULL: check on)
+    FtCtl *tctl;
 };
 // global column of local column l in the 1-D block-column cyclic layout; local column ncl
 // is the replicated row-checksum column r (global n)
@@ -150,6 +160,8 @@ struct GemmLeftParams {
     double *Fr;
     FtCtl *ectl;
     FtCtl *pre_reset;  // non-NULL: CTA (0,0) clears the fused pre-update sums for the next panel
+    FtCtl *tctl;       // non-NULL: a set tctl->tbad (T checksum failed in the right update) makes the
+                       // launch a no-op and raises the halt (stage 3) instead
     // 1: row r_hi-1 and column c_hi-1 are the checksum row c and column r (= n, ABFT); they are
     // updated by CUDA-core dot products in the CTAs owning the last row tile / column strip
     // instead of as an extra 64-row tile and 64-column strip of DMMA work (n % 64 == 0 would
@@ -206,3 +218,12 @@ cudaError_t ft_larft(const double *V, int64_t ldw, const double *tau, double *T,
 cudaError_t ft_set_identity(double *Q, int64_t ldq, int n, cudaStream_t s);
 
 extern int64_t g_ft_launches;
+extern int64_t g_ft_wide_launches;  // launches of the two-reduction (wide) panel kernel
+
+// Bit of the current device in a per-device "attribute set" mask: kernel attributes such as the
+// dynamic shared-memory opt-in belong to a device context, so one-time setup is keyed by device.
+inline unsigned ft_dev_bit() {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    return 1u << (dev & 31);
+}

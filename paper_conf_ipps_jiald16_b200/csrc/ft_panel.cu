@@ -1027,12 +1027,19 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
                 p.ctl->tmax = m;
             }
         }
+        if (p.abft && tid < 4 * FT_NBMAX) {  // T checksum (R15 extended to T), read by the right update
+            double ts, tsa;
+            t_row_checksum([&](int a, int bb) { return S.Ts[a][bb]; }, tid >> 2, tid & 3, ib, ts, tsa);
+            if ((tid & 3) == 0 && (tid >> 2) < ib) p.ctl->tchk[tid >> 2] = ts;
+        }
     }
 }
 
 cudaError_t ft_launch_panel_multi(const PanelLaunch &L, int nsm, cudaStream_t s) {
     static int max_smem = 0;
-    if (!max_smem) {
+    static unsigned attr = 0;
+    const unsigned dbit = ft_dev_bit();
+    if (!(attr & dbit)) {
         int dev = 0;
         cudaGetDevice(&dev);
         cudaDeviceGetAttribute(&max_smem, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
@@ -1043,6 +1050,7 @@ cudaError_t ft_launch_panel_multi(const PanelLaunch &L, int nsm, cudaStream_t s)
             cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem);
             if (e != cudaSuccess) return e;
         }
+        attr |= dbit;
     }
     static int ctas = -1, explicit_path = 0;
     if (ctas < 0) {

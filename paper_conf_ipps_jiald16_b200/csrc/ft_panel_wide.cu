@@ -731,12 +731,19 @@ __global__ void __launch_bounds__(PT, 1) k_panel_wide(const __grid_constant__ Pa
                 p.ctl->tmax = m;
             }
         }
+        if (p.abft && tid < 4 * FT_NBMAX) {  // T checksum (R15 extended to T), read by the right update
+            double ts, tsa;
+            t_row_checksum([&](int a, int bb) { return S.Ts[a][bb]; }, tid >> 2, tid & 3, ib, ts, tsa);
+            if ((tid & 3) == 0 && (tid >> 2) < ib) p.ctl->tchk[tid >> 2] = ts;
+        }
     }
 }
 
 cudaError_t ft_launch_panel_wide(const PanelLaunch &L, int nsm, cudaStream_t s) {
     static int max_smem = 0;
-    if (!max_smem) {
+    static unsigned attr = 0;
+    const unsigned dbit = ft_dev_bit();
+    if (!(attr & dbit)) {
         int dev = 0;
         cudaGetDevice(&dev);
         cudaDeviceGetAttribute(&max_smem, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
@@ -745,6 +752,7 @@ cudaError_t ft_launch_panel_wide(const PanelLaunch &L, int nsm, cudaStream_t s) 
             cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem);
             if (e != cudaSuccess) return e;
         }
+        attr |= dbit;
     }
     if (L.nr != 1) return cudaErrorInvalidValue;
     int grid = nsm < L.r[0].ngroups ? nsm : L.r[0].ngroups;
@@ -758,6 +766,7 @@ cudaError_t ft_launch_panel_wide(const PanelLaunch &L, int nsm, cudaStream_t s) 
     const bool cache = want <= (size_t)max_smem;
     void *args[] = {const_cast<PanelLaunch *>(&L)};
     g_ft_launches++;
+    g_ft_wide_launches++;
     const void *fn = cache ? (const void *)k_panel_wide<true, false> : (const void *)k_panel_wide<false, false>;
     return cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(PT), args, cache ? want : fixed, s);
 }

@@ -18,7 +18,7 @@ _lib = None
 
 FT_E_UNCORRECTABLE, FT_E_CUDA, FT_E_NCCL, FT_E_NOMEM = 1, 2, 3, 4
 PHASE_BEFORE_PANEL, PHASE_AFTER_PANEL, PHASE_AFTER_RIGHT, PHASE_AFTER_UPDATE, PHASE_AT_END = range(5)
-SITE_A, SITE_R, SITE_C, SITE_K, SITE_Y, SITE_V = range(6)
+SITE_A, SITE_R, SITE_C, SITE_K, SITE_Y, SITE_V, SITE_T = range(7)
 EV_NAMES = ["INJECT", "DETECT", "FIX_DATA", "FIX_R", "FIX_C", "FIX_K", "FIX_Q", "FIX_QR", "FIX_QC",
             "FIX_QK", "UNCORRECTABLE", "ROLLBACK", "PANEL_REDO"]
 POLICY_EAGER, POLICY_PAPER = 0, 1

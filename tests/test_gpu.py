@@ -444,3 +444,46 @@ def test_wide_panel_kernel_large():
     resid = n1(Ad - Q @ H @ Q.T) / (n * n1(Ad) * eps)
     orth = n1(torch.eye(n, dtype=torch.float64, device="cuda") - Q.T @ Q) / (n * eps)
     assert resid <= 30 and orth <= 30, (resid, orth)
+
+
+# ------------------------------------------------------------------ T (block-reflector factor)
+@pytest.mark.parametrize("n,nb,i,j,bit", [(128, 32, 3, 10, 55), (128, 32, 0, 0, 52), (128, 32, 7, 31, 62),
+                                          (600, 32, 5, 20, 45), (300, 64, 40, 60, 63)])
+def test_t_fault_after_panel_rolled_back(n, nb, i, j, bit):
+    """R15 extended to T: a flip in the upper triangle of T between the panel and the updates
+    (the entries W' = T^T W reads) fails the T checksum where the right update forms W'; the
+    right update is rolled back and the panel redone.  Result at the oracle bar."""
+    A = synth.matrix(n)
+    dA, tau, res = faulty(A, nb, [(1, ft.PHASE_AFTER_PANEL, ft.SITE_T, i, j, bit)])
+    assert res.info == 0, res.events
+    assert any(e[0] == "ROLLBACK" and e[1] == 1 and e[2] == 32 for e in res.events), res.events
+    assert res.report.rollbacks >= 1
+    check_against_oracle(A, dA, tau, nb=nb)
+
+
+@pytest.mark.parametrize("phase,i,j", [(ft.PHASE_AFTER_PANEL, 10, 3),   # strict lower triangle: never read
+                                       (ft.PHASE_AFTER_RIGHT, 3, 10),   # after W' = T^T W was formed
+                                       (ft.PHASE_AFTER_UPDATE, 2, 2)])
+def test_t_fault_harmless_positions(phase, i, j):
+    """T words the remaining steps of the iteration never read: no detection, no effect."""
+    n, nb = 128, 32
+    A = synth.matrix(n)
+    dA, tau, res = faulty(A, nb, [(1, phase, ft.SITE_T, i, j, 61)])
+    assert res.info == 0, res.events
+    assert res.report.detected == 0 and res.report.rollbacks == 0, res.events
+    check_against_oracle(A, dA, tau, nb=nb)
+
+
+def test_policy_paper_fault_detect_rollback_locate_redo():
+    """POLICY_PAPER (R11, the paper's own detection): the scalar |sum r - sum c| test at the end of
+    the iteration (Alg. 3 l.12-13) -> reverse computation (l.14) -> location by recomputation and
+    correction -> redo.  A flip mid-update in area 2 and one before the panel."""
+    n, nb = 256, 32
+    A = synth.matrix(n)
+    for f in [(2, ft.PHASE_AFTER_RIGHT, ft.SITE_A, 150, 200, 55), (3, ft.PHASE_AFTER_UPDATE, ft.SITE_A, 130, 220, 57),
+              (2, ft.PHASE_BEFORE_PANEL, ft.SITE_A, 120, 230, 54)]:
+        dA, tau, res = faulty(A, nb, [f], policy=ft.POLICY_PAPER)
+        assert res.info == 0, (f, res.events)
+        assert res.report.rollbacks >= 1, (f, res.events)
+        assert ("FIX_DATA", f[3], f[4]) in fixes(res.events), (f, res.events)
+        check_against_oracle(A, dA, tau, nb=nb)
