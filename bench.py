@@ -1,19 +1,22 @@
 #!/usr/bin/env python3
 """Benchmark: ABFT Hessenberg reduction (BASELINE.json metric) on B200.
 
-  python bench.py [--gpus N] [--steps K] [--warmup W] [--n 2048] [--nb 32] [--impl ours|reference]
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--n 16384] [--nb 64] [--impl ours|reference]
 
-One step = one full ft_dgehrd (panel + updates + checksum encode / verify / final
-verification) of a fresh synthetic n x n FP64 matrix already resident in HBM.
-Timing: CUDA events on the call's stream around each step, L2 flushed (256 MiB
-write) and the input restored between steps, outside the timed events; the
-job time is the max over ranks of the summed step times.  ABFT-off steps (the
-"optimized but fault-prone" baseline of P:358) are interleaved to report the
-resilience overhead.  Prints ONE JSON line on rank 0.
+Workload: BASELINE config C3 (n = 16384, nb = 64, ABFT on, EAGER policy) -- the largest
+single-GPU configuration of BASELINE.json (its metric names no config), one reduction per GPU.
+One step = one full ft_dgehrd (encode, panels, updates, verification, final verification) of
+the synthetic n x n FP64 matrix already resident in HBM; ABFT-off steps (the "optimized but
+fault-prone" baseline of P:358) are interleaved with the ABFT-on steps to report the resilience
+overhead.  Timing: CUDA events on the call's stream around each step; the input (2.1 GB, larger
+than L2) is restored between steps outside the events; job time = max over ranks of the summed
+ABFT-on step times.  Config C2 (n = 2048, nb = 32, L2 flushed between steps) is measured the same
+way and reported under "c2".  Prints ONE JSON line on rank 0.
 """
 from __future__ import annotations
 
 import argparse
+import ctypes
 import json
 import os
 import subprocess
@@ -25,30 +28,49 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 METRIC = "FP64 Hessenberg Gflop/s (10/3·n^3) at 1/2/4/8 B200; ABFT overhead %"
+ORACLE_PREFIX_PANELS = 1  # the oracle's bounded sample: the first panel (nb columns) of the workload
 
 
 def flops(n: int) -> float:
     return 10.0 / 3.0 * n ** 3
 
 
-def gemv_bytes(n: int, nb: int, ilo: int = 1, ihi: int | None = None) -> list[float]:
-    """Algorithmic GEMV bytes of each panel launch: 8 * sum_c (ihi-k-1)(ihi-c-1)."""
+def panels(n: int, nb: int, ilo: int = 1, ihi: int | None = None):
     ihi = n if ihi is None else ihi
-    out = []
     k = ilo - 1
     while k < ihi - 2:
-        ib = min(nb, ihi - 2 - k)
-        out.append(8.0 * sum((ihi - k - 1) * (ihi - c - 1) for c in range(k, k + ib)))
+        yield k, min(nb, ihi - 2 - k)
         k += nb
-    return out
 
 
-def measured_peaks():
-    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+def gemv_bytes(n: int, nb: int) -> list[float]:
+    """Algorithmic GEMV bytes of each panel launch: 8 * sum_c (n-k-1)(n-c-1)."""
+    return [8.0 * sum((n - k - 1) * (n - c - 1) for c in range(k, k + ib)) for k, ib in panels(n, nb)]
+
+
+def gemm_flops(n: int, nb: int) -> list[float]:
+    """Algorithmic flops of each iteration's right-update launch (A(0:n, e:n) -= Y V^T, fused with
+    W = V^T A(k+1:n, e:n)) plus its left update (A(k+1:n, e:n) -= V (T^T W)): 2 ib n (n-e) +
+    4 ib (n-k-1)(n-e) (checksum row / column excluded)."""
+    return [2.0 * ib * n * (n - k - ib) + 4.0 * ib * (n - k - 1) * (n - k - ib) for k, ib in panels(n, nb)]
+
+
+def dgehd2_prefix_flops(n: int, ncols: int) -> float:
+    """Exact flops of the unblocked reduction's first ncols reflectors (ihi = n): right step
+    y = A v and A -= tau y v^T (4 n m), left step w = v^T A and A -= tau v w (4 m (n-c-1)),
+    m = n-c-1.  Summed over all n-2 columns this is the metric's 10/3 n^3 (to leading order)."""
+    return float(sum(4 * n * (n - c - 1) + 4 * (n - c - 1) ** 2 for c in range(min(ncols, n - 2))))
+
+
+def load_json(rel):
     try:
-        return json.load(open(p))
+        return json.load(open(os.path.join(ROOT, rel)))
     except Exception:
         return None
+
+
+def workload_name(n: int, nb: int) -> str:
+    return {(16384, 64): "C3", (2048, 32): "C2", (64, 16): "C1"}.get((n, nb), "custom")
 
 
 class ClockSampler:
@@ -89,72 +111,210 @@ class ClockSampler:
             self.proc.kill()
         if self.thread:
             self.thread.join(timeout=2)
-        sms = [float(r[1]) for r in self.rows if len(r) >= 9 and r[1].replace(".", "").isdigit()]
-        mx = [float(r[2]) for r in self.rows if len(r) >= 9 and r[2].replace(".", "").isdigit()]
+        ok = [r for r in self.rows if len(r) >= 9 and r[1].replace(".", "").isdigit()]
+        sms = sorted(float(r[1]) for r in ok)
+        mx = [float(r[2]) for r in ok if r[2].replace(".", "").isdigit()]
+        pw = [float(r[3]) for r in ok if r[3].replace(".", "").isdigit()]
         reasons = set()
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for r in self.rows:
-            if len(r) >= 9:
-                for nm, v in zip(names, r[5:9]):
-                    if v.lower().startswith("active"):
-                        reasons.add(nm)
+        for r in ok:
+            for nm, v in zip(names, r[5:9]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
         if not sms:
             return None
-        sms.sort()
         return {"sm_mhz": sms[len(sms) // 2], "sm_max_mhz": max(mx) if mx else None,
-                "reasons": sorted(reasons), "samples": len(sms)}
+                "reasons": sorted(reasons), "samples": len(sms), "power_w_max": max(pw) if pw else None}
 
 
-def oracle_sample(n: int, nb: int, seconds_cap: float = 30.0):
-    """Time the CPU oracle (as it stands) on the host cores: full ABFT reduction of the
-    same workload if it fits the cap, else a prefix of panels (scaled to Gflop/s)."""
+# ------------------------------------------------------------------------------------------ oracle
+def oracle_prefix(A, nb: int):
+    """The CPU oracle as it stands on the first ORACLE_PREFIX_PANELS panel(s) of the workload:
+    encode, the boundary verification and nb unblocked reflector steps with their checksum
+    bookkeeping (ora_ft_dgehd2 stopped by its verify hook).  Gflop/s on the prefix's exact
+    DGEHD2 flop count (the encode and verification are not counted)."""
     import oracle
-    import synth
-    A = synth.matrix(n)
+    n = A.shape[0]
+    ncols = min(ORACLE_PREFIX_PANELS * nb, n - 2)
     t0 = time.perf_counter()
-    info, _, _, _, _ = oracle.ft_dgehd2(A, nb)
+    info, _, _, _, _ = oracle.ft_dgehd2(A, nb, stop_after_panel=ORACLE_PREFIX_PANELS - 1)
     dt = time.perf_counter() - t0
-    return {"value": flops(n) / dt / 1e9, "unit": "Gflop/s", "cores": oracle.num_threads(), "kind": "oracle",
-            "sample": f"one full ABFT reduction n={n} nb={nb} (unblocked DGEHD2 + checksum bookkeeping, C/OpenMP), "
-                      f"{dt:.2f} s", "seconds": dt}
+    if info != 0:
+        raise RuntimeError(f"oracle info={info}")
+    return dgehd2_prefix_flops(n, ncols) / dt / 1e9, dt, ncols
+
+
+def oracle_sample(A, nb: int):
+    import oracle
+    val, dt, ncols = oracle_prefix(A, nb)
+    n = A.shape[0]
+    return {"value": val, "unit": "Gflop/s", "cores": oracle.num_threads(), "kind": "oracle",
+            "sample": f"the first {ncols} columns (panel 0) of the {workload_name(n, nb)} workload n={n}: "
+                      f"ora_ft_dgehd2 (unblocked DGEHD2 + Theorem-1 bookkeeping, encode and one boundary "
+                      f"verification included, C/OpenMP) stopped after panel 0, {dt:.2f} s; Gflop/s on the "
+                      f"prefix's exact DGEHD2 flops ({dgehd2_prefix_flops(n, ncols):.3e})",
+            "prefix_columns": ncols, "seconds": dt}
 
 
 def run_reference(args, rank: int, world: int):
-    """--impl reference: the oracle is this tier's reference arm (no installable reference code)."""
+    """--impl reference: the oracle is this tier's reference arm (no installable reference code).
+    Each step is the bounded sample of the workload oracle_prefix() describes."""
     if rank != 0:
         return
     import oracle
     import synth
     n, nb = args.n, args.nb
-    A = synth.matrix(n)
     oracle.build()
+    A = synth.matrix(n)
+    ncols = min(ORACLE_PREFIX_PANELS * nb, n - 2)
+    pf = dgehd2_prefix_flops(n, ncols)
     times = []
     for it in range(args.warmup + args.steps):
-        t0 = time.perf_counter()
-        info, _, _, _, _ = oracle.ft_dgehd2(A, nb)
-        dt = time.perf_counter() - t0
+        _, dt, _ = oracle_prefix(A, nb)
         if it >= args.warmup:
             times.append(dt)
     T = sum(times)
-    val = flops(n) * len(times) / T / 1e9
+    val = pf * len(times) / T / 1e9
+    sample = (f"per step: the first {ncols} columns (panel 0) of n={n}: ora_ft_dgehd2 stopped after panel 0 "
+              f"(encode + one boundary verification + {ncols} reflector steps); Gflop/s on the prefix's exact "
+              f"DGEHD2 flops {pf:.3e}")
     line = {"metric": METRIC, "value": val, "unit": "Gflop/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": 1e3 * T / len(times), "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic U(0,1), seed 20160523+n",
-            "impl": "reference",
-            "config": {"workload": f"C2: n={n} nb={nb} ABFT on", "n": n, "nb": nb, "abft": 1,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic U(0,1) (splitmix64 counter generator, seed 20160523+n)", "impl": "reference",
+            "config": {"workload": f"{workload_name(n, nb)}: n={n} nb={nb} ABFT on, oracle prefix sample",
+                       "n": n, "nb": nb, "abft": 1, "prefix_columns": ncols,
                        "parallelism": "host cores (OpenMP)"},
             "cpu_baseline": {"value": val, "unit": "Gflop/s", "cores": oracle.num_threads(), "kind": "oracle",
-                             "sample": f"full ABFT reduction n={n} per step"},
+                             "sample": sample, "prefix_columns": ncols},
             "e2e": {"value": val, "unit": "Gflop/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
 
-def run_sharded(args, rank: int, world: int, local: int, dist):
-    """N > 1: ONE n x n reduction, 1-D block-column cyclic over the N GPUs (SURVEY 8(e));
-    the per-column GEMV partials move through peer memory inside the panel kernel.  Strong
-    scaling: value = steps * 10/3 n^3 / (max over ranks of the summed step times)."""
-    import ctypes
+# ------------------------------------------------------------------------------------------ GPU arm
+def measure(ft, torch, A, n, nb, steps, warmup, flush_l2, stream, clocks=None):
+    """Interleaved ABFT-on / ABFT-off steps; returns (on_ms, off_ms, launches during on-steps)."""
+    dA0 = ft.fortran(torch.from_numpy(A).cuda())
+    dA = ft.fortran(torch.empty((n, n), dtype=torch.float64, device="cuda"))
+    tau = torch.zeros(n, dtype=torch.float64, device="cuda")
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda") if flush_l2 else None
 
+    def one(abft: bool):
+        dA.copy_(dA0)
+        if flush is not None:
+            flush.fill_(1.0)  # evict the matrix from L2 between steps
+        torch.cuda.synchronize()
+        l0 = ft.launch_count()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        _, res = ft.dgehrd(dA, tau=tau, nb=nb, abft=abft, stream=stream)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        if res.info != 0:
+            raise RuntimeError(f"ft_dgehrd info={res.info}: {ft.strerror(res.info)} {res.events}")
+        return e0.elapsed_time(e1), ft.launch_count() - l0
+
+    for _ in range(warmup):
+        one(True)
+        one(False)
+    if clocks:
+        clocks.start()
+    on_ms, off_ms, launches = [], [], 0
+    for _ in range(steps):
+        t, nl = one(True)
+        on_ms.append(t)
+        launches += nl
+        off_ms.append(one(False)[0])
+    torch.cuda.synchronize()
+    return on_ms, off_ms, launches, (dA0, dA, tau)
+
+
+def roofline(ft, torch, bufs, n, nb, stream, step_ms):
+    """Dominant kernel (the DLAHR2 panel with its trailing GEMV, HBM-bound) and the update GEMMs
+    (FP64 DMMA), from one extra reduction with live per-launch CUDA events (graph replay off for
+    that call; its own total is the step time the shares refer to)."""
+    L = ft.lib()
+    L.ft_debug_time_kernels.argtypes = [ctypes.c_int]
+    L.ft_debug_kernel_ms.argtypes = [ctypes.c_int]
+    L.ft_debug_kernel_ms.restype = ctypes.c_double
+    L.ft_debug_kernel_launches.argtypes = [ctypes.c_int]
+    L.ft_debug_kernel_launches.restype = ctypes.c_int
+    dA0, dA, tau = bufs
+    dA.copy_(dA0)
+    torch.cuda.synchronize()
+    L.ft_debug_time_kernels(1)
+    _, res = ft.dgehrd(dA, tau=tau, nb=nb, abft=True, stream=stream, timing=True)
+    torch.cuda.synchronize()
+    L.ft_debug_time_kernels(0)
+    total_ms = res.report.ms[0]
+    kms = [L.ft_debug_kernel_ms(q) for q in range(3)]
+    kn = [L.ft_debug_kernel_launches(q) for q in range(3)]
+    pb, gf = gemv_bytes(n, nb), gemm_flops(n, nb)
+    if kn[0] != len(pb) or kms[0] <= 0:
+        return None
+    peaks = load_json("MEASURED_PEAKS.json")
+    hbm = peaks["hbm_gbs"] if peaks and "hbm_gbs" in peaks else 6650.0
+    hbm_src = "MEASURED_PEAKS.json hbm_gbs (measured copy bandwidth)" if peaks else "fallback 6.65 TB/s (B200_PROFILING.md)"
+    fp = load_json("profiles/fp64_peak.json") or {}
+    fp64 = fp.get("dmma_tflops_sustained") or fp.get("dmma_tflops") or 37.1
+    fp64_src = ("profiles/fp64_peak.json dmma_tflops_sustained (measured on this pool: scripts/mb_dmma.cu, "
+                "register-resident DMMA.8x8x4 loop, seconds-long)") if fp else "37.1 TFLOP/s (profiles/r01/mb_dmma.txt)"
+    traffic, tsrc = None, None
+    tj = load_json(f"profiles/panel_traffic_n{n}_nb{nb}.json") or load_json("profiles/panel_traffic.json")
+    if tj and tj.get("n") == n and tj.get("nb") == nb:
+        traffic, tsrc = tj.get("dram_bytes_per_launch"), tj.get("source")
+    achieved = sum(pb) / (kms[0] / 1e3) / 1e9
+    l2_note = ("matrix (%.1f MB) fits in the 126 MB L2: frac can exceed 1" % (8e-6 * n * n)) if 8 * n * n < 100e6 \
+        else "matrix (%.2f GB) is larger than L2: the GEMV streams from HBM" % (8e-9 * n * n)
+    out = {"bound": "hbm", "kernel": "k_panel / k_panel_wide (DLAHR2 panel incl. the trailing GEMV)",
+           "achieved": achieved, "peak": hbm, "unit": "GB/s", "frac": achieved / hbm, "traffic": traffic,
+           "traffic_source": tsrc, "share_of_step": kms[0] / total_ms,
+           "algorithmic_bytes_per_launch": sum(pb) / len(pb), "launches": kn[0],
+           "avg_launch_ms": kms[0] / kn[0], "peak_source": hbm_src, "note": l2_note}
+    if kn[1] == len(gf) and kn[2] == len(gf) and kms[1] + kms[2] > 0:
+        g_ach = sum(gf) / ((kms[1] + kms[2]) / 1e3) / 1e12
+        out["gemm"] = {"bound": "tensor", "kernel": "k_gemm_right (+W) + k_gemm_left (DMMA m8n8k4 f64)",
+                       "achieved": g_ach, "peak": fp64, "unit": "TFLOP/s", "frac": g_ach / fp64,
+                       "share_of_step": (kms[1] + kms[2]) / total_ms, "right_ms": kms[1], "left_ms": kms[2],
+                       "algorithmic_flops": sum(gf), "peak_source": fp64_src}
+    # whole-step additive roofline (north star): GEMV bytes at HBM bandwidth + the rest of the flops at FP64 peak
+    t_roof = sum(pb) / (hbm * 1e9) + (flops(n) - sum(pb) / 4) / (fp64 * 1e12)
+    out["step_roofline_ms"] = 1e3 * t_roof
+    out["step_frac"] = 1e3 * t_roof / step_ms
+    out["timing_run_total_ms"] = total_ms
+    out["phases_ms"] = {k: res.report.ms[i] for i, k in enumerate(
+        ["total", "panel+Ytop", "right", "left", "verify", "recovery", "copy", "encode"])}
+    return out
+
+
+def e2e_host(ft, torch, np, A, n, nb, stream, steps, warmup):
+    """End to end through the C ABI with HOST buffers (pinned): H2D of A, the reduction, D2H of
+    H/V and tau, all inside ft_dgehrd_host and inside the timed region."""
+    L = ft.lib()
+    hA0 = torch.from_numpy(np.asfortranarray(A).T.copy()).pin_memory()  # row-major transpose == Fortran A
+    hA = torch.empty_like(hA0).pin_memory()
+    htau = torch.zeros(n, dtype=torch.float64).pin_memory()
+    opts = ft.ftgehrd.make_opts(nb=nb, abft=True, stream=stream)
+    times = []
+    for it in range(warmup + steps):
+        hA.copy_(hA0)
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        info = L.ft_dgehrd_host(n, 1, n, ctypes.c_void_p(hA.data_ptr()), n, ctypes.c_void_p(htau.data_ptr()),
+                                ctypes.byref(opts))
+        t1 = time.perf_counter()
+        if info != 0:
+            raise RuntimeError(f"ft_dgehrd_host info={info}")
+        if it >= warmup:
+            times.append(t1 - t0)
+    return times
+
+
+def run_sharded(args, rank: int, world: int, local: int, dist):
+    """N > 1: ONE n x n reduction, 1-D block-column cyclic over the N GPUs; the
+    per-column GEMV partials move through peer memory inside the panel kernel.  Strong scaling:
+    value = steps * 10/3 n^3 / (max over ranks of the summed step times)."""
     import numpy as np
     import torch
 
@@ -165,16 +325,14 @@ def run_sharded(args, rank: int, world: int, local: int, dist):
     A = synth.matrix(n)  # the same matrix on every rank (seed 20160523 + n)
     cols = ft.cyclic_columns(n, nb, rank, world)
     slab0 = ft.fortran(torch.from_numpy(np.ascontiguousarray(A[:, cols])).cuda())
-    slab = slab0.clone()
-    slab = ft.fortran(slab)
+    slab = ft.fortran(slab0.clone())
     tau = torch.zeros(n, dtype=torch.float64, device="cuda")
-    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda")
     stream = torch.cuda.current_stream()
     ft.mgpu_init(n)
 
     def one(abft: bool):
         slab.copy_(slab0)
-        flush.fill_(1.0)
+        torch.cuda.synchronize()
         e0 = torch.cuda.Event(enable_timing=True)
         e1 = torch.cuda.Event(enable_timing=True)
         e0.record(stream)
@@ -192,10 +350,12 @@ def run_sharded(args, rank: int, world: int, local: int, dist):
     sampler.start()
     dist.barrier()
     torch.cuda.synchronize()
-    launches0 = ft.launch_count()
-    on_ms = [one(True)[0] for _ in range(args.steps)]
-    launches = ft.launch_count() - launches0
-    off_ms = [one(False)[0] for _ in range(args.steps)]
+    on_ms, off_ms, launches = [], [], 0
+    for _ in range(args.steps):
+        l0 = ft.launch_count()
+        on_ms.append(one(True)[0])
+        launches += ft.launch_count() - l0
+        off_ms.append(one(False)[0])
     torch.cuda.synchronize()
     dist.barrier()
     clocks = sampler.stop()
@@ -203,13 +363,12 @@ def run_sharded(args, rank: int, world: int, local: int, dist):
     dist.all_reduce(tt, op=dist.ReduceOp.MAX)
     T_on, T_off = tt.tolist()
     value = args.steps * flops(n) / T_on / 1e9
-    # e2e: this rank's slab from pinned host memory, the reduction, H/V slab + tau back
     hs0 = slab0.cpu().pin_memory()
     hs = torch.empty_like(hs0).pin_memory()
     htau = torch.zeros(n, dtype=torch.float64).pin_memory()
     times = []
-    for it in range(args.warmup + args.steps):
-        flush.fill_(1.0)
+    esteps = min(args.steps, 5)
+    for it in range(2 + esteps):
         torch.cuda.synchronize()
         dist.barrier()
         t0 = time.perf_counter()
@@ -219,21 +378,21 @@ def run_sharded(args, rank: int, world: int, local: int, dist):
         htau.copy_(tau, non_blocking=True)
         torch.cuda.synchronize()
         t1 = time.perf_counter()
-        if it >= args.warmup:
+        if it >= 2:
             times.append(t1 - t0)
     te = torch.tensor([sum(times)], dtype=torch.float64, device="cuda")
     dist.all_reduce(te, op=dist.ReduceOp.MAX)
     e2e = {"value": len(times) * flops(n) / te.item() / 1e9, "unit": "Gflop/s",
            "h2d_bytes_per_step": 8 * n * len(cols), "d2h_bytes_per_step": 8 * n * len(cols) + 8 * n,
-           "api": "ft_dgehrd_mgpu (per-rank slab from pinned host memory)"}
+           "steps": len(times), "api": "ft_dgehrd_mgpu (per-rank slab from pinned host memory)"}
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": "Gflop/s", "n_gpus": world, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": 1e3 * T_on / args.steps, "higher_is_better": True,
                 "scaling": "strong", "vs_baseline": None, "dtype": "f64",
                 "data": "synthetic U(0,1) (splitmix64 counter generator, seed 20160523+n)",
-                "config": {"workload": f"C4-style: one n={n} nb={nb} ABFT reduction, 1-D block-column cyclic "
-                                       f"over {world} GPUs", "n": n, "nb": nb, "abft": 1,
-                           "l2": "flushed between steps (256 MiB write), input restored outside the timed events",
+                "config": {"workload": f"{workload_name(n, nb)} sharded: one n={n} nb={nb} ABFT reduction, 1-D "
+                                       f"block-column cyclic over {world} GPUs", "n": n, "nb": nb, "abft": 1,
+                           "l2": "inputs larger than L2" if 8 * n * n > 200e6 else "L2-resident matrix",
                            "parallelism": f"column-cyclic x{world} (peer-memory exchange per column)"},
                 "abft_overhead_pct": 100.0 * (T_on - T_off) / T_off,
                 "abft_off_value": args.steps * flops(n) / T_off / 1e9,
@@ -246,12 +405,13 @@ def run_sharded(args, rank: int, world: int, local: int, dist):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--n", type=int, default=2048)
-    ap.add_argument("--nb", type=int, default=32)
+    ap.add_argument("--n", type=int, default=16384)
+    ap.add_argument("--nb", type=int, default=64)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-c2", action="store_true", help="skip the extra C2 (n = 2048) measurement")
     ap.add_argument("--replicas", action="store_true",
                     help="N > 1: independent replicas instead of one sharded reduction")
     args = ap.parse_args()
@@ -283,51 +443,18 @@ def main():
     if world > 1 and not args.replicas:
         run_sharded(args, rank, world, local, dist)
         return
-    A = synth.matrix(n, seed=synth.default_seed(n) + rank)
-    dA0 = ft.fortran(torch.from_numpy(A).cuda())
-    dA = ft.fortran(torch.empty((n, n), dtype=torch.float64, device="cuda"))
-    tau = torch.zeros(n, dtype=torch.float64, device="cuda")
-    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda")
     stream = torch.cuda.current_stream()
-
-    def one(abft: bool, timed_events=None):
-        dA.copy_(dA0)
-        flush.fill_(1.0)  # evict the matrix from L2 between steps
-        e0 = torch.cuda.Event(enable_timing=True)
-        e1 = torch.cuda.Event(enable_timing=True)
-        e0.record(stream)
-        _, res = ft.dgehrd(dA, tau=tau, nb=nb, abft=abft, stream=stream)
-        e1.record(stream)
-        torch.cuda.synchronize()
-        if res.info != 0:
-            raise RuntimeError(f"ft_dgehrd info={res.info}: {ft.strerror(res.info)} {res.events}")
-        return e0.elapsed_time(e1), res
-
-    for _ in range(args.warmup):
-        one(True)
-        one(False)
-
+    A = synth.matrix(n, seed=synth.default_seed(n) + rank)
+    big = 8 * n * n > 200e6  # inputs larger than L2 (126 MB): no flush needed between steps
     sampler = ClockSampler(local)
-    sampler.start()
     if dist:
         dist.barrier()
-    torch.cuda.synchronize()
-    launches0 = ft.launch_count()
-    on_ms, off_ms = [], []
-    for _ in range(args.steps):
-        t, _ = one(True)
-        on_ms.append(t)
-    launches = ft.launch_count() - launches0
-    for _ in range(args.steps):
-        t, _ = one(False)
-        off_ms.append(t)
-    torch.cuda.synchronize()
+    on_ms, off_ms, launches, bufs = measure(ft, torch, A, n, nb, args.steps, args.warmup, not big, stream,
+                                            clocks=sampler)
     if dist:
         dist.barrier()
     clocks = sampler.stop()
-
-    T_on = sum(on_ms) / 1e3
-    T_off = sum(off_ms) / 1e3
+    T_on, T_off = sum(on_ms) / 1e3, sum(off_ms) / 1e3
     if dist:
         tt = torch.tensor([T_on, T_off], dtype=torch.float64, device="cuda")
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
@@ -336,69 +463,17 @@ def main():
     off_value = world * args.steps * flops(n) / T_off / 1e9
     overhead = 100.0 * (T_on - T_off) / T_off
 
-    # ---- roofline of the dominant kernel (the panel GEMV), live CUDA-event timing per launch
-    L = ft.lib()
-    import ctypes
-    roofline = None
     try:
-        L.ft_debug_time_panels.argtypes = [ctypes.c_int]
-        L.ft_debug_panel_ms.restype = ctypes.c_double
-        L.ft_debug_panel_launches.restype = ctypes.c_int
-        L.ft_debug_time_panels(1)
-        one(True)
-        L.ft_debug_time_panels(0)
-        panel_ms = L.ft_debug_panel_ms()
-        nlaunch = L.ft_debug_panel_launches()
-        pb = gemv_bytes(n, nb)
-        step_ms = sum(on_ms) / len(on_ms)
-        if nlaunch == len(pb) and panel_ms > 0:
-            achieved = sum(pb) / (panel_ms / 1e3) / 1e9
-            peaks = measured_peaks()
-            peak = peaks["hbm_gbs"] if peaks else 6650.0
-            traffic = None
-            tp = os.path.join(ROOT, "profiles", "panel_traffic.json")
-            if os.path.exists(tp):
-                try:
-                    tj = json.load(open(tp))
-                    if tj.get("n") == n and tj.get("nb") == nb:
-                        traffic = tj.get("dram_bytes_per_launch")
-                except Exception:
-                    pass
-            roofline = {"bound": "hbm", "kernel": "k_panel (DLAHR2 panel incl. trailing GEMV)",
-                        "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                        "traffic": traffic, "share_of_step": panel_ms / step_ms,
-                        "algorithmic_bytes_per_launch": sum(pb) / len(pb), "launches": nlaunch,
-                        "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured)" if peaks else "fallback 6.65 TB/s",
-                        "note": "n=2048 matrix (33.5 MB) is L2-resident inside a step; frac can exceed 1"}
-            # whole-step additive roofline (GEMV bytes at HBM BW + update flops at FP64 peak)
-            fp64_peak = 37.0e12
-            t_roof = sum(pb) / (peak * 1e9) + (flops(n) - sum(pb) / 4) / fp64_peak
-            roofline["step_roofline_ms"] = 1e3 * t_roof
-            roofline["step_frac"] = 1e3 * t_roof / step_ms
+        roof = roofline(ft, torch, bufs, n, nb, stream, 1e3 * T_on / args.steps)
     except AttributeError:
-        roofline = None
+        roof = None
+    del bufs
+    torch.cuda.empty_cache()
 
-    # ---- end to end through the C ABI with host buffers (pinned), copies inside the timed region
     e2e = None
     try:
-        hA0 = torch.from_numpy(np.asfortranarray(A).T.copy()).pin_memory()  # row-major transpose == Fortran A
-        hA = torch.empty_like(hA0).pin_memory()
-        htau = torch.zeros(n, dtype=torch.float64).pin_memory()
-        Lh = L.ft_dgehrd_host
-        opts = ft.ftgehrd.make_opts(nb=nb, abft=True, stream=stream)
-        times = []
-        for it in range(args.warmup + args.steps):
-            hA.copy_(hA0)
-            flush.fill_(1.0)
-            torch.cuda.synchronize()
-            t0 = time.perf_counter()
-            info = Lh(n, 1, n, ctypes.c_void_p(hA.data_ptr()), n, ctypes.c_void_p(htau.data_ptr()),
-                      ctypes.byref(opts))
-            t1 = time.perf_counter()
-            if info != 0:
-                raise RuntimeError(f"ft_dgehrd_host info={info}")
-            if it >= args.warmup:
-                times.append(t1 - t0)
+        esteps = min(args.steps, 5) if big else args.steps
+        times = e2e_host(ft, torch, np, A, n, nb, stream, esteps, 2)
         Te = sum(times)
         if dist:
             tt = torch.tensor([Te], dtype=torch.float64, device="cuda")
@@ -406,30 +481,50 @@ def main():
             Te = tt.item()
         e2e = {"value": world * len(times) * flops(n) / Te / 1e9, "unit": "Gflop/s",
                "h2d_bytes_per_step": 8 * n * n, "d2h_bytes_per_step": 8 * n * n + 8 * (n - 1),
-               "ms_per_step": 1e3 * Te / len(times), "api": "ft_dgehrd_host (pinned host buffers)"}
+               "ms_per_step": 1e3 * Te / len(times), "steps": len(times),
+               "api": "ft_dgehrd_host (pinned host buffers; H2D + reduction + D2H inside the call)"}
     except Exception as ex:  # pragma: no cover
         e2e = {"value": None, "unit": "Gflop/s", "error": str(ex)[:200]}
+
+    c2 = None
+    if not args.no_c2 and (n, nb) != (2048, 32):
+        n2, nb2 = 2048, 32
+        A2 = synth.matrix(n2, seed=synth.default_seed(n2) + rank)
+        s2 = max(args.steps, 10)
+        on2, off2, _, b2 = measure(ft, torch, A2, n2, nb2, s2, args.warmup, True, stream)
+        r2 = roofline(ft, torch, b2, n2, nb2, stream, sum(on2) / len(on2))
+        c2 = {"workload": "C2: n=2048 nb=32 ABFT on (EAGER), one reduction per GPU", "n": n2, "nb": nb2,
+              "steps": s2, "value": s2 * flops(n2) / (sum(on2) / 1e3) / 1e9,
+              "ms_per_step": sum(on2) / s2, "abft_off_value": s2 * flops(n2) / (sum(off2) / 1e3) / 1e9,
+              "ms_per_step_abft_off": sum(off2) / s2,
+              "abft_overhead_pct": 100.0 * (sum(on2) - sum(off2)) / sum(off2),
+              "l2": "flushed between steps (256 MiB write), input restored outside the timed events",
+              "panel_frac": r2["frac"] if r2 else None, "panel_share": r2["share_of_step"] if r2 else None}
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         try:
-            cpu = oracle_sample(n, nb)
+            cpu = oracle_sample(A, nb)
         except Exception as ex:  # pragma: no cover
             cpu = {"value": None, "error": str(ex)[:200]}
 
     if rank == 0:
+        wl = workload_name(n, nb)
         line = {"metric": METRIC, "value": value, "unit": "Gflop/s", "n_gpus": world, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": 1e3 * T_on / args.steps, "higher_is_better": True,
                 "scaling": "weak", "vs_baseline": None, "dtype": "f64",
                 "data": "synthetic U(0,1) (splitmix64 counter generator, seed 20160523+n+rank)",
-                "config": {"workload": f"C2: n={n} nb={nb} ABFT on (EAGER policy), one reduction per GPU",
+                "config": {"workload": f"{wl}: n={n} nb={nb} ABFT on (EAGER policy), one reduction per GPU",
                            "n": n, "nb": nb, "abft": 1, "policy": "eager",
-                           "l2": "flushed between steps (256 MiB write), input restored outside the timed events",
-                           "parallelism": "replicas" if world > 1 else "single GPU"},
+                           "l2": ("inputs larger than L2 (%.2f GB matrix); input restored between steps outside "
+                                  "the timed events" % (8e-9 * n * n)) if big else
+                                 "flushed between steps (256 MiB write), input restored outside the timed events",
+                           "parallelism": "replicas" if world > 1 else "single GPU",
+                           "abft_off_interleaved": True},
                 "abft_overhead_pct": overhead, "abft_off_value": off_value,
                 "ms_per_step_abft_off": 1e3 * T_off / args.steps,
-                "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
-                "clocks": clocks}
+                "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
+                "clocks": clocks, "c2": c2}
         print(json.dumps(line), flush=True)
     if dist:
         dist.destroy_process_group()

@@ -82,8 +82,12 @@ typedef struct {
 typedef struct {
     int32_t detected, corrected, rollbacks, panel_redos, uncorrectable, nevents;
     double max_drift_rel;       /* max |maintained - recomputed| / (n eps ||A||_F) seen */
-    double ms[8];               /* per-phase device ms: 0 total, 1 panel, 2 right, 3 left,
-                                   4 verify, 5 recovery, 6 copy, 7 encode */
+    double ms[8];               /* device ms (CUDA events on the call's stream): 0 the whole call;
+                                   with opts.timing = 1 the phases 1 panel (DLAHR2 kernel + Y_top),
+                                   2 right update (+ W), 3 left update, 4 separate verification
+                                   launches (unfused checks, final verification; fused checks are
+                                   inside 1-3), 5 recovery (rollback, restore, locate, correct),
+                                   6 copy-in/out, 7 encode; -1 when opts.timing = 0 */
     ft_event events[FT_MAX_EVENTS];
 } ft_report;
 
@@ -104,6 +108,8 @@ typedef struct {
                                  [r(0:n) | c(0:n) | kappa] to dchk_out                   */
     double *dchk_out;         /* device buffer of 2n+1 doubles, or NULL                  */
     void *stream;             /* cudaStream_t; NULL -> the legacy default stream          */
+    int32_t timing;           /* 1: record the per-phase times report->ms[1..7] (an event pair
+                                 around each phase; such calls are never graph-replayed)     */
 } ft_opts;
 
 /* Fill *o with defaults (nb 0, abft 1, policy EAGER, c_thr 2, no faults, run to end). */
@@ -190,6 +196,11 @@ int64_t ft_launch_count(int reset);
 void ft_debug_time_panels(int on);
 double ft_debug_panel_ms(void);
 int ft_debug_panel_launches(void);
+/* The same for the bench's kernel classes cls = 0 panel kernel, 1 right-update launch (+ W),
+ * 2 left-update launch: ft_debug_time_kernels(1) resets and starts (graph replay off while on). */
+void ft_debug_time_kernels(int on);
+double ft_debug_kernel_ms(int cls);
+int ft_debug_kernel_launches(int cls);
 void ft_debug_probe_panel(int panel, unsigned long long *dbuf);
 /* ft_debug_panel_path(8) sends every column of every later panel through the explicit
  * two-reduction path (the one-reduction path's cancellation fallback); 64 / 128 force the

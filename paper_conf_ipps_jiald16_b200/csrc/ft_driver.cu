@@ -38,32 +38,27 @@ extern "C" void ft_debug_probe_panel(int panel, unsigned long long *dbuf) {
     g_dbg_panel = panel;
     g_dbg_buf = dbuf;
 }
-// live per-launch timing of the panel kernel (CUDA events on the launching stream)
-static bool g_time_panels = false;
-static double g_panel_ms = 0.0;
-static int g_panel_launches = 0;
-static std::vector<std::pair<cudaEvent_t, cudaEvent_t>> g_panel_events;
-extern "C" void ft_debug_time_panels(int on) {
-    g_time_panels = on != 0;
-    if (on) {
-        g_panel_ms = 0.0;
-        g_panel_launches = 0;
-    }
-}
-extern "C" double ft_debug_panel_ms(void) { return g_panel_ms; }
-extern "C" int ft_debug_panel_launches(void) { return g_panel_launches; }
-static void collect_panel_events() {
-    for (auto &pr : g_panel_events) {
-        float ms = 0.f;
-        if (cudaEventElapsedTime(&ms, pr.first, pr.second) == cudaSuccess) {
-            g_panel_ms += ms;
-            g_panel_launches++;
+// Live device timing with CUDA events on the launching stream.  Categories 1..7 are the report's
+// phases (ft_report.ms, opts.timing); 8..10 the kernel classes of the bench's roofline (panel
+// kernel, right-update launch, left-update launch; ft_debug_time_kernels).
+enum { TC_PANEL = 1, TC_RIGHT = 2, TC_LEFT = 3, TC_VERIFY = 4, TC_RECOVERY = 5, TC_COPY = 6, TC_ENCODE = 7,
+       TK_PANEL = 8, TK_RIGHT = 9, TK_LEFT = 10, TC_N = 11 };
+static bool g_time_kernels = false;
+static double g_kms[3] = {0.0, 0.0, 0.0};
+static int g_kn[3] = {0, 0, 0};
+extern "C" void ft_debug_time_kernels(int on) {
+    g_time_kernels = on != 0;
+    if (on)
+        for (int q = 0; q < 3; q++) {
+            g_kms[q] = 0.0;
+            g_kn[q] = 0;
         }
-        cudaEventDestroy(pr.first);
-        cudaEventDestroy(pr.second);
-    }
-    g_panel_events.clear();
 }
+extern "C" double ft_debug_kernel_ms(int cls) { return cls >= 0 && cls < 3 ? g_kms[cls] : 0.0; }
+extern "C" int ft_debug_kernel_launches(int cls) { return cls >= 0 && cls < 3 ? g_kn[cls] : 0; }
+extern "C" void ft_debug_time_panels(int on) { ft_debug_time_kernels(on); }
+extern "C" double ft_debug_panel_ms(void) { return g_kms[0]; }
+extern "C" int ft_debug_panel_launches(void) { return g_kn[0]; }
 
 namespace {
 
@@ -406,6 +401,9 @@ struct Call {
     // panel ride through the panel's GEMV and Y recurrence (DLAHRD's formulation), and the
     // M-part of the right update is the b0 of those rows (written by the panel)
     bool fused_ytop = false;
+    // event spans (category, start, stop) when this call is timed (opts.timing or kernel timing)
+    bool timing = false;
+    std::vector<std::tuple<int, cudaEvent_t, cudaEvent_t>> spans;
     int rend() const { return abft ? n + 1 : ihi; }
     int cend() const { return abft ? n + 1 : n; }
     int pk(int t) const { return ilo - 1 + t * nb; }
@@ -420,6 +418,36 @@ struct Call {
         events.push_back(e);
     }
 };
+
+// open a timed span of category cat on the call's stream (-1: the call is not timed)
+int span_begin(Call &C, int cat) {
+    if (!C.timing) return -1;
+    cudaEvent_t a = nullptr, b = nullptr;
+    if (cudaEventCreate(&a) != cudaSuccess || cudaEventCreate(&b) != cudaSuccess) return -1;
+    cudaEventRecord(a, C.s);
+    C.spans.emplace_back(cat, a, b);
+    return (int)C.spans.size() - 1;
+}
+void span_end(Call &C, int idx) {
+    if (idx >= 0) cudaEventRecord(std::get<2>(C.spans[idx]), C.s);
+}
+// after the stream has finished: per-category sums (ms) and counts, events released
+void spans_collect(Call &C, double *ms, int *cnt) {
+    for (int q = 0; q < TC_N; q++) {
+        ms[q] = 0.0;
+        cnt[q] = 0;
+    }
+    for (auto &sp : C.spans) {
+        float t = 0.f;
+        if (cudaEventElapsedTime(&t, std::get<1>(sp), std::get<2>(sp)) == cudaSuccess) {
+            ms[std::get<0>(sp)] += t;
+            cnt[std::get<0>(sp)]++;
+        }
+        cudaEventDestroy(std::get<1>(sp));
+        cudaEventDestroy(std::get<2>(sp));
+    }
+    C.spans.clear();
+}
 
 double *site_addr(Call &C, const ft_fault &f) {
     Work &w = *C.w;
@@ -652,17 +680,10 @@ int enqueue_panel(Call &C, int t) {
     p.ytop = C.fused_ytop ? 1 : 0;
     int rendp = (C.rend() + gr - 1) / gr * gr;
     p.ngroups = (rendp - p.rbase) / gr;
-    cudaEvent_t pe0 = nullptr, pe1 = nullptr;
-    if (g_time_panels) {
-        CK(cudaEventCreate(&pe0));
-        CK(cudaEventCreate(&pe1));
-        CK(cudaEventRecord(pe0, C.s));
-    }
+    const int sp_panel = span_begin(C, TC_PANEL);
+    const int sp_kpanel = span_begin(C, TK_PANEL);
     CK(ft_launch_panel(p, w.nsm, C.s));
-    if (g_time_panels) {
-        CK(cudaEventRecord(pe1, C.s));
-        g_panel_events.push_back({pe0, pe1});
-    }
+    span_end(C, sp_kpanel);
     // Y_top = A(0:k+1, k+1:ihi) V T (+ area-1 row sums), unless the panel formed it
     YtopParams y{};
     y.A = w.Aw;
@@ -688,19 +709,36 @@ int enqueue_panel(Call &C, int t) {
     while ((int64_t)ns * (k + 1) > kYtopRows) ns--;
     y.nsplit = std::max(ns, 1);
     if (!C.fused_ytop) CK(ft_launch_ytop(y, C.s));
+    span_end(C, sp_panel);
     if (inject_at(C, t, FT_PHASE_AFTER_PANEL)) return FT_E_CUDA;
     if (eager && !fuse_pre) {
         // a fault is scheduled after the panel: recompute the check sums after it
+        const int sp = span_begin(C, TC_VERIFY);
         CK(cudaMemsetAsync(w.ctl->eY, 0, sizeof(double) * 2 * FT_NBMAX * FT_ESTR, C.s));
         CK(ft_precheck(w.Y, w.V, w.ldw, n, C.ihi, k, ib, w.ctl, C.s));
         CK(ft_decide(w.Y, w.V, w.T, w.ldw, n, k, ib, t, w.ctl, C.s));
+        span_end(C, sp);
     }
-    if (right_update(C, t, -1.0, 1, fuse_pre)) return FT_E_CUDA;
+    {
+        const int sp = span_begin(C, TC_RIGHT), sk = span_begin(C, TK_RIGHT);
+        if (right_update(C, t, -1.0, 1, fuse_pre)) return FT_E_CUDA;
+        span_end(C, sk);
+        span_end(C, sp);
+    }
     if (inject_at(C, t, FT_PHASE_AFTER_RIGHT)) return FT_E_CUDA;
     const bool fuse_end = C.abft && !has_fault(C, t, FT_PHASE_AFTER_UPDATE);
-    if (left_update(C, t, -1.0, trailing_nsplit(C, t), fuse_end ? 1 : 0, fuse_pre)) return FT_E_CUDA;
+    {
+        const int sp = span_begin(C, TC_LEFT), sk = span_begin(C, TK_LEFT);
+        if (left_update(C, t, -1.0, trailing_nsplit(C, t), fuse_end ? 1 : 0, fuse_pre)) return FT_E_CUDA;
+        span_end(C, sk);
+        span_end(C, sp);
+    }
     if (inject_at(C, t, FT_PHASE_AFTER_UPDATE)) return FT_E_CUDA;
-    if (C.abft && !fuse_end) CK(ft_endcheck(w.Aw, w.ldw, n, C.ihi, k, ib, t, C.policy, w.Fr, w.ctl, C.s));
+    if (C.abft && !fuse_end) {
+        const int sp = span_begin(C, TC_VERIFY);
+        CK(ft_endcheck(w.Aw, w.ldw, n, C.ihi, k, ib, t, C.policy, w.Fr, w.ctl, C.s));
+        span_end(C, sp);
+    }
     if (C.hA) {  // columns [k, e) are final: back to the host beside the next panels
         CK(cudaEventRecord(w.copy_ev, C.s));
         CK(cudaStreamWaitEvent(w.copy_stream, w.copy_ev, 0));
@@ -795,7 +833,14 @@ int verify_and_correct(Call &C, int panel, int cdone, int mode, bool *found) {
     return 0;
 }
 
+int recover_body(Call &C, const FtCtl &h);
 int recover(Call &C, const FtCtl &h) {
+    const int sp = span_begin(C, TC_RECOVERY);
+    const int rc = recover_body(C, h);
+    span_end(C, sp);
+    return rc;
+}
+int recover_body(Call &C, const FtCtl &h) {
     Work &w = *C.w;
     const int t = h.halt_panel;
     const int k = C.pk(t);
@@ -839,6 +884,7 @@ int enqueue_start(Call &C, const double *dA, int lda) {
     cudaStream_t s = C.s;
     if (n > 1) CK(cudaMemsetAsync(C.tau, 0, (n - 1) * sizeof(double), s));
     CK(ft_ctl_init(w.ctl, C.c_thr, s));
+    const int sp_copy = span_begin(C, TC_COPY);
     CK(cudaMemsetAsync(w.Aw, 0, (size_t)w.ldw * (n + 1) * sizeof(double), s));
     CK(cudaMemsetAsync(w.V, 0, (size_t)w.ldw * FT_NBMAX * sizeof(double), s));
     CK(cudaMemsetAsync(w.Y, 0, (size_t)w.ldw * FT_NBMAX * sizeof(double), s));
@@ -847,14 +893,17 @@ int enqueue_start(Call &C, const double *dA, int lda) {
                              n * sizeof(double), n, cudaMemcpyHostToDevice, s));
     else
         CK(ft_copy_in(dA, lda, w.Aw, w.ldw, n, s));
+    span_end(C, sp_copy);
     CK(cudaMemsetAsync(w.bvec, 0, (size_t)4 * w.ldw * sizeof(double), s));  // b(q >= ihi) must read 0
     if (reset_panel_state(C)) return FT_E_CUDA;
     if (C.abft) {
+        const int sp_enc = span_begin(C, TC_ENCODE);
         CK(ft_encode(w.Aw, w.ldw, n, w.ctl, w.scratch, w.linepart, s));
         CK(cudaMemsetAsync(w.Fr, 0, w.ldw * sizeof(double), s));
         if (C.ilo > 1) CK(ft_frozen_init(w.Aw, w.ldw, n, C.ilo - 1, w.Fr, s));
         CK(cudaMemsetAsync(w.Qr, 0, w.ldw * sizeof(double), s));
         CK(cudaMemsetAsync(w.Qc, 0, w.ldw * sizeof(double), s));
+        span_end(C, sp_enc);
     }
     return 0;
 }
@@ -874,6 +923,7 @@ int validate(int n, int ilo, int ihi, const void *A, int lda, const void *tau, c
         if (o->c_thr < 0.0 || !(o->c_thr == o->c_thr)) return -7;
         if (o->nfaults < 0 || o->nfaults > FT_MAXFAULTS || (o->nfaults > 0 && !o->faults)) return -7;
         if (o->stop_after_panel < -1) return -7;
+        if (o->timing != 0 && o->timing != 1) return -7;
     }
     return 0;
 }
@@ -897,6 +947,7 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
     C.c_thr = o.c_thr > 0 ? o.c_thr : 2.0;
     C.s = s;
     C.tau = dtau;
+    C.timing = o.timing != 0 || g_time_kernels;
     for (int q = 0; q < o.nfaults; q++) C.faults.push_back(o.faults[q]);
     int rc = get_work(n, &C.w);
     if (rc) return rc;
@@ -921,7 +972,7 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
     // Fault-free calls replay one CUDA graph of the whole launch sequence (start-up kernels and
     // every iteration), captured on the second call with the same shape and buffers; the halt
     // protocol is unchanged (a halted graph's remaining kernels are no-ops, recovery follows).
-    const bool graphable = C.faults.empty() && o.stop_after_panel < 0 && g_dbg_panel < 0 && !g_time_panels &&
+    const bool graphable = C.faults.empty() && o.stop_after_panel < 0 && g_dbg_panel < 0 && !C.timing &&
                            !g_panel_path && g_left_fold &&
                            !getenv("FT_NO_GRAPH");
     bool launched = false;
@@ -1008,8 +1059,10 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
             // final verification of the finished H (a12) and of the Householder vectors
             bool found = false;
             const int cdone = std::max(ihi - 1, ilo - 1);
+            const int sp = span_begin(C, TC_VERIFY);
             int r1 = verify_and_correct(C, -1, cdone, 0, &found);
             if (r1 == 0) r1 = verify_and_correct(C, -1, cdone, 1, &found);
+            span_end(C, sp);
             if (r1 == FT_E_UNCORRECTABLE) info = r1;
             else if (r1) return r1;
         }
@@ -1035,7 +1088,9 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
             CK(d2h(std::max(e1, k0), n));
         }
     } else {
+        const int sp = span_begin(C, TC_COPY);
         CK(ft_copy_out(w.Aw, w.ldw, dA, lda, n, s));
+        span_end(C, sp);
     }
     if (o.stop_after_panel >= 0 && o.dchk_out && C.abft) {
         CK(cudaMemcpyAsync(o.dchk_out, w.Aw + (int64_t)n * w.ldw, n * sizeof(double), cudaMemcpyDeviceToDevice, s));
@@ -1050,7 +1105,14 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
     CK(cudaStreamSynchronize(s));
     float ms = 0.f;
     cudaEventElapsedTime(&ms, ev0, ev1);
-    collect_panel_events();
+    double span_ms[TC_N];
+    int span_cnt[TC_N];
+    spans_collect(C, span_ms, span_cnt);
+    if (g_time_kernels)
+        for (int q = 0; q < 3; q++) {
+            g_kms[q] += span_ms[TK_PANEL + q];
+            g_kn[q] += span_cnt[TK_PANEL + q];
+        }
     cudaEventDestroy(ev0);
     cudaEventDestroy(ev1);
     if (o.report) {
@@ -1080,6 +1142,7 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
         memcpy(&drift, &hf.drift_bits, 8);
         R.max_drift_rel = drift;
         R.ms[0] = ms;
+        for (int q = 1; q < 8; q++) R.ms[q] = o.timing ? span_ms[q] : -1.0;
     }
     return info;
 }

@@ -55,7 +55,7 @@ class Opts(ctypes.Structure):
                 ("policy", ctypes.c_int32), ("c_thr", ctypes.c_double),
                 ("faults", ctypes.POINTER(Fault)), ("nfaults", ctypes.c_int32),
                 ("report", ctypes.POINTER(Report)), ("stop_after_panel", ctypes.c_int32),
-                ("dchk_out", ctypes.c_void_p), ("stream", ctypes.c_void_p)]
+                ("dchk_out", ctypes.c_void_p), ("stream", ctypes.c_void_p), ("timing", ctypes.c_int32)]
 
 
 def build(force: bool = False) -> str:
@@ -129,7 +129,7 @@ def fortran(x):
 
 
 def make_opts(nb=0, abft=True, policy=POLICY_EAGER, c_thr=2.0, faults=(), report=None,
-              stop_after_panel=-1, dchk_out=None, stream=None):
+              stop_after_panel=-1, dchk_out=None, stream=None, timing=False):
     o = Opts()
     lib().ft_opts_default(ctypes.byref(o))
     o.nb = nb
@@ -150,6 +150,7 @@ def make_opts(nb=0, abft=True, policy=POLICY_EAGER, c_thr=2.0, faults=(), report
     o.stop_after_panel = stop_after_panel
     o.dchk_out = ctypes.c_void_p(dchk_out.data_ptr()) if dchk_out is not None else None
     o.stream = _stream_ptr(stream)
+    o.timing = 1 if timing else 0
     o._keep = farr  # keep the fault array alive
     return o
 
