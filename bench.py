@@ -288,6 +288,38 @@ def roofline(ft, torch, bufs, n, nb, stream, step_ms):
     return out
 
 
+def q_formation(ft, torch, bufs, n, nb, stream, reps=3):
+    """NEXT-3: ft_dorghr (checksum-protected and plain) on the reduced workload matrix, CUDA events;
+    Gflop/s on DORGHR's 4/3 n^3 and the fraction of the measured FP64 DMMA peak (GEMM-bound)."""
+    dA0, dA, tau = bufs
+    dA.copy_(dA0)
+    _, res = ft.dgehrd(dA, tau=tau, nb=nb, stream=stream)
+    torch.cuda.synchronize()
+    Q = ft.fortran(torch.empty((n, n), dtype=torch.float64, device="cuda"))
+    out = {}
+    for _ in range(2):
+        for abft in (True, False):
+            ts = []
+            for _ in range(reps):
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record(stream)
+                _, r = ft.dorghr(dA, tau, Q=Q, nb=nb, abft=abft, stream=stream, full=True)
+                e1.record(stream)
+                torch.cuda.synchronize()
+                if r.info != 0:
+                    raise RuntimeError(f"ft_dorghr info={r.info}")
+                ts.append(e0.elapsed_time(e1))
+            out["ms_abft" if abft else "ms_plain"] = sorted(ts)[len(ts) // 2]
+    del Q
+    fl = 4.0 / 3.0 * n ** 3
+    fp = load_json("profiles/fp64_peak.json") or {}
+    peak = fp.get("dmma_tflops_sustained") or 37.1
+    return {"api": "ft_dorghr (opts.abft = 1: Q with row / column checksums through every update)",
+            "ms_per_call": out["ms_abft"], "value": fl / out["ms_abft"] / 1e6, "unit": "Gflop/s (4/3 n^3)",
+            "frac_of_fp64_peak": fl / out["ms_abft"] / 1e9 / peak, "peak_tflops": peak,
+            "ms_plain": out["ms_plain"], "abft_overhead_pct": 100.0 * (out["ms_abft"] - out["ms_plain"]) / out["ms_plain"]}
+
+
 def e2e_host(ft, torch, np, A, n, nb, stream, steps, warmup):
     """End to end through the C ABI with HOST buffers (pinned): H2D of A, the reduction, D2H of
     H/V and tau, all inside ft_dgehrd_host and inside the timed region."""
@@ -467,6 +499,11 @@ def main():
         roof = roofline(ft, torch, bufs, n, nb, stream, 1e3 * T_on / args.steps)
     except AttributeError:
         roof = None
+    qf = None
+    try:
+        qf = q_formation(ft, torch, bufs, n, nb, stream, reps=3 if big else 10)
+    except Exception as ex:  # pragma: no cover
+        qf = {"error": str(ex)[:200]}
     del bufs
     torch.cuda.empty_cache()
 
@@ -524,7 +561,7 @@ def main():
                 "abft_overhead_pct": overhead, "abft_off_value": off_value,
                 "ms_per_step_abft_off": 1e3 * T_off / args.steps,
                 "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
-                "clocks": clocks, "c2": c2}
+                "clocks": clocks, "c2": c2, "q_formation": qf}
         print(json.dumps(line), flush=True)
     if dist:
         dist.destroy_process_group()

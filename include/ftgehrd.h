@@ -128,10 +128,17 @@ int ft_dgehrd(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const 
  * (the end-to-end entry point bench.py times). */
 int ft_dgehrd_host(int n, int ilo, int ihi, double *hA, int lda, double *htau, const ft_opts *opts);
 
-/* Form the explicit orthogonal Q = H(ilo) H(ilo+1) ... H(ihi-1) from the output
- * of ft_dgehrd (LAPACK DORGHR semantics; Q is the identity outside rows/cols
- * ilo..ihi and Q e1 = e1 when ilo = 1).  dQ may alias dA only if ldq == lda.
- * opts may be NULL (only opts->nb and opts->stream are read). */
+/* Form the explicit orthogonal Q = H(ilo) H(ilo+1) ... H(ihi-1) (Q = Q1 Q2 ... Qn-1) from the
+ * output of ft_dgehrd (LAPACK DORGHR semantics; Q is the identity outside rows/cols ilo..ihi and
+ * Q e1 = e1 when ilo = 1).  dQ may alias dA only if ldq == lda.  Blocked and backward: panel
+ * t = npanels-1 .. 0 (columns k = ilo-1 + t nb ..) applies Q = (I - V T V^T) Q with the DMMA kernels.
+ * opts NULL: the plain formation.  opts->abft = 1 (NEXT-3): checksum-protected accumulation -- Q
+ * carries a row checksum r = Q e, a column checksum c = e^T Q and kappa through every update
+ * (Theorem 1), each iteration ends with the sum check (rolled back and located on a
+ * mismatch), and Q is verified and corrected at the end (R12 decoder).  Read: nb, abft,
+ * c_thr, faults (sites A = Q(i,j), R, C, K of Q's checksums; phases BEFORE_PANEL / AFTER_UPDATE of
+ * panel t, AT_END), report, stream, timing.  Returns 0, FT_E_UNCORRECTABLE (Q undefined), or the
+ * argument / runtime codes of ft_dgehrd (-8 dQ, -9 ldq). */
 int ft_dorghr(int n, int ilo, int ihi, const double *dA, int lda, const double *dtau,
               double *dQ, int ldq, const ft_opts *opts);
 

@@ -7,6 +7,8 @@
 //   full verify       D_r = r - L e, D_c = c - e^T L             P:272 (Sec. IV-F, location)
 //   fix               A(i,j) = r(i) - sum_{k!=j} A(i,k) (or col)
 //   inject            XOR one bit of a binary64 word             P:48-52 failure model, R16
+#include <algorithm>
+
 #include "ft_common.cuh"
 #include "ft_internal.h"
 
@@ -344,10 +346,13 @@ cudaError_t ft_endcheck(double *Aw, int64_t ldw, int n, int ihi, int k, int ib, 
                         double *Fr, FtCtl *ctl, cudaStream_t s) {
     int nblk = (n + 1023) / 1024;
     if (nblk > 16) nblk = 16;
-    g_ft_launches += 2;
+    g_ft_launches++;
     k_endcheck<<<nblk, 1024, 0, s>>>(Aw, ldw, n, ihi, k, ib, panel, policy, Fr, ctl);
     int e = k + ib;
-    k_frozen_rows<<<(e + 1 + 255) / 256, 256, 0, s>>>(Aw, ldw, n, k, e, Fr, ctl);
+    if (Fr) {
+        g_ft_launches++;
+        k_frozen_rows<<<(e + 1 + 255) / 256, 256, 0, s>>>(Aw, ldw, n, k, e, Fr, ctl);
+    }
     return cudaGetLastError();
 }
 
@@ -489,7 +494,8 @@ cudaError_t ft_apply_fixes(double *Aw, int64_t ldw, int n, int ilo, int ihi, int
 // ---------------------------------------------------------------------------
 // Q formation helpers (ft_dorghr): dense V from the stored reflectors, and T (DLARFT)
 // ---------------------------------------------------------------------------
-__global__ void k_build_v(const double *Aw, int64_t ldw, double *V, int n, int ihi, int k, int ib) {
+__global__ void k_build_v(const double *Aw, int64_t ldw, double *V, int n, int ihi, int k, int ib, const FtCtl *ctl) {
+    if (ctl && ctl->halt) return;
     int i = blockIdx.x * blockDim.x + threadIdx.x;
     int j = blockIdx.y;
     if (i >= n || j >= ib) return;
@@ -499,23 +505,72 @@ __global__ void k_build_v(const double *Aw, int64_t ldw, double *V, int n, int i
     else if (i >= c + 2 && i < ihi) v = Aw[i + (int64_t)c * ldw];
     V[i + (int64_t)j * ldw] = v;
 }
-cudaError_t ft_build_v(const double *Aw, int64_t ldw, double *V, int n, int ihi, int k, int ib, cudaStream_t s) {
+// V_chk = e^T V as row n of V (the column-checksum coefficients of the protected Q formation: the
+// checksum row c of Q is updated as one more row of the left update, Theorem 1)
+__global__ void k_vchk(double *V, int64_t ldw, int n, int k, int ihi, const FtCtl *ctl) {
+    if (ctl && ctl->halt) return;
+    __shared__ double ws[32];
+    const int j = blockIdx.x;
+    double sum = 0.0;
+    for (int i = k + 1 + threadIdx.x; i < ihi; i += blockDim.x) sum += V[i + (int64_t)j * ldw];
+    sum = warp_sum(sum);
+    if ((threadIdx.x & 31) == 0) ws[threadIdx.x >> 5] = sum;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double t = 0.0;
+        for (int w = 0; w < (int)(blockDim.x >> 5); w++) t += ws[w];
+        V[n + (int64_t)j * ldw] = t;
+    }
+}
+cudaError_t ft_build_v(const double *Aw, int64_t ldw, double *V, int n, int ihi, int k, int ib, cudaStream_t s,
+                       const FtCtl *ctl, int vchk) {
     g_ft_launches++;
-    k_build_v<<<dim3((n + 255) / 256, ib), 256, 0, s>>>(Aw, ldw, V, n, ihi, k, ib);
+    k_build_v<<<dim3((n + 255) / 256, ib), 256, 0, s>>>(Aw, ldw, V, n, ihi, k, ib, ctl);
+    if (vchk) {
+        g_ft_launches++;
+        k_vchk<<<ib, 256, 0, s>>>(V, ldw, n, k, ihi, ctl);
+    }
     return cudaGetLastError();
 }
-// T(0:j, j) = -tau_j T(0:j,0:j) (V(:,0:j)^T v_j), T(j,j) = tau_j  (one block; G = V^T V first)
-__global__ void k_larft(const double *V, int64_t ldw, const double *tau, double *T, int ihi, int k, int ib) {
+// Gram partials of the panel's V over row chunks (DLARFT's V^T V, P:40's compact WY), all SMs:
+// block b sums rows [k+1 + b*GR_ROWS, ...) of V(:, a) V(:, bcol) for a < bcol into gpart[b]
+#define GR_ROWS 64
+__global__ void __launch_bounds__(256) k_gram_part(const double *V, int64_t ldw, int ihi, int k, int ib,
+                                                   double *gpart, const FtCtl *ctl) {
+    if (ctl && ctl->halt) return;
+    __shared__ double Vs[GR_ROWS][FT_NBMAX + 1];
+    const int r0 = k + 1 + blockIdx.x * GR_ROWS, r1 = min(ihi, r0 + GR_ROWS), R = r1 - r0;
+    for (int x = threadIdx.x; x < GR_ROWS * FT_NBMAX; x += blockDim.x) {
+        const int rl = x % GR_ROWS, jj = x / GR_ROWS;
+        Vs[rl][jj] = (rl < R && jj < ib) ? V[r0 + rl + (int64_t)jj * ldw] : 0.0;
+    }
+    __syncthreads();
+    double *g = gpart + (int64_t)blockIdx.x * FT_NBMAX * FT_NBMAX;
+    for (int pidx = threadIdx.x; pidx < FT_NBMAX * FT_NBMAX; pidx += blockDim.x) {
+        const int a = pidx % FT_NBMAX, b = pidx / FT_NBMAX;
+        double s0 = 0.0, s1 = 0.0;
+        if (a < b && b < ib) {
+            int rl = 0;
+            for (; rl + 1 < R; rl += 2) {
+                s0 += Vs[rl][a] * Vs[rl][b];
+                s1 += Vs[rl + 1][a] * Vs[rl + 1][b];
+            }
+            if (rl < R) s0 += Vs[rl][a] * Vs[rl][b];
+        }
+        g[pidx] = s0 + s1;
+    }
+}
+// T(0:j, j) = -tau_j T(0:j,0:j) (V(:,0:j)^T v_j), T(j,j) = tau_j  (one block; G = sum of the
+// k_gram_part partials in chunk order: deterministic)
+__global__ void k_larft(const double *gpart, int nchunk, const double *tau, double *T, int k, int ib,
+                        const FtCtl *ctl) {
+    if (ctl && ctl->halt) return;
     extern __shared__ double larft_smem[];
     double *G = larft_smem, *Ts = larft_smem + FT_NBMAX * FT_NBMAX, *tmp = Ts + FT_NBMAX * FT_NBMAX;
-    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
-    for (int pidx = wid; pidx < ib * ib; pidx += nw) {
-        int a = pidx % ib, b = pidx / ib;
+    for (int pidx = threadIdx.x; pidx < FT_NBMAX * FT_NBMAX; pidx += blockDim.x) {
         double s = 0.0;
-        if (a < b)
-            for (int i = k + 1 + lane; i < ihi; i += 32) s += V[i + (int64_t)a * ldw] * V[i + (int64_t)b * ldw];
-        s = warp_sum(s);
-        if (lane == 0) G[a + b * FT_NBMAX] = s;
+        for (int c = 0; c < nchunk; c++) s += __ldcg(gpart + (int64_t)c * FT_NBMAX * FT_NBMAX + pidx);
+        G[pidx] = s;
     }
     for (int i = threadIdx.x; i < FT_NBMAX * FT_NBMAX; i += blockDim.x) Ts[i] = 0.0;
     __syncthreads();
@@ -537,7 +592,7 @@ __global__ void k_larft(const double *V, int64_t ldw, const double *tau, double 
     }
 }
 cudaError_t ft_larft(const double *V, int64_t ldw, const double *tau, double *T, int n, int ihi, int k, int ib,
-                     cudaStream_t s) {
+                     cudaStream_t s, const FtCtl *ctl, double *gpart) {
     static unsigned attr = 0;
     const unsigned dbit = ft_dev_bit();
     const int smem = (2 * FT_NBMAX * FT_NBMAX + FT_NBMAX) * sizeof(double);
@@ -547,7 +602,10 @@ cudaError_t ft_larft(const double *V, int64_t ldw, const double *tau, double *T,
         attr |= dbit;
     }
     g_ft_launches++;
-    k_larft<<<1, 512, smem, s>>>(V, ldw, tau, T, ihi, k, ib);
+    const int nchunk = std::max(1, (ihi - k - 1 + GR_ROWS - 1) / GR_ROWS);
+    g_ft_launches++;
+    k_gram_part<<<nchunk, 256, 0, s>>>(V, ldw, ihi, k, ib, gpart, ctl);
+    k_larft<<<1, 512, smem, s>>>(gpart, nchunk, tau, T, k, ib, ctl);
     return cudaGetLastError();
 }
 __global__ void k_identity(double *Q, int64_t ldq, int n) {
@@ -559,6 +617,30 @@ cudaError_t ft_set_identity(double *Q, int64_t ldq, int n, cudaStream_t s) {
     if (n <= 0) return cudaSuccess;
     g_ft_launches++;
     k_identity<<<dim3((n + 255) / 256, n), 256, 0, s>>>(Q, ldq, n);
+    return cudaGetLastError();
+}
+// augmented identity of the protected Q formation: Q = I, r = Q e = e (column n), c = e^T Q = e^T
+// (row n), kappa = e^T Q e = n (encode, applied to the initial Q)
+__global__ void k_identity_aug(double *Q, int64_t ldq, int n) {
+    int i = blockIdx.x * blockDim.x + threadIdx.x;
+    int64_t j = blockIdx.y;
+    if (i > n) return;
+    double v;
+    if (i < n && j < n) v = (i == j) ? 1.0 : 0.0;
+    else if (i == n && j == n) v = (double)n;
+    else v = 1.0;
+    Q[i + j * ldq] = v;
+}
+cudaError_t ft_set_identity_aug(double *Q, int64_t ldq, int n, cudaStream_t s) {
+    if (n <= 0) return cudaSuccess;
+    g_ft_launches++;
+    k_identity_aug<<<dim3((n + 1 + 255) / 256, n + 1), 256, 0, s>>>(Q, ldq, n);
+    return cudaGetLastError();
+}
+__global__ void k_ctl_norm(FtCtl *ctl, double v) { ctl->normF = v; }
+cudaError_t ft_ctl_set_norm(FtCtl *ctl, double v, cudaStream_t s) {
+    g_ft_launches++;
+    k_ctl_norm<<<1, 1, 0, s>>>(ctl, v);
     return cudaGetLastError();
 }
 

@@ -192,7 +192,8 @@ int get_work(int n, Work **out) {
     A(dalloc(&w.ypart, (size_t)kYtopRows * FT_NBMAX, b));
     A(dalloc(&w.rowpart, (size_t)kYtopRows, b));
     A(dalloc(&w.scratch, (size_t)64 * ((n + 255) / 256) + 8, b));
-    A(dalloc(&w.linepart, (size_t)64 * ldw, b));
+    // row-sum partials of the verification ([64][ldw]) / Gram partials of Q formation's DLARFT
+    A(dalloc(&w.linepart, (size_t)std::max<int64_t>(64 * ldw, 4096 * ((int64_t)n / 64 + 2)), b));
     A(dalloc(&w.deltas, (size_t)FT_MAX_EVENTS, b));
     A(dalloc(&w.bar, 4, b));
     A(dalloc(&w.strip_done, (N1 + 63) / 64 + 2, b));
@@ -479,6 +480,12 @@ double *site_addr(Call &C, const ft_fault &f) {
     return nullptr;
 }
 
+void fill_report(Call &C, const ft_opts &o, const FtCtl &hf, float ms, const double *span_ms, ft_report &R);
+bool q_has_fault_after(const Call &C, int panel) {
+    for (size_t q = 0; q < C.faults.size() && q < FT_MAXFAULTS; q++)
+        if (C.faults[q].phase == FT_PHASE_AFTER_UPDATE && C.faults[q].panel == panel) return true;
+    return false;
+}
 bool has_fault(const Call &C, int panel, int phase) {
     for (size_t q = 0; q < C.faults.size() && q < FT_MAXFAULTS; q++)
         if (C.faults[q].phase == phase && (phase == FT_PHASE_AT_END || C.faults[q].panel == panel)) return true;
@@ -751,15 +758,18 @@ int enqueue_panel(Call &C, int t) {
 
 // full verify + decode + correct + re-verify.  mode 0: H (cdone finished columns), 1: Q.
 // Returns 0 ok (clean or corrected), FT_E_UNCORRECTABLE, or an error.
-int verify_and_correct(Call &C, int panel, int cdone, int mode, bool *found) {
+// M: the augmented working array (the reduction's Aw, or ft_dorghr's augmented Q); mode 0 reads its
+// checksum column n / row n / corner, mode 1 the Q checksums of the Householder vectors
+int verify_and_correct(Call &C, int panel, int cdone, int mode, bool *found, double *M = nullptr) {
     Work &w = *C.w;
     const int n = C.n;
     const int64_t ldw = w.ldw;
-    double *r = mode == 0 ? w.Aw + (int64_t)n * ldw : w.Qr;
+    if (!M) M = w.Aw;
+    double *r = mode == 0 ? M + (int64_t)n * ldw : w.Qr;
     int64_t rinc = 1;
-    double *c = mode == 0 ? w.Aw + n : w.Qc;
+    double *c = mode == 0 ? M + n : w.Qc;
     int64_t cinc = mode == 0 ? ldw : 1;
-    double *kap = mode == 0 ? w.Aw + n + (int64_t)n * ldw : w.Qc + n;
+    double *kap = mode == 0 ? M + n + (int64_t)n * ldw : w.Qc + n;
     FtCtl hctl;
     CK(cudaMemcpyAsync(&hctl, w.ctl, sizeof(FtCtl), cudaMemcpyDeviceToHost, C.s));
     CK(cudaStreamSynchronize(C.s));
@@ -768,7 +778,7 @@ int verify_and_correct(Call &C, int panel, int cdone, int mode, bool *found) {
     double sums[2], kh;
     *found = false;
     for (int pass = 0; pass < 2; pass++) {
-        CK(ft_full_verify(w.Aw, ldw, n, C.ilo, C.ihi, cdone, mode, r, rinc, c, cinc, nullptr, w.Dr, w.Dc, w.sums,
+        CK(ft_full_verify(M, ldw, n, C.ilo, C.ihi, cdone, mode, r, rinc, c, cinc, nullptr, w.Dr, w.Dc, w.sums,
                           w.linepart, C.s));
         CK(cudaMemcpyAsync(Dr.data(), w.Dr, n * sizeof(double), cudaMemcpyDeviceToHost, C.s));
         CK(cudaMemcpyAsync(Dc.data(), w.Dc, n * sizeof(double), cudaMemcpyDeviceToHost, C.s));
@@ -806,13 +816,19 @@ int verify_and_correct(Call &C, int panel, int cdone, int mode, bool *found) {
                 C.uncorrectable++;
                 return FT_E_UNCORRECTABLE;
             }
-            int nf = (int)std::min<size_t>(P.fixes.size(), FT_MAX_EVENTS);
-            CK(cudaMemcpyAsync(w.fixes, P.fixes.data(), nf * sizeof(FtFix), cudaMemcpyHostToDevice, C.s));
-            CK(ft_apply_fixes(w.Aw, ldw, n, C.ilo, C.ihi, cdone, mode, r, rinc, c, cinc, kap, w.fixes, nf, w.deltas,
-                              C.s));
+            // data fixes first, then the checksum refreshes (they read the repaired data); in chunks
+            // of FT_MAX_EVENTS (a data error that propagated along its column before the final
+            // verification of ft_dorghr is one fix per polluted row)
+            const int nf = (int)P.fixes.size();
             std::vector<double> dl(nf);
-            CK(cudaMemcpyAsync(dl.data(), w.deltas, nf * sizeof(double), cudaMemcpyDeviceToHost, C.s));
-            CK(cudaStreamSynchronize(C.s));
+            for (int q0 = 0; q0 < nf; q0 += FT_MAX_EVENTS) {
+                const int m = std::min(FT_MAX_EVENTS, nf - q0);
+                CK(cudaMemcpyAsync(w.fixes, P.fixes.data() + q0, m * sizeof(FtFix), cudaMemcpyHostToDevice, C.s));
+                CK(ft_apply_fixes(M, ldw, n, C.ilo, C.ihi, cdone, mode, r, rinc, c, cinc, kap, w.fixes, m, w.deltas,
+                                  C.s));
+                CK(cudaMemcpyAsync(dl.data() + q0, w.deltas, m * sizeof(double), cudaMemcpyDeviceToHost, C.s));
+                CK(cudaStreamSynchronize(C.s));
+            }
             for (int q = 0; q < nf; q++) {
                 const FtFix &f = P.fixes[q];
                 int kind = f.kind == 0 || f.kind == 1 ? (mode == 0 ? FT_EV_FIX_DATA : FT_EV_FIX_Q)
@@ -1115,8 +1131,13 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
         }
     cudaEventDestroy(ev0);
     cudaEventDestroy(ev1);
-    if (o.report) {
-        ft_report &R = *o.report;
+    if (o.report) fill_report(C, o, hf, ms, span_ms, *o.report);
+    return info;
+}
+
+// the caller's report: injection events (fault order), then the detection / correction log
+void fill_report(Call &C, const ft_opts &o, const FtCtl &hf, float ms, const double *span_ms, ft_report &R) {
+    {
         memset(&R, 0, sizeof(R));
         // injection events first (in fault order), then the detection/correction log
         std::vector<ft_event> all;
@@ -1144,7 +1165,263 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
         R.ms[0] = ms;
         for (int q = 1; q < 8; q++) R.ms[q] = o.timing ? span_ms[q] : -1.0;
     }
-    return info;
+}
+
+// ---------------------------------------------------------------------------
+// Q formation (DORGHR semantics; Q = H(ilo) ... H(ihi-1)), blocked and backward: for panel
+// t = npanels-1 .. 0, Q(k+1:, k+1:) = (I - V T V^T) Q(k+1:, k+1:) (DLARFB 'L','N','F','C') as
+// W = V^T Q (the right-update kernel's W pass) and Q -= V (T W) (the left-update kernel).
+// With opts.abft = 1 (NEXT-3; P:266/P:278 protect Q's Householder vectors, this protects
+// the accumulation): Q is carried augmented -- column n = r = Q e, row n = c = e^T Q, corner
+// kappa = e^T Q e, encoded from Q = I -- and the same Theorem-1 algebra keeps them
+// valid through every left update (V_chk = e^T V as row n of V; the left kernel folds r, c, kappa).
+// Every iteration ends with the fused sum check (sum r = sum c = kappa; catches checksum-vector
+// errors, rolled back with the retained W' and located); the end verifies Q against r, c and
+// corrects with the R12 decoder.  A data error only ever mixes within its own column (left
+// multiplications), so it is located at the end as one column with many rows, each repaired with
+// the row formula.
+// ---------------------------------------------------------------------------
+double *q_scratch(int n, int64_t ldw, size_t cols, int *rc) {
+    static std::map<int, std::pair<size_t, double *>> qscratch;
+    int dev = 0;
+    *rc = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) {
+        *rc = FT_E_CUDA;
+        return nullptr;
+    }
+    auto &qs = qscratch[dev];
+    size_t need = (size_t)ldw * cols;
+    if (qs.first < need) {
+        if (qs.second) cudaFree(qs.second);
+        qs.second = nullptr;
+        qs.first = 0;
+        if (cudaMalloc(&qs.second, need * sizeof(double)) != cudaSuccess) {
+            cudaGetLastError();
+            *rc = FT_E_NOMEM;
+            return nullptr;
+        }
+        qs.first = need;
+    }
+    return qs.second;
+}
+
+int q_inject(Call &C, double *Qa, int panel, int phase) {
+    const int64_t ldw = C.w->ldw;
+    const int n = C.n;
+    for (size_t q = 0; q < C.faults.size() && q < FT_MAXFAULTS; q++) {
+        const ft_fault &f = C.faults[q];
+        if (f.phase != phase || (phase != FT_PHASE_AT_END && f.panel != panel)) continue;
+        double *a = nullptr;
+        if (f.site == FT_SITE_A && f.i >= 0 && f.i < n && f.j >= 0 && f.j < n) a = Qa + f.i + f.j * ldw;
+        else if (f.site == FT_SITE_R && f.i >= 0 && f.i < n) a = Qa + f.i + (int64_t)n * ldw;
+        else if (f.site == FT_SITE_C && f.j >= 0 && f.j < n) a = Qa + n + f.j * ldw;
+        else if (f.site == FT_SITE_K) a = Qa + n + (int64_t)n * ldw;
+        if (a) CK(ft_inject(a, (int)q, f.bit, C.w->ctl, C.s));
+    }
+    return 0;
+}
+
+int dorghr_run(int n, int ilo, int ihi, const double *dA, int lda, const double *dtau, double *dQ, int ldq,
+               const ft_opts &o) {
+    cudaStream_t s = (cudaStream_t)o.stream;
+    Call C;
+    C.n = n;
+    C.ilo = ilo;
+    C.ihi = ihi;
+    C.nb = o.nb > 0 ? o.nb : (n < 4096 ? 32 : 64);
+    C.abft = o.abft;
+    C.policy = FT_POLICY_EAGER;
+    C.c_thr = o.c_thr > 0 ? o.c_thr : 2.0;
+    C.s = s;
+    C.timing = o.timing != 0;
+    for (int q = 0; q < o.nfaults; q++) C.faults.push_back(o.faults[q]);
+    int rc = get_work(n, &C.w);
+    if (rc) return rc;
+    Work &w = *C.w;
+    const bool ab = C.abft != 0;
+    cudaEvent_t ev0, ev1;
+    CK(cudaEventCreate(&ev0));
+    CK(cudaEventCreate(&ev1));
+    CK(cudaEventRecord(ev0, s));
+    CK(ft_ctl_init(w.ctl, C.c_thr, s));
+    if (ab) CK(ft_ctl_set_norm(w.ctl, std::sqrt((double)n), s));  // ||Q||_F = sqrt(n) (R10 scale of Q)
+    CK(ft_copy_in(dA, lda, w.Aw, w.ldw, n, s));  // private copy of V (dQ may alias dA)
+    // the DMMA tiles move 16-byte chunks: work in an aligned scratch if dQ / ldq are not (and always
+    // with ABFT: the augmented Q has a checksum row and column)
+    double *Qw = dQ;
+    int64_t ldqw = ldq;
+    if (ab || (ldq & 1) || (((uintptr_t)dQ) & 15)) {
+        Qw = q_scratch(n, w.ldw, (size_t)n + 1, &rc);
+        if (rc) return rc;
+        ldqw = w.ldw;
+    }
+    if (ab) CK(ft_set_identity_aug(Qw, ldqw, n, s));
+    else CK(ft_set_identity(Qw, ldqw, n, s));
+    int npanels = 0;
+    for (int k = ilo - 1; k < ihi - 2; k += C.nb) npanels++;
+    C.npanels = npanels;
+    const int rend = ab ? n + 1 : ihi, cend = ab ? n + 1 : ihi;
+    auto enqueue_q = [&](int t) -> int {
+        const int k = ilo - 1 + t * C.nb, ib = std::min(C.nb, ihi - 2 - k);
+        if (ab && q_inject(C, Qw, t, FT_PHASE_BEFORE_PANEL)) return FT_E_CUDA;
+        CK(ft_build_v(w.Aw, w.ldw, w.V, n, ihi, k, ib, s, ab ? w.ctl : nullptr, ab ? 1 : 0));
+        CK(ft_larft(w.V, w.ldw, dtau, w.T, n, ihi, k, ib, s, ab ? w.ctl : nullptr, w.linepart));
+        GemmRightParams g{};
+        g.A = Qw;
+        g.lda = ldqw;
+        g.ldw = w.ldw;
+        g.Y = nullptr;
+        g.V = w.V;
+        g.r_lo = k + 1;
+        g.r_hi = ihi;
+        g.c_lo = k + 1;
+        g.c_hi = cend;
+        g.K = ib;
+        g.wr_lo = k + 1;
+        g.wr_hi = ihi;
+        g.do_right = 0;
+        g.do_w = 1;
+        g.sign = 1.0;
+        g.Wpart = w.Wpart;
+        g.wsplit_stride = ((int64_t)n + 1 + 64) * FT_NBMAX;
+        const int ns = ft_gemm_splits(k + 1, ihi, k + 1, cend, w.nsm);
+        g.nsplit = ns;
+        g.ctl = ab ? w.ctl : nullptr;
+        g.Wt = w.Wt;
+        g.T = w.T;
+        g.transT = 0;
+        g.strip_done = w.strip_done;
+        {
+            const int sp = span_begin(C, TC_RIGHT);
+            CK(ft_launch_gemm_right(g, s));
+            span_end(C, sp);
+        }
+        GemmLeftParams L{};
+        L.A = Qw;
+        L.lda = ldqw;
+        L.ldw = w.ldw;
+        L.V = w.V;
+        L.T = w.T;
+        L.Wpart = w.Wpart;
+        L.Wt = w.Wt;
+        L.r_lo = k + 1;
+        L.r_hi = rend;
+        L.c_lo = k + 1;
+        L.c_hi = cend;
+        L.K = ib;
+        L.nsplit = ns;
+        L.wsplit_stride = g.wsplit_stride;
+        L.transT = 0;
+        L.sign = -1.0;
+        L.ctl = ab ? w.ctl : nullptr;
+        L.wt_ready = 1;
+        if (ab) {  // checksum row / column folded, fused end-of-iteration sum check (no frozen sums)
+            L.fold = 1;
+            L.endcheck = q_has_fault_after(C, t) ? 0 : 1;
+            L.panel = t;
+            L.policy = FT_POLICY_EAGER;
+            L.n = n;
+            L.Fr = nullptr;
+            L.ectl = w.ctl;
+        }
+        {
+            const int sp = span_begin(C, TC_LEFT);
+            CK(ft_launch_gemm_left(L, s));
+            span_end(C, sp);
+        }
+        if (ab) {
+            if (q_inject(C, Qw, t, FT_PHASE_AFTER_UPDATE)) return FT_E_CUDA;
+            if (!L.endcheck) CK(ft_endcheck(Qw, ldqw, n, ihi, k, ib, t, FT_POLICY_EAGER, nullptr, w.ctl, s));
+        }
+        return 0;
+    };
+    int t0 = npanels - 1, attempts = 0;
+    int result = 0;
+    while (true) {
+        for (int t = t0; t >= 0; t--) {
+            rc = enqueue_q(t);
+            if (rc) return rc;
+        }
+        if (!ab) break;
+        FtCtl h;
+        CK(cudaMemcpyAsync(&h, w.ctl, sizeof(FtCtl), cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        if (!h.halt) break;
+        if (++attempts > 4 * (npanels + 1) + (int)C.faults.size() * 4) {
+            C.ev(FT_EV_UNCORRECTABLE, h.halt_panel, -1, -1, 0.0);
+            C.uncorrectable++;
+            result = FT_E_UNCORRECTABLE;
+            break;
+        }
+        // reverse computation of the halted iteration (its V, T, W' are still in the workspace:
+        // every later launch was a no-op), then locate and correct, redo
+        const int sp = span_begin(C, TC_RECOVERY);
+        const int t = h.halt_panel, k = ilo - 1 + t * C.nb, ib = std::min(C.nb, ihi - 2 - k);
+        int zero = 0;
+        CK(cudaMemcpyAsync(&w.ctl->halt, &zero, sizeof(int), cudaMemcpyHostToDevice, s));
+        CK(cudaMemsetAsync(w.ctl->sums, 0, sizeof(double) * 4, s));
+        CK(cudaMemsetAsync(&w.ctl->done_count, 0, 3 * sizeof(int), s));
+        GemmLeftParams L{};
+        L.A = Qw;
+        L.lda = ldqw;
+        L.ldw = w.ldw;
+        L.V = w.V;
+        L.T = w.T;
+        L.Wpart = w.Wpart;
+        L.Wt = w.Wt;
+        L.r_lo = k + 1;
+        L.r_hi = rend;
+        L.c_lo = k + 1;
+        L.c_hi = cend;
+        L.K = ib;
+        L.nsplit = 1;
+        L.wsplit_stride = ((int64_t)n + 1 + 64) * FT_NBMAX;
+        L.transT = 0;
+        L.sign = +1.0;
+        L.wt_ready = 1;
+        L.fold = 1;
+        L.n = n;
+        CK(ft_launch_gemm_left(L, s));
+        C.ev(FT_EV_ROLLBACK, t, h.halt_reason, 0, 0.0);
+        C.rollbacks++;
+        bool found = false;
+        const int r1 = verify_and_correct(C, t, ilo - 1, 0, &found, Qw);
+        span_end(C, sp);
+        if (r1 == FT_E_UNCORRECTABLE) {
+            result = r1;
+            break;
+        }
+        if (r1) return r1;
+        t0 = t;
+    }
+    if (ab && result == 0) {
+        if (q_inject(C, Qw, -1, FT_PHASE_AT_END)) return FT_E_CUDA;
+        bool found = false;
+        const int sp = span_begin(C, TC_VERIFY);
+        const int r1 = verify_and_correct(C, -1, ilo - 1, 0, &found, Qw);  // final verification of Q
+        span_end(C, sp);
+        if (r1 == FT_E_UNCORRECTABLE) result = r1;
+        else if (r1) return r1;
+    }
+    if (Qw != dQ) {
+        const int sp = span_begin(C, TC_COPY);
+        CK(cudaMemcpy2DAsync(dQ, (size_t)ldq * sizeof(double), Qw, (size_t)ldqw * sizeof(double),
+                             (size_t)n * sizeof(double), n, cudaMemcpyDeviceToDevice, s));
+        span_end(C, sp);
+    }
+    CK(cudaEventRecord(ev1, s));
+    FtCtl hf;
+    CK(cudaMemcpyAsync(&hf, w.ctl, sizeof(FtCtl), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    float ms = 0.f;
+    cudaEventElapsedTime(&ms, ev0, ev1);
+    cudaEventDestroy(ev0);
+    cudaEventDestroy(ev1);
+    double span_ms[TC_N];
+    int span_cnt[TC_N];
+    spans_collect(C, span_ms, span_cnt);
+    if (o.report) fill_report(C, o, hf, ms, span_ms, *o.report);
+    return result;
 }
 
 }  // namespace
@@ -1213,96 +1490,14 @@ int ft_dorghr(int n, int ilo, int ihi, const double *dA, int lda, const double *
     ft_opts o;
     ft_opts_default(&o);
     if (opts) o = *opts;
-    int info = validate(n, ilo, ihi, dA, lda, dtau, nullptr);
+    else o.abft = 0;  // NULL opts: the plain formation (documented)
+    int info = validate(n, ilo, ihi, dA, lda, dtau, opts ? &o : nullptr);
     if (info) return info;
     if (n > 0 && !dQ) return -8;
     if (ldq < std::max(1, n)) return -9;
     if (o.nb < 0 || o.nb > FT_NBMAX) return -7;
     if (n == 0) return 0;
-    cudaStream_t s = (cudaStream_t)o.stream;
-    Work *wp = nullptr;
-    int rc = get_work(n, &wp);
-    if (rc) return rc;
-    Work &w = *wp;
-    const int nb = o.nb > 0 ? o.nb : (n < 4096 ? 32 : 64);
-    CK(ft_copy_in(dA, lda, w.Aw, w.ldw, n, s));  // private copy of V (dQ may alias dA)
-    // the DMMA tiles move 16-byte chunks: work in an aligned scratch if dQ / ldq are not
-    double *Qw = dQ;
-    int64_t ldqw = ldq;
-    static std::map<int, std::pair<size_t, double *>> qscratch;
-    if ((ldq & 1) || (((uintptr_t)dQ) & 15)) {
-        int dev = 0;
-        CK(cudaGetDevice(&dev));
-        auto &qs = qscratch[dev];
-        size_t need = (size_t)w.ldw * n;
-        if (qs.first < need) {
-            if (qs.second) cudaFree(qs.second);
-            qs.second = nullptr;
-            CK(cudaMalloc(&qs.second, need * sizeof(double)));
-            qs.first = need;
-        }
-        Qw = qs.second;
-        ldqw = w.ldw;
-    }
-    CK(ft_set_identity(Qw, ldqw, n, s));
-    int npanels = 0;
-    for (int k = ilo - 1; k < ihi - 2; k += nb) npanels++;
-    for (int t = npanels - 1; t >= 0; t--) {
-        const int k = ilo - 1 + t * nb, ib = std::min(nb, ihi - 2 - k);
-        CK(ft_build_v(w.Aw, w.ldw, w.V, n, ihi, k, ib, s));
-        CK(ft_larft(w.V, w.ldw, dtau, w.T, n, ihi, k, ib, s));
-        GemmRightParams g{};
-        g.A = Qw;
-        g.lda = ldqw;
-        g.ldw = w.ldw;
-        g.Y = nullptr;
-        g.V = w.V;
-        g.r_lo = k + 1;
-        g.r_hi = ihi;
-        g.c_lo = k + 1;
-        g.c_hi = ihi;
-        g.K = ib;
-        g.wr_lo = k + 1;
-        g.wr_hi = ihi;
-        g.do_right = 0;
-        g.do_w = 1;
-        g.sign = 1.0;
-        g.Wpart = w.Wpart;
-        g.wsplit_stride = ((int64_t)n + 1 + 64) * FT_NBMAX;
-        const int ns = ft_gemm_splits(k + 1, ihi, k + 1, ihi, w.nsm);
-        g.nsplit = ns;
-        g.ctl = nullptr;
-        g.Wt = w.Wt;
-        g.T = w.T;
-        g.transT = 0;
-        g.strip_done = w.strip_done;
-        CK(ft_launch_gemm_right(g, s));
-        GemmLeftParams L{};
-        L.A = Qw;
-        L.lda = ldqw;
-        L.ldw = w.ldw;
-        L.V = w.V;
-        L.T = w.T;
-        L.Wpart = w.Wpart;
-        L.Wt = w.Wt;
-        L.r_lo = k + 1;
-        L.r_hi = ihi;
-        L.c_lo = k + 1;
-        L.c_hi = ihi;
-        L.K = ib;
-        L.nsplit = ns;
-        L.wsplit_stride = g.wsplit_stride;
-        L.transT = 0;
-        L.sign = -1.0;
-        L.ctl = nullptr;
-        L.wt_ready = 1;
-        CK(ft_launch_gemm_left(L, s));
-    }
-    if (Qw != dQ)
-        CK(cudaMemcpy2DAsync(dQ, (size_t)ldq * sizeof(double), Qw, (size_t)ldqw * sizeof(double),
-                             (size_t)n * sizeof(double), n, cudaMemcpyDeviceToDevice, s));
-    CK(cudaStreamSynchronize(s));
-    return 0;
+    return dorghr_run(n, ilo, ihi, dA, lda, dtau, dQ, ldq, o);
 }
 
 const char *ft_strerror(int info) {

@@ -747,7 +747,7 @@ static cudaError_t launch_left_kt(const GemmLeftParams &p, cudaStream_t s) {
     q.c_hi = c_hi;
     q.ny = ny;
     int nyf = 0;  // extra CTA rows for the frozen row sums (one row of A per thread)
-    if (p.endcheck) {
+    if (p.endcheck && p.Fr) {
         const int rows = std::min(p.c_lo + 1, p.n);
         nyf = ((rows + UT - 1) / UT + nstrip - 1) / nstrip;
     }

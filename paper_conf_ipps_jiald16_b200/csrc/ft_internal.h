@@ -212,10 +212,14 @@ cudaError_t ft_apply_fixes(double *Aw, int64_t ldw, int n, int ilo, int ihi, int
                            double *r, int64_t rinc, double *c, int64_t cinc, double *kappa,
                            const FtFix *fixes, int nfix, double *deltas, cudaStream_t s);
 cudaError_t ft_frob_to_ctl(const double *A, int lda, int n, FtCtl *ctl, cudaStream_t s);
-cudaError_t ft_build_v(const double *Aw, int64_t ldw, double *V, int n, int ihi, int k, int ib, cudaStream_t s);
+cudaError_t ft_build_v(const double *Aw, int64_t ldw, double *V, int n, int ihi, int k, int ib, cudaStream_t s,
+                       const FtCtl *ctl = nullptr, int vchk = 0);
+// gpart: Gram partial workspace of (ihi-k-1)/128 + 1 blocks of 64 x 64 doubles
 cudaError_t ft_larft(const double *V, int64_t ldw, const double *tau, double *T, int n, int ihi, int k,
-                     int ib, cudaStream_t s);
+                     int ib, cudaStream_t s, const FtCtl *ctl, double *gpart);
 cudaError_t ft_set_identity(double *Q, int64_t ldq, int n, cudaStream_t s);
+cudaError_t ft_set_identity_aug(double *Q, int64_t ldq, int n, cudaStream_t s);
+cudaError_t ft_ctl_set_norm(FtCtl *ctl, double v, cudaStream_t s);
 
 extern int64_t g_ft_launches;
 extern int64_t g_ft_wide_launches;  // launches of the two-reduction (wide) panel kernel

@@ -186,17 +186,23 @@ def dgehrd_host(A_np, ilo=1, ihi=None, **kw):
     return tau[: max(n - 1, 0)], Result(info, rep, rep.event_list())
 
 
-def dorghr(A, tau, ilo=1, ihi=None, Q=None, nb=0, stream=None):
-    """Explicit Q from ft_dgehrd's output (DORGHR semantics). Returns (Q, info)."""
+def dorghr(A, tau, ilo=1, ihi=None, Q=None, nb=0, stream=None, abft=True, faults=(), c_thr=2.0, timing=False,
+           full=False):
+    """Explicit Q from ft_dgehrd's output (DORGHR semantics).  abft: checksum-protected accumulation
+    (NEXT-3); faults: (panel, phase, site, i, j, bit) on Q (sites A, R, C, K; phases BEFORE_PANEL /
+    AFTER_UPDATE of panel t, AT_END).  Returns (Q, info), or (Q, Result) with full=True."""
     import torch
     n, lda = _check_fortran(A)
     ihi = n if ihi is None else ihi
     if Q is None:
         Q = fortran(torch.empty((n, n), dtype=torch.float64, device=A.device))
     _, ldq = _check_fortran(Q, "Q")
-    o = make_opts(nb=nb, stream=stream)
+    rep = Report()
+    o = make_opts(nb=nb, stream=stream, abft=abft, faults=faults, c_thr=c_thr, report=rep, timing=timing)
     info = lib().ft_dorghr(n, ilo, ihi, ctypes.c_void_p(A.data_ptr()), lda, ctypes.c_void_p(tau.data_ptr()),
                            ctypes.c_void_p(Q.data_ptr()), ldq, ctypes.byref(o))
+    if full:
+        return Q, Result(info, rep, rep.event_list())
     return Q, info
 
 
