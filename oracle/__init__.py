@@ -16,11 +16,11 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 _LIB_PATH = os.path.join(_HERE, "liboracle.so")
 _lib = None
 
-SITE_A, SITE_R, SITE_C, SITE_K, SITE_QR, SITE_QC = range(6)
+SITE_A, SITE_R, SITE_C, SITE_K, SITE_QR, SITE_QC, SITE_RW, SITE_CW = range(8)
 (EV_INJECT, EV_DETECT, EV_FIX_DATA, EV_FIX_R, EV_FIX_C, EV_FIX_K, EV_FIX_Q,
- EV_FIX_QR, EV_FIX_QC, EV_FIX_QK, EV_UNCORRECTABLE) = range(11)
+ EV_FIX_QR, EV_FIX_QC, EV_FIX_QK, EV_UNCORRECTABLE, EV_FIX_RW, EV_FIX_CW, EV_FIX_KW) = range(14)
 EV_NAMES = ["INJECT", "DETECT", "FIX_DATA", "FIX_R", "FIX_C", "FIX_K", "FIX_Q",
-            "FIX_QR", "FIX_QC", "FIX_QK", "UNCORRECTABLE"]
+            "FIX_QR", "FIX_QC", "FIX_QK", "UNCORRECTABLE", "FIX_RW", "FIX_CW", "FIX_KW"]
 MAX_EVENTS = 1024
 
 
@@ -65,6 +65,11 @@ def lib():
         L.ora_ft_dgehd2.argtypes = [ctypes.c_int, ctypes.c_int, ctypes.c_int, dp, ctypes.c_int, dp,
                                     ctypes.c_int, ctypes.c_double, ctypes.POINTER(Fault),
                                     ctypes.c_int, ctypes.POINTER(Report), ctypes.c_int, dp]
+        L.ora_ft_dgehd2_ex.argtypes = [ctypes.c_int, ctypes.c_int, ctypes.c_int, dp, ctypes.c_int, dp,
+                                       ctypes.c_int, ctypes.c_double, ctypes.c_int, ctypes.POINTER(Fault),
+                                       ctypes.c_int, ctypes.POINTER(Report), ctypes.c_int, dp]
+        L.ora_decode_w.argtypes = [ctypes.c_int, dp, ctypes.c_int, dp, dp, dp, dp, dp, dp, dp, ctypes.c_double,
+                                   ctypes.POINTER(Report), ctypes.c_int]
         L.ora_decode.argtypes = [ctypes.c_int, dp, ctypes.c_int, dp, dp, dp, ctypes.c_double,
                                  ctypes.POINTER(Report), ctypes.c_int, ctypes.c_int]
         L.ora_encode.argtypes = [ctypes.c_int, dp, ctypes.c_int, dp, dp, dp]
@@ -109,9 +114,10 @@ def dorghr(Aout: np.ndarray, tau: np.ndarray, ilo: int = 1, ihi: int | None = No
 
 
 def ft_dgehd2(A: np.ndarray, nb: int, ilo: int = 1, ihi: int | None = None, c_thr: float = 2.0,
-              faults=(), stop_after_panel: int = -1):
+              faults=(), stop_after_panel: int = -1, weighted: bool = False):
     """ABFT oracle.  faults: iterable of (panel, site, i, j, bit).
-    Returns (info, A_out, tau, report, chk) with chk = [r | c | kappa] when stopping."""
+    Returns (info, A_out, tau, report, chk) with chk = [r | c | kappa] when stopping
+    (weighted: [r | c | kappa | r_w | c_w | e^T L w | w^T L e])."""
     A = _fmat(A)
     n = A.shape[0]
     ihi = n if ihi is None else ihi
@@ -121,9 +127,9 @@ def ft_dgehd2(A: np.ndarray, nb: int, ilo: int = 1, ihi: int | None = None, c_th
     for k, (p, s, i, j, b) in enumerate(fl):
         farr[k] = Fault(p, s, i, j, b, 0)
     rep = Report()
-    chk = np.zeros(2 * n + 1)
-    info = lib().ora_ft_dgehd2(n, ilo, ihi, _dp(A), max(n, 1), _dp(tau), nb, c_thr, farr, len(fl),
-                               ctypes.byref(rep), stop_after_panel, _dp(chk))
+    chk = np.zeros(4 * n + 3 if weighted else 2 * n + 1)
+    info = lib().ora_ft_dgehd2_ex(n, ilo, ihi, _dp(A), max(n, 1), _dp(tau), nb, c_thr, 1 if weighted else 0,
+                                  farr, len(fl), ctypes.byref(rep), stop_after_panel, _dp(chk))
     if info < 0:
         raise ValueError(f"ora_ft_dgehd2 info={info}")
     return info, A, tau[: max(n - 1, 0)], rep, chk
@@ -139,6 +145,21 @@ def decode(L: np.ndarray, r: np.ndarray, c: np.ndarray, kappa: float, tau_abs: f
     n = L.shape[0]
     res = lib().ora_decode(n, _dp(L), max(n, 1), _dp(r), _dp(c), _dp(k), tau_abs, ctypes.byref(rep), 0, mode)
     return res, L, r, c, float(k[0]), rep
+
+
+def decode_w(L: np.ndarray, r, c, kappa: float, rw, cw, krw: float, kcw: float, tau_abs: float):
+    """Run decoder v3 (weighted pair, w_i = i + 1).
+    Returns (result, L, r, c, kappa, rw, cw, krw, kcw, report); result 0/1/2."""
+    L = _fmat(L)
+    r, c, rw, cw = (np.array(x, dtype=np.float64) for x in (r, c, rw, cw))
+    k = np.array([kappa, krw, kcw], dtype=np.float64)
+    rep = Report()
+    n = L.shape[0]
+    kp = k.ctypes.data
+    res = lib().ora_decode_w(n, _dp(L), max(n, 1), _dp(r), _dp(c), ctypes.cast(kp, ctypes.POINTER(ctypes.c_double)),
+                             _dp(rw), _dp(cw), ctypes.cast(kp + 8, ctypes.POINTER(ctypes.c_double)),
+                             ctypes.cast(kp + 16, ctypes.POINTER(ctypes.c_double)), tau_abs, ctypes.byref(rep), 0)
+    return res, L, r, c, float(k[0]), rw, cw, float(k[1]), float(k[2]), rep
 
 
 def encode(A: np.ndarray):

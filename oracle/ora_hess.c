@@ -95,7 +95,12 @@ static int check_args(int n, int ilo, int ihi, const void *A, int lda, const voi
 typedef struct {
     double *r, *c, *kap;     /* H checksums (length n, n, 1) */
     double *qr, *qc, *qk;    /* Q checksums */
+    /* weighted pair (NEXT-1), w_i = i + 1, or NULL: r_w = L w, c_w = w^T L and the corners
+     * krw = e^T L w, kcw = w^T L e */
+    double *rw, *cw, *krw, *kcw;
 } chk_t;
+
+#define WGT(i) ((double)(i) + 1.0) /* weight of 0-based index i (NEXT-1) */
 
 static double reflector_step(int n, int ihi, double *A, int lda, int c,
                              double *y, double *w, chk_t *chk) {
@@ -122,9 +127,12 @@ static double reflector_step(int n, int ihi, double *A, int lda, int c,
     double ev = 1.0;                     /* e^T v */
     for (int i = c + 2; i < ihi; i++) ev += V(i);
 
+    double wv = WGT(c + 1);              /* w^T v (weighted pair) */
+    for (int i = c + 2; i < ihi; i++) wv += WGT(i) * V(i);
     if (chk) {
         /* reduced column c: left term of its own reflector (R7): c[c] -= (e^T v)(alpha - beta) */
         chk->c[c] -= ev * (alpha0 - beta);
+        if (chk->rw) chk->cw[c] -= wv * (alpha0 - beta);
         /* Q checksums of the new Householder vector (Fig. 5) */
         chk->qc[c] = ev - 1.0;
         for (int i = c + 2; i < ihi; i++) chk->qr[i] += V(i);
@@ -149,6 +157,16 @@ static double reflector_step(int n, int ihi, double *A, int lda, int c,
         double cv = 0.0;
         for (int j = c + 1; j < ihi; j++) cv += chk->c[j] * V(j);
         *chk->kap -= tau * cv * ev;
+        if (chk->rw) {
+            /* the same algebra with w: r_w' = A (I - tau v v^T) w = r_w - tau (w^T v) y,
+             * c_w' = c_w - tau (c_w.v) v^T, e^T A' w and w^T A' e likewise */
+            double cwv = 0.0;
+            for (int j = c + 1; j < ihi; j++) cwv += chk->cw[j] * V(j);
+            *chk->krw -= tau * cv * wv;
+            *chk->kcw -= tau * cwv * ev;
+            for (int j = c + 1; j < ihi; j++) chk->cw[j] -= tau * cwv * V(j);
+            for (int i = 0; i < ihi; i++) chk->rw[i] -= tau * wv * y[i];
+        }
         for (int j = c + 1; j < ihi; j++) chk->c[j] -= tau * cv * V(j);
         for (int i = 0; i < ihi; i++) chk->r[i] -= tau * ev * y[i];
     }
@@ -170,6 +188,15 @@ static double reflector_step(int n, int ihi, double *A, int lda, int c,
         double vr = 0.0;
         for (int i = c + 1; i < ihi; i++) vr += V(i) * chk->r[i];
         *chk->kap -= tau * ev * vr;
+        if (chk->rw) {
+            /* r_w' = (I - tau v v^T) r_w, c_w' = c_w - tau (w^T v) (v^T A), corners likewise */
+            double vrw = 0.0;
+            for (int i = c + 1; i < ihi; i++) vrw += V(i) * chk->rw[i];
+            *chk->krw -= tau * ev * vrw;
+            *chk->kcw -= tau * wv * vr;
+            for (int i = c + 1; i < ihi; i++) chk->rw[i] -= tau * vrw * V(i);
+            for (int j = c + 1; j < n; j++) chk->cw[j] -= tau * wv * w[j];
+        }
         for (int i = c + 1; i < ihi; i++) chk->r[i] -= tau * vr * V(i);
         for (int j = c + 1; j < n; j++) chk->c[j] -= tau * ev * w[j];
     }
@@ -504,6 +531,264 @@ done:
     return result;
 }
 
+/* ------------------------------------------------------------------ */
+/* Weighted checksum pair (NEXT-1): w_i = i + 1.           */
+/* r_w = L w, c_w = w^T L, krw = e^T L w, kcw = w^T L e.                 */
+/* ------------------------------------------------------------------ */
+static void encode_w(int n, const double *L, int ldl, double *rw, double *cw, double *krw, double *kcw) {
+#pragma omp parallel for schedule(static)
+    for (int i0 = 0; i0 < n; i0 += row_block(n)) {
+        const int rb = row_block(n), i1 = i0 + rb < n ? i0 + rb : n;
+        for (int i = i0; i < i1; i++) rw[i] = 0.0;
+        for (int j = 0; j < n; j++) {
+            const double wj = WGT(j);
+            for (int i = i0; i < i1; i++) rw[i] += AT(L, ldl, i, j) * wj;
+        }
+    }
+#pragma omp parallel for schedule(static)
+    for (int j = 0; j < n; j++) {
+        double t = 0.0;
+        for (int i = 0; i < n; i++) t += WGT(i) * AT(L, ldl, i, j);
+        cw[j] = t;
+    }
+    double a = 0.0, b = 0.0;
+    for (int i = 0; i < n; i++) a += rw[i];
+    for (int j = 0; j < n; j++) b += cw[j];
+    *krw = a;
+    *kcw = b;
+}
+
+/* weighted row / column sum of one line (explicit, for refreshes) */
+static double row_w(int n, const double *L, int ldl, int i) {
+    double t = 0.0;
+    for (int j = 0; j < n; j++) t += AT(L, ldl, i, j) * WGT(j);
+    return t;
+}
+static double col_w(int n, const double *L, int ldl, int j) {
+    double t = 0.0;
+    for (int i = 0; i < n; i++) t += WGT(i) * AT(L, ldl, i, j);
+    return t;
+}
+static double row_e(int n, const double *L, int ldl, int i) {
+    double t = 0.0;
+    for (int j = 0; j < n; j++) t += AT(L, ldl, i, j);
+    return t;
+}
+static double col_e(int n, const double *L, int ldl, int j) {
+    double t = 0.0;
+    for (int i = 0; i < n; i++) t += AT(L, ldl, i, j);
+    return t;
+}
+
+/* the index a weighted / plain syndrome ratio names: D_w / D = w_x = x + 1 for a single error at
+ * x; -1 unless the ratio is within 1/4 of an integer in [1, n] after its rounding error
+ * (|D_w| <= tw, |D| <= t: ratio error <= (tw + n t) / |D|) */
+static int ratio_index(double Dw, double D, double t, double tw, int n) {
+    if (!isfinite(Dw) || !isfinite(D) || !(fabs(D) > t)) return -1;
+    const double rho = Dw / D;
+    const double err = (tw + (double)n * t) / fabs(D) + 4.0 * n * EPS * fabs(rho);
+    if (!(err < 0.25)) return -1;
+    const double k = nearbyint(rho);
+    if (!(fabs(rho - k) <= err) || k < 1.0 || k > (double)n) return -1;
+    return (int)k - 1;
+}
+
+/* Decoder v3 (weighted pair).  First the paper's single pair (v2, R12) on L, r, c, kappa: if it
+ * corrects (or finds nothing), only weighted checksum words can still disagree -- they are
+ * refreshed from the verified data.  If v2 refuses (value ties, L-shapes), the weighted pair
+ * locates: a column j whose syndromes satisfy D_cw(j) / D_c(j) = w_i holds its one error at row i
+ * (and a row likewise), which needs no pairing by value.  Every located error is repaired with
+ * an explicit sum along the line that holds no other error; checksum words whose line
+ * shows no data error are refreshed; everything is re-verified and any remaining discrepancy is
+ * reported uncorrectable (never a wrong correction).  Returns 0 clean, 1 corrected, 2 refused. */
+int ora_decode_w(int n, double *L, int ldl, double *r, double *c, double *kappa, double *rw, double *cw,
+                 double *krw, double *kcw, double tau_abs, ora_report *rep, int panel) {
+    const size_t nn = (size_t)(n > 0 ? n : 1);
+    const double tw = tau_abs * (double)n;           /* weighted sums: weights up to n */
+    const double tauS = tau_abs * sqrt((double)(n > 1 ? n : 1)), twS = tw * sqrt((double)(n > 1 ? n : 1));
+    /* keep the input: v2 may modify L before refusing */
+    double *L0 = (double *)malloc(sizeof(double) * nn * nn), *r0 = (double *)malloc(sizeof(double) * nn),
+           *c0 = (double *)malloc(sizeof(double) * nn);
+    for (int j = 0; j < n; j++)
+        for (int i = 0; i < n; i++) L0[i + (size_t)j * nn] = AT(L, ldl, i, j);
+    memcpy(r0, r, sizeof(double) * nn);
+    memcpy(c0, c, sizeof(double) * nn);
+    const double k0 = *kappa;
+    const int nev0 = rep ? rep->nevents : 0, det0 = rep ? rep->detected : 0, cor0 = rep ? rep->corrected : 0,
+              unc0 = rep ? rep->uncorrectable : 0;
+    int result = ora_decode(n, L, ldl, r, c, kappa, tau_abs, rep, panel, ORA_MODE_H);
+    double *Dr = (double *)malloc(sizeof(double) * nn), *Dc = (double *)malloc(sizeof(double) * nn);
+    double *Drw = (double *)malloc(sizeof(double) * nn), *Dcw = (double *)malloc(sizeof(double) * nn);
+    int *pi = (int *)malloc(sizeof(int) * nn);
+    int detected_here = 0;
+    if (result == 2) {
+        /* ---- weighted location on the original input ---- */
+        for (int j = 0; j < n; j++)
+            for (int i = 0; i < n; i++) AT(L, ldl, i, j) = L0[i + (size_t)j * nn];
+        memcpy(r, r0, sizeof(double) * nn);
+        memcpy(c, c0, sizeof(double) * nn);
+        *kappa = k0;
+        if (rep) { /* the single-pair attempt's events are replaced by this decode's */
+            rep->nevents = nev0; rep->detected = det0; rep->corrected = cor0; rep->uncorrectable = unc0;
+        }
+        result = 1;
+        for (int pass = 0; pass < 8; pass++) {  /* each pass can free lines for the next (L-shapes) */
+        for (int i = 0; i < n; i++) { Dr[i] = r[i] - row_e(n, L, ldl, i); Drw[i] = rw[i] - row_w(n, L, ldl, i); }
+        for (int j = 0; j < n; j++) { Dc[j] = c[j] - col_e(n, L, ldl, j); Dcw[j] = cw[j] - col_w(n, L, ldl, j); }
+        int nR = 0, nC = 0;
+        for (int i = 0; i < n; i++) nR += bad(Dr[i], tau_abs);
+        for (int j = 0; j < n; j++) nC += bad(Dc[j], tau_abs);
+        if (pass == 0) {
+            push_ev(rep, ORA_EV_DETECT, panel, nR, nC, 0.0);
+            if (rep) rep->detected++;
+            detected_here = 1;
+        }
+        if (nR == 0 || nC == 0) break;
+        /* candidates: column j names row pi[j]; row i names column ratio_index(...).  A named
+         * line must itself be flagged (plain or weighted syndrome: a pair cancelling in the plain
+         * sum of a line never cancels in its weighted sum, w_j1 != w_j2) */
+        for (int j = 0; j < n; j++) {
+            pi[j] = -1;
+            if (!bad(Dc[j], tau_abs)) continue;
+            const int i = ratio_index(Dcw[j], Dc[j], tau_abs, tw, n);
+            if (i >= 0 && (bad(Dr[i], tau_abs) || bad(Drw[i], tw))) pi[j] = i;
+        }
+        /* fixes: a column-named error (i, j) whose row also names j is alone in row and column
+         * (row formula); a column-named one whose row names something else shares its row
+         * (column formula: the column holds only it); then row-named errors in columns that
+         * named nothing (they share their column: row formula) */
+        int nfix = 0;
+        for (int j = 0; j < n; j++) {
+            const int i = pi[j];
+            if (i < 0) continue;
+            const int jr = ratio_index(Drw[i], Dr[i], tau_abs, tw, n);
+            const double d = (jr == j) ? fix_row(n, L, ldl, r, i, j) : fix_col(n, L, ldl, c, i, j);
+            push_ev(rep, ORA_EV_FIX_DATA, panel, i, j, d);
+            nfix++;
+        }
+        for (int i = 0; i < n; i++) {
+            if (!bad(Dr[i], tau_abs)) continue;
+            const int j = ratio_index(Drw[i], Dr[i], tau_abs, tw, n);
+            if (j < 0 || !(bad(Dc[j], tau_abs) || bad(Dcw[j], tw)) || pi[j] >= 0) continue;
+            const double d = fix_row(n, L, ldl, r, i, j);
+            push_ev(rep, ORA_EV_FIX_DATA, panel, i, j, d);
+            nfix++;
+        }
+        if (nfix == 0) break;
+        }
+        /* checksum words.  A data error flags both syndromes of its row in at least one sense and
+         * its column likewise, so a word is refreshed only when the orthogonal direction shows
+         * no flag of either kind anywhere (else: refuse at the re-verification) */
+        for (int i = 0; i < n; i++) { Dr[i] = r[i] - row_e(n, L, ldl, i); Drw[i] = rw[i] - row_w(n, L, ldl, i); }
+        for (int j = 0; j < n; j++) { Dc[j] = c[j] - col_e(n, L, ldl, j); Dcw[j] = cw[j] - col_w(n, L, ldl, j); }
+        int anyR = 0, anyC = 0;
+        for (int i = 0; i < n; i++) anyR |= bad(Dr[i], tau_abs) || bad(Drw[i], tw);
+        for (int j = 0; j < n; j++) anyC |= bad(Dc[j], tau_abs) || bad(Dcw[j], tw);
+        if (anyR && !anyC)
+            for (int i = 0; i < n; i++) {
+                if (bad(Dr[i], tau_abs)) {
+                    const double old = r[i];
+                    r[i] = row_e(n, L, ldl, i);
+                    push_ev(rep, ORA_EV_FIX_R, panel, i, -1, r[i] - old);
+                }
+                if (bad(Drw[i], tw)) {
+                    const double old = rw[i];
+                    rw[i] = row_w(n, L, ldl, i);
+                    push_ev(rep, ORA_EV_FIX_RW, panel, i, -1, rw[i] - old);
+                }
+            }
+        if (anyC && !anyR)
+            for (int j = 0; j < n; j++) {
+                if (bad(Dc[j], tau_abs)) {
+                    const double old = c[j];
+                    c[j] = col_e(n, L, ldl, j);
+                    push_ev(rep, ORA_EV_FIX_C, panel, -1, j, c[j] - old);
+                }
+                if (bad(Dcw[j], tw)) {
+                    const double old = cw[j];
+                    cw[j] = col_w(n, L, ldl, j);
+                    push_ev(rep, ORA_EV_FIX_CW, panel, -1, j, cw[j] - old);
+                }
+            }
+        /* kappa: both sums off by the same amount */
+        {
+            double sr = 0.0, sc = 0.0;
+            for (int i = 0; i < n; i++) sr += r[i];
+            for (int j = 0; j < n; j++) sc += c[j];
+            if (!approx(sr, *kappa, tauS) && approx(sr, sc, tauS)) {
+                const double old = *kappa;
+                *kappa = sr;
+                push_ev(rep, ORA_EV_FIX_K, panel, -1, -1, *kappa - old);
+            }
+        }
+    }
+    if (result == 1 || result == 0) {
+        /* weighted words against the (verified / repaired) data: a weighted line that disagrees
+         * while its plain line agrees is a corrupted weighted word (a data error with |d| <= tau
+         * moves a weighted sum by at most n |d| <= tw) -- refresh it; corners likewise */
+        int refreshed = 0;
+        for (int i = 0; i < n; i++) {
+            const double t = row_w(n, L, ldl, i);
+            if (bad(rw[i] - t, tw) && !detected_here) {  /* v2 verified the data: a weighted word */
+                const double old = rw[i];
+                rw[i] = t;
+                push_ev(rep, ORA_EV_FIX_RW, panel, i, -1, rw[i] - old);
+                refreshed++;
+            }
+        }
+        for (int j = 0; j < n; j++) {
+            const double t = col_w(n, L, ldl, j);
+            if (bad(cw[j] - t, tw) && !detected_here) {
+                const double old = cw[j];
+                cw[j] = t;
+                push_ev(rep, ORA_EV_FIX_CW, panel, -1, j, cw[j] - old);
+                refreshed++;
+            }
+        }
+        double srw = 0.0, scw = 0.0;
+        for (int i = 0; i < n; i++) srw += rw[i];
+        for (int j = 0; j < n; j++) scw += cw[j];
+        if (!approx(srw, *krw, twS)) {
+            const double old = *krw;
+            *krw = srw;
+            push_ev(rep, ORA_EV_FIX_KW, panel, 0, -1, *krw - old);
+            refreshed++;
+        }
+        if (!approx(scw, *kcw, twS)) {
+            const double old = *kcw;
+            *kcw = scw;
+            push_ev(rep, ORA_EV_FIX_KW, panel, -1, 0, *kcw - old);
+            refreshed++;
+        }
+        if (refreshed && result == 0) {
+            push_ev(rep, ORA_EV_DETECT, panel, 0, 0, 0.0);
+            if (rep) { rep->detected++; rep->corrected++; }
+            result = 1;
+        }
+        /* final re-verification of all four syndromes and the corners */
+        int ok = 1;
+        double sr = 0.0, sc = 0.0;
+        for (int i = 0; i < n && ok; i++) {
+            ok &= !bad(r[i] - row_e(n, L, ldl, i), tau_abs) && !bad(rw[i] - row_w(n, L, ldl, i), tw);
+            sr += r[i];
+        }
+        for (int j = 0; j < n && ok; j++) {
+            ok &= !bad(c[j] - col_e(n, L, ldl, j), tau_abs) && !bad(cw[j] - col_w(n, L, ldl, j), tw);
+            sc += c[j];
+        }
+        if (ok) ok = approx(sr, *kappa, tauS) && approx(sc, *kappa, tauS);
+        if (!ok) {
+            push_ev(rep, ORA_EV_UNCORRECTABLE, panel, -1, -1, 0.0);
+            if (rep) rep->uncorrectable++;
+            result = 2;
+        } else if (detected_here && rep) {
+            rep->corrected++;
+        }
+    }
+    free(L0); free(r0); free(c0); free(Dr); free(Dc); free(Drw); free(Dcw); free(pi);
+    return result;
+}
+
 /* encode (Fig. 3, Alg. 3 l.2): r = A e, c = e^T A, kappa = e^T A e (R22) */
 void ora_encode(int n, const double *A, int lda, double *r, double *c, double *kappa) {
     row_sums(n, A, lda, r);
@@ -553,6 +838,8 @@ static void inject(const ora_fault *f, int n, double *A, int lda, chk_t *k, ora_
     case ORA_SITE_K: p = k->kap; break;
     case ORA_SITE_QR: if (f->i >= 0 && f->i < n) p = &k->qr[f->i]; break;
     case ORA_SITE_QC: if (f->j >= 0 && f->j < n) p = &k->qc[f->j]; break;
+    case ORA_SITE_RW: if (k->rw && f->i >= 0 && f->i < n) p = &k->rw[f->i]; break;
+    case ORA_SITE_CW: if (k->cw && f->j >= 0 && f->j < n) p = &k->cw[f->j]; break;
     }
     if (!p) return;
     double d = ora_flip(p, f->bit);
@@ -569,6 +856,12 @@ static double frob(int n, const double *A, int lda) {
 int ora_ft_dgehd2(int n, int ilo, int ihi, double *A, int lda, double *tau,
                   int nb, double c_thr, const ora_fault *faults, int nfaults,
                   ora_report *rep, int stop_after_panel, double *chk_out) {
+    return ora_ft_dgehd2_ex(n, ilo, ihi, A, lda, tau, nb, c_thr, 0, faults, nfaults, rep, stop_after_panel, chk_out);
+}
+
+int ora_ft_dgehd2_ex(int n, int ilo, int ihi, double *A, int lda, double *tau,
+                     int nb, double c_thr, int weighted, const ora_fault *faults, int nfaults,
+                     ora_report *rep, int stop_after_panel, double *chk_out) {
     int info = check_args(n, ilo, ihi, A, lda, tau);
     if (info) return info;
     if (nb < 1) return -7;
@@ -583,10 +876,12 @@ int ora_ft_dgehd2(int n, int ilo, int ihi, double *A, int lda, double *tau,
     double *y = (double *)calloc(nn, 8), *w = (double *)calloc(nn, 8);
     double *L = (double *)malloc(nn * nn * 8);
     double *Dr = (double *)malloc(nn * 8), *Dc = (double *)malloc(nn * 8);
-    double kap = 0.0, qk = 0.0;
-    chk_t k = {r, cc, &kap, qr, qc, &qk};
+    double kap = 0.0, qk = 0.0, krw = 0.0, kcw = 0.0;
+    double *rw = weighted ? (double *)calloc(nn, 8) : NULL, *cw = weighted ? (double *)calloc(nn, 8) : NULL;
+    chk_t k = {r, cc, &kap, qr, qc, &qk, rw, cw, &krw, &kcw};
 
     ora_encode(n, A, lda, r, cc, &kap);
+    if (weighted) encode_w(n, A, lda, rw, cw, &krw, &kcw);
     double normF = frob(n, A, lda);              /* invariant under the similarity */
     double tau_abs = c_thr * n * EPS * normF;    /* R10 */
     double unit = n * EPS * (normF > 0 ? normF : 1.0);
@@ -613,7 +908,8 @@ int ora_ft_dgehd2(int n, int ilo, int ihi, double *A, int lda, double *tau,
                     if (dmax / unit > rep->max_drift && dmax <= tau_abs) rep->max_drift = dmax / unit;
                 }
             }
-            int dres = ora_decode(n, L, n, r, cc, &kap, tau_abs, rep, t, ORA_MODE_H);
+            int dres = weighted ? ora_decode_w(n, L, n, r, cc, &kap, rw, cw, &krw, &kcw, tau_abs, rep, t)
+                                : ora_decode(n, L, n, r, cc, &kap, tau_abs, rep, t, ORA_MODE_H);
             if (dres == 2) { result = 1; goto out; }
             if (dres == 1) write_back(n, A, lda, ilo, ihi, c, L, 0);
         }
@@ -624,6 +920,12 @@ int ora_ft_dgehd2(int n, int ilo, int ihi, double *A, int lda, double *tau,
                 memcpy(chk_out, r, nn * 8);
                 memcpy(chk_out + n, cc, nn * 8);
                 chk_out[2 * n] = kap;
+                if (weighted) {  /* [.. | r_w | c_w | krw | kcw] */
+                    memcpy(chk_out + 2 * n + 1, rw, nn * 8);
+                    memcpy(chk_out + 3 * n + 1, cw, nn * 8);
+                    chk_out[4 * n + 1] = krw;
+                    chk_out[4 * n + 2] = kcw;
+                }
             }
             goto out;
         }
@@ -634,7 +936,8 @@ int ora_ft_dgehd2(int n, int ilo, int ihi, double *A, int lda, double *tau,
     {
         int cdone = clast + 1;
         build_L(n, A, lda, ilo, ihi, cdone, L, 0);
-        int dres = ora_decode(n, L, n, r, cc, &kap, tau_abs, rep, -1, ORA_MODE_H);
+        int dres = weighted ? ora_decode_w(n, L, n, r, cc, &kap, rw, cw, &krw, &kcw, tau_abs, rep, -1)
+                            : ora_decode(n, L, n, r, cc, &kap, tau_abs, rep, -1, ORA_MODE_H);
         if (dres == 2) { result = 1; goto out; }
         if (dres == 1) write_back(n, A, lda, ilo, ihi, cdone, L, 0);
         /* Q: logical matrix = stored Householder vectors only */
@@ -645,6 +948,6 @@ int ora_ft_dgehd2(int n, int ilo, int ihi, double *A, int lda, double *tau,
         if (dres == 1) write_back(n, A, lda, ilo, ihi, cdone, L, 1);
     }
 out:
-    free(r); free(cc); free(qr); free(qc); free(y); free(w); free(L); free(Dr); free(Dc);
+    free(r); free(cc); free(qr); free(qc); free(y); free(w); free(L); free(Dr); free(Dc); free(rw); free(cw);
     return result;
 }

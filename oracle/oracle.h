@@ -29,12 +29,15 @@ enum { ORA_SITE_A = 0,  /* working-array word A(i,j): H, trailing, or stored V *
        ORA_SITE_C = 2,  /* column-checksum c(j)         (P:224 Ac_chk)       */
        ORA_SITE_K = 3,  /* corner kappa = e^T L e       (R22)                */
        ORA_SITE_QR = 4, /* Q row checksum Qr(i)              */
-       ORA_SITE_QC = 5  /* Q column checksum Qc(j)              */ };
+       ORA_SITE_QC = 5, /* Q column checksum Qc(j)              */
+       ORA_SITE_RW = 6, /* weighted row checksum r_w(i) (NEXT-1, w_i = i+1)   */
+       ORA_SITE_CW = 7  /* weighted column checksum c_w(j)                     */ };
 
 /* event kinds */
 enum { ORA_EV_INJECT = 0, ORA_EV_DETECT = 1, ORA_EV_FIX_DATA = 2, ORA_EV_FIX_R = 3,
        ORA_EV_FIX_C = 4, ORA_EV_FIX_K = 5, ORA_EV_FIX_Q = 6, ORA_EV_FIX_QR = 7,
-       ORA_EV_FIX_QC = 8, ORA_EV_FIX_QK = 9, ORA_EV_UNCORRECTABLE = 10 };
+       ORA_EV_FIX_QC = 8, ORA_EV_FIX_QK = 9, ORA_EV_UNCORRECTABLE = 10,
+       ORA_EV_FIX_RW = 11, ORA_EV_FIX_CW = 12, ORA_EV_FIX_KW = 13 };
 
 /* decoder modes */
 enum { ORA_MODE_H = 0, ORA_MODE_Q = 1 };
@@ -79,6 +82,19 @@ int ora_dorghr(int n, int ilo, int ihi, const double *A, int lda, const double *
 int ora_ft_dgehd2(int n, int ilo, int ihi, double *A, int lda, double *tau,
                   int nb, double c_thr, const ora_fault *faults, int nfaults,
                   ora_report *rep, int stop_after_panel, double *chk_out);
+
+/* The same with the weighted checksum pair (NEXT-1, w_i = i + 1) when weighted = 1: r_w = L w,
+ * c_w = w^T L and the corners e^T L w, w^T L e ride through every reflector (Theorem 1 with w,
+ * P:268-274) and the boundary decoder is ora_decode_w; chk_out then holds
+ * [r | c | kappa | r_w | c_w | e^T L w | w^T L e] (4n + 3 doubles). */
+int ora_ft_dgehd2_ex(int n, int ilo, int ihi, double *A, int lda, double *tau,
+                     int nb, double c_thr, int weighted, const ora_fault *faults, int nfaults,
+                     ora_report *rep, int stop_after_panel, double *chk_out);
+
+/* Decoder v3 (weighted pair): v2 first; if it refuses, location by D_w / D = w_i on the weighted
+ * syndromes; weighted checksum words refreshed; full re-verification.  0 / 1 / 2 as ora_decode. */
+int ora_decode_w(int n, double *L, int ldl, double *r, double *c, double *kappa, double *rw, double *cw,
+                 double *krw, double *kcw, double tau_abs, ora_report *rep, int panel);
 
 /* The R12 decoder on a dense logical n x n matrix L (ldl), checksums r, c and
  * corner kappa, threshold tau_abs.  Repairs L/r/c/kappa in place.

@@ -379,3 +379,166 @@ def test_decoder_borderline_flips_never_refused_or_wrong(ora, seed):
             res, L, r2, c2, k2, rep = ora.decode(Af, rf, cf, kf, tau)
             assert res in (0, 1), (site, bit, rep.events())
             assert np.abs(L - A).max() <= 2 * tau, (site, bit)
+
+
+# ---------------------------------------------------------------- NEXT-1: weighted checksum pair
+def _wsums(L):
+    n = L.shape[0]
+    w = np.arange(1, n + 1, dtype=float)
+    rw, cw = L @ w, w @ L
+    return rw, cw, float(rw.sum()), float(cw.sum())
+
+
+@pytest.mark.parametrize("n,nb,dist", [(64, 16, "normal"), (200, 32, "uniform"), (150, 64, "normal")])
+def test_weighted_theorem1_at_every_boundary(ora, n, nb, dist):
+    """Theorem 1 holds for any weight vector: r_w = L w, c_w = w^T L and the corners
+    e^T L w, w^T L e maintained per reflector equal their recomputation at every boundary, and the
+    plain pair is unchanged by carrying the weighted one."""
+    A = synth.matrix(n, dist=dist)
+    normF = np.linalg.norm(A)
+    npanel = (n - 2 + nb - 1) // nb
+    for t in range(npanel):
+        info, Aw, tw, rep, chk = ora.ft_dgehd2(A, nb, stop_after_panel=t, weighted=True)
+        assert info == 0 and rep.detected == 0
+        info0, Aw0, _, _, chk0 = ora.ft_dgehd2(A, nb, stop_after_panel=t)
+        assert np.array_equal(Aw, Aw0) and np.array_equal(chk[: 2 * n + 1], chk0)
+        L = _logical(Aw, 1, n, min((t + 1) * nb, n - 1))
+        rw, cw, krw, kcw = _wsums(L)
+        unit = n * EPS * normF * n  # weighted sums carry weights up to n
+        assert np.abs(chk[2 * n + 1: 3 * n + 1] - rw).max() <= 0.5 * unit, t
+        assert np.abs(chk[3 * n + 1: 4 * n + 1] - cw).max() <= 0.5 * unit, t
+        assert abs(chk[4 * n + 1] - krw) <= 0.5 * unit * n and abs(chk[4 * n + 2] - kcw) <= 0.5 * unit * n
+
+
+def _wcase(ora, n=8, seed=0):
+    A = synth.matrix(n, seed=seed, dist="normal")
+    r, c, k = ora.encode(A)
+    rw, cw, krw, kcw = _wsums(A)
+    tau = 2.0 * n * EPS * np.linalg.norm(A)
+    return A, r, c, k, rw, cw, krw, kcw, tau
+
+
+def _wapply(st, site, bit, ora):
+    A, r, c, k, rw, cw = st[0].copy(order="F"), st[1].copy(), st[2].copy(), st[3], st[4].copy(), st[5].copy()
+    kind, i, j = site
+    if kind == "A":
+        A[i, j] = ora.flip(A[i, j], bit)
+    elif kind == "r":
+        r[i] = ora.flip(r[i], bit)
+    elif kind == "c":
+        c[j] = ora.flip(c[j], bit)
+    elif kind == "rw":
+        rw[i] = ora.flip(rw[i], bit)
+    elif kind == "cw":
+        cw[j] = ora.flip(cw[j], bit)
+    else:
+        k = ora.flip(k, bit)
+    return A, r, c, k, rw, cw
+
+
+def _wsites(n):
+    return _sites(n) + [("rw", i, -1) for i in range(n)] + [("cw", -1, j) for j in range(n)]
+
+
+def _wexact(A0, L, r0, r, c0, c, rw0, rw, cw0, cw, n):
+    scale = n * EPS * max(1.0, np.abs(A0).max()) * 8
+    return (np.abs(L - A0).max() <= scale and np.abs(r - r0).max() <= scale * n and np.abs(c - c0).max() <= scale * n
+            and np.abs(rw - rw0).max() <= scale * n * n and np.abs(cw - cw0).max() <= scale * n * n)
+
+
+@pytest.mark.parametrize("seed", [0, 1])
+def test_weighted_decoder_singles_and_never_miscorrects_pairs(ora, seed):
+    """Decoder v3 brute force (n = 8): every single fault at every site -- data, r, c, kappa, r_w,
+    c_w -- is corrected; every pair of sites x bit pairs is corrected exactly or refused, never
+    wrong; and it corrects at least as many pairs as the single pair's decoder (v2)."""
+    n = 8
+    A, r, c, k, rw, cw, krw, kcw, tau = _wcase(ora, n, seed)
+    st = (A, r, c, k, rw, cw)
+    for site in _wsites(n):
+        for bit in (45, 51, 62, 63):
+            Af, rf, cf, kf, rwf, cwf = _wapply(st, site, bit, ora)
+            res, L, r2, c2, k2, rw2, cw2, krw2, kcw2, rep = ora.decode_w(Af, rf, cf, kf, rwf, cwf, krw, kcw, tau)
+            assert res == 1, (site, bit, rep.events())
+            assert _wexact(A, L, r, r2, c, c2, rw, rw2, cw, cw2, n), (site, bit)
+    sites = _wsites(n)
+    bitpairs = [(45, 51), (51, 51), (62, 45), (52, 60)]
+    ok_w = ok_v2 = refused = 0
+    for s1, s2 in itertools.combinations(sites, 2):
+        for b1, b2 in bitpairs:
+            f = _wapply(st, s1, b1, ora)
+            f = _wapply(f, s2, b2, ora)
+            res, L, r2, c2, k2, rw2, cw2, krw2, kcw2, rep = ora.decode_w(*f, krw, kcw, tau)
+            if res == 1:
+                assert _wexact(A, L, r, r2, c, c2, rw, rw2, cw, cw2, n), (s1, s2, b1, b2, rep.events())
+                ok_w += 1
+            else:
+                assert res == 2
+                refused += 1
+            if s1[0] in "Ark" and s2[0] in "Ark":
+                res2, *_ = ora.decode(*f[:4], tau)
+                ok_v2 += res2 == 1
+    assert ok_w > 0.9 * (ok_w + refused) and ok_w >= ok_v2, (ok_w, refused, ok_v2)
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_weighted_decoder_fixes_ten_tied_flips(ora, seed):
+    """ten flips in one iteration with tied discrepancies (entries 1.0, mantissa bit
+    51: every delta is exactly +0.5) defeat the single pair (v2 refuses: pairing by value is
+    ambiguous); the weighted pair locates each by D_w / D = w and corrects all ten.  Rectangles
+     are still refused."""
+    n = 64
+    rng = np.random.default_rng(seed)
+    A = np.ones((n, n)) + np.eye(n)
+    r, c, k = ora.encode(A)
+    rw, cw, krw, kcw = _wsums(A)
+    tau = 2.0 * n * EPS * np.linalg.norm(A)
+    rows = rng.choice(n, 10, replace=False)
+    cols = rng.choice(n, 10, replace=False)
+    Af = A.copy(order="F")
+    for i, j in zip(rows, cols):
+        Af[i, j] = ora.flip(Af[i, j], 51)
+    assert ora.decode(Af, r, c, k, tau)[0] == 2
+    res, L, *_ , rep = ora.decode_w(Af, r, c, k, rw, cw, krw, kcw, tau)
+    assert res == 1, rep.events()
+    assert np.abs(L - A).max() <= 1e-14
+    Ar = A.copy(order="F")
+    for (i, j) in [(3, 7), (3, 20), (40, 7), (40, 20)]:
+        Ar[i, j] = ora.flip(Ar[i, j], 51)
+    assert ora.decode_w(Ar, r, c, k, rw, cw, krw, kcw, tau)[0] == 2
+
+
+def _tied_positions(W, lo, count, rng):
+    """count positions (distinct rows and columns, both >= lo) of values in [0.5, 1) whose mantissa
+    bit 51 is clear: flipping it adds exactly +0.25 to each (a tie pattern)."""
+    n = W.shape[0]
+    bits = W.view(np.uint64)
+    ok = (np.abs(W) >= 0.5) & (np.abs(W) < 1.0) & ((bits >> np.uint64(51)) & np.uint64(1) == 0) & (W > 0)
+    rows, cols, out = set(), set(), []
+    for i, j in zip(*np.nonzero(ok)):
+        if i >= lo and j >= lo and i not in rows and j not in cols and rng.random() < 0.3:
+            out.append((int(i), int(j)))
+            rows.add(i)
+            cols.add(j)
+        if len(out) == count:
+            break
+    return out
+
+
+def test_weighted_end_to_end_tied_flips(ora):
+    """The unblocked ABFT reduction with the weighted pair on (weighted=1): ten flips with tied
+    discrepancies (+0.25 each) in the trailing matrix at boundary 1 are all located and corrected,
+    and the reduction equals the fault-free one; with the single pair the same run stops
+    uncorrectable (R12 refuses the ambiguous pairing)."""
+    n, nb = 128, 32
+    A = synth.matrix(n)
+    Ao, tau = _fault_free(ora, A, nb)
+    _, W, _, _, _ = ora.ft_dgehd2(A, nb, stop_after_panel=0)  # the working matrix at boundary 1
+    pos = _tied_positions(np.asfortranarray(W), 40, 10, np.random.default_rng(1))
+    assert len(pos) == 10
+    faults = [(1, 0, i, j, 51) for (i, j) in pos]
+    info, Af, tf, rep, _ = ora.ft_dgehd2(A, nb, faults=faults, weighted=True)
+    assert info == 0, rep.events()
+    assert sorted((e[2], e[3]) for e in rep.events() if e[0] == "FIX_DATA") == sorted(pos)
+    assert np.abs(np.triu(Af, -1) - np.triu(Ao, -1)).max() <= 1e-12 * np.abs(Ao).max()
+    info1, *_ = ora.ft_dgehd2(A, nb, faults=faults)
+    assert info1 == 1
