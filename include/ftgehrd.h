@@ -58,7 +58,9 @@ enum { FT_PHASE_BEFORE_PANEL = 0, FT_PHASE_AFTER_PANEL = 1, FT_PHASE_AFTER_RIGHT
  *   V   panel workspace V(i,j)   (the copy the updates read; R15)
  *   T   block-reflector factor T(i,j), 0 <= i, j < 64 (the nb x nb upper triangle is what the
  *       left update W' = T^T V^T A reads; R15 extended to T) */
-enum { FT_SITE_A = 0, FT_SITE_R = 1, FT_SITE_C = 2, FT_SITE_K = 3, FT_SITE_Y = 4, FT_SITE_V = 5, FT_SITE_T = 6 };
+/*   RW, CW  weighted checksum words r_w(i), c_w(j) (opts.weighted = 1, NEXT-1) */
+enum { FT_SITE_A = 0, FT_SITE_R = 1, FT_SITE_C = 2, FT_SITE_K = 3, FT_SITE_Y = 4, FT_SITE_V = 5, FT_SITE_T = 6,
+       FT_SITE_RW = 7, FT_SITE_CW = 8 };
 
 typedef struct {
     int32_t panel;  /* iteration t >= 0 (ignored for AT_END) */
@@ -70,7 +72,8 @@ typedef struct {
 
 enum { FT_EV_INJECT = 0, FT_EV_DETECT = 1, FT_EV_FIX_DATA = 2, FT_EV_FIX_R = 3, FT_EV_FIX_C = 4,
        FT_EV_FIX_K = 5, FT_EV_FIX_Q = 6, FT_EV_FIX_QR = 7, FT_EV_FIX_QC = 8, FT_EV_FIX_QK = 9,
-       FT_EV_UNCORRECTABLE = 10, FT_EV_ROLLBACK = 11, FT_EV_PANEL_REDO = 12 };
+       FT_EV_UNCORRECTABLE = 10, FT_EV_ROLLBACK = 11, FT_EV_PANEL_REDO = 12,
+       FT_EV_FIX_RW = 13, FT_EV_FIX_CW = 14, FT_EV_FIX_KW = 15 /* weighted pair words (NEXT-1) */ };
 
 typedef struct {
     int32_t kind, panel;  /* FT_EV_*, iteration (-1 = final verification) */
@@ -96,7 +99,11 @@ enum { FT_POLICY_EAGER = 0, FT_POLICY_PAPER = 1 };
 typedef struct {
     int32_t nb;          /* panel width; 0 -> 32 if n < 4096 else 64 (R4); max 64      */
     int32_t abft;        /* 0 = fault-prone baseline (no checksums), 1 = protected     */
-    int32_t weighted;    /* reserved (weighted checksum pair, NEXT-1); must be 0       */
+    int32_t weighted;    /* 1 (with abft = 1): + the weighted checksum pair r_w = L w, c_w = w^T L,
+                            w_i = i + 1 (NEXT-1), riding as row / column n+1 through every update;
+                            the decoder then locates tied and L-shaped multiple errors;
+                            the stop hook's dchk_out holds 4n+3 doubles
+                            [r | c | kappa | r_w | c_w | e^T L w | w^T L e]                     */
     int32_t policy;      /* FT_POLICY_EAGER (default) or FT_POLICY_PAPER (R11)         */
     double c_thr;        /* threshold constant; 0 -> 2.0; tau_abs = c_thr*n*eps*||A||_F (R10) */
     const ft_fault *faults;   /* host array, may be NULL                                 */

@@ -67,12 +67,19 @@ __device__ __forceinline__ bool in_v(int i, int j, int ilo, int ihi, int cdone) 
 }
 __global__ void __launch_bounds__(LS_RB) k_rowsum_part(const double *__restrict__ Aw, int64_t ldw, int n, int nchunk,
                                                        int mode, int ilo, int ihi, int cdone, double *rowpart,
-                                                       double *sq_part) {
+                                                       double *sq_part, int wgt = 0) {
     const int i = blockIdx.x * LS_RB + threadIdx.x;
     const int cw = (n + nchunk - 1) / nchunk;
     const int j0 = blockIdx.y * cw, j1 = min(n, j0 + cw);
     double s = 0.0, q = 0.0;
-    if (i < n) {
+    if (i < n && wgt) {  // weighted pair (NEXT-1): sum_j w_j A(i, j), w_j = j + 1
+        const double *a = Aw + i;
+        for (int j = j0; j < j1; j++) {
+            const bool v = mode >= 0 && in_v(i, j, ilo, ihi, cdone);
+            if (mode < 0 || (mode == 0 ? !v : v)) s += a[(int64_t)j * ldw] * (double)(j + 1);
+        }
+        rowpart[(int64_t)blockIdx.y * n + i] = s;
+    } else if (i < n) {
         const double *a = Aw + i;
         if (mode < 0) {
 #pragma unroll 8
@@ -279,30 +286,44 @@ cudaError_t ft_decide(const double *Y, const double *V, const double *T, int64_t
 //   Fr(i) += sum_{col in [k,e), i <= col+1} A(i,col)   for i <= e (columns frozen now)
 // ---------------------------------------------------------------------------
 __global__ void k_endcheck(double *Aw, int64_t ldw, int n, int ihi, int k, int ib, int panel, int policy,
-                           double *Fr, FtCtl *ctl) {
+                           double *Fr, FtCtl *ctl, int weighted) {
     if (ctl->halt) return;
-    __shared__ double ws[2][32];
+    __shared__ double ws[4][32];
     __shared__ int last;
-    double sr = 0.0, sc = 0.0;
+    double sr = 0.0, sc = 0.0, srw = 0.0, scw = 0.0;
     for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
         sr += Aw[i + (int64_t)n * ldw];
         sc += Aw[n + (int64_t)i * ldw];
+        if (weighted) {  // the weighted pair's sums (NEXT-1): sum r_w = e^T L w, sum c_w = w^T L e
+            srw += Aw[i + (int64_t)(n + 1) * ldw];
+            scw += Aw[n + 1 + (int64_t)i * ldw];
+        }
     }
     sr = warp_sum(sr);
     sc = warp_sum(sc);
+    srw = warp_sum(srw);
+    scw = warp_sum(scw);
     if ((threadIdx.x & 31) == 0) {
         ws[0][threadIdx.x >> 5] = sr;
         ws[1][threadIdx.x >> 5] = sc;
+        ws[2][threadIdx.x >> 5] = srw;
+        ws[3][threadIdx.x >> 5] = scw;
     }
     __syncthreads();
     if (threadIdx.x == 0) {
-        double a = 0.0, b = 0.0;
+        double a = 0.0, b = 0.0, c2 = 0.0, d2 = 0.0;
         for (int w = 0; w < (int)(blockDim.x >> 5); w++) {
             a += ws[0][w];
             b += ws[1][w];
+            c2 += ws[2][w];
+            d2 += ws[3][w];
         }
         atomicAdd(&ctl->sums[0], a);
         atomicAdd(&ctl->sums[1], b);
+        if (weighted) {
+            atomicAdd(&ctl->wsums[0], c2);
+            atomicAdd(&ctl->wsums[1], d2);
+        }
         __threadfence();
         last = (atomicAdd(&ctl->done_count, 1) == (int)gridDim.x - 1);
     }
@@ -319,6 +340,13 @@ __global__ void k_endcheck(double *Aw, int64_t ldw, int n, int ihi, int k, int i
             if (not_within(Sr - Sc, tauS)) reason |= 8;
         } else {
             if (not_within(Sr - kap, tauS) || not_within(Sc - kap, tauS)) reason |= 8;
+        }
+        if (weighted) {
+            const double Srw = atomicAdd(&ctl->wsums[0], 0.0), Scw = atomicAdd(&ctl->wsums[1], 0.0);
+            const double krw = Aw[n + (int64_t)(n + 1) * ldw], kcw = Aw[n + 1 + (int64_t)n * ldw];
+            if (not_within(Srw - krw, tauS * n) || not_within(Scw - kcw, tauS * n)) reason |= 64;
+            ctl->wsums[0] = 0.0;
+            ctl->wsums[1] = 0.0;
         }
         ctl->sums[0] = 0.0;
         ctl->sums[1] = 0.0;
@@ -343,11 +371,11 @@ __global__ void k_frozen_rows(const double *Aw, int64_t ldw, int n, int k, int e
     Fr[i] += s;
 }
 cudaError_t ft_endcheck(double *Aw, int64_t ldw, int n, int ihi, int k, int ib, int panel, int policy,
-                        double *Fr, FtCtl *ctl, cudaStream_t s) {
+                        double *Fr, FtCtl *ctl, cudaStream_t s, int weighted) {
     int nblk = (n + 1023) / 1024;
     if (nblk > 16) nblk = 16;
     g_ft_launches++;
-    k_endcheck<<<nblk, 1024, 0, s>>>(Aw, ldw, n, ihi, k, ib, panel, policy, Fr, ctl);
+    k_endcheck<<<nblk, 1024, 0, s>>>(Aw, ldw, n, ihi, k, ib, panel, policy, Fr, ctl, weighted);
     int e = k + ib;
     if (Fr) {
         g_ft_launches++;
@@ -383,14 +411,14 @@ cudaError_t ft_inject(double *addr, int fidx, int bit, FtCtl *ctl, cudaStream_t 
 // sums[0] = sum r, sums[1] = sum c.
 // ---------------------------------------------------------------------------
 __global__ void k_fv_cols(const double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdone, int mode,
-                          const double *c, int64_t cinc, double *Dc) {
+                          const double *c, int64_t cinc, double *Dc, int wgt = 0) {
     int j = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
     int lane = threadIdx.x & 31;
     if (j >= n) return;
     double s = 0.0;
     for (int i = lane; i < n; i += 32) {
         bool v = in_v(i, j, ilo, ihi, cdone);
-        if (mode == 0 ? !v : v) s += Aw[i + (int64_t)j * ldw];
+        if (mode == 0 ? !v : v) s += wgt ? (double)(i + 1) * Aw[i + (int64_t)j * ldw] : Aw[i + (int64_t)j * ldw];
     }
     s = warp_sum(s);
     if (lane == 0) Dc[j] = c[(int64_t)j * cinc] - s;
@@ -432,6 +460,179 @@ cudaError_t ft_full_verify(const double *Aw, int64_t ldw, int n, int ilo, int ih
     return cudaGetLastError();
 }
 
+// ---------------------------------------------------------------------------
+// Weighted checksum pair (NEXT-1; w_i = i + 1), opts.weighted = 1.  Column n+1 of the
+// working array is r_w = L w, row n+1 is c_w = w^T L; (n, n+1) = e^T L w, (n+1, n) = w^T L e,
+// (n+1, n+1) = w^T L w.  They ride through the update GEMMs as one more row / column (Theorem 1 holds
+// for any weight vector); the panel's rows n+1 of V and Y (w^T V and c_w V T) are formed
+// after the panel by k_wchk_*; the finished panel columns' c_w entries are re-encoded (k_cw_panel).
+// ---------------------------------------------------------------------------
+// corners of the weighted pair after encode: (n, n+1) = sum r_w, (n+1, n) = sum c_w, (n+1, n+1) = sum w_j c_w(j)
+__global__ void k_encode_w_finish(double *Aw, int64_t ldw, int n) {
+    __shared__ double ws[3][32];
+    double a = 0.0, b = 0.0, c = 0.0;
+    const double *rw = Aw + (int64_t)(n + 1) * ldw;
+    for (int i = threadIdx.x; i < n; i += blockDim.x) {
+        a += rw[i];
+        const double cwj = Aw[n + 1 + (int64_t)i * ldw];
+        b += cwj;
+        c += (double)(i + 1) * cwj;
+    }
+    a = warp_sum(a);
+    b = warp_sum(b);
+    c = warp_sum(c);
+    if ((threadIdx.x & 31) == 0) {
+        ws[0][threadIdx.x >> 5] = a;
+        ws[1][threadIdx.x >> 5] = b;
+        ws[2][threadIdx.x >> 5] = c;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double x = 0.0, y = 0.0, z = 0.0;
+        for (int w = 0; w < (int)(blockDim.x >> 5); w++) {
+            x += ws[0][w];
+            y += ws[1][w];
+            z += ws[2][w];
+        }
+        Aw[n + (int64_t)(n + 1) * ldw] = x;
+        Aw[n + 1 + (int64_t)n * ldw] = y;
+        Aw[n + 1 + (int64_t)(n + 1) * ldw] = z;
+    }
+}
+// c_w(j) = sum_i w_i A(i, j) into row n+1 (warp per column, fixed order)
+__global__ void k_encode_cols_w(double *Aw, int64_t ldw, int n) {
+    int j = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+    int lane = threadIdx.x & 31;
+    if (j >= n) return;
+    double s = 0.0;
+    for (int i = lane; i < n; i += 32) s += (double)(i + 1) * Aw[i + (int64_t)j * ldw];
+    s = warp_sum(s);
+    if (lane == 0) Aw[n + 1 + (int64_t)j * ldw] = s;
+}
+cudaError_t ft_encode_w(double *Aw, int64_t ldw, int n, double *linepart, cudaStream_t s) {
+    if (n <= 0) return cudaSuccess;
+    const int nrb = (n + LS_RB - 1) / LS_RB, nch = ls_chunks(n);
+    g_ft_launches += 4;
+    k_rowsum_part<<<dim3(nrb, nch), LS_RB, 0, s>>>(Aw, ldw, n, nch, -1, 0, 0, 0, linepart, nullptr, 1);
+    k_rowsum_finish<<<(n + 255) / 256, 256, 0, s>>>(linepart, n, nch, nullptr, 0, Aw + (int64_t)(n + 1) * ldw, 1);
+    k_encode_cols_w<<<(n + 7) / 8, 256, 0, s>>>(Aw, ldw, n);
+    k_encode_w_finish<<<1, 1024, 0, s>>>(Aw, ldw, n);
+    return cudaGetLastError();
+}
+
+// weighted syndromes of the full verification: D_rw = r_w - L w, D_cw = c_w - w^T L (mode 0, H logical)
+cudaError_t ft_full_verify_w(const double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdone, const double *rw,
+                             const double *cw, int64_t cinc, double *Drw, double *Dcw, double *linepart,
+                             cudaStream_t s) {
+    if (n <= 0) return cudaSuccess;
+    g_ft_launches += 3;
+    const int nrb = (n + LS_RB - 1) / LS_RB, nch = ls_chunks(n);
+    k_rowsum_part<<<dim3(nrb, nch), LS_RB, 0, s>>>(Aw, ldw, n, nch, 0, ilo, ihi, cdone, linepart, nullptr, 1);
+    k_rowsum_finish<<<(n + 255) / 256, 256, 0, s>>>(linepart, n, nch, rw, 1, Drw, 1);
+    k_fv_cols<<<(n + 7) / 8, 256, 0, s>>>(Aw, ldw, n, ilo, ihi, cdone, 0, cw, cinc, Dcw, 1);
+    return cudaGetLastError();
+}
+
+// after the panel: V(n+1, j) = sum_i w_i V(i, j) and s(j) = sum_i c_w0(i) V(i, j) over the reflector
+// rows k+1 .. ihi-1 (c_w0 = row n+1 at panel start: the panel does not touch it), as per-chunk partials
+#define WCHK_ROWS 256
+__global__ void __launch_bounds__(256) k_wchk_part(const double *Aw, int64_t ldw, const double *V, int n, int ihi,
+                                                   int k, int ib, double *part, const FtCtl *ctl) {
+    if (ctl->halt) return;
+    const int j = threadIdx.x & 63, q = threadIdx.x >> 6;  // 4 row phases x 64 columns
+    const int r0 = k + 1 + blockIdx.x * WCHK_ROWS, r1 = min(ihi, r0 + WCHK_ROWS);
+    double sw = 0.0, sc = 0.0;
+    if (j < ib)
+        for (int i = r0 + q; i < r1; i += 4) {
+            const double v = V[i + (int64_t)j * ldw];
+            sw += (double)(i + 1) * v;
+            sc += Aw[n + 1 + (int64_t)i * ldw] * v;
+        }
+    __shared__ double red[2][4][64];
+    red[0][q][j] = sw;
+    red[1][q][j] = sc;
+    __syncthreads();
+    if (q == 0) {
+        part[(int64_t)blockIdx.x * 128 + j] = ((red[0][0][j] + red[0][1][j]) + (red[0][2][j] + red[0][3][j]));
+        part[(int64_t)blockIdx.x * 128 + 64 + j] = ((red[1][0][j] + red[1][1][j]) + (red[1][2][j] + red[1][3][j]));
+    }
+}
+// chunk partials in chunk order; V(n+1, :) = w^T V, Y(n+1, :) = (c_w0 V) T  (Y = A V T, DLAHR2)
+__global__ void k_wchk_finish(double *V, double *Y, const double *T, int64_t ldw, int n, int ib, const double *part,
+                              int nchunk, const FtCtl *ctl) {
+    if (ctl->halt) return;
+    __shared__ double sc[64];
+    const int j = threadIdx.x;
+    double a = 0.0, b = 0.0;
+    for (int c = 0; c < nchunk; c++) {
+        a += part[(int64_t)c * 128 + j];
+        b += part[(int64_t)c * 128 + 64 + j];
+    }
+    sc[j] = b;
+    __syncthreads();
+    if (j < ib) {
+        double y = 0.0;
+        for (int bb = 0; bb <= j; bb++) y += sc[bb] * T[bb + j * FT_NBMAX];
+        V[n + 1 + (int64_t)j * ldw] = a;
+        Y[n + 1 + (int64_t)j * ldw] = y;
+    }
+}
+cudaError_t ft_wchk(const double *Aw, double *V, double *Y, const double *T, int64_t ldw, int n, int ihi, int k,
+                    int ib, double *part, const FtCtl *ctl, cudaStream_t s) {
+    const int nchunk = std::max(1, (ihi - k - 1 + WCHK_ROWS - 1) / WCHK_ROWS);
+    g_ft_launches += 2;
+    k_wchk_part<<<nchunk, 256, 0, s>>>(Aw, ldw, V, n, ihi, k, ib, part, ctl);
+    k_wchk_finish<<<1, 64, 0, s>>>(V, Y, T, ldw, n, ib, part, nchunk, ctl);
+    return cudaGetLastError();
+}
+
+// the finished panel columns [k, e): c_w(col) re-encoded from the logical column (rows outside the
+// stored Householder vectors; R6), once the iteration has made them final
+__global__ void k_cw_panel(double *Aw, int64_t ldw, int n, int ilo, int ihi, int k, int e, const FtCtl *ctl) {
+    if (ctl->halt) return;
+    const int col = k + blockIdx.x;
+    if (col >= e) return;
+    __shared__ double ws[32];
+    double s = 0.0;
+    for (int i = threadIdx.x; i < n; i += blockDim.x)
+        if (!in_v(i, col, ilo, ihi, e)) s += (double)(i + 1) * Aw[i + (int64_t)col * ldw];
+    s = warp_sum(s);
+    if ((threadIdx.x & 31) == 0) ws[threadIdx.x >> 5] = s;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double t = 0.0;
+        for (int w = 0; w < (int)(blockDim.x >> 5); w++) t += ws[w];
+        Aw[n + 1 + (int64_t)col * ldw] = t;
+    }
+}
+cudaError_t ft_cw_panel(double *Aw, int64_t ldw, int n, int ilo, int ihi, int k, int e, const FtCtl *ctl,
+                        cudaStream_t s) {
+    if (e <= k) return cudaSuccess;
+    g_ft_launches++;
+    k_cw_panel<<<e - k, 256, 0, s>>>(Aw, ldw, n, ilo, ihi, k, e, ctl);
+    return cudaGetLastError();
+}
+
+// diskless checkpoint of the weighted pair: column n+1 (rows 0..n+1) and row n+1 (columns 0..n+1)
+__global__ void k_ckpt_w(double *Aw, int64_t ldw, int n, double *ck, int restore, const FtCtl *ctl) {
+    if (!restore && ctl->halt) return;
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i <= n + 1; i += gridDim.x * blockDim.x) {
+        double *a = Aw + i + (int64_t)(n + 1) * ldw, *b = Aw + n + 1 + (int64_t)i * ldw;
+        if (restore) {
+            *a = ck[i];
+            *b = ck[n + 2 + i];
+        } else {
+            ck[i] = *a;
+            ck[n + 2 + i] = *b;
+        }
+    }
+}
+cudaError_t ft_ckpt_w(double *Aw, int64_t ldw, int n, double *ck, int restore, const FtCtl *ctl, cudaStream_t s) {
+    g_ft_launches++;
+    k_ckpt_w<<<std::max(1, std::min((n + 2 + 255) / 256, 64)), 256, 0, s>>>(Aw, ldw, n, ck, restore, ctl);
+    return cudaGetLastError();
+}
+
 // one block per fix: explicit sum excluding the bad element
 __global__ void k_fix(double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdone, int mode, double *r,
                       int64_t rinc, double *c, int64_t cinc, double *kappa, const FtFix *fixes, double *deltas) {
@@ -439,18 +640,22 @@ __global__ void k_fix(double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdon
     __shared__ double ws[32];
     double s = 0.0;
     const int i0 = (int)f.i, j0 = (int)f.j;
-    if (f.kind == 0 || f.kind == 2) {  // along row i
+    if (f.kind == 0 || f.kind == 2 || f.kind == 5) {  // along row i (5: weighted)
         for (int j = threadIdx.x; j < n; j += blockDim.x) {
             if (f.kind == 0 && j == j0) continue;
             bool v = in_v(i0, j, ilo, ihi, cdone);
-            if (mode == 0 ? !v : v) s += Aw[i0 + (int64_t)j * ldw];
+            if (mode == 0 ? !v : v) s += (f.kind == 5 ? (double)(j + 1) : 1.0) * Aw[i0 + (int64_t)j * ldw];
         }
-    } else if (f.kind == 1 || f.kind == 3) {  // along column j
+    } else if (f.kind == 1 || f.kind == 3 || f.kind == 6) {  // along column j (6: weighted)
         for (int i = threadIdx.x; i < n; i += blockDim.x) {
             if (f.kind == 1 && i == i0) continue;
             bool v = in_v(i, j0, ilo, ihi, cdone);
-            if (mode == 0 ? !v : v) s += Aw[i + (int64_t)j0 * ldw];
+            if (mode == 0 ? !v : v) s += (f.kind == 6 ? (double)(i + 1) : 1.0) * Aw[i + (int64_t)j0 * ldw];
         }
+    } else if (f.kind == 7) {  // e^T L w = sum r_w (column n+1)
+        for (int i = threadIdx.x; i < n; i += blockDim.x) s += Aw[i + (int64_t)(n + 1) * ldw];
+    } else if (f.kind == 8) {  // w^T L e = sum c_w (row n+1)
+        for (int j = threadIdx.x; j < n; j += blockDim.x) s += Aw[n + 1 + (int64_t)j * ldw];
     } else {  // kappa = sum r
         for (int i = threadIdx.x; i < n; i += blockDim.x) s += r[(int64_t)i * rinc];
     }
@@ -473,6 +678,18 @@ __global__ void k_fix(double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdon
             nv = t;
         } else if (f.kind == 3) {
             dst = c + (int64_t)j0 * cinc;
+            nv = t;
+        } else if (f.kind == 5) {
+            dst = Aw + i0 + (int64_t)(n + 1) * ldw;
+            nv = t;
+        } else if (f.kind == 6) {
+            dst = Aw + n + 1 + (int64_t)j0 * ldw;
+            nv = t;
+        } else if (f.kind == 7) {
+            dst = Aw + n + (int64_t)(n + 1) * ldw;
+            nv = t;
+        } else if (f.kind == 8) {
+            dst = Aw + n + 1 + (int64_t)n * ldw;
             nv = t;
         } else {
             dst = kappa;

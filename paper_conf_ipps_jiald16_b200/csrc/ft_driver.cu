@@ -87,7 +87,8 @@ struct Work {
     double *Aw = nullptr, *V = nullptr, *Y = nullptr, *Z = nullptr, *T = nullptr, *Wpart = nullptr, *bvec = nullptr,
            *acc = nullptr, *ckpt = nullptr, *ck_r = nullptr, *ck_c = nullptr, *ck_q = nullptr, *Fr = nullptr,
            *Qr = nullptr, *Qc = nullptr, *Dr = nullptr, *Dc = nullptr, *sums = nullptr, *ypart = nullptr,
-           *rowpart = nullptr, *linepart = nullptr, *scratch = nullptr, *deltas = nullptr, *hA = nullptr, *htau = nullptr;
+           *rowpart = nullptr, *linepart = nullptr, *scratch = nullptr, *deltas = nullptr, *hA = nullptr, *htau = nullptr,
+           *ck_w = nullptr, *Dr2 = nullptr, *Dc2 = nullptr, *wpart = nullptr;
     unsigned *bar = nullptr;
     int *strip_done = nullptr;
     cudaStream_t cap_stream = nullptr;  // graph capture stream (library-owned)
@@ -99,7 +100,7 @@ struct Work {
     size_t bytes = 0;
     void release() {
         double **ps[] = {&Wt, &Aw, &V, &Y, &Z, &T, &Wpart, &bvec, &acc, &ckpt, &ck_r, &ck_c, &ck_q, &Fr, &Qr, &Qc, &Dr, &Dc,
-                         &sums, &ypart, &rowpart, &linepart, &scratch, &deltas, &hA, &htau};
+                         &sums, &ypart, &rowpart, &linepart, &scratch, &deltas, &hA, &htau, &ck_w, &Dr2, &Dc2, &wpart};
         for (auto p : ps) {
             if (*p) cudaFree(*p);
             *p = nullptr;
@@ -120,14 +121,14 @@ std::map<int, Work> g_work;
 
 // CUDA graphs of fault-free calls, keyed by device, shape, options and caller buffers
 struct GraphKey {
-    int dev, n, ilo, ihi, nb, abft, policy;
+    int dev, n, ilo, ihi, nb, abft, policy, weighted;
     double c_thr;
     const void *dA;
     int lda;
     const void *dtau;
     bool operator<(const GraphKey &o) const {
-        return std::tie(dev, n, ilo, ihi, nb, abft, policy, c_thr, dA, lda, dtau) <
-               std::tie(o.dev, o.n, o.ilo, o.ihi, o.nb, o.abft, o.policy, o.c_thr, o.dA, o.lda, o.dtau);
+        return std::tie(dev, n, ilo, ihi, nb, abft, policy, weighted, c_thr, dA, lda, dtau) <
+               std::tie(o.dev, o.n, o.ilo, o.ihi, o.nb, o.abft, o.policy, o.weighted, o.c_thr, o.dA, o.lda, o.dtau);
     }
 };
 struct GraphEntry {
@@ -195,6 +196,10 @@ int get_work(int n, Work **out) {
     // row-sum partials of the verification ([64][ldw]) / Gram partials of Q formation's DLARFT
     A(dalloc(&w.linepart, (size_t)std::max<int64_t>(64 * ldw, 4096 * ((int64_t)n / 64 + 2)), b));
     A(dalloc(&w.deltas, (size_t)FT_MAX_EVENTS, b));
+    A(dalloc(&w.ck_w, (size_t)2 * (n + 2), b));  // weighted pair (NEXT-1): checkpoint, syndromes, partials
+    A(dalloc(&w.Dr2, (size_t)ldw, b));
+    A(dalloc(&w.Dc2, (size_t)ldw, b));
+    A(dalloc(&w.wpart, (size_t)128 * (n / 256 + 2), b));
     A(dalloc(&w.bar, 4, b));
     A(dalloc(&w.strip_done, (N1 + 63) / 64 + 2, b));
     A(dalloc(&w.ctl, 1, b));
@@ -385,6 +390,7 @@ Plan decode(int n, const std::vector<double> &Dr, const std::vector<double> &Dc,
 // ---------------------------------------------------------------------------
 struct Call {
     int n, ilo, ihi, nb, abft, policy;
+    int weighted = 0;  // NEXT-1: the weighted checksum pair rides as row / column n+1
     double c_thr;
     cudaStream_t s;
     Work *w;
@@ -476,6 +482,12 @@ double *site_addr(Call &C, const ft_fault &f) {
     case FT_SITE_T:
         if (f.i < 0 || f.i >= FT_NBMAX || f.j < 0 || f.j >= FT_NBMAX) return nullptr;
         return w.T + f.i + f.j * FT_NBMAX;
+    case FT_SITE_RW:
+        if (!C.weighted || f.i < 0 || f.i >= n) return nullptr;
+        return w.Aw + f.i + (int64_t)(n + 1) * ldw;
+    case FT_SITE_CW:
+        if (!C.weighted || f.j < 0 || f.j >= n) return nullptr;
+        return w.Aw + n + 1 + f.j * ldw;
     }
     return nullptr;
 }
@@ -573,9 +585,9 @@ int right_update(Call &C, int t, double sign, int do_w, bool precheck = false) {
     // trailing block (+ checksum row/column), fused with W = V^T A_new and W' = T^T W
     g.do_right = 1;
     g.r_lo = 0;
-    g.r_hi = C.rend();
+    g.r_hi = C.rend() + C.weighted;  // + row n+1 (c_w) / column n+1 (r_w) of the weighted pair
     g.c_lo = e;
-    g.c_hi = C.cend();
+    g.c_hi = C.cend() + C.weighted;
     g.wr_lo = k + 1;
     g.wr_hi = C.ihi;
     g.do_w = do_w;
@@ -608,9 +620,9 @@ int left_update(Call &C, int t, double sign, int nsplit, int endcheck = 0, bool 
     g.Wpart = w.Wpart;
     g.Wt = w.Wt;
     g.r_lo = k + 1;
-    g.r_hi = C.rend();
+    g.r_hi = C.rend() + C.weighted;
     g.c_lo = e;
-    g.c_hi = C.cend();
+    g.c_hi = C.cend() + C.weighted;
     g.K = ib;
     g.nsplit = nsplit;
     g.wsplit_stride = ((int64_t)C.n + 1 + 64) * FT_NBMAX;
@@ -633,7 +645,7 @@ int left_update(Call &C, int t, double sign, int nsplit, int endcheck = 0, bool 
 
 int trailing_nsplit(Call &C, int t) {
     const int e = C.pk(t) + C.pib(t);
-    return ft_gemm_splits(0, C.rend(), e, C.cend(), C.w->nsm);
+    return ft_gemm_splits(0, C.rend() + C.weighted, e, C.cend() + C.weighted, C.w->nsm);
 }
 
 // panel-kernel sync state: barrier counters and accumulator sets must be zero when a
@@ -687,6 +699,7 @@ int enqueue_panel(Call &C, int t) {
     p.ytop = C.fused_ytop ? 1 : 0;
     int rendp = (C.rend() + gr - 1) / gr * gr;
     p.ngroups = (rendp - p.rbase) / gr;
+    if (C.weighted) CK(ft_ckpt_w(w.Aw, w.ldw, n, w.ck_w, 0, w.ctl, C.s));
     const int sp_panel = span_begin(C, TC_PANEL);
     const int sp_kpanel = span_begin(C, TK_PANEL);
     CK(ft_launch_panel(p, w.nsm, C.s));
@@ -716,6 +729,8 @@ int enqueue_panel(Call &C, int t) {
     while ((int64_t)ns * (k + 1) > kYtopRows) ns--;
     y.nsplit = std::max(ns, 1);
     if (!C.fused_ytop) CK(ft_launch_ytop(y, C.s));
+    // weighted pair: rows n+1 of V and Y (w^T V, c_w V T), part of the panel's output
+    if (C.weighted) CK(ft_wchk(w.Aw, w.V, w.Y, w.T, w.ldw, n, C.ihi, k, ib, w.wpart, w.ctl, C.s));
     span_end(C, sp_panel);
     if (inject_at(C, t, FT_PHASE_AFTER_PANEL)) return FT_E_CUDA;
     if (eager && !fuse_pre) {
@@ -733,17 +748,21 @@ int enqueue_panel(Call &C, int t) {
         span_end(C, sp);
     }
     if (inject_at(C, t, FT_PHASE_AFTER_RIGHT)) return FT_E_CUDA;
-    const bool fuse_end = C.abft && !has_fault(C, t, FT_PHASE_AFTER_UPDATE);
+    // the weighted pair (NEXT-1) takes the separate end check, which also sums r_w and c_w
+    const bool fuse_end = C.abft && !C.weighted && !has_fault(C, t, FT_PHASE_AFTER_UPDATE);
     {
         const int sp = span_begin(C, TC_LEFT), sk = span_begin(C, TK_LEFT);
         if (left_update(C, t, -1.0, trailing_nsplit(C, t), fuse_end ? 1 : 0, fuse_pre)) return FT_E_CUDA;
         span_end(C, sk);
         span_end(C, sp);
     }
+    // weighted pair: the panel columns are final now -- their c_w entries (row n+1, which no update
+    // kernel writes for them) re-encoded before the end check compares sum c_w with w^T L e
+    if (C.weighted) CK(ft_cw_panel(w.Aw, w.ldw, n, C.ilo, C.ihi, k, k + ib, w.ctl, C.s));
     if (inject_at(C, t, FT_PHASE_AFTER_UPDATE)) return FT_E_CUDA;
     if (C.abft && !fuse_end) {
         const int sp = span_begin(C, TC_VERIFY);
-        CK(ft_endcheck(w.Aw, w.ldw, n, C.ihi, k, ib, t, C.policy, w.Fr, w.ctl, C.s));
+        CK(ft_endcheck(w.Aw, w.ldw, n, C.ihi, k, ib, t, C.policy, w.Fr, w.ctl, C.s, C.weighted));
         span_end(C, sp);
     }
     if (C.hA) {  // columns [k, e) are final: back to the host beside the next panels
@@ -758,9 +777,209 @@ int enqueue_panel(Call &C, int t) {
 
 // full verify + decode + correct + re-verify.  mode 0: H (cdone finished columns), 1: Q.
 // Returns 0 ok (clean or corrected), FT_E_UNCORRECTABLE, or an error.
+// ---------------------------------------------------------------------------
+// Weighted pair (NEXT-1, w_i = i + 1): decoder v3 on the host (written apart from the oracle's).
+// v2 first on the plain syndromes; if it corrects, weighted words that still disagree are refreshed;
+// if it refuses, the weighted syndromes locate: D_cw(j) / D_c(j) = w_i names row i of column j's one
+// error (and a row likewise), repaired along the line that holds no other error; checksum words
+// whose orthogonal direction is clean are refreshed; the result is re-verified.
+// ---------------------------------------------------------------------------
+struct WSyn {
+    std::vector<double> Dr, Dc, Drw, Dcw, rw, cw;
+    double sumr = 0, sumc = 0, kap = 0, krw = 0, kcw = 0;
+};
+
+int fetch_wsyn(Call &C, int cdone, WSyn &S) {
+    Work &w = *C.w;
+    const int n = C.n;
+    const int64_t ldw = w.ldw;
+    double *M = w.Aw;
+    S.Dr.resize(n);
+    S.Dc.resize(n);
+    S.Drw.resize(n);
+    S.Dcw.resize(n);
+    S.rw.resize(n);
+    S.cw.resize(n);
+    CK(ft_full_verify(M, ldw, n, C.ilo, C.ihi, cdone, 0, M + (int64_t)n * ldw, 1, M + n, ldw, nullptr, w.Dr, w.Dc,
+                      w.sums, w.linepart, C.s));
+    CK(cudaMemcpyAsync(S.Dr.data(), w.Dr, n * sizeof(double), cudaMemcpyDeviceToHost, C.s));
+    CK(cudaMemcpyAsync(S.Dc.data(), w.Dc, n * sizeof(double), cudaMemcpyDeviceToHost, C.s));
+    double sums[2];
+    CK(cudaMemcpyAsync(sums, w.sums, 2 * sizeof(double), cudaMemcpyDeviceToHost, C.s));
+    CK(ft_full_verify_w(M, ldw, n, C.ilo, C.ihi, cdone, M + (int64_t)(n + 1) * ldw, M + n + 1, ldw, w.Dr2, w.Dc2,
+                        w.linepart, C.s));
+    CK(cudaMemcpyAsync(S.Drw.data(), w.Dr2, n * sizeof(double), cudaMemcpyDeviceToHost, C.s));
+    CK(cudaMemcpyAsync(S.Dcw.data(), w.Dc2, n * sizeof(double), cudaMemcpyDeviceToHost, C.s));
+    CK(cudaMemcpyAsync(S.rw.data(), M + (int64_t)(n + 1) * ldw, n * sizeof(double), cudaMemcpyDeviceToHost, C.s));
+    CK(cudaMemcpy2DAsync(S.cw.data(), sizeof(double), M + n + 1, ldw * sizeof(double), sizeof(double), n,
+                         cudaMemcpyDeviceToHost, C.s));
+    double corner[3];
+    CK(cudaMemcpyAsync(&corner[0], M + n + (int64_t)n * ldw, sizeof(double), cudaMemcpyDeviceToHost, C.s));
+    CK(cudaMemcpyAsync(&corner[1], M + n + (int64_t)(n + 1) * ldw, sizeof(double), cudaMemcpyDeviceToHost, C.s));
+    CK(cudaMemcpyAsync(&corner[2], M + n + 1 + (int64_t)n * ldw, sizeof(double), cudaMemcpyDeviceToHost, C.s));
+    CK(cudaStreamSynchronize(C.s));
+    S.sumr = sums[0];
+    S.sumc = sums[1];
+    S.kap = corner[0];
+    S.krw = corner[1];
+    S.kcw = corner[2];
+    return 0;
+}
+
+// fixes one launch at a time, in order (a later fix may read a word an earlier one repaired)
+int apply_seq(Call &C, int panel, int cdone, const std::vector<FtFix> &fx) {
+    Work &w = *C.w;
+    const int n = C.n;
+    const int64_t ldw = w.ldw;
+    double *M = w.Aw;
+    for (const FtFix &f : fx) {
+        CK(cudaMemcpyAsync(w.fixes, &f, sizeof(FtFix), cudaMemcpyHostToDevice, C.s));
+        CK(ft_apply_fixes(M, ldw, n, C.ilo, C.ihi, cdone, 0, M + (int64_t)n * ldw, 1, M + n, ldw,
+                          M + n + (int64_t)n * ldw, w.fixes, 1, w.deltas, C.s));
+        double d = 0.0;
+        CK(cudaMemcpyAsync(&d, w.deltas, sizeof(double), cudaMemcpyDeviceToHost, C.s));
+        CK(cudaStreamSynchronize(C.s));
+        const int kind = f.kind <= 1 ? FT_EV_FIX_DATA : f.kind == 2 ? FT_EV_FIX_R : f.kind == 3 ? FT_EV_FIX_C
+                         : f.kind == 4 ? FT_EV_FIX_K : f.kind == 5 ? FT_EV_FIX_RW : f.kind == 6 ? FT_EV_FIX_CW
+                                                                                     : FT_EV_FIX_KW;
+        C.ev(kind, panel, f.i, f.j, d);
+    }
+    return 0;
+}
+
+// the index named by a weighted / plain syndrome ratio (w_x = x + 1), or -1 when the ratio is not
+// within 1/4 of an integer in [1, n] after its rounding error (t, tw: the two thresholds)
+int named_index(double Dw, double D, double t, double tw, int n) {
+    if (!std::isfinite(Dw) || !std::isfinite(D) || !(std::fabs(D) > t)) return -1;
+    const double rho = Dw / D;
+    const double err = (tw + (double)n * t) / std::fabs(D) + 4.0 * n * kEps * std::fabs(rho);
+    if (!(err < 0.25)) return -1;
+    const double k = std::nearbyint(rho);
+    if (!(std::fabs(rho - k) <= err) || k < 1.0 || k > (double)n) return -1;
+    return (int)k - 1;
+}
+
+int verify_and_correct_w(Call &C, int panel, int cdone, bool *found) {
+    Work &w = *C.w;
+    const int n = C.n;
+    FtCtl hctl;
+    CK(cudaMemcpyAsync(&hctl, w.ctl, sizeof(FtCtl), cudaMemcpyDeviceToHost, C.s));
+    CK(cudaStreamSynchronize(C.s));
+    const double tau = C.c_thr * n * kEps * hctl.normF, tw = tau * n;
+    const double tauS = tau * std::sqrt((double)std::max(n, 1)), twS = tw * std::sqrt((double)std::max(n, 1));
+    auto flagged_w = [&](const WSyn &S, int *nr, int *nc) {
+        int a = 0, b = 0;
+        for (int i = 0; i < n; i++) a += bad(S.Dr[i], tau) || bad(S.Drw[i], tw);
+        for (int j = 0; j < n; j++) b += bad(S.Dc[j], tau) || bad(S.Dcw[j], tw);
+        if (nr) *nr = a;
+        if (nc) *nc = b;
+        return a + b;
+    };
+    auto sums_ok = [&](const WSyn &S) {
+        double srw = 0.0, scw = 0.0;
+        for (int i = 0; i < n; i++) srw += S.rw[i];
+        for (int j = 0; j < n; j++) scw += S.cw[j];
+        return same(S.sumr, S.kap, tauS) && same(S.sumc, S.kap, tauS) && same(srw, S.krw, twS) && same(scw, S.kcw, twS);
+    };
+    WSyn S;
+    if (fetch_wsyn(C, cdone, S)) return FT_E_CUDA;
+    *found = false;
+    int nr = 0, nc = 0;
+    if (flagged_w(S, &nr, &nc) == 0 && sums_ok(S)) return 0;
+    *found = true;
+    C.ev(FT_EV_DETECT, panel, nr, nc, 0.0);
+    C.detected++;
+    auto fail = [&]() {
+        C.ev(FT_EV_UNCORRECTABLE, panel, -1, -1, 0.0);
+        C.uncorrectable++;
+        return FT_E_UNCORRECTABLE;
+    };
+    Plan P = decode(n, S.Dr, S.Dc, S.sumr - S.kap, S.sumc - S.kap, tau);
+    if (P.status == 1) {
+        if (apply_seq(C, panel, cdone, P.fixes)) return FT_E_CUDA;
+        if (fetch_wsyn(C, cdone, S)) return FT_E_CUDA;
+    }
+    std::vector<FtFix> fx;
+    if (P.status != 2) {
+        // the data are verified: weighted words that still disagree are refreshed
+        for (int i = 0; i < n; i++)
+            if (bad(S.Drw[i], tw)) fx.push_back({i, -1, 5, 0});
+        for (int j = 0; j < n; j++)
+            if (bad(S.Dcw[j], tw)) fx.push_back({-1, j, 6, 0});
+    } else {
+        // weighted location, pass by pass (each pass can free lines for the next: L-shapes)
+        for (int pass = 0; pass < 8; pass++) {
+            int a = 0, b = 0;
+            for (int i = 0; i < n; i++) a += bad(S.Dr[i], tau);
+            for (int j = 0; j < n; j++) b += bad(S.Dc[j], tau);
+            if (a == 0 || b == 0) break;
+            std::vector<int> pi(n, -1);
+            std::vector<FtFix> step;
+            for (int j = 0; j < n; j++) {
+                if (!bad(S.Dc[j], tau)) continue;
+                const int i = named_index(S.Dcw[j], S.Dc[j], tau, tw, n);
+                if (i >= 0 && (bad(S.Dr[i], tau) || bad(S.Drw[i], tw))) pi[j] = i;
+            }
+            for (int j = 0; j < n; j++) {
+                const int i = pi[j];
+                if (i < 0) continue;
+                const int jr = named_index(S.Drw[i], S.Dr[i], tau, tw, n);
+                step.push_back({i, j, jr == j ? 0 : 1, 0});  // alone in its row: row formula; else column
+            }
+            for (int i = 0; i < n; i++) {
+                if (!bad(S.Dr[i], tau)) continue;
+                const int j = named_index(S.Drw[i], S.Dr[i], tau, tw, n);
+                if (j < 0 || !(bad(S.Dc[j], tau) || bad(S.Dcw[j], tw)) || pi[j] >= 0) continue;
+                step.push_back({i, j, 0, 0});
+            }
+            if (step.empty()) break;
+            if (apply_seq(C, panel, cdone, step)) return FT_E_CUDA;
+            if (fetch_wsyn(C, cdone, S)) return FT_E_CUDA;
+        }
+        // checksum words: refreshed only when the orthogonal direction shows no flag anywhere
+        int anyR = 0, anyC = 0;
+        flagged_w(S, &anyR, &anyC);
+        if (anyR && !anyC)
+            for (int i = 0; i < n; i++) {
+                if (bad(S.Dr[i], tau)) fx.push_back({i, -1, 2, 0});
+                if (bad(S.Drw[i], tw)) fx.push_back({i, -1, 5, 0});
+            }
+        if (anyC && !anyR)
+            for (int j = 0; j < n; j++) {
+                if (bad(S.Dc[j], tau)) fx.push_back({-1, j, 3, 0});
+                if (bad(S.Dcw[j], tw)) fx.push_back({-1, j, 6, 0});
+            }
+    }
+    if (!fx.empty()) {
+        if (apply_seq(C, panel, cdone, fx)) return FT_E_CUDA;
+        if (fetch_wsyn(C, cdone, S)) return FT_E_CUDA;
+    }
+    // corners: kappa when both plain sums are off by the same amount; the weighted corners from the
+    // (now verified) weighted vectors
+    fx.clear();
+    if (!same(S.sumr, S.kap, tauS) && same(S.sumr, S.sumc, tauS)) fx.push_back({-1, -1, 4, 0});
+    {
+        double srw = 0.0, scw = 0.0;
+        for (int i = 0; i < n; i++) srw += S.rw[i];
+        for (int j = 0; j < n; j++) scw += S.cw[j];
+        if (flagged_w(S, nullptr, nullptr) == 0) {
+            if (!same(srw, S.krw, twS)) fx.push_back({-1, -1, 7, 0});
+            if (!same(scw, S.kcw, twS)) fx.push_back({-1, -1, 8, 0});
+        }
+    }
+    if (!fx.empty()) {
+        if (apply_seq(C, panel, cdone, fx)) return FT_E_CUDA;
+        if (fetch_wsyn(C, cdone, S)) return FT_E_CUDA;
+    }
+    if (flagged_w(S, nullptr, nullptr) != 0 || !sums_ok(S)) return fail();
+    C.corrected++;
+    return 0;
+}
+
 // M: the augmented working array (the reduction's Aw, or ft_dorghr's augmented Q); mode 0 reads its
 // checksum column n / row n / corner, mode 1 the Q checksums of the Householder vectors
 int verify_and_correct(Call &C, int panel, int cdone, int mode, bool *found, double *M = nullptr) {
+    if (C.weighted && mode == 0 && (!M || M == C.w->Aw)) return verify_and_correct_w(C, panel, cdone, found);
     Work &w = *C.w;
     const int n = C.n;
     const int64_t ldw = w.ldw;
@@ -866,6 +1085,7 @@ int recover_body(Call &C, const FtCtl &h) {
     CK(cudaMemcpyAsync(&w.ctl->nflag, &zero, sizeof(int), cudaMemcpyHostToDevice, C.s));
     CK(cudaMemsetAsync(w.ctl->eY, 0, sizeof(double) * 2 * FT_NBMAX * FT_ESTR, C.s));
     CK(cudaMemsetAsync(w.ctl->sums, 0, sizeof(double) * 4, C.s));
+    CK(cudaMemsetAsync(w.ctl->wsums, 0, sizeof(double) * 2, C.s));
     CK(cudaMemsetAsync(&w.ctl->done_count, 0, 3 * sizeof(int), C.s));  // done_count, done_ytop, done_left
     CK(cudaMemsetAsync(&w.ctl->tbad, 0, sizeof(int), C.s));
     if (h.halt_stage == 3) {
@@ -886,6 +1106,7 @@ int recover_body(Call &C, const FtCtl &h) {
     }
     // restore the pre-factorized panel and the checksum vectors (diskless checkpoint)
     if (checkpoint(C, t, 1)) return FT_E_CUDA;
+    if (C.weighted) CK(ft_ckpt_w(w.Aw, w.ldw, C.n, w.ck_w, 1, w.ctl, C.s));
     if (reset_panel_state(C)) return FT_E_CUDA;
     bool found = false;
     int info = verify_and_correct(C, t, k, 0, &found);
@@ -915,6 +1136,7 @@ int enqueue_start(Call &C, const double *dA, int lda) {
     if (C.abft) {
         const int sp_enc = span_begin(C, TC_ENCODE);
         CK(ft_encode(w.Aw, w.ldw, n, w.ctl, w.scratch, w.linepart, s));
+        if (C.weighted) CK(ft_encode_w(w.Aw, w.ldw, n, w.linepart, s));
         CK(cudaMemsetAsync(w.Fr, 0, w.ldw * sizeof(double), s));
         if (C.ilo > 1) CK(ft_frozen_init(w.Aw, w.ldw, n, C.ilo - 1, w.Fr, s));
         CK(cudaMemsetAsync(w.Qr, 0, w.ldw * sizeof(double), s));
@@ -934,7 +1156,7 @@ int validate(int n, int ilo, int ihi, const void *A, int lda, const void *tau, c
     if (o) {
         if (o->nb < 0 || o->nb > FT_NBMAX) return -7;
         if (o->abft != 0 && o->abft != 1) return -7;
-        if (o->weighted != 0) return -7;
+        if (o->weighted != 0 && (o->weighted != 1 || o->abft != 1)) return -7;  // NEXT-1 needs ABFT
         if (o->policy != FT_POLICY_EAGER && o->policy != FT_POLICY_PAPER) return -7;
         if (o->c_thr < 0.0 || !(o->c_thr == o->c_thr)) return -7;
         if (o->nfaults < 0 || o->nfaults > FT_MAXFAULTS || (o->nfaults > 0 && !o->faults)) return -7;
@@ -959,6 +1181,7 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
     C.ihi = ihi;
     C.nb = o.nb > 0 ? o.nb : (n < 4096 ? 32 : 64);
     C.abft = o.abft;
+    C.weighted = o.abft ? o.weighted : 0;
     C.policy = o.policy;
     C.c_thr = o.c_thr > 0 ? o.c_thr : 2.0;
     C.s = s;
@@ -995,7 +1218,7 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
     if (graphable) {
         int dev = 0;
         CK(cudaGetDevice(&dev));
-        GraphKey key{dev, n, ilo, ihi, C.nb, C.abft, C.policy, C.c_thr, C.hA ? (const void *)C.hA : (const void *)dA,
+        GraphKey key{dev, n, ilo, ihi, C.nb, C.abft, C.policy, C.weighted, C.c_thr, C.hA ? (const void *)C.hA : (const void *)dA,
                      C.hA ? (int)C.hlda : lda, (const void *)dtau};
         auto it = g_graphs.find(key);
         if (it != g_graphs.end() && it->second.exec) {
@@ -1114,6 +1337,16 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
                              cudaMemcpyDeviceToDevice, s));
         CK(cudaMemcpyAsync(o.dchk_out + 2 * n, w.Aw + n + (int64_t)n * w.ldw, sizeof(double),
                            cudaMemcpyDeviceToDevice, s));
+        if (C.weighted) {  // [.. | r_w | c_w | e^T L w | w^T L e]
+            CK(cudaMemcpyAsync(o.dchk_out + 2 * n + 1, w.Aw + (int64_t)(n + 1) * w.ldw, n * sizeof(double),
+                               cudaMemcpyDeviceToDevice, s));
+            CK(cudaMemcpy2DAsync(o.dchk_out + 3 * n + 1, sizeof(double), w.Aw + n + 1, w.ldw * sizeof(double),
+                                 sizeof(double), n, cudaMemcpyDeviceToDevice, s));
+            CK(cudaMemcpyAsync(o.dchk_out + 4 * n + 1, w.Aw + n + (int64_t)(n + 1) * w.ldw, sizeof(double),
+                               cudaMemcpyDeviceToDevice, s));
+            CK(cudaMemcpyAsync(o.dchk_out + 4 * n + 2, w.Aw + n + 1 + (int64_t)n * w.ldw, sizeof(double),
+                               cudaMemcpyDeviceToDevice, s));
+        }
     }
     CK(cudaEventRecord(ev1, s));
     FtCtl hf;

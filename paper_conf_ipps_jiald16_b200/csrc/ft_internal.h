@@ -24,7 +24,8 @@ struct FtCtl {
     int halt_panel;   // iteration at which the halt was raised
     int halt_stage;   // 1 = pre-update (verify-before-consume / workspace check), 2 = post-update,
                       // 3 = T checksum failed after the right update (only the right update to undo)
-    int halt_reason;  // bit 0: D_r flag, 1: Y check, 2: V check, 3: scalar check (paper), 4: kappa, 5: T check
+    int halt_reason;  // bit 0: D_r flag, 1: Y check, 2: V check, 3: scalar check (paper), 4: kappa, 5: T check,
+                      // 6: weighted sums (NEXT-1)
     int nflag;        // flagged rows in the fused verify of the current iteration
     int done_count;   // last-block-done counter (k_endcheck)
     int done_ytop;    // last-block-done counter (fused pre-update decision in the Y_top finalize)
@@ -37,6 +38,7 @@ struct FtCtl {
     double eY[64 * FT_ESTR];
     double eV[64 * FT_ESTR];
     double sums[4];       // end check: sum r, sum c
+    double wsums[2];      // end check of the weighted pair: sum r_w, sum c_w (NEXT-1)
     double tmax;          // max |T| of the last panel (written by the panel kernel; pre-update tolerance)
     // T checksum (reading R15 extended to T): row sums of the upper triangle of the panel's T, written
     // by the panel kernel with T; re-evaluated from T in memory by the right-update CTAs that form
@@ -200,14 +202,25 @@ cudaError_t ft_precheck(const double *Y, const double *V, int64_t ldw, int n, in
 cudaError_t ft_decide(const double *Y, const double *V, const double *T, int64_t ldw, int n, int k,
                       int ib, int panel, FtCtl *ctl, cudaStream_t s);
 cudaError_t ft_endcheck(double *Aw, int64_t ldw, int n, int ihi, int k, int ib, int panel, int policy,
-                        double *Fr, FtCtl *ctl, cudaStream_t s);
+                        double *Fr, FtCtl *ctl, cudaStream_t s, int weighted = 0);
 cudaError_t ft_zero_if_running(double *p, size_t n, const FtCtl *ctl, cudaStream_t s);
 cudaError_t ft_inject(double *addr, int fidx, int bit, FtCtl *ctl, cudaStream_t s);
 // full verification (recovery path / final): mode 0 = H logical, 1 = Q (V region)
 cudaError_t ft_full_verify(const double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdone, int mode,
                            const double *r, int64_t rinc, const double *c, int64_t cinc, const double *Fr,
                            double *Dr, double *Dc, double *sums, double *linepart, cudaStream_t s);
-struct FtFix { int64_t i, j; int kind; int pad; };  // kind: 0 row formula, 1 col formula, 2 refresh r(i), 3 refresh c(j), 4 kappa
+// kind: 0 row formula, 1 col formula, 2 refresh r(i), 3 refresh c(j), 4 kappa; weighted pair (NEXT-1):
+// 5 refresh r_w(i), 6 refresh c_w(j), 7 e^T L w = sum r_w, 8 w^T L e = sum c_w
+struct FtFix { int64_t i, j; int kind; int pad; };
+cudaError_t ft_encode_w(double *Aw, int64_t ldw, int n, double *linepart, cudaStream_t s);
+cudaError_t ft_full_verify_w(const double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdone, const double *rw,
+                             const double *cw, int64_t cinc, double *Drw, double *Dcw, double *linepart,
+                             cudaStream_t s);
+cudaError_t ft_wchk(const double *Aw, double *V, double *Y, const double *T, int64_t ldw, int n, int ihi, int k,
+                    int ib, double *part, const FtCtl *ctl, cudaStream_t s);
+cudaError_t ft_cw_panel(double *Aw, int64_t ldw, int n, int ilo, int ihi, int k, int e, const FtCtl *ctl,
+                        cudaStream_t s);
+cudaError_t ft_ckpt_w(double *Aw, int64_t ldw, int n, double *ck, int restore, const FtCtl *ctl, cudaStream_t s);
 cudaError_t ft_apply_fixes(double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdone, int mode,
                            double *r, int64_t rinc, double *c, int64_t cinc, double *kappa,
                            const FtFix *fixes, int nfix, double *deltas, cudaStream_t s);

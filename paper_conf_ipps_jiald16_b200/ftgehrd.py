@@ -18,9 +18,9 @@ _lib = None
 
 FT_E_UNCORRECTABLE, FT_E_CUDA, FT_E_NCCL, FT_E_NOMEM = 1, 2, 3, 4
 PHASE_BEFORE_PANEL, PHASE_AFTER_PANEL, PHASE_AFTER_RIGHT, PHASE_AFTER_UPDATE, PHASE_AT_END = range(5)
-SITE_A, SITE_R, SITE_C, SITE_K, SITE_Y, SITE_V, SITE_T = range(7)
+SITE_A, SITE_R, SITE_C, SITE_K, SITE_Y, SITE_V, SITE_T, SITE_RW, SITE_CW = range(9)
 EV_NAMES = ["INJECT", "DETECT", "FIX_DATA", "FIX_R", "FIX_C", "FIX_K", "FIX_Q", "FIX_QR", "FIX_QC",
-            "FIX_QK", "UNCORRECTABLE", "ROLLBACK", "PANEL_REDO"]
+            "FIX_QK", "UNCORRECTABLE", "ROLLBACK", "PANEL_REDO", "FIX_RW", "FIX_CW", "FIX_KW"]
 POLICY_EAGER, POLICY_PAPER = 0, 1
 MAX_EVENTS = 256
 
@@ -129,11 +129,12 @@ def fortran(x):
 
 
 def make_opts(nb=0, abft=True, policy=POLICY_EAGER, c_thr=2.0, faults=(), report=None,
-              stop_after_panel=-1, dchk_out=None, stream=None, timing=False):
+              stop_after_panel=-1, dchk_out=None, stream=None, timing=False, weighted=False):
     o = Opts()
     lib().ft_opts_default(ctypes.byref(o))
     o.nb = nb
     o.abft = 1 if abft else 0
+    o.weighted = 1 if weighted else 0
     o.policy = policy
     o.c_thr = c_thr
     fl = list(faults)
