@@ -82,7 +82,14 @@ def test_bad_opts_rejected_without_gpu(ft):
     o.nb = 65
     assert ft.lib().ft_dgehrd(4, 1, 4, ctypes.c_void_p(8), 4, ctypes.c_void_p(8), ctypes.byref(o)) == -7
     o.nb = 0
+    o.weighted = 2  # 0 or 1
+    assert ft.lib().ft_dgehrd(4, 1, 4, ctypes.c_void_p(8), 4, ctypes.c_void_p(8), ctypes.byref(o)) == -7
     o.weighted = 1
+    o.abft = 0  # the weighted pair (NEXT-1) needs the checksums
+    assert ft.lib().ft_dgehrd(4, 1, 4, ctypes.c_void_p(8), 4, ctypes.c_void_p(8), ctypes.byref(o)) == -7
+    o.weighted = 0
+    o.abft = 1
+    o.timing = 3
     assert ft.lib().ft_dgehrd(4, 1, 4, ctypes.c_void_p(8), 4, ctypes.c_void_p(8), ctypes.byref(o)) == -7
 
 
