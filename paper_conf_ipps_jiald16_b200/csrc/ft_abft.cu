@@ -633,6 +633,58 @@ cudaError_t ft_ckpt_w(double *Aw, int64_t ldw, int n, double *ck, int restore, c
     return cudaGetLastError();
 }
 
+// ---------------------------------------------------------------------------
+// device-side decision of the final verification (a12 / P:278), fault-free path: from the full
+// verification's syndromes, flag (ctl->fflag bit mode) whether anything needs the host decoder and
+// record the fault-free drift; the host only looks again when a bit is set (no extra round trip)
+// ---------------------------------------------------------------------------
+__global__ void k_final_flags(const double *Dr, const double *Dc, const double *sums, const double *kap, int n,
+                              int mode, FtCtl *ctl) {
+    if (ctl->halt) return;
+    __shared__ double wm[32];
+    __shared__ int wf[32];
+    const double unit = (double)n * EPS * (mode == 0 ? ctl->normF : sqrt((double)n));
+    const double tau = ctl->c_thr * unit, tauS = tau * sqrt((double)(n > 1 ? n : 1));
+    double mx = 0.0;
+    int fl = 0;
+    for (int i = threadIdx.x; i < n; i += blockDim.x) {
+        const double a = Dr[i], b = Dc[i];
+        if (not_within(a, tau)) fl = 1;
+        else mx = fmax(mx, fabs(a));
+        if (not_within(b, tau)) fl = 1;
+        else mx = fmax(mx, fabs(b));
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        mx = fmax(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+        fl |= __shfl_xor_sync(0xffffffffu, fl, o);
+    }
+    if ((threadIdx.x & 31) == 0) {
+        wm[threadIdx.x >> 5] = mx;
+        wf[threadIdx.x >> 5] = fl;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        for (int w = 0; w < (int)(blockDim.x >> 5); w++) {
+            mx = fmax(mx, wm[w]);
+            fl |= wf[w];
+        }
+        const double k = *kap;
+        if (not_within(sums[0] - k, tauS) || not_within(sums[1] - k, tauS)) fl = 1;
+        if (fl) ctl->fflag |= 1 << mode;
+        if (mode == 0 && unit > 0.0) {
+            const double rel = mx / unit;
+            atomicMax(&ctl->drift_bits, (unsigned long long)__double_as_longlong(rel));
+        }
+    }
+}
+cudaError_t ft_final_flags(const double *Dr, const double *Dc, const double *sums, const double *kap, int n, int mode,
+                           FtCtl *ctl, cudaStream_t s) {
+    g_ft_launches++;
+    k_final_flags<<<1, 1024, 0, s>>>(Dr, Dc, sums, kap, n, mode, ctl);
+    return cudaGetLastError();
+}
+
 // one block per fix: explicit sum excluding the bad element
 __global__ void k_fix(double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdone, int mode, double *r,
                       int64_t rinc, double *c, int64_t cinc, double *kappa, const FtFix *fixes, double *deltas) {

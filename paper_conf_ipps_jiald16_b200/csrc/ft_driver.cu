@@ -78,7 +78,9 @@ const double kEps = 2.220446049250313e-16;
 // workspace (cached per device, grown on demand)
 // ---------------------------------------------------------------------------
 constexpr int kMaxWsplit = FT_WSPLIT_MAX;
-constexpr int kYtopRows = 296 * 64;  // max (Y_top splits x rows) kept in ypart
+// Y_top split partials: up to kYtopSplits x (n+1) rows (or 296 x 64 rows for small n) kept in ypart
+constexpr int kYtopSplits = 16;
+int64_t ytop_rows_cap(int n) { return std::max<int64_t>(296 * 64, (int64_t)kYtopSplits * (n + 1)); }
 
 struct Work {
     int n_cap = -1;
@@ -190,8 +192,8 @@ int get_work(int n, Work **out) {
     A(dalloc(&w.Dr, (size_t)ldw, b));
     A(dalloc(&w.Dc, (size_t)ldw, b));
     A(dalloc(&w.sums, 8, b));
-    A(dalloc(&w.ypart, (size_t)kYtopRows * FT_NBMAX, b));
-    A(dalloc(&w.rowpart, (size_t)kYtopRows, b));
+    A(dalloc(&w.ypart, (size_t)ytop_rows_cap(n) * FT_NBMAX, b));
+    A(dalloc(&w.rowpart, (size_t)ytop_rows_cap(n), b));
     A(dalloc(&w.scratch, (size_t)64 * ((n + 255) / 256) + 8, b));
     // row-sum partials of the verification ([64][ldw]) / Gram partials of Q formation's DLARFT
     A(dalloc(&w.linepart, (size_t)std::max<int64_t>(64 * ldw, 4096 * ((int64_t)n / 64 + 2)), b));
@@ -725,8 +727,10 @@ int enqueue_panel(Call &C, int t) {
     y.panel = t;
     int nm = (k + 1 + 63) / 64;
     int nkt = (C.ihi - k - 1 + 31) / 32;
-    int ns = std::max(1, std::min({(2 * w.nsm) / nm, nkt / 2, 64}));
-    while ((int64_t)ns * (k + 1) > kYtopRows) ns--;
+    // splits over the long inner dimension: about ytop_f CTAs per SM in total (4 warps each)
+    static const int ytop_f = getenv("FT_YTOP_F") ? atoi(getenv("FT_YTOP_F")) : 12;  // measured: 2 -> 12 saves 42 ms at C3
+    int ns = std::max(1, std::min({(ytop_f * w.nsm) / nm, nkt / 2, 64}));
+    while ((int64_t)ns * (k + 1) > ytop_rows_cap(w.n_cap)) ns--;
     y.nsplit = std::max(ns, 1);
     if (!C.fused_ytop) CK(ft_launch_ytop(y, C.s));
     // weighted pair: rows n+1 of V and Y (w^T V, c_w V T), part of the panel's output
@@ -1146,6 +1150,25 @@ int enqueue_start(Call &C, const double *dA, int lda) {
     return 0;
 }
 
+// final verification of the finished H (a12) and of the Householder vectors, enqueued with
+// the panels: syndromes and the flag / drift decision on the device (k_final_flags); the host decoder
+// runs only if a flag is set
+int enqueue_final(Call &C) {
+    Work &w = *C.w;
+    const int n = C.n;
+    const int64_t ldw = w.ldw;
+    const int cdone = std::max(C.ihi - 1, C.ilo - 1);
+    const int sp = span_begin(C, TC_VERIFY);
+    CK(ft_full_verify(w.Aw, ldw, n, C.ilo, C.ihi, cdone, 0, w.Aw + (int64_t)n * ldw, 1, w.Aw + n, ldw, nullptr, w.Dr,
+                      w.Dc, w.sums, w.linepart, C.s));
+    CK(ft_final_flags(w.Dr, w.Dc, w.sums, w.Aw + n + (int64_t)n * ldw, n, 0, w.ctl, C.s));
+    CK(ft_full_verify(w.Aw, ldw, n, C.ilo, C.ihi, cdone, 1, w.Qr, 1, w.Qc, 1, nullptr, w.Dr, w.Dc, w.sums,
+                      w.linepart, C.s));
+    CK(ft_final_flags(w.Dr, w.Dc, w.sums, w.Qc + n, n, 1, w.ctl, C.s));
+    span_end(C, sp);
+    return 0;
+}
+
 int validate(int n, int ilo, int ihi, const void *A, int lda, const void *tau, const ft_opts *o) {
     if (n < 0) return -1;
     if (ilo < 1 || ilo > std::max(1, n)) return -2;
@@ -1215,6 +1238,9 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
                            !g_panel_path && g_left_fold &&
                            !getenv("FT_NO_GRAPH");
     bool launched = false;
+    // the fault-free final verification's decision is taken on the device (not for the weighted pair,
+    // whose final verification always runs the host decoder v3)
+    const bool dev_final = C.abft && !C.weighted && o.stop_after_panel < 0;
     if (graphable) {
         int dev = 0;
         CK(cudaGetDevice(&dev));
@@ -1237,6 +1263,7 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
                 C.s = w.cap_stream;
                 rc2 = enqueue_start(C, dA, lda);
                 for (int t = 0; t < last && !rc2; t++) rc2 = enqueue_panel(C, t);
+                if (!rc2 && dev_final) rc2 = enqueue_final(C);
                 if (C.hA && !rc2) {  // join the copy stream back into the capture
                     if (cudaEventRecord(w.copy_ev, w.copy_stream) != cudaSuccess ||
                         cudaStreamWaitEvent(w.cap_stream, w.copy_ev, 0) != cudaSuccess)
@@ -1269,12 +1296,18 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
     }
     int t0 = launched ? last : 0, attempts = 0;
     info = 0;
+    FtCtl h;
+    bool final_enqueued = launched && dev_final;  // the captured graph holds it
     while (true) {
         for (int t = t0; t < last; t++) {
             rc = enqueue_panel(C, t);
             if (rc) return rc;
         }
-        FtCtl h;
+        if (o.stop_after_panel < 0 && !final_enqueued) {
+            if (inject_at(C, -1, FT_PHASE_AT_END)) return FT_E_CUDA;
+            if (dev_final && enqueue_final(C)) return FT_E_CUDA;
+        }
+        final_enqueued = false;
         CK(cudaMemcpyAsync(&h, w.ctl, sizeof(FtCtl), cudaMemcpyDeviceToHost, s));
         CK(cudaStreamSynchronize(s));
         if (!h.halt) break;
@@ -1292,15 +1325,16 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
         if (rc) return rc;
         t0 = h.halt_panel;
     }
-    if (info == 0 && o.stop_after_panel < 0) {
-        inject_at(C, -1, FT_PHASE_AT_END);
-        if (C.abft) {
-            // final verification of the finished H (a12) and of the Householder vectors
+    if (info == 0 && o.stop_after_panel < 0 && C.abft) {
+        // final verification (a12): the host decoder only where the device flagged (or always
+        // for the weighted pair)
+        const bool doH = !dev_final || (h.fflag & 1), doQ = !dev_final || (h.fflag & 2);
+        if (doH || doQ) {
             bool found = false;
             const int cdone = std::max(ihi - 1, ilo - 1);
             const int sp = span_begin(C, TC_VERIFY);
-            int r1 = verify_and_correct(C, -1, cdone, 0, &found);
-            if (r1 == 0) r1 = verify_and_correct(C, -1, cdone, 1, &found);
+            int r1 = doH ? verify_and_correct(C, -1, cdone, 0, &found) : 0;
+            if (r1 == 0 && doQ) r1 = verify_and_correct(C, -1, cdone, 1, &found);
             span_end(C, sp);
             if (r1 == FT_E_UNCORRECTABLE) info = r1;
             else if (r1) return r1;

@@ -46,6 +46,7 @@ struct FtCtl {
     // update launch turns it into a halt of stage 3 (roll back the right update, redo the panel)
     double tchk[64];
     int tbad;
+    int fflag;  // device-side final verification: bit 0 H, bit 1 Q needs the host decoder
     double inj_delta[FT_MAXFAULTS];
     int inj_done[FT_MAXFAULTS];
 };
@@ -213,6 +214,8 @@ cudaError_t ft_full_verify(const double *Aw, int64_t ldw, int n, int ilo, int ih
 // 5 refresh r_w(i), 6 refresh c_w(j), 7 e^T L w = sum r_w, 8 w^T L e = sum c_w
 struct FtFix { int64_t i, j; int kind; int pad; };
 cudaError_t ft_encode_w(double *Aw, int64_t ldw, int n, double *linepart, cudaStream_t s);
+cudaError_t ft_final_flags(const double *Dr, const double *Dc, const double *sums, const double *kap, int n, int mode,
+                           FtCtl *ctl, cudaStream_t s);
 cudaError_t ft_full_verify_w(const double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdone, const double *rw,
                              const double *cw, int64_t cinc, double *Drw, double *Dcw, double *linepart,
                              cudaStream_t s);
