@@ -95,6 +95,41 @@ FT_DEV void cp_async_wait() {
     asm volatile("cp.async.wait_group %0;\n" ::"n"(N) : "memory");
 }
 
+// ---------------------------------------------------------------------------
+// Bulk asynchronous copies (the TMA unit's 1-D cp.async.bulk, SASS UBLKCP) completing on an
+// mbarrier transaction count: one lane moves a whole contiguous column segment of an operand tile
+// into its (padded, bank-conflict-free) row of shared memory.  src, dst 16-byte aligned, bytes a
+// multiple of 16.
+// ---------------------------------------------------------------------------
+FT_DEV unsigned smem_u32(const void *p) { return (unsigned)__cvta_generic_to_shared(p); }
+FT_DEV void mbar_init(unsigned long long *bar, unsigned count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;\n" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+FT_DEV void mbar_fence_init() { asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory"); }
+// generic-proxy accesses of this thread (made visible by a preceding bar.sync) before async-proxy writes
+FT_DEV void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory"); }
+FT_DEV void mbar_expect_tx(unsigned long long *bar, unsigned bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(smem_u32(bar)), "r"(bytes)
+                 : "memory");
+}
+FT_DEV void bulk_g2s(void *dst, const void *src, unsigned bytes, unsigned long long *bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];\n" ::"r"(
+                     smem_u32(dst)),
+                 "l"(src), "r"(bytes), "r"(smem_u32(bar))
+                 : "memory");
+}
+FT_DEV void mbar_wait(unsigned long long *bar, unsigned parity) {
+    asm volatile(
+        "{\n"
+        ".reg .pred p;\n"
+        "WAIT_%=:\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+        "@!p bra WAIT_%=;\n"
+        "}\n" ::"r"(smem_u32(bar)),
+        "r"(parity)
+        : "memory");
+}
+
 // element coordinates owned by this lane in fragment (mi, ni), v = 0/1
 FT_DEV int frag_row(int mi) { return mi * 8 + ((threadIdx.x & 31) >> 2); }
 FT_DEV int frag_col(int ni, int v) { return ni * 8 + 2 * (threadIdx.x & 3) + v; }

@@ -170,13 +170,37 @@ __global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
     double wacc[NJ][2];
 #pragma unroll
     for (int a = 0; a < NJ; a++) wacc[a][0] = wacc[a][1] = 0.0;
+    cp_async_commit();  // the Vc strip
 
-    // pipeline invariant at the top of tile tt: groups [Ys(tt), Vr(tt)] in flight
+    // Y / V row tiles: bulk copies (TMA, one column segment per lane of warp 0) into the padded tiles,
+    // completing on one mbarrier per tile buffer (parity = use count & 1).  Ys columns k >= K meet
+    // zero Vc entries and every Vr row meets the W pass (masked rows are zero there), so those words
+    // start as zeros (stale shared memory could hold NaN patterns); later tiles leave finite V rows
+    __shared__ __align__(8) unsigned long long ybar, vbar;
+    if (tid == 0) {
+        mbar_init(&ybar, 1);
+        mbar_init(&vbar, 1);
+        mbar_fence_init();
+    }
+    if (K < KT && p.do_right)
+        for (int i = tid; i < (KT - K) * SK; i += UT) S.Ys[K + i / SK][i % SK] = 0.0;
+    if (do_w)
+        for (int i = tid; i < KT * SK; i += UT) S.Vr[i / SK][i % SK] = 0.0;
+    __syncthreads();
+    // issued by all eight warps (lanes 0..7 of warp w: columns 8w..8w+7), so no warp stalls its
+    // barrier partners on a long serial issue; tid 0's arrive carries the expected byte count
+    auto issue_tile = [&](double (*T)[SK], const double *M, int r, unsigned long long *bar) {
+        const unsigned bytes = (unsigned)min(UB, (int)(p.ldw - r)) * 8u;
+        const int kk = warp * 8 + lane;
+        if (lane < 8 && kk < K) {
+            fence_proxy_async();  // the buffer's earlier reads (ordered by the last bar.sync) precede the copies
+            bulk_g2s(&T[kk][0], M + (int64_t)kk * p.ldw + r, bytes, bar);
+        }
+        if (tid == 0) mbar_expect_tx(bar, bytes * (unsigned)K);
+    };
     if (t0 < t1) {
-        if (p.do_right) issue_ktile<KT>(S.Ys, p.Y, p.ldw, rbase + t0 * UB, r_hi, K);
-        cp_async_commit();
-        if (do_w) issue_ktile<KT>(S.Vr, p.V, p.ldw, rbase + t0 * UB, r_hi, K);
-        cp_async_commit();
+        if (p.do_right) issue_tile(S.Ys, p.Y, rbase + t0 * UB, &ybar);
+        if (do_w) issue_tile(S.Vr, p.V, rbase + t0 * UB, &vbar);
     }
     // C tile of tile tt into registers (16-byte loads; masked pairs at the edges)
     auto load_c = [&](int tt, double2 (&dst)[8]) {
@@ -202,9 +226,12 @@ __global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
             acc[ni][1] = sg * cn[ni].y;
         }
         if (tt + 1 < t1) load_c(tt + 1, cn);
-        cp_async_wait<1>();
-        __syncthreads();
-        if (tt == t0 && pre_abort()) return;
+        if (tt == t0) {
+            cp_async_wait<0>();  // the Vc strip
+            __syncthreads();
+            if (pre_abort()) return;
+        }
+        if (p.do_right) mbar_wait(&ybar, (unsigned)(tt - t0) & 1u);
         if (p.do_right) {
 #pragma unroll 4
             for (int k0 = 0; k0 < KT; k0 += 4) {
@@ -225,11 +252,9 @@ __global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
             }
         }
         __syncthreads();  // every warp is done with Ys(tt)
-        if (p.do_right && tt + 1 < t1) issue_ktile<KT>(S.Ys, p.Y, p.ldw, r + UB, r_hi, K);
-        cp_async_commit();
+        if (p.do_right && tt + 1 < t1) issue_tile(S.Ys, p.Y, r + UB, &ybar);
         if (do_w) {
-            cp_async_wait<1>();
-            __syncthreads();
+            mbar_wait(&vbar, (unsigned)(tt - t0) & 1u);
             // only rows in [wr_lo, wr_hi) take part in W
             const int wlo = max(lo, p.wr_lo), whi = min(hi, p.wr_hi);
 #pragma unroll
@@ -254,9 +279,8 @@ __global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
                 }
             }
             __syncthreads();  // every warp is done with Vr(tt)
-            if (tt + 1 < t1) issue_ktile<KT>(S.Vr, p.V, p.ldw, r + UB, r_hi, K);
+            if (tt + 1 < t1) issue_tile(S.Vr, p.V, r + UB, &vbar);
         }
-        cp_async_commit();
     }
     cp_async_wait<0>();
     if (t0 >= t1) {  // no tile: take the pre-update decision here (no strip counter on a halt)
@@ -509,14 +533,40 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
         if (tid == 0) p.pre_reset->nflag = 0;
     }
 
-    // W'^T for the strip: Wt [col][64] -> Wc[k][col] (asynchronous, with the first V tile)
+    // W'^T for the strip: Wt [col][64] -> Wc[k][col] (cp.async, joined before the first tile)
     for (int i = tid; i < KT * UB; i += UT) {
         const int cc = i / KT, kk = i % KT;
         const bool ok = kk < K && cc < ncols;
         cp_async8(&S.Wc[kk][cc], ok ? p.Wpart + (int64_t)(cb + cc) * FT_NBMAX + kk : p.Wpart, ok ? 8 : 0);
     }
-    if (t0 < t1) issue_ktile<KT>(S.Vr[0], p.V, p.ldw, rbase + t0 * UB, p.r_hi, K);
     cp_async_commit();
+    // V tiles: bulk copies (TMA, one 512-byte column segment per lane of warp 0) into the padded
+    // double buffer, completing on an mbarrier per buffer (parity = use count & 1).  Rows past the
+    // tile's copy extent only feed masked outputs; columns k >= K meet zero W' entries, so they are
+    // zeroed once (stale shared memory could hold NaN patterns)
+    __shared__ __align__(8) unsigned long long vbar[2];
+    if (tid == 0) {
+        mbar_init(&vbar[0], 1);
+        mbar_init(&vbar[1], 1);
+        mbar_fence_init();
+    }
+    if (K < KT)
+        for (int i = tid; i < 2 * (KT - K) * SK; i += UT) {
+            const int b = i / ((KT - K) * SK), rem = i % ((KT - K) * SK);
+            S.Vr[b][K + rem / SK][rem % SK] = 0.0;
+        }
+    __syncthreads();
+    auto issue_v = [&](int tt, int b) {  // all eight warps issue (lanes 0..7: columns 8w..8w+7)
+        const int r = rbase + tt * UB;
+        const unsigned bytes = (unsigned)min(UB, (int)(p.ldw - r)) * 8u;
+        const int kk = warp * 8 + lane;
+        if (lane < 8 && kk < K) {
+            fence_proxy_async();  // this buffer's earlier reads (ordered by the last bar.sync) precede the copies
+            bulk_g2s(&S.Vr[b][kk][0], p.V + (int64_t)kk * p.ldw + r, bytes, &vbar[b]);
+        }
+        if (tid == 0) mbar_expect_tx(&vbar[b], bytes * (unsigned)K);
+    };
+    if (t0 < t1) issue_v(t0, 0);
     // fold (ABFT): column n (r) rides with the last strip, row n (c) with the last row tile
     if (p.fold && tid < KT) {
         S.Wr[tid] = tid < K ? p.Wpart[(int64_t)p.n * FT_NBMAX + tid] : 0.0;
@@ -552,6 +602,8 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
             else es_c += __ldcg(p.A + en + (int64_t)(x - nr) * p.lda);
         }
     }
+    cp_async_wait<0>();
+    __syncthreads();  // every thread's part of W' landed
     for (int tt = t0; tt < t1; tt++) {
         const int st = (tt - t0) & 1;
         const int r = rbase + tt * UB;
@@ -568,10 +620,8 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
                 acc[mi][ni][0] = sg * c.x;
                 acc[mi][ni][1] = sg * c.y;
             }
-        if (tt + 1 < t1) issue_ktile<KT>(S.Vr[st ^ 1], p.V, p.ldw, r + UB, p.r_hi, K);
-        cp_async_commit();
-        cp_async_wait<1>();
-        __syncthreads();
+        if (tt + 1 < t1) issue_v(tt + 1, st ^ 1);  // released by the bar.sync that ended tile tt-1
+        mbar_wait(&vbar[st], (unsigned)((tt - t0) >> 1) & 1u);
 #pragma unroll 4
         for (int k0 = 0; k0 < KT; k0 += 4) {
             double a[2], b[4];
@@ -592,7 +642,7 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
                 const double x = sg * acc[mi][ni][0], y = sg * acc[mi][ni][1];
                 if (full) *reinterpret_cast<double2 *>(colp[mi] + row) = make_double2(x, y);
                 else store_pair(colp[mi], row, lo, hi, colok[mi], x, y);
-                if (p.endcheck && colok[mi]) {
+                if (p.endcheck && !p.fold && colok[mi]) {  // fold: r, c are written by the fold code below
                     const int gc = cb + cols[mi];
                     const bool in0 = row >= lo && row < hi, in1 = row + 1 >= lo && row + 1 < hi;
                     if (gc == en) {  // r entries (kappa = row n excluded)
@@ -625,9 +675,8 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
         }
         __syncthreads();  // Vr[st] is refilled two tiles later
     }
-    cp_async_wait<0>();
     if (fold_row) {  // c(cols) += sg V(n, :) W'(:, cols), and kappa with the last strip
-        __syncthreads();  // Wc landed (cp.async) for every thread
+        __syncthreads();
         const int cc = tid >> 2, q4 = tid & 3;
         double s0 = 0.0, s1 = 0.0, k0 = 0.0, k1 = 0.0;
 #pragma unroll
