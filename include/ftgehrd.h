@@ -159,11 +159,15 @@ int ft_dorghr(int n, int ilo, int ihi, const double *dA, int lda, const double *
  * sums are exchanged CTA by CTA through peer memory inside the persistent panel kernel
  * (no host collective per column); Y_top is a per-rank partial summed by a peer
  * allreduce; the block-reflector updates are rank-local.  tau is replicated on return.
- * Round-1 scope: ilo = 1, ihi = n, no fault plan, no stop hook (-7 otherwise); with
- * abft = 1 the checksums ride through every update and the finished H is verified
- * against them at the end -- report->detected counts flagged rows/columns,
- * report->max_drift_rel the largest discrepancy in units of n eps ||A||_F; correction
- * and rollback run on the single-GPU entry only.
+ * Scope: ilo = 1, ihi = n, no stop hook (-2 / -3 / -7 otherwise).  With abft = 1 the checksums
+ * ride through every update (r replicated, c with its columns); every iteration ends with the
+ * paper's sum check on rank-ordered allreduced sums, so every rank halts identically;
+ * the iteration is then added back (reverse computation), the checkpoint restored, the error
+ * located from the summed row sums and the gathered column discrepancies, and repaired by the
+ * owner of its column (R12 decoder); the finished H is verified and corrected at the end.
+ * Fault plans: sites A and C (j = the GLOBAL column; the owner's word) at BEFORE_PANEL,
+ * AFTER_RIGHT, AFTER_UPDATE and AT_END (-7 for the replicated r / kappa and the per-rank
+ * V, Y, T copies, and for AFTER_PANEL).
  *
  * Bootstrap (one process per GPU): ft_mgpu_setup allocates this rank's workspace,
  * including a peer-visible region, for matrices up to n_max and returns its CUDA IPC
@@ -184,6 +188,12 @@ int ft_dgehrd_mgpu(int n, int ilo, int ihi, double *dA_local, int lda_local, dou
  * measure the multi-GPU path on one GPU. */
 int ft_dgehrd_vranks(int n, int ilo, int ihi, double *const *dA_local, int lda_local,
                      double *const *dtau, int nranks, const ft_opts *opts);
+
+/* Bootstrap probe of the IPC mappings (no kernel): ft_mgpu_probe_put(v) writes v into slot `rank` of
+ * every rank's symmetric region through the peer mappings (ordinary copies); after a barrier between
+ * the processes, ft_mgpu_probe_get(out) reads this rank's nranks slots.  -9 before setup/connect. */
+int ft_mgpu_probe_put(double v);
+int ft_mgpu_probe_get(double *out);
 
 /* Release the multi-rank workspaces (virtual ranks and this process's rank). */
 void ft_mgpu_finalize(void);

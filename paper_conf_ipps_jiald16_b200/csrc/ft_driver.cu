@@ -387,6 +387,20 @@ Plan decode(int n, const std::vector<double> &Dr, const std::vector<double> &Dc,
     return P;
 }
 
+}  // namespace
+
+// the R12 decoder for other translation units (the multi-rank path, ft_mgpu.cu): status 0 clean,
+// 1 fixes planned, 2 uncorrectable
+int ft_host_decode(int n, const double *Dr, const double *Dc, double sr, double sc, double tau,
+                   std::vector<FtFix> *fixes) {
+    std::vector<double> r(Dr, Dr + n), c(Dc, Dc + n);
+    Plan P = decode(n, r, c, sr, sc, tau);
+    if (fixes) *fixes = P.fixes;
+    return P.status;
+}
+
+namespace {
+
 // ---------------------------------------------------------------------------
 // one call's state
 // ---------------------------------------------------------------------------

@@ -155,24 +155,35 @@ __global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
     const int t0 = (int)((long long)blockIdx.y * nrt / gridDim.y);
     const int t1 = (int)((long long)(blockIdx.y + 1) * nrt / gridDim.y);
     constexpr int NJ = KT / 8;
-    const int wcol = warp * 8 + lr;  // this lane's column inside the strip (D row)
-    const bool colok = wcol < ncols;
-    double *colp = p.A + (int64_t)(cb + (colok ? wcol : 0)) * p.lda;
+    // warp tile: 16 columns x 32 rows (warp (wc, wr): columns wc*16.., rows wr*32.. of each tile):
+    // per k step 2 + 4 fragment loads feed 8 DMMA (the W pass: 4 shuffles + 8 loads feed 16)
+    const int wc = warp & 3, wr = warp >> 2;
+    int cols2[2];
+    bool colok2[2];
+    double *colp2[2];
+#pragma unroll
+    for (int mi = 0; mi < 2; mi++) {
+        cols2[mi] = wc * 16 + mi * 8 + lr;
+        colok2[mi] = cols2[mi] < ncols;
+        colp2[mi] = p.A + (int64_t)(cb + (colok2[mi] ? cols2[mi] : 0)) * p.lda;
+    }
 
     if (p.do_right) {  // V(cols, :) once per CTA (plain loads: cb may be odd)
-        for (int i = tid; i < KT * UB; i += UT) {  // asynchronous: joins the first Ys group
+        for (int i = tid; i < KT * UB; i += UT) {
             const int kk = i / UB, cc = i % UB;
             const bool ok = kk < K && cc < ncols;
             const int vrow = ft_cmap(cb + cc, p.cm_G, p.cm_rank, p.cm_nb, p.cm_ncl, p.cm_n);
             cp_async8(&S.Vc[kk][cc], ok ? p.V + vrow + (int64_t)kk * p.ldw : p.V, ok ? 8 : 0);
         }
     }
-    double wacc[NJ][2];
+    double wacc[2][NJ][2];
 #pragma unroll
-    for (int a = 0; a < NJ; a++) wacc[a][0] = wacc[a][1] = 0.0;
+    for (int mi = 0; mi < 2; mi++)
+#pragma unroll
+        for (int a = 0; a < NJ; a++) wacc[mi][a][0] = wacc[mi][a][1] = 0.0;
     cp_async_commit();  // the Vc strip
 
-    // Y / V row tiles: bulk copies (TMA, one column segment per lane of warp 0) into the padded tiles,
+    // Y / V row tiles: bulk copies (TMA, one column segment per lane) into the padded tiles,
     // completing on one mbarrier per tile buffer (parity = use count & 1).  Ys columns k >= K meet
     // zero Vc entries and every Vr row meets the W pass (masked rows are zero there), so those words
     // start as zeros (stale shared memory could hold NaN patterns); later tiles leave finite V rows
@@ -203,53 +214,63 @@ __global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
         if (do_w) issue_tile(S.Vr, p.V, rbase + t0 * UB, &vbar);
     }
     // C tile of tile tt into registers (16-byte loads; masked pairs at the edges)
-    auto load_c = [&](int tt, double2 (&dst)[8]) {
+    auto load_c = [&](int tt, double2 (&dst)[2][4]) {
         const int r = rbase + tt * UB;
         const int lo = max(r, r_lo), hi = min(r + UB, r_hi);
         const bool full = lo == r && hi == r + UB && ncols == UB;
 #pragma unroll
-        for (int ni = 0; ni < 8; ni++) {
-            const int row = r + ni * 8 + 2 * lc;
-            dst[ni] = full ? *reinterpret_cast<const double2 *>(colp + row) : load_pair(colp, row, lo, hi, colok);
-        }
+        for (int mi = 0; mi < 2; mi++)
+#pragma unroll
+            for (int ni = 0; ni < 4; ni++) {
+                const int row = r + wr * 32 + ni * 8 + 2 * lc;
+                dst[mi][ni] = full ? *reinterpret_cast<const double2 *>(colp2[mi] + row)
+                                   : load_pair(colp2[mi], row, lo, hi, colok2[mi]);
+            }
     };
-    double2 cn[8];  // the next tile's C, prefetched a whole tile ahead
+    double2 cn[2][4];  // the next tile's C, prefetched a whole tile ahead
     if (t0 < t1) load_c(t0, cn);
     for (int tt = t0; tt < t1; tt++) {
         const int r = rbase + tt * UB;
         const int lo = max(r, r_lo), hi = min(r + UB, r_hi);
         const bool full = lo == r && hi == r + UB && ncols == UB;  // interior tile: no masks
-        double acc[8][2];
+        double acc[2][4][2];
 #pragma unroll
-        for (int ni = 0; ni < 8; ni++) {
-            acc[ni][0] = sg * cn[ni].x;
-            acc[ni][1] = sg * cn[ni].y;
-        }
+        for (int mi = 0; mi < 2; mi++)
+#pragma unroll
+            for (int ni = 0; ni < 4; ni++) {
+                acc[mi][ni][0] = sg * cn[mi][ni].x;
+                acc[mi][ni][1] = sg * cn[mi][ni].y;
+            }
         if (tt + 1 < t1) load_c(tt + 1, cn);
         if (tt == t0) {
             cp_async_wait<0>();  // the Vc strip
             __syncthreads();
             if (pre_abort()) return;
         }
-        if (p.do_right) mbar_wait(&ybar, (unsigned)(tt - t0) & 1u);
         if (p.do_right) {
+            mbar_wait(&ybar, (unsigned)(tt - t0) & 1u);
 #pragma unroll 4
             for (int k0 = 0; k0 < KT; k0 += 4) {
-                const double a = S.Vc[k0 + lc][wcol];
-                double b[8];
+                double a[2], b[4];
 #pragma unroll
-                for (int ni = 0; ni < 8; ni++) b[ni] = S.Ys[k0 + lc][ni * 8 + lr];
+                for (int mi = 0; mi < 2; mi++) a[mi] = S.Vc[k0 + lc][wc * 16 + mi * 8 + lr];
 #pragma unroll
-                for (int ni = 0; ni < 8; ni++) dmma_8x8x4(acc[ni][0], acc[ni][1], a, b[ni]);
+                for (int ni = 0; ni < 4; ni++) b[ni] = S.Ys[k0 + lc][wr * 32 + ni * 8 + lr];
+#pragma unroll
+                for (int mi = 0; mi < 2; mi++)
+#pragma unroll
+                    for (int ni = 0; ni < 4; ni++) dmma_8x8x4(acc[mi][ni][0], acc[mi][ni][1], a[mi], b[ni]);
             }
 #pragma unroll
-            for (int ni = 0; ni < 8; ni++) {
-                acc[ni][0] *= sg;
-                acc[ni][1] *= sg;
-                const int row = r + ni * 8 + 2 * lc;
-                if (full) *reinterpret_cast<double2 *>(colp + row) = make_double2(acc[ni][0], acc[ni][1]);
-                else store_pair(colp, row, lo, hi, colok, acc[ni][0], acc[ni][1]);
-            }
+            for (int mi = 0; mi < 2; mi++)
+#pragma unroll
+                for (int ni = 0; ni < 4; ni++) {
+                    acc[mi][ni][0] *= sg;
+                    acc[mi][ni][1] *= sg;
+                    const int row = r + wr * 32 + ni * 8 + 2 * lc;
+                    if (full) *reinterpret_cast<double2 *>(colp2[mi] + row) = make_double2(acc[mi][ni][0], acc[mi][ni][1]);
+                    else store_pair(colp2[mi], row, lo, hi, colok2[mi], acc[mi][ni][0], acc[mi][ni][1]);
+                }
         }
         __syncthreads();  // every warp is done with Ys(tt)
         if (p.do_right && tt + 1 < t1) issue_tile(S.Ys, p.Y, r + UB, &ybar);
@@ -258,24 +279,31 @@ __global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
             // only rows in [wr_lo, wr_hi) take part in W
             const int wlo = max(lo, p.wr_lo), whi = min(hi, p.wr_hi);
 #pragma unroll
-            for (int ni = 0; ni < 8; ni++) {
-                const int row = r + ni * 8 + 2 * lc;
-                if (row < wlo || row >= whi) acc[ni][0] = 0.0;
-                if (row + 1 < wlo || row + 1 >= whi) acc[ni][1] = 0.0;
-            }
-            // W^T(cols, j) += C_new^T(cols, rows) V(rows, j); the A fragment (col lr, row
-            // ks*4 + lc) sits in lane lr*4 + 2h + lc/2, element lc & 1 (ks = 2 ni + h)
+            for (int mi = 0; mi < 2; mi++)
 #pragma unroll
-            for (int ks = 0; ks < 16; ks++) {
+                for (int ni = 0; ni < 4; ni++) {
+                    const int row = r + wr * 32 + ni * 8 + 2 * lc;
+                    if (row < wlo || row >= whi) acc[mi][ni][0] = 0.0;
+                    if (row + 1 < wlo || row + 1 >= whi) acc[mi][ni][1] = 0.0;
+                }
+            // W^T(cols, j) += C_new^T(cols, rows) V(rows, j) over this warp's 32 rows; the A fragment
+            // (col lr, row ks*4 + lc) sits in lane lr*4 + 2h + lc/2, element lc & 1 (ks = 2 ni + h)
+#pragma unroll
+            for (int ks = 0; ks < 8; ks++) {
                 const int ni = ks >> 1, h = ks & 1;
                 const int src = lr * 4 + 2 * h + (lc >> 1);
-                const double x0 = __shfl_sync(0xffffffffu, acc[ni][0], src);
-                const double x1 = __shfl_sync(0xffffffffu, acc[ni][1], src);
-                const double a = (lc & 1) ? x1 : x0;
+                double a[2];
+#pragma unroll
+                for (int mi = 0; mi < 2; mi++) {
+                    const double x0 = __shfl_sync(0xffffffffu, acc[mi][ni][0], src);
+                    const double x1 = __shfl_sync(0xffffffffu, acc[mi][ni][1], src);
+                    a[mi] = (lc & 1) ? x1 : x0;
+                }
 #pragma unroll
                 for (int nj = 0; nj < NJ; nj++) {
-                    const double b = S.Vr[nj * 8 + lr][ks * 4 + lc];
-                    dmma_8x8x4(wacc[nj][0], wacc[nj][1], a, b);
+                    const double b = S.Vr[nj * 8 + lr][wr * 32 + ks * 4 + lc];
+#pragma unroll
+                    for (int mi = 0; mi < 2; mi++) dmma_8x8x4(wacc[mi][nj][0], wacc[mi][nj][1], a[mi], b);
                 }
             }
             __syncthreads();  // every warp is done with Vr(tt)
@@ -288,16 +316,32 @@ __global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
         if (pre_abort()) return;
     }
     if (do_w) {
-        // deterministic partial of this row split: Wpart[split][col][j]
+        // deterministic partial of this row split: Wpart[split][col][j]; the two row warps of each
+        // column group meet in shared memory first (wr = 1 stores, wr = 0 adds and writes out)
         double *Wp = p.Wpart + (int64_t)blockIdx.y * p.wsplit_stride;
-        if (colok)
+        double *red = &S.Ys[0][0];  // [col][64] scratch: every copy into Ys has completed
+        __syncthreads();
+        if (wr == 1)
 #pragma unroll
-            for (int nj = 0; nj < NJ; nj++)
+            for (int mi = 0; mi < 2; mi++)
 #pragma unroll
-                for (int v = 0; v < 2; v++) {
-                    const int jj = nj * 8 + 2 * lc + v;
-                    if (jj < K) Wp[(int64_t)(cb + wcol) * FT_NBMAX + jj] = wacc[nj][v];
-                }
+                for (int nj = 0; nj < NJ; nj++)
+#pragma unroll
+                    for (int v = 0; v < 2; v++) red[cols2[mi] * FT_NBMAX + nj * 8 + 2 * lc + v] = wacc[mi][nj][v];
+        __syncthreads();
+        if (wr == 0)
+#pragma unroll
+            for (int mi = 0; mi < 2; mi++)
+                if (colok2[mi])
+#pragma unroll
+                    for (int nj = 0; nj < NJ; nj++)
+#pragma unroll
+                        for (int v = 0; v < 2; v++) {
+                            const int jj = nj * 8 + 2 * lc + v;
+                            if (jj < K)
+                                Wp[(int64_t)(cb + cols2[mi]) * FT_NBMAX + jj] =
+                                    wacc[mi][nj][v] + red[cols2[mi] * FT_NBMAX + jj];
+                        }
         if (p.Wt) {
             // the last CTA of the strip sums the partials (fixed order) and forms W' = op(T) W
             __shared__ int last;

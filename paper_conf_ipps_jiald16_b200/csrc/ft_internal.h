@@ -237,6 +237,13 @@ cudaError_t ft_set_identity(double *Q, int64_t ldq, int n, cudaStream_t s);
 cudaError_t ft_set_identity_aug(double *Q, int64_t ldq, int n, cudaStream_t s);
 cudaError_t ft_ctl_set_norm(FtCtl *ctl, double v, cudaStream_t s);
 
+#ifdef __cplusplus
+#include <vector>
+// the host R12 decoder (ft_driver.cu), shared with the multi-rank path: 0 clean, 1 fixes, 2 refused
+int ft_host_decode(int n, const double *Dr, const double *Dc, double sr, double sc, double tau,
+                   std::vector<FtFix> *fixes);
+#endif
+
 extern int64_t g_ft_launches;
 extern int64_t g_ft_wide_launches;  // launches of the two-reduction (wide) panel kernel
 

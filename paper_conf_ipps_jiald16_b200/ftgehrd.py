@@ -83,6 +83,8 @@ def lib():
         L.ft_mgpu_connect.argtypes = [ctypes.POINTER(IpcHandle), i32, i32]
         L.ft_dgehrd_vranks.argtypes = [i32, i32, i32, ctypes.POINTER(vp), i32, ctypes.POINTER(vp), i32,
                                        ctypes.POINTER(Opts)]
+        L.ft_mgpu_probe_put.argtypes = [ctypes.c_double]
+        L.ft_mgpu_probe_get.argtypes = [vp]
         L.ft_strerror.argtypes = [i32]
         L.ft_strerror.restype = ctypes.c_char_p
         L.ft_version.restype = ctypes.c_char_p
@@ -94,6 +96,7 @@ def lib():
 
 EXPORTS = ["ft_opts_default", "ft_dgehrd", "ft_dgehrd_host", "ft_dorghr", "ft_dgehrd_mgpu",
            "ft_mgpu_setup", "ft_mgpu_connect", "ft_dgehrd_vranks", "ft_mgpu_finalize",
+           "ft_mgpu_probe_put", "ft_mgpu_probe_get",
            "ft_strerror", "ft_finalize", "ft_version", "ft_launch_count"]
 
 
@@ -285,10 +288,11 @@ def _slab_ld(S, n):
     return max(S.stride(1) if S.shape[1] > 1 else n, n, 1)
 
 
-def dgehrd_vranks(slabs: list, nb: int = 0, abft: bool = True, taus=None, stream=None):
+def dgehrd_vranks(slabs: list, nb: int = 0, abft: bool = True, taus=None, stream=None, faults=(), c_thr=2.0):
     """Sharded reduction with len(slabs) VIRTUAL ranks on the current GPU (ft_dgehrd_vranks).
 
     slabs: the ranks' n x ncols CUDA float64 column-major slabs (modified in place).
+    faults: (panel, phase, site, i, J, bit) with J a GLOBAL column (sites A, C; the owner's word).
     Returns (taus, Result)."""
     import torch
     G = len(slabs)
@@ -305,7 +309,7 @@ def dgehrd_vranks(slabs: list, nb: int = 0, abft: bool = True, taus=None, stream
     pa = (ctypes.c_void_p * G)(*[S.data_ptr() for S in slabs])
     pt = (ctypes.c_void_p * G)(*[t.data_ptr() for t in taus])
     rep = Report()
-    o = make_opts(nb=nb, abft=abft, report=rep, stream=stream)
+    o = make_opts(nb=nb, abft=abft, report=rep, stream=stream, faults=faults, c_thr=c_thr)
     info = lib().ft_dgehrd_vranks(n, 1, n, pa, lda, pt, G, ctypes.byref(o))
     return taus, Result(info, rep, rep.event_list())
 
@@ -326,7 +330,8 @@ def mgpu_init(n_max: int, group=None) -> None:
     info = lib().ft_mgpu_setup(n_max, rank, nranks, ctypes.byref(h))
     if info:
         raise RuntimeError(f"ft_mgpu_setup: {strerror(info)}")
-    hs = exchange_handles(h.bytes.ljust(64, b"\0")[:64], group)
+    # the raw 64 bytes (ctypes' c_char-array value would stop at the first NUL byte of the handle)
+    hs = exchange_handles(ctypes.string_at(ctypes.addressof(h), 64), group)
     arr = (IpcHandle * nranks)()
     for g, b in enumerate(hs):
         ctypes.memmove(ctypes.byref(arr[g]), b, 64)
@@ -335,7 +340,7 @@ def mgpu_init(n_max: int, group=None) -> None:
         raise RuntimeError(f"ft_mgpu_connect: {strerror(info)}")
 
 
-def dgehrd_mgpu(slab, rank: int, nranks: int, nb: int = 0, abft: bool = True, tau=None, stream=None):
+def dgehrd_mgpu(slab, rank: int, nranks: int, nb: int = 0, abft: bool = True, tau=None, stream=None, faults=()):
     """This rank's part of the sharded reduction (after mgpu_init). Returns (tau, Result)."""
     import torch
     n = slab.shape[0]
@@ -343,7 +348,7 @@ def dgehrd_mgpu(slab, rank: int, nranks: int, nb: int = 0, abft: bool = True, ta
     if tau is None:
         tau = torch.zeros(max(n - 1, 1), dtype=torch.float64, device=slab.device)
     rep = Report()
-    o = make_opts(nb=nb, abft=abft, report=rep, stream=stream)
+    o = make_opts(nb=nb, abft=abft, report=rep, stream=stream, faults=faults)
     info = lib().ft_dgehrd_mgpu(n, 1, n, ctypes.c_void_p(slab.data_ptr()), lda, ctypes.c_void_p(tau.data_ptr()),
                                 rank, nranks, ctypes.byref(o))
     return tau, Result(info, rep, rep.event_list())

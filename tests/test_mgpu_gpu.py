@@ -116,3 +116,77 @@ def test_vranks_bad_arguments():
     pt = (ctypes.c_void_p * 2)(*[s.data_ptr() for s in slabs])
     assert L.ft_dgehrd_vranks(n, 2, n, pa, n, pt, 2, ctypes.byref(o)) == -2   # ilo != 1 (round-1 scope)
     assert L.ft_dgehrd_vranks(n, 1, n, pa, n, pt, 9, ctypes.byref(o)) == -9   # > 8 ranks
+
+
+# ------------------------------------------------------------------ resilience on the sharded layout
+def run_vranks_faults(A, G, nb, faults):
+    n = A.shape[0]
+    dA = torch.from_numpy(A).cuda()
+    slabs = ft.shard(dA, nb, G)
+    taus, res = ft.dgehrd_vranks(slabs, nb=nb, faults=faults)
+    torch.cuda.synchronize()
+    return ft.unshard(slabs, n, nb).cpu().numpy(), [t.cpu().numpy()[: n - 1] for t in taus], res
+
+
+MG_FAULTS = [
+    (2, ft.PHASE_BEFORE_PANEL, ft.SITE_A, 150, 200, 55),   # trailing word: consumed by the panel, caught by the end check
+    (1, ft.PHASE_BEFORE_PANEL, ft.SITE_C, -1, 250, 52),    # the owner's column checksum
+    (3, ft.PHASE_AFTER_RIGHT, ft.SITE_A, 200, 260, 54),    # mid-update
+    (2, ft.PHASE_AFTER_UPDATE, ft.SITE_A, 170, 230, 57),
+    (0, ft.PHASE_AT_END, ft.SITE_A, 100, 150, 50),         # finished H, final verification
+    (4, ft.PHASE_BEFORE_PANEL, ft.SITE_A, 140, 140, 63),   # the panel's own column (sign)
+]
+
+
+@pytest.mark.parametrize("G", [2, 4, 8])
+@pytest.mark.parametrize("fault", MG_FAULTS, ids=lambda f: f"p{f[0]}-ph{f[1]}-s{f[2]}-{f[3]}-{f[4]}")
+def test_vranks_fault_detected_and_corrected(G, fault):
+    """SURVEY 8(e) resilience: the end-of-iteration check on rank-ordered allreduced sums halts every
+    rank identically; the iteration is added back (reverse computation), the checkpoint restored, the
+    error located from the summed row sums and the gathered column sums and repaired by the owner of
+    its column; the result meets the oracle bar."""
+    n, nb = 300, 32
+    A = synth.matrix(n)
+    Ag, taus, res = run_vranks_faults(A, G, nb, [fault])
+    assert res.info == 0, res.events
+    assert res.report.detected >= 1, res.events
+    fx = [(e[0], e[2], e[3]) for e in res.events if e[0].startswith("FIX")]
+    if fault[2] == ft.SITE_A:
+        assert ("FIX_DATA", fault[3], fault[4]) in fx, res.events
+    else:
+        assert ("FIX_C", -1, fault[4]) in fx, res.events
+    Ao, to = oracle.dgehd2(A)
+    assert rel(np.triu(Ag, -1), np.triu(Ao, -1)) <= TOL
+    assert np.abs(taus[0] - to).max() <= TOL * max(1.0, np.abs(to).max())
+
+
+@pytest.mark.parametrize("nfaults", [1, 10])
+def test_vranks_c5_style_fault_runs(nfaults):
+    """C5-style runs at 8 (virtual) GPUs: 1 and 10 soft errors per reduction, each in a different
+    iteration, drawn (seeded) over the live trailing block and the column checksums, bits from the
+    exponent / high mantissa; every one is corrected and the result meets the oracle bar."""
+    n, nb, G = 517, 32, 8
+    A = synth.matrix(n)
+    rng = np.random.default_rng(20160523 + nfaults)
+    faults = []
+    for q, t in enumerate(rng.choice(np.arange(1, (n - 2) // nb - 1), nfaults, replace=False)):
+        k = int(t) * nb
+        i = int(rng.integers(k + 2, n))
+        j = int(rng.integers(k + nb + 1, n))
+        site = ft.SITE_C if q % 4 == 3 else ft.SITE_A
+        faults.append((int(t), ft.PHASE_BEFORE_PANEL, site, i if site == ft.SITE_A else -1, j,
+                       int(rng.choice([52, 53, 54, 55, 56, 58, 60, 63]))))
+    Ag, taus, res = run_vranks_faults(A, G, nb, faults)
+    assert res.info == 0, res.events
+    assert res.report.detected >= nfaults // 2, res.events
+    Ao, to = oracle.dgehd2(A)
+    assert rel(np.triu(Ag, -1), np.triu(Ao, -1)) <= TOL
+
+
+def test_vranks_unsupported_fault_sites_rejected():
+    n = 128
+    slabs = ft.shard(torch.from_numpy(synth.matrix(n)).cuda(), 16, 2)
+    for f in [(1, ft.PHASE_BEFORE_PANEL, ft.SITE_R, 5, -1, 50), (1, ft.PHASE_AFTER_PANEL, ft.SITE_A, 40, 50, 50),
+              (1, ft.PHASE_BEFORE_PANEL, ft.SITE_Y, 40, 3, 50)]:
+        _, res = ft.dgehrd_vranks(slabs, nb=16, faults=[f])
+        assert res.info == -7
