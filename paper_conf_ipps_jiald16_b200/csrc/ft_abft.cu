@@ -685,9 +685,287 @@ cudaError_t ft_final_flags(const double *Dr, const double *Dc, const double *sum
     return cudaGetLastError();
 }
 
+// ---------------------------------------------------------------------------
+// R12 decoder v2 on the device (one block; written apart from the host copy in ft_driver.cu and
+// from the oracle's).  Never miscorrect: refuse whenever two explanations exist.  Input: the full
+// verification's syndromes D_r, D_c, the sums of r and c, kappa; output: status (0 clean, 1 fixes
+// planned, 2 uncorrectable, 3 too large for the device: the host decides), the fix list (the order
+// of the host decoder: data fixes, then r refreshes, then c refreshes) and the flagged counts.
+// ---------------------------------------------------------------------------
+#define DEC_T 256
+__device__ __forceinline__ bool d_bad(double d, double tau) { return !(fabs(d) <= tau); }
+__device__ __forceinline__ bool d_same(double a, double b, double tol) {
+    const bool fa = isfinite(a), fb = isfinite(b);
+    if (!fa || !fb) return !fa && !fb;
+    return fabs(a - b) <= tol;
+}
+// ordered compaction of {i < n : flagged(D[i])} into out (block-wide scan over contiguous chunks)
+__device__ int d_compact(const double *D, int n, double tau, int *out, int *scan) {
+    const int t = threadIdx.x, chunk = (n + DEC_T - 1) / DEC_T;
+    const int i0 = min(n, t * chunk), i1 = min(n, i0 + chunk);
+    int c = 0;
+    for (int i = i0; i < i1; i++) c += d_bad(D[i], tau);
+    scan[t] = c;
+    __syncthreads();
+    for (int o = 1; o < DEC_T; o <<= 1) {  // inclusive Hillis-Steele scan
+        const int v = t >= o ? scan[t - o] : 0;
+        __syncthreads();
+        scan[t] += v;
+        __syncthreads();
+    }
+    int pos = scan[t] - c;
+    for (int i = i0; i < i1; i++)
+        if (d_bad(D[i], tau)) out[pos++] = i;
+    __syncthreads();
+    const int total = scan[DEC_T - 1];
+    __syncthreads();
+    return total;
+}
+// members of S (size m) whose syndromes add up to target (|subset| <= 3), unique; block-parallel
+// over the first member.  Returns the subset size (0..3) into sub, or -1
+__device__ int d_explain(const int *S, int m, const double *D, double target, double tauS, int n, int *sub,
+                         int *hits, unsigned long long *best) {
+    if (d_same(target, 0.0, tauS)) return 0;
+    if (!isfinite(target)) {
+        int k = 0;
+        for (int a = 0; a < m; a++)
+            if (!isfinite(D[S[a]])) {
+                if (k == 3) return -1;
+                sub[k++] = S[a];
+            }
+        return k > 0 ? k : -1;
+    }
+    if (m > 256) return -1;
+    if (threadIdx.x == 0) {
+        *hits = 0;
+        *best = 0ull;
+    }
+    __syncthreads();
+    const double e2 = 2.0 * n * EPS;
+    for (int a = threadIdx.x; a < m; a += DEC_T) {
+        const double da = D[S[a]];
+        if (d_same(da, target, tauS + e2 * fabs(da))) {
+            atomicAdd(hits, 1);
+            atomicExch(best, (unsigned long long)(a + 1));
+        }
+        for (int b = a + 1; b < m; b++) {
+            const double db = D[S[b]];
+            if (d_same(da + db, target, tauS + e2 * (fabs(da) + fabs(db)))) {
+                atomicAdd(hits, 1);
+                atomicExch(best, (unsigned long long)(a + 1) | ((unsigned long long)(b + 1) << 20));
+            }
+            for (int c = b + 1; c < m; c++) {
+                const double dc = D[S[c]];
+                if (d_same(da + db + dc, target, tauS + e2 * (fabs(da) + fabs(db) + fabs(dc)))) {
+                    atomicAdd(hits, 1);
+                    atomicExch(best, (unsigned long long)(a + 1) | ((unsigned long long)(b + 1) << 20) |
+                                         ((unsigned long long)(c + 1) << 40));
+                }
+            }
+        }
+    }
+    __syncthreads();
+    const int h = *hits;
+    const unsigned long long bb = *best;
+    __syncthreads();
+    if (h != 1) return -1;
+    int k = 0;
+    for (int q = 0; q < 3; q++) {
+        const int v = (int)((bb >> (20 * q)) & 0xFFFFF);
+        if (v) sub[k++] = S[v - 1];
+    }
+    return k;
+}
+__global__ void __launch_bounds__(DEC_T) k_decode(const double *Dr, const double *Dc, const double *sums,
+                                                  const double *kap, int n, int mode, const FtCtl *ctl, int *idx,
+                                                  FtFix *fixes, int cap, FtDecOut *out) {
+    __shared__ int scan[DEC_T];
+    __shared__ int hits;
+    __shared__ unsigned long long best;
+    __shared__ int Rc[3], Cc[3], nRc, nCc;
+    const double tau = ctl->c_thr * (double)n * EPS * (mode == 0 ? ctl->normF : sqrt((double)n));
+    const double tauS = tau * sqrt((double)(n > 1 ? n : 1));
+    int *R = idx, *C = idx + n;
+    const int nR = d_compact(Dr, n, tau, R, scan);
+    const int nC = d_compact(Dc, n, tau, C, scan);
+    const double sr = sums[0] - *kap, sc = sums[1] - *kap;
+    const bool sr0 = d_same(sr, 0.0, tauS), sc0 = d_same(sc, 0.0, tauS);
+    const bool amb = !sr0 && !sc0 && d_same(sr, sc, tauS);
+    if (threadIdx.x == 0) {
+        out->nR = nR;
+        out->nC = nC;
+        out->nfix = 0;
+        out->status = 2;
+    }
+    if (nR == 0 && nC == 0) {
+        if (threadIdx.x == 0) {
+            if (sr0 && sc0) out->status = 0;
+            else if (amb) {  // only the corner: both sums off by the same amount
+                fixes[0] = FtFix{-1, -1, 4, 0};
+                out->nfix = 1;
+                out->status = 1;
+            }
+        }
+        return;
+    }
+    if (amb) return;  // equally explained by "corner + data errors": refuse
+    {
+        int sub[3];
+        const int k1 = d_explain(R, nR, Dr, sr, tauS, n, sub, &hits, &best);
+        if (threadIdx.x == 0) {
+            nRc = k1;
+            for (int q = 0; q < 3; q++) Rc[q] = q < k1 ? sub[q] : -1;
+        }
+        __syncthreads();
+        const int k2 = d_explain(C, nC, Dc, sc, tauS, n, sub, &hits, &best);
+        if (threadIdx.x == 0) {
+            nCc = k2;
+            for (int q = 0; q < 3; q++) Cc[q] = q < k2 ? sub[q] : -1;
+        }
+        __syncthreads();
+    }
+    if (threadIdx.x != 0) return;
+    if (nRc < 0 || nCc < 0) return;
+    auto inset = [](int v, const int *s3, int m) {
+        for (int q = 0; q < m; q++)
+            if (s3[q] == v) return true;
+        return false;
+    };
+    int rc[3] = {Rc[0], Rc[1], Rc[2]}, cc[3] = {Cc[0], Cc[1], Cc[2]};
+    int nrc = nRc, ncc = nCc;
+    int nRd = 0, nCd = 0;
+    for (int a = 0; a < nR; a++) nRd += !inset(R[a], rc, nrc);
+    for (int b = 0; b < nC; b++) nCd += !inset(C[b], cc, ncc);
+    // a flagged line without a flagged partner is a checksum word whose syndrome hid inside the
+    // sum tolerance (tau < |d| <= tau sqrt(n)): accept if the whole set explains s_r / s_c
+    auto whole_set = [&](const int *S, int m, const double *D, double target) {
+        if (m > 3) return false;
+        double sum = 0.0, sa = 0.0;
+        for (int a = 0; a < m; a++) {
+            const double d = D[S[a]];
+            if (!(fabs(d) <= tauS)) return false;
+            sum += d;
+            sa += fabs(d);
+        }
+        return d_same(sum, target, tauS + 2.0 * n * EPS * sa);
+    };
+    if (nRd > 0 && nCd == 0 && whole_set(R, nR, Dr, sr)) {
+        nrc = nR;
+        for (int a = 0; a < nR; a++) rc[a] = R[a];
+        nRd = 0;
+    }
+    if (nCd > 0 && nRd == 0 && whole_set(C, nC, Dc, sc)) {
+        ncc = nC;
+        for (int b = 0; b < nC; b++) cc[b] = C[b];
+        nCd = 0;
+    }
+    if ((nRd == 0) != (nCd == 0)) return;
+    int nf = 0;
+    auto push = [&](int64_t i, int64_t j, int kind) {
+        if (nf < cap) fixes[nf] = FtFix{i, j, kind, 0};
+        nf++;
+    };
+    auto pair_tol = [&](double a, double b) { return 2.0 * tau + 2.0 * n * EPS * (fabs(a) + fabs(b)); };
+    // the data rows / columns (flagged, not checksum words), in index order
+    auto nth_d = [&](const int *S, int m, const int *s3, int m3, int q) {
+        for (int a = 0, c = 0; a < m; a++)
+            if (!inset(S[a], s3, m3)) {
+                if (c == q) return S[a];
+                c++;
+            }
+        return -1;
+    };
+    if (nRd > 0) {
+        if (nRd == 1 && nCd == 1) {
+            const int i = nth_d(R, nR, rc, nrc, 0), j = nth_d(C, nC, cc, ncc, 0);
+            if (!d_same(Dr[i], Dc[j], pair_tol(Dr[i], Dc[j]))) return;
+            push(i, j, 0);
+        } else if (nRd == 1 || nCd == 1) {
+            // one shared line holds all errors: fix each along the orthogonal line
+            const bool shared_row = nRd == 1;
+            const int one_i = shared_row ? nth_d(R, nR, rc, nrc, 0) : nth_d(C, nC, cc, ncc, 0);
+            const double one = shared_row ? Dr[one_i] : Dc[one_i];
+            const int *S = shared_row ? C : R;
+            const int m = shared_row ? nC : nR;
+            const int *s3 = shared_row ? cc : rc;
+            const int m3 = shared_row ? ncc : nrc;
+            const double *Dm = shared_row ? Dc : Dr;
+            double sum = 0.0, sa = 0.0;
+            bool nonfin = false;
+            for (int a = 0; a < m; a++)
+                if (!inset(S[a], s3, m3)) {
+                    sum += Dm[S[a]];
+                    sa += fabs(Dm[S[a]]);
+                    nonfin |= !isfinite(Dm[S[a]]);
+                }
+            if (nonfin) {
+                if (isfinite(one)) return;
+            } else if (!d_same(sum, one, 2.0 * tauS + 2.0 * n * EPS * (sa + fabs(one)))) {
+                return;
+            }
+            for (int a = 0; a < m; a++)
+                if (!inset(S[a], s3, m3)) {
+                    if (shared_row) push(one_i, S[a], 1);  // column formula
+                    else push(S[a], one_i, 0);            // row formula
+                }
+        } else if (nRd == nCd) {
+            // distinct rows and columns: pair by value, uniquely in both directions
+            for (int a = 0; a < nRd; a++) {
+                const int i = nth_d(R, nR, rc, nrc, a);
+                int cnt = 0, match = -1;
+                for (int b = 0; b < nCd; b++) {
+                    const int j = nth_d(C, nC, cc, ncc, b);
+                    if (d_same(Dr[i], Dc[j], pair_tol(Dr[i], Dc[j]))) {
+                        cnt++;
+                        match = j;
+                    }
+                }
+                if (cnt != 1) return;
+                int cnt2 = 0;
+                for (int a2 = 0; a2 < nRd; a2++) {
+                    const int i2 = nth_d(R, nR, rc, nrc, a2);
+                    if (d_same(Dr[i2], Dc[match], pair_tol(Dr[i2], Dc[match]))) cnt2++;
+                }
+                if (cnt2 != 1) return;
+                push(i, match, 0);
+            }
+        } else {
+            return;
+        }
+    }
+    for (int q = 0; q < nrc; q++) push(rc[q], -1, 2);
+    for (int q = 0; q < ncc; q++) push(-1, cc[q], 3);
+    out->nfix = nf;
+    out->status = nf > cap ? 3 : 1;
+}
+cudaError_t ft_decode(const double *Dr, const double *Dc, const double *sums, const double *kap, int n, int mode,
+                      const FtCtl *ctl, int *idx, FtFix *fixes, int cap, FtDecOut *out, cudaStream_t s) {
+    g_ft_launches++;
+    k_decode<<<1, DEC_T, 0, s>>>(Dr, Dc, sums, kap, n, mode, ctl, idx, fixes, cap, out);
+    return cudaGetLastError();
+}
+// the planned fixes (count from the device: blocks past it return), one block per fix
+__global__ void k_fix(double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdone, int mode, double *r,
+                      int64_t rinc, double *c, int64_t cinc, double *kappa, const FtFix *fixes, double *deltas);
+__global__ void k_fix_dev(double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdone, int mode, double *r,
+                          int64_t rinc, double *c, int64_t cinc, double *kappa, const FtFix *fixes, double *deltas,
+                          const FtDecOut *dec);
+
 // one block per fix: explicit sum excluding the bad element
+__device__ void fix_one(double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdone, int mode, double *r,
+                        int64_t rinc, double *c, int64_t cinc, double *kappa, const FtFix *fixes, double *deltas);
 __global__ void k_fix(double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdone, int mode, double *r,
                       int64_t rinc, double *c, int64_t cinc, double *kappa, const FtFix *fixes, double *deltas) {
+    fix_one(Aw, ldw, n, ilo, ihi, cdone, mode, r, rinc, c, cinc, kappa, fixes, deltas);
+}
+__global__ void k_fix_dev(double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdone, int mode, double *r,
+                          int64_t rinc, double *c, int64_t cinc, double *kappa, const FtFix *fixes, double *deltas,
+                          const FtDecOut *dec) {
+    if (dec->status != 1 || (int)blockIdx.x >= dec->nfix) return;
+    fix_one(Aw, ldw, n, ilo, ihi, cdone, mode, r, rinc, c, cinc, kappa, fixes, deltas);
+}
+__device__ void fix_one(double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdone, int mode, double *r,
+                        int64_t rinc, double *c, int64_t cinc, double *kappa, const FtFix *fixes, double *deltas) {
     const FtFix f = fixes[blockIdx.x];
     __shared__ double ws[32];
     double s = 0.0;
@@ -750,6 +1028,13 @@ __global__ void k_fix(double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdon
         deltas[blockIdx.x] = nv - *dst;
         *dst = nv;
     }
+}
+cudaError_t ft_apply_fixes_dev(double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdone, int mode, double *r,
+                               int64_t rinc, double *c, int64_t cinc, double *kappa, const FtFix *fixes, int cap,
+                               double *deltas, const FtDecOut *dec, cudaStream_t s) {
+    g_ft_launches++;
+    k_fix_dev<<<cap, 256, 0, s>>>(Aw, ldw, n, ilo, ihi, cdone, mode, r, rinc, c, cinc, kappa, fixes, deltas, dec);
+    return cudaGetLastError();
 }
 cudaError_t ft_apply_fixes(double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdone, int mode, double *r,
                            int64_t rinc, double *c, int64_t cinc, double *kappa, const FtFix *fixes, int nfix,

@@ -90,7 +90,10 @@ struct Work {
            *acc = nullptr, *ckpt = nullptr, *ck_r = nullptr, *ck_c = nullptr, *ck_q = nullptr, *Fr = nullptr,
            *Qr = nullptr, *Qc = nullptr, *Dr = nullptr, *Dc = nullptr, *sums = nullptr, *ypart = nullptr,
            *rowpart = nullptr, *linepart = nullptr, *scratch = nullptr, *deltas = nullptr, *hA = nullptr, *htau = nullptr,
-           *ck_w = nullptr, *Dr2 = nullptr, *Dc2 = nullptr, *wpart = nullptr;
+           *ck_w = nullptr, *Dr2 = nullptr, *Dc2 = nullptr, *wpart = nullptr, *dec_delta = nullptr;
+    int *dec_idx = nullptr;       // device decoder: compacted flagged rows / columns (2n)
+    FtFix *dec_fix = nullptr;     // its fix plan (n + 8)
+    FtDecOut *dec_out = nullptr;  // [pass 1, pass 2]
     unsigned *bar = nullptr;
     int *strip_done = nullptr;
     cudaStream_t cap_stream = nullptr;  // graph capture stream (library-owned)
@@ -108,6 +111,14 @@ struct Work {
             *p = nullptr;
         }
         if (bar) cudaFree(bar);
+        if (dec_idx) cudaFree(dec_idx);
+        if (dec_fix) cudaFree(dec_fix);
+        if (dec_out) cudaFree(dec_out);
+        if (dec_delta) cudaFree(dec_delta);
+        dec_idx = nullptr;
+        dec_fix = nullptr;
+        dec_out = nullptr;
+        dec_delta = nullptr;
         if (strip_done) cudaFree(strip_done);
         strip_done = nullptr;
         if (ctl) cudaFree(ctl);
@@ -202,6 +213,10 @@ int get_work(int n, Work **out) {
     A(dalloc(&w.Dr2, (size_t)ldw, b));
     A(dalloc(&w.Dc2, (size_t)ldw, b));
     A(dalloc(&w.wpart, (size_t)128 * (n / 256 + 2), b));
+    A(dalloc(&w.dec_idx, (size_t)2 * n + 2, b));
+    A(dalloc(&w.dec_fix, (size_t)n + 8, b));
+    A(dalloc(&w.dec_out, 2, b));
+    A(dalloc(&w.dec_delta, (size_t)n + 8, b));
     A(dalloc(&w.bar, 4, b));
     A(dalloc(&w.strip_done, (N1 + 63) / 64 + 2, b));
     A(dalloc(&w.ctl, 1, b));
@@ -996,8 +1011,67 @@ int verify_and_correct_w(Call &C, int panel, int cdone, bool *found) {
 
 // M: the augmented working array (the reduction's Aw, or ft_dorghr's augmented Q); mode 0 reads its
 // checksum column n / row n / corner, mode 1 the Q checksums of the Householder vectors
+int verify_and_correct_host(Call &C, int panel, int cdone, int mode, bool *found, double *M);
+
+// full verify -> R12 decode -> explicit-sum fixes -> re-verify -> decode, all enqueued on the device
+// (k_decode, k_fix_dev); the host reads the outcome and the fix list once, for the report
 int verify_and_correct(Call &C, int panel, int cdone, int mode, bool *found, double *M = nullptr) {
     if (C.weighted && mode == 0 && (!M || M == C.w->Aw)) return verify_and_correct_w(C, panel, cdone, found);
+    Work &w = *C.w;
+    const int n = C.n;
+    const int64_t ldw = w.ldw;
+    if (!M) M = w.Aw;
+    double *r = mode == 0 ? M + (int64_t)n * ldw : w.Qr;
+    double *c = mode == 0 ? M + n : w.Qc;
+    const int64_t cinc = mode == 0 ? ldw : 1;
+    double *kap = mode == 0 ? M + n + (int64_t)n * ldw : w.Qc + n;
+    const int cap = n + 8;
+    for (int pass = 0; pass < 2; pass++) {
+        CK(ft_full_verify(M, ldw, n, C.ilo, C.ihi, cdone, mode, r, 1, c, cinc, nullptr, w.Dr, w.Dc, w.sums,
+                          w.linepart, C.s));
+        CK(ft_decode(w.Dr, w.Dc, w.sums, kap, n, mode, w.ctl, w.dec_idx, w.dec_fix, cap, w.dec_out + pass, C.s));
+        if (pass == 0)
+            CK(ft_apply_fixes_dev(M, ldw, n, C.ilo, C.ihi, cdone, mode, r, 1, c, cinc, kap, w.dec_fix, cap,
+                                  w.dec_delta, w.dec_out, C.s));
+    }
+    FtDecOut d[2];
+    CK(cudaMemcpyAsync(d, w.dec_out, 2 * sizeof(FtDecOut), cudaMemcpyDeviceToHost, C.s));
+    CK(cudaStreamSynchronize(C.s));
+    *found = false;
+    if (d[0].status == 0) return 0;
+    if (d[0].status == 3) return verify_and_correct_host(C, panel, cdone, mode, found, M);  // (unreachable: cap)
+    *found = true;
+    C.ev(FT_EV_DETECT, panel, d[0].nR, d[0].nC, 0.0);
+    C.detected++;
+    if (d[0].status == 2) {
+        C.ev(FT_EV_UNCORRECTABLE, panel, d[0].nR, d[0].nC, 0.0);
+        C.uncorrectable++;
+        return FT_E_UNCORRECTABLE;
+    }
+    const int nf = d[0].nfix;
+    std::vector<FtFix> fx(nf);
+    std::vector<double> dl(nf);
+    CK(cudaMemcpy(fx.data(), w.dec_fix, nf * sizeof(FtFix), cudaMemcpyDeviceToHost));
+    CK(cudaMemcpy(dl.data(), w.dec_delta, nf * sizeof(double), cudaMemcpyDeviceToHost));
+    for (int q = 0; q < nf; q++) {
+        const FtFix &f = fx[q];
+        const int kind = f.kind == 0 || f.kind == 1 ? (mode == 0 ? FT_EV_FIX_DATA : FT_EV_FIX_Q)
+                         : f.kind == 2             ? (mode == 0 ? FT_EV_FIX_R : FT_EV_FIX_QR)
+                         : f.kind == 3             ? (mode == 0 ? FT_EV_FIX_C : FT_EV_FIX_QC)
+                                                   : (mode == 0 ? FT_EV_FIX_K : FT_EV_FIX_QK);
+        C.ev(kind, panel, f.i, f.j, dl[q]);
+    }
+    if (d[1].status != 0) {
+        C.ev(FT_EV_UNCORRECTABLE, panel, -1, -1, 0.0);
+        C.uncorrectable++;
+        return FT_E_UNCORRECTABLE;
+    }
+    C.corrected++;
+    return 0;
+}
+
+// the host copy of the same decision (R12), kept for a plan larger than the device's fix buffer
+int verify_and_correct_host(Call &C, int panel, int cdone, int mode, bool *found, double *M) {
     Work &w = *C.w;
     const int n = C.n;
     const int64_t ldw = w.ldw;

@@ -214,6 +214,14 @@ cudaError_t ft_full_verify(const double *Aw, int64_t ldw, int n, int ilo, int ih
 // 5 refresh r_w(i), 6 refresh c_w(j), 7 e^T L w = sum r_w, 8 w^T L e = sum c_w
 struct FtFix { int64_t i, j; int kind; int pad; };
 cudaError_t ft_encode_w(double *Aw, int64_t ldw, int n, double *linepart, cudaStream_t s);
+// R12 decoder v2 on the device (one block): status 0 clean, 1 fixes planned, 2 uncorrectable, 3 the plan
+// exceeds cap (the host decides)
+struct FtDecOut { int status, nfix, nR, nC; };
+cudaError_t ft_decode(const double *Dr, const double *Dc, const double *sums, const double *kap, int n, int mode,
+                      const FtCtl *ctl, int *idx, FtFix *fixes, int cap, FtDecOut *out, cudaStream_t s);
+cudaError_t ft_apply_fixes_dev(double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdone, int mode, double *r,
+                               int64_t rinc, double *c, int64_t cinc, double *kappa, const FtFix *fixes, int cap,
+                               double *deltas, const FtDecOut *dec, cudaStream_t s);
 cudaError_t ft_final_flags(const double *Dr, const double *Dc, const double *sums, const double *kap, int n, int mode,
                            FtCtl *ctl, cudaStream_t s);
 cudaError_t ft_full_verify_w(const double *Aw, int64_t ldw, int n, int ilo, int ihi, int cdone, const double *rw,
