@@ -646,6 +646,22 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
             else es_c += __ldcg(p.A + en + (int64_t)(x - nr) * p.lda);
         }
     }
+    // C tile of tile tt into registers, prefetched a whole tile ahead (16-byte loads, masked edges)
+    auto load_c = [&](int tt, double2 (&dst)[2][4]) {
+        const int r = rbase + tt * UB;
+        const int lo = max(r, p.r_lo), hi = min(r + UB, p.r_hi);
+        const bool full = lo == r && hi == r + UB && ncols == UB;
+#pragma unroll
+        for (int mi = 0; mi < 2; mi++)
+#pragma unroll
+            for (int ni = 0; ni < 4; ni++) {
+                const int row = r + wr * 32 + ni * 8 + 2 * lc;
+                dst[mi][ni] = full ? *reinterpret_cast<const double2 *>(colp[mi] + row)
+                                   : load_pair(colp[mi], row, lo, hi, colok[mi]);
+            }
+    };
+    double2 cn[2][4];
+    if (t0 < t1) load_c(t0, cn);
     cp_async_wait<0>();
     __syncthreads();  // every thread's part of W' landed
     for (int tt = t0; tt < t1; tt++) {
@@ -658,13 +674,13 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
         for (int mi = 0; mi < 2; mi++)
 #pragma unroll
             for (int ni = 0; ni < 4; ni++) {
-                const int row = r + wr * 32 + ni * 8 + 2 * lc;
-                const double2 c = full ? *reinterpret_cast<const double2 *>(colp[mi] + row)
-                                       : load_pair(colp[mi], row, lo, hi, colok[mi]);
-                acc[mi][ni][0] = sg * c.x;
-                acc[mi][ni][1] = sg * c.y;
+                acc[mi][ni][0] = sg * cn[mi][ni].x;
+                acc[mi][ni][1] = sg * cn[mi][ni].y;
             }
-        if (tt + 1 < t1) issue_v(tt + 1, st ^ 1);  // released by the bar.sync that ended tile tt-1
+        if (tt + 1 < t1) {
+            issue_v(tt + 1, st ^ 1);  // released by the bar.sync that ended tile tt-1
+            load_c(tt + 1, cn);
+        }
         mbar_wait(&vbar[st], (unsigned)((tt - t0) >> 1) & 1u);
 #pragma unroll 4
         for (int k0 = 0; k0 < KT; k0 += 4) {
