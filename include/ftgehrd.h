@@ -130,6 +130,17 @@ void ft_opts_default(ft_opts *o);
  * in rows/columns 1:ilo-1 and ihi+1:n.  lda >= max(1, n). */
 int ft_dgehrd(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opts *opts);
 
+/* NEXT-4 (the paper's generalisation claim): symmetric tridiagonal reduction A = Q T Q^T with
+ * LAPACK DSYTRD semantics for uplo = 'L', on the protected path.  For symmetric A the Householder
+ * Hessenberg reduction IS the tridiagonal reduction (same reflectors, same DLARFG convention: H is
+ * tridiagonal, v(i+2:n) of H(i) stored below the subdiagonal), so the call runs ft_dgehrd's ABFT
+ * machinery (checksums, verification, rollback, correction, fault plan) on the symmetric matrix the
+ * lower triangle of dA defines (the strict upper triangle is not referenced).  It does not exploit the
+ * symmetry (no SYMV / SYR2K: about 2.5x the flops of a symmetric-specific code).  On exit: d (n) the
+ * diagonal, e (n-1) the subdiagonal of T, tau (n-1), V below the subdiagonal of dA; Q by ft_dorghr.
+ * Device pointers; errors as ft_dgehrd (-4 d, -5 e / lda, -6 tau). */
+int ft_dsytrd(int n, double *dA, int lda, double *dd, double *de, double *dtau, const ft_opts *opts);
+
 /* Same contract with HOST buffers hA / htau: the host->device copy of A, the
  * reduction and the device->host copy of H/V and tau all run inside the call
  * (the end-to-end entry point bench.py times). */

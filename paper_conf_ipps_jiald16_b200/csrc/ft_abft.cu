@@ -30,6 +30,37 @@ __global__ void k_copy_out(const double *__restrict__ Aw, int64_t ldw, double *_
     for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x)
         A[i + j * (int64_t)lda] = Aw[i + j * ldw];
 }
+// symmetric input (ft_dsytrd, uplo 'L'): the working copy's strict upper triangle from the lower one
+__global__ void k_mirror_lower(double *Aw, int64_t ldw, int n) {
+    const int64_t j = blockIdx.y;
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < j; i += gridDim.x * blockDim.x)
+        Aw[i + j * ldw] = Aw[j + (int64_t)i * ldw];
+}
+cudaError_t ft_mirror_lower(double *Aw, int64_t ldw, int n, cudaStream_t s) {
+    if (n <= 1) return cudaSuccess;
+    g_ft_launches++;
+    k_mirror_lower<<<dim3((n + 255) / 256 < 8 ? (n + 255) / 256 : 8, n), 256, 0, s>>>(Aw, ldw, n);
+    return cudaGetLastError();
+}
+// copy-out of the lower triangle only (the caller's strict upper part is not referenced), and the
+// tridiagonal's diagonal d and subdiagonal e
+__global__ void k_copy_out_lower(const double *__restrict__ Aw, int64_t ldw, double *__restrict__ A, int lda, int n,
+                                 double *d, double *e) {
+    const int64_t j = blockIdx.y;
+    for (int i = (int)j + blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+        const double v = Aw[i + j * ldw];
+        A[i + j * (int64_t)lda] = v;
+        if (i == j) d[i] = v;
+        else if (i == j + 1) e[j] = v;
+    }
+}
+cudaError_t ft_copy_out_lower(const double *Aw, int64_t ldw, double *A, int lda, int n, double *d, double *e,
+                              cudaStream_t s) {
+    if (n <= 0) return cudaSuccess;
+    g_ft_launches++;
+    k_copy_out_lower<<<dim3((n + 255) / 256 < 8 ? (n + 255) / 256 : 8, n), 256, 0, s>>>(Aw, ldw, A, lda, n, d, e);
+    return cudaGetLastError();
+}
 cudaError_t ft_copy_out(const double *Aw, int64_t ldw, double *A, int lda, int n, cudaStream_t s) {
     if (n <= 0) return cudaSuccess;
     g_ft_launches++;

@@ -195,6 +195,9 @@ cudaError_t ft_launch_ytop(const YtopParams &p, cudaStream_t s);
 cudaError_t ft_ctl_init(FtCtl *ctl, double c_thr, cudaStream_t s);
 cudaError_t ft_copy_in(const double *A, int lda, double *Aw, int64_t ldw, int n, cudaStream_t s);
 cudaError_t ft_copy_out(const double *Aw, int64_t ldw, double *A, int lda, int n, cudaStream_t s);
+cudaError_t ft_mirror_lower(double *Aw, int64_t ldw, int n, cudaStream_t s);
+cudaError_t ft_copy_out_lower(const double *Aw, int64_t ldw, double *A, int lda, int n, double *d, double *e,
+                              cudaStream_t s);
 cudaError_t ft_encode(double *Aw, int64_t ldw, int n, FtCtl *ctl, double *scratch, double *linepart,
                       cudaStream_t s);
 cudaError_t ft_frozen_init(const double *Aw, int64_t ldw, int n, int ncols, double *Fr, cudaStream_t s);

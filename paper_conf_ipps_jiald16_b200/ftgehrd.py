@@ -78,6 +78,7 @@ def lib():
         L.ft_dgehrd.argtypes = [i32, i32, i32, vp, i32, vp, ctypes.POINTER(Opts)]
         L.ft_dgehrd_host.argtypes = [i32, i32, i32, vp, i32, vp, ctypes.POINTER(Opts)]
         L.ft_dorghr.argtypes = [i32, i32, i32, vp, i32, vp, vp, i32, ctypes.POINTER(Opts)]
+        L.ft_dsytrd.argtypes = [i32, vp, i32, vp, vp, vp, ctypes.POINTER(Opts)]
         L.ft_dgehrd_mgpu.argtypes = [i32, i32, i32, vp, i32, vp, i32, i32, ctypes.POINTER(Opts)]
         L.ft_mgpu_setup.argtypes = [i32, i32, i32, ctypes.POINTER(IpcHandle)]
         L.ft_mgpu_connect.argtypes = [ctypes.POINTER(IpcHandle), i32, i32]
@@ -94,7 +95,7 @@ def lib():
     return _lib
 
 
-EXPORTS = ["ft_opts_default", "ft_dgehrd", "ft_dgehrd_host", "ft_dorghr", "ft_dgehrd_mgpu",
+EXPORTS = ["ft_opts_default", "ft_dgehrd", "ft_dgehrd_host", "ft_dorghr", "ft_dsytrd", "ft_dgehrd_mgpu",
            "ft_mgpu_setup", "ft_mgpu_connect", "ft_dgehrd_vranks", "ft_mgpu_finalize",
            "ft_mgpu_probe_put", "ft_mgpu_probe_get",
            "ft_strerror", "ft_finalize", "ft_version", "ft_launch_count"]
@@ -173,6 +174,21 @@ def dgehrd(A, tau=None, ilo=1, ihi=None, **kw):
     info = lib().ft_dgehrd(n, ilo, ihi, ctypes.c_void_p(A.data_ptr()), lda, ctypes.c_void_p(tau.data_ptr()),
                            ctypes.byref(o))
     return tau, Result(info, rep, rep.event_list())
+
+
+def dsytrd(A, **kw):
+    """Symmetric tridiagonal reduction (DSYTRD, uplo 'L') of the column-major CUDA float64 matrix A
+    (lower triangle read; NEXT-4 on the protected path).  Returns (d, e, tau, Result)."""
+    import torch
+    n, lda = _check_fortran(A)
+    d = torch.zeros(max(n, 1), dtype=torch.float64, device=A.device)
+    e = torch.zeros(max(n - 1, 1), dtype=torch.float64, device=A.device)
+    tau = torch.zeros(max(n - 1, 1), dtype=torch.float64, device=A.device)
+    rep = Report()
+    o = make_opts(report=rep, **kw)
+    info = lib().ft_dsytrd(n, ctypes.c_void_p(A.data_ptr()), lda, ctypes.c_void_p(d.data_ptr()),
+                           ctypes.c_void_p(e.data_ptr()), ctypes.c_void_p(tau.data_ptr()), ctypes.byref(o))
+    return d[:n], e[: max(n - 1, 0)], tau[: max(n - 1, 0)], Result(info, rep, rep.event_list())
 
 
 def dgehrd_host(A_np, ilo=1, ihi=None, **kw):

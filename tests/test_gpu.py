@@ -506,3 +506,43 @@ def test_policy_paper_fault_detect_rollback_locate_redo():
         assert res.report.rollbacks >= 1, (f, res.events)
         assert ("FIX_DATA", f[3], f[4]) in fixes(res.events), (f, res.events)
         check_against_oracle(A, dA, tau, nb=nb)
+
+
+# ------------------------------------------------------------------ NEXT-4: symmetric tridiagonal reduction
+@pytest.mark.parametrize("n,nb", [(64, 16), (300, 32), (1000, 64)])
+def test_dsytrd_matches_oracle(n, nb):
+    """ft_dsytrd (DSYTRD 'L' semantics on the protected path): d, e, tau and V equal the oracle's
+    reduction of the symmetric matrix (pinned to LAPACK dsytrd in test_oracle.py) at the parity bar;
+    the strict upper triangle of the caller's array is not touched; Q T Q^T reproduces A."""
+    S = synth.symmetric_matrix(n)
+    A = np.asfortranarray(np.tril(S) + 7.0 * np.triu(np.ones((n, n)), 1))  # garbage above: not referenced
+    dA = ft.fortran(torch.from_numpy(A).cuda())
+    d, e, tau, res = ft.dsytrd(dA, nb=nb)
+    torch.cuda.synchronize()
+    assert res.info == 0 and res.report.detected == 0, res.events
+    Ao, to = oracle.dgehd2(S)
+    sc = np.abs(Ao).max()
+    assert np.abs(d.cpu().numpy() - np.diag(Ao)).max() <= TOL * sc
+    assert np.abs(e.cpu().numpy() - np.diag(Ao, -1)).max() <= TOL * sc
+    assert np.abs(tau.cpu().numpy() - to).max() <= TOL
+    Ag = dA.cpu().numpy()
+    assert np.abs(np.tril(Ag, -2) - np.tril(Ao, -2)).max() <= TOL
+    assert np.array_equal(np.triu(Ag, 1), np.triu(A, 1))
+    tpad = torch.cat([tau, torch.zeros(1, dtype=torch.float64, device="cuda")])
+    Q, info = ft.dorghr(dA, tpad, nb=nb)
+    Qg = Q.cpu().numpy()
+    T = np.diag(d.cpu().numpy()) + np.diag(e.cpu().numpy(), -1) + np.diag(e.cpu().numpy(), 1)
+    assert np.linalg.norm(S - Qg @ T @ Qg.T, 1) / (n * np.linalg.norm(S, 1) * EPS) <= 30
+
+
+def test_dsytrd_fault_corrected():
+    """The ABFT machinery on the symmetric path: a flip in the trailing block before a panel is located
+    and corrected; the tridiagonal meets the oracle bar."""
+    n, nb = 300, 32
+    S = synth.symmetric_matrix(n)
+    dA = ft.fortran(torch.from_numpy(S).cuda())
+    d, e, tau, res = ft.dsytrd(dA, nb=nb, faults=[(2, ft.PHASE_BEFORE_PANEL, ft.SITE_A, 150, 200, 55)])
+    torch.cuda.synchronize()
+    assert res.info == 0 and ("FIX_DATA", 150, 200) in fixes(res.events), res.events
+    Ao, to = oracle.dgehd2(S)
+    assert np.abs(e.cpu().numpy() - np.diag(Ao, -1)).max() <= TOL * np.abs(Ao).max()

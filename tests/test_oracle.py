@@ -542,3 +542,19 @@ def test_weighted_end_to_end_tied_flips(ora):
     assert np.abs(np.triu(Af, -1) - np.triu(Ao, -1)).max() <= 1e-12 * np.abs(Ao).max()
     info1, *_ = ora.ft_dgehd2(A, nb, faults=faults)
     assert info1 == 1
+
+
+def test_symmetric_hessenberg_is_lapack_dsytrd(ora):
+    """NEXT-4 pin: for symmetric A the unblocked Householder Hessenberg reduction (DGEHD2 conventions,
+    R1) is LAPACK's DSYTRD (uplo 'L'): the same diagonal d, subdiagonal e, tau and reflectors V."""
+    from scipy.linalg import lapack
+    for n in (17, 120, 333):
+        S = synth.symmetric_matrix(n)
+        c, d, e, tau, info = lapack.dsytrd(S, lower=1)
+        assert info == 0
+        Ao, to = ora.dgehd2(S)
+        sc = max(np.abs(d).max(), np.abs(e).max())  # norm-wise (R18)
+        assert np.abs(np.diag(Ao) - d).max() <= 1e-12 * sc
+        assert np.abs(np.diag(Ao, -1) - e).max() <= 1e-12 * sc
+        assert np.abs(to - tau).max() <= 1e-12
+        assert np.abs(np.tril(Ao, -2) - np.tril(c, -2)).max() <= 1e-11
