@@ -556,5 +556,7 @@ def test_symmetric_hessenberg_is_lapack_dsytrd(ora):
         sc = max(np.abs(d).max(), np.abs(e).max())  # norm-wise (R18)
         assert np.abs(np.diag(Ao) - d).max() <= 1e-12 * sc
         assert np.abs(np.diag(Ao, -1) - e).max() <= 1e-12 * sc
-        assert np.abs(to - tau).max() <= 1e-12
-        assert np.abs(np.tril(Ao, -2) - np.tril(c, -2)).max() <= 1e-11
+        # the last reflectors are ill-conditioned functions of the data (R18): two correct codes differ
+        # by ~1e-12 there; a convention error (sign, scaling, index) would be O(1)
+        assert np.abs(to - tau).max() <= 1e-10
+        assert np.abs(np.tril(Ao, -2) - np.tril(c, -2)).max() <= 1e-10
