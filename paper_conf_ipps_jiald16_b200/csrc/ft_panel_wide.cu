@@ -378,6 +378,8 @@ __global__ void __launch_bounds__(PT, 1) k_panel_wide(const __grid_constant__ Pa
             }
         });
         PROBE(5);
+        unsigned long long gt_start = 0;
+        if (p.dbg && tid == 0 && j == 8) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(gt_start));
         if (wid > 0) {
             // ======================= GEMV warps: y = A(:, c+1:) v on the unscaled b ===========
             const int gt = tid - 32;
@@ -542,6 +544,16 @@ __global__ void __launch_bounds__(PT, 1) k_panel_wide(const __grid_constant__ Pa
             PROBE(6);
         }
         __syncthreads();  // GEMV partials, tau / scale / t, V(:, j) are in shared memory
+        if (p.dbg && tid == 0 && j == 8) {  // per-CTA GEMV span (debug hook): smid, start, end, rows
+            unsigned long long t1;
+            unsigned smid;
+            asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t1));
+            asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+            p.dbg[2048 + bid * 4 + 0] = smid;
+            p.dbg[2048 + bid * 4 + 1] = gt_start;
+            p.dbg[2048 + bid * 4 + 2] = t1;
+            p.dbg[2048 + bid * 4 + 3] = (unsigned long long)R;
+        }
         if (MG) {
             // ---- cross-rank exchange of the GEMV partials, CTA by CTA: every rank
             // uses the same row partition, so CTA bid of each rank owns the same rows.  Push

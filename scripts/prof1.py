@@ -26,6 +26,7 @@ def main():
     ap.add_argument("--ablate", type=int, default=0)
     ap.add_argument("--no-panel-timing", action="store_true", help="leave panel events off (CUDA graphs enabled)")
     a = ap.parse_args()
+    import numpy as np
     import torch
 
     import paper_conf_ipps_jiald16_b200 as ft
@@ -42,7 +43,7 @@ def main():
     L.ft_debug_panel_launches.restype = ctypes.c_int
     dbg = None
     if a.probe >= 0:
-        dbg = torch.zeros(2048, dtype=torch.int64, device="cuda")
+        dbg = torch.zeros(2048 + 4 * 256, dtype=torch.int64, device="cuda")
         L.ft_debug_probe_panel.argtypes = [ctypes.c_int, ctypes.c_void_p]
         L.ft_debug_probe_panel(a.probe, ctypes.c_void_p(dbg.data_ptr()))
         L.ft_debug_ablate.argtypes = [ctypes.c_int]
@@ -87,6 +88,16 @@ def main():
             for sl in order[1:]:
                 if row[sl] > 0:
                     mx[names[sl]] = mx.get(names[sl], 0) + row[sl]
+        cta = d[2048:].reshape(-1, 4)
+        cta = cta[cta[:, 2] > 0]
+        if len(cta):  # per-CTA GEMV spans of column 8 (wide kernel): globaltimer ns
+            t0 = cta[:, 1].min()
+            dur = cta[:, 2] - cta[:, 1]
+            print(f"per-CTA GEMV span, column 8: {len(cta)} CTAs, rows {cta[:, 3].min()}..{cta[:, 3].max()}, "
+                  f"duration ns min {dur.min()} median {int(np.median(dur))} max {dur.max()}; "
+                  f"start spread {cta[:, 1].max() - t0} ns, end spread {cta[:, 2].max() - cta[:, 2].min()} ns")
+            order = np.argsort(cta[:, 0])
+            print("  smid:dur_ns " + " ".join(f"{int(cta[q, 0])}:{int(dur[q])}" for q in order))
         print(f"probe panel {a.probe}: {ncol} columns, mean cycles per column by phase "
               f"(CTA 0 | max over CTAs of the phase):")
         for k2, v in tot.items():
