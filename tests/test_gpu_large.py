@@ -216,3 +216,27 @@ def test_c3_fault_pattern_full(a16):
     dB, tB, resB, _, _ = gpu_run(A, keep_device=True)
     assert resB.info == 0 and resB.report.detected == 0
     assert float((torch.triu(dA, -1) - torch.triu(dB, -1)).abs().max()) <= TOL * float(torch.triu(dB, -1).abs().max())
+
+
+# ------------------------------------------------------------------ sharded path at the C3 size
+def test_sharded_path_c3_size(a16):
+    """The 1-D block-column cyclic path (what bench.py --gpus N runs) at n = 16384: two virtual ranks
+    on this GPU (74 CTAs each, ~221 rows per CTA) give the single-GPU H to the parity bar, fault-free
+    and with a data flip at panel 3 that the sharded verification corrects."""
+    A = a16
+    n = A.shape[0]
+    dA = ft.fortran(torch.from_numpy(A).cuda())
+    tau1, r1 = ft.dgehrd(dA, nb=NB)
+    assert r1.info == 0
+    H1 = torch.triu(dA, -1)
+    s = float(H1.abs().max())
+    for faults in ((), ((3, ft.PHASE_BEFORE_PANEL, ft.SITE_A, n // 2 + 7, n // 2 + 100, 55),)):
+        slabs = ft.shard(torch.from_numpy(A).cuda(), NB, 2)
+        taus, res = ft.dgehrd_vranks(slabs, nb=NB, faults=faults)
+        torch.cuda.synchronize()
+        assert res.info == 0, res.events
+        assert res.report.detected == len(faults), res.events
+        Hv = torch.triu(ft.unshard(slabs, n, NB), -1)
+        assert float((Hv - H1).abs().max()) <= TOL * s
+        assert float((taus[0][: n - 1] - tau1[: n - 1]).abs().max()) <= TOL
+        del slabs, Hv
