@@ -247,6 +247,11 @@ void ft_debug_panel_path(int bits);
  * the CTAs of the last tile row / strip (1, the default).  Results agree
  * up to rounding; CUDA-graph replay is off while 0. */
 void ft_debug_left_fold(int on);
+/* ft_debug_right_fold(0) makes the ABFT right update carry the column checksum c (row n) as one
+ * more DMMA tile row instead of a GEMV by the CTAs of the last row split (1, the default; the
+ * row splits then see the data rows only).  Results agree up to rounding; CUDA-graph replay is
+ * off while 0. */
+void ft_debug_right_fold(int on);
 /* Number of panel launches that ran the two-reduction wide kernel (>= 32 rows per CTA, the large-n
  * path) since load / the last reset: tests use it to show which panel kernel a run exercised. */
 int64_t ft_debug_wide_launches(int reset);

@@ -355,13 +355,11 @@ __global__ void k_endcheck(double *Aw, int64_t ldw, int n, int ihi, int k, int i
             atomicAdd(&ctl->wsums[0], c2);
             atomicAdd(&ctl->wsums[1], d2);
         }
-        __threadfence();
-        last = (atomicAdd(&ctl->done_count, 1) == (int)gridDim.x - 1);
+        last = (atom_add_acqrel_s32(&ctl->done_count, 1) == (int)gridDim.x - 1);
     }
     __syncthreads();
     if (!last) return;
     if (threadIdx.x == 0) {
-        __threadfence();
         double Sr = atomicAdd(&ctl->sums[0], 0.0), Sc = atomicAdd(&ctl->sums[1], 0.0);
         double kap = Aw[n + (int64_t)n * ldw];
         double unit = (double)n * EPS * ctl->normF;

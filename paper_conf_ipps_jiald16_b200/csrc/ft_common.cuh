@@ -147,6 +147,14 @@ FT_DEV unsigned ld_acquire_u32(const unsigned *p) {
 FT_DEV void red_release_add_u32(unsigned *p, unsigned v) {
     asm volatile("red.release.gpu.global.add.u32 [%0], %1;\n" ::"l"(p), "r"(v) : "memory");
 }
+// last-CTA-done counters: one acq_rel atomic replaces fence + atomic + fence (the release is
+// cumulative over the CTA's writes ordered before it by bar.sync, the acquire over the last
+// CTA's reads ordered after it by the next bar.sync)
+FT_DEV int atom_add_acqrel_s32(int *p, int v) {
+    int old;
+    asm volatile("atom.acq_rel.gpu.global.add.s32 %0, [%1], %2;\n" : "=r"(old) : "l"(p), "r"(v) : "memory");
+    return old;
+}
 FT_DEV void grid_barrier(unsigned *count, unsigned &epoch, unsigned nblocks) {
     __syncthreads();
     if (threadIdx.x == 0) {

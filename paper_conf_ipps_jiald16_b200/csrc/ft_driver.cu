@@ -34,6 +34,8 @@ static int g_panel_path = 0;  // OR'ed into every panel launch's mode bits (8: e
 extern "C" void ft_debug_panel_path(int bits) { g_panel_path = bits & (8 | 64 | 128); }
 static int g_left_fold = 1;  // ABFT left update: checksum row/column folded (1) or as DMMA tiles (0)
 extern "C" void ft_debug_left_fold(int on) { g_left_fold = on ? 1 : 0; }
+static int g_right_fold = 1;  // ABFT right update: checksum row c as a GEMV of the last row split (1) or a tile row (0)
+extern "C" void ft_debug_right_fold(int on) { g_right_fold = on ? 1 : 0; }
 extern "C" void ft_debug_probe_panel(int panel, unsigned long long *dbuf) {
     g_dbg_panel = panel;
     g_dbg_buf = dbuf;
@@ -625,7 +627,8 @@ int right_update(Call &C, int t, double sign, int do_w, bool precheck = false) {
     g.wr_lo = k + 1;
     g.wr_hi = C.ihi;
     g.do_w = do_w;
-    g.nsplit = ft_gemm_splits(g.r_lo, g.r_hi, g.c_lo, g.c_hi, w.nsm);
+    g.fold_row = (C.abft && !C.weighted) ? g_right_fold : 0;  // row n (c) as a GEMV of the last row split
+    g.nsplit = ft_gemm_splits(g.r_lo, g.r_hi - g.fold_row, g.c_lo, g.c_hi, w.nsm);
     if (do_w) {
         g.Wt = w.Wt;
         g.T = w.T;
@@ -1330,7 +1333,7 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
     // every iteration), captured on the second call with the same shape and buffers; the halt
     // protocol is unchanged (a halted graph's remaining kernels are no-ops, recovery follows).
     const bool graphable = C.faults.empty() && o.stop_after_panel < 0 && g_dbg_panel < 0 && !C.timing && !C.sym &&
-                           !g_panel_path && g_left_fold &&
+                           !g_panel_path && g_left_fold && g_right_fold &&
                            !getenv("FT_NO_GRAPH");
     bool launched = false;
     // the fault-free final verification's decision is taken on the device (not for the weighted pair,

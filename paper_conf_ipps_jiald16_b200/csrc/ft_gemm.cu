@@ -57,6 +57,7 @@ struct RightSmemT {
     double Vc[KT][SK];  // V(cols, k) as [k][col]   (A operand of the right update)
     double Ys[KT][SK];  // Y(rows, k) as [k][row]   (B operand of the right update)
     double Vr[KT][SK];  // V(rows, j) as [j][row]   (B operand of W^T = C_new^T V)
+    double Yn[KT];      // fold_row: Y(n, :) = Y_chk
 };
 
 // k-major operand tile: M(r .. r+63, 0:KT) (column-major, leading dim ld) -> T[k][row];
@@ -118,7 +119,9 @@ __device__ int pre_update_reason(const GemmRightParams &p) {
 
 template <int KT>
 __global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
-    if (p.ctl && p.ctl->halt) return;
+    // the halt flag is loaded here but first used at the first tile's barrier (before any store),
+    // so its round trip overlaps the operand loads instead of delaying them
+    const int halted = p.ctl ? __ldcg(&p.ctl->halt) : 0;
     // fused pre-update check: warp 0 evaluates it while the other warps start the operand and
     // C-tile loads; the decision is read at the first tile's barrier, before any store
     __shared__ int s_reason;
@@ -126,18 +129,6 @@ __global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
         const int reason = pre_update_reason(p);
         if (threadIdx.x == 0) s_reason = reason;
     }
-    auto pre_abort = [&]() -> bool {  // after a __syncthreads that follows the evaluation
-        if (!p.pre_ctl || !s_reason) return false;
-        if (threadIdx.x == 0 && blockIdx.x == 0 && blockIdx.y == 0) {
-            FtCtl *ctl = p.pre_ctl;
-            ctl->halt_panel = p.pre_panel;
-            ctl->halt_stage = 1;
-            ctl->halt_reason = s_reason;
-            __threadfence();
-            ctl->halt = 1;
-        }
-        return true;  // nothing consumed: the panel is redone from its checkpoint
-    };
     extern __shared__ __align__(16) unsigned char smem_raw[];
     RightSmemT<KT> &S = *reinterpret_cast<RightSmemT<KT> *>(smem_raw);
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -155,6 +146,11 @@ __global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
     const int t0 = (int)((long long)blockIdx.y * nrt / gridDim.y);
     const int t1 = (int)((long long)(blockIdx.y + 1) * nrt / gridDim.y);
     constexpr int NJ = KT / 8;
+    // fold_row: row p.r_hi (= n, the column checksum c) is updated by the last row split as a GEMV,
+    // 4 lanes per strip column; c(col) is prefetched here, its use is after the tile loop
+    const bool foldr = p.fold_row && !mpart && (int)blockIdx.y == (int)gridDim.y - 1;
+    const int fcol = tid >> 2, fq = tid & 3;
+    const double cold = (foldr && fq == 0 && fcol < ncols) ? __ldcg(p.A + p.r_hi + (int64_t)(cb + fcol) * p.lda) : 0.0;
     // warp tile: 16 columns x 32 rows (warp (wc, wr): columns wc*16.., rows wr*32.. of each tile):
     // per k step 2 + 4 fragment loads feed 8 DMMA (the W pass: 4 shuffles + 8 loads feed 16)
     const int wc = warp & 3, wr = warp >> 2;
@@ -197,6 +193,7 @@ __global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
         for (int i = tid; i < (KT - K) * SK; i += UT) S.Ys[K + i / SK][i % SK] = 0.0;
     if (do_w)
         for (int i = tid; i < KT * SK; i += UT) S.Vr[i / SK][i % SK] = 0.0;
+    if (foldr && tid < KT) S.Yn[tid] = tid < K ? __ldcg(p.Y + p.r_hi + (int64_t)tid * p.ldw) : 0.0;
     __syncthreads();
     // issued by all eight warps (lanes 0..7 of warp w: columns 8w..8w+7), so no warp stalls its
     // barrier partners on a long serial issue; tid 0's arrive carries the expected byte count
@@ -213,6 +210,23 @@ __global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
         if (p.do_right) issue_tile(S.Ys, p.Y, rbase + t0 * UB, &ybar);
         if (do_w) issue_tile(S.Vr, p.V, rbase + t0 * UB, &vbar);
     }
+    auto pre_abort = [&]() -> bool {  // after a __syncthreads that follows the evaluation
+        const bool raise = !halted && p.pre_ctl && s_reason;
+        if (!halted && !raise) return false;
+        if (raise && threadIdx.x == 0 && blockIdx.x == 0 && blockIdx.y == 0) {
+            FtCtl *ctl = p.pre_ctl;
+            ctl->halt_panel = p.pre_panel;
+            ctl->halt_stage = 1;
+            ctl->halt_reason = s_reason;
+            __threadfence();
+            ctl->halt = 1;
+        }
+        if (t0 < t1) {  // the first tiles' bulk copies land before the CTA's shared memory is released
+            if (p.do_right) mbar_wait(&ybar, 0u);
+            if (do_w) mbar_wait(&vbar, 0u);
+        }
+        return true;  // nothing consumed: the panel is redone from its checkpoint
+    };
     // C tile of tile tt into registers (16-byte loads; masked pairs at the edges)
     auto load_c = [&](int tt, double2 (&dst)[2][4]) {
         const int r = rbase + tt * UB;
@@ -315,6 +329,18 @@ __global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
         __syncthreads();
         if (pre_abort()) return;
     }
+    if (foldr) {  // c(cols) += sg Y(n, :) V(cols, :)^T (Vc and Yn in shared memory)
+        double s0 = 0.0, s1 = 0.0;
+#pragma unroll
+        for (int kk = fq; kk < KT; kk += 8) {
+            s0 += S.Vc[kk][fcol] * S.Yn[kk];
+            s1 += S.Vc[kk + 4][fcol] * S.Yn[kk + 4];
+        }
+        s0 += s1;
+        s0 += __shfl_xor_sync(0xffffffffu, s0, 1);
+        s0 += __shfl_xor_sync(0xffffffffu, s0, 2);
+        if (fq == 0 && fcol < ncols) p.A[p.r_hi + (int64_t)(cb + fcol) * p.lda] = cold + sg * s0;
+    }
     if (do_w) {
         // deterministic partial of this row split: Wpart[split][col][j]; the two row warps of each
         // column group meet in shared memory first (wr = 1 stores, wr = 0 adds and writes out)
@@ -345,12 +371,10 @@ __global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
         if (p.Wt) {
             // the last CTA of the strip sums the partials (fixed order) and forms W' = op(T) W
             __shared__ int last;
-            __threadfence();
             __syncthreads();
-            if (tid == 0) last = atomicAdd(&p.strip_done[blockIdx.x], 1) == (int)gridDim.y - 1;
+            if (tid == 0) last = atom_add_acqrel_s32(&p.strip_done[blockIdx.x], 1) == (int)gridDim.y - 1;
             __syncthreads();
             if (last) {
-                __threadfence();
                 double(*Ts)[SK] = S.Vc;  // reuse: T as Ts[a][b] (KT x KT)
                 double(*Ws)[SK] = S.Ys;  // W as Ws[col][b] (64 x KT): spans Ys and Vr (contiguous)
                 for (int i = tid; i < KT * KT; i += UT) {
@@ -434,10 +458,13 @@ static cudaError_t launch_right_kt(const GemmRightParams &p, cudaStream_t s) {
         if (e != cudaSuccess) return e;
         attr |= dbit;
     }
-    const int nstrip = (p.c_hi - p.c_lo + UB - 1) / UB + (p.has_m ? 1 : 0);
-    const int ny = p.nsplit > 0 ? p.nsplit : 1;
+    GemmRightParams q = p;
+    q.fold_row = p.fold_row && p.do_right && p.cm_G <= 1 && p.r_hi - 1 > p.r_lo ? 1 : 0;
+    if (q.fold_row) q.r_hi = p.r_hi - 1;  // row r_hi-1 (c) is folded into the last row split
+    const int nstrip = (q.c_hi - q.c_lo + UB - 1) / UB + (q.has_m ? 1 : 0);
+    const int ny = q.nsplit > 0 ? q.nsplit : 1;
     g_ft_launches++;
-    k_gemm_right<KT><<<dim3(nstrip, ny), UT, smem, s>>>(p);
+    k_gemm_right<KT><<<dim3(nstrip, ny), UT, smem, s>>>(q);
     return cudaGetLastError();
 }
 cudaError_t ft_launch_gemm_right(const GemmRightParams &p, cudaStream_t s) {
@@ -518,8 +545,11 @@ __global__ void k_wprep(const double *__restrict__ Wpart, int64_t wstride, int n
 
 template <int KT>
 __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
-    if (p.ctl && p.ctl->halt) return;
-    if (p.tctl && __ldcg(&p.tctl->tbad)) {  // the right update consumed a corrupted T: nothing here runs
+    // both flags in flight together (one round trip before the launch's first load)
+    const int halted = p.ctl ? __ldcg(&p.ctl->halt) : 0;
+    const int tbad = p.tctl ? __ldcg(&p.tctl->tbad) : 0;
+    if (halted) return;
+    if (tbad) {  // the right update consumed a corrupted T: nothing here runs
         if (blockIdx.x == 0 && blockIdx.y == 0 && threadIdx.x == 0) {
             FtCtl *ctl = p.tctl;
             ctl->halt_panel = p.panel;
@@ -763,8 +793,7 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
             *pk = *pk + sg * k0;
         }
     }
-    if (p.fold && part) __threadfence();  // the fold's stores precede this CTA's done_left increment
-    if (!p.endcheck || !part) return;
+    if (!p.endcheck || !part) return;  // (the fold's stores reach the last CTA through the acq_rel below)
     // fused end-of-iteration check (Alg. 3 l.12-13; R11/R22): the CTA's partial sums go into
     // ctl->sums[2:4]; once every CTA has finished, the last one compares sum r and sum c with
     // kappa (EAGER) or with each other (PAPER)
@@ -785,12 +814,10 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
         }
         atomicAdd(&p.ectl->sums[2], a);
         atomicAdd(&p.ectl->sums[3], b);
-        __threadfence();
-        last = atomicAdd(&p.ectl->done_left, 1) == pcnt - 1;
+        last = atom_add_acqrel_s32(&p.ectl->done_left, 1) == pcnt - 1;
     }
     __syncthreads();
     if (!last || tid != 0) return;
-    __threadfence();
     const int n = p.n;
     const double Sr = __ldcg(&p.ectl->sums[2]), Sc = __ldcg(&p.ectl->sums[3]);
     p.ectl->sums[2] = 0.0;

@@ -132,6 +132,11 @@ struct GemmRightParams {
     // T checksum check (ABFT): the last CTA of each strip verifies the T it read against ctl->tchk
     // before forming W' = op(T) W; on a mismatch it sets ctl->tbad (non-NULL: check on)
     FtCtl *tctl;
+    // fold (ABFT, single rank): the column-checksum row c = row r_hi-1 (= n) is not a tile row;
+    // the CTAs of the last row split update it as a GEMV c(cols) += sign Y(n, :) V(cols, :)^T
+    // (kappa with the column-n strip), so a whole 64-row tile is not spent on one row and the row
+    // splits see the data rows only (nsplit: ft_gemm_splits over [r_lo, r_hi-1))
+    int fold_row;
 };
 // global column of local column l in the 1-D block-column cyclic layout; local column ncl
 // is the replicated row-checksum column r (global n)

@@ -264,6 +264,39 @@ def test_checksums_at_every_boundary(n, nb):
         assert rel(dA.cpu().numpy(), Aw) <= TOL, t
 
 
+@pytest.mark.parametrize("n,nb", [(256, 64), (320, 32), (513, 64), (1024, 32), (2048, 32)])
+def test_right_update_row_fold_matches_tiles(n, nb):
+    """The ABFT right update's column-checksum row c as a GEMV of the last row split (default)
+    against c as one more DMMA tile row (ft_debug_right_fold(0)): H, tau and the maintained
+    checksums at a mid boundary agree to rounding and both meet the oracle; flips of c before
+    the panel and after the right update are still handled (located, or rolled back to the
+    checkpoint that predates them)."""
+    A = synth.matrix(n, dist="normal")
+    L = ft.lib()
+    L.ft_debug_right_fold.argtypes = [ctypes.c_int]
+    t = ((n - 2 + nb - 1) // nb) // 2
+    out = []
+    for fold in (1, 0):
+        L.ft_debug_right_fold(fold)
+        try:
+            chk = torch.zeros(2 * n + 1, dtype=torch.float64, device="cuda")
+            dAs, _, rs = gpu_reduce(A, nb=nb, stop_after_panel=t, dchk_out=chk)
+            dA, tau, res = gpu_reduce(A, nb=nb)
+        finally:
+            L.ft_debug_right_fold(1)
+        assert rs.info == 0 and res.info == 0 and res.report.detected == 0, res.events
+        check_against_oracle(A, dA, tau, nb=nb)
+        out.append((dA.cpu().numpy(), chk.cpu().numpy()))
+    (H1, c1), (H0, c0) = out
+    assert rel(np.triu(H1, -1), np.triu(H0, -1)) <= 1e-11
+    assert np.abs(c1 - c0).max() <= 1e-11 * np.linalg.norm(A)
+    for ph, site, i, j in ((ft.PHASE_BEFORE_PANEL, ft.SITE_C, -1, n - 3), (ft.PHASE_AFTER_RIGHT, ft.SITE_C, -1, n - 3),
+                           (ft.PHASE_AFTER_RIGHT, ft.SITE_K, -1, -1)):
+        dA, tau, res = gpu_reduce(A, nb=nb, faults=[(1, ph, site, i, j, 52)])
+        assert res.info == 0 and res.report.detected + res.report.rollbacks >= 1, res.events
+        check_against_oracle(A, dA, tau, nb=nb)
+
+
 @pytest.mark.parametrize("n,nb", [(256, 64), (320, 32), (513, 64), (1024, 32)])
 def test_left_update_fold_matches_tiles(n, nb):
     """The ABFT left update's checksum row/column folded into the last tile row / strip
