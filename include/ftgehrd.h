@@ -226,8 +226,10 @@ int64_t ft_launch_count(int reset);
  * ft_debug_time_panels(1) resets and starts recording CUDA events around every panel
  * kernel launch on its stream; ft_debug_panel_ms() / ft_debug_panel_launches() return the
  * summed device time and launch count of completed calls.  ft_debug_probe_panel(t, dbuf)
- * makes CTA 0 of panel t write per-column phase timestamps (%globaltimer, 16 slots per
- * column, device buffer of 64*16 uint64) -- t = -1 disables. */
+ * makes CTA 0 of panel t write per-column phase timestamps (clock64, 16 slots per column at
+ * [j*16], the max over CTAs of each phase at [1024 + j*16]; the wide kernel's per-CTA GEMV spans
+ * at [2048 + 4*cta]; CTA 0's kernel entry / epilogue end at [3072] / [3073]: a device buffer of
+ * 3088 uint64) -- t = -1 disables. */
 void ft_debug_time_panels(int on);
 double ft_debug_panel_ms(void);
 int ft_debug_panel_launches(void);

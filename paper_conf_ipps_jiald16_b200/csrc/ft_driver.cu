@@ -435,6 +435,8 @@ struct Call {
     std::vector<ft_event> events;
     int detected = 0, corrected = 0, rollbacks = 0, redos = 0, uncorrectable = 0;
     int npanels = 0;
+    int last = 0;           // panels enqueued by this call (stop_after_panel)
+    int defer_from = -1;    // the next panel launch evaluates the end check of this iteration
     // host-buffer call (ft_dgehrd_host): the input is copied straight into the working array and
     // every iteration's finished columns [k, e) are copied back on w->copy_stream while the
     // following panels run (they are never touched again, except by a recovery: re-copied)
@@ -729,6 +731,12 @@ int enqueue_panel(Call &C, int t) {
     p.verify = eager ? 1 : 0;
     const bool fuse_pre = eager && !has_fault(C, t, FT_PHASE_AFTER_PANEL);
     p.precheck_sums = fuse_pre ? 1 : 0;
+    if (C.defer_from == t - 1 && t > 0) {  // the end check of iteration t-1, at this launch's entry
+        p.echeck = 1;
+        p.echeck_panel = t - 1;
+        p.echeck_policy = C.policy;
+    }
+    C.defer_from = -1;
     p.dbg = (t == g_dbg_panel) ? g_dbg_buf : nullptr;
     p.dbg_mode = ((t == g_dbg_panel) ? g_dbg_mode : 0) | g_panel_path;
     const int gr = ft_panel_group_rows();
@@ -789,9 +797,14 @@ int enqueue_panel(Call &C, int t) {
     if (inject_at(C, t, FT_PHASE_AFTER_RIGHT)) return FT_E_CUDA;
     // the weighted pair (NEXT-1) takes the separate end check, which also sums r_w and c_w
     const bool fuse_end = C.abft && !C.weighted && !has_fault(C, t, FT_PHASE_AFTER_UPDATE);
+    // deferred to the next panel launch's entry (no last-CTA chain on this launch's tail) when one
+    // follows in this sequence with nothing injected in between
+    const bool defer_end = fuse_end && t + 1 < C.last && !has_fault(C, t + 1, FT_PHASE_BEFORE_PANEL);
     {
         const int sp = span_begin(C, TC_LEFT), sk = span_begin(C, TK_LEFT);
-        if (left_update(C, t, -1.0, trailing_nsplit(C, t), fuse_end ? 1 : 0, fuse_pre)) return FT_E_CUDA;
+        if (left_update(C, t, -1.0, trailing_nsplit(C, t), fuse_end ? (defer_end ? 2 : 1) : 0, fuse_pre))
+            return FT_E_CUDA;
+        if (defer_end) C.defer_from = t;
         span_end(C, sk);
         span_end(C, sp);
     }
@@ -1329,6 +1342,7 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
     C.npanels = 0;
     for (int k = ilo - 1; k < ihi - 2; k += C.nb) C.npanels++;
     const int last = (o.stop_after_panel >= 0) ? std::min(o.stop_after_panel + 1, C.npanels) : C.npanels;
+    C.last = last;
     // Fault-free calls replay one CUDA graph of the whole launch sequence (start-up kernels and
     // every iteration), captured on the second call with the same shape and buffers; the halt
     // protocol is unchanged (a halted graph's remaining kernels are no-ops, recovery follows).
@@ -1415,6 +1429,7 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
             info = FT_E_UNCORRECTABLE;
             break;
         }
+        C.defer_from = -1;  // recovery re-checks: the redo starts without a pending end check
         rc = recover(C, h);
         if (rc == FT_E_UNCORRECTABLE) {
             info = rc;

@@ -122,6 +122,10 @@ __global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
     // the halt flag is loaded here but first used at the first tile's barrier (before any store),
     // so its round trip overlaps the operand loads instead of delaying them
     const int halted = p.ctl ? __ldcg(&p.ctl->halt) : 0;
+    // the panel's T row sums for the T check of the strip's last CTA (which CTA is last is known
+    // only at the end: every CTA prefetches, so the check carries no load round trip)
+    const double tchk_pre = (p.tctl && p.Wt && (threadIdx.x & 3) == 0 && (int)(threadIdx.x >> 2) < p.K)
+                                ? __ldcg(&p.tctl->tchk[threadIdx.x >> 2]) : 0.0;
     // fused pre-update check: warp 0 evaluates it while the other warps start the operand and
     // C-tile loads; the decision is read at the first tile's barrier, before any store
     __shared__ int s_reason;
@@ -419,7 +423,7 @@ __global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
                     t_row_checksum([&](int a, int bb) { return Ts[a][bb]; }, tid >> 2, tid & 3, K, ts, tsa);
                     const int a = tid >> 2;
                     if ((tid & 3) == 0 && a < K &&
-                        not_within(ts - __ldcg(&p.tctl->tchk[a]), (double)K * 2.220446049250313e-16 * tsa))
+                        not_within(ts - tchk_pre, (double)K * 2.220446049250313e-16 * tsa))
                         p.tctl->tbad = 1;
                 }
                 // W' = op(T) W: this thread's NE outputs as independent chains (one pass over b)
@@ -814,7 +818,8 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
         }
         atomicAdd(&p.ectl->sums[2], a);
         atomicAdd(&p.ectl->sums[3], b);
-        last = atom_add_acqrel_s32(&p.ectl->done_left, 1) == pcnt - 1;
+        // deferred: the next panel launch compares the sums (kernel boundary orders them)
+        last = p.endcheck == 2 ? 0 : atom_add_acqrel_s32(&p.ectl->done_left, 1) == pcnt - 1;
     }
     __syncthreads();
     if (!last || tid != 0) return;

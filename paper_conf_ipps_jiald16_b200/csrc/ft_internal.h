@@ -69,6 +69,12 @@ struct PanelParams {
     // diskless checkpoint of the panel, taken in the kernel's prologue, or NULL
     double *ckpt, *ck_r, *ck_c, *ck_q, *Fr;
     int precheck_sums;  // add e^T Y, e^T V of the own rows into ctl->eY / eV (fused pre-update check)
+    // deferred end check of the previous iteration (left update with endcheck = 2): every CTA
+    // reads ctl->sums[2:4] and kappa at entry, with the halt flag, and compares them before its
+    // first store (EAGER: sum r and sum c against kappa; PAPER: with each other); a failure
+    // raises the halt for panel echeck_panel (stage 2) and the launch does nothing.  CTA 0 clears
+    // the sums after the first grid barrier.
+    int echeck, echeck_panel, echeck_policy;
     unsigned long long *dbg;          // optional per-column phase timestamps (CTA 0), or NULL
     int dbg_mode;                     // timing ablations (wrong results): 1 no grid barriers, 2 no GEMV, 4 no atomics;
                                       // 8: every column on the explicit (two-reduction) path (exact)
@@ -163,7 +169,8 @@ struct GemmLeftParams {
     double sign;    // -1 update, +1 rollback
     const FtCtl *ctl;
     int wt_ready;   // 1: Wt already holds op(T) W (formed by the right-update launch)
-    // fused end-of-iteration check (Alg. 3 l.12-13) + frozen row sums; last CTA decides
+    // end-of-iteration check (Alg. 3 l.12-13) + frozen row sums: endcheck 1 = fused, the last CTA
+    // decides; 2 = the partial sums only (the next panel launch decides, PanelParams::echeck)
     int endcheck, panel, policy, n;
     double *Fr;
     FtCtl *ectl;

@@ -89,6 +89,7 @@ struct PanelSmem {
     double b0[RMAX];                    // b0 of the current column
     double bmA[RMAX];                   // b0 masked to the data rows
     double bmX[RMAX];                   // b0 (or x) masked to the data rows >= c+2
+    double rref[RMAX];                  // verify: r(row) - Fr(row) of the own rows (loaded in the prologue)
     double2 red[PT];                    // GEMV partials  (y pairs)
     double2 rsr[PT];                    // GEMV partials  (row sums, verify pass)
     unsigned long long drift;           // max fault-free |D_r| of the CTA's rows (reduced once per panel)
@@ -255,7 +256,36 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
     const int vr = MG ? (int)(blockIdx.x / P) : 0;
     const PanelParams &p = L.r[vr];
     const int bid = (int)(blockIdx.x - vr * P);
-    if (p.ctl->halt) return;  // uniform for the whole grid (nobody writes halt in this launch)
+    {
+        // the halt flag and, when deferred here, the previous iteration's end-check sums: one round
+        // trip, every CTA on the same words (a uniform decision; nobody writes them in this launch)
+        const int halted = __ldcg(&p.ctl->halt);
+        double e_sr = 0.0, e_sc = 0.0, e_kap = 0.0, e_nf = 0.0, e_thr = 0.0;
+        if (p.echeck) {
+            e_sr = __ldcg(&p.ctl->sums[2]);
+            e_sc = __ldcg(&p.ctl->sums[3]);
+            e_kap = __ldcg(p.A + p.n + (int64_t)p.n * p.ldw);
+            e_nf = __ldcg(&p.ctl->normF);
+            e_thr = __ldcg(&p.ctl->c_thr);
+        }
+        if (halted) return;
+        if (p.echeck) {  // Alg. 3 l.12-13 of iteration echeck_panel (R11/R22), as the fused check
+            const double tauS = e_thr * (double)p.n * 2.220446049250313e-16 * e_nf * sqrt((double)p.n);
+            const bool bad = p.echeck_policy == FT_POLICY_PAPER
+                                 ? not_within(e_sr - e_sc, tauS)
+                                 : (not_within(e_sr - e_kap, tauS) || not_within(e_sc - e_kap, tauS));
+            if (bad) {
+                if (blockIdx.x == 0 && threadIdx.x == 0) {
+                    p.ctl->halt_panel = p.echeck_panel;
+                    p.ctl->halt_stage = 2;
+                    p.ctl->halt_reason = 8;
+                    __threadfence();
+                    p.ctl->halt = 1;
+                }
+                return;  // nothing touched: the previous iteration is rolled back
+            }
+        }
+    }
     extern __shared__ __align__(16) unsigned char smem_raw[];
     PanelSmem &S = *reinterpret_cast<PanelSmem *>(smem_raw);
 
@@ -437,6 +467,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
     unsigned epoch = 0;
     long long probe_last = 0;
     int j = 0;  // (PROBE)
+    if (p.dbg && bid == 0 && tid == 0) p.dbg[3072] = clock64();  // kernel entry (CTA 0): prologue = dbg[0] - this
     // ======================= the trailing GEMV (warps with IS_GEMV_WARP) =========================
     // partials of A(rows, c+2:cend) bv(c+2:cend) (and of the row sums when vfy) into S.red / S.rsr
     auto gemv = [&](const double *bv, int c, bool vfy) {
@@ -553,29 +584,80 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
         (&S.Ts[0][0])[i] = 0.0;
         (&S.Km[0][0])[i] = 0.0;
     }
+    if (ncc > 0) {
+        // the row slab of columns [k+2, k+2+ncc) into shared memory: at panel start they hold
+        // A0, and column c's GEMV reads only columns >= c+2, which this panel has not written yet.
+        // Issued first: the checkpoint and column-k loads below overlap its flight
+        const int R2c = R >> 1;
+        for (int x = tid; x < ncc * R2c; x += PT) {
+            const int cc = x / R2c, rq = x - cc * R2c;
+            cp_async16(Ac + (int64_t)cc * R + 2 * rq, A + (r0 + 2 * rq) + (int64_t)(k + 2 + cc) * ldw, 16);
+        }
+        cp_async_commit();
+    }
     if (p.ckpt) {
         // diskless checkpoint of the panel columns, r, c, kappa, Qr, Qc, Fr, taken
         // before anything is modified: own rows by their owner, the rest grid-strided; all of it
         // precedes this CTA's first arrival
+        // (every loop issues its loads before its stores: one round trip per batch, not per word)
         const int rend = p.abft ? n + 1 : ihi;
-        for (int x = tid; x < R * ib; x += PT) {
-            const int rl = x % R, jj = x / R, row = r0 + rl;
-            if (row < rend) p.ckpt[row + (int64_t)jj * ldw] = Apan[row + (int64_t)(k + jj) * ldw];
-        }
+        // r, Qr, Qc, Fr and the checksum row c, grid-strided: loaded here, in flight with the first
+        // batch of panel columns, stored after it (the owner of row n rewrites c(k:e) only after
+        // the first grid sync, which every copy precedes)
         const int gstride = (int)P * PT, gi = bid * PT + tid;
-        for (int x = gi; x < p.rbase * ib; x += gstride) {
-            const int i = x % p.rbase, jj = x / p.rbase;
-            p.ckpt[i + (int64_t)jj * ldw] = Apan[i + (int64_t)(k + jj) * ldw];
+        // interleaved over the CTAs (entry bid + P * tid), so CTAs 0..4 carry no extra copies
+        const int vi = bid + (int)P * tid;
+        double vr = 0.0, vq = 0.0, vc = 0.0, vf = 0.0, vk = 0.0;
+        if (vi <= n) {
+            vr = p.rcol[vi];
+            vq = p.Qr[vi];
+            vc = p.Qc[vi];
+            vf = p.Fr[vi];
+            vk = A[n + (int64_t)vi * ldw];
         }
-        for (int i = gi; i <= n; i += gstride) {
-            p.ck_r[i] = p.rcol[i];
-            p.ck_q[i] = p.Qr[i];
-            p.ck_q[ldw + i] = p.Qc[i];
-            p.ck_q[2 * ldw + i] = p.Fr[i];
+#pragma unroll 1
+        for (int x0 = tid; x0 < R * ib; x0 += 4 * PT) {
+            double v[4];
+#pragma unroll
+            for (int u = 0; u < 4; u++) {
+                const int x = x0 + u * PT, rl = x % R, jj = x / R, row = r0 + rl;
+                v[u] = (x < R * ib && row < rend) ? Apan[row + (int64_t)(k + jj) * ldw] : 0.0;
+            }
+#pragma unroll
+            for (int u = 0; u < 4; u++) {
+                const int x = x0 + u * PT, rl = x % R, jj = x / R, row = r0 + rl;
+                if (x < R * ib && row < rend) p.ckpt[row + (int64_t)jj * ldw] = v[u];
+            }
         }
-        // the checksum row c, grid-strided: every copy precedes its CTA's first arrival, and the
-        // owner of row n rewrites c(k:e) only after that first grid sync
-        for (int i = gi; i <= n; i += gstride) p.ck_c[i] = A[n + (int64_t)i * ldw];
+#pragma unroll 1
+        for (int x0 = gi; x0 < p.rbase * ib; x0 += 4 * gstride) {  // rows above the panel
+            double v[4];
+#pragma unroll
+            for (int u = 0; u < 4; u++) {
+                const int x = x0 + u * gstride;
+                v[u] = x < p.rbase * ib ? Apan[x % p.rbase + (int64_t)(k + x / p.rbase) * ldw] : 0.0;
+            }
+#pragma unroll
+            for (int u = 0; u < 4; u++) {
+                const int x = x0 + u * gstride;
+                if (x < p.rbase * ib) p.ckpt[x % p.rbase + (int64_t)(x / p.rbase) * ldw] = v[u];
+            }
+        }
+        if (vi <= n) {
+            p.ck_r[vi] = vr;
+            p.ck_q[vi] = vq;
+            p.ck_q[ldw + vi] = vc;
+            p.ck_q[2 * ldw + vi] = vf;
+            p.ck_c[vi] = vk;
+        }
+        for (int i = gi + gstride; i <= n; i += gstride) {  // n >= P * PT only (entries past the first P * PT)
+            const double wr = p.rcol[i], wq = p.Qr[i], wc = p.Qc[i], wf = p.Fr[i], wk = A[n + (int64_t)i * ldw];
+            p.ck_r[i] = wr;
+            p.ck_q[i] = wq;
+            p.ck_q[ldw + i] = wc;
+            p.ck_q[2 * ldw + i] = wf;
+            p.ck_c[i] = wk;
+        }
     }
     {
         // column k: b0 = A(:, k); publish its x part (rows >= k+2) and b0(k+1)
@@ -584,6 +666,8 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
         for (int rl = tid; rl < R; rl += PT) {
             const int row = r0 + rl;
             const double b = is_valid(row) ? Apan[row + (int64_t)k * ldw] : 0.0;
+            if (p.verify && (is_data(row) || is_top(row)))  // the D_r reference, in flight with b
+                S.rref[rl] = p.rcol[row] - (is_top(row) ? p.Fr[row] : 0.0);
             const bool d = is_data(row), xr = d && row >= k + 2;
             S.acol[rl] = b;
             S.b0[rl] = b;
@@ -594,17 +678,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
         }
     }
     if (tid < FT_NBMAX) S.ep[tid] = 0.0;
-    if (ncc > 0) {
-        // the row slab of columns [k+2, k+2+ncc) into shared memory: at panel start they hold
-        // A0, and column c's GEMV reads only columns >= c+2, which this panel has not written yet
-        const int R2c = R >> 1;
-        for (int x = tid; x < ncc * R2c; x += PT) {
-            const int cc = x / R2c, rq = x - cc * R2c;
-            cp_async16(Ac + (int64_t)cc * R + 2 * rq, A + (r0 + 2 * rq) + (int64_t)(k + 2 + cc) * ldw, 16);
-        }
-        cp_async_commit();
-        cp_async_wait<0>();
-    }
+    if (ncc > 0) cp_async_wait<0>();  // the row slab (issued first in the prologue)
     if (tid == 0 && bid == 0) *p.bar_next = 0u;  // the next panel launch's counter
     if (tid == 0) S.drift = 0ull;
     __syncthreads();
@@ -649,6 +723,10 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
         PROBE(1);
         double s1a = 0.0, s1b = 0.0, sxa = 0.0, sxb = 0.0, vra = 0.0, vrb = 0.0, bb = 0.0, eb = 0.0, b0c1 = 0.0;
         grid_sync(epoch, [&]() {
+            if (j == 0 && bid == 0 && lane == 0 && p.echeck) {  // every CTA has read the deferred sums
+                p.ctl->sums[2] = 0.0;
+                p.ctl->sums[3] = 0.0;
+            }
             bb = ldcg(acc + ACC_BB * FT_ACC_PAD);
             eb = ldcg(acc + ACC_EB * FT_ACC_PAD);
             b0c1 = ldcg(acc + ACC_B0 * FT_ACC_PAD);
@@ -942,7 +1020,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
                             // D_r(row) = r(row) - sum_{col >= k} L(row, col); columns < k are logical zero
                             // for data rows, the frozen finished-H sums Fr for the rows above (area 1)
                             rsum += S.acol[rl] + an;
-                            const double d = p.rcol[row] - (is_top(row) ? p.Fr[row] : 0.0) - rsum;
+                            const double d = S.rref[rl] - rsum;
                             if (not_within(d, tau_abs)) {
                                 atomicAdd(&p.ctl->nflag, 1);
                             } else if (tau_abs > 0.0) {
@@ -997,41 +1075,49 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
             double s = 0.0;
             for (int jj = 0; jj < ib; jj++)
                 if (row >= k + jj + 2) s += Vl[rl * XR + jj * XC];
-            p.Qr[row] += s;
+            atomicAdd(&p.Qr[row], s);  // one writer per row: a plain Qr + s, without the load round trip
         }
-    if (p.precheck_sums)  // e^T Y, e^T V over the own data rows (pre-update check R15, fused): a warp per column
-        for (int o = wid; o < 2 * ib; o += NW) {
-            const int jj = o % ib;
+    if (p.precheck_sums) {  // e^T Y, e^T V over the own data rows (pre-update check R15, fused): 8 lanes per sum
+        const int l8 = tid & 7;  // 2 ib <= 128 sums over 64 groups; the loop bound is warp-uniform
+        for (int base = (tid >> 5) * 4; base < 2 * ib; base += PT / 8) {
+            const int oo = base + ((tid >> 3) & 3), jj = oo % ib;
             double s = 0.0;
-            for (int rl = lane; rl < R; rl += 32)
-                if (is_data(r0 + rl) || is_top(r0 + rl)) s += o < ib ? Yl[rl * YR + jj * YCS] : Vl[rl * XR + jj * XC];
-            s = warp_sum(s);
-            if (lane == 0) atomicAdd(o < ib ? &p.ctl->eY[jj * FT_ESTR] : &p.ctl->eV[jj * FT_ESTR], s);
+            if (oo < 2 * ib)
+                for (int rl = l8; rl < R; rl += 8)
+                    if (is_data(r0 + rl) || is_top(r0 + rl)) s += oo < ib ? Yl[rl * YR + jj * YCS] : Vl[rl * XR + jj * XC];
+            s += __shfl_xor_sync(0xffffffffu, s, 1);
+            s += __shfl_xor_sync(0xffffffffu, s, 2);
+            s += __shfl_xor_sync(0xffffffffu, s, 4);
+            if (l8 == 0 && oo < 2 * ib) atomicAdd(oo < ib ? &p.ctl->eY[jj * FT_ESTR] : &p.ctl->eV[jj * FT_ESTR], s);
         }
-    if (bid == 0 && tid == 0 && p.abft) p.Qc[n] += qc_corner;
-    if (bid == 0) {
+    }
+    if (bid == 0 && tid == 0 && p.abft) atomicAdd(&p.Qc[n], qc_corner);  // single writer: Qc(n) + corner
+    // T, max |T| and the T checksum from three different CTAs (every CTA holds T in shared memory),
+    // so no CTA carries all three serial tails
+    const int P3 = (int)P;
+    if (bid == (P3 > 1 ? 1 : 0))
+        for (int i = tid; i < ib * ib; i += PT) p.T[i % ib + (i / ib) * FT_NBMAX] = S.Ts[i % ib][i / ib];
+    if (p.precheck_sums && bid == (P3 > 2 ? 2 : 0)) {  // max |T| for the pre-update tolerance (R15)
         double tm = 0.0;
-        for (int i = tid; i < ib * ib; i += PT) {
-            int a = i % ib, bb = i / ib;
-            p.T[a + bb * FT_NBMAX] = S.Ts[a][bb];
-            tm = fmax(tm, fabs(S.Ts[a][bb]));
-        }
-        if (p.precheck_sums) {  // max |T| for the pre-update tolerance (R15), read by the right update
+        for (int i = tid; i < ib * ib; i += PT) tm = fmax(tm, fabs(S.Ts[i % ib][i / ib]));
 #pragma unroll
-            for (int o = 16; o > 0; o >>= 1) tm = fmax(tm, __shfl_xor_sync(0xffffffffu, tm, o));
-            if (lane == 0) S.red[wid].x = tm;
-            __syncthreads();
-            if (tid == 0) {
-                double m = 0.0;
-                for (int w = 0; w < NW; w++) m = fmax(m, S.red[w].x);
-                p.ctl->tmax = m;
-            }
+        for (int o = 16; o > 0; o >>= 1) tm = fmax(tm, __shfl_xor_sync(0xffffffffu, tm, o));
+        if (lane == 0) S.red[wid].x = tm;
+        __syncthreads();
+        if (tid == 0) {
+            double m = 0.0;
+            for (int w = 0; w < NW; w++) m = fmax(m, S.red[w].x);
+            p.ctl->tmax = m;
         }
-        if (p.abft && tid < 4 * FT_NBMAX) {  // T checksum (R15 extended to T), read by the right update
-            double ts, tsa;
-            t_row_checksum([&](int a, int bb) { return S.Ts[a][bb]; }, tid >> 2, tid & 3, ib, ts, tsa);
-            if ((tid & 3) == 0 && (tid >> 2) < ib) p.ctl->tchk[tid >> 2] = ts;
-        }
+    }
+    if (p.abft && bid == (P3 > 3 ? 3 : 0) && tid < 4 * FT_NBMAX) {  // T checksum (R15 extended to T)
+        double ts, tsa;
+        t_row_checksum([&](int a, int bb) { return S.Ts[a][bb]; }, tid >> 2, tid & 3, ib, ts, tsa);
+        if ((tid & 3) == 0 && (tid >> 2) < ib) p.ctl->tchk[tid >> 2] = ts;
+    }
+    if (p.dbg && bid == 0) {  // epilogue end (CTA 0): epilogue = this - the last column's end
+        __syncthreads();
+        if (tid == 0) p.dbg[3073] = clock64();
     }
 }
 

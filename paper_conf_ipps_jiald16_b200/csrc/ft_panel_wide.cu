@@ -148,7 +148,36 @@ __global__ void __launch_bounds__(PT, 1) k_panel_wide(const __grid_constant__ Pa
     const int vr = MG ? (int)(blockIdx.x / P) : 0;
     const PanelParams &p = L.r[vr];
     const int bid = (int)(blockIdx.x - vr * P);
-    if (p.ctl->halt) return;  // uniform for the whole grid (nobody writes halt in this launch)
+    {
+        // the halt flag and, when deferred here, the previous iteration's end-check sums: one round
+        // trip, every CTA on the same words (a uniform decision; nobody writes them in this launch)
+        const int halted = __ldcg(&p.ctl->halt);
+        double e_sr = 0.0, e_sc = 0.0, e_kap = 0.0, e_nf = 0.0, e_thr = 0.0;
+        if (p.echeck) {
+            e_sr = __ldcg(&p.ctl->sums[2]);
+            e_sc = __ldcg(&p.ctl->sums[3]);
+            e_kap = __ldcg(p.A + p.n + (int64_t)p.n * p.ldw);
+            e_nf = __ldcg(&p.ctl->normF);
+            e_thr = __ldcg(&p.ctl->c_thr);
+        }
+        if (halted) return;
+        if (p.echeck) {  // Alg. 3 l.12-13 of iteration echeck_panel (R11/R22), as the fused check
+            const double tauS = e_thr * (double)p.n * 2.220446049250313e-16 * e_nf * sqrt((double)p.n);
+            const bool bad = p.echeck_policy == FT_POLICY_PAPER
+                                 ? not_within(e_sr - e_sc, tauS)
+                                 : (not_within(e_sr - e_kap, tauS) || not_within(e_sc - e_kap, tauS));
+            if (bad) {
+                if (blockIdx.x == 0 && threadIdx.x == 0) {
+                    p.ctl->halt_panel = p.echeck_panel;
+                    p.ctl->halt_stage = 2;
+                    p.ctl->halt_reason = 8;
+                    __threadfence();
+                    p.ctl->halt = 1;
+                }
+                return;  // nothing touched: the previous iteration is rolled back
+            }
+        }
+    }
     extern __shared__ __align__(16) unsigned char smem_raw[];
     PanelSmemW &S = *reinterpret_cast<PanelSmemW *>(smem_raw);
 
@@ -264,25 +293,47 @@ __global__ void __launch_bounds__(PT, 1) k_panel_wide(const __grid_constant__ Pa
         // diskless checkpoint of the panel columns, r, c, kappa, Qr, Qc, Fr, taken
         // before anything is modified: own rows by their owner, the rest grid-strided; all of it
         // precedes this CTA's first arrival
+        // (every loop issues its loads before its stores: one round trip per batch, not per word)
         const int rend = p.abft ? n + 1 : ihi;
-        for (int x = tid; x < R * ib; x += PT) {
-            const int rl = x % R, jj = x / R, row = r0 + rl;
-            if (row < rend) p.ckpt[row + (int64_t)jj * ldw] = Apan[row + (int64_t)(k + jj) * ldw];
+#pragma unroll 1
+        for (int x0 = tid; x0 < R * ib; x0 += 8 * PT) {
+            double v[8];
+#pragma unroll
+            for (int u = 0; u < 8; u++) {
+                const int x = x0 + u * PT, rl = x % R, jj = x / R, row = r0 + rl;
+                v[u] = (x < R * ib && row < rend) ? Apan[row + (int64_t)(k + jj) * ldw] : 0.0;
+            }
+#pragma unroll
+            for (int u = 0; u < 8; u++) {
+                const int x = x0 + u * PT, rl = x % R, jj = x / R, row = r0 + rl;
+                if (x < R * ib && row < rend) p.ckpt[row + (int64_t)jj * ldw] = v[u];
+            }
         }
         const int gstride = (int)P * PT, gi = bid * PT + tid;
-        for (int x = gi; x < p.rbase * ib; x += gstride) {
-            const int i = x % p.rbase, jj = x / p.rbase;
-            p.ckpt[i + (int64_t)jj * ldw] = Apan[i + (int64_t)(k + jj) * ldw];
+#pragma unroll 1
+        for (int x0 = gi; x0 < p.rbase * ib; x0 += 4 * gstride) {  // rows above the panel
+            double v[4];
+#pragma unroll
+            for (int u = 0; u < 4; u++) {
+                const int x = x0 + u * gstride;
+                v[u] = x < p.rbase * ib ? Apan[x % p.rbase + (int64_t)(k + x / p.rbase) * ldw] : 0.0;
+            }
+#pragma unroll
+            for (int u = 0; u < 4; u++) {
+                const int x = x0 + u * gstride;
+                if (x < p.rbase * ib) p.ckpt[x % p.rbase + (int64_t)(x / p.rbase) * ldw] = v[u];
+            }
         }
+        // r, Qr, Qc, Fr and the checksum row c, grid-strided: every copy precedes its CTA's first
+        // arrival, and the owner of row n rewrites c(k:e) only after that first grid sync
         for (int i = gi; i <= n; i += gstride) {
-            p.ck_r[i] = p.rcol[i];
-            p.ck_q[i] = p.Qr[i];
-            p.ck_q[ldw + i] = p.Qc[i];
-            p.ck_q[2 * ldw + i] = p.Fr[i];
+            const double vr = p.rcol[i], vq = p.Qr[i], vc = p.Qc[i], vf = p.Fr[i], vk = A[n + (int64_t)i * ldw];
+            p.ck_r[i] = vr;
+            p.ck_q[i] = vq;
+            p.ck_q[ldw + i] = vc;
+            p.ck_q[2 * ldw + i] = vf;
+            p.ck_c[i] = vk;
         }
-        // the checksum row c, grid-strided: every copy precedes its CTA's first arrival, and the
-        // owner of row n rewrites c(k:e) only after that first grid sync
-        for (int i = gi; i <= n; i += gstride) p.ck_c[i] = A[n + (int64_t)i * ldw];
     }
     for (int rl = tid; rl < R; rl += PT) {
         const int row = r0 + rl;
@@ -365,6 +416,10 @@ __global__ void __launch_bounds__(PT, 1) k_panel_wide(const __grid_constant__ Pa
         // control scalars of DLARFG, loaded by warp 0 as soon as the barrier opens
         double nrm2 = 0.0, sx = 0.0, alpha = 0.0, vn0 = 0.0, vt0 = 0.0, vn1 = 0.0, vt1 = 0.0;
         grid_sync(epoch, [&]() {
+            if (j == 0 && bid == 0 && lane == 0 && p.echeck) {  // every CTA has read the deferred sums
+                p.ctl->sums[2] = 0.0;
+                p.ctl->sums[3] = 0.0;
+            }
             nrm2 = ldcg(acc + ACC_NRM * FT_ACC_PAD);
             sx = ldcg(acc + ACC_SX * FT_ACC_PAD);
             alpha = ldcg(acc + ACC_ALPHA * FT_ACC_PAD);
@@ -714,40 +769,41 @@ __global__ void __launch_bounds__(PT, 1) k_panel_wide(const __grid_constant__ Pa
             double s = 0.0;
             for (int jj = 0; jj < ib; jj++)
                 if (row >= k + jj + 2) s += Vl[rl * XR + jj * XC];
-            p.Qr[row] += s;
+            atomicAdd(&p.Qr[row], s);  // one writer per row: a plain Qr + s, without the load round trip
         }
-    if (p.precheck_sums && tid < 2 * ib) {  // e^T Y, e^T V over the own data rows (pre-update check R15, fused)
-        const int jj = tid % ib;
-        const double *X = tid < ib ? Yl : Vl;
+    if (p.precheck_sums) {  // e^T Y, e^T V over the own data rows (pre-update check R15, fused): 4 lanes per sum
+        const int o = tid >> 2, q = tid & 3, jj = o % ib;
+        const double *X = o < ib ? Yl : Vl;
         double s = 0.0;
-        for (int rl = 0; rl < R; rl++)
-            if (is_data(r0 + rl)) s += X[rl * XR + jj * XC];
-        atomicAdd(tid < ib ? &p.ctl->eY[jj * FT_ESTR] : &p.ctl->eV[jj * FT_ESTR], s);
+        if (o < 2 * ib)
+            for (int rl = q; rl < R; rl += 4)
+                if (is_data(r0 + rl)) s += X[rl * XR + jj * XC];
+        s += __shfl_xor_sync(0xffffffffu, s, 1);
+        s += __shfl_xor_sync(0xffffffffu, s, 2);
+        if (q == 0 && o < 2 * ib) atomicAdd(o < ib ? &p.ctl->eY[jj * FT_ESTR] : &p.ctl->eV[jj * FT_ESTR], s);
     }
-    if (bid == 0 && tid == 0 && p.abft) p.Qc[n] += qc_corner;
-    if (bid == 0) {
+    if (bid == 0 && tid == 0 && p.abft) atomicAdd(&p.Qc[n], qc_corner);  // single writer: Qc(n) + corner
+    // T, max |T| and the T checksum from three different CTAs (every CTA holds T in shared memory)
+    const int P3 = (int)P;
+    if (bid == (P3 > 1 ? 1 : 0))
+        for (int i = tid; i < ib * ib; i += PT) p.T[i % ib + (i / ib) * FT_NBMAX] = S.Ts[i % ib][i / ib];
+    if (p.precheck_sums && bid == (P3 > 2 ? 2 : 0)) {  // max |T| for the pre-update tolerance (R15)
         double tm = 0.0;
-        for (int i = tid; i < ib * ib; i += PT) {
-            int a = i % ib, bb = i / ib;
-            p.T[a + bb * FT_NBMAX] = S.Ts[a][bb];
-            tm = fmax(tm, fabs(S.Ts[a][bb]));
-        }
-        if (p.precheck_sums) {  // max |T| for the pre-update tolerance (R15), read by the right update
+        for (int i = tid; i < ib * ib; i += PT) tm = fmax(tm, fabs(S.Ts[i % ib][i / ib]));
 #pragma unroll
-            for (int o = 16; o > 0; o >>= 1) tm = fmax(tm, __shfl_xor_sync(0xffffffffu, tm, o));
-            if (lane == 0) S.red[wid].x = tm;
-            __syncthreads();
-            if (tid == 0) {
-                double m = 0.0;
-                for (int w = 0; w < NW; w++) m = fmax(m, S.red[w].x);
-                p.ctl->tmax = m;
-            }
+        for (int o = 16; o > 0; o >>= 1) tm = fmax(tm, __shfl_xor_sync(0xffffffffu, tm, o));
+        if (lane == 0) S.red[wid].x = tm;
+        __syncthreads();
+        if (tid == 0) {
+            double m = 0.0;
+            for (int w = 0; w < NW; w++) m = fmax(m, S.red[w].x);
+            p.ctl->tmax = m;
         }
-        if (p.abft && tid < 4 * FT_NBMAX) {  // T checksum (R15 extended to T), read by the right update
-            double ts, tsa;
-            t_row_checksum([&](int a, int bb) { return S.Ts[a][bb]; }, tid >> 2, tid & 3, ib, ts, tsa);
-            if ((tid & 3) == 0 && (tid >> 2) < ib) p.ctl->tchk[tid >> 2] = ts;
-        }
+    }
+    if (p.abft && bid == (P3 > 3 ? 3 : 0) && tid < 4 * FT_NBMAX) {  // T checksum (R15 extended to T)
+        double ts, tsa;
+        t_row_checksum([&](int a, int bb) { return S.Ts[a][bb]; }, tid >> 2, tid & 3, ib, ts, tsa);
+        if ((tid & 3) == 0 && (tid >> 2) < ib) p.ctl->tchk[tid >> 2] = ts;
     }
 }
 

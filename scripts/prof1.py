@@ -43,7 +43,7 @@ def main():
     L.ft_debug_panel_launches.restype = ctypes.c_int
     dbg = None
     if a.probe >= 0:
-        dbg = torch.zeros(2048 + 4 * 256, dtype=torch.int64, device="cuda")
+        dbg = torch.zeros(2048 + 4 * 256 + 16, dtype=torch.int64, device="cuda")
         L.ft_debug_probe_panel.argtypes = [ctypes.c_int, ctypes.c_void_p]
         L.ft_debug_probe_panel(a.probe, ctypes.c_void_p(dbg.data_ptr()))
         L.ft_debug_ablate.argtypes = [ctypes.c_int]
@@ -98,6 +98,10 @@ def main():
                   f"start spread {cta[:, 1].max() - t0} ns, end spread {cta[:, 2].max() - cta[:, 2].min()} ns")
             order = np.argsort(cta[:, 0])
             print("  smid:dur_ns " + " ".join(f"{int(cta[q, 0])}:{int(dur[q])}" for q in order))
+        last_end = max(d[j * 16 + 8] for j in range(64))
+        if d[3072] and d[3073]:
+            print(f"CTA 0: prologue {d[0] - d[3072]} cycles, epilogue {d[3073] - last_end} cycles, "
+                  f"kernel {d[3073] - d[3072]} cycles")
         print(f"probe panel {a.probe}: {ncol} columns, mean cycles per column by phase "
               f"(CTA 0 | max over CTAs of the phase):")
         for k2, v in tot.items():

@@ -297,6 +297,25 @@ def test_right_update_row_fold_matches_tiles(n, nb):
         check_against_oracle(A, dA, tau, nb=nb)
 
 
+@pytest.mark.parametrize("n,nb", [(300, 32), (2048, 32), (3000, 64)])
+@pytest.mark.parametrize("site", [ft.SITE_R, ft.SITE_C, ft.SITE_K])
+def test_end_check_deferred_and_fused(n, nb, site):
+    """The end-of-iteration check (Alg. 3 l.12-13) of every iteration but the last is evaluated at
+    the entry of the next panel launch (deferred, no last-CTA chain on the left update's tail); the
+    last iteration's in the left update itself (fused).  A checksum flip after the right update
+    fails it either way: the iteration is rolled back (ROLLBACK at that panel, reason 8) before
+    anything of the next panel is stored, and the result meets the oracle."""
+    A = synth.matrix(n)
+    npan = (n - 2 + nb - 1) // nb
+    i, j = (n // 3, -1) if site == ft.SITE_R else ((-1, n - 5) if site == ft.SITE_C else (-1, -1))
+    for t in (1, npan - 1):  # deferred, fused
+        dA, tau, res = gpu_reduce(A, nb=nb, faults=[(t, ft.PHASE_AFTER_RIGHT, site, i, j, 53)])
+        assert res.info == 0, res.events
+        rb = [e for e in res.events if e[0] == "ROLLBACK"]
+        assert rb and rb[0][1] == t and rb[0][2] == 8, res.events
+        check_against_oracle(A, dA, tau, nb=nb)
+
+
 @pytest.mark.parametrize("n,nb", [(256, 64), (320, 32), (513, 64), (1024, 32)])
 def test_left_update_fold_matches_tiles(n, nb):
     """The ABFT left update's checksum row/column folded into the last tile row / strip
