@@ -939,11 +939,11 @@ __global__ void __launch_bounds__(128) k_ytop_partial(YtopParams p) {
     auto issue = [&](int kt, int st) {
         const int kc = K0 + kt * YT_K;
         const int nk = min(YT_K, K1 - kc);
-        for (int i = threadIdx.x; i < YT_K * YT_M; i += blockDim.x) {
-            const int m = i % YT_M, kk = i / YT_M;
-            const bool ok = m < mrows && kk < nk;
-            cp_async8(&S.As[st][kk * (YT_M + 4) + m], ok ? p.A + (m_lo + m) + (int64_t)(kc + kk) * p.ldw : p.A,
-                      ok ? 8 : 0);
+        for (int i = threadIdx.x; i < YT_K * (YT_M / 2); i += blockDim.x) {  // 16-byte row pairs
+            const int m2 = (i % (YT_M / 2)) * 2, kk = i / (YT_M / 2);
+            const int bytes = kk < nk ? (m2 + 1 < mrows ? 16 : (m2 < mrows ? 8 : 0)) : 0;
+            cp_async16(&S.As[st][kk * (YT_M + 4) + m2], bytes ? p.A + (m_lo + m2) + (int64_t)(kc + kk) * p.ldw : p.A,
+                       bytes);
         }
         for (int i = threadIdx.x; i < FT_NBMAX * YT_K; i += blockDim.x) {
             const int kk = i % YT_K, jj = i / YT_K;
@@ -961,8 +961,8 @@ __global__ void __launch_bounds__(128) k_ytop_partial(YtopParams p) {
         cp_async_commit();
         cp_async_wait<1>();
         __syncthreads();
-        if (p.verify && threadIdx.x < YT_M)
-            for (int kk = 0; kk < nk; kk++) rs += S.As[st][kk * (YT_M + 4) + threadIdx.x];
+        if (p.verify)  // row sums: row threadIdx.x % 64, alternate k of the tile per half of the CTA
+            for (int kk = threadIdx.x >> 6; kk < nk; kk += 2) rs += S.As[st][kk * (YT_M + 4) + (threadIdx.x & 63)];
         // warp tile: rows warp*16..+16, cols 0..63 (MI=2, NI=8)
         warp_mma<2, 8, true>(acc, S.As[st], YT_M + 4, S.Vs[st], YT_K + 4, warp * 16, 0, YT_K);
         __syncthreads();  // buffer st is refilled by the next iteration's issue
@@ -978,23 +978,39 @@ __global__ void __launch_bounds__(128) k_ytop_partial(YtopParams p) {
                 int m = warp * 16 + frag_row(mi), jj = frag_col(ni, v);
                 if (m < mrows && jj < ib) yp[(int64_t)(m_lo + m) * FT_NBMAX + jj] = acc[mi][ni][v];
             }
-    if (p.verify && threadIdx.x < mrows) p.rowpart[(int64_t)blockIdx.y * (p.k + 1) + m_lo + threadIdx.x] = rs;
+    if (p.verify) {  // the two halves' row sums meet in shared memory (the A tiles are free now)
+        __syncthreads();
+        double *half = &S.As[0][0];
+        if (threadIdx.x >= 64) half[threadIdx.x - 64] = rs;
+        __syncthreads();
+        if (threadIdx.x < mrows) p.rowpart[(int64_t)blockIdx.y * (p.k + 1) + m_lo + threadIdx.x] = rs + half[threadIdx.x];
+    }
 }
 
 // Y_top rows: sum the split partials, multiply by T; row-sum verify of area 1.
 // Block = 16 rows x 64 columns of Y.
 #define YF_R 16
 __global__ void __launch_bounds__(YF_R * 64) k_ytop_finalize(YtopParams p) {
-    if (p.ctl->halt) return;
     __shared__ double Ts[FT_NBMAX * FT_NBMAX];
     __shared__ double y0[YF_R][FT_NBMAX + 1];
     const int jb = threadIdx.x & 63, rl = threadIdx.x >> 6;
     const int row = blockIdx.x * YF_R + rl;
     const int ib = p.ib;
-    for (int i = threadIdx.x; i < ib * ib; i += blockDim.x) {
-        int a = i % ib, b = i / ib;
-        Ts[a + b * FT_NBMAX] = p.T[a + b * FT_NBMAX];
+    // the halt flag, this row's verify operands and T: every load in flight together
+    const bool vrow = p.verify && row <= p.k && jb == 0;
+    const int halted = __ldcg(&p.ctl->halt);
+    const double a_k = vrow ? p.A[row + (int64_t)p.k * p.ldw] : 0.0;
+    const double a_n = vrow ? p.A[row + (int64_t)p.n * p.ldw] : 0.0;
+    const double f_r = vrow ? p.Fr[row] : 0.0;
+    double tv[FT_NBMAX * FT_NBMAX / (YF_R * 64)];
+#pragma unroll
+    for (int u = 0; u < FT_NBMAX * FT_NBMAX / (YF_R * 64); u++) {
+        const int i = threadIdx.x + u * YF_R * 64, a = i % FT_NBMAX, b = i / FT_NBMAX;
+        tv[u] = (a < ib && b < ib) ? p.T[i] : 0.0;
     }
+    if (halted) return;
+#pragma unroll
+    for (int u = 0; u < FT_NBMAX * FT_NBMAX / (YF_R * 64); u++) Ts[threadIdx.x + u * YF_R * 64] = tv[u];
     double acc = 0.0;
     if (row <= p.k && jb < ib) {
         // the split partials, 16 loads in flight at a time (fixed summation order)
@@ -1024,12 +1040,12 @@ __global__ void __launch_bounds__(YF_R * 64) k_ytop_finalize(YtopParams p) {
         yv = (yv + y1) + (y2 + y3);
         p.Y[row + (int64_t)jb * p.ldw] = yv;
     }
-    if (p.verify && row <= p.k && jb == 0) {
+    if (vrow) {
         double rsum = 0.0;
         rsum = sum_strided(p.rowpart + row, p.k + 1, p.nsplit);
-        rsum += p.A[row + (int64_t)p.k * p.ldw];
+        rsum += a_k;
         if (p.ihi < p.n) rsum += sum_strided(p.A + row + (int64_t)p.ihi * p.ldw, p.ldw, p.n - p.ihi);
-        double d = p.A[row + (int64_t)p.n * p.ldw] - p.Fr[row] - rsum;
+        double d = a_n - f_r - rsum;
         double tau_abs = p.ctl->c_thr * (double)p.n * 2.220446049250313e-16 * p.ctl->normF;
         if (not_within(d, tau_abs)) atomicAdd(&p.ctl->nflag, 1);
     }
