@@ -118,6 +118,24 @@ FT_DEV void bulk_g2s(void *dst, const void *src, unsigned bytes, unsigned long l
                  "l"(src), "r"(bytes), "r"(smem_u32(bar))
                  : "memory");
 }
+// consumer release of a pipeline buffer (the arrive orders this thread's earlier shared-memory
+// reads before the producer's next async-proxy write into the buffer, as in a TMA pipeline)
+FT_DEV void mbar_arrive(unsigned long long *bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];\n" ::"r"(smem_u32(bar)) : "memory");
+}
+// 2-D tensor TMA (SASS UTMALDG): the box at element coordinates (c0 = row, c1 = column) of the
+// tensor map `map` (a __grid_constant__ kernel parameter) into shared memory at dst (128-byte
+// aligned), completing on bar's transaction count; out-of-bounds elements are zero-filled
+FT_DEV void tma_load_2d(void *dst, const void *map, int c0, int c1, unsigned long long *bar) {
+    asm volatile(
+        "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], "
+        "[%4];\n" ::"r"(smem_u32(dst)),
+        "l"(map), "r"(c0), "r"(c1), "r"(smem_u32(bar))
+        : "memory");
+}
+FT_DEV void tma_prefetch_map(const void *map) {
+    asm volatile("prefetch.tensormap [%0];\n" ::"l"(map) : "memory");
+}
 FT_DEV void mbar_wait(unsigned long long *bar, unsigned parity) {
     asm volatile(
         "{\n"

@@ -8,6 +8,10 @@
 // Rollback (reverse computation, Alg. 3 l.14) is the same kernels with sign +1.
 //
 #include <cstdlib>
+#include <cstring>
+
+#include <cuda.h>
+#include <cudaTypedefs.h>
 
 #include "ft_common.cuh"
 #include "ft_internal.h"
@@ -44,20 +48,53 @@ static int best_splits(int nstrip, int nrt, int nsm, int cap, int per_sm, int ov
     }
     return best;
 }
-int ft_gemm_splits(int r_lo, int r_hi, int c_lo, int c_hi, int nsm) {
-    const int nstrip = (c_hi - c_lo + UB - 1) / UB;
+int ft_gemm_splits(int r_lo, int r_hi, int c_lo, int c_hi, int nsm, int extra_strips) {
+    // extra_strips: strips of the same launch outside [c_lo, c_hi) (the M-part strip); they take
+    // grid slots like the others (counted as full strips: the model stays an upper bound)
+    const int nstrip = (c_hi - c_lo + UB - 1) / UB + extra_strips;
     const int nrt = (r_hi - (r_lo / UB) * UB + UB - 1) / UB;
     // right update: one CTA per SM (the next C tile is prefetched in registers)
     static const int ovh = getenv("FT_RIGHT_OVH") ? atoi(getenv("FT_RIGHT_OVH")) : 0;
     return best_splits(nstrip > 0 ? nstrip : 1, nrt > 0 ? nrt : 1, nsm, FT_WSPLIT_MAX, 1, ovh);
 }
 
+// 2-D tensor map of a column-major ldw x K operand panel (V or Y; element (row, col) at
+// base[row + col * ldw]) with a box of `rows` x K elements: one TMA copy moves rows r .. r+rows-1 of
+// all K columns into a [col][rows] shared-memory tile (rows = SK: the padded, conflict-free stride);
+// rows past ldw are zero-filled.  The driver entry point is resolved once through the runtime.
+int ft_panel_tmap(CUtensorMap *m, const double *base, int64_t ldw, int K, int rows) {
+    static PFN_cuTensorMapEncodeTiled_v12000 enc = nullptr;
+    if (!enc) {
+        void *fn = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) != cudaSuccess ||
+            q != cudaDriverEntryPointSuccess || !fn)
+            return 1;
+        enc = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
+    }
+    if (!base || K <= 0 || K > FT_NBMAX || (ldw * 8) % 16 != 0 || (((uintptr_t)base) & 15)) return 1;
+    const cuuint64_t dims[2] = {(cuuint64_t)ldw, (cuuint64_t)K};
+    const cuuint64_t strides[1] = {(cuuint64_t)ldw * sizeof(double)};
+    const cuuint32_t box[2] = {(cuuint32_t)rows, (cuuint32_t)K};
+    const cuuint32_t estr[2] = {1, 1};
+    const CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 2, const_cast<double *>(base), dims, strides, box, estr,
+                           CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                           CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    return r == CUDA_SUCCESS ? 0 : 1;
+}
+
+// dynamic shared memory rounded up to a 128-byte boundary (TMA destinations); the offset is added
+// to the shared array itself, so the compiler keeps the shared address space (LDS, not generic LD)
+__device__ __forceinline__ unsigned char *align128(unsigned char *p) {
+    return p + ((128u - (smem_u32(p) & 127u)) & 127u);
+}
+
 template <int KT>
 struct RightSmemT {
-    double Vc[KT][SK];  // V(cols, k) as [k][col]   (A operand of the right update)
-    double Ys[KT][SK];  // Y(rows, k) as [k][row]   (B operand of the right update)
-    double Vr[KT][SK];  // V(rows, j) as [j][row]   (B operand of W^T = C_new^T V)
-    double Yn[KT];      // fold_row: Y(n, :) = Y_chk
+    double Vc[KT][SK];     // sign * V(cols, k) as [k][col]   (A operand of the right update)
+    double Ys[2][KT][SK];  // Y(rows, k) as [k][row], double-buffered TMA tiles (B operand of the right update)
+    double Vr[2][KT][SK];  // V(rows, j) as [j][row], double-buffered TMA tiles (B operand of W^T = C_new^T V)
+    double Yn[KT];         // fold_row: Y(n, :) = Y_chk
 };
 
 // k-major operand tile: M(r .. r+63, 0:KT) (column-major, leading dim ld) -> T[k][row];
@@ -118,7 +155,8 @@ __device__ int pre_update_reason(const GemmRightParams &p) {
 }
 
 template <int KT>
-__global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
+__global__ void __launch_bounds__(UT, 1)
+    k_gemm_right(const GemmRightParams p, const __grid_constant__ CUtensorMap tmY, const __grid_constant__ CUtensorMap tmV) {
     // the halt flag is loaded here but first used at the first tile's barrier (before any store),
     // so its round trip overlaps the operand loads instead of delaying them
     const int halted = p.ctl ? __ldcg(&p.ctl->halt) : 0;
@@ -133,8 +171,8 @@ __global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
         const int reason = pre_update_reason(p);
         if (threadIdx.x == 0) s_reason = reason;
     }
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    RightSmemT<KT> &S = *reinterpret_cast<RightSmemT<KT> *>(smem_raw);
+    extern __shared__ unsigned char smem_raw[];
+    RightSmemT<KT> &S = *reinterpret_cast<RightSmemT<KT> *>(align128(smem_raw));
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int lr = lane >> 2, lc = lane & 3;
     // the last strip of the grid is the M-part when present (rows 0..m_r_hi, no W)
@@ -168,12 +206,63 @@ __global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
         colp2[mi] = p.A + (int64_t)(cb + (colok2[mi] ? cols2[mi] : 0)) * p.lda;
     }
 
-    if (p.do_right) {  // V(cols, :) once per CTA (plain loads: cb may be odd)
-        for (int i = tid; i < KT * UB; i += UT) {
-            const int kk = i / UB, cc = i % UB;
+    // Operand pipeline: the Y / V row tiles (rows r .. r+SK-1, columns 0..K-1) arrive by 2-D tensor
+    // TMA, one instruction per tile issued by thread 0, into double buffers; full[b] completes on the
+    // copy's transaction count, empty[b] when all eight warps have read the buffer (mbarrier arrive:
+    // no CTA-wide barrier inside the tile loop, so warps drift and the DMMA pipe stays fed while one
+    // warp stores or shuffles).  Ys columns k >= K meet zero Vc entries: they start as zeros (stale
+    // shared memory could hold NaN patterns); rows past the matrix are zero-filled by the TMA unit.
+    __shared__ __align__(8) unsigned long long yfull[2], vfull[2], yempty[2], vempty[2];
+    if (tid == 0) {
+        for (int b = 0; b < 2; b++) {
+            mbar_init(&yfull[b], 1);
+            mbar_init(&vfull[b], 1);
+            mbar_init(&yempty[b], UT / 32);
+            mbar_init(&vempty[b], UT / 32);
+        }
+        mbar_fence_init();
+        if (p.do_right) tma_prefetch_map(&tmY);
+        if (do_w) tma_prefetch_map(&tmV);
+    }
+    const unsigned tile_bytes = (unsigned)(SK * K * 8);
+    auto issue = [&](int tt, int b) {  // thread 0: tile tt's operands into buffers b
+        const int r = rbase + tt * UB;
+        if (p.do_right) {
+            mbar_expect_tx(&yfull[b], tile_bytes);
+            tma_load_2d(&S.Ys[b][0][0], &tmY, r, 0, &yfull[b]);
+        }
+        if (do_w) {
+            mbar_expect_tx(&vfull[b], tile_bytes);
+            tma_load_2d(&S.Vr[b][0][0], &tmV, r, 0, &vfull[b]);
+        }
+    };
+    if (K < KT && p.do_right)
+        for (int i = tid; i < 2 * (KT - K) * SK; i += UT) {
+            const int b = i / ((KT - K) * SK), rem = i % ((KT - K) * SK);
+            S.Ys[b][K + rem / SK][rem % SK] = 0.0;
+        }
+    if (foldr && tid < KT) S.Yn[tid] = tid < K ? __ldcg(p.Y + p.r_hi + (int64_t)tid * p.ldw) : 0.0;
+    __syncthreads();  // barrier init visible before the first copies
+    if (tid == 0 && t0 < t1) {
+        issue(t0, 0);
+        if (t0 + 1 < t1) issue(t0 + 1, 1);
+    }
+    // sign * V(cols, :) once per CTA (sign folded into the A operand: the accumulators start from C
+    // itself and hold C_new at the end -- the same roundings as sign * (sign C + V Y^T))
+    if (p.do_right) {
+        constexpr int NV = KT * UB / UT;
+        double vv[NV];
+#pragma unroll
+        for (int m = 0; m < NV; m++) {
+            const int i = tid + m * UT, kk = i / UB, cc = i % UB;
             const bool ok = kk < K && cc < ncols;
             const int vrow = ft_cmap(cb + cc, p.cm_G, p.cm_rank, p.cm_nb, p.cm_ncl, p.cm_n);
-            cp_async8(&S.Vc[kk][cc], ok ? p.V + vrow + (int64_t)kk * p.ldw : p.V, ok ? 8 : 0);
+            vv[m] = ok ? __ldg(p.V + vrow + (int64_t)kk * p.ldw) : 0.0;
+        }
+#pragma unroll
+        for (int m = 0; m < NV; m++) {
+            const int i = tid + m * UT;
+            S.Vc[i / UB][i % UB] = sg * vv[m];
         }
     }
     double wacc[2][NJ][2];
@@ -181,39 +270,7 @@ __global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
     for (int mi = 0; mi < 2; mi++)
 #pragma unroll
         for (int a = 0; a < NJ; a++) wacc[mi][a][0] = wacc[mi][a][1] = 0.0;
-    cp_async_commit();  // the Vc strip
-
-    // Y / V row tiles: bulk copies (TMA, one column segment per lane) into the padded tiles,
-    // completing on one mbarrier per tile buffer (parity = use count & 1).  Ys columns k >= K meet
-    // zero Vc entries and every Vr row meets the W pass (masked rows are zero there), so those words
-    // start as zeros (stale shared memory could hold NaN patterns); later tiles leave finite V rows
-    __shared__ __align__(8) unsigned long long ybar, vbar;
-    if (tid == 0) {
-        mbar_init(&ybar, 1);
-        mbar_init(&vbar, 1);
-        mbar_fence_init();
-    }
-    if (K < KT && p.do_right)
-        for (int i = tid; i < (KT - K) * SK; i += UT) S.Ys[K + i / SK][i % SK] = 0.0;
-    if (do_w)
-        for (int i = tid; i < KT * SK; i += UT) S.Vr[i / SK][i % SK] = 0.0;
-    if (foldr && tid < KT) S.Yn[tid] = tid < K ? __ldcg(p.Y + p.r_hi + (int64_t)tid * p.ldw) : 0.0;
-    __syncthreads();
-    // issued by all eight warps (lanes 0..7 of warp w: columns 8w..8w+7), so no warp stalls its
-    // barrier partners on a long serial issue; tid 0's arrive carries the expected byte count
-    auto issue_tile = [&](double (*T)[SK], const double *M, int r, unsigned long long *bar) {
-        const unsigned bytes = (unsigned)min(UB, (int)(p.ldw - r)) * 8u;
-        const int kk = warp * 8 + lane;
-        if (lane < 8 && kk < K) {
-            fence_proxy_async();  // the buffer's earlier reads (ordered by the last bar.sync) precede the copies
-            bulk_g2s(&T[kk][0], M + (int64_t)kk * p.ldw + r, bytes, bar);
-        }
-        if (tid == 0) mbar_expect_tx(bar, bytes * (unsigned)K);
-    };
-    if (t0 < t1) {
-        if (p.do_right) issue_tile(S.Ys, p.Y, rbase + t0 * UB, &ybar);
-        if (do_w) issue_tile(S.Vr, p.V, rbase + t0 * UB, &vbar);
-    }
+    const int ntile_issued = t0 < t1 ? min(2, t1 - t0) : 0;
     auto pre_abort = [&]() -> bool {  // after a __syncthreads that follows the evaluation
         const bool raise = !halted && p.pre_ctl && s_reason;
         if (!halted && !raise) return false;
@@ -225,9 +282,10 @@ __global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
             __threadfence();
             ctl->halt = 1;
         }
-        if (t0 < t1) {  // the first tiles' bulk copies land before the CTA's shared memory is released
-            if (p.do_right) mbar_wait(&ybar, 0u);
-            if (do_w) mbar_wait(&vbar, 0u);
+        // the copies in flight land before the CTA's shared memory is released
+        for (int b = 0; b < ntile_issued; b++) {
+            if (p.do_right) mbar_wait(&yfull[b], 0u);
+            if (do_w) mbar_wait(&vfull[b], 0u);
         }
         return true;  // nothing consumed: the panel is redone from its checkpoint
     };
@@ -248,6 +306,8 @@ __global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
     double2 cn[2][4];  // the next tile's C, prefetched a whole tile ahead
     if (t0 < t1) load_c(t0, cn);
     for (int tt = t0; tt < t1; tt++) {
+        const int it = tt - t0, b = it & 1;
+        const unsigned ph = (unsigned)(it >> 1) & 1u;
         const int r = rbase + tt * UB;
         const int lo = max(r, r_lo), hi = min(r + UB, r_hi);
         const bool full = lo == r && hi == r + UB && ncols == UB;  // interior tile: no masks
@@ -256,84 +316,88 @@ __global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
         for (int mi = 0; mi < 2; mi++)
 #pragma unroll
             for (int ni = 0; ni < 4; ni++) {
-                acc[mi][ni][0] = sg * cn[mi][ni].x;
-                acc[mi][ni][1] = sg * cn[mi][ni].y;
+                acc[mi][ni][0] = cn[mi][ni].x;
+                acc[mi][ni][1] = cn[mi][ni].y;
             }
         if (tt + 1 < t1) load_c(tt + 1, cn);
         if (tt == t0) {
-            cp_async_wait<0>();  // the Vc strip
-            __syncthreads();
+            __syncthreads();  // Vc and the pre-update decision
             if (pre_abort()) return;
+        } else if (tid == 0 && tt + 1 < t1) {
+            // refill the buffers of tile tt-1 with tile tt+1 once every warp has released them
+            const unsigned pho = (unsigned)((it - 1) >> 1) & 1u;
+            if (p.do_right) mbar_wait(&yempty[b ^ 1], pho);
+            if (do_w) mbar_wait(&vempty[b ^ 1], pho);
+            issue(tt + 1, b ^ 1);
         }
         if (p.do_right) {
-            mbar_wait(&ybar, (unsigned)(tt - t0) & 1u);
+            mbar_wait(&yfull[b], ph);
 #pragma unroll 4
             for (int k0 = 0; k0 < KT; k0 += 4) {
-                double a[2], b[4];
+                double a[2], bb[4];
 #pragma unroll
                 for (int mi = 0; mi < 2; mi++) a[mi] = S.Vc[k0 + lc][wc * 16 + mi * 8 + lr];
 #pragma unroll
-                for (int ni = 0; ni < 4; ni++) b[ni] = S.Ys[k0 + lc][wr * 32 + ni * 8 + lr];
+                for (int ni = 0; ni < 4; ni++) bb[ni] = S.Ys[b][k0 + lc][wr * 32 + ni * 8 + lr];
 #pragma unroll
                 for (int mi = 0; mi < 2; mi++)
 #pragma unroll
-                    for (int ni = 0; ni < 4; ni++) dmma_8x8x4(acc[mi][ni][0], acc[mi][ni][1], a[mi], b[ni]);
+                    for (int ni = 0; ni < 4; ni++) dmma_8x8x4(acc[mi][ni][0], acc[mi][ni][1], a[mi], bb[ni]);
             }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&yempty[b]);
 #pragma unroll
             for (int mi = 0; mi < 2; mi++)
 #pragma unroll
                 for (int ni = 0; ni < 4; ni++) {
-                    acc[mi][ni][0] *= sg;
-                    acc[mi][ni][1] *= sg;
                     const int row = r + wr * 32 + ni * 8 + 2 * lc;
                     if (full) *reinterpret_cast<double2 *>(colp2[mi] + row) = make_double2(acc[mi][ni][0], acc[mi][ni][1]);
                     else store_pair(colp2[mi], row, lo, hi, colok2[mi], acc[mi][ni][0], acc[mi][ni][1]);
                 }
         }
-        __syncthreads();  // every warp is done with Ys(tt)
-        if (p.do_right && tt + 1 < t1) issue_tile(S.Ys, p.Y, r + UB, &ybar);
         if (do_w) {
-            mbar_wait(&vbar, (unsigned)(tt - t0) & 1u);
-            // only rows in [wr_lo, wr_hi) take part in W
+            mbar_wait(&vfull[b], ph);
+            // only rows in [wr_lo, wr_hi) take part in W (a uniform test: interior tiles skip the masks)
             const int wlo = max(lo, p.wr_lo), whi = min(hi, p.wr_hi);
+            if (!(wlo == r && whi == r + UB)) {
 #pragma unroll
-            for (int mi = 0; mi < 2; mi++)
+                for (int mi = 0; mi < 2; mi++)
 #pragma unroll
-                for (int ni = 0; ni < 4; ni++) {
-                    const int row = r + wr * 32 + ni * 8 + 2 * lc;
-                    if (row < wlo || row >= whi) acc[mi][ni][0] = 0.0;
-                    if (row + 1 < wlo || row + 1 >= whi) acc[mi][ni][1] = 0.0;
-                }
-            // W^T(cols, j) += C_new^T(cols, rows) V(rows, j) over this warp's 32 rows; the A fragment
-            // (col lr, row ks*4 + lc) sits in lane lr*4 + 2h + lc/2, element lc & 1 (ks = 2 ni + h)
+                    for (int ni = 0; ni < 4; ni++) {
+                        const int row = r + wr * 32 + ni * 8 + 2 * lc;
+                        if (row < wlo || row >= whi) acc[mi][ni][0] = 0.0;
+                        if (row + 1 < wlo || row + 1 >= whi) acc[mi][ni][1] = 0.0;
+                    }
+            }
+            // W^T(cols, j) += C_new^T(cols, rows) V(rows, j) over this warp's 32 rows.  The rows are
+            // taken in a permuted order so that every A fragment is an accumulator the lane already
+            // holds (no shuffles): k-step (ni, e) gives lane (lr, lc) the row 8 ni + 2 lc + (e ^ lc/2),
+            // i.e. acc[mi][ni][e ^ lc/2]; the matching B rows V(row, j) then hit every shared-memory
+            // bank exactly twice per warp (stride SK = 4 mod 16), like the other fragment loads
+            const int sw = lc >> 1;
 #pragma unroll
             for (int ks = 0; ks < 8; ks++) {
-                const int ni = ks >> 1, h = ks & 1;
-                const int src = lr * 4 + 2 * h + (lc >> 1);
+                const int ni = ks >> 1, e = ks & 1;
                 double a[2];
 #pragma unroll
-                for (int mi = 0; mi < 2; mi++) {
-                    const double x0 = __shfl_sync(0xffffffffu, acc[mi][ni][0], src);
-                    const double x1 = __shfl_sync(0xffffffffu, acc[mi][ni][1], src);
-                    a[mi] = (lc & 1) ? x1 : x0;
-                }
+                for (int mi = 0; mi < 2; mi++) a[mi] = sw ? acc[mi][ni][e ^ 1] : acc[mi][ni][e];
+                const int row = wr * 32 + ni * 8 + 2 * lc + (e ^ sw);
 #pragma unroll
                 for (int nj = 0; nj < NJ; nj++) {
-                    const double b = S.Vr[nj * 8 + lr][wr * 32 + ks * 4 + lc];
+                    const double bv = S.Vr[b][nj * 8 + lr][row];
 #pragma unroll
-                    for (int mi = 0; mi < 2; mi++) dmma_8x8x4(wacc[mi][nj][0], wacc[mi][nj][1], a[mi], b);
+                    for (int mi = 0; mi < 2; mi++) dmma_8x8x4(wacc[mi][nj][0], wacc[mi][nj][1], a[mi], bv);
                 }
             }
-            __syncthreads();  // every warp is done with Vr(tt)
-            if (tt + 1 < t1) issue_tile(S.Vr, p.V, r + UB, &vbar);
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&vempty[b]);
         }
     }
-    cp_async_wait<0>();
     if (t0 >= t1) {  // no tile: take the pre-update decision here (no strip counter on a halt)
         __syncthreads();
         if (pre_abort()) return;
     }
-    if (foldr) {  // c(cols) += sg Y(n, :) V(cols, :)^T (Vc and Yn in shared memory)
+    if (foldr) {  // c(cols) += Y(n, :) (sign V(cols, :))^T (Vc and Yn in shared memory)
         double s0 = 0.0, s1 = 0.0;
 #pragma unroll
         for (int kk = fq; kk < KT; kk += 8) {
@@ -343,13 +407,13 @@ __global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
         s0 += s1;
         s0 += __shfl_xor_sync(0xffffffffu, s0, 1);
         s0 += __shfl_xor_sync(0xffffffffu, s0, 2);
-        if (fq == 0 && fcol < ncols) p.A[p.r_hi + (int64_t)(cb + fcol) * p.lda] = cold + sg * s0;
+        if (fq == 0 && fcol < ncols) p.A[p.r_hi + (int64_t)(cb + fcol) * p.lda] = cold + s0;
     }
     if (do_w) {
         // deterministic partial of this row split: Wpart[split][col][j]; the two row warps of each
         // column group meet in shared memory first (wr = 1 stores, wr = 0 adds and writes out)
         double *Wp = p.Wpart + (int64_t)blockIdx.y * p.wsplit_stride;
-        double *red = &S.Ys[0][0];  // [col][64] scratch: every copy into Ys has completed
+        double *red = &S.Ys[0][0][0];  // [col][64] scratch: every copy into Ys has completed
         __syncthreads();
         if (wr == 1)
 #pragma unroll
@@ -380,7 +444,7 @@ __global__ void __launch_bounds__(UT, 1) k_gemm_right(GemmRightParams p) {
             __syncthreads();
             if (last) {
                 double(*Ts)[SK] = S.Vc;  // reuse: T as Ts[a][b] (KT x KT)
-                double(*Ws)[SK] = S.Ys;  // W as Ws[col][b] (64 x KT): spans Ys and Vr (contiguous)
+                double(*Ws)[SK] = reinterpret_cast<double(*)[SK]>(&S.Ys[0][0][0]);  // W as Ws[col][b] (64 x KT): spans both Ys buffers
                 for (int i = tid; i < KT * KT; i += UT) {
                     const int a = i % KT, b = i / KT;
                     const bool ok = a < K && b < K;
@@ -456,7 +520,7 @@ template <int KT>
 static cudaError_t launch_right_kt(const GemmRightParams &p, cudaStream_t s) {
     static unsigned attr = 0;
     const unsigned dbit = ft_dev_bit();
-    const size_t smem = sizeof(RightSmemT<KT>);
+    const size_t smem = sizeof(RightSmemT<KT>) + 128;  // + alignment slack (TMA destinations)
     if (!(attr & dbit)) {
         cudaError_t e = cudaFuncSetAttribute(k_gemm_right<KT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return e;
@@ -467,8 +531,13 @@ static cudaError_t launch_right_kt(const GemmRightParams &p, cudaStream_t s) {
     if (q.fold_row) q.r_hi = p.r_hi - 1;  // row r_hi-1 (c) is folded into the last row split
     const int nstrip = (q.c_hi - q.c_lo + UB - 1) / UB + (q.has_m ? 1 : 0);
     const int ny = q.nsplit > 0 ? q.nsplit : 1;
+    CUtensorMap tmY, tmV;
+    memset(&tmY, 0, sizeof(tmY));
+    memset(&tmV, 0, sizeof(tmV));
+    if (q.do_right && ft_panel_tmap(&tmY, q.Y, q.ldw, q.K, SK)) return cudaErrorInvalidValue;
+    if (q.do_w && ft_panel_tmap(&tmV, q.V, q.ldw, q.K, SK)) return cudaErrorInvalidValue;
     g_ft_launches++;
-    k_gemm_right<KT><<<dim3(nstrip, ny), UT, smem, s>>>(q);
+    k_gemm_right<KT><<<dim3(nstrip, ny), UT, smem, s>>>(q, tmY, tmV);
     return cudaGetLastError();
 }
 cudaError_t ft_launch_gemm_right(const GemmRightParams &p, cudaStream_t s) {
@@ -503,8 +572,8 @@ cudaError_t ft_launch_gemm_right(const GemmRightParams &p, cudaStream_t s) {
 // ---------------------------------------------------------------------------
 template <int KT>
 struct LeftSmemT {
-    double Wc[KT][SK];     // W' = op(T) W as [k][col]  (A operand, W'^T)
-    double Vr[2][KT][SK];  // V(rows, k) as [k][row]    (B operand), double-buffered
+    double Wc[UB][SK];     // sign * W' (W' = op(T) W) as [col][k]  (A operand, W'^T; stride SK: conflict free)
+    double Vr[2][KT][SK];  // V(rows, k) as [k][row]    (B operand), double-buffered TMA tiles
     double Wr[KT];         // fold: W'(:, n), the r column's coefficients
     double Vn[KT];         // fold: V(n, :) = V_chk
 };
@@ -548,7 +617,7 @@ __global__ void k_wprep(const double *__restrict__ Wpart, int64_t wstride, int n
 }
 
 template <int KT>
-__global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
+__global__ void __launch_bounds__(UT, 2) k_gemm_left(const GemmLeftParams p, const __grid_constant__ CUtensorMap tmV) {
     // both flags in flight together (one round trip before the launch's first load)
     const int halted = p.ctl ? __ldcg(&p.ctl->halt) : 0;
     const int tbad = p.tctl ? __ldcg(&p.tctl->tbad) : 0;
@@ -587,8 +656,8 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
         p.Fr[i] += ((s[0] + s[1]) + (s[2] + s[3])) + ((s[4] + s[5]) + (s[6] + s[7]));
         return;
     }
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    LeftSmemT<KT> &S = *reinterpret_cast<LeftSmemT<KT> *>(smem_raw);
+    extern __shared__ unsigned char smem_raw[];
+    LeftSmemT<KT> &S = *reinterpret_cast<LeftSmemT<KT> *>(align128(smem_raw));
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int lr = lane >> 2, lc = lane & 3;
     const int wc = warp & 3, wr = warp >> 2;
@@ -611,44 +680,56 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
         if (tid == 0) p.pre_reset->nflag = 0;
     }
 
-    // W'^T for the strip: Wt [col][64] -> Wc[k][col] (cp.async, joined before the first tile)
-    for (int i = tid; i < KT * UB; i += UT) {
-        const int cc = i / KT, kk = i % KT;
-        const bool ok = kk < K && cc < ncols;
-        cp_async8(&S.Wc[kk][cc], ok ? p.Wpart + (int64_t)(cb + cc) * FT_NBMAX + kk : p.Wpart, ok ? 8 : 0);
-    }
-    cp_async_commit();
-    // V tiles: bulk copies (TMA, one 512-byte column segment per lane of warp 0) into the padded
-    // double buffer, completing on an mbarrier per buffer (parity = use count & 1).  Rows past the
-    // tile's copy extent only feed masked outputs; columns k >= K meet zero W' entries, so they are
-    // zeroed once (stale shared memory could hold NaN patterns)
-    __shared__ __align__(8) unsigned long long vbar[2];
+    // V tiles (rows r .. r+SK-1, columns 0..K-1) by 2-D tensor TMA, one instruction per tile issued
+    // by thread 0, into a double buffer: full[b] completes on the copy's transaction count, empty[b]
+    // when all eight warps have read the buffer (no CTA-wide barrier inside the tile loop).  Columns
+    // k >= K meet zero W' entries, so they are zeroed once (stale shared memory could hold NaN
+    // patterns); rows past the matrix are zero-filled by the TMA unit.
+    __shared__ __align__(8) unsigned long long vfull[2], vempty[2];
     if (tid == 0) {
-        mbar_init(&vbar[0], 1);
-        mbar_init(&vbar[1], 1);
+        for (int b = 0; b < 2; b++) {
+            mbar_init(&vfull[b], 1);
+            mbar_init(&vempty[b], UT / 32);
+        }
         mbar_fence_init();
+        tma_prefetch_map(&tmV);
     }
     if (K < KT)
         for (int i = tid; i < 2 * (KT - K) * SK; i += UT) {
             const int b = i / ((KT - K) * SK), rem = i % ((KT - K) * SK);
             S.Vr[b][K + rem / SK][rem % SK] = 0.0;
         }
-    __syncthreads();
-    auto issue_v = [&](int tt, int b) {  // all eight warps issue (lanes 0..7: columns 8w..8w+7)
-        const int r = rbase + tt * UB;
-        const unsigned bytes = (unsigned)min(UB, (int)(p.ldw - r)) * 8u;
-        const int kk = warp * 8 + lane;
-        if (lane < 8 && kk < K) {
-            fence_proxy_async();  // this buffer's earlier reads (ordered by the last bar.sync) precede the copies
-            bulk_g2s(&S.Vr[b][kk][0], p.V + (int64_t)kk * p.ldw + r, bytes, &vbar[b]);
-        }
-        if (tid == 0) mbar_expect_tx(&vbar[b], bytes * (unsigned)K);
-    };
-    if (t0 < t1) issue_v(t0, 0);
     // fold (ABFT): column n (r) rides with the last strip, row n (c) with the last row tile
     if (p.fold && tid < KT) {
         S.Wr[tid] = tid < K ? p.Wpart[(int64_t)p.n * FT_NBMAX + tid] : 0.0;
         S.Vn[tid] = tid < K ? p.V[p.n + (int64_t)tid * p.ldw] : 0.0;
+    }
+    __syncthreads();  // barrier init visible before the first copies
+    const unsigned tile_bytes = (unsigned)(SK * K * 8);
+    auto issue_v = [&](int tt, int b) {  // thread 0
+        mbar_expect_tx(&vfull[b], tile_bytes);
+        tma_load_2d(&S.Vr[b][0][0], &tmV, rbase + tt * UB, 0, &vfull[b]);
+    };
+    if (tid == 0 && t0 < t1) {
+        issue_v(t0, 0);
+        if (t0 + 1 < t1) issue_v(t0 + 1, 1);
+    }
+    // sign * W'^T for the strip: Wt [col][64] -> Wc[k][col] (sign folded into the A operand: the
+    // accumulators start from C itself -- the same roundings as sign * (sign C + W'^T V^T))
+    {
+        constexpr int NW = KT * UB / UT;
+        double wv[NW];
+#pragma unroll
+        for (int m = 0; m < NW; m++) {
+            const int i = tid + m * UT, cc = i / KT, kk = i % KT;
+            const bool ok = kk < K && cc < ncols;
+            wv[m] = ok ? __ldcg(p.Wpart + (int64_t)(cb + cc) * FT_NBMAX + kk) : 0.0;
+        }
+#pragma unroll
+        for (int m = 0; m < NW; m++) {
+            const int i = tid + m * UT;
+            S.Wc[i / KT][i % KT] = sg * wv[m];
+        }
     }
     int cols[2];
     bool colok[2];
@@ -696,10 +777,9 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
     };
     double2 cn[2][4];
     if (t0 < t1) load_c(t0, cn);
-    cp_async_wait<0>();
-    __syncthreads();  // every thread's part of W' landed
+    __syncthreads();  // every thread's part of sign * W' landed
     for (int tt = t0; tt < t1; tt++) {
-        const int st = (tt - t0) & 1;
+        const int it = tt - t0, st = it & 1;
         const int r = rbase + tt * UB;
         const int lo = max(r, p.r_lo), hi = min(r + UB, p.r_hi);
         const bool full = lo == r && hi == r + UB && ncols == UB;  // interior tile: no masks
@@ -708,19 +788,22 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
         for (int mi = 0; mi < 2; mi++)
 #pragma unroll
             for (int ni = 0; ni < 4; ni++) {
-                acc[mi][ni][0] = sg * cn[mi][ni].x;
-                acc[mi][ni][1] = sg * cn[mi][ni].y;
+                acc[mi][ni][0] = cn[mi][ni].x;
+                acc[mi][ni][1] = cn[mi][ni].y;
             }
         if (tt + 1 < t1) {
-            issue_v(tt + 1, st ^ 1);  // released by the bar.sync that ended tile tt-1
             load_c(tt + 1, cn);
+            if (tid == 0 && it >= 1) {  // refill tile tt-1's buffer with tile tt+1 once every warp released it
+                mbar_wait(&vempty[st ^ 1], (unsigned)((it - 1) >> 1) & 1u);
+                issue_v(tt + 1, st ^ 1);
+            }
         }
-        mbar_wait(&vbar[st], (unsigned)((tt - t0) >> 1) & 1u);
+        mbar_wait(&vfull[st], (unsigned)(it >> 1) & 1u);
 #pragma unroll 4
         for (int k0 = 0; k0 < KT; k0 += 4) {
             double a[2], b[4];
 #pragma unroll
-            for (int mi = 0; mi < 2; mi++) a[mi] = S.Wc[k0 + lc][wc * 16 + mi * 8 + lr];
+            for (int mi = 0; mi < 2; mi++) a[mi] = S.Wc[wc * 16 + mi * 8 + lr][k0 + lc];
 #pragma unroll
             for (int ni = 0; ni < 4; ni++) b[ni] = S.Vr[st][k0 + lc][wr * 32 + ni * 8 + lr];
 #pragma unroll
@@ -728,26 +811,6 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
 #pragma unroll
                 for (int ni = 0; ni < 4; ni++) dmma_8x8x4(acc[mi][ni][0], acc[mi][ni][1], a[mi], b[ni]);
         }
-#pragma unroll
-        for (int mi = 0; mi < 2; mi++)
-#pragma unroll
-            for (int ni = 0; ni < 4; ni++) {
-                const int row = r + wr * 32 + ni * 8 + 2 * lc;
-                const double x = sg * acc[mi][ni][0], y = sg * acc[mi][ni][1];
-                if (full) *reinterpret_cast<double2 *>(colp[mi] + row) = make_double2(x, y);
-                else store_pair(colp[mi], row, lo, hi, colok[mi], x, y);
-                if (p.endcheck && !p.fold && colok[mi]) {  // fold: r, c are written by the fold code below
-                    const int gc = cb + cols[mi];
-                    const bool in0 = row >= lo && row < hi, in1 = row + 1 >= lo && row + 1 < hi;
-                    if (gc == en) {  // r entries (kappa = row n excluded)
-                        if (in0 && row < en) es_r += x;
-                        if (in1 && row + 1 < en) es_r += y;
-                    } else if (gc < en) {  // c entries
-                        if (in0 && row == en) es_c += x;
-                        if (in1 && row + 1 == en) es_c += y;
-                    }
-                }
-            }
         if (fold_col) {  // r(rows) += sg V(rows, :) W'(:, n): 4 lanes per row, two chains each
             const int rr = tid >> 2, q4 = tid & 3;
             double s0 = 0.0, s1 = 0.0;
@@ -767,7 +830,28 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
                 es_r += v;
             }
         }
-        __syncthreads();  // Vr[st] is refilled two tiles later
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&vempty[st]);  // this warp is done with Vr[st]
+#pragma unroll
+        for (int mi = 0; mi < 2; mi++)
+#pragma unroll
+            for (int ni = 0; ni < 4; ni++) {
+                const int row = r + wr * 32 + ni * 8 + 2 * lc;
+                const double x = acc[mi][ni][0], y = acc[mi][ni][1];
+                if (full) *reinterpret_cast<double2 *>(colp[mi] + row) = make_double2(x, y);
+                else store_pair(colp[mi], row, lo, hi, colok[mi], x, y);
+                if (p.endcheck && !p.fold && colok[mi]) {  // fold: r, c are written by the fold code
+                    const int gc = cb + cols[mi];
+                    const bool in0 = row >= lo && row < hi, in1 = row + 1 >= lo && row + 1 < hi;
+                    if (gc == en) {  // r entries (kappa = row n excluded)
+                        if (in0 && row < en) es_r += x;
+                        if (in1 && row + 1 < en) es_r += y;
+                    } else if (gc < en) {  // c entries
+                        if (in0 && row == en) es_c += x;
+                        if (in1 && row + 1 == en) es_c += y;
+                    }
+                }
+            }
     }
     if (fold_row) {  // c(cols) += sg V(n, :) W'(:, cols), and kappa with the last strip
         __syncthreads();
@@ -775,8 +859,8 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
         double s0 = 0.0, s1 = 0.0, k0 = 0.0, k1 = 0.0;
 #pragma unroll
         for (int kk = q4; kk < KT; kk += 8) {
-            s0 += S.Vn[kk] * S.Wc[kk][cc];
-            s1 += S.Vn[kk + 4] * S.Wc[kk + 4][cc];
+            s0 += S.Vn[kk] * S.Wc[cc][kk];  // Wc = sign * W': the sign is in s0
+            s1 += S.Vn[kk + 4] * S.Wc[cc][kk + 4];
             k0 += S.Vn[kk] * S.Wr[kk];
             k1 += S.Vn[kk + 4] * S.Wr[kk + 4];
         }
@@ -788,7 +872,7 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(GemmLeftParams p) {
         k0 += __shfl_xor_sync(0xffffffffu, k0, 2);
         if (q4 == 0 && cc < ncols) {
             double *pc = p.A + p.n + (int64_t)(cb + cc) * p.lda;
-            const double v = *pc + sg * s0;
+            const double v = *pc + s0;
             *pc = v;
             es_c += v;
         }
@@ -850,7 +934,7 @@ template <int KT>
 static cudaError_t launch_left_kt(const GemmLeftParams &p, cudaStream_t s) {
     static unsigned attr = 0;
     const unsigned dbit = ft_dev_bit();
-    const size_t smem = sizeof(LeftSmemT<KT>);
+    const size_t smem = sizeof(LeftSmemT<KT>) + 128;  // + alignment slack (TMA destinations)
     if (!(attr & dbit)) {
         cudaError_t e = cudaFuncSetAttribute(k_gemm_left<KT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return e;
@@ -893,7 +977,10 @@ static cudaError_t launch_left_kt(const GemmLeftParams &p, cudaStream_t s) {
         nyf = ((rows + UT - 1) / UT + nstrip - 1) / nstrip;
     }
     q.nyf = nyf;
-    k_gemm_left<KT><<<dim3(nstrip, ny + nyf), UT, smem, s>>>(q);
+    CUtensorMap tmV;
+    memset(&tmV, 0, sizeof(tmV));
+    if (ft_panel_tmap(&tmV, q.V, q.ldw, q.K, SK)) return cudaErrorInvalidValue;
+    k_gemm_left<KT><<<dim3(nstrip, ny + nyf), UT, smem, s>>>(q, tmV);
     return cudaGetLastError();
 }
 cudaError_t ft_launch_gemm_left(const GemmLeftParams &p, cudaStream_t s) {

@@ -152,9 +152,12 @@ __host__ __device__ inline int ft_cmap(int l, int G, int rank, int nb, int ncl, 
     return (l / nb) * nb * G + rank * nb + l % nb;
 }
 cudaError_t ft_launch_gemm_right(const GemmRightParams &p, cudaStream_t s);
-#define FT_WSPLIT_MAX 16  // max row splits of the right update (deterministic W partials)
+struct CUtensorMap_st;
+// 2-D TMA map of a column-major ldw x K panel, box rows x K (ft_gemm.cu); 0 on success
+int ft_panel_tmap(struct CUtensorMap_st *m, const double *base, int64_t ldw, int K, int rows);
+#define FT_WSPLIT_MAX 32  // max row splits of the right update (deterministic W partials)
 // row splits the right-update launch uses for this block (the left update's k_wprep sums them)
-int ft_gemm_splits(int r_lo, int r_hi, int c_lo, int c_hi, int nsm);
+int ft_gemm_splits(int r_lo, int r_hi, int c_lo, int c_hi, int nsm, int extra_strips = 0);
 
 struct GemmLeftParams {
     double *A;
