@@ -54,7 +54,10 @@ int ft_gemm_splits(int r_lo, int r_hi, int c_lo, int c_hi, int nsm, int extra_st
     const int nstrip = (c_hi - c_lo + UB - 1) / UB + extra_strips;
     const int nrt = (r_hi - (r_lo / UB) * UB + UB - 1) / UB;
     // right update: one CTA per SM (the next C tile is prefetched in registers)
-    static const int ovh = getenv("FT_RIGHT_OVH") ? atoi(getenv("FT_RIGHT_OVH")) : 0;
+    // per-CTA prologue / epilogue (V strip, first copies, W partials) of 1.5 tiles: with the split cap
+    // at 32 a zero term picks many short CTAs (right update at C3: 356 ms at 0, 340 ms at 3-10;
+    // profiles/r02/gemm_tma/right_ovh_sweep.txt); FT_RIGHT_OVH overrides for sweeps
+    static const int ovh = getenv("FT_RIGHT_OVH") ? atoi(getenv("FT_RIGHT_OVH")) : 6;
     return best_splits(nstrip > 0 ? nstrip : 1, nrt > 0 ? nrt : 1, nsm, FT_WSPLIT_MAX, 1, ovh);
 }
 
