@@ -117,6 +117,12 @@ typedef struct {
     void *stream;             /* cudaStream_t; NULL -> the legacy default stream          */
     int32_t timing;           /* 1: record the per-phase times report->ms[1..7] (an event pair
                                  around each phase; such calls are never graph-replayed)     */
+    int32_t deterministic;    /* 1: bitwise reproducible results -- the panel's cross-CTA column
+                                 dots are summed in a fixed order (each CTA stores its partial,
+                                 every CTA sums them after the grid barrier) instead of by FP64
+                                 atomics, so two identical calls (and the ranks of a multi-GPU
+                                 call) give bitwise-equal H, tau, Q; costs one L2 round trip
+                                 per column reduction                          */
 } ft_opts;
 
 /* Fill *o with defaults (nb 0, abft 1, policy EAGER, c_thr 2, no faults, run to end). */

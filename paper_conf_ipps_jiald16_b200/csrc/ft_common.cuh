@@ -7,6 +7,9 @@
 #ifndef FT_NBMAX
 #define FT_NBMAX 64  // max panel width (opts.nb <= 64)
 #endif
+#ifndef FT_DPMAX
+#define FT_DPMAX 160  // deterministic mode: max CTAs per panel launch (rank group)
+#endif
 #define FT_KPAD (FT_NBMAX + 4)  // smem row stride for K <= 64 operands (conflict-free DMMA frags)
 
 #define FT_DEV __device__ __forceinline__
@@ -214,6 +217,41 @@ FT_DEV double sum_strided(const double *p, int64_t stride, int N) {
         s3 += v[3] + v[7];
     }
     return (s0 + s1) + (s2 + s3);
+}
+
+// Deterministic sums of CTA partials (opts.deterministic): out[v] = the sum over the P CTAs of
+// accumulator idx(v) of one set, idx running over [a0, a0+n0) then [a1, a1+n1) then [a2, a2+n2);
+// part points at the set's block of [FT_ACC_STRIDE][FT_DPMAX] partials.  Warp w takes values
+// w, w + nw, ... four at a time (all their loads in flight), lane l the CTAs l, l + 32, ... in
+// order, then a fixed xor tree: the same additions in the same order on every call and in every
+// CTA.  Called by every thread of the CTA; a __syncthreads must follow before out is read.
+FT_DEV void det_sum(const double *part, int P, int a0, int n0, int a1, int n1, int a2, int n2, double *out) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    const int nv = n0 + n1 + n2;
+    for (int v0 = w; v0 < nv; v0 += 4 * nw) {
+        double s[4];
+#pragma unroll
+        for (int u = 0; u < 4; u++) {
+            const int v = v0 + u * nw;
+            s[u] = 0.0;
+            if (v < nv) {
+                const int idx = v < n0 ? a0 + v : (v < n0 + n1 ? a1 + (v - n0) : a2 + (v - n0 - n1));
+                const double *q = part + (int64_t)idx * FT_DPMAX;
+                double x[(FT_DPMAX + 31) / 32];
+#pragma unroll
+                for (int b = 0; b < (FT_DPMAX + 31) / 32; b++) x[b] = lane + 32 * b < P ? __ldcg(q + lane + 32 * b) : 0.0;
+#pragma unroll
+                for (int b = 0; b < (FT_DPMAX + 31) / 32; b++) s[u] += x[b];
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < 4; u++) {
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) s[u] += __shfl_xor_sync(0xffffffffu, s[u], o);
+            const int v = v0 + u * nw;
+            if (lane == 0 && v < nv) out[v] = s[u];
+        }
+    }
 }
 
 FT_DEV double warp_sum(double v) {

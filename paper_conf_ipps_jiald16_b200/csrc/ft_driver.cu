@@ -92,7 +92,8 @@ struct Work {
            *acc = nullptr, *ckpt = nullptr, *ck_r = nullptr, *ck_c = nullptr, *ck_q = nullptr, *Fr = nullptr,
            *Qr = nullptr, *Qc = nullptr, *Dr = nullptr, *Dc = nullptr, *sums = nullptr, *ypart = nullptr,
            *rowpart = nullptr, *linepart = nullptr, *scratch = nullptr, *deltas = nullptr, *hA = nullptr, *htau = nullptr,
-           *ck_w = nullptr, *Dr2 = nullptr, *Dc2 = nullptr, *wpart = nullptr, *dec_delta = nullptr;
+           *ck_w = nullptr, *Dr2 = nullptr, *Dc2 = nullptr, *wpart = nullptr, *dec_delta = nullptr,
+           *dpart = nullptr;  // deterministic mode: per-CTA column-dot partials (PanelParams::dpart)
     int *dec_idx = nullptr;       // device decoder: compacted flagged rows / columns (2n)
     FtFix *dec_fix = nullptr;     // its fix plan (n + 8)
     FtDecOut *dec_out = nullptr;  // [pass 1, pass 2]
@@ -107,7 +108,8 @@ struct Work {
     size_t bytes = 0;
     void release() {
         double **ps[] = {&Wt, &Aw, &V, &Y, &Z, &T, &Wpart, &bvec, &acc, &ckpt, &ck_r, &ck_c, &ck_q, &Fr, &Qr, &Qc, &Dr, &Dc,
-                         &sums, &ypart, &rowpart, &linepart, &scratch, &deltas, &hA, &htau, &ck_w, &Dr2, &Dc2, &wpart};
+                         &sums, &ypart, &rowpart, &linepart, &scratch, &deltas, &hA, &htau, &ck_w, &Dr2, &Dc2, &wpart,
+                         &dpart};
         for (auto p : ps) {
             if (*p) cudaFree(*p);
             *p = nullptr;
@@ -136,14 +138,15 @@ std::map<int, Work> g_work;
 
 // CUDA graphs of fault-free calls, keyed by device, shape, options and caller buffers
 struct GraphKey {
-    int dev, n, ilo, ihi, nb, abft, policy, weighted;
+    int dev, n, ilo, ihi, nb, abft, policy, weighted, det;
     double c_thr;
     const void *dA;
     int lda;
     const void *dtau;
     bool operator<(const GraphKey &o) const {
-        return std::tie(dev, n, ilo, ihi, nb, abft, policy, weighted, c_thr, dA, lda, dtau) <
-               std::tie(o.dev, o.n, o.ilo, o.ihi, o.nb, o.abft, o.policy, o.weighted, o.c_thr, o.dA, o.lda, o.dtau);
+        return std::tie(dev, n, ilo, ihi, nb, abft, policy, weighted, det, c_thr, dA, lda, dtau) <
+               std::tie(o.dev, o.n, o.ilo, o.ihi, o.nb, o.abft, o.policy, o.weighted, o.det, o.c_thr, o.dA, o.lda,
+                        o.dtau);
     }
 };
 struct GraphEntry {
@@ -195,6 +198,7 @@ int get_work(int n, Work **out) {
     A(dalloc(&w.Z, (size_t)ldw * FT_NBMAX, b));
     A(dalloc(&w.bvec, (size_t)4 * ldw, b));
     A(dalloc(&w.acc, (size_t)FT_ACC_SETS * FT_ACC_SET_DOUBLES, b));
+    A(dalloc(&w.dpart, (size_t)FT_ACC_SETS * FT_ACC_STRIDE * FT_DPMAX, b));
     A(dalloc(&w.ckpt, (size_t)ldw * FT_NBMAX, b));
     A(dalloc(&w.ck_r, (size_t)ldw, b));
     A(dalloc(&w.ck_c, N1, b));
@@ -424,6 +428,7 @@ namespace {
 struct Call {
     int n, ilo, ihi, nb, abft, policy;
     int weighted = 0;  // NEXT-1: the weighted checksum pair rides as row / column n+1
+    int det = 0;       // opts.deterministic: fixed-order column-dot sums in the panel kernels
     // NEXT-4 (ft_dsytrd): symmetric input given by its lower triangle; d, e of the tridiagonal out
     int sym = 0;
     double *sym_d = nullptr, *sym_e = nullptr;
@@ -718,6 +723,7 @@ int enqueue_panel(Call &C, int t) {
     p.bvec = w.bvec;
     p.Z = w.Z;
     p.acc = w.acc;
+    p.dpart = C.det ? w.dpart : nullptr;
     p.bar = w.bar + (t & 1);
     p.bar_next = w.bar + ((t + 1) & 1);
     p.ctl = w.ctl;
@@ -1293,6 +1299,7 @@ int validate(int n, int ilo, int ihi, const void *A, int lda, const void *tau, c
         if (o->nfaults < 0 || o->nfaults > FT_MAXFAULTS || (o->nfaults > 0 && !o->faults)) return -7;
         if (o->stop_after_panel < -1) return -7;
         if (o->timing != 0 && o->timing != 1) return -7;
+        if (o->deterministic != 0 && o->deterministic != 1) return -7;
     }
     return 0;
 }
@@ -1313,6 +1320,7 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
     C.nb = o.nb > 0 ? o.nb : (n < 4096 ? 32 : 64);
     C.abft = o.abft;
     C.weighted = o.abft ? o.weighted : 0;
+    C.det = o.deterministic;
     C.policy = o.policy;
     C.c_thr = o.c_thr > 0 ? o.c_thr : 2.0;
     C.s = s;
@@ -1356,7 +1364,7 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
     if (graphable) {
         int dev = 0;
         CK(cudaGetDevice(&dev));
-        GraphKey key{dev, n, ilo, ihi, C.nb, C.abft, C.policy, C.weighted, C.c_thr, C.hA ? (const void *)C.hA : (const void *)dA,
+        GraphKey key{dev, n, ilo, ihi, C.nb, C.abft, C.policy, C.weighted, C.det, C.c_thr, C.hA ? (const void *)C.hA : (const void *)dA,
                      C.hA ? (int)C.hlda : lda, (const void *)dtau};
         auto it = g_graphs.find(key);
         if (it != g_graphs.end() && it->second.exec) {

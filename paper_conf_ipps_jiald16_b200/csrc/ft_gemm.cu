@@ -228,16 +228,17 @@ __global__ void __launch_bounds__(UT, 1)
         if (do_w) tma_prefetch_map(&tmV);
     }
     const unsigned tile_bytes = (unsigned)(SK * K * 8);
-    auto issue = [&](int tt, int b) {  // thread 0: tile tt's operands into buffers b
-        const int r = rbase + tt * UB;
-        if (p.do_right) {
-            mbar_expect_tx(&yfull[b], tile_bytes);
-            tma_load_2d(&S.Ys[b][0][0], &tmY, r, 0, &yfull[b]);
-        }
-        if (do_w) {
-            mbar_expect_tx(&vfull[b], tile_bytes);
-            tma_load_2d(&S.Vr[b][0][0], &tmV, r, 0, &vfull[b]);
-        }
+    auto issue_y = [&](int tt, int b) {  // thread 0: tile tt's Y rows into buffer b
+        mbar_expect_tx(&yfull[b], tile_bytes);
+        tma_load_2d(&S.Ys[b][0][0], &tmY, rbase + tt * UB, 0, &yfull[b]);
+    };
+    auto issue_v = [&](int tt, int b) {  // thread 0: tile tt's V rows into buffer b
+        mbar_expect_tx(&vfull[b], tile_bytes);
+        tma_load_2d(&S.Vr[b][0][0], &tmV, rbase + tt * UB, 0, &vfull[b]);
+    };
+    auto issue = [&](int tt, int b) {
+        if (p.do_right) issue_y(tt, b);
+        if (do_w) issue_v(tt, b);
     };
     if (K < KT && p.do_right)
         for (int i = tid; i < 2 * (KT - K) * SK; i += UT) {
@@ -326,12 +327,11 @@ __global__ void __launch_bounds__(UT, 1)
         if (tt == t0) {
             __syncthreads();  // Vc and the pre-update decision
             if (pre_abort()) return;
-        } else if (tid == 0 && tt + 1 < t1) {
-            // refill the buffers of tile tt-1 with tile tt+1 once every warp has released them
-            const unsigned pho = (unsigned)((it - 1) >> 1) & 1u;
-            if (p.do_right) mbar_wait(&yempty[b ^ 1], pho);
-            if (do_w) mbar_wait(&vempty[b ^ 1], pho);
-            issue(tt + 1, b ^ 1);
+        } else if (tid == 0 && tt + 1 < t1 && p.do_right) {
+            // refill tile tt-1's Y buffer with tile tt+1 once every warp has released it (its right
+            // pass: long done); the V buffer follows after this warp's own right pass, below
+            mbar_wait(&yempty[b ^ 1], (unsigned)((it - 1) >> 1) & 1u);
+            issue_y(tt + 1, b ^ 1);
         }
         if (p.do_right) {
             mbar_wait(&yfull[b], ph);
@@ -359,6 +359,12 @@ __global__ void __launch_bounds__(UT, 1)
                 }
         }
         if (do_w) {
+            if (tid == 0 && tt > t0 && tt + 1 < t1) {
+                // refill tile tt-1's V buffer with tile tt+1: by now every warp is normally past the
+                // W pass of tile tt-1, so this wait rarely blocks (and never blocks the Y refill)
+                mbar_wait(&vempty[b ^ 1], (unsigned)((it - 1) >> 1) & 1u);
+                issue_v(tt + 1, b ^ 1);
+            }
             mbar_wait(&vfull[b], ph);
             // only rows in [wr_lo, wr_hi) take part in W (a uniform test: interior tiles skip the masks)
             const int wlo = max(lo, p.wr_lo), whi = min(hi, p.wr_hi);

@@ -17,6 +17,9 @@
 #define FT_ACC_SETS 4               // sets indexed by the global column mod 4 (recycled in-kernel)
 #define FT_ACC_PAD 32               // doubles between accumulators: one 256-byte block (own L2 slice) each
 #define FT_ACC_SET_DOUBLES (FT_ACC_STRIDE * FT_ACC_PAD)
+#ifndef FT_DPMAX
+#define FT_DPMAX 160  // deterministic mode: max CTAs per panel launch (rank group)
+#endif
 
 // Device-resident control block: halt protocol, fused-verify flags, injector log.
 struct FtCtl {
@@ -55,6 +58,10 @@ struct PanelParams {
     double *A;
     int64_t ldw;
     double *V, *Y, *T, *tau, *acc;
+    // deterministic mode (opts.deterministic): the column dots' CTA partials are stored, not added,
+    // at dpart[(set * FT_ACC_STRIDE + i) * FT_DPMAX + cta] and summed in a fixed order after the grid
+    // barrier (ft_common.cuh det_sum): bitwise reproducible panels.  NULL: FP64 atomics into acc
+    double *dpart;
     double *bvec;        // [4][ldw]: b0 of columns c (parity c & 1), x of the explicit path (2 + parity)
     double *Z;           // ldw x FT_NBMAX: A(:, c+2:) V_x of the own rows when they do not fit in smem
     unsigned *bar;       // grid-barrier counter of this launch (zero at launch)

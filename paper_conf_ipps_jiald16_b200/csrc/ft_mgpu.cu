@@ -346,7 +346,8 @@ struct MgRank {
     int64_t ldw = 0;
     double *Aw = nullptr, *V = nullptr, *Y = nullptr, *Z = nullptr, *T = nullptr, *Wpart = nullptr, *Wt = nullptr, *bvec = nullptr,
            *acc = nullptr, *Qr = nullptr, *Qc = nullptr, *ypart = nullptr, *rowpart = nullptr, *vec = nullptr,
-           *vec2 = nullptr, *ck = nullptr, *full = nullptr;
+           *vec2 = nullptr, *ck = nullptr, *full = nullptr,
+           *dpart = nullptr;  // deterministic mode: per-CTA column-dot partials (PanelParams::dpart)
     void *ops = nullptr;  // MgOp list of a correction
     unsigned *bar = nullptr;
     int *strip_done = nullptr;
@@ -367,7 +368,8 @@ struct MgRank {
     unsigned *flags(int g) const { return reinterpret_cast<unsigned *>(peer[g] + lay.flags); }
     unsigned *xflags(int g) const { return reinterpret_cast<unsigned *>(peer[g] + lay.xflags); }
     void release() {
-        double **ps[] = {&Aw, &V, &Y, &Z, &T, &Wpart, &Wt, &bvec, &acc, &Qr, &Qc, &ypart, &rowpart, &vec, &vec2, &ck, &full};
+        double **ps[] = {&Aw, &V, &Y, &Z, &T, &Wpart, &Wt, &bvec, &acc, &Qr, &Qc, &ypart, &rowpart, &vec, &vec2, &ck, &full,
+                         &dpart};
         for (auto p : ps) {
             if (*p) cudaFree(*p);
             *p = nullptr;
@@ -418,6 +420,7 @@ int mg_alloc(MgRank &R, int n, int G, int rank) {
     A(cudaMalloc(&R.Z, (size_t)ldw * FT_NBMAX * sizeof(double)));
     A(cudaMalloc(&R.bvec, (size_t)4 * ldw * sizeof(double)));
     A(cudaMalloc(&R.acc, (size_t)FT_ACC_SETS * FT_ACC_SET_DOUBLES * sizeof(double)));
+    A(cudaMalloc(&R.dpart, (size_t)FT_ACC_SETS * FT_ACC_STRIDE * FT_DPMAX * sizeof(double)));
     A(cudaMalloc(&R.Qr, (size_t)ldw * sizeof(double)));
     A(cudaMalloc(&R.Qc, (size_t)ldw * sizeof(double)));
     A(cudaMalloc(&R.ypart, (size_t)std::min<int64_t>(kYtopRowsM, 64 * N1) * FT_NBMAX * sizeof(double)));
@@ -483,6 +486,7 @@ int mg_xchg(std::vector<MgRank *> &Rs, int mode, int root, std::vector<XchgRank>
 
 struct MgCall {
     int n, nb, G, abft, npanels;
+    int det = 0;  // opts.deterministic: fixed-order column dots (ranks then agree bitwise)
     double c_thr = 2.0;
     std::vector<ft_fault> faults;  // sites A and C (the owner's words); phases BEFORE_PANEL,
                                    // AFTER_RIGHT, AFTER_UPDATE, AT_END
@@ -662,6 +666,7 @@ int mg_panel(MgCall &C, int t) {
         p.bvec = R.bvec;
         p.Z = R.Z;
         p.acc = R.acc;
+        p.dpart = C.det ? R.dpart : nullptr;
         p.bar = R.bar + (t & 1);
         p.bar_next = R.bar + ((t + 1) & 1);
         p.ctl = R.ctl;
@@ -1051,6 +1056,7 @@ int mg_validate(int n, int ilo, int ihi, int lda, int nranks, const ft_opts &o) 
     if (o.nb < 0 || o.nb > FT_NBMAX) return -7;
     if (o.abft != 0 && o.abft != 1) return -7;
     if (o.stop_after_panel != -1 || o.weighted != 0) return -7;  // single-GPU path only
+    if (o.deterministic != 0 && o.deterministic != 1) return -7;
     if (o.nfaults < 0 || o.nfaults > FT_MAXFAULTS || (o.nfaults > 0 && (!o.faults || !o.abft))) return -7;
     for (int q = 0; q < o.nfaults; q++) {
         const ft_fault &f = o.faults[q];
@@ -1098,6 +1104,7 @@ int ft_dgehrd_vranks(int n, int ilo, int ihi, double *const *dA_local, int lda_l
     C.nb = o.nb > 0 ? o.nb : (n < 4096 ? 32 : 64);
     C.G = nranks;
     C.abft = o.abft;
+    C.det = o.deterministic;
     C.npanels = (n - 2 + C.nb - 1) / C.nb;
     C.s = (cudaStream_t)o.stream;
     C.lda = lda_local;
@@ -1162,6 +1169,7 @@ int ft_dgehrd_mgpu(int n, int ilo, int ihi, double *dA_local, int lda_local, dou
     C.nb = o.nb > 0 ? o.nb : (n < 4096 ? 32 : 64);
     C.G = nranks;
     C.abft = o.abft;
+    C.det = o.deterministic;
     C.npanels = (n - 2 + C.nb - 1) / C.nb;
     C.s = (cudaStream_t)o.stream;
     C.lda = lda_local;

@@ -84,6 +84,7 @@ struct PanelSmem {
     double s1[FT_NBMAX], w[FT_NBMAX], t[FT_NBMAX], ep[FT_NBMAX];  // ep: e^T V over rows >= c+1
     double vr1[FT_NBMAX + 1];           // V(c+1, 0:j)
     double scal[16];                    // SC_*
+    double dsum[2 * FT_NBMAX + 4];      // deterministic mode: the reduced column dots (det_sum)
     double acol[RMAX];                  // A(row, c) of the own rows
     double anext[RMAX];                 // A(row, c+1)
     double b0[RMAX];                    // b0 of the current column
@@ -369,6 +370,17 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
     //   then zB.zB -> acc[oE], sum zB -> acc[oE + 1]
     // An aligned group of LPO lanes per output (4..32, ~2 rows per lane), lanes stride the
     // rows, shuffle tree inside the warp; the group leader adds the CTA partial.
+    // a CTA partial of accumulator dst of set acc: FP64 atomic, or (deterministic mode) a store into
+    // the CTA's own slot, summed in a fixed order after the grid barrier (det_sum)
+    auto acc_add = [&](double *acc, int dst, double s) {
+        if (p.dpart)
+            p.dpart[((acc - p.acc) / FT_ACC_SET_DOUBLES * FT_ACC_STRIDE + dst) * FT_DPMAX + bid] = s;
+        else
+            atomicAdd(acc + dst * FT_ACC_PAD, s);
+    };
+    auto dset = [&](const double *acc) -> const double * {
+        return p.dpart + (acc - p.acc) / FT_ACC_SET_DOUBLES * FT_ACC_STRIDE * FT_DPMAX;
+    };
     auto coldot_add = [&](const double *zA, int JA, const double *zB, int JB, double *acc, int oA, int oB,
                           int oE) {
         const int NO = JA + JB + 2;
@@ -401,7 +413,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
                 }
                 if (!(p.dbg_mode & 4)) {
                     const int dst = o < JA ? oA + o : (o < JA + JB ? oB + o - JA : oE + (o - JA - JB));
-                    atomicAdd(acc + dst * FT_ACC_PAD, s0 + s1);
+                    acc_add(acc, dst, s0 + s1);
                 }
             }
             return;
@@ -441,7 +453,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
                 if (off < LPO) s += __shfl_xor_sync(0xffffffffu, s, off);
             if (o < NO && gl == 0 && !(p.dbg_mode & 4)) {
                 const int dst = o < JA ? oA + o : (o < JA + JB ? oB + o - JA : oE + (o - JA - JB));
-                atomicAdd(acc + dst * FT_ACC_PAD, s);
+                acc_add(acc, dst, s);
             }
         }
     };
@@ -727,20 +739,33 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
                 p.ctl->sums[2] = 0.0;
                 p.ctl->sums[3] = 0.0;
             }
+            b0c1 = ldcg(acc + ACC_B0 * FT_ACC_PAD);  // single writer
+            if (lane < j) vra = ldcg(V + (c + 1) + (int64_t)lane * ldw);
+            if (lane + 32 < j) vrb = ldcg(V + (c + 1) + (int64_t)(lane + 32) * ldw);
+            if (p.dpart) return;
             bb = ldcg(acc + ACC_BB * FT_ACC_PAD);
             eb = ldcg(acc + ACC_EB * FT_ACC_PAD);
-            b0c1 = ldcg(acc + ACC_B0 * FT_ACC_PAD);
             if (lane < j) {
                 s1a = ldcg(acc + (ACC_S1 + lane) * FT_ACC_PAD);
                 sxa = ldcg(acc + (ACC_SX + lane) * FT_ACC_PAD);
-                vra = ldcg(V + (c + 1) + (int64_t)lane * ldw);
             }
             if (lane + 32 < j) {
                 s1b = ldcg(acc + (ACC_S1 + lane + 32) * FT_ACC_PAD);
                 sxb = ldcg(acc + (ACC_SX + lane + 32) * FT_ACC_PAD);
-                vrb = ldcg(V + (c + 1) + (int64_t)(lane + 32) * ldw);
             }
         });
+        if (p.dpart) {  // deterministic mode: s1, sx, bb, eb from the CTA partials in a fixed order
+            det_sum(dset(acc), (int)P, ACC_S1, j, ACC_SX, j, ACC_BB, 2, S.dsum);
+            __syncthreads();
+            if (wid == 0) {
+                s1a = lane < j ? S.dsum[lane] : 0.0;
+                s1b = lane + 32 < j ? S.dsum[lane + 32] : 0.0;
+                sxa = lane < j ? S.dsum[j + lane] : 0.0;
+                sxb = lane + 32 < j ? S.dsum[j + lane + 32] : 0.0;
+                bb = S.dsum[2 * j];
+                eb = S.dsum[2 * j + 1];
+            }
+        }
         PROBE(2);
         if (gw) {
             // speculative: y = A(:, c+1) + scale (A(:, c+2:) b0_x - Z w); MG takes the explicit path
@@ -849,12 +874,23 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
             coldot_add(nullptr, 0, S.bmX, j, acc, 0, ACC_FVX, ACC_FNRM);
             double fnrm = 0.0, fex = 0.0, fal = 0.0, fva = 0.0, fvb = 0.0;
             grid_sync(epoch, [&]() {
+                fal = ldcg(acc + ACC_FAL * FT_ACC_PAD);  // single writer
+                if (p.dpart) return;
                 fnrm = ldcg(acc + ACC_FNRM * FT_ACC_PAD);
                 fex = ldcg(acc + ACC_FEX * FT_ACC_PAD);
-                fal = ldcg(acc + ACC_FAL * FT_ACC_PAD);
                 if (lane < j) fva = ldcg(acc + (ACC_FVX + lane) * FT_ACC_PAD);
                 if (lane + 32 < j) fvb = ldcg(acc + (ACC_FVX + lane + 32) * FT_ACC_PAD);
             });
+            if (p.dpart) {  // deterministic mode
+                det_sum(dset(acc), (int)P, ACC_FVX, j, ACC_FNRM, 2, 0, 0, S.dsum);
+                __syncthreads();
+                if (wid == 0) {
+                    fva = lane < j ? S.dsum[lane] : 0.0;
+                    fvb = lane + 32 < j ? S.dsum[lane + 32] : 0.0;
+                    fnrm = S.dsum[j];
+                    fex = S.dsum[j + 1];
+                }
+            }
             if (gw) {
                 gemv(bvx, c, false);
             } else if (wid == 0) {
@@ -1189,6 +1225,7 @@ cudaError_t ft_launch_panel_multi(const PanelLaunch &L, int nsm, cudaStream_t s)
         Lx.r[i].ncc = ncc;
         if (explicit_path) Lx.r[i].dbg_mode |= ((explicit_path & 0xff) ? 8 : 0) | (explicit_path >> 8);
     }
+    if (L.r[0].dpart && grid > FT_DPMAX) return cudaErrorInvalidValue;  // deterministic mode: partial slots
     const PanelLaunch *Lp = &Lx;
     void *args[] = {const_cast<PanelLaunch *>(Lp)};
     g_ft_launches++;

@@ -64,6 +64,7 @@ struct PanelSmemW {
     double t[FT_NBMAX];                 // V^T v
     double s1[FT_NBMAX];                // V^T b0 (reduced)
     double scal[8];                     // tau, beta, scale, vchk, alpha
+    double dsum[2 * FT_NBMAX + 4];      // deterministic mode: the reduced column dots (det_sum)
     double acol[RMAX];                  // A(row, c) of the own rows
     double anext[RMAX];                 // A(row, c+1)
     double b0[RMAX];                    // b0 (rows), then b
@@ -211,6 +212,10 @@ __global__ void __launch_bounds__(PT, 1) k_panel_wide(const __grid_constant__ Pa
     const int npart = R2p <= 32 ? NGW : ncl;  // partials per row pair
 
     auto is_data = [&](int row) { return row >= k + 1 && row < ihi; };
+    // deterministic mode: the partial block of the accumulator set `acc` belongs to
+    auto dset = [&](const double *acc) -> const double * {
+        return p.dpart + (acc - p.acc) / FT_ACC_SET_DOUBLES * FT_ACC_STRIDE * FT_DPMAX;
+    };
     auto is_valid = [&](int row) { return (row >= k + 1 && row < ihi) || (p.abft && row == n); };
 
     // ---- CTA-parallel building blocks of the column chain --------------------------------
@@ -265,7 +270,10 @@ __global__ void __launch_bounds__(PT, 1) k_panel_wide(const __grid_constant__ Pa
             if (off < LPO) s += __shfl_xor_sync(0xffffffffu, s, off);
         if (o < NO && gl == 0 && !(p.dbg_mode & 4)) {
             const int dst = o < J ? acc_o0 + o : acc_extra0 + (o - J);
-            atomicAdd(acc + dst * FT_ACC_PAD, s);
+            if (p.dpart)  // deterministic mode: this CTA's partial in its own slot
+                p.dpart[((acc - p.acc) / FT_ACC_SET_DOUBLES * FT_ACC_STRIDE + dst) * FT_DPMAX + bid] = s;
+            else
+                atomicAdd(acc + dst * FT_ACC_PAD, s);
         }
     };
     // grid barrier: thread 0 arrives (release, cumulative over the CTA's writes ordered by the
@@ -367,9 +375,14 @@ __global__ void __launch_bounds__(PT, 1) k_panel_wide(const __grid_constant__ Pa
             coldot_add(Vl, S.bm, j, false, acc, 0, 0);
             PROBE(1);
             grid_sync(epoch, [&]() {
+                if (p.dpart) return;
                 if (lane < j) S.s1[lane] = ldcg(acc + lane * FT_ACC_PAD);
                 if (lane + 32 < j) S.s1[lane + 32] = ldcg(acc + (lane + 32) * FT_ACC_PAD);
             });
+            if (p.dpart) {  // deterministic mode: fixed-order sums of the CTA partials
+                det_sum(dset(acc), (int)P, 0, j, 0, 0, 0, 0, S.s1);
+                __syncthreads();
+            }
             PROBE(2);
             // w = T^T s1 (an 8-lane group per output)
             {
@@ -420,18 +433,25 @@ __global__ void __launch_bounds__(PT, 1) k_panel_wide(const __grid_constant__ Pa
                 p.ctl->sums[2] = 0.0;
                 p.ctl->sums[3] = 0.0;
             }
+            alpha = ldcg(acc + ACC_ALPHA * FT_ACC_PAD);  // single writer
+            if (lane < j) vn0 = ldcg(V + (c + 1) + (int64_t)lane * ldw);
+            if (lane + 32 < j) vn1 = ldcg(V + (c + 1) + (int64_t)(lane + 32) * ldw);
+            if (p.dpart) return;
             nrm2 = ldcg(acc + ACC_NRM * FT_ACC_PAD);
             sx = ldcg(acc + ACC_SX * FT_ACC_PAD);
-            alpha = ldcg(acc + ACC_ALPHA * FT_ACC_PAD);
-            if (lane < j) {
-                vn0 = ldcg(V + (c + 1) + (int64_t)lane * ldw);
-                vt0 = ldcg(acc + (ACC_VTB + lane) * FT_ACC_PAD);
-            }
-            if (lane + 32 < j) {
-                vn1 = ldcg(V + (c + 1) + (int64_t)(lane + 32) * ldw);
-                vt1 = ldcg(acc + (ACC_VTB + lane + 32) * FT_ACC_PAD);
-            }
+            if (lane < j) vt0 = ldcg(acc + (ACC_VTB + lane) * FT_ACC_PAD);
+            if (lane + 32 < j) vt1 = ldcg(acc + (ACC_VTB + lane + 32) * FT_ACC_PAD);
         });
+        if (p.dpart) {  // deterministic mode: V^T x, ||x||^2, e^T x from the CTA partials in a fixed order
+            det_sum(dset(acc), (int)P, ACC_VTB, j, ACC_NRM, 2, 0, 0, S.dsum);
+            __syncthreads();
+            if (wid == 0) {
+                vt0 = lane < j ? S.dsum[lane] : 0.0;
+                vt1 = lane + 32 < j ? S.dsum[lane + 32] : 0.0;
+                nrm2 = S.dsum[j];
+                sx = S.dsum[j + 1];
+            }
+        }
         PROBE(5);
         unsigned long long gt_start = 0;
         if (p.dbg && tid == 0 && j == 8) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(gt_start));
@@ -832,6 +852,7 @@ cudaError_t ft_launch_panel_wide(const PanelLaunch &L, int nsm, cudaStream_t s) 
     const size_t fixed = sizeof(PanelSmemW);
     const size_t want = fixed + (size_t)2 * VS * rmax * sizeof(double);
     const bool cache = want <= (size_t)max_smem;
+    if (L.r[0].dpart && grid > FT_DPMAX) return cudaErrorInvalidValue;  // deterministic mode: partial slots
     void *args[] = {const_cast<PanelLaunch *>(&L)};
     g_ft_launches++;
     g_ft_wide_launches++;

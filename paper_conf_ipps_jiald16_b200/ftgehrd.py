@@ -55,7 +55,8 @@ class Opts(ctypes.Structure):
                 ("policy", ctypes.c_int32), ("c_thr", ctypes.c_double),
                 ("faults", ctypes.POINTER(Fault)), ("nfaults", ctypes.c_int32),
                 ("report", ctypes.POINTER(Report)), ("stop_after_panel", ctypes.c_int32),
-                ("dchk_out", ctypes.c_void_p), ("stream", ctypes.c_void_p), ("timing", ctypes.c_int32)]
+                ("dchk_out", ctypes.c_void_p), ("stream", ctypes.c_void_p), ("timing", ctypes.c_int32),
+                ("deterministic", ctypes.c_int32)]
 
 
 def build(force: bool = False) -> str:
@@ -133,7 +134,7 @@ def fortran(x):
 
 
 def make_opts(nb=0, abft=True, policy=POLICY_EAGER, c_thr=2.0, faults=(), report=None,
-              stop_after_panel=-1, dchk_out=None, stream=None, timing=False, weighted=False):
+              stop_after_panel=-1, dchk_out=None, stream=None, timing=False, weighted=False, deterministic=False):
     o = Opts()
     lib().ft_opts_default(ctypes.byref(o))
     o.nb = nb
@@ -156,6 +157,7 @@ def make_opts(nb=0, abft=True, policy=POLICY_EAGER, c_thr=2.0, faults=(), report
     o.dchk_out = ctypes.c_void_p(dchk_out.data_ptr()) if dchk_out is not None else None
     o.stream = _stream_ptr(stream)
     o.timing = 1 if timing else 0
+    o.deterministic = 1 if deterministic else 0
     o._keep = farr  # keep the fault array alive
     return o
 
@@ -304,7 +306,8 @@ def _slab_ld(S, n):
     return max(S.stride(1) if S.shape[1] > 1 else n, n, 1)
 
 
-def dgehrd_vranks(slabs: list, nb: int = 0, abft: bool = True, taus=None, stream=None, faults=(), c_thr=2.0):
+def dgehrd_vranks(slabs: list, nb: int = 0, abft: bool = True, taus=None, stream=None, faults=(), c_thr=2.0,
+                  deterministic=False):
     """Sharded reduction with len(slabs) VIRTUAL ranks on the current GPU (ft_dgehrd_vranks).
 
     slabs: the ranks' n x ncols CUDA float64 column-major slabs (modified in place).
@@ -325,7 +328,7 @@ def dgehrd_vranks(slabs: list, nb: int = 0, abft: bool = True, taus=None, stream
     pa = (ctypes.c_void_p * G)(*[S.data_ptr() for S in slabs])
     pt = (ctypes.c_void_p * G)(*[t.data_ptr() for t in taus])
     rep = Report()
-    o = make_opts(nb=nb, abft=abft, report=rep, stream=stream, faults=faults, c_thr=c_thr)
+    o = make_opts(nb=nb, abft=abft, report=rep, stream=stream, faults=faults, c_thr=c_thr, deterministic=deterministic)
     info = lib().ft_dgehrd_vranks(n, 1, n, pa, lda, pt, G, ctypes.byref(o))
     return taus, Result(info, rep, rep.event_list())
 
@@ -356,7 +359,8 @@ def mgpu_init(n_max: int, group=None) -> None:
         raise RuntimeError(f"ft_mgpu_connect: {strerror(info)}")
 
 
-def dgehrd_mgpu(slab, rank: int, nranks: int, nb: int = 0, abft: bool = True, tau=None, stream=None, faults=()):
+def dgehrd_mgpu(slab, rank: int, nranks: int, nb: int = 0, abft: bool = True, tau=None, stream=None, faults=(),
+                deterministic=False):
     """This rank's part of the sharded reduction (after mgpu_init). Returns (tau, Result)."""
     import torch
     n = slab.shape[0]
@@ -364,7 +368,7 @@ def dgehrd_mgpu(slab, rank: int, nranks: int, nb: int = 0, abft: bool = True, ta
     if tau is None:
         tau = torch.zeros(max(n - 1, 1), dtype=torch.float64, device=slab.device)
     rep = Report()
-    o = make_opts(nb=nb, abft=abft, report=rep, stream=stream, faults=faults)
+    o = make_opts(nb=nb, abft=abft, report=rep, stream=stream, faults=faults, deterministic=deterministic)
     info = lib().ft_dgehrd_mgpu(n, 1, n, ctypes.c_void_p(slab.data_ptr()), lda, ctypes.c_void_p(tau.data_ptr()),
                                 rank, nranks, ctypes.byref(o))
     return tau, Result(info, rep, rep.event_list())
