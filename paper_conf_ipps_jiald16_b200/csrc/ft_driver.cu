@@ -635,7 +635,7 @@ int right_update(Call &C, int t, double sign, int do_w, bool precheck = false) {
     g.wr_hi = C.ihi;
     g.do_w = do_w;
     g.fold_row = (C.abft && !C.weighted) ? g_right_fold : 0;  // row n (c) as a GEMV of the last row split
-    g.nsplit = ft_gemm_splits(g.r_lo, g.r_hi - g.fold_row, g.c_lo, g.c_hi, w.nsm, g.has_m);
+    g.nsplit = ft_gemm_splits(g.r_lo, g.r_hi - g.fold_row, g.c_lo, g.c_hi, w.nsm, g.has_m, do_w ? g.wr_lo : g.r_hi);
     if (do_w) {
         g.Wt = w.Wt;
         g.T = w.T;

@@ -7,6 +7,7 @@
 // the column checksum c -- so Theorem 1 is carried by the same tiles.
 // Rollback (reverse computation, Alg. 3 l.14) is the same kernels with sign +1.
 //
+#include <algorithm>
 #include <cstdlib>
 #include <cstring>
 
@@ -48,17 +49,54 @@ static int best_splits(int nstrip, int nrt, int nsm, int cap, int per_sm, int ov
     }
     return best;
 }
-int ft_gemm_splits(int r_lo, int r_hi, int c_lo, int c_hi, int nsm, int extra_strips) {
+// Right-update tile weights: a tile above the W rows (rows < wr_lo: the rows 0..k the update
+// reaches but W = V^T A_new does not) runs the right pass only and counts 1; a tile that also runs
+// the W pass counts 2 (twice the DMMA work, the same HBM traffic).  The row splits of a strip cut
+// it into equal WEIGHTS (the kernel maps split y to its tiles with right_split_tile), so at late
+// panels -- where most rows are above the panel -- the CTAs holding W tiles are no longer the tail.
+// tw: the number of right-only tiles at the top of the strip (nrt: none takes part in W).
+__host__ __device__ inline int right_split_tile(long long u, int tw) {
+    return u <= tw ? (int)u : tw + (int)((u - tw + 1) / 2);
+}
+static inline int right_tw(int wr_lo, int rbase, int nrt) {
+    if (wr_lo < 0) return 0;
+    const int t = (wr_lo - rbase) / UB;
+    return t < 0 ? 0 : (t > nrt ? nrt : t);
+}
+int ft_gemm_splits(int r_lo, int r_hi, int c_lo, int c_hi, int nsm, int extra_strips, int wr_lo) {
     // extra_strips: strips of the same launch outside [c_lo, c_hi) (the M-part strip); they take
     // grid slots like the others (counted as full strips: the model stays an upper bound)
     const int nstrip = (c_hi - c_lo + UB - 1) / UB + extra_strips;
-    const int nrt = (r_hi - (r_lo / UB) * UB + UB - 1) / UB;
+    const int rbase = (r_lo / UB) * UB;
+    const int nrt = (r_hi - rbase + UB - 1) / UB;
     // right update: one CTA per SM (the next C tile is prefetched in registers)
     // per-CTA prologue / epilogue (V strip, first copies, W partials) of 1.5 tiles: with the split cap
     // at 32 a zero term picks many short CTAs (right update at C3: 356 ms at 0, 340 ms at 3-10;
     // profiles/r02/gemm_tma/right_ovh_sweep.txt); FT_RIGHT_OVH overrides for sweeps
     static const int ovh = getenv("FT_RIGHT_OVH") ? atoi(getenv("FT_RIGHT_OVH")) : 6;
-    return best_splits(nstrip > 0 ? nstrip : 1, nrt > 0 ? nrt : 1, nsm, FT_WSPLIT_MAX, 1, ovh);
+    if (nstrip <= 0 || nrt <= 0) return 1;
+    const int tw = right_tw(wr_lo, rbase, nrt);
+    const long long units = (long long)tw + 2LL * (nrt - tw);  // weights: right-only 1, right + W 2
+    const int slots = nsm;
+    int best = 1;
+    long long best_cost = -1;
+    for (int ns = 1; ns <= FT_WSPLIT_MAX && ns <= nrt; ns++) {
+        const long long waves = ((long long)nstrip * ns + slots - 1) / slots;
+        // heaviest split in quarter tiles (a right-only tile is half a right + W tile = 2 quarters)
+        long long umax = 0;
+        for (int y = 0; y < ns; y++) {
+            const long long u0 = (long long)y * units / ns, u1 = (long long)(y + 1) * units / ns;
+            const int a = right_split_tile(u0, tw), b = right_split_tile(u1, tw);
+            const long long w = (long long)(b - a) * 4 - 2LL * std::max(0, std::min(b, tw) - std::min(a, tw));
+            if (w > umax) umax = w;
+        }
+        const long long cost = waves * (umax + ovh);
+        if (best_cost < 0 || cost < best_cost) {
+            best_cost = cost;
+            best = ns;
+        }
+    }
+    return best;
 }
 
 // 2-D tensor map of a column-major ldw x K operand panel (V or Y; element (row, col) at
@@ -188,8 +226,11 @@ __global__ void __launch_bounds__(UT, 1)
     const double sg = p.sign;
     const int rbase = (r_lo / UB) * UB;
     const int nrt = (r_hi - rbase + UB - 1) / UB;
-    const int t0 = (int)((long long)blockIdx.y * nrt / gridDim.y);
-    const int t1 = (int)((long long)(blockIdx.y + 1) * nrt / gridDim.y);
+    // this split's tiles: equal weights per split (right-only tiles 1, right + W tiles 2)
+    const int tw = do_w ? (p.wr_lo <= rbase ? 0 : min(nrt, (p.wr_lo - rbase) / UB)) : nrt;
+    const long long units = (long long)tw + 2LL * (nrt - tw);
+    const int t0 = right_split_tile((long long)blockIdx.y * units / gridDim.y, tw);
+    const int t1 = right_split_tile((long long)(blockIdx.y + 1) * units / gridDim.y, tw);
     constexpr int NJ = KT / 8;
     // fold_row: row p.r_hi (= n, the column checksum c) is updated by the last row split as a GEMV,
     // 4 lanes per strip column; c(col) is prefetched here, its use is after the tile loop

@@ -164,7 +164,8 @@ struct CUtensorMap_st;
 int ft_panel_tmap(struct CUtensorMap_st *m, const double *base, int64_t ldw, int K, int rows);
 #define FT_WSPLIT_MAX 32  // max row splits of the right update (deterministic W partials)
 // row splits the right-update launch uses for this block (the left update's k_wprep sums them)
-int ft_gemm_splits(int r_lo, int r_hi, int c_lo, int c_hi, int nsm, int extra_strips = 0);
+// wr_lo: first row of the W pass (tiles above it are weighted as right-only, see ft_gemm.cu); -1: all
+int ft_gemm_splits(int r_lo, int r_hi, int c_lo, int c_hi, int nsm, int extra_strips = 0, int wr_lo = -1);
 
 struct GemmLeftParams {
     double *A;

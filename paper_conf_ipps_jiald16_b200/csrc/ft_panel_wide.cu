@@ -47,7 +47,10 @@
 #define RMAX PT       // max rows per CTA
 #define NSLOT (PT / 8)  // 8-lane groups per CTA (rows / outputs handled at once)
 #ifndef GB
-#define GB 8          // GEMV load batch (double2 of A + b per lane)
+// GEMV load batch (double2 of A + b per lane): 12 streams at 0.9 of the HBM copy bandwidth at C3
+// (8: -1.4 % panel time; 16 spills; a software-pipelined 2 x 6 / 2 x 8 batch: +8 %,
+// profiles/r02/s3/gemv_batch_ab.txt)
+#define GB 12
 #endif
 
 // accumulator set layout (FT_ACC_STRIDE doubles): [0,64) s1 = V^T b0 | [64,128) V^T x |
@@ -520,6 +523,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel_wide(const __grid_constant__ Pa
                         rs.y += a[u].y;
                     }
                 }
+
                 if (col < cend) {  // ragged tail: one predicated batch (all loads in flight together)
                     double2 a[GB];
                     double v[GB];

@@ -139,7 +139,7 @@ def test_deterministic_option_validated():
     A = synth.matrix(64)
     dA = ft.fortran(torch.from_numpy(A).cuda())
     tau = torch.zeros(64, dtype=torch.float64, device="cuda")
-    o = ft.make_opts()
+    o = ft.ftgehrd.make_opts()
     o.deterministic = 2
     assert ft.lib().ft_dgehrd(64, 1, 64, ctypes.c_void_p(dA.data_ptr()), 64, ctypes.c_void_p(tau.data_ptr()),
                               ctypes.byref(o)) == -7
