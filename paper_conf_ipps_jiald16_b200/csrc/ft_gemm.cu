@@ -277,10 +277,6 @@ __global__ void __launch_bounds__(UT, 1)
         mbar_expect_tx(&vfull[b], tile_bytes);
         tma_load_2d(&S.Vr[b][0][0], &tmV, rbase + tt * UB, 0, &vfull[b]);
     };
-    auto issue = [&](int tt, int b) {
-        if (p.do_right) issue_y(tt, b);
-        if (do_w) issue_v(tt, b);
-    };
     if (K < KT && p.do_right)
         for (int i = tid; i < 2 * (KT - K) * SK; i += UT) {
             const int b = i / ((KT - K) * SK), rem = i % ((KT - K) * SK);
@@ -288,9 +284,14 @@ __global__ void __launch_bounds__(UT, 1)
         }
     if (foldr && tid < KT) S.Yn[tid] = tid < K ? __ldcg(p.Y + p.r_hi + (int64_t)tid * p.ldw) : 0.0;
     __syncthreads();  // barrier init visible before the first copies
-    if (tid == 0 && t0 < t1) {
-        issue(t0, 0);
-        if (t0 + 1 < t1) issue(t0 + 1, 1);
+    // tiles above the W rows (tt < tw) run the right pass only: no V tile, no W pass (their W rows
+    // are all masked); the V pipeline runs over this CTA's W tiles tv0 .. t1-1
+    const int tv0 = max(t0, tw);
+    const int ny_issued = (p.do_right && t0 < t1) ? min(2, t1 - t0) : 0;
+    const int nv_issued = (do_w && tv0 < t1) ? min(2, t1 - tv0) : 0;
+    if (tid == 0) {
+        for (int b = 0; b < ny_issued; b++) issue_y(t0 + b, b);
+        for (int b = 0; b < nv_issued; b++) issue_v(tv0 + b, b);
     }
     // sign * V(cols, :) once per CTA (sign folded into the A operand: the accumulators start from C
     // itself and hold C_new at the end -- the same roundings as sign * (sign C + V Y^T))
@@ -315,7 +316,6 @@ __global__ void __launch_bounds__(UT, 1)
     for (int mi = 0; mi < 2; mi++)
 #pragma unroll
         for (int a = 0; a < NJ; a++) wacc[mi][a][0] = wacc[mi][a][1] = 0.0;
-    const int ntile_issued = t0 < t1 ? min(2, t1 - t0) : 0;
     auto pre_abort = [&]() -> bool {  // after a __syncthreads that follows the evaluation
         const bool raise = !halted && p.pre_ctl && s_reason;
         if (!halted && !raise) return false;
@@ -328,10 +328,8 @@ __global__ void __launch_bounds__(UT, 1)
             ctl->halt = 1;
         }
         // the copies in flight land before the CTA's shared memory is released
-        for (int b = 0; b < ntile_issued; b++) {
-            if (p.do_right) mbar_wait(&yfull[b], 0u);
-            if (do_w) mbar_wait(&vfull[b], 0u);
-        }
+        for (int b = 0; b < ny_issued; b++) mbar_wait(&yfull[b], 0u);
+        for (int b = 0; b < nv_issued; b++) mbar_wait(&vfull[b], 0u);
         return true;  // nothing consumed: the panel is redone from its checkpoint
     };
     // C tile of tile tt into registers (16-byte loads; masked pairs at the edges)
@@ -399,14 +397,15 @@ __global__ void __launch_bounds__(UT, 1)
                     else store_pair(colp2[mi], row, lo, hi, colok2[mi], acc[mi][ni][0], acc[mi][ni][1]);
                 }
         }
-        if (do_w) {
-            if (tid == 0 && tt > t0 && tt + 1 < t1) {
-                // refill tile tt-1's V buffer with tile tt+1: by now every warp is normally past the
-                // W pass of tile tt-1, so this wait rarely blocks (and never blocks the Y refill)
-                mbar_wait(&vempty[b ^ 1], (unsigned)((it - 1) >> 1) & 1u);
-                issue_v(tt + 1, b ^ 1);
+        if (do_w && tt >= tw) {
+            const int jv = tt - tv0, bv = jv & 1;  // this tile's place in the V pipeline
+            if (tid == 0 && jv > 0 && tt + 1 < t1) {
+                // refill the V buffer of the previous W tile with tile tt+1: by now every warp is
+                // normally past that W pass, so this wait rarely blocks (and never blocks the Y refill)
+                mbar_wait(&vempty[bv ^ 1], (unsigned)((jv - 1) >> 1) & 1u);
+                issue_v(tt + 1, bv ^ 1);
             }
-            mbar_wait(&vfull[b], ph);
+            mbar_wait(&vfull[bv], (unsigned)(jv >> 1) & 1u);
             // only rows in [wr_lo, wr_hi) take part in W (a uniform test: interior tiles skip the masks)
             const int wlo = max(lo, p.wr_lo), whi = min(hi, p.wr_hi);
             if (!(wlo == r && whi == r + UB)) {
@@ -434,13 +433,13 @@ __global__ void __launch_bounds__(UT, 1)
                 const int row = wr * 32 + ni * 8 + 2 * lc + (e ^ sw);
 #pragma unroll
                 for (int nj = 0; nj < NJ; nj++) {
-                    const double bv = S.Vr[b][nj * 8 + lr][row];
+                    const double vb = S.Vr[bv][nj * 8 + lr][row];
 #pragma unroll
-                    for (int mi = 0; mi < 2; mi++) dmma_8x8x4(wacc[mi][nj][0], wacc[mi][nj][1], a[mi], bv);
+                    for (int mi = 0; mi < 2; mi++) dmma_8x8x4(wacc[mi][nj][0], wacc[mi][nj][1], a[mi], vb);
                 }
             }
             __syncwarp();
-            if (lane == 0) mbar_arrive(&vempty[b]);
+            if (lane == 0) mbar_arrive(&vempty[bv]);
         }
     }
     if (t0 >= t1) {  // no tile: take the pre-update decision here (no strip counter on a halt)
