@@ -41,8 +41,12 @@
 
 #define PT 512        // threads per CTA
 #define NW (PT / 32)  // warps per CTA
-#define NGW (NW - 1)  // GEMV warps (warp 0 is the control warp)
-#define GR 8          // row-group granularity (64 bytes of a column)
+#define NGW NW  // GEMV warps (warp 0, the control warp, joins after its chain work)
+// row-group granularity of the CTA row blocks (64 bytes of a column; the driver's ft_panel_group_rows).
+// 2-row groups (equal rows per CTA to one double2) measured no faster at C3: the slowest CTAs of a
+// column are set by the address position of their rows, not by the +8-row blocks
+#define GR 8
+#define GR_DRIVER 8
 #define VS 65         // shared-memory row stride of the V / Y row caches (doubles)
 #define RMAX PT       // max rows per CTA
 #define NSLOT (PT / 8)  // 8-lane groups per CTA (rows / outputs handled at once)
@@ -458,9 +462,73 @@ __global__ void __launch_bounds__(PT, 1) k_panel_wide(const __grid_constant__ Pa
         PROBE(5);
         unsigned long long gt_start = 0;
         if (p.dbg && tid == 0 && j == 8) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(gt_start));
-        if (wid > 0) {
-            // ======================= GEMV warps: y = A(:, c+1:) v on the unscaled b ===========
-            const int gt = tid - 32;
+        if (wid == 0) {
+            // ======================= control warp: (iii) DLARFG (R1), V(:, j) ================
+            const Refl rf = dlarfg_scalars(nrm2, alpha, c + 2 >= ihi);
+            const double tau = rf.tau, beta = rf.beta, scale = rf.scale;
+            const double vchk = 1.0 + scale * sx;  // V_chk(j) = e^T v
+            // t = V^T v = V(c+1,:)^T + scale * V^T x; V(c+1, :) is also the next column's vrow
+            if (lane < j) {
+                S.t[lane] = vn0 + scale * vt0;
+                S.vrow[lane] = vn0;
+            }
+            if (lane + 32 < j) {
+                S.t[lane + 32] = vn1 + scale * vt1;
+                S.vrow[lane + 32] = vn1;
+            }
+            if (lane == 0) {
+                S.vrow[j] = 1.0;
+                S.scal[0] = tau;
+                S.scal[2] = scale;
+            }
+            PROBE(9);
+            // V(:, j) and the reduced column c of the own rows
+#pragma unroll 1
+            for (int rl = lane; rl < R; rl += 32) {
+                const int row = r0 + rl;
+                const double b = S.b0[rl];
+                if (row == n && p.abft) {
+                    V[row + (int64_t)j * ldw] = vchk;
+                    if (CACHE) Vl[rl * XR + j * XC] = vchk;
+                    Apan[row + (int64_t)c * ldw] = (tau != 0.0) ? b - vchk * (alpha - beta) : b;  // left term (R7)
+                } else if (is_data(row)) {
+                    double vv, av;
+                    if (row <= c) {
+                        vv = 0.0;
+                        av = b;
+                    } else if (row == c + 1) {
+                        vv = 1.0;
+                        av = beta;
+                    } else {
+                        vv = scale * b;
+                        av = vv;
+                    }
+                    V[row + (int64_t)j * ldw] = vv;
+                    if (CACHE) Vl[rl * XR + j * XC] = vv;
+                    Apan[row + (int64_t)c * ldw] = av;
+                } else if (CACHE) {
+                    Vl[rl * XR + j * XC] = 0.0;  // rows outside the panel take no part in the dots
+                }
+            }
+            if (bid == 0 && lane == 0) {
+                p.tau[c] = tau;
+                if (p.abft) {
+                    p.Qc[c] = vchk - 1.0;  // Q column checksum (P:266)
+                    qc_corner += vchk - 1.0;
+                }
+            }
+            // recycle the accumulator set of column c+2 (= that of column c-2): every CTA has
+            // finished reading it, and column c+2 adds into it only after two more syncs
+            if (bid == 0)
+                for (int i = lane; i < FT_ACC_STRIDE; i += 32) p.acc[((c + 2) & 3) * FT_ACC_SET_DOUBLES + i * FT_ACC_PAD] = 0.0;
+            PROBE(6);
+        }
+        {
+            // ======================= GEMV, all 16 warps: y = A(:, c+1:) v on the unscaled b ===
+            // (warp 0 joins after its DLARFG / V(:, j) work above: with 512 lanes a CTA of 112 rows
+            // streams 9 columns at a time instead of 8 -- the CTAs with the most rows set the
+            // column's barrier)
+            const int gt = tid;
             const int rp = gt % R2p, cl = gt / R2p;
             const bool gemv_on = rp < R2 && cl < ncl;
             const double2 *__restrict__ A2 = reinterpret_cast<const double2 *>(A + r0);
@@ -554,73 +622,13 @@ __global__ void __launch_bounds__(PT, 1) k_panel_wide(const __grid_constant__ Pa
                         }
                     }
                 if (lane < R2p) {
-                    S.red[(wid - 1) * R2p + lane] = ya;
-                    if (vfy) S.rsr[(wid - 1) * R2p + lane] = rs;
+                    S.red[wid * R2p + lane] = ya;
+                    if (vfy) S.rsr[wid * R2p + lane] = rs;
                 }
             } else if (cl < ncl) {
                 S.red[cl * R2p + rp] = ya;
                 if (vfy) S.rsr[cl * R2p + rp] = rs;
             }
-        } else {
-            // ======================= control warp: (iii) DLARFG (R1), V(:, j) ================
-            const Refl rf = dlarfg_scalars(nrm2, alpha, c + 2 >= ihi);
-            const double tau = rf.tau, beta = rf.beta, scale = rf.scale;
-            const double vchk = 1.0 + scale * sx;  // V_chk(j) = e^T v
-            // t = V^T v = V(c+1,:)^T + scale * V^T x; V(c+1, :) is also the next column's vrow
-            if (lane < j) {
-                S.t[lane] = vn0 + scale * vt0;
-                S.vrow[lane] = vn0;
-            }
-            if (lane + 32 < j) {
-                S.t[lane + 32] = vn1 + scale * vt1;
-                S.vrow[lane + 32] = vn1;
-            }
-            if (lane == 0) {
-                S.vrow[j] = 1.0;
-                S.scal[0] = tau;
-                S.scal[2] = scale;
-            }
-            PROBE(9);
-            // V(:, j) and the reduced column c of the own rows
-#pragma unroll 1
-            for (int rl = lane; rl < R; rl += 32) {
-                const int row = r0 + rl;
-                const double b = S.b0[rl];
-                if (row == n && p.abft) {
-                    V[row + (int64_t)j * ldw] = vchk;
-                    if (CACHE) Vl[rl * XR + j * XC] = vchk;
-                    Apan[row + (int64_t)c * ldw] = (tau != 0.0) ? b - vchk * (alpha - beta) : b;  // left term (R7)
-                } else if (is_data(row)) {
-                    double vv, av;
-                    if (row <= c) {
-                        vv = 0.0;
-                        av = b;
-                    } else if (row == c + 1) {
-                        vv = 1.0;
-                        av = beta;
-                    } else {
-                        vv = scale * b;
-                        av = vv;
-                    }
-                    V[row + (int64_t)j * ldw] = vv;
-                    if (CACHE) Vl[rl * XR + j * XC] = vv;
-                    Apan[row + (int64_t)c * ldw] = av;
-                } else if (CACHE) {
-                    Vl[rl * XR + j * XC] = 0.0;  // rows outside the panel take no part in the dots
-                }
-            }
-            if (bid == 0 && lane == 0) {
-                p.tau[c] = tau;
-                if (p.abft) {
-                    p.Qc[c] = vchk - 1.0;  // Q column checksum (P:266)
-                    qc_corner += vchk - 1.0;
-                }
-            }
-            // recycle the accumulator set of column c+2 (= that of column c-2): every CTA has
-            // finished reading it, and column c+2 adds into it only after two more syncs
-            if (bid == 0)
-                for (int i = lane; i < FT_ACC_STRIDE; i += 32) p.acc[((c + 2) & 3) * FT_ACC_SET_DOUBLES + i * FT_ACC_PAD] = 0.0;
-            PROBE(6);
         }
         __syncthreads();  // GEMV partials, tau / scale / t, V(:, j) are in shared memory
         if (p.dbg && tid == 0 && j == 8) {  // per-CTA GEMV span (debug hook): smid, start, end, rows
@@ -847,17 +855,19 @@ cudaError_t ft_launch_panel_wide(const PanelLaunch &L, int nsm, cudaStream_t s) 
         attr |= dbit;
     }
     if (L.nr != 1) return cudaErrorInvalidValue;
+    PanelLaunch Lw = L;  // ngroups in GR-row units (rbase is a multiple of GR_DRIVER)
+    Lw.r[0].ngroups = L.r[0].ngroups * (GR_DRIVER / GR);
     int grid = nsm < L.r[0].ngroups ? nsm : L.r[0].ngroups;
     if (grid > FT_FLAG_STRIDE) grid = FT_FLAG_STRIDE;
     if (grid < 1) grid = 1;
-    const int gmax = (L.r[0].ngroups + grid - 1) / grid;
+    const int gmax = (Lw.r[0].ngroups + grid - 1) / grid;
     const int rmax = GR * gmax;
     if (rmax > RMAX) return cudaErrorInvalidConfiguration;
     const size_t fixed = sizeof(PanelSmemW);
     const size_t want = fixed + (size_t)2 * VS * rmax * sizeof(double);
     const bool cache = want <= (size_t)max_smem;
     if (L.r[0].dpart && grid > FT_DPMAX) return cudaErrorInvalidValue;  // deterministic mode: partial slots
-    void *args[] = {const_cast<PanelLaunch *>(&L)};
+    void *args[] = {&Lw};
     g_ft_launches++;
     g_ft_wide_launches++;
     const void *fn = cache ? (const void *)k_panel_wide<true, false> : (const void *)k_panel_wide<false, false>;

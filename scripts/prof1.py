@@ -98,6 +98,7 @@ def main():
                   f"start spread {cta[:, 1].max() - t0} ns, end spread {cta[:, 2].max() - cta[:, 2].min()} ns")
             order = np.argsort(cta[:, 0])
             print("  smid:dur_ns " + " ".join(f"{int(cta[q, 0])}:{int(dur[q])}" for q in order))
+            print("  by CTA (bid:smid:dur_us) " + " ".join(f"{q}:{int(cta[q, 0])}:{dur[q] / 1e3:.0f}" for q in range(len(cta))))
         last_end = max(d[j * 16 + 8] for j in range(64))
         if d[3072] and d[3073]:
             print(f"CTA 0: prologue {d[0] - d[3072]} cycles, epilogue {d[3073] - last_end} cycles, "

@@ -95,7 +95,7 @@ def test_deterministic_bitwise_wide():
     # ill-conditioned (two valid summation orders move tau by ~1e-9, R18), so the
     # deterministic factorisation itself is held to the residual / orthogonality bar
     A3, t3, _ = reduce_once(A, nb=64)
-    assert rel(np.triu(A3, -1), np.triu(A1, -1)) <= 1e-11
+    assert rel(np.triu(A3, -1), np.triu(A1, -1)) <= TOL
     dA0 = torch.from_numpy(A).cuda()
     Qd, Hd = torch.from_numpy(Q1).cuda(), torch.triu(torch.from_numpy(A1).cuda(), -1)
     eps = 2.0 ** -52
