@@ -50,6 +50,10 @@
 #define VS 65         // shared-memory row stride of the V / Y row caches (doubles)
 #define RMAX PT       // max rows per CTA
 #define NSLOT (PT / 8)  // 8-lane groups per CTA (rows / outputs handled at once)
+// GEMV loads of A: L2 only (ld.global.cg) -- A streams once per column and never hits L1, and
+// bypassing L1 measured -1.2 % panel time at C3; evict-first: +3 %; nc.no_allocate: 0
+// (profiles/r02/s3b/gemv_loads_ab.txt)
+#define GLOAD(p) __ldcg(p)
 #ifndef GB
 // GEMV load batch (double2 of A + b per lane): 12 streams at 0.9 of the HBM copy bandwidth at C3
 // (8: -1.4 % panel time; 16 spills; a software-pipelined 2 x 6 / 2 x 8 batch: +8 %,
@@ -580,7 +584,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel_wide(const __grid_constant__ Pa
 #pragma unroll
                     for (int u = 0; u < GB; u++) {
                         const int q = col + u * ncl;
-                        a[u] = A2[(int64_t)q * ldw2 + rp];
+                        a[u] = GLOAD(A2 + (int64_t)q * ldw2 + rp);
                         v[u] = bv[q];
                     }
 #pragma unroll
@@ -598,7 +602,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel_wide(const __grid_constant__ Pa
 #pragma unroll
                     for (int u = 0; u < GB; u++) {
                         const int q = col + u * ncl;
-                        a[u] = q < cend ? A2[(int64_t)q * ldw2 + rp] : make_double2(0.0, 0.0);
+                        a[u] = q < cend ? GLOAD(A2 + (int64_t)q * ldw2 + rp) : make_double2(0.0, 0.0);
                         v[u] = q < cend ? bv[q] : 0.0;
                     }
 #pragma unroll
