@@ -33,6 +33,8 @@
 // V(:, j), Y(:, j), Z(:, j) and the next column's b0 and its reduction partials.
 // Accumulator sets are indexed by the global column (mod 4) and recycled in-kernel,
 // barrier counters alternate between consecutive panel launches: no memsets per panel.
+#include <type_traits>
+
 #include "ft_common.cuh"
 #include "ft_internal.h"
 
@@ -58,6 +60,14 @@
 #define VS 68         // row stride of the V / Y / Z row caches (doubles; = 4 mod 16: the combine's 8-lane row groups hit distinct banks)
 #define RMAX PT       // max rows per CTA
 #define NSLOT (PT / 8)  // 8-lane groups per CTA (rows / outputs handled at once)
+#ifndef NGLOAD_CG
+#define NGLOAD_CG 1
+#endif
+#if NGLOAD_CG
+#define NGLOAD(p) __ldcg(p)
+#else
+#define NGLOAD(p) (*(p))
+#endif
 #ifndef GB
 #define GB 8          // GEMV load batch (double2 of A + b per lane)
 #endif
@@ -527,7 +537,9 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
             // invalidated this SM's L1 before the trailing bar.sync released us.
             // Columns [k+2, k+2+ncc) come from the CTA's shared-memory copy of its row slab
             // (loaded once per panel), the rest from L2 / HBM.
-            auto run = [&](const double2 *__restrict__ base, int64_t cs2, int coff, int cbeg, int cstop) {
+            auto run = [&](const double2 *__restrict__ base, int64_t cs2, int coff, int cbeg, int cstop, auto glb) {
+                // glb: the operand streams from L2 / HBM -- L2-only loads (ld.global.cg, as the wide kernel)
+                auto ld = [&](const double2 *ptr) { return decltype(glb)::value ? NGLOAD(ptr) : *ptr; };
                 int col = cbeg + cl;
 #pragma unroll 1
                 for (; col + (GB - 1) * ncl < cstop; col += GB * ncl) {
@@ -536,7 +548,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
 #pragma unroll
                     for (int u = 0; u < GB; u++) {
                         const int q = col + u * ncl;
-                        a[u] = base[(int64_t)(q - coff) * cs2 + rp];
+                        a[u] = ld(base + (int64_t)(q - coff) * cs2 + rp);
                         v[u] = bv[q];
                     }
 #pragma unroll
@@ -553,7 +565,7 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
 #pragma unroll
                     for (int u = 0; u < GB; u++) {
                         const int q = col + u * ncl;
-                        a[u] = q < cstop ? base[(int64_t)(q - coff) * cs2 + rp] : make_double2(0.0, 0.0);
+                        a[u] = q < cstop ? ld(base + (int64_t)(q - coff) * cs2 + rp) : make_double2(0.0, 0.0);
                         v[u] = q < cstop ? bv[q] : 0.0;
                     }
 #pragma unroll
@@ -566,9 +578,10 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
                 }
             };
             const int csplit = min(cend, k + 2 + ncc);
-            if (c + 2 < csplit) run(reinterpret_cast<const double2 *>(Ac), R2, k + 2, c + 2, csplit);
+            if (c + 2 < csplit)
+                run(reinterpret_cast<const double2 *>(Ac), R2, k + 2, c + 2, csplit, std::integral_constant<bool, false>());
             const int cbeg = max(c + 2, csplit);
-            if (cbeg < cend) run(A2, ldw2, 0, cbeg, cend);
+            if (cbeg < cend) run(A2, ldw2, 0, cbeg, cend, std::integral_constant<bool, true>());
         }
         if (R2p <= 32) {
 #pragma unroll
