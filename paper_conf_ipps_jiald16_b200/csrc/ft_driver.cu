@@ -774,7 +774,8 @@ int enqueue_panel(Call &C, int t) {
     y.verify = eager ? 1 : 0;
     y.decide = fuse_pre ? 1 : 0;
     y.panel = t;
-    int nm = (k + 1 + 63) / 64;
+    const int ytm = ft_ytop_rows_per_cta();
+    int nm = (k + 1 + ytm - 1) / ytm;
     int nkt = (C.ihi - k - 1 + 31) / 32;
     // splits over the long inner dimension: about ytop_f CTAs per SM in total (4 warps each)
     static const int ytop_f = getenv("FT_YTOP_F") ? atoi(getenv("FT_YTOP_F")) : 12;  // measured: 2 -> 12 saves 42 ms at C3

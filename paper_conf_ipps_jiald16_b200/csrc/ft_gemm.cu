@@ -1045,14 +1045,17 @@ cudaError_t ft_launch_gemm_left(const GemmLeftParams &p, cudaStream_t s) {
 // split over the long inner dimension; the same pass sums A's rows for the
 // verify-before-consume check of the rows above the panel (area 1).
 // ---------------------------------------------------------------------------
-#define YT_M 64
+#ifndef YT_M
+#define YT_M 64  // rows per CTA (16 per warp)
+#endif
+#define YT_T (2 * YT_M)  // threads per CTA
 #define YT_K 32
 struct YtopSmem {
     double As[2][YT_K * (YT_M + 4)];      // A tile [col][row], double-buffered
     double Vs[2][FT_NBMAX * (YT_K + 4)];  // V [j][col]
 };
 
-__global__ void __launch_bounds__(128) k_ytop_partial(YtopParams p) {
+__global__ void __launch_bounds__(YT_T) k_ytop_partial(YtopParams p) {
     if (p.ctl->halt) return;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     YtopSmem &S = *reinterpret_cast<YtopSmem *>(smem_raw);
@@ -1098,7 +1101,7 @@ __global__ void __launch_bounds__(128) k_ytop_partial(YtopParams p) {
         cp_async_wait<1>();
         __syncthreads();
         if (p.verify)  // row sums: row threadIdx.x % 64, alternate k of the tile per half of the CTA
-            for (int kk = threadIdx.x >> 6; kk < nk; kk += 2) rs += S.As[st][kk * (YT_M + 4) + (threadIdx.x & 63)];
+            for (int kk = threadIdx.x / YT_M; kk < nk; kk += 2) rs += S.As[st][kk * (YT_M + 4) + (threadIdx.x % YT_M)];
         // warp tile: rows warp*16..+16, cols 0..63 (MI=2, NI=8)
         warp_mma<2, 8, true>(acc, S.As[st], YT_M + 4, S.Vs[st], YT_K + 4, warp * 16, 0, YT_K);
         __syncthreads();  // buffer st is refilled by the next iteration's issue
@@ -1117,7 +1120,7 @@ __global__ void __launch_bounds__(128) k_ytop_partial(YtopParams p) {
     if (p.verify) {  // the two halves' row sums meet in shared memory (the A tiles are free now)
         __syncthreads();
         double *half = &S.As[0][0];
-        if (threadIdx.x >= 64) half[threadIdx.x - 64] = rs;
+        if (threadIdx.x >= YT_M) half[threadIdx.x - YT_M] = rs;
         __syncthreads();
         if (threadIdx.x < mrows) p.rowpart[(int64_t)blockIdx.y * (p.k + 1) + m_lo + threadIdx.x] = rs + half[threadIdx.x];
     }
@@ -1125,19 +1128,14 @@ __global__ void __launch_bounds__(128) k_ytop_partial(YtopParams p) {
 
 // Y_top rows: sum the split partials, multiply by T; row-sum verify of area 1.
 // Block = 16 rows x 64 columns of Y.
-#define YF_R 16
+#define YF_R 16  // rows per row group (a thread per (row, j) of the group)
+#define YF_G 4   // row groups per CTA: T is loaded once per CTA for YF_G * YF_R rows
 __global__ void __launch_bounds__(YF_R * 64) k_ytop_finalize(YtopParams p) {
     __shared__ double Ts[FT_NBMAX * FT_NBMAX];
     __shared__ double y0[YF_R][FT_NBMAX + 1];
     const int jb = threadIdx.x & 63, rl = threadIdx.x >> 6;
-    const int row = blockIdx.x * YF_R + rl;
     const int ib = p.ib;
-    // the halt flag, this row's verify operands and T: every load in flight together
-    const bool vrow = p.verify && row <= p.k && jb == 0;
     const int halted = __ldcg(&p.ctl->halt);
-    const double a_k = vrow ? p.A[row + (int64_t)p.k * p.ldw] : 0.0;
-    const double a_n = vrow ? p.A[row + (int64_t)p.n * p.ldw] : 0.0;
-    const double f_r = vrow ? p.Fr[row] : 0.0;
     double tv[FT_NBMAX * FT_NBMAX / (YF_R * 64)];
 #pragma unroll
     for (int u = 0; u < FT_NBMAX * FT_NBMAX / (YF_R * 64); u++) {
@@ -1147,48 +1145,61 @@ __global__ void __launch_bounds__(YF_R * 64) k_ytop_finalize(YtopParams p) {
     if (halted) return;
 #pragma unroll
     for (int u = 0; u < FT_NBMAX * FT_NBMAX / (YF_R * 64); u++) Ts[threadIdx.x + u * YF_R * 64] = tv[u];
-    double acc = 0.0;
-    if (row <= p.k && jb < ib) {
-        // the split partials, 16 loads in flight at a time (fixed summation order)
-        const double *src = p.ypart + (int64_t)row * FT_NBMAX + jb;
-        const int64_t st = (int64_t)(p.k + 1) * FT_NBMAX;
-        for (int s0 = 0; s0 < p.nsplit; s0 += 16) {
-            double v[16];
+    const int64_t st = (int64_t)(p.k + 1) * FT_NBMAX;
+    double ey = 0.0;  // fused pre-update check: this thread's share of e^T Y(:, jb) over its rows
+#pragma unroll 1
+    for (int grp = 0; grp < YF_G; grp++) {
+        const int row = (blockIdx.x * YF_G + grp) * YF_R + rl;
+        if ((blockIdx.x * YF_G + grp) * YF_R > p.k) break;  // no row of this group exists (uniform)
+        // this row's verify operands and the split partials: every load in flight together
+        const bool vrow = p.verify && row <= p.k && jb == 0;
+        const double a_k = vrow ? p.A[row + (int64_t)p.k * p.ldw] : 0.0;
+        const double a_n = vrow ? p.A[row + (int64_t)p.n * p.ldw] : 0.0;
+        const double f_r = vrow ? p.Fr[row] : 0.0;
+        double acc = 0.0;
+        if (row <= p.k && jb < ib) {
+            // the split partials, 16 loads in flight at a time (fixed summation order)
+            const double *src = p.ypart + (int64_t)row * FT_NBMAX + jb;
+            for (int s0 = 0; s0 < p.nsplit; s0 += 16) {
+                double v[16];
 #pragma unroll
-            for (int u = 0; u < 16; u++) v[u] = s0 + u < p.nsplit ? __ldcg(src + (int64_t)(s0 + u) * st) : 0.0;
+                for (int u = 0; u < 16; u++) v[u] = s0 + u < p.nsplit ? __ldcg(src + (int64_t)(s0 + u) * st) : 0.0;
 #pragma unroll
-            for (int u = 0; u < 16; u++) acc += v[u];
+                for (int u = 0; u < 16; u++) acc += v[u];
+            }
         }
-    }
-    y0[rl][jb] = acc;
-    __syncthreads();
-    double yv = 0.0;
-    if (row <= p.k && jb < ib) {
-        double y1 = 0.0, y2 = 0.0, y3 = 0.0;  // four independent chains
-        int b = 0;
-        for (; b + 3 <= jb; b += 4) {
-            yv += y0[rl][b] * Ts[b + jb * FT_NBMAX];
-            y1 += y0[rl][b + 1] * Ts[b + 1 + jb * FT_NBMAX];
-            y2 += y0[rl][b + 2] * Ts[b + 2 + jb * FT_NBMAX];
-            y3 += y0[rl][b + 3] * Ts[b + 3 + jb * FT_NBMAX];
+        __syncthreads();  // Ts written (first group) / the previous group's y0 reads are done
+        y0[rl][jb] = acc;
+        __syncthreads();
+        double yv = 0.0;
+        if (row <= p.k && jb < ib) {
+            double y1 = 0.0, y2 = 0.0, y3 = 0.0;  // four independent chains
+            int b = 0;
+            for (; b + 3 <= jb; b += 4) {
+                yv += y0[rl][b] * Ts[b + jb * FT_NBMAX];
+                y1 += y0[rl][b + 1] * Ts[b + 1 + jb * FT_NBMAX];
+                y2 += y0[rl][b + 2] * Ts[b + 2 + jb * FT_NBMAX];
+                y3 += y0[rl][b + 3] * Ts[b + 3 + jb * FT_NBMAX];
+            }
+            for (; b <= jb; b++) yv += y0[rl][b] * Ts[b + jb * FT_NBMAX];
+            yv = (yv + y1) + (y2 + y3);
+            p.Y[row + (int64_t)jb * p.ldw] = yv;
+            ey += yv;
         }
-        for (; b <= jb; b++) yv += y0[rl][b] * Ts[b + jb * FT_NBMAX];
-        yv = (yv + y1) + (y2 + y3);
-        p.Y[row + (int64_t)jb * p.ldw] = yv;
-    }
-    if (vrow) {
-        double rsum = 0.0;
-        rsum = sum_strided(p.rowpart + row, p.k + 1, p.nsplit);
-        rsum += a_k;
-        if (p.ihi < p.n) rsum += sum_strided(p.A + row + (int64_t)p.ihi * p.ldw, p.ldw, p.n - p.ihi);
-        double d = a_n - f_r - rsum;
-        double tau_abs = p.ctl->c_thr * (double)p.n * 2.220446049250313e-16 * p.ctl->normF;
-        if (not_within(d, tau_abs)) atomicAdd(&p.ctl->nflag, 1);
+        if (vrow) {
+            double rsum = 0.0;
+            rsum = sum_strided(p.rowpart + row, p.k + 1, p.nsplit);
+            rsum += a_k;
+            if (p.ihi < p.n) rsum += sum_strided(p.A + row + (int64_t)p.ihi * p.ldw, p.ldw, p.n - p.ihi);
+            double d = a_n - f_r - rsum;
+            double tau_abs = p.ctl->c_thr * (double)p.n * 2.220446049250313e-16 * p.ctl->normF;
+            if (not_within(d, tau_abs)) atomicAdd(&p.ctl->nflag, 1);
+        }
     }
     if (!p.decide) return;
-    // fused pre-update check (reading R15): e^T Y of rows 0..k
+    // fused pre-update check (reading R15): e^T Y of rows 0..k, one add per column per CTA
     __syncthreads();
-    y0[rl][jb] = yv;
+    y0[rl][jb] = ey;
     __syncthreads();
     if (rl == 0 && jb < ib) {
         double s = 0.0;
@@ -1197,7 +1208,7 @@ __global__ void __launch_bounds__(YF_R * 64) k_ytop_finalize(YtopParams p) {
     }
     // the decision itself is taken by every CTA of the right update (GemmRightParams::pre_ctl)
 }
-
+int ft_ytop_rows_per_cta() { return YT_M; }
 cudaError_t ft_launch_ytop(const YtopParams &p, cudaStream_t s) {
     static unsigned attr = 0;
     const unsigned dbit = ft_dev_bit();
@@ -1209,9 +1220,9 @@ cudaError_t ft_launch_ytop(const YtopParams &p, cudaStream_t s) {
     }
     int nm = (p.k + 1 + YT_M - 1) / YT_M;
     g_ft_launches += 2;
-    k_ytop_partial<<<dim3(nm, p.nsplit), 128, smem, s>>>(p);
+    k_ytop_partial<<<dim3(nm, p.nsplit), YT_T, smem, s>>>(p);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
-    k_ytop_finalize<<<(p.k + 1 + YF_R - 1) / YF_R, YF_R * 64, 0, s>>>(p);
+    k_ytop_finalize<<<(p.k + 1 + YF_R * YF_G - 1) / (YF_R * YF_G), YF_R * 64, 0, s>>>(p);
     return cudaGetLastError();
 }

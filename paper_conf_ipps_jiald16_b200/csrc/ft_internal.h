@@ -212,6 +212,7 @@ struct YtopParams {
     // V rows through the column map; Y(0:k+1, :) is then this rank's partial
     int cm_G, cm_rank, cm_nb, cm_ncl, kc0, kc1;
 };
+int ft_ytop_rows_per_cta();  // rows of A per Y_top partial CTA (split sizing)
 cudaError_t ft_launch_ytop(const YtopParams &p, cudaStream_t s);
 
 // ABFT / utility kernels (ft_abft.cu)

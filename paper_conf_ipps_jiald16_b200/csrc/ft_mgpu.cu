@@ -731,7 +731,7 @@ int mg_panel(MgCall &C, int t) {
         y.cm_ncl = ncl;
         y.kc0 = C.lfirst(R.rank, k + 1);
         y.kc1 = ncl;
-        const int nm = (k + 1 + 63) / 64;
+        const int nm = (k + 1 + ft_ytop_rows_per_cta() - 1) / ft_ytop_rows_per_cta();
         const int nkt = (y.kc1 - y.kc0 + 31) / 32;
         int ns = std::max(1, std::min({(2 * R.nsm) / nm, std::max(nkt / 2, 1), 64}));
         while ((int64_t)ns * (k + 1) > kYtopRowsM) ns--;
