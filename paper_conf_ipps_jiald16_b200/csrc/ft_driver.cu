@@ -745,6 +745,10 @@ int enqueue_panel(Call &C, int t) {
     C.defer_from = -1;
     p.dbg = (t == g_dbg_panel) ? g_dbg_buf : nullptr;
     p.dbg_mode = ((t == g_dbg_panel) ? g_dbg_mode : 0) | g_panel_path;
+    {
+        static const int rot = getenv("FT_PANEL_ROT") ? atoi(getenv("FT_PANEL_ROT")) : 0;  // probe experiments
+        p.dbg_mode |= rot << 16;
+    }
     const int gr = ft_panel_group_rows();
     p.rbase = C.fused_ytop ? 0 : ((k + 1) / gr) * gr;
     p.ytop = C.fused_ytop ? 1 : 0;

@@ -45,7 +45,9 @@
 // row-group granularity of the CTA row blocks (64 bytes of a column; the driver's ft_panel_group_rows).
 // 2-row groups (equal rows per CTA to one double2) measured no faster at C3: the slowest CTAs of a
 // column are set by the address position of their rows, not by the +8-row blocks
+#ifndef GR
 #define GR 8
+#endif
 #define GR_DRIVER 8
 #define VS 65         // shared-memory row stride of the V / Y row caches (doubles)
 #define RMAX PT       // max rows per CTA
@@ -195,8 +197,10 @@ __global__ void __launch_bounds__(PT, 1) k_panel_wide(const __grid_constant__ Pa
 
     const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
     const int slot = tid >> 3, g = tid & 7;  // 8-lane groups: NSLOT row / output slots
-    const int g0 = (int)((long long)bid * p.ngroups / P);
-    const int g1 = (int)((long long)(bid + 1) * p.ngroups / P);
+    // row block of this CTA (dbg_mode >> 16: a rotation of the block <-> CTA map, probe experiments)
+    const int pbid = (int)((bid + (unsigned)(p.dbg_mode >> 16)) % P);
+    const int g0 = (int)((long long)pbid * p.ngroups / P);
+    const int g1 = (int)((long long)(pbid + 1) * p.ngroups / P);
     const int r0 = p.rbase + GR * g0, r1 = p.rbase + GR * g1;
     const int R = r1 - r0, R2 = R >> 1;
     const int n = p.n, ihi = p.ihi, k = p.k, ib = p.ib;
