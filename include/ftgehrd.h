@@ -21,9 +21,10 @@
  * Every call returns only after its stream has finished (info depends on the
  * device-side verification outcome).
  *
- * Threading: the library is NOT reentrant.  Its workspace, cached CUDA graphs and
- * counters are per device and process-global; calls from several host threads
- * (on one device or several) must be serialised by the caller.
+ * Threading: the workspace, cached CUDA graphs and counters are per device and
+ * process-global, so every entry point holds one process-wide lock for the whole call:
+ * calls from several host threads (on one device or several) are serialised by the
+ * library, not run concurrently.
  */
 #ifndef FTGEHRD_H
 #define FTGEHRD_H

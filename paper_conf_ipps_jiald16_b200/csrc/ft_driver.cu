@@ -19,6 +19,16 @@
 
 #include "ft_internal.h"
 
+#include <mutex>
+// Every public entry point holds this process-wide lock for the whole call: the workspace, the cached
+// graphs and the counters are shared per device, so calls from several host threads are serialised
+// here instead of racing (a call blocks until its stream has finished anyway).  Recursive: entry
+// points call each other (ft_dsytrd -> run, ft_dgehrd_host -> run).
+std::recursive_mutex &ft_api_mutex() {
+    static std::recursive_mutex mu;
+    return mu;
+}
+
 int64_t g_ft_launches = 0;
 int64_t g_ft_wide_launches = 0;
 extern "C" int64_t ft_debug_wide_launches(int reset) {
@@ -1837,10 +1847,12 @@ void ft_opts_default(ft_opts *o) {
 }
 
 int ft_dgehrd(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opts *opts) {
+    std::lock_guard<std::recursive_mutex> api_lock(ft_api_mutex());
     return run(n, ilo, ihi, dA, lda, dtau, opts);
 }
 
 int ft_dsytrd(int n, double *dA, int lda, double *dd, double *de, double *dtau, const ft_opts *opts) {
+    std::lock_guard<std::recursive_mutex> api_lock(ft_api_mutex());
     int info = validate(n, 1, n, dA, lda, dtau, nullptr);
     if (info) return info;
     if (n > 0 && !dd) return -4;
@@ -1855,6 +1867,7 @@ int ft_dsytrd(int n, double *dA, int lda, double *dd, double *de, double *dtau, 
 }
 
 int ft_dgehrd_host(int n, int ilo, int ihi, double *hA, int lda, double *htau, const ft_opts *opts) {
+    std::lock_guard<std::recursive_mutex> api_lock(ft_api_mutex());
     ft_opts o;
     ft_opts_default(&o);
     if (opts) o = *opts;
@@ -1895,6 +1908,7 @@ int ft_dgehrd_host(int n, int ilo, int ihi, double *hA, int lda, double *htau, c
 
 int ft_dorghr(int n, int ilo, int ihi, const double *dA, int lda, const double *dtau, double *dQ, int ldq,
               const ft_opts *opts) {
+    std::lock_guard<std::recursive_mutex> api_lock(ft_api_mutex());
     ft_opts o;
     ft_opts_default(&o);
     if (opts) o = *opts;

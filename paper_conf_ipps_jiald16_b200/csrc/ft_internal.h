@@ -274,6 +274,8 @@ cudaError_t ft_ctl_set_norm(FtCtl *ctl, double v, cudaStream_t s);
 
 #ifdef __cplusplus
 #include <vector>
+#include <mutex>
+std::recursive_mutex &ft_api_mutex();  // held by every public entry point (ft_driver.cu)
 // the host R12 decoder (ft_driver.cu), shared with the multi-rank path: 0 clean, 1 fixes, 2 refused
 int ft_host_decode(int n, const double *Dr, const double *Dc, double sr, double sc, double tau,
                    std::vector<FtFix> *fixes);

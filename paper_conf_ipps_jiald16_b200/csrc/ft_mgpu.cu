@@ -32,6 +32,8 @@
 #include "ft_common.cuh"
 #include "ft_internal.h"
 
+#include <mutex>
+
 #define CK(x)                                                                                       \
     do {                                                                                            \
         cudaError_t e_ = (x);                                                                       \
@@ -1079,6 +1081,7 @@ extern "C" {
 
 int ft_dgehrd_vranks(int n, int ilo, int ihi, double *const *dA_local, int lda_local, double *const *dtau,
                      int nranks, const ft_opts *opts) {
+    std::lock_guard<std::recursive_mutex> api_lock(ft_api_mutex());
     ft_opts o;
     ft_opts_default(&o);
     if (opts) o = *opts;
@@ -1119,6 +1122,7 @@ int ft_dgehrd_vranks(int n, int ilo, int ihi, double *const *dA_local, int lda_l
 }
 
 int ft_mgpu_setup(int n_max, int rank, int nranks, ft_ipc_handle *handle_out) {
+    std::lock_guard<std::recursive_mutex> api_lock(ft_api_mutex());
     if (nranks < 1 || nranks > FT_MAX_VRANKS || rank < 0 || rank >= nranks || n_max < 0 || !handle_out) return -9;
     int rc = mg_alloc(g_rank, std::max(n_max, 3), nranks, rank);
     if (rc) return rc;
@@ -1131,6 +1135,7 @@ int ft_mgpu_setup(int n_max, int rank, int nranks, ft_ipc_handle *handle_out) {
 }
 
 int ft_mgpu_connect(const ft_ipc_handle *handles, int rank, int nranks) {
+    std::lock_guard<std::recursive_mutex> api_lock(ft_api_mutex());
     if (!handles || g_rank.n_cap < 0 || nranks != g_rank.G || rank != g_rank.rank) return -9;
     for (int g = 0; g < nranks; g++) {
         if (g == rank) continue;
@@ -1153,6 +1158,7 @@ int ft_mgpu_connect(const ft_ipc_handle *handles, int rank, int nranks) {
 
 int ft_dgehrd_mgpu(int n, int ilo, int ihi, double *dA_local, int lda_local, double *dtau, int rank, int nranks,
                    const ft_opts *opts) {
+    std::lock_guard<std::recursive_mutex> api_lock(ft_api_mutex());
     ft_opts o;
     ft_opts_default(&o);
     if (opts) o = *opts;

@@ -143,3 +143,31 @@ def test_deterministic_option_validated():
     o.deterministic = 2
     assert ft.lib().ft_dgehrd(64, 1, 64, ctypes.c_void_p(dA.data_ptr()), 64, ctypes.c_void_p(tau.data_ptr()),
                               ctypes.byref(o)) == -7
+
+
+def test_concurrent_host_threads_are_serialised():
+    """Two host threads calling the library at once (own streams): the process-wide API lock
+    serialises them, and each result equals the sequential deterministic result bitwise."""
+    import threading
+    mats = [synth.matrix(257, dist="uniform"), synth.matrix(300, seed=7)]
+    ref = [reduce_once(A, nb=32, deterministic=True)[:2] for A in mats]
+    out = [None, None]
+
+    def work(q):
+        s = torch.cuda.Stream()
+        with torch.cuda.stream(s):
+            for _ in range(3):
+                dA = ft.fortran(torch.from_numpy(mats[q]).cuda())
+                tau, res = ft.dgehrd(dA, nb=32, deterministic=True, stream=s)
+                s.synchronize()
+                assert res.info == 0
+                out[q] = (dA.cpu().numpy(), tau.cpu().numpy()[: mats[q].shape[0] - 1])
+
+    th = [threading.Thread(target=work, args=(q,)) for q in range(2)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join()
+    for q in range(2):
+        assert out[q] is not None
+        assert np.array_equal(out[q][0], ref[q][0]) and np.array_equal(out[q][1], ref[q][1])
