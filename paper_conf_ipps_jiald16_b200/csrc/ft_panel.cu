@@ -1230,7 +1230,9 @@ cudaError_t ft_launch_panel_multi(const PanelLaunch &L, int nsm, cudaStream_t s)
         want += (size_t)ncc * rmax * sizeof(double);
     }
     // wide single-GPU launches: the two-reduction kernel (ft_panel_wide.cu), see its header
-    if (L.nr == 1 && !mg && rmax >= 32 && !(L.r[0].dbg_mode & (8 | 64 | 128)) && !explicit_path)
+    // (FT_WIDE_MIN_ROWS: the rows-per-CTA threshold of the wide kernel, for A/B runs)
+    static const int wide_min = getenv("FT_WIDE_MIN_ROWS") ? atoi(getenv("FT_WIDE_MIN_ROWS")) : 32;
+    if (L.nr == 1 && !mg && rmax >= wide_min && !(L.r[0].dbg_mode & (8 | 64 | 128)) && !explicit_path)
         return ft_launch_panel_wide(L, nsm, s);
     PanelLaunch Lx = L;
     for (int i = 0; i < Lx.nr; i++) {
