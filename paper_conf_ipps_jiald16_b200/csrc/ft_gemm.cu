@@ -1129,7 +1129,7 @@ __global__ void __launch_bounds__(YT_T) k_ytop_partial(YtopParams p) {
 // Y_top rows: sum the split partials, multiply by T; row-sum verify of area 1.
 // Block = 16 rows x 64 columns of Y.
 #define YF_R 16  // rows per row group (a thread per (row, j) of the group)
-#define YF_G 4   // row groups per CTA: T is loaded once per CTA for YF_G * YF_R rows
+#define YF_G 1  // row groups per CTA (4: +8 ms of finalize under the ncu launch list, profiles/r02/s3c)
 __global__ void __launch_bounds__(YF_R * 64) k_ytop_finalize(YtopParams p) {
     __shared__ double Ts[FT_NBMAX * FT_NBMAX];
     __shared__ double y0[YF_R][FT_NBMAX + 1];
