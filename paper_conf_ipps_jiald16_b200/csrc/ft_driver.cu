@@ -1351,7 +1351,8 @@ int run(int n, int ilo, int ihi, double *dA, int lda, double *dtau, const ft_opt
     // Y_top fused into the panel when every panel launch is narrow (<= 24 rows per CTA) and the
     // rows above the panel are cheap to stream per column (measured: faster at n = 1024 / 2048,
     // slower at n = 3200, where the GEMV's L2 traffic starts to dominate the column)
-    C.fused_ytop = (n + 1 + 7) / 8 <= 3 * w.nsm && n <= 2560 && !getenv("FT_NO_FUSED_YTOP");
+    const int pctas = ft_panel_cta_cap() > 0 ? std::min(ft_panel_cta_cap(), w.nsm) : w.nsm;
+    C.fused_ytop = (n + 1 + 7) / 8 <= 3 * pctas && n <= 2560 && !getenv("FT_NO_FUSED_YTOP");
     if (hA && o.stop_after_panel < 0) {
         C.hA = hA;
         C.hlda = hlda;

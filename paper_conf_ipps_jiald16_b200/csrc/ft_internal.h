@@ -113,6 +113,7 @@ cudaError_t ft_launch_panel_multi(const PanelLaunch &L, int nsm, cudaStream_t s)
 cudaError_t ft_launch_panel_wide(const PanelLaunch &L, int nsm, cudaStream_t s);  // two-reduction kernel
 size_t ft_panel_smem_bytes();
 int ft_panel_group_rows();
+int ft_panel_cta_cap();  // FT_PANEL_CTAS experiment cap on the panel grid (0: none)
 
 struct GemmRightParams {
     double *A;

@@ -1189,8 +1189,7 @@ cudaError_t ft_launch_panel_multi(const PanelLaunch &L, int nsm, cudaStream_t s)
     }
     static int ctas = -1, explicit_path = 0;
     if (ctas < 0) {
-        const char *e = getenv("FT_PANEL_CTAS");  // experiment knob: cap on the panel grid
-        ctas = e ? atoi(e) : 0;
+        ctas = ft_panel_cta_cap();
         const char *x = getenv("FT_PANEL_EXPLICIT");  // experiment knob: every column on the explicit path
         explicit_path = x ? atoi(x) : 0;
         const char *d = getenv("FT_PANEL_DBG");  // experiment knob: dbg_mode bits for every launch
@@ -1263,3 +1262,14 @@ cudaError_t ft_launch_panel(const PanelParams &p, int nsm, cudaStream_t s) {
 }
 
 int ft_panel_group_rows() { return GR; }
+// FT_PANEL_CTAS (experiment knob): a cap on the panel grid (0: one CTA per SM); the driver's fused-Y_top
+// decision (<= 24 rows per CTA) uses the same effective count
+int ft_panel_cta_cap() {
+    static int cap = -1;
+    if (cap < 0) {
+        const char *e = getenv("FT_PANEL_CTAS");
+        cap = e ? atoi(e) : 0;
+        if (cap < 0) cap = 0;
+    }
+    return cap;
+}
