@@ -190,6 +190,18 @@ FT_DEV void grid_barrier(unsigned *count, unsigned &epoch, unsigned nblocks) {
     __syncthreads();
 }
 
+// Watchdog for spins on flags written by OTHER GPUs (multi-rank exchanges): a peer that never
+// arrives (a dead rank, a broken peer mapping) ends the kernel with a trap after 60 s -- the call
+// then fails with a CUDA error instead of hanging the job.  Cheap: the timer is read once per 1024
+// polls.
+FT_DEV void peer_spin_guard(unsigned long long &t0, unsigned &polls) {
+    if ((++polls & 1023u) != 0u) return;
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    if (t0 == 0ull) t0 = t;
+    else if (t - t0 > 60ull * 1000000000ull) __trap();
+}
+
 // L2-coherent loads for data written by other CTAs inside the same launch
 FT_DEV double ldcg(const double *p) { return __ldcg(p); }
 

@@ -106,9 +106,13 @@ __global__ void __launch_bounds__(256) k_xchg(const __grid_constant__ XchgLaunch
     if (threadIdx.x < 32) {
         const int g = threadIdx.x;
         const bool need = g < x.G && (x.mode == 0 || g == x.root);
-        if (need)
+        if (need) {
+            unsigned long long t0 = 0ull;
+            unsigned polls = 0u;
             while (ld_acq_sys(own + g * FT_FLAG_STRIDE + bid) < x.seq) {
+                peer_spin_guard(t0, polls);
             }
+        }
     }
     __syncthreads();
     if (x.mode == 0) {

@@ -950,9 +950,13 @@ __global__ void __launch_bounds__(PT, 1) k_panel(const __grid_constant__ PanelLa
                 __threadfence_system();
                 for (int gg = 0; gg < p.G; gg++) st_relaxed_sys_u32(p.fpeer[gg] + p.rank * FT_FLAG_STRIDE + bid, seq);
             }
-            if (wid == 0 && lane < p.G)
+            if (wid == 0 && lane < p.G) {
+                unsigned long long t0 = 0ull;
+                unsigned polls = 0u;
                 while (ld_acquire_sys_u32(p.flags + lane * FT_FLAG_STRIDE + bid) < seq) {
+                    peer_spin_guard(t0, polls);
                 }
+            }
             __syncthreads();
         }
         if ((p.dbg_mode & 16) && !fb) {
