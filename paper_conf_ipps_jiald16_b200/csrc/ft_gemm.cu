@@ -494,9 +494,9 @@ __global__ void __launch_bounds__(UT, 1)
             if (last) {
                 double(*Ts)[SK] = S.Vc;  // reuse: T as Ts[a][b] (KT x KT)
                 double(*Ws)[SK] = reinterpret_cast<double(*)[SK]>(&S.Ys[0][0][0]);  // W as Ws[col][b] (64 x KT): spans both Ys buffers
-                for (int i = tid; i < KT * KT; i += UT) {
+                for (int i = tid; i < KT * KT; i += UT) {  // the upper triangle of T; zeros below it
                     const int a = i % KT, b = i / KT;
-                    const bool ok = a < K && b < K;
+                    const bool ok = a < K && b < K && a <= b;
                     cp_async8(&Ts[a][b], ok ? p.T + a + b * FT_NBMAX : p.T, ok ? 8 : 0);
                 }
                 cp_async_commit();
@@ -539,25 +539,32 @@ __global__ void __launch_bounds__(UT, 1)
                         not_within(ts - tchk_pre, (double)K * 2.220446049250313e-16 * tsa))
                         p.tctl->tbad = 1;
                 }
-                // W' = op(T) W: this thread's NE outputs as independent chains (one pass over b)
-                double so[NE];
+                // W' = op(T) W as a 64 x KT x KT DMMA product, D(col, a) = sum_b W(col, b) B(b, a) with
+                // B = T^T (transT: T(b, a), b <= a) or T (T(a, b), b >= a); the zeros below T's diagonal
+                // restrict the sums.  Warp tile 16 x 32 as in the update (conflict-free fragments)
+                {
+                    const int wc = warp & 3, wr = warp >> 2;
+                    double wacc2[2][4][2];
 #pragma unroll
-                for (int m = 0; m < NE; m++) so[m] = 0.0;
-#pragma unroll 2
-                for (int bb = 0; bb < K; bb++) {
+                    for (int mi = 0; mi < 2; mi++)
 #pragma unroll
-                    for (int m = 0; m < NE; m++) {
-                        const int i = tid + m * UT, cc = i / KT, a = i % KT;
-                        // transT: W'(a) = sum_{b <= a} T(b, a) W(b); else sum_{b >= a} T(a, b) W(b)
-                        const bool on = p.transT ? bb <= a : bb >= a;
-                        const double tv = p.transT ? Ts[bb][a] : Ts[a][bb];
-                        if (on) so[m] += tv * Ws[cc][bb];
+                        for (int ni = 0; ni < 4; ni++) wacc2[mi][ni][0] = wacc2[mi][ni][1] = 0.0;
+                    if (KT == 64 ? wr * 32 < KT : true) {
+                        if (p.transT)
+                            warp_mma2<2, 4, false, true>(wacc2, &Ws[0][0], SK, &Ts[0][0], SK, wc * 16, wr * 32 % KT, KT);
+                        else
+                            warp_mma2<2, 4, false, false>(wacc2, &Ws[0][0], SK, &Ts[0][0], SK, wc * 16, wr * 32 % KT, KT);
                     }
-                }
 #pragma unroll
-                for (int m = 0; m < NE; m++) {
-                    const int i = tid + m * UT, cc = i / KT, a = i % KT;
-                    if (cc < ncols && a < K) p.Wt[(int64_t)(cb + cc) * FT_NBMAX + a] = so[m];
+                    for (int mi = 0; mi < 2; mi++)
+#pragma unroll
+                        for (int ni = 0; ni < 4; ni++)
+#pragma unroll
+                            for (int v = 0; v < 2; v++) {
+                                const int cc = wc * 16 + mi * 8 + lr, a = (wr * 32 % KT) + ni * 8 + 2 * lc + v;
+                                if (cc < ncols && a < K && (KT == 64 || wr == 0))
+                                    p.Wt[(int64_t)(cb + cc) * FT_NBMAX + a] = wacc2[mi][ni][v];
+                            }
                 }
                 if (tid == 0) p.strip_done[blockIdx.x] = 0;
             }
