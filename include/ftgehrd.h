@@ -264,6 +264,13 @@ void ft_debug_right_fold(int on);
 /* Number of panel launches that ran the two-reduction wide kernel (>= 32 rows per CTA, the large-n
  * path) since load / the last reset: tests use it to show which panel kernel a run exercised. */
 int64_t ft_debug_wide_launches(int reset);
+/* Host-side diagnostics of the right update's row-split model (no device work): the number of row
+ * splits chosen for the block rows [r_lo, r_hi) x columns [c_lo, c_hi) on nsm SMs (extra_strips:
+ * the M-part strip; wr_lo: the first row of the W pass, -1 for none), and the tile range [t0, t1)
+ * that split y of ns gets when a strip of nrt tiles has tw right-only tiles at the top (weights 1
+ * and 2: the splits cut the strip into equal weights). */
+int ft_debug_right_splits(int r_lo, int r_hi, int c_lo, int c_hi, int nsm, int extra_strips, int wr_lo);
+void ft_debug_right_split_range(int nrt, int tw, int ns, int y, int *t0, int *t1);
 
 #ifdef __cplusplus
 }

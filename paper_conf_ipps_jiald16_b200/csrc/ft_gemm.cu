@@ -130,6 +130,15 @@ __device__ __forceinline__ unsigned char *align128(unsigned char *p) {
     return p + ((128u - (smem_u32(p) & 127u)) & 127u);
 }
 
+extern "C" int ft_debug_right_splits(int r_lo, int r_hi, int c_lo, int c_hi, int nsm, int extra_strips, int wr_lo) {
+    return ft_gemm_splits(r_lo, r_hi, c_lo, c_hi, nsm, extra_strips, wr_lo);
+}
+extern "C" void ft_debug_right_split_range(int nrt, int tw, int ns, int y, int *t0, int *t1) {
+    const long long units = (long long)tw + 2LL * (nrt - tw);
+    if (t0) *t0 = right_split_tile((long long)y * units / ns, tw);
+    if (t1) *t1 = right_split_tile((long long)(y + 1) * units / ns, tw);
+}
+
 template <int KT>
 struct RightSmemT {
     double Vc[KT][SK];     // sign * V(cols, k) as [k][col]   (A operand of the right update)

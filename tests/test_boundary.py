@@ -48,6 +48,7 @@ def test_library_is_sm100a_native(ft):
     assert "sm_100a" in out
     sass = subprocess.run(["cuobjdump", "-sass", ft.ftgehrd.LIB_PATH], capture_output=True, text=True).stdout
     assert "DMMA" in sass  # the block-reflector updates run on the FP64 tensor pipe
+    assert "UTMALDG" in sass  # their operand tiles arrive by 2-D tensor TMA
 
 
 def test_struct_layouts_match_header(ft):
@@ -58,6 +59,7 @@ def test_struct_layouts_match_header(ft):
     o = m.Opts()
     ft.lib().ft_opts_default(ctypes.byref(o))
     assert o.abft == 1 and o.nb == 0 and o.c_thr == 2.0 and o.stop_after_panel == -1 and o.weighted == 0
+    assert o.deterministic == 0 and o.timing == 0
 
 
 @pytest.mark.parametrize("args,expect", [
@@ -111,3 +113,38 @@ def test_product_package_does_not_import_oracle():
             if f.endswith((".py", ".cu", ".cuh", ".h", ".cpp")):
                 txt = open(os.path.join(dirpath, f)).read()
                 assert "import oracle" not in txt and "oracle.h" not in txt and "liboracle" not in txt, f
+
+
+def test_right_update_row_splits_partition_each_strip(ft):
+    """Host logic of the right update's weighted row splits (ft_gemm.cu): every split of a strip
+    gets a contiguous tile range, the ranges cover the strip exactly once, and the weights
+    (right-only tiles above the W rows 1, right + W tiles 2) differ by at most one tile."""
+    L = ft.lib()
+    L.ft_debug_right_split_range.argtypes = [ctypes.c_int] * 4 + [ctypes.POINTER(ctypes.c_int)] * 2
+    t0, t1 = ctypes.c_int(), ctypes.c_int()
+    for nrt in (1, 2, 3, 17, 64, 256, 257):
+        for tw in sorted({0, 1, nrt // 3, nrt // 2, nrt - 1, nrt}):
+            if tw < 0 or tw > nrt:
+                continue
+            for ns in (1, 2, 3, 5, 16, 32):
+                ranges = []
+                for y in range(ns):
+                    L.ft_debug_right_split_range(nrt, tw, ns, y, ctypes.byref(t0), ctypes.byref(t1))
+                    ranges.append((t0.value, t1.value))
+                assert ranges[0][0] == 0 and ranges[-1][1] == nrt
+                assert all(a <= b for a, b in ranges)
+                assert all(ranges[i][1] == ranges[i + 1][0] for i in range(ns - 1))
+                w = [sum(1 if t < tw else 2 for t in range(a, b)) for a, b in ranges]
+                total = tw + 2 * (nrt - tw)
+                assert max(w) - min(w) <= 3 and abs(max(w) - total / ns) <= 2.5, (nrt, tw, ns, w)
+
+
+def test_right_update_split_count_is_bounded(ft):
+    L = ft.lib()
+    L.ft_debug_right_splits.argtypes = [ctypes.c_int] * 7
+    for n in (300, 2048, 16384):
+        for e in (64, n // 2, n - 64):
+            for wr in (-1, 0, e - 63):
+                ns = L.ft_debug_right_splits(0, n, e, n + 1, 148, 1, wr)
+                nrt = (n + 63) // 64
+                assert 1 <= ns <= min(32, nrt), (n, e, wr, ns)
