@@ -69,7 +69,9 @@
 #define NGLOAD(p) (*(p))
 #endif
 #ifndef GB
-#define GB 8          // GEMV load batch (double2 of A + b per lane)
+// GEMV load batch (double2 of A + b per lane): 6 measured best at C2 (8: +1.5 % panel time, 4: +1 %,
+// 12 spills; C3 neutral), profiles/r02/s3b/gemv_loads_ab.txt
+#define GB 6
 #endif
 #define GAMMA (1.0 / 64.0)  // cancellation guard of the one-reduction column (see above)
 
