@@ -683,11 +683,14 @@ __global__ void k_wprep(const double *__restrict__ Wpart, int64_t wstride, int n
 
 template <int KT>
 __global__ void __launch_bounds__(UT, 2) k_gemm_left(const GemmLeftParams p, const __grid_constant__ CUtensorMap tmV) {
-    // both flags in flight together (one round trip before the launch's first load)
+    // both flags in flight together; they are first needed before this CTA's first global store,
+    // so their round trip overlaps the CTA's first loads (the operand strip, the first tiles)
     const int halted = p.ctl ? __ldcg(&p.ctl->halt) : 0;
     const int tbad = p.tctl ? __ldcg(&p.tctl->tbad) : 0;
-    if (halted) return;
-    if (tbad) {  // the right update consumed a corrupted T: nothing here runs
+    // the right update consumed a corrupted T: nothing here runs, CTA (0, 0) raises the halt
+    auto stop = [&]() -> bool {
+        if (halted) return true;
+        if (!tbad) return false;
         if (blockIdx.x == 0 && blockIdx.y == 0 && threadIdx.x == 0) {
             FtCtl *ctl = p.tctl;
             ctl->halt_panel = p.panel;
@@ -696,8 +699,8 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(const GemmLeftParams p, con
             __threadfence();
             ctl->halt = 1;
         }
-        return;
-    }
+        return true;
+    };
     if ((int)blockIdx.y < p.nyf) {
         // frozen row sums of the panel columns k..e-1 (final now, untouched by this launch; R6):
         // Fr(i) += sum_{col in [max(k, i-1), e)} A(i, col) for i <= e -- one row per thread in
@@ -705,7 +708,10 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(const GemmLeftParams p, con
         // they come first in the grid (scheduled first, off the launch's tail)
         const int k = p.r_lo - 1, e = p.c_lo, rows = min(e + 1, p.n);
         const int i = (blockIdx.y * gridDim.x + blockIdx.x) * UT + threadIdx.x;
-        if (i >= rows) return;
+        if (i >= rows) {
+            stop();
+            return;
+        }
         const double *a = p.A + i;
         // all of a row's loads in flight together (<= 64 columns): 8 at a time into 8 chains
         double s[8] = {0.0, 0.0, 0.0, 0.0, 0.0, 0.0, 0.0, 0.0};
@@ -718,6 +724,7 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(const GemmLeftParams p, con
 #pragma unroll
         for (int u = 0; u < 7; u++)
             if (c + u < e) s[u] += __ldcg(a + (int64_t)(c + u) * p.lda);
+        if (stop()) return;
         p.Fr[i] += ((s[0] + s[1]) + (s[2] + s[3])) + ((s[4] + s[5]) + (s[6] + s[7]));
         return;
     }
@@ -737,13 +744,6 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(const GemmLeftParams p, con
     const int nrt = (p.r_hi - rbase + UB - 1) / UB;
     const int t0 = (int)((long long)by * nrt / p.ny);
     const int t1 = (int)((long long)(by + 1) * nrt / p.ny);
-    if (p.pre_reset && bx == 0 && by == 0) {  // the right update has read them
-        for (int j = tid; j < FT_NBMAX; j += UT) {
-            p.pre_reset->eY[j * FT_ESTR] = 0.0;
-            p.pre_reset->eV[j * FT_ESTR] = 0.0;
-        }
-        if (tid == 0) p.pre_reset->nflag = 0;
-    }
 
     // V tiles (rows r .. r+SK-1, columns 0..K-1) by 2-D tensor TMA, one instruction per tile issued
     // by thread 0, into a double buffer: full[b] completes on the copy's transaction count, empty[b]
@@ -842,6 +842,17 @@ __global__ void __launch_bounds__(UT, 2) k_gemm_left(const GemmLeftParams p, con
     };
     double2 cn[2][4];
     if (t0 < t1) load_c(t0, cn);
+    if (stop()) {  // before any global store; the copies in flight land before the CTA exits
+        for (int b = 0; b < 2 && t0 + b < t1; b++) mbar_wait(&vfull[b], 0u);
+        return;
+    }
+    if (p.pre_reset && bx == 0 && by == 0) {  // the right update has read them
+        for (int j = tid; j < FT_NBMAX; j += UT) {
+            p.pre_reset->eY[j * FT_ESTR] = 0.0;
+            p.pre_reset->eV[j * FT_ESTR] = 0.0;
+        }
+        if (tid == 0) p.pre_reset->nflag = 0;
+    }
     __syncthreads();  // every thread's part of sign * W' landed
     for (int tt = t0; tt < t1; tt++) {
         const int it = tt - t0, st = it & 1;
